@@ -1,0 +1,287 @@
+"""Pins of the CPU oracle against the paper and mathematics (never against itself).
+
+P:n = PAPER.md line n.  Each test says what it pins and where the expected
+value comes from: a closed form (oracle/closed_forms.py, computed two ways), a
+worked example of the paper, brute force on tiny inputs, or a magnitude the
+paper prints.
+"""
+import os
+
+import numpy as np
+import pytest
+
+import atfspec as A
+from atfspec import (Spec, X, C, P, DIVIDES, MULOF, interval, pow2, set_, divides,
+                     is_multiple_of, E)
+from oracle import closed_forms as cf
+from oracle import run as orc
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def sizes(d):
+    return [g["size"] for g in d["groups"]]
+
+
+def fs(d, g=0):
+    return [lv["f"] for lv in d["groups"][g]["levels"]]
+
+
+# ---------------------------------------------------------------- closed forms
+def test_c1_closed_form(oracle_bin):
+    d = orc.info(A.c1_toy())
+    assert int(d["S"]) == cf.c1_size() == 46
+    assert fs(d) == [cf.count_divisors_upto(64, 64), 46]
+    assert [lv["evals"] for lv in d["groups"][0]["levels"]] == [64, 7 * 64]
+
+
+@pytest.mark.parametrize("n", [1, 12, 64, 360, 1000, 4096])
+def test_saxpy_closed_form(oracle_bin, n):
+    """WPT|N, LS|(N/WPT)  =>  S = sum_{d|N} tau(d) = prod (a+1)(a+2)/2."""
+    d = orc.info(A.saxpy(n))
+    assert int(d["S"]) == cf.saxpy_size_by_divisor_sum(n) == cf.saxpy_size_by_exponents(n)
+    assert fs(d)[0] == cf.tau(n)
+    assert len(d["groups"]) == 1
+
+
+def test_saxpy_named_values(oracle_bin):
+    # N = 64 -> 28, N = 1000 -> 100, N = 4096 -> 91 (closed form)
+    for n, s in [(64, 28), (1000, 100), (4096, 91)]:
+        assert cf.saxpy_size_by_exponents(n) == s
+        assert int(orc.info(A.saxpy(n))["S"]) == s
+
+
+def test_fig1_worked_example(oracle_bin):
+    """Fig. 1: two groups {tp1,tp2}, {tp3,tp4}; 3 configs each; S = 9."""
+    s = A.fig1()
+    d = orc.info(s)
+    assert [g["members"] for g in d["groups"]] == [[0, 1], [2, 3]]
+    assert sizes(d) == [3, 3] and int(d["S"]) == 9
+    assert fs(d, 0) == [2, 3] and fs(d, 1) == [2, 3]
+    gold = np.loadtxt(os.path.join(GOLDEN, "fig1_rows.txt"), dtype=np.int32, comments="#")
+    info, soa = orc.decode(s, np.arange(9, dtype=np.uint64))
+    assert np.array_equal(soa.T, gold)
+    _, rows = orc.o1(s)
+    assert np.array_equal(rows, gold)
+
+
+@pytest.mark.parametrize("R,E", [(64, 64), (100, 360), (10, 360), (4096, 2**12), (37, 1)])
+def test_interval_divisibility_counts(oracle_bin, R, E):
+    s = Spec("div"); s.add("x", interval(1, R), divides(E))
+    assert int(orc.info(s)["S"]) == cf.count_divisors_upto(E, R)
+    s = Spec("mul"); s.add("x", interval(1, R), is_multiple_of(E))
+    assert int(orc.info(s)["S"]) == cf.count_multiples_upto(E, R)
+
+
+@pytest.mark.parametrize("R", [1, 17, 64, 500])
+def test_divisor_pairs_hyperbola(oracle_bin, R):
+    s = Spec("pairs"); s.add("a", interval(1, R)); s.add("b", interval(1, R), divides(P(0)))
+    assert int(orc.info(s)["S"]) == cf.dirichlet_hyperbola_D2(R) == cf.piltz_D(R, 2)[1]
+
+
+def test_piltz_two_routes():
+    # D_k(R) by the Dirichlet recurrence vs a literal chain count on a tiny range
+    R, k = 24, 4
+    def chains(depth, top):
+        if depth == 0:
+            return 1
+        return sum(chains(depth - 1, d) for d in range(1, top + 1) if top % d == 0)
+    brute = [sum(chains(j, x) for x in range(1, R + 1)) for j in range(k)]
+    assert brute == cf.piltz_D(R, k)
+    assert cf.piltz_D(4096, 2)[1] == 34720          # SURVEY.md §8(c) interval pin
+
+
+@pytest.mark.parametrize("R,L", [(60, 5), (128, 8)])
+def test_c5_chains_piltz(oracle_bin, R, L):
+    d = orc.info(A.c5_chains(R, L), threads=8)
+    want = cf.c5_level_sizes(R, L)
+    assert [fs(d, g) for g in range(3)] == want
+    S = 1
+    for w in want:
+        S *= w[-1]
+    assert int(d["S"]) == S
+    for g in range(3):
+        lv = d["groups"][g]["levels"]
+        prev = 1
+        for l in lv:
+            assert l["evals"] == prev * l["r"]     # evals_k = f_{k-1} * r_k
+            prev = l["f"]
+
+
+# ---------------------------------------------------------------- paper magnitudes
+def test_c2_paper_magnitudes(oracle_bin):
+    """at 2^10 x 2^10 the unconstrained XgemmDirect space has > 10^19 configs while
+    ATF's constrained space has 'nearly 10^7'."""
+    d = orc.info(A.c2_xgemm_direct(1024), threads=8)
+    assert int(d["unconstrained"]) == 1024 ** 6 * 4 * 4 * 2 * 2 > 10 ** 19
+    S = int(d["S"])
+    assert 5 * 10 ** 6 < S < 10 ** 7
+    # without the anchor (WGD|M, WGD|N) the size is far from 10^7: the anchor is confirmed
+    assert [g["members"] for g in d["groups"]] == [[0, 1, 2, 3, 4, 5, 6, 7], [8], [9]]
+
+
+def test_empty_space_cltune_limits(oracle_bin):
+    """CLTune's WGD in {8,16,32} with WGD | rows and WGD | cols empties the space for
+    the deep-learning shapes (rows 20, cols 576)."""
+    s = Spec("cltune_wgd"); s.add("WGD", set_(8, 16, 32), divides(20) & divides(576))
+    s.add("KWID", interval(1, 32), divides(P(0)))
+    d = orc.info(s)
+    assert int(d["S"]) == 0 and sizes(d) == [0]
+
+
+def test_pow2_first_ten(oracle_bin):
+    """interval<size_t>(1, 10, pow(2,i)) 'represents the first ten powers of 2'."""
+    s = Spec("pow2"); s.add("x", pow2(1, 10))
+    assert int(orc.info(s)["S"]) == 10
+    info, soa = orc.decode(s, np.arange(10, dtype=np.uint64))
+    assert soa[0].tolist() == [2 ** i for i in range(1, 11)]
+    s = Spec("even"); s.add("z", interval(2, 4096, 2))
+    assert int(orc.info(s)["S"]) == 2048
+
+
+def test_duplicate_set_rejected(oracle_bin):
+    s = Spec("dup"); s.add("x", set_(1, 2, 2))
+    with pytest.raises(ValueError):
+        orc.info(s)
+
+
+# ---------------------------------------------------------------- metamorphic
+@pytest.mark.parametrize("n", [16, 32])
+def test_c2_implied_constraints_change_nothing(oracle_bin, n):
+    a = orc.info(A.c2_xgemm_direct(n, implied=True), hash=True)
+    b = orc.info(A.c2_xgemm_direct(n, implied=False), hash=True)
+    assert a["S"] == b["S"]
+    assert [g["hash"] for g in a["groups"]] == [g["hash"] for g in b["groups"]]
+
+
+def test_tautology_changes_nothing(oracle_bin):
+    s1 = A.c3_xgemm((6, 8, 4))
+    s2 = A.c3_xgemm((6, 8, 4))
+    s2.params[5].constraints.append((X >= 1).code)          # MDIMA >= 1 holds on its range
+    a, b = orc.info(s1, hash=True), orc.info(s2, hash=True)
+    assert a["groups"][0]["hash"] == b["groups"][0]["hash"]
+
+
+# ---------------------------------------------------------------- O1 == O2 (brute force)
+def _o1_vs_decode(spec):
+    d1, rows = orc.o1(spec)
+    d2 = orc.info(spec)
+    assert int(d2["S"]) == d1["S"] == rows.shape[0]
+    if rows.shape[0]:
+        _, soa = orc.decode(spec, np.arange(rows.shape[0], dtype=np.uint64))
+        assert np.array_equal(soa.T, rows)
+
+
+@pytest.mark.parametrize("name", ["c1", "fig1", "saxpy12", "c2_8", "c3_tiny", "c3_tiny_anch"])
+def test_o1_equals_o2_named(oracle_bin, name):
+    spec = {"c1": A.c1_toy, "fig1": A.fig1, "saxpy12": lambda: A.saxpy(12),
+            "c2_8": lambda: A.c2_xgemm_direct(8), "c3_tiny": lambda: A.c3_xgemm((4, 6, 2)),
+            "c3_tiny_anch": lambda: A.c3_xgemm((3, 2, 2), anchored=True)}[name]()
+    _o1_vs_decode(spec)
+
+
+@pytest.mark.parametrize("seed", range(60))
+def test_o1_equals_o2_fuzz(oracle_bin, seed):
+    _o1_vs_decode(A.random_spec(seed))
+
+
+# ---------------------------------------------------------------- two encodings agree
+@pytest.mark.parametrize("spec,native", [
+    (lambda: A.c1_toy(), "c1"),
+    (lambda: A.c2_xgemm_direct(256), "c2:256"),
+    (lambda: A.c3_xgemm("IS1"), "c3:"),
+    (lambda: A.c3_xgemm("IS3"), "c3:"),
+    (lambda: A.c3_xgemm((12, 30, 8)), "c3:"),
+    (lambda: A.saxpy(360), "saxpy:360"),
+])
+def test_bytecode_matches_native_predicates(oracle_bin, spec, native):
+    d = orc.info(spec(), threads=4, native=native, native_check=True)
+    assert d["native_mismatch"] == 0
+    d2 = orc.info(spec(), threads=4, native=native)
+    assert d2["S"] == d["S"]
+
+
+# ---------------------------------------------------------------- decode = mixed radix
+def test_decode_mixed_radix_c4_structure(oracle_bin):
+    """SURVEY.md §8(c) C4 pin: with contiguous groups and the four binary singletons last,
+    decode(i) = (G0 tuple floor(i/16), bits of i mod 16 for STRM, STRN, SA, SB)."""
+    s = A.c3_xgemm((4, 8, 4))
+    d = orc.info(s)
+    g0 = orc.leaves(s, 0, 10)
+    S = int(d["S"])
+    assert S == g0.shape[0] * 16
+    idx = np.arange(S, dtype=np.uint64)
+    _, soa = orc.decode(s, idx)
+    i = np.arange(S)
+    assert np.array_equal(soa[:10].T, g0[i // 16])
+    for b, p in enumerate([10, 11, 12, 13]):
+        assert np.array_equal(soa[p], (i >> (3 - b)) & 1)
+    # lexicographic extremes
+    assert soa[:, 0].tolist()[:3] == [1, 1, 1]
+
+
+def test_decode_out_of_range(oracle_bin):
+    s = A.fig1()
+    info, soa = orc.decode(s, np.array([9, 10, 2 ** 63], dtype=np.uint64))
+    assert info["invalid"] == 3
+    assert (soa == np.iinfo(np.int32).min).all()
+
+
+# ---------------------------------------------------------------- opcode semantics
+def _accepted(code, lo=-6, hi=6):
+    s = Spec("op"); s.add("x", interval(lo, hi), code)
+    n = int(orc.info(s)["S"])
+    if n == 0:
+        return []
+    _, soa = orc.decode(s, np.arange(n, dtype=np.uint64))
+    return soa[0].tolist()
+
+
+def test_opcode_semantics_reading_table(oracle_bin):
+    """Readings #6-#8: aliases, strict evaluation, zero divisor rejects, C truncation."""
+    xs = range(-6, 7)
+    trunc_div = lambda a, b: abs(a) // abs(b) * (1 if (a >= 0) == (b >= 0) else -1)
+    trunc_mod = lambda a, b: a - b * trunc_div(a, b)
+    assert _accepted(divides(12)) == [x for x in xs if x != 0 and 12 % abs(x) == 0]
+    # x % 3 == 0 includes x = 0 (MULOF: [b != 0 and a mod b == 0], b = 3)
+    assert _accepted(is_multiple_of(3)) == [x for x in xs if trunc_mod(x, 3) == 0]
+    assert _accepted(X < 2) == [x for x in xs if x < 2]
+    assert _accepted(X <= 2) == [x for x in xs if x <= 2]
+    assert _accepted(X.eq(-3)) == [-3]
+    assert _accepted(X.ne(-3)) == [x for x in xs if x != -3]
+    # DIV truncates toward zero; -7 / 2 = -3
+    assert _accepted((C(-7) // X).eq(-3)) == [x for x in xs if x != 0 and trunc_div(-7, x) == -3]
+    assert _accepted((C(-7) % X).eq(-1)) == [x for x in xs if x != 0 and trunc_mod(-7, x) == -1]
+    # zero divisor rejects even under OR with a true operand (strict evaluation, reading #7)
+    assert 0 not in _accepted(((C(5) // X) > 100) | C(1))
+    assert 0 not in _accepted(~DIVIDES(X, 7))
+    assert _accepted(~DIVIDES(X, 7)) == [x for x in xs if x != 0 and 7 % abs(x) != 0]
+    # integer result used as a boolean: nonzero accepts
+    assert _accepted(X - 2) == [x for x in xs if x != 2]
+    assert _accepted(E((X * X).code)) == [x for x in xs if x != 0]
+    assert _accepted(A.min_(X, 3).eq(3)) == [x for x in xs if x >= 3]
+    assert _accepted(A.max_(X, 3).eq(3)) == [x for x in xs if x <= 3]
+
+
+def test_cltune_zero_range_same_space(oracle_bin):
+    """CLTune's saxpy ranges start at 0; with reading #7 a zero divisor rejects the
+    candidate, so the 0..N ranges define the same space as 1..N."""
+    n = 360
+    s = Spec("saxpy0"); s.add("WPT", interval(0, n), divides(n))
+    s.add("LS", interval(0, n), divides(C(n) // P(0)))
+    assert int(orc.info(s)["S"]) == cf.saxpy_size_by_exponents(n)
+
+
+def test_overflow_is_reported(oracle_bin):
+    s = Spec("ovf"); s.add("x", interval(1, 4), (C(2 ** 62) * X) > 0)
+    assert orc.info(s)["overflow"] is True
+
+
+# ---------------------------------------------------------------- survey cross-check
+def test_c3_small_shapes_match_survey_appendix(oracle_bin):
+    """SURVEY.md Appendix A (an independent counter): C3 IS1 and IS3 per-level f_k."""
+    d = orc.info(A.c3_xgemm("IS1"), threads=8)
+    assert fs(d) == [20, 11520, 11520, 38016, 248424, 85055, 90173, 90173, 129716, 239741]
+    d = orc.info(A.c3_xgemm("IS3"), threads=8)
+    assert fs(d) == [50, 3200, 3200, 13248, 57960, 35070, 30555, 30555, 48298, 80124]
+    assert int(d["S"]) == 80124 * 16
