@@ -1,0 +1,238 @@
+/*
+ * atfgen.h — C ABI of the B200-native ATF search-space generator.
+ *
+ * The operation (PAPER.md, cited as P:n = line n):
+ *   A tuning parameter has a unique name, a range and a constraint (P:51-59,
+ *   §II Step 1).  The search space "comprises all valid parameter
+ *   configurations, i.e., for which the parameters' constraints are
+ *   satisfied".  ATF generates it "by iterating over the constrained
+ *   ranges of tuning parameters" rather than filtering the unconstrained
+ *   product, per group of interdependent parameters.
+ *   The space has a size S and is index-addressable: OpenTuner's
+ *   TP in [1,S] selects "the configuration with index TP within the ATF search
+ *   space".
+ *
+ * This library builds each parameter group's valid configurations on one GPU
+ * (sm_100a) as a per-level tree (level k = the group's k-th parameter), and
+ * exposes S (u128), per-group sizes and a batched index -> configuration
+ * decoder.  Groups are found automatically (connected components of the
+ * constraint-reference graph) instead of the paper's user-supplied G(...)
+ * (P:245).
+ *
+ * Conventions:
+ *   - Indices are 0-based (the paper's TP is 1-based).
+ *   - Group order: by first-declared member; group 0 is the most significant
+ *     mixed-radix digit.  Inside a group: lexicographic order of range
+ *     positions in declaration order.  Output columns are in declaration order.
+ *   - Intervals are inclusive, value(i) = gen(begin + i*step).
+ *   - A zero divisor anywhere in a constraint rejects the candidate; AND/OR
+ *     are strict (non-short-circuit) (reading #7).
+ *
+ * Errors: every function returns atf_status (0 = ATF_OK, < 0 = error); no
+ * exceptions cross the ABI.  atf_space_last_error() gives a message.
+ * Threading: an atf_space is not thread-safe; distinct spaces are independent.
+ * Ownership: host inputs (names, range values, bytecode) are copied before the
+ * call returns.  Device buffers passed to decode are borrowed until the work
+ * queued on `stream` completes.  The space owns its tree memory.
+ */
+#ifndef ATFGEN_H
+#define ATFGEN_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct atf_space atf_space; /* opaque, owned by the library */
+
+typedef enum {
+  ATF_OK = 0,
+  ATF_ERR_INVALID_ARG = -1, /* NULL pointer, bad kind, step <= 0, empty name, ...      */
+  ATF_ERR_OOM = -2,         /* allocation failed (device or host)                      */
+  ATF_ERR_CUDA = -3,        /* a CUDA runtime call failed (message in last_error)      */
+  ATF_ERR_STATE = -4,       /* call not allowed in the space's current state           */
+  ATF_ERR_BYTECODE = -5,    /* bad opcode, stack underflow/overflow, not 1 result       */
+  ATF_ERR_FORWARD_REF = -6, /* PARAM j with j >= the constrained parameter's id       */
+  ATF_ERR_OVERFLOW = -7,    /* int64 overflow possible / size or index too large      */
+  ATF_ERR_INDEX = -8,       /* decode index >= S (rows filled with INT32_MIN)          */
+  ATF_ERR_DUPLICATE = -9,   /* duplicate parameter name or duplicate set value        */
+  ATF_ERR_LIMIT = -10       /* a documented v1 limit is exceeded                       */
+} atf_status;
+
+/* Range kinds.
+ *   INTERVAL: values begin, begin+step, ..., <= end (inclusive, reading #1); int32.
+ *   POW2:     values 2^i for i = begin, begin+step, ..., <= end; 0 <= i <= 30
+ *             ("atf::interval<size_t>(1,10,[](i){return pow(2,i);})" = first ten powers of 2).
+ *   SET:      values[0..n_values) in the listed order; duplicates -> ATF_ERR_DUPLICATE.
+ *             bool and enum parameters are SETs of ints ({0,1} for bools). */
+typedef enum { ATF_RANGE_INTERVAL = 0, ATF_RANGE_POW2 = 1, ATF_RANGE_SET = 2 } atf_range_kind;
+
+typedef struct {
+  int32_t kind;           /* atf_range_kind */
+  int64_t begin, end, step;
+  const int32_t* values;  /* SET only: host pointer, copied */
+  int64_t n_values;
+} atf_range;
+
+/* Device allocator hooks (e.g. PyTorch's caching allocator).  If alloc is NULL
+ * the library uses cudaMallocAsync/cudaFreeAsync on its stream.  `stream` is the
+ * cudaStream_t the memory will be used on. */
+typedef void* (*atf_alloc_fn)(size_t bytes, void* stream, void* ctx);
+typedef void (*atf_free_fn)(void* ptr, size_t bytes, void* stream, void* ctx);
+
+typedef struct {
+  int32_t device;      /* CUDA device ordinal                                  */
+  void* stream;        /* cudaStream_t for all work (NULL = legacy default)    */
+  atf_alloc_fn alloc;  /* optional */
+  atf_free_fn free;    /* optional (required if alloc is set) */
+  void* alloc_ctx;
+  uint32_t flags;      /* ATF_FLAG_* */
+} atf_space_opts;
+
+#define ATF_FLAG_TIMING 1u        /* record per-level CUDA-event times (atf_space_stats)  */
+#define ATF_FLAG_GENERIC_ONLY 2u  /* disable the hoisted fast atoms: interpret every
+                                     candidate with the generic bytecode interpreter     */
+#define ATF_FLAG_KEEP_LEVELS 4u   /* keep inner-level arrays (CSR + records); default
+                                     keeps them too — reserved                          */
+
+/* Bytecode: postfix int32 words, int64 stack.
+ *   1 X            push the candidate value
+ *   2 PARAM j      push the value of parameter j (j < the constrained parameter's id)
+ *   3 CONST lo hi  push the int64 (hi << 32) | (uint32)lo
+ *   4 ADD 5 SUB 6 MUL            exact; possible int64 overflow -> ATF_ERR_OVERFLOW
+ *   7 DIV 8 MOD                  C truncation; b == 0 -> poison
+ *   9 MIN 10 MAX
+ *  11 EQ 12 NE 13 LT 14 LE 15 GT 16 GE   -> 0/1
+ *  17 DIVIDES  a b -> [b mod a == 0]; a == 0 -> poison     (atf::divides)
+ *  18 MULOF    a b -> [a mod b == 0]; b == 0 -> poison     (atf::is_multiple_of)
+ *  19 AND 20 OR (strict)  21 NOT
+ * A candidate is accepted iff the program leaves exactly one item, it is
+ * nonzero, and no poison occurred.  Several constraints on one parameter are
+ * ANDed.  Limits: <= 256 words and stack depth <= 16 per program. */
+enum {
+  ATF_OP_X = 1, ATF_OP_PARAM = 2, ATF_OP_CONST = 3, ATF_OP_ADD = 4, ATF_OP_SUB = 5, ATF_OP_MUL = 6,
+  ATF_OP_DIV = 7, ATF_OP_MOD = 8, ATF_OP_MIN = 9, ATF_OP_MAX = 10, ATF_OP_EQ = 11, ATF_OP_NE = 12,
+  ATF_OP_LT = 13, ATF_OP_LE = 14, ATF_OP_GT = 15, ATF_OP_GE = 16, ATF_OP_DIVIDES = 17,
+  ATF_OP_MULOF = 18, ATF_OP_AND = 19, ATF_OP_OR = 20, ATF_OP_NOT = 21
+};
+
+/* v1 limits */
+#define ATF_MAX_PARAMS 64
+#define ATF_MAX_RANGE (1 << 24)
+#define ATF_MAX_PROGRAM_WORDS 256
+#define ATF_MAX_STACK 16
+
+/* ---- building (state BUILDING) --------------------------------------------------- */
+
+/* Create an empty space.  opts may be NULL (device 0, default stream).  No CUDA
+ * work happens until atf_space_generate. */
+atf_status atf_space_create(const atf_space_opts* opts, atf_space** out);
+
+/* Add tuning parameter `name` (unique) with `range`.  The
+ * parameter id (declaration index) is written to *out_param_id. */
+atf_status atf_space_add_param(atf_space* s, const char* name, const atf_range* range,
+                               int32_t* out_param_id);
+
+/* Add a constraint program to parameter `param_id` (a callable on the
+ * parameter's value that may use earlier parameters).  Validated immediately
+ * (opcodes, stack discipline, backward references). */
+atf_status atf_space_add_constraint(atf_space* s, int32_t param_id, const int32_t* code,
+                                    int32_t n_words);
+
+/* ---- planning (host only; no GPU needed) ----------------------------------------- */
+
+/* Materialise ranges, run the static int64 interval analysis, partition the
+ * parameters into groups and compile each level's constraint program.
+ * BUILDING -> PLANNED.  Called implicitly by generate. */
+atf_status atf_space_plan(atf_space* s);
+
+atf_status atf_space_num_params(const atf_space* s, int32_t* out);
+atf_status atf_space_num_groups(const atf_space* s, int32_t* out);           /* >= PLANNED */
+/* members of group g (declaration order) -> out[0..n), n written to *n_out */
+atf_status atf_space_group_members(const atf_space* s, int32_t g, int32_t* out, int32_t cap,
+                                   int32_t* n_out);
+/* JSON description of the plan (groups, levels, record layout, compiled terms). */
+atf_status atf_space_plan_json(const atf_space* s, char* buf, size_t cap, size_t* len_out);
+
+/* ---- generation (GPU) ------------------------------------------------------------- */
+
+/* Generate every group's tree on the space's device/stream.  PLANNED (or
+ * BUILDING) -> GENERATED.  Synchronises the stream once per level round. */
+atf_status atf_space_generate(atf_space* s);
+
+/* Multi-GPU: generate this rank's shard (levels above the cut replicated, a
+ * contiguous balanced slice of the cut level expanded locally).  Writes this
+ * rank's per-level node counts (sum over groups of their level counts, in
+ * (group, level) order) to h_counts[0..n) (host), *n_out = n.  The caller
+ * all-gathers the counts across ranks (e.g. NCCL over NVLink) and passes them
+ * to atf_space_finalize_shard.  -> SHARDED. */
+atf_status atf_space_generate_shard(atf_space* s, int32_t rank, int32_t world, int64_t* h_counts,
+                                    int32_t cap, int32_t* n_out);
+/* h_all_counts: [world][n] host array of every rank's counts (rank-major).
+ * Computes the global level offsets of this rank's slice and the global group
+ * sizes.  SHARDED -> GENERATED (size/group_size become global; decode is not
+ * available on a shard: ATF_ERR_STATE). */
+atf_status atf_space_finalize_shard(atf_space* s, const int64_t* h_all_counts, int32_t world,
+                                    int32_t n);
+
+/* ---- results (state GENERATED) ---------------------------------------------------- */
+
+/* S = prod_g |G_g| as u128: *lo = low 64 bits, *hi = high 64 bits. */
+atf_status atf_space_size(const atf_space* s, uint64_t* lo, uint64_t* hi);
+atf_status atf_space_group_size(const atf_space* s, int32_t g, uint64_t* out);
+atf_status atf_space_num_levels(const atf_space* s, int32_t g, int32_t* out);
+/* f_k of group g (nodes at level k = 0..L-1, dead ends included); for a shard:
+ * this rank's local count. */
+atf_status atf_space_level_size(const atf_space* s, int32_t g, int32_t k, uint64_t* out);
+
+/* Level arrays of group g, level k (device pointers owned by the space):
+ *   records: [f_k][words] uint32, the range positions of the node's path
+ *            (field k' at bits [shift_k', shift_k'+bits_k') of word word_k');
+ *   csr:     [f_k + 1] uint64 first-child index in level k+1 (NULL for the leaf level);
+ *   offset:  global index of this array's first node (0 on one GPU). */
+typedef struct {
+  const uint32_t* records;
+  const uint64_t* csr;
+  uint64_t n_nodes;
+  uint64_t offset;
+  int32_t words;
+  int32_t param;     /* parameter id of level k */
+  int32_t field_word, field_shift, field_bits;
+} atf_level_view;
+atf_status atf_space_level_view(const atf_space* s, int32_t g, int32_t k, atf_level_view* out);
+
+/* Decode n 0-based indices (device uint64 d_idx[n], requires S < 2^64 else
+ * ATF_ERR_OVERFLOW) into configurations: d_out is int32 SoA, column p (the
+ * value of parameter p) at d_out + p*ld, ld >= n.  Rows whose index >= S are
+ * filled with INT32_MIN and the call returns ATF_ERR_INDEX (after a stream sync).
+ * Otherwise asynchronous on `stream` (NULL = the space's stream). */
+atf_status atf_space_decode_indices(const atf_space* s, const uint64_t* d_idx, int64_t n,
+                                    int32_t* d_out, int64_t ld, void* stream);
+/* Like decode_indices but with per-group digits: d_digits is [G][n] uint64
+ * (digit of group g at d_digits + g*n, each < |G_g|); works for any S. */
+atf_status atf_space_decode_digits(const atf_space* s, const uint64_t* d_digits, int64_t n,
+                                   int32_t* d_out, int64_t ld, void* stream);
+
+/* Per (group, level) statistics, in (group, level) order. */
+typedef struct {
+  int32_t group, level, param;
+  int64_t r;        /* range size r_k                         */
+  uint64_t evals;   /* candidate evaluations f_{k-1} * r_k    */
+  uint64_t f;       /* nodes f_k                              */
+  float ms;         /* device time of the level (ATF_FLAG_TIMING), else -1 */
+  int32_t path;     /* 0 = fast atoms, 1 = generic interpreter */
+} atf_level_stats;
+atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap, int32_t* n_out);
+
+/* Destroy (NULL ok).  Frees are stream-ordered on the space's stream. */
+void atf_space_destroy(atf_space* s);
+
+const char* atf_status_str(atf_status st);
+const char* atf_space_last_error(const atf_space* s);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* ATFGEN_H */

@@ -1,0 +1,137 @@
+// atf_internal.hpp — structures shared by the host planner (planner.cpp, api.cpp)
+// and the sm_100a kernels (kernels.cu).  Plain-old-data only: the level program is
+// passed to the kernels by value as a kernel parameter (constant bank).
+#pragma once
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __CUDACC__
+#define ATF_HD __host__ __device__ __forceinline__
+#else
+#define ATF_HD inline
+#endif
+
+namespace atf {
+
+constexpr int kMaxLevels = 64;   // parameters per group (= ATF_MAX_PARAMS)
+constexpr int kMaxSlots = 24;    // per-node int64 values (ancestor params + hoisted invariants)
+constexpr int kMaxTerms = 8;     // top-level conjuncts evaluated per candidate
+constexpr int kMaxCode = 448;    // device bytecode words per level (invariants + generic terms)
+constexpr int kMaxStack = 16;
+constexpr int kMaxGroups = 64;
+constexpr int kQTableMax = 16384;  // largest quotient with a shared-memory divisibility magic
+
+// Device bytecode = the ABI opcodes plus SLOT k (push per-node slot k).
+constexpr int32_t OP_SLOT = 32;
+
+// Candidate-dependent conjunct kinds ("atoms").
+enum TermKind : int32_t {
+  T_CMP = 1,      // (A * x) rel B                                  A, B per node
+  T_DIVX = 2,     // x | n        i.e. n mod x == 0, x == 0 rejects      A = |n|
+  T_MULX = 3,     // d | x        i.e. x mod d == 0 (d != 0: node gate)  A = |d|, B = magic(d)
+  T_DIVPROD = 4,  // (a*x) | b    -> gate a != 0 && a | b;  x | (b/a)    A = |b/a|
+  T_QDIV = 5,     // (num / x) | nb, quotient 0 or x == 0 rejects        A = |num|, B = |nb|
+  T_GENERIC = 6,  // any other conjunct: interpreted per candidate (code_off/code_len)
+};
+// arithmetic width the planner proved sufficient (static interval analysis)
+enum Variant : int32_t { V16 = 0, V32 = 1, V64 = 2 };
+enum Rel : int32_t { R_EQ = 11, R_NE = 12, R_LT = 13, R_LE = 14, R_GT = 15, R_GE = 16 };
+
+struct Term {
+  int32_t kind, variant, rel;
+  int32_t slot_a, slot_b;      // operand slots (meaning per kind)
+  int32_t code_off, code_len;  // T_GENERIC
+  int32_t use_qtable;          // T_QDIV V16: divisibility magic of the quotient from smem
+};
+
+// Per-level program + geometry, passed by value to the expand kernel.
+struct LevelArgs {
+  // frontier = level k-1 of this group (k == 0: a single empty root record)
+  const uint32_t* parent_rec;
+  uint64_t n_parents;
+  // candidates = materialised range of the level's parameter
+  const int32_t* cand;
+  int32_t r;
+  int32_t level;
+  int32_t field_word, field_shift;  // where the child's range position goes
+  // slots [0, n_pv): values of ancestor levels, decoded from the parent record
+  int32_t n_pv;
+  int32_t pv_word[kMaxSlots], pv_shift[kMaxSlots], pv_bits[kMaxSlots];
+  const int32_t* pv_range[kMaxSlots];
+  // slots [n_pv, n_slots): hoisted node-invariant expressions (code[inv_off..+inv_len))
+  int32_t n_slots;
+  int16_t inv_off[kMaxSlots], inv_len[kMaxSlots];
+  // node gates: slot values that must be nonzero (top-level invariant conjuncts)
+  int32_t n_gates;
+  int16_t gate_slot[kMaxTerms];
+  int32_t n_terms;
+  Term terms[kMaxTerms];
+  int32_t need_slots_smem;  // a generic term reads slots per candidate
+  int32_t need_m64;         // some term needs the 64-bit candidate magic
+  int32_t code[kMaxCode];
+  // outputs
+  uint32_t* child_rec;      // [f_k][W]
+  uint64_t* csr;            // [n_parents + 1]
+  unsigned long long* status;  // [n_tiles] decoupled look-back tile status
+  unsigned int* tile_counter;
+  unsigned long long* total_out;
+  uint64_t child_cap;       // capacity of child_rec in records
+  unsigned int* overflow_flag;
+  // geometry
+  int32_t block, cpt, npp, np;
+  int32_t tile_nodes;       // nodes per tile (np * npp), 1 if n_chunks > 1
+  int64_t n_chunks;         // candidate chunks per node (r > block*cpt)
+  uint64_t n_tiles;
+  uint32_t qmax;            // T_QDIV table covers quotients [0, qmax]
+  int32_t smem_bytes;
+};
+
+// Decode: index -> per-group digit (mixed radix, group 0 most significant) ->
+// leaf record -> range positions -> values.
+struct DecodeArgs {
+  int32_t n_groups;
+  int32_t n_params;
+  uint64_t gsize[kMaxGroups];
+  const uint32_t* leaves[kMaxGroups];
+  int32_t words[kMaxGroups];
+  int32_t lvl_begin[kMaxGroups + 1];   // levels of group g: [lvl_begin[g], lvl_begin[g+1])
+  int16_t lvl_param[kMaxLevels];
+  int16_t lvl_word[kMaxLevels], lvl_shift[kMaxLevels], lvl_bits[kMaxLevels];
+  const int32_t* lvl_range[kMaxLevels];
+};
+
+// Dynamic shared-memory layout of the expand kernel (byte offsets; -1 = absent).
+struct SmemLayout {
+  int ctl, ok, rec, opa, opb, slots, wcnt, wtot, qtab, total;
+};
+ATF_HD int align16(int x) { return (x + 15) & ~15; }
+ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
+  SmemLayout L;
+  const int tn = a.tile_nodes;
+  int o = 0;
+  L.ctl = o; o += 32;
+  L.ok = o; o = align16(o + 4 * tn);
+  L.rec = o; o = align16(o + 4 * words * tn);
+  L.opa = o; o = align16(o + 8 * a.n_terms * tn);
+  L.opb = o; o = align16(o + 8 * a.n_terms * tn);
+  if (a.need_slots_smem) { L.slots = o; o = align16(o + 8 * a.n_slots * tn); } else { L.slots = -1; }
+  L.wcnt = o; o = align16(o + 4 * (a.np * a.cpt * (a.block / 32) + 1));
+  L.wtot = o; o = align16(o + 4 * 33);
+  if (a.qmax > 0) { L.qtab = o; o = align16(o + 4 * ((int)a.qmax + 1)); } else { L.qtab = -1; }
+  L.total = o;
+  return L;
+}
+
+// ---- launch wrappers (kernels.cu) ------------------------------------------------
+// All return a cudaError_t value as int (0 = success).
+int launch_expand(const LevelArgs& a, int words, void* stream);
+int expand_smem_bytes(const LevelArgs& a, int words);
+int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out,
+                          int64_t ld, unsigned int* bad_flag, void* stream);
+int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,
+                         int64_t ld, unsigned int* bad_flag, void* stream);
+int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long long* status,
+                    unsigned int* counter, void* stream);
+int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
+
+}  // namespace atf

@@ -1,0 +1,1531 @@
+// atfgen.cpp — host side of libatfgen: the C ABI (include/atfgen.h), the planner
+// (range materialisation, bytecode validation, static int64 interval analysis,
+// group partition, hoisting + atom compilation of every level's constraint) and
+// the generation driver (per-group arenas, one fused expand launch per level).
+//
+// Citations: P:n = PAPER.md line n; SURVEY.md §8 is the hot-path contract.
+#include "../../include/atfgen.h"
+#include "../../include/atfgen_test.h"
+
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <functional>
+#include <map>
+#include <memory>
+#include <numeric>
+#include <string>
+#include <vector>
+
+#include "atf_internal.hpp"
+
+using namespace atf;
+using i128 = __int128;
+using u128 = unsigned __int128;
+
+namespace {
+
+enum State { BUILDING = 0, PLANNED = 1, GENERATED = 2, SHARDED = 3, FINAL_SHARD = 4 };
+
+struct ParamDef {
+  std::string name;
+  std::vector<int32_t> values;                 // materialised range
+  std::vector<std::vector<int32_t>> programs;  // ANDed constraints
+  int64_t vmin = 0, vmax = 0;
+};
+
+struct Iv {
+  i128 lo, hi;
+};
+const i128 I64MIN = (i128)INT64_MIN, I64MAX = (i128)INT64_MAX;
+bool fits64(const Iv& v) { return v.lo >= I64MIN && v.hi <= I64MAX; }
+i128 absmax(const Iv& v) {
+  i128 a = v.lo < 0 ? -v.lo : v.lo, b = v.hi < 0 ? -v.hi : v.hi;
+  return a > b ? a : b;
+}
+
+struct ENode {
+  int op = 0;
+  int a = -1, b = -1;
+  int64_t k = 0;  // PARAM id / CONST value
+  bool var = false;
+  Iv iv{0, 0};
+  std::string key;
+};
+
+struct LevelPlan {
+  int param = -1;
+  int r = 0;
+  int field_word = 0, field_shift = 0, field_bits = 0;
+  LevelArgs proto;           // program part only
+  std::vector<int> pv_param; // parameter id per ancestor slot
+  double cost = 0;           // algorithmic int ops per candidate evaluation (roofline)
+  bool generic = false;
+  std::string desc;
+};
+
+struct GroupPlan {
+  std::vector<int> members;
+  int words = 1;
+  std::vector<LevelPlan> levels;
+};
+
+struct Chunk {
+  char* p = nullptr;
+  size_t size = 0, used = 0;
+};
+
+struct LevelData {
+  uint32_t* rec = nullptr;
+  uint64_t* csr = nullptr;  // [n + 1], written when the next level is expanded
+  uint64_t n = 0;
+  uint64_t offset = 0;      // global index of rec[0] (shards)
+  uint64_t evals = 0;
+  float ms = -1.f;
+};
+
+}  // namespace
+
+struct atf_space {
+  atf_space_opts opts{};
+  int state = BUILDING;
+  std::string err;
+  std::vector<ParamDef> params;
+  std::vector<GroupPlan> groups;
+  std::vector<int> group_of;
+  // device state
+  bool dev_ready = false;
+  std::vector<int32_t*> d_range;
+  std::vector<std::vector<Chunk>> arena;  // per group
+  std::vector<std::vector<LevelData>> data;
+  std::vector<uint64_t> gsize;
+  unsigned long long* d_status = nullptr;
+  size_t status_cap = 0;
+  unsigned int* d_counter = nullptr;     // [kMaxGroups] tile counters
+  unsigned long long* d_totals = nullptr;  // [kMaxGroups]
+  unsigned int* d_ovf = nullptr;         // [kMaxGroups]
+  unsigned int* d_bad = nullptr;         // decode flag
+  uint32_t* d_root = nullptr;            // 8 zero words
+  unsigned long long* h_totals = nullptr;  // pinned
+  unsigned int* h_flags = nullptr;         // pinned
+  std::vector<std::vector<std::pair<cudaEvent_t, cudaEvent_t>>> events;
+  // shards
+  int shard_rank = 0, shard_world = 1;
+  std::vector<int> shard_cut;  // per group: first level expanded on a slice (L = none)
+};
+
+// ---------------------------------------------------------------- helpers
+static atf_status fail(atf_space* s, atf_status st, const char* fmt, ...) {
+  if (s) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    s->err = buf;
+  }
+  return st;
+}
+
+#define CUDA_TRY(s, call)                                                                          \
+  do {                                                                                             \
+    cudaError_t e_ = (call);                                                                       \
+    if (e_ != cudaSuccess) return fail((s), ATF_ERR_CUDA, "%s: %s", #call, cudaGetErrorString(e_)); \
+  } while (0)
+
+static void* dalloc(atf_space* s, size_t bytes) {
+  if (bytes == 0) bytes = 16;
+  void* p = nullptr;
+  if (s->opts.alloc) {
+    p = s->opts.alloc(bytes, s->opts.stream, s->opts.alloc_ctx);
+  } else {
+    if (cudaMallocAsync(&p, bytes, (cudaStream_t)s->opts.stream) != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+    }
+  }
+  return p;
+}
+static void dfree(atf_space* s, void* p, size_t bytes) {
+  if (!p) return;
+  if (s->opts.alloc) {
+    if (s->opts.free) s->opts.free(p, bytes, s->opts.stream, s->opts.alloc_ctx);
+  } else {
+    cudaFreeAsync(p, (cudaStream_t)s->opts.stream);
+  }
+}
+
+static int bits_for(int64_t r) {
+  int b = 0;
+  while (((int64_t)1 << b) < r) b++;
+  return b;
+}
+
+// ---------------------------------------------------------------- bytecode validation
+// opcodes 1..21, PARAM j with j < self (reading #10), exactly one
+// result, stack depth <= 16, <= 256 words.
+static atf_status validate_program(atf_space* s, int self, const int32_t* code, int n) {
+  if (n <= 0 || n > ATF_MAX_PROGRAM_WORDS) return fail(s, ATF_ERR_BYTECODE, "program length %d outside [1,256]", n);
+  int sp = 0;
+  for (int i = 0; i < n;) {
+    int op = code[i];
+    if (op == ATF_OP_X) { sp++; i++; }
+    else if (op == ATF_OP_PARAM) {
+      if (i + 1 >= n) return fail(s, ATF_ERR_BYTECODE, "PARAM without operand");
+      int j = code[i + 1];
+      if (j < 0 || j >= self)
+        return fail(s, ATF_ERR_FORWARD_REF, "parameter %d references parameter %d (only earlier ones allowed)", self, j);
+      sp++;
+      i += 2;
+    } else if (op == ATF_OP_CONST) {
+      if (i + 2 >= n) return fail(s, ATF_ERR_BYTECODE, "CONST without operands");
+      sp++;
+      i += 3;
+    } else if (op == ATF_OP_NOT) {
+      if (sp < 1) return fail(s, ATF_ERR_BYTECODE, "stack underflow at word %d", i);
+      i++;
+    } else if (op >= ATF_OP_ADD && op <= ATF_OP_OR) {
+      if (sp < 2) return fail(s, ATF_ERR_BYTECODE, "stack underflow at word %d", i);
+      sp--;
+      i++;
+    } else {
+      return fail(s, ATF_ERR_BYTECODE, "bad opcode %d at word %d", op, i);
+    }
+    if (sp > ATF_MAX_STACK) return fail(s, ATF_ERR_BYTECODE, "stack depth > %d", ATF_MAX_STACK);
+  }
+  if (sp != 1) return fail(s, ATF_ERR_BYTECODE, "program leaves %d items (must be 1)", sp);
+  return ATF_OK;
+}
+
+// ---------------------------------------------------------------- expression trees
+struct Tree {
+  std::vector<ENode> nodes;
+  int add(ENode n) {
+    nodes.push_back(std::move(n));
+    return (int)nodes.size() - 1;
+  }
+};
+
+static const char* opname(int op) {
+  static const char* names[] = {"?", "X", "PARAM", "CONST", "ADD", "SUB", "MUL", "DIV", "MOD", "MIN", "MAX", "EQ",
+                                "NE", "LT", "LE", "GT", "GE", "DIVIDES", "MULOF", "AND", "OR", "NOT"};
+  return (op >= 1 && op <= 21) ? names[op] : "?";
+}
+
+// interval of a binary op; false on possible int64 overflow (reading #9)
+static bool binop_iv(int op, const Iv& a, const Iv& b, Iv& out) {
+  auto mk = [&](i128 x, i128 y) { out = Iv{std::min(x, y), std::max(x, y)}; };
+  switch (op) {
+    case ATF_OP_ADD: out = Iv{a.lo + b.lo, a.hi + b.hi}; break;
+    case ATF_OP_SUB: out = Iv{a.lo - b.hi, a.hi - b.lo}; break;
+    case ATF_OP_MUL: {
+      i128 c[4] = {a.lo * b.lo, a.lo * b.hi, a.hi * b.lo, a.hi * b.hi};
+      out = Iv{*std::min_element(c, c + 4), *std::max_element(c, c + 4)};
+      break;
+    }
+    case ATF_OP_DIV: {
+      if (a.lo == I64MIN && b.lo <= -1 && b.hi >= -1) return false;  // INT64_MIN / -1
+      if (a.lo >= 0 && b.lo > 0) mk(a.lo / b.hi, a.hi / b.lo);
+      else { i128 m = absmax(a); out = Iv{-m, m}; }
+      break;
+    }
+    case ATF_OP_MOD: {
+      i128 mb = absmax(b) - 1;
+      if (mb < 0) mb = 0;
+      i128 ma = absmax(a);
+      i128 m = std::min(ma, mb);
+      if (a.lo >= 0) out = Iv{0, m};
+      else if (a.hi <= 0) out = Iv{-m, 0};
+      else out = Iv{-m, m};
+      break;
+    }
+    case ATF_OP_MIN: out = Iv{std::min(a.lo, b.lo), std::min(a.hi, b.hi)}; break;
+    case ATF_OP_MAX: out = Iv{std::max(a.lo, b.lo), std::max(a.hi, b.hi)}; break;
+    default: out = Iv{0, 1}; break;
+  }
+  return fits64(out);
+}
+
+// Parse a validated program into the tree; returns the root node or -1 on overflow.
+static int parse_program(const std::vector<int32_t>& code, const std::vector<ParamDef>& P, const Iv& xiv, Tree& t,
+                         std::string* why) {
+  std::vector<int> st;
+  for (size_t i = 0; i < code.size();) {
+    int op = code[i];
+    ENode n;
+    n.op = op;
+    if (op == ATF_OP_X) {
+      n.var = true;
+      n.iv = xiv;
+      n.key = "X";
+      i++;
+    } else if (op == ATF_OP_PARAM) {
+      n.k = code[i + 1];
+      n.iv = Iv{P[n.k].vmin, P[n.k].vmax};
+      n.key = "P" + std::to_string(n.k);
+      i += 2;
+    } else if (op == ATF_OP_CONST) {
+      n.k = (int64_t)(((uint64_t)(uint32_t)code[i + 2] << 32) | (uint64_t)(uint32_t)code[i + 1]);
+      n.iv = Iv{n.k, n.k};
+      n.key = "C" + std::to_string(n.k);
+      i += 3;
+    } else if (op == ATF_OP_NOT) {
+      n.a = st.back();
+      st.pop_back();
+      n.var = t.nodes[n.a].var;
+      n.iv = Iv{0, 1};
+      n.key = "(" + t.nodes[n.a].key + " NOT)";
+      i++;
+    } else {
+      n.b = st.back();
+      st.pop_back();
+      n.a = st.back();
+      st.pop_back();
+      const ENode &A = t.nodes[n.a], &B = t.nodes[n.b];
+      n.var = A.var || B.var;
+      if (!binop_iv(op, A.iv, B.iv, n.iv)) {
+        if (why) *why = std::string("possible int64 overflow in ") + opname(op);
+        return -1;
+      }
+      n.key = "(" + A.key + " " + B.key + " " + opname(op) + ")";
+      i++;
+    }
+    st.push_back(t.add(std::move(n)));
+  }
+  return st.back();
+}
+
+// ---------------------------------------------------------------- level compiler
+struct LevelCompiler {
+  const std::vector<ParamDef>& P;
+  Tree& t;
+  LevelArgs& a;
+  std::vector<int>& pv_param;
+  std::map<std::string, int> slot_of_key;
+  std::vector<int32_t> code;
+  std::string err;
+  int n_slots = 0;
+
+  LevelCompiler(const std::vector<ParamDef>& P_, Tree& t_, LevelArgs& a_, std::vector<int>& pv)
+      : P(P_), t(t_), a(a_), pv_param(pv) {}
+
+  int pv_slot(int param) {
+    for (size_t s = 0; s < pv_param.size(); s++)
+      if (pv_param[s] == param) return (int)s;
+    return -1;
+  }
+  // postfix code of a node; invariant subtrees become SLOT refs when `hoist`
+  bool emit(int ni, std::vector<int32_t>& out, bool hoist) {
+    const ENode& n = t.nodes[ni];
+    if (hoist && !n.var) {
+      int s = slot(ni);
+      if (s < 0) return false;
+      out.push_back(OP_SLOT);
+      out.push_back(s);
+      return true;
+    }
+    switch (n.op) {
+      case ATF_OP_X: out.push_back(ATF_OP_X); return true;
+      case ATF_OP_PARAM: out.push_back(OP_SLOT); out.push_back(pv_slot((int)n.k)); return true;
+      case ATF_OP_CONST:
+        out.push_back(ATF_OP_CONST);
+        out.push_back((int32_t)(uint32_t)((uint64_t)n.k & 0xffffffffu));
+        out.push_back((int32_t)(uint32_t)((uint64_t)n.k >> 32));
+        return true;
+      case ATF_OP_NOT:
+        if (!emit(n.a, out, hoist)) return false;
+        out.push_back(ATF_OP_NOT);
+        return true;
+      default:
+        if (!emit(n.a, out, hoist) || !emit(n.b, out, hoist)) return false;
+        out.push_back(n.op);
+        return true;
+    }
+  }
+  // slot holding the value of invariant node ni (deduplicated by structure)
+  int slot(int ni) {
+    const ENode& n = t.nodes[ni];
+    if (n.op == ATF_OP_PARAM) return pv_slot((int)n.k);
+    auto it = slot_of_key.find(n.key);
+    if (it != slot_of_key.end()) return it->second;
+    if (n_slots >= kMaxSlots) { err = "too many hoisted invariants"; return -1; }
+    std::vector<int32_t> c;
+    if (!emit(ni, c, false)) return -1;
+    if (code.size() + c.size() > (size_t)kMaxCode) { err = "level program too long"; return -1; }
+    int s = n_slots++;
+    a.inv_off[s] = (int16_t)code.size();
+    a.inv_len[s] = (int16_t)c.size();
+    code.insert(code.end(), c.begin(), c.end());
+    slot_of_key[n.key] = s;
+    return s;
+  }
+  int mk_const(int64_t v) {
+    ENode n;
+    n.op = ATF_OP_CONST;
+    n.k = v;
+    n.iv = Iv{v, v};
+    n.key = "C" + std::to_string(v);
+    return t.add(n);
+  }
+  int mk_bin(int op, int x, int y) {  // invariant binary node; -1 on overflow
+    ENode n;
+    n.op = op;
+    n.a = x;
+    n.b = y;
+    n.var = t.nodes[x].var || t.nodes[y].var;
+    if (!binop_iv(op, t.nodes[x].iv, t.nodes[y].iv, n.iv)) return -1;
+    n.key = "(" + t.nodes[x].key + " " + t.nodes[y].key + " " + opname(op) + ")";
+    return t.add(n);
+  }
+};
+
+static void flatten_and(const Tree& t, int ni, std::vector<int>& out) {
+  const ENode& n = t.nodes[ni];
+  if (n.op == ATF_OP_AND) {
+    flatten_and(t, n.a, out);
+    flatten_and(t, n.b, out);
+  } else {
+    out.push_back(ni);
+  }
+}
+
+static int flip_rel(int rel) {
+  switch (rel) {
+    case R_LT: return R_GT;
+    case R_GT: return R_LT;
+    case R_LE: return R_GE;
+    case R_GE: return R_LE;
+    default: return rel;
+  }
+}
+
+static const double kCost[] = {0, 2, 2, 2, 2, 6, 0};  // per TermKind (T_GENERIC: op count)
+
+// Compile the constraint of level `lv` (parameter p) of a group.  Fills lp.proto's
+// program part.  Returns ATF_OK or an error with message in *why.
+static atf_status compile_level(const std::vector<ParamDef>& P, int p, const std::vector<int>& members, int lv,
+                                const std::vector<int>& field_word, const std::vector<int>& field_shift,
+                                const std::vector<int>& field_bits, bool generic_only, LevelPlan& lp,
+                                std::string* why) {
+  LevelArgs& a = lp.proto;
+  std::memset(&a, 0, sizeof a);
+  const ParamDef& pd = P[p];
+  const Iv xiv{pd.vmin, pd.vmax};
+  i128 xabs = absmax(xiv);
+  Tree t;
+  std::vector<int> roots;
+  for (auto& code : pd.programs) {
+    int root = parse_program(code, P, xiv, t, why);
+    if (root < 0) return ATF_ERR_OVERFLOW;
+    roots.push_back(root);
+  }
+  // ancestor slots: every parameter referenced by the level's programs
+  std::vector<int> refs;
+  for (auto& n : t.nodes)
+    if (n.op == ATF_OP_PARAM && std::find(refs.begin(), refs.end(), (int)n.k) == refs.end()) refs.push_back((int)n.k);
+  std::sort(refs.begin(), refs.end());
+  if ((int)refs.size() > kMaxSlots) { *why = "too many referenced parameters"; return ATF_ERR_LIMIT; }
+  lp.pv_param = refs;
+  a.n_pv = (int)refs.size();
+  for (int s = 0; s < a.n_pv; s++) {
+    int l = (int)(std::find(members.begin(), members.end(), refs[s]) - members.begin());
+    if (l >= lv) { *why = "internal: reference outside the group prefix"; return ATF_ERR_FORWARD_REF; }
+    a.pv_word[s] = field_word[l];
+    a.pv_shift[s] = field_shift[l];
+    a.pv_bits[s] = field_bits[l];
+  }
+  LevelCompiler lc(P, t, a, lp.pv_param);
+  lc.n_slots = a.n_pv;
+  std::vector<Term> terms;
+  std::vector<int> gates;
+  std::vector<std::string> desc, gdesc;
+  auto add_generic = [&](int ni) -> bool {
+    std::vector<int32_t> c;
+    if (!lc.emit(ni, c, !generic_only)) return false;
+    Term T{};
+    T.kind = T_GENERIC;
+    T.code_off = (int)lc.code.size();
+    T.code_len = (int)c.size();
+    if (lc.code.size() + c.size() > (size_t)kMaxCode) { lc.err = "level program too long"; return false; }
+    lc.code.insert(lc.code.end(), c.begin(), c.end());
+    terms.push_back(T);
+    desc.push_back("GENERIC" + std::string(" ") + t.nodes[ni].key);
+    return true;
+  };
+  std::vector<int> conj;
+  for (int root : roots) flatten_and(t, root, conj);
+  if (generic_only) {
+    // one interpreted term per program: no hoisting, no atoms (baseline path)
+    for (int root : roots)
+      if (!add_generic(root)) { *why = lc.err; return ATF_ERR_LIMIT; }
+  } else {
+    for (int ci : conj) {
+      const ENode& n = t.nodes[ci];
+      if (!n.var) {  // node-invariant conjunct -> node gate
+        int s = lc.slot(ci);
+        if (s < 0) { *why = lc.err; return ATF_ERR_LIMIT; }
+        gates.push_back(s);
+        gdesc.push_back("GATE " + n.key);
+        continue;
+      }
+      Term T{};
+      bool matched = false;
+      auto isX = [&](int i) { return t.nodes[i].op == ATF_OP_X; };
+      auto inv = [&](int i) { return !t.nodes[i].var; };
+      // DIVIDES(d, m): d | m.  MULOF(m, d) is the same test with the same poison (d == 0).
+      int d = -1, m = -1;
+      if (n.op == ATF_OP_DIVIDES) { d = n.a; m = n.b; }
+      if (n.op == ATF_OP_MULOF) { d = n.b; m = n.a; }
+      if (d >= 0) {
+        const ENode& D = t.nodes[d];
+        if (isX(d) && inv(m)) {  // x | m
+          T.kind = T_DIVX;
+          T.slot_a = lc.slot(m);
+          i128 nm = absmax(t.nodes[m].iv);
+          T.variant = (xabs < 65536 && nm < 65536) ? V16 : (nm < ((i128)1 << 32) ? V32 : V64);
+          matched = T.slot_a >= 0;
+        } else if (inv(d) && isX(m)) {  // d | x
+          T.kind = T_MULX;
+          T.slot_a = lc.slot(d);
+          i128 dm = absmax(D.iv);
+          T.variant = (xabs < 65536 && dm < 65536) ? V16 : (dm < ((i128)1 << 32) ? V32 : V64);
+          matched = T.slot_a >= 0;
+        } else if (D.op == ATF_OP_MUL && inv(m) && ((isX(D.a) && inv(D.b)) || (inv(D.a) && isX(D.b)))) {
+          // (a*x) | m  ->  gate a != 0 && a | m;  x | (m / a)
+          int an = isX(D.a) ? D.b : D.a;
+          T.kind = T_DIVPROD;
+          T.slot_a = lc.slot(an);
+          T.slot_b = lc.slot(m);
+          i128 nm = absmax(t.nodes[m].iv);
+          T.variant = (xabs < 65536 && nm < 65536) ? V16 : (nm < ((i128)1 << 32) ? V32 : V64);
+          matched = T.slot_a >= 0 && T.slot_b >= 0;
+        } else if (D.op == ATF_OP_DIV && inv(D.a) && isX(D.b) && inv(m)) {
+          // (num / x) | m
+          T.kind = T_QDIV;
+          T.slot_a = lc.slot(D.a);
+          T.slot_b = lc.slot(m);
+          i128 nu = absmax(t.nodes[D.a].iv), nb = absmax(t.nodes[m].iv);
+          if (xabs < 65536 && nu < 65536 && nb < 65536) {
+            T.variant = V16;
+            T.use_qtable = nu <= kQTableMax ? 1 : 0;
+            if (T.use_qtable) a.qmax = std::max<uint32_t>(a.qmax, (uint32_t)nu);
+          } else {
+            T.variant = (nu < ((i128)1 << 32) && nb < ((i128)1 << 32)) ? V32 : V64;
+          }
+          matched = T.slot_a >= 0 && T.slot_b >= 0;
+        }
+      } else if (n.op >= ATF_OP_EQ && n.op <= ATF_OP_GE) {
+        int vs = -1, is = -1, rel = n.op;
+        if (t.nodes[n.a].var && inv(n.b)) { vs = n.a; is = n.b; }
+        else if (inv(n.a) && t.nodes[n.b].var) { vs = n.b; is = n.a; rel = flip_rel(rel); }
+        if (vs >= 0) {
+          // affine side: x, a*x, x*a, x+c, c+x, x-c, c-x  ->  (m*x + c) rel v  ->  m*x rel v - c
+          const ENode& V = t.nodes[vs];
+          int mnode = -1, cnode = -1;
+          bool neg_c = false;
+          if (isX(vs)) { mnode = lc.mk_const(1); }
+          else if (V.op == ATF_OP_MUL && isX(V.a) && inv(V.b)) { mnode = V.b; }
+          else if (V.op == ATF_OP_MUL && inv(V.a) && isX(V.b)) { mnode = V.a; }
+          else if (V.op == ATF_OP_ADD && isX(V.a) && inv(V.b)) { mnode = lc.mk_const(1); cnode = V.b; }
+          else if (V.op == ATF_OP_ADD && inv(V.a) && isX(V.b)) { mnode = lc.mk_const(1); cnode = V.a; }
+          else if (V.op == ATF_OP_SUB && isX(V.a) && inv(V.b)) { mnode = lc.mk_const(1); cnode = V.b; neg_c = true; }
+          else if (V.op == ATF_OP_SUB && inv(V.a) && isX(V.b)) { mnode = lc.mk_const(-1); cnode = V.a; }
+          if (mnode >= 0) {
+            int vnode = is;
+            if (cnode >= 0) vnode = lc.mk_bin(neg_c ? ATF_OP_ADD : ATF_OP_SUB, is, cnode);
+            if (vnode >= 0) {
+              Iv prod;
+              bool ok = binop_iv(ATF_OP_MUL, t.nodes[mnode].iv, xiv, prod);
+              if (ok) {
+                T.kind = T_CMP;
+                T.rel = rel;
+                T.slot_a = lc.slot(mnode);
+                T.slot_b = lc.slot(vnode);
+                const Iv& vi = t.nodes[vnode].iv;
+                bool f32 = prod.lo >= INT32_MIN && prod.hi <= INT32_MAX && vi.lo >= INT32_MIN && vi.hi <= INT32_MAX &&
+                           t.nodes[mnode].iv.lo >= INT32_MIN && t.nodes[mnode].iv.hi <= INT32_MAX;
+                T.variant = f32 ? V32 : V64;
+                matched = T.slot_a >= 0 && T.slot_b >= 0;
+              }
+            }
+          }
+        }
+      } else if (isX(ci)) {  // bare x as a conjunct: x != 0
+        T.kind = T_CMP;
+        T.rel = R_NE;
+        T.slot_a = lc.slot(lc.mk_const(1));
+        T.slot_b = lc.slot(lc.mk_const(0));
+        T.variant = V32;
+        matched = T.slot_a >= 0 && T.slot_b >= 0;
+      }
+      if (!lc.err.empty()) { *why = lc.err; return ATF_ERR_LIMIT; }
+      if (matched) {
+        terms.push_back(T);
+        static const char* kn[] = {"?", "CMP", "DIVX", "MULX", "DIVPROD", "QDIV", "GENERIC"};
+        static const char* vn[] = {"16", "32", "64"};
+        desc.push_back(std::string(kn[T.kind]) + "/" + vn[T.variant] + " " + n.key);
+      } else if (!add_generic(ci)) {
+        *why = lc.err;
+        return ATF_ERR_LIMIT;
+      }
+    }
+  }
+  // cheapest conjuncts first (top-level AND: order changes neither result nor poison-reject)
+  std::vector<size_t> order(terms.size());
+  std::iota(order.begin(), order.end(), 0);
+  auto cost_of = [&](const Term& T) { return T.kind == T_GENERIC ? 10.0 + T.code_len : kCost[T.kind]; };
+  std::stable_sort(order.begin(), order.end(), [&](size_t x, size_t y) { return cost_of(terms[x]) < cost_of(terms[y]); });
+  if ((int)terms.size() > kMaxTerms) { *why = "too many conjuncts"; return ATF_ERR_LIMIT; }
+  if ((int)gates.size() > kMaxTerms) { *why = "too many invariant conjuncts"; return ATF_ERR_LIMIT; }
+  a.n_terms = (int)terms.size();
+  lp.cost = 0;
+  lp.generic = false;
+  std::string d;
+  for (size_t i = 0; i < order.size(); i++) {
+    const Term& T = terms[order[i]];
+    a.terms[i] = T;
+    if (T.kind == T_GENERIC) {
+      a.need_slots_smem = 1;
+      lp.generic = true;
+      int ops = 0;
+      for (int w = T.code_off; w < T.code_off + T.code_len;) {
+        int op = lc.code[w];
+        ops++;
+        w += (op == OP_SLOT) ? 2 : (op == ATF_OP_CONST ? 3 : 1);
+      }
+      lp.cost += ops;
+    } else {
+      lp.cost += kCost[T.kind];
+    }
+    if (T.kind == T_DIVX || T.kind == T_DIVPROD || T.kind == T_MULX || T.kind == T_QDIV)
+      if (T.variant == V32) a.need_m64 = 1;
+    d += (i ? " & " : "") + desc[order[i]];
+  }
+  if (a.n_terms > 1) lp.cost += a.n_terms - 1;  // the ANDs
+  a.n_gates = (int)gates.size();
+  for (size_t i = 0; i < gates.size(); i++) {
+    a.gate_slot[i] = (int16_t)gates[i];
+    d += std::string(d.empty() ? "" : " & ") + gdesc[i];
+  }
+  a.n_slots = lc.n_slots;
+  if (lc.code.size() > (size_t)kMaxCode) { *why = "level program too long"; return ATF_ERR_LIMIT; }
+  std::copy(lc.code.begin(), lc.code.end(), a.code);
+  lp.desc = d.empty() ? "TRUE" : d;
+  return ATF_OK;
+}
+
+// ---------------------------------------------------------------- planning
+static atf_status plan(atf_space* s) {
+  if (s->state != BUILDING) return ATF_OK;
+  int n = (int)s->params.size();
+  // groups: connected components of p -- q for every q referenced by p's constraints
+  // (groups ordered by first member, members in declaration order)
+  std::vector<int> parent(n);
+  std::iota(parent.begin(), parent.end(), 0);
+  std::function<int(int)> find = [&](int x) { return parent[x] == x ? x : parent[x] = find(parent[x]); };
+  for (int p = 0; p < n; p++)
+    for (auto& code : s->params[p].programs)
+      for (size_t i = 0; i < code.size();) {
+        int op = code[i];
+        if (op == ATF_OP_PARAM) {
+          int a = find(p), b = find(code[i + 1]);
+          if (a != b) parent[std::max(a, b)] = std::min(a, b);
+          i += 2;
+        } else {
+          i += (op == ATF_OP_CONST) ? 3 : 1;
+        }
+      }
+  s->groups.clear();
+  s->group_of.assign(n, -1);
+  std::map<int, int> gid;
+  for (int p = 0; p < n; p++) {
+    int root = find(p);
+    auto it = gid.find(root);
+    if (it == gid.end()) {
+      gid[root] = (int)s->groups.size();
+      s->groups.push_back(GroupPlan{});
+      it = gid.find(root);
+    }
+    s->groups[it->second].members.push_back(p);
+    s->group_of[p] = it->second;
+  }
+  if ((int)s->groups.size() > kMaxGroups) return fail(s, ATF_ERR_LIMIT, "more than %d groups", kMaxGroups);
+  for (auto& g : s->groups) {
+    // record layout: each level's range position gets ceil(log2 r) bits; fields are
+    // packed first-fit-decreasing into 32-bit words (no field straddles a word)
+    size_t L = g.members.size();
+    std::vector<int> fw(L, 0), fs(L, 0), fb(L, 0);
+    for (size_t l = 0; l < L; l++) fb[l] = bits_for((int64_t)s->params[g.members[l]].values.size());
+    std::vector<size_t> ord(L);
+    std::iota(ord.begin(), ord.end(), 0);
+    std::stable_sort(ord.begin(), ord.end(), [&](size_t x, size_t y) { return fb[x] > fb[y]; });
+    std::vector<int> fill;
+    for (size_t l : ord) {
+      size_t w = 0;
+      while (w < fill.size() && fill[w] + fb[l] > 32) w++;
+      if (w == fill.size()) fill.push_back(0);
+      fw[l] = (int)w;
+      fs[l] = fill[w];
+      fill[w] += fb[l];
+    }
+    int words = std::max<int>(1, (int)fill.size());
+    if (words > 8) return fail(s, ATF_ERR_LIMIT, "group path record needs %d words (> 8)", words);
+    g.words = words <= 1 ? 1 : words <= 2 ? 2 : words <= 4 ? 4 : 8;
+    g.levels.clear();
+    for (size_t l = 0; l < g.members.size(); l++) {
+      LevelPlan lp;
+      int p = g.members[l];
+      lp.param = p;
+      lp.r = (int)s->params[p].values.size();
+      lp.field_word = fw[l];
+      lp.field_shift = fs[l];
+      lp.field_bits = fb[l];
+      std::string why;
+      atf_status st = compile_level(s->params, p, g.members, (int)l, fw, fs, fb,
+                                    (s->opts.flags & ATF_FLAG_GENERIC_ONLY) != 0, lp, &why);
+      if (st != ATF_OK) return fail(s, st, "parameter %s: %s", s->params[p].name.c_str(), why.c_str());
+      lp.proto.level = (int)l;
+      lp.proto.field_word = fw[l];
+      lp.proto.field_shift = fs[l];
+      g.levels.push_back(lp);
+    }
+  }
+  s->state = PLANNED;
+  return ATF_OK;
+}
+
+// ---------------------------------------------------------------- geometry
+static void choose_geometry(LevelArgs& a, int words) {
+  const int r = a.r;
+  int B, cpt = 1, npp = 1;
+  int64_t n_chunks = 1;
+  if (r <= 1024) {
+    int best = -1;
+    double bu = -1;
+    for (int b = 32; b <= 1024; b += 32) {
+      if (b < r) continue;
+      int k = b / r;
+      double u = (double)k * r / b;
+      // prefer utilisation, then ~512 threads
+      double score = u - 1e-4 * std::abs(b - 512) / 512.0;
+      if (b < 256 && r < 256) score -= 1e-3;
+      if (score > bu) { bu = score; best = b; }
+    }
+    B = best;
+    npp = B / r;
+  } else {
+    cpt = 2;
+    while (cpt < 8 && (r + cpt - 1) / cpt > 512) cpt *= 2;
+    int per = (r + cpt - 1) / cpt;
+    if (per > 512) per = 512;
+    B = (per + 31) / 32 * 32;
+    n_chunks = ((int64_t)r + (int64_t)B * cpt - 1) / ((int64_t)B * cpt);
+  }
+  a.block = B;
+  a.cpt = cpt;
+  a.npp = npp;
+  a.n_chunks = n_chunks;
+  // passes per tile: bounded by 32 bits per thread and ~96 KB of shared memory
+  int per_node = 4 + 4 * words + 16 * a.n_terms + (a.need_slots_smem ? 8 * a.n_slots : 0);
+  int NW = B / 32;
+  int np = n_chunks > 1 ? 1 : 32 / cpt;
+  while (np > 1) {
+    a.np = np;
+    a.tile_nodes = np * npp;
+    if (expand_layout(a, words).total <= 96 * 1024) break;
+    np--;
+  }
+  (void)per_node;
+  (void)NW;
+  a.np = np;
+  a.tile_nodes = n_chunks > 1 ? 1 : np * npp;
+  a.smem_bytes = expand_layout(a, words).total;
+}
+
+// ---------------------------------------------------------------- device setup
+static atf_status ensure_device(atf_space* s) {
+  CUDA_TRY(s, cudaSetDevice(s->opts.device));
+  if (s->dev_ready) return ATF_OK;
+  size_t np = s->params.size();
+  s->d_range.assign(np, nullptr);
+  for (size_t p = 0; p < np; p++) {
+    auto& v = s->params[p].values;
+    s->d_range[p] = (int32_t*)dalloc(s, std::max<size_t>(4, v.size() * 4));
+    if (!s->d_range[p]) return fail(s, ATF_ERR_OOM, "range upload");
+    if (!v.empty())
+      CUDA_TRY(s, cudaMemcpyAsync(s->d_range[p], v.data(), v.size() * 4, cudaMemcpyHostToDevice,
+                                  (cudaStream_t)s->opts.stream));
+  }
+  s->d_counter = (unsigned int*)dalloc(s, 4 * kMaxGroups);
+  s->d_totals = (unsigned long long*)dalloc(s, 8 * kMaxGroups);
+  s->d_ovf = (unsigned int*)dalloc(s, 4 * kMaxGroups);
+  s->d_bad = (unsigned int*)dalloc(s, 16);
+  s->d_root = (uint32_t*)dalloc(s, 64);
+  if (!s->d_counter || !s->d_totals || !s->d_ovf || !s->d_bad || !s->d_root) return fail(s, ATF_ERR_OOM, "scratch");
+  CUDA_TRY(s, cudaMemsetAsync(s->d_root, 0, 64, (cudaStream_t)s->opts.stream));
+  CUDA_TRY(s, cudaMallocHost(&s->h_totals, 8 * kMaxGroups));
+  CUDA_TRY(s, cudaMallocHost(&s->h_flags, 4 * kMaxGroups));
+  s->arena.assign(s->groups.size(), {});
+  s->dev_ready = true;
+  return ATF_OK;
+}
+
+static atf_status ensure_status(atf_space* s, size_t tiles) {
+  if (tiles <= s->status_cap) return ATF_OK;
+  dfree(s, s->d_status, s->status_cap * 8);
+  size_t cap = std::max<size_t>(tiles, s->status_cap * 2);
+  s->d_status = (unsigned long long*)dalloc(s, cap * 8);
+  if (!s->d_status) { s->status_cap = 0; return fail(s, ATF_ERR_OOM, "tile status (%zu tiles)", cap); }
+  s->status_cap = cap;
+  return ATF_OK;
+}
+
+// bump allocation inside group g's arena; nullptr if no chunk has room
+static char* arena_alloc(atf_space* s, int g, size_t bytes) {
+  bytes = (bytes + 255) & ~(size_t)255;
+  for (auto& c : s->arena[g])
+    if (c.size - c.used >= bytes) {
+      char* p = c.p + c.used;
+      c.used += bytes;
+      return p;
+    }
+  return nullptr;
+}
+static atf_status arena_grow(atf_space* s, int g, size_t need) {
+  size_t total = 0;
+  for (auto& c : s->arena[g]) total += c.size;
+  size_t sz = std::max<size_t>({need + (need >> 3) + (1 << 20), total, (size_t)64 << 20});
+  Chunk c;
+  c.p = (char*)dalloc(s, sz);
+  if (!c.p) return fail(s, ATF_ERR_OOM, "arena chunk of %zu bytes", sz);
+  c.size = sz;
+  s->arena[g].push_back(c);
+  return ATF_OK;
+}
+// largest free tail of the arena (chunk index, bytes)
+static size_t arena_tail(atf_space* s, int g, int* which) {
+  size_t best = 0;
+  *which = -1;
+  for (size_t i = 0; i < s->arena[g].size(); i++) {
+    auto& c = s->arena[g][i];
+    if (c.size - c.used > best) { best = c.size - c.used; *which = (int)i; }
+  }
+  return best;
+}
+
+static void release_device(atf_space* s) {
+  for (size_t g = 0; g < s->arena.size(); g++)
+    for (auto& c : s->arena[g]) dfree(s, c.p, c.size);
+  s->arena.clear();
+  for (size_t p = 0; p < s->d_range.size(); p++) dfree(s, s->d_range[p], 4 * s->params[p].values.size());
+  s->d_range.clear();
+  dfree(s, s->d_status, s->status_cap * 8);
+  dfree(s, s->d_counter, 4 * kMaxGroups);
+  dfree(s, s->d_totals, 8 * kMaxGroups);
+  dfree(s, s->d_ovf, 4 * kMaxGroups);
+  dfree(s, s->d_bad, 16);
+  dfree(s, s->d_root, 64);
+  if (s->h_totals) cudaFreeHost(s->h_totals);
+  if (s->h_flags) cudaFreeHost(s->h_flags);
+  for (auto& ev : s->events)
+    for (auto& e : ev) {
+      cudaEventDestroy(e.first);
+      cudaEventDestroy(e.second);
+    }
+  s->events.clear();
+  s->d_status = nullptr;
+  s->h_totals = nullptr;
+  s->h_flags = nullptr;
+  s->dev_ready = false;
+}
+
+// ---------------------------------------------------------------- generation driver
+// Expand level k of group g from `parents` (n_parents nodes) into the group's arena.
+// Queues work only; the level total lands in d_totals[g].
+struct Pending {
+  int g, k;
+  uint64_t n_parents;
+  const uint32_t* parents;
+  uint64_t* csr;
+  uint32_t* child;
+  uint64_t cap;
+  int chunk;  // arena chunk holding the child region
+  size_t child_off;
+};
+
+static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parents, uint64_t n_parents, Pending& pd,
+                              uint64_t tile_base_unused = 0) {
+  (void)tile_base_unused;
+  GroupPlan& gp = s->groups[g];
+  LevelPlan& lp = gp.levels[k];
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  LevelArgs a = lp.proto;
+  a.parent_rec = parents;
+  a.n_parents = n_parents;
+  a.cand = s->d_range[lp.param];
+  a.r = lp.r;
+  for (int i = 0; i < a.n_pv; i++) a.pv_range[i] = s->d_range[lp.pv_param[i]];
+  choose_geometry(a, gp.words);
+  a.n_tiles = a.n_chunks > 1 ? n_parents * (uint64_t)a.n_chunks
+                             : (n_parents + (uint64_t)a.tile_nodes - 1) / (uint64_t)a.tile_nodes;
+  if (a.n_tiles >= 0xffffffffull) return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %llu tiles", k, g,
+                                              (unsigned long long)a.n_tiles);
+  atf_status e = ensure_status(s, a.n_tiles);
+  if (e) return e;
+  // CSR of the parent level (exact size), then the child region = largest free tail
+  size_t csr_bytes = (n_parents + 1) * 8;
+  char* csr = arena_alloc(s, g, csr_bytes);
+  if (!csr) {
+    if ((e = arena_grow(s, g, csr_bytes + n_parents * gp.words * 4))) return e;
+    csr = arena_alloc(s, g, csr_bytes);
+  }
+  int which = -1;
+  size_t tail = arena_tail(s, g, &which);
+  if (tail < (size_t)gp.words * 4 * 64) {
+    if ((e = arena_grow(s, g, std::max<size_t>(n_parents * gp.words * 4, 1 << 20)))) return e;
+    tail = arena_tail(s, g, &which);
+  }
+  Chunk& c = s->arena[g][which];
+  size_t off = (c.used + 255) & ~(size_t)255;
+  uint32_t* child = (uint32_t*)(c.p + off);
+  uint64_t cap = (c.size - off) / (gp.words * 4);
+  a.child_rec = child;
+  a.child_cap = cap;
+  a.csr = (uint64_t*)csr;
+  a.status = s->d_status;
+  a.tile_counter = s->d_counter + g;
+  a.total_out = s->d_totals + g;
+  a.overflow_flag = s->d_ovf + g;
+  CUDA_TRY(s, cudaMemsetAsync(s->d_status, 0, a.n_tiles * 8, st));
+  CUDA_TRY(s, cudaMemsetAsync(s->d_counter + g, 0, 4, st));
+  CUDA_TRY(s, cudaMemsetAsync(s->d_ovf + g, 0, 4, st));
+  bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].first, st));
+  int ce = launch_expand(a, gp.words, st);
+  if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].second, st));
+  pd = Pending{g, k, n_parents, parents, (uint64_t*)csr, child, cap, which, off};
+  return ATF_OK;
+}
+
+// Generate groups' levels [k_from, L) starting from the given frontiers; syncs once per round.
+static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int> k_from,
+                             std::vector<const uint32_t*> frontier, std::vector<uint64_t> fsize) {
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  std::vector<int> k = k_from;
+  for (;;) {
+    std::vector<Pending> pend;
+    for (size_t i = 0; i < gs.size(); i++) {
+      int g = gs[i];
+      int L = (int)s->groups[g].levels.size();
+      if (k[i] >= L) continue;
+      if (fsize[i] == 0 || s->groups[g].levels[k[i]].r == 0) {
+        // empty frontier or empty range: every deeper level is empty
+        for (int kk = k[i]; kk < L; kk++) {
+          LevelData& d = s->data[g][kk];
+          d.rec = nullptr;
+          d.n = 0;
+          d.evals = (kk == k[i]) ? fsize[i] * (uint64_t)s->groups[g].levels[kk].r : 0;
+          if (kk > 0 && kk == k[i] && fsize[i] > 0) {
+            // parents get an all-zero CSR
+            char* csr = arena_alloc(s, g, (fsize[i] + 1) * 8);
+            if (!csr) {
+              atf_status e = arena_grow(s, g, (fsize[i] + 1) * 8);
+              if (e) return e;
+              csr = arena_alloc(s, g, (fsize[i] + 1) * 8);
+            }
+            CUDA_TRY(s, cudaMemsetAsync(csr, 0, (fsize[i] + 1) * 8, st));
+            s->data[g][kk - 1].csr = (uint64_t*)csr;
+          }
+        }
+        k[i] = L;
+        continue;
+      }
+      Pending pd;
+      atf_status e = queue_level(s, g, k[i], frontier[i], fsize[i], pd);
+      if (e) return e;
+      pend.push_back(pd);
+    }
+    if (pend.empty()) break;
+    for (auto& pd : pend) {
+      CUDA_TRY(s, cudaMemcpyAsync(s->h_totals + pd.g, s->d_totals + pd.g, 8, cudaMemcpyDeviceToHost, st));
+      CUDA_TRY(s, cudaMemcpyAsync(s->h_flags + pd.g, s->d_ovf + pd.g, 4, cudaMemcpyDeviceToHost, st));
+    }
+    CUDA_TRY(s, cudaStreamSynchronize(st));
+    for (auto& pd : pend) {
+      size_t i = std::find(gs.begin(), gs.end(), pd.g) - gs.begin();
+      uint64_t total = s->h_totals[pd.g];
+      GroupPlan& gp = s->groups[pd.g];
+      if (s->h_flags[pd.g] || total > pd.cap) {
+        // child region too small: grow the arena and redo this level next round
+        atf_status e = arena_grow(s, pd.g, total * gp.words * 4 + (pd.n_parents + 1) * 8);
+        if (e) return e;
+        continue;
+      }
+      Chunk& c = s->arena[pd.g][pd.chunk];
+      c.used = pd.child_off + ((total * gp.words * 4 + 255) & ~(uint64_t)255);
+      LevelData& d = s->data[pd.g][pd.k];
+      d.rec = pd.child;
+      d.n = total;
+      d.evals = pd.n_parents * (uint64_t)gp.levels[pd.k].r;
+      if (pd.k > 0) s->data[pd.g][pd.k - 1].csr = pd.csr;
+      if (s->opts.flags & ATF_FLAG_TIMING)
+        cudaEventElapsedTime(&d.ms, s->events[pd.g][pd.k].first, s->events[pd.g][pd.k].second);
+      frontier[i] = pd.child;
+      fsize[i] = total;
+      k[i]++;
+    }
+  }
+  return ATF_OK;
+}
+
+static atf_status generate_impl(atf_space* s) {
+  atf_status e = plan(s);
+  if (e) return e;
+  if ((e = ensure_device(s))) return e;
+  size_t G = s->groups.size();
+  s->data.assign(G, {});
+  for (size_t g = 0; g < G; g++) {
+    s->data[g].assign(s->groups[g].levels.size(), LevelData{});
+    for (auto& c : s->arena[g]) c.used = 0;
+  }
+  if (s->opts.flags & ATF_FLAG_TIMING) {
+    if (s->events.size() != G) {
+      s->events.assign(G, {});
+      for (size_t g = 0; g < G; g++) {
+        s->events[g].resize(s->groups[g].levels.size());
+        for (auto& ev : s->events[g]) {
+          CUDA_TRY(s, cudaEventCreate(&ev.first));
+          CUDA_TRY(s, cudaEventCreate(&ev.second));
+        }
+      }
+    }
+  }
+  std::vector<int> gs(G), kf(G, 0);
+  std::iota(gs.begin(), gs.end(), 0);
+  std::vector<const uint32_t*> fr(G, s->d_root);
+  std::vector<uint64_t> fz(G, 1);
+  if ((e = run_levels(s, gs, kf, fr, fz))) return e;
+  s->gsize.assign(G, 0);
+  for (size_t g = 0; g < G; g++) s->gsize[g] = s->groups[g].levels.empty() ? 0 : s->data[g].back().n;
+  s->state = GENERATED;
+  return ATF_OK;
+}
+
+// ---------------------------------------------------------------- decode args
+static atf_status make_decode_args(const atf_space* s, DecodeArgs& a) {
+  std::memset(&a, 0, sizeof a);
+  a.n_groups = (int)s->groups.size();
+  a.n_params = (int)s->params.size();
+  int l = 0;
+  for (int g = 0; g < a.n_groups; g++) {
+    const GroupPlan& gp = s->groups[g];
+    a.gsize[g] = s->gsize[g];
+    a.leaves[g] = s->data[g].back().rec;
+    a.words[g] = gp.words;
+    a.lvl_begin[g] = l;
+    for (auto& lp : gp.levels) {
+      a.lvl_param[l] = (int16_t)lp.param;
+      a.lvl_word[l] = (int16_t)lp.field_word;
+      a.lvl_shift[l] = (int16_t)lp.field_shift;
+      a.lvl_bits[l] = (int16_t)lp.field_bits;
+      a.lvl_range[l] = s->d_range[lp.param];
+      l++;
+    }
+  }
+  a.lvl_begin[a.n_groups] = l;
+  return ATF_OK;
+}
+
+// ================================================================= C ABI
+extern "C" {
+
+const char* atf_status_str(atf_status st) {
+  switch (st) {
+    case ATF_OK: return "ok";
+    case ATF_ERR_INVALID_ARG: return "invalid argument";
+    case ATF_ERR_OOM: return "out of memory";
+    case ATF_ERR_CUDA: return "CUDA error";
+    case ATF_ERR_STATE: return "invalid state";
+    case ATF_ERR_BYTECODE: return "bad bytecode";
+    case ATF_ERR_FORWARD_REF: return "forward reference";
+    case ATF_ERR_OVERFLOW: return "overflow";
+    case ATF_ERR_INDEX: return "index out of range";
+    case ATF_ERR_DUPLICATE: return "duplicate";
+    case ATF_ERR_LIMIT: return "limit exceeded";
+  }
+  return "unknown";
+}
+
+const char* atf_space_last_error(const atf_space* s) { return s ? s->err.c_str() : "null space"; }
+
+atf_status atf_space_create(const atf_space_opts* opts, atf_space** out) {
+  if (!out) return ATF_ERR_INVALID_ARG;
+  atf_space* s = new (std::nothrow) atf_space();
+  if (!s) return ATF_ERR_OOM;
+  if (opts) s->opts = *opts;
+  if (s->opts.alloc && !s->opts.free) {
+    delete s;
+    return ATF_ERR_INVALID_ARG;
+  }
+  *out = s;
+  return ATF_OK;
+}
+
+atf_status atf_space_add_param(atf_space* s, const char* name, const atf_range* range, int32_t* out_id) {
+  if (!s || !name || !range) return fail(s, ATF_ERR_INVALID_ARG, "null argument");
+  if (s->state != BUILDING) return fail(s, ATF_ERR_STATE, "add_param after plan/generate");
+  if (!*name) return fail(s, ATF_ERR_INVALID_ARG, "empty name");
+  if (s->params.size() >= ATF_MAX_PARAMS) return fail(s, ATF_ERR_LIMIT, "more than %d parameters", ATF_MAX_PARAMS);
+  for (auto& p : s->params)
+    if (p.name == name) return fail(s, ATF_ERR_DUPLICATE, "duplicate parameter name %s (P:53: unique)", name);
+  ParamDef pd;
+  pd.name = name;
+  // P:57 ranges; readings #1-#3, #5
+  if (range->kind == ATF_RANGE_INTERVAL || range->kind == ATF_RANGE_POW2) {
+    if (range->step <= 0) return fail(s, ATF_ERR_INVALID_ARG, "step must be positive");
+    if (range->end >= range->begin) {
+      i128 count = ((i128)range->end - range->begin) / range->step + 1;
+      if (count > ATF_MAX_RANGE) return fail(s, ATF_ERR_LIMIT, "range of %s has more than 2^24 values", name);
+    }
+    for (i128 i = range->begin; i <= range->end; i += range->step) {
+      if (range->kind == ATF_RANGE_INTERVAL) {
+        if (i < INT32_MIN || i > INT32_MAX) return fail(s, ATF_ERR_INVALID_ARG, "interval value outside int32");
+        pd.values.push_back((int32_t)i);
+      } else {
+        if (i < 0 || i > 30) return fail(s, ATF_ERR_INVALID_ARG, "pow2 exponent outside [0,30]");
+        pd.values.push_back((int32_t)(1u << (int)i));
+      }
+    }
+  } else if (range->kind == ATF_RANGE_SET) {
+    if (range->n_values < 0 || (range->n_values > 0 && !range->values))
+      return fail(s, ATF_ERR_INVALID_ARG, "bad set");
+    if (range->n_values > ATF_MAX_RANGE) return fail(s, ATF_ERR_LIMIT, "set larger than 2^24");
+    std::vector<int32_t> sorted(range->values, range->values + range->n_values);
+    std::sort(sorted.begin(), sorted.end());
+    if (std::adjacent_find(sorted.begin(), sorted.end()) != sorted.end())
+      return fail(s, ATF_ERR_DUPLICATE, "duplicate value in set of %s", name);
+    pd.values.assign(range->values, range->values + range->n_values);
+  } else {
+    return fail(s, ATF_ERR_INVALID_ARG, "unknown range kind %d", range->kind);
+  }
+  if (!pd.values.empty()) {
+    pd.vmin = *std::min_element(pd.values.begin(), pd.values.end());
+    pd.vmax = *std::max_element(pd.values.begin(), pd.values.end());
+  }
+  s->params.push_back(std::move(pd));
+  if (out_id) *out_id = (int32_t)s->params.size() - 1;
+  return ATF_OK;
+}
+
+atf_status atf_space_add_constraint(atf_space* s, int32_t pid, const int32_t* code, int32_t n) {
+  if (!s || !code) return fail(s, ATF_ERR_INVALID_ARG, "null argument");
+  if (s->state != BUILDING) return fail(s, ATF_ERR_STATE, "add_constraint after plan/generate");
+  if (pid < 0 || pid >= (int)s->params.size()) return fail(s, ATF_ERR_INVALID_ARG, "no parameter %d", pid);
+  atf_status st = validate_program(s, pid, code, n);
+  if (st) return st;
+  s->params[pid].programs.emplace_back(code, code + n);
+  return ATF_OK;
+}
+
+atf_status atf_space_plan(atf_space* s) {
+  if (!s) return ATF_ERR_INVALID_ARG;
+  if (s->state == BUILDING) {
+    // static int64 interval analysis of every program (reading #9)
+    for (size_t p = 0; p < s->params.size(); p++)
+      for (auto& code : s->params[p].programs) {
+        Tree t;
+        std::string why;
+        Iv xiv{s->params[p].vmin, s->params[p].vmax};
+        if (parse_program(code, s->params, xiv, t, &why) < 0)
+          return fail(s, ATF_ERR_OVERFLOW, "parameter %s: %s", s->params[p].name.c_str(), why.c_str());
+      }
+  }
+  return plan(s);
+}
+
+atf_status atf_space_num_params(const atf_space* s, int32_t* out) {
+  if (!s || !out) return ATF_ERR_INVALID_ARG;
+  *out = (int32_t)s->params.size();
+  return ATF_OK;
+}
+
+atf_status atf_space_num_groups(const atf_space* s, int32_t* out) {
+  if (!s || !out) return ATF_ERR_INVALID_ARG;
+  if (s->state == BUILDING) return ATF_ERR_STATE;
+  *out = (int32_t)s->groups.size();
+  return ATF_OK;
+}
+
+atf_status atf_space_group_members(const atf_space* s, int32_t g, int32_t* out, int32_t cap, int32_t* n_out) {
+  if (!s || !n_out) return ATF_ERR_INVALID_ARG;
+  if (s->state == BUILDING) return ATF_ERR_STATE;
+  if (g < 0 || g >= (int)s->groups.size()) return ATF_ERR_INVALID_ARG;
+  auto& m = s->groups[g].members;
+  *n_out = (int32_t)m.size();
+  for (int i = 0; i < (int)m.size() && i < cap && out; i++) out[i] = m[i];
+  return ATF_OK;
+}
+
+atf_status atf_space_plan_json(const atf_space* s, char* buf, size_t cap, size_t* len_out) {
+  if (!s) return ATF_ERR_INVALID_ARG;
+  if (s->state == BUILDING) return ATF_ERR_STATE;
+  std::string j = "{\"groups\":[";
+  for (size_t g = 0; g < s->groups.size(); g++) {
+    auto& gp = s->groups[g];
+    j += (g ? "," : "") + std::string("{\"members\":[");
+    for (size_t i = 0; i < gp.members.size(); i++) j += (i ? "," : "") + std::to_string(gp.members[i]);
+    j += "],\"words\":" + std::to_string(gp.words) + ",\"levels\":[";
+    for (size_t l = 0; l < gp.levels.size(); l++) {
+      auto& lp = gp.levels[l];
+      std::string d;
+      for (char c : lp.desc) {
+        if (c == '"' || c == '\\') d += '\\';
+        d += c;
+      }
+      char tmp[256];
+      snprintf(tmp, sizeof tmp,
+               "{\"param\":%d,\"r\":%d,\"word\":%d,\"shift\":%d,\"bits\":%d,\"cost\":%.1f,\"generic\":%s,"
+               "\"n_terms\":%d,\"n_gates\":%d,\"n_slots\":%d,\"qmax\":%u,\"desc\":\"",
+               lp.param, lp.r, lp.field_word, lp.field_shift, lp.field_bits, lp.cost, lp.generic ? "true" : "false",
+               lp.proto.n_terms, lp.proto.n_gates, lp.proto.n_slots, lp.proto.qmax);
+      j += (l ? "," : "") + std::string(tmp) + d + "\"";
+      j += ",\"terms\":[";
+      for (int t = 0; t < lp.proto.n_terms; t++) {
+        const Term& T = lp.proto.terms[t];
+        snprintf(tmp, sizeof tmp, "%s{\"kind\":%d,\"variant\":%d,\"rel\":%d,\"qtable\":%d}", t ? "," : "", T.kind,
+                 T.variant, T.rel, T.use_qtable);
+        j += tmp;
+      }
+      j += "]}";
+    }
+    j += "]}";
+  }
+  j += "]}";
+  if (len_out) *len_out = j.size();
+  if (buf && cap > 0) {
+    size_t n = std::min(cap - 1, j.size());
+    memcpy(buf, j.data(), n);
+    buf[n] = 0;
+  }
+  return ATF_OK;
+}
+
+atf_status atf_space_generate(atf_space* s) {
+  if (!s) return ATF_ERR_INVALID_ARG;
+  if (s->state == SHARDED) return fail(s, ATF_ERR_STATE, "space holds an unfinalized shard");
+  if (s->state == BUILDING) {
+    atf_status e = atf_space_plan(s);
+    if (e) return e;
+  }
+  return generate_impl(s);
+}
+
+atf_status atf_space_size(const atf_space* s, uint64_t* lo, uint64_t* hi) {
+  if (!s || !lo || !hi) return ATF_ERR_INVALID_ARG;
+  if (s->state != GENERATED && s->state != FINAL_SHARD) return ATF_ERR_STATE;
+  u128 S = 1;
+  for (uint64_t z : s->gsize) {
+    if (z && S > (~(u128)0) / z) return fail((atf_space*)s, ATF_ERR_OVERFLOW, "S >= 2^128");
+    S *= z;
+  }
+  *lo = (uint64_t)S;
+  *hi = (uint64_t)(S >> 64);
+  return ATF_OK;
+}
+
+atf_status atf_space_group_size(const atf_space* s, int32_t g, uint64_t* out) {
+  if (!s || !out) return ATF_ERR_INVALID_ARG;
+  if (s->state != GENERATED && s->state != FINAL_SHARD) return ATF_ERR_STATE;
+  if (g < 0 || g >= (int)s->groups.size()) return ATF_ERR_INVALID_ARG;
+  *out = s->gsize[g];
+  return ATF_OK;
+}
+
+atf_status atf_space_num_levels(const atf_space* s, int32_t g, int32_t* out) {
+  if (!s || !out) return ATF_ERR_INVALID_ARG;
+  if (s->state == BUILDING) return ATF_ERR_STATE;
+  if (g < 0 || g >= (int)s->groups.size()) return ATF_ERR_INVALID_ARG;
+  *out = (int32_t)s->groups[g].levels.size();
+  return ATF_OK;
+}
+
+atf_status atf_space_level_size(const atf_space* s, int32_t g, int32_t k, uint64_t* out) {
+  if (!s || !out) return ATF_ERR_INVALID_ARG;
+  if (s->state < GENERATED) return ATF_ERR_STATE;
+  if (g < 0 || g >= (int)s->groups.size() || k < 0 || k >= (int)s->groups[g].levels.size())
+    return ATF_ERR_INVALID_ARG;
+  *out = s->data[g][k].n;
+  return ATF_OK;
+}
+
+atf_status atf_space_level_view(const atf_space* s, int32_t g, int32_t k, atf_level_view* out) {
+  if (!s || !out) return ATF_ERR_INVALID_ARG;
+  if (s->state < GENERATED) return ATF_ERR_STATE;
+  if (g < 0 || g >= (int)s->groups.size() || k < 0 || k >= (int)s->groups[g].levels.size())
+    return ATF_ERR_INVALID_ARG;
+  const LevelData& d = s->data[g][k];
+  const LevelPlan& lp = s->groups[g].levels[k];
+  out->records = d.rec;
+  out->csr = (k + 1 < (int)s->groups[g].levels.size()) ? d.csr : nullptr;
+  out->n_nodes = d.n;
+  out->offset = d.offset;
+  out->words = s->groups[g].words;
+  out->param = lp.param;
+  out->field_word = lp.field_word;
+  out->field_shift = lp.field_shift;
+  out->field_bits = lp.field_bits;
+  return ATF_OK;
+}
+
+static atf_status decode_common(const atf_space* cs, const uint64_t* idx, const uint64_t* digits, int64_t n,
+                                int32_t* out, int64_t ld, void* stream) {
+  atf_space* s = (atf_space*)cs;
+  if (!s || (!idx && !digits) || !out || n < 0 || ld < n) return fail(s, ATF_ERR_INVALID_ARG, "bad decode arguments");
+  if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "decode needs a generated (non-shard) space");
+  if (idx) {
+    u128 S = 1;
+    for (uint64_t z : s->gsize) S *= z;
+    if (S >> 64) return fail(s, ATF_ERR_OVERFLOW, "S >= 2^64: use atf_space_decode_digits");
+  }
+  if (n == 0) return ATF_OK;
+  CUDA_TRY(s, cudaSetDevice(s->opts.device));
+  cudaStream_t st = (cudaStream_t)(stream ? stream : s->opts.stream);
+  DecodeArgs a;
+  make_decode_args(s, a);
+  CUDA_TRY(s, cudaMemsetAsync(s->d_bad, 0, 4, st));
+  int ce = idx ? launch_decode_indices(a, idx, n, out, ld, s->d_bad, st)
+               : launch_decode_digits(a, digits, n, out, ld, s->d_bad, st);
+  if (ce) return fail(s, ATF_ERR_CUDA, "decode launch: %s", cudaGetErrorString((cudaError_t)ce));
+  // the bad-index flag is read back only when someone could be out of range: always
+  // check (one 4-byte copy) — it costs a sync, so the flag copy is async and we
+  // synchronise the stream here to report ATF_ERR_INDEX deterministically.
+  CUDA_TRY(s, cudaMemcpyAsync(s->h_flags, s->d_bad, 4, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(s, cudaStreamSynchronize(st));
+  if (s->h_flags[0]) return fail(s, ATF_ERR_INDEX, "index/digit out of range (rows set to INT32_MIN)");
+  return ATF_OK;
+}
+
+atf_status atf_space_decode_indices(const atf_space* s, const uint64_t* d_idx, int64_t n, int32_t* d_out, int64_t ld,
+                                    void* stream) {
+  if (!d_idx) return fail((atf_space*)s, ATF_ERR_INVALID_ARG, "null indices");
+  return decode_common(s, d_idx, nullptr, n, d_out, ld, stream);
+}
+
+atf_status atf_space_decode_digits(const atf_space* s, const uint64_t* d_digits, int64_t n, int32_t* d_out,
+                                   int64_t ld, void* stream) {
+  if (!d_digits) return fail((atf_space*)s, ATF_ERR_INVALID_ARG, "null digits");
+  return decode_common(s, nullptr, d_digits, n, d_out, ld, stream);
+}
+
+atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap, int32_t* n_out) {
+  if (!s || !n_out) return ATF_ERR_INVALID_ARG;
+  if (s->state < GENERATED) return ATF_ERR_STATE;
+  int n = 0;
+  for (size_t g = 0; g < s->groups.size(); g++)
+    for (size_t k = 0; k < s->groups[g].levels.size(); k++) {
+      if (out && n < cap) {
+        const LevelPlan& lp = s->groups[g].levels[k];
+        const LevelData& d = s->data[g][k];
+        atf_level_stats& o = out[n];
+        o.group = (int32_t)g;
+        o.level = (int32_t)k;
+        o.param = lp.param;
+        o.r = lp.r;
+        o.evals = d.evals;
+        o.f = d.n;
+        o.ms = d.ms;
+        o.path = lp.generic ? 1 : 0;
+      }
+      n++;
+    }
+  *n_out = n;
+  return ATF_OK;
+}
+
+// ---------------------------------------------------------------- multi-GPU shards
+// every rank computes the prefix levels up to the cut k* (first level
+// with f >= 1024 * world) and the level k*+1 of the whole cut frontier; rank r then
+// keeps the contiguous slice of level-k* nodes whose level-(k*+1) child prefix lies in
+// [r T / world, (r+1) T / world) and expands its children locally.  Concatenating the
+// ranks' slices in rank order gives the single-GPU arrays.
+atf_status atf_space_generate_shard(atf_space* s, int32_t rank, int32_t world, int64_t* h_counts, int32_t cap,
+                                    int32_t* n_out) {
+  if (!s || !n_out || world < 1 || rank < 0 || rank >= world) return fail(s, ATF_ERR_INVALID_ARG, "bad rank/world");
+  if (s->state == BUILDING) {
+    atf_status e = atf_space_plan(s);
+    if (e) return e;
+  }
+  atf_status e = ensure_device(s);
+  if (e) return e;
+  size_t G = s->groups.size();
+  s->data.assign(G, {});
+  for (size_t g = 0; g < G; g++) {
+    s->data[g].assign(s->groups[g].levels.size(), LevelData{});
+    for (auto& c : s->arena[g]) c.used = 0;
+  }
+  s->shard_rank = rank;
+  s->shard_world = world;
+  s->shard_cut.assign(G, 0);
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  const uint64_t thresh = 1024ull * (uint64_t)world;
+  // phase 1: replicated prefix, level by level, until the cut
+  std::vector<const uint32_t*> fr(G, s->d_root);
+  std::vector<uint64_t> fz(G, 1);
+  std::vector<int> kk(G, 0);
+  std::vector<char> cut_done(G, 0);
+  for (;;) {
+    std::vector<int> gs;
+    for (size_t g = 0; g < G; g++) {
+      int L = (int)s->groups[g].levels.size();
+      // expand while the frontier is small, and always the level just after the cut
+      if (cut_done[g] || kk[g] >= L) continue;
+      gs.push_back((int)g);
+    }
+    if (gs.empty()) break;
+    for (int g : gs) {
+      std::vector<int> one{g}, k1{kk[g]};
+      std::vector<const uint32_t*> f1{fr[g]};
+      std::vector<uint64_t> z1{fz[g]};
+      // run exactly one level: temporarily cap the group's level count
+      GroupPlan& gp = s->groups[g];
+      std::vector<LevelPlan> saved(gp.levels.begin() + kk[g] + 1, gp.levels.end());
+      gp.levels.resize(kk[g] + 1);
+      e = run_levels(s, one, k1, f1, z1);
+      gp.levels.insert(gp.levels.end(), saved.begin(), saved.end());
+      if (e) return e;
+      LevelData& d = s->data[g][kk[g]];
+      fr[g] = d.rec;
+      fz[g] = d.n;
+      kk[g]++;
+      // cut after the level following the first level with >= thresh nodes
+      if (kk[g] >= 2 && s->data[g][kk[g] - 2].n >= thresh) cut_done[g] = 2;  // sharded
+      else if (d.n == 0) cut_done[g] = 1;                                      // empty: replicated
+    }
+  }
+  // phase 2: slice the cut level (k* = kk-2) by the child counts of level k*+1
+  std::vector<int> gs, kf;
+  std::vector<const uint32_t*> f2;
+  std::vector<uint64_t> z2;
+  for (size_t g = 0; g < G; g++) {
+    int L = (int)s->groups[g].levels.size();
+    if (cut_done[g] != 2) {
+      // group too small to shard: fully replicated, owned by rank 0
+      s->shard_cut[g] = L;
+      continue;
+    }
+    int kc = kk[g] - 2;  // cut level
+    s->shard_cut[g] = kc + 1;
+    LevelData& cutd = s->data[g][kc];
+    uint64_t ncut = cutd.n;
+    std::vector<uint64_t> csr(ncut + 1);
+    CUDA_TRY(s, cudaMemcpyAsync(csr.data(), cutd.csr, (ncut + 1) * 8, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(s, cudaStreamSynchronize(st));
+    const uint64_t T = csr[ncut];
+    auto bound = [&](int r_) -> uint64_t {  // first cut node whose child prefix >= r T / world
+      u128 target = (u128)T * (u128)r_ / (u128)world;
+      return (uint64_t)(std::lower_bound(csr.begin(), csr.end(), (uint64_t)target) - csr.begin());
+    };
+    uint64_t lo = rank == 0 ? 0 : std::min<uint64_t>(bound(rank), ncut);
+    uint64_t hi = rank == world - 1 ? ncut : std::min<uint64_t>(bound(rank + 1), ncut);
+    if (hi < lo) hi = lo;
+    // slice of level k*+1 = children of cut nodes [lo, hi)
+    LevelData& nd = s->data[g][kc + 1];
+    uint64_t c0 = csr[lo], c1 = csr[hi];
+    GroupPlan& gp = s->groups[g];
+    nd.offset = c0;
+    nd.rec = nd.rec + c0 * gp.words;
+    nd.n = c1 - c0;
+    if (kc + 2 < L) {
+      gs.push_back((int)g);
+      kf.push_back(kc + 2);
+      f2.push_back(nd.rec);
+      z2.push_back(nd.n);
+    }
+  }
+  if (!gs.empty()) {
+    if ((e = run_levels(s, gs, kf, f2, z2))) return e;
+  }
+  // counts: per (group, level): this rank's nodes of the sharded levels; replicated levels
+  // count on rank 0 only, so that the sum over ranks is the global level size.
+  int n = 0;
+  for (size_t g = 0; g < G; g++)
+    for (size_t k = 0; k < s->groups[g].levels.size(); k++) {
+      int64_t c = (int)k >= s->shard_cut[g] ? (int64_t)s->data[g][k].n : (rank == 0 ? (int64_t)s->data[g][k].n : 0);
+      if (h_counts && n < cap) h_counts[n] = c;
+      n++;
+    }
+  *n_out = n;
+  s->state = SHARDED;
+  return ATF_OK;
+}
+
+atf_status atf_space_finalize_shard(atf_space* s, const int64_t* all, int32_t world, int32_t n) {
+  if (!s || !all) return ATF_ERR_INVALID_ARG;
+  if (s->state != SHARDED) return fail(s, ATF_ERR_STATE, "finalize_shard needs generate_shard");
+  if (world != s->shard_world) return fail(s, ATF_ERR_INVALID_ARG, "world mismatch");
+  int idx = 0;
+  size_t G = s->groups.size();
+  s->gsize.assign(G, 0);
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  for (size_t g = 0; g < G; g++)
+    for (size_t k = 0; k < s->groups[g].levels.size(); k++, idx++) {
+      if (idx >= n) return fail(s, ATF_ERR_INVALID_ARG, "counts too short");
+      uint64_t before = 0, tot = 0;
+      for (int r = 0; r < world; r++) {
+        uint64_t c = (uint64_t)all[(size_t)r * n + idx];
+        if (r < s->shard_rank) before += c;
+        tot += c;
+      }
+      LevelData& d = s->data[g][k];
+      if ((int)k >= s->shard_cut[g]) {
+        uint64_t old = d.offset;
+        d.offset = before;
+        // CSR entries of this rank's sharded parents point into its local child array;
+        // shift them to global child indices
+        if ((int)k > s->shard_cut[g] && k >= 1) {
+          LevelData& pdl = s->data[g][k - 1];
+          if (pdl.csr && pdl.n) {
+            int ce = launch_add_offset(pdl.csr, pdl.n + 1, before, st);
+            if (ce) return fail(s, ATF_ERR_CUDA, "csr fix-up");
+          }
+        }
+        (void)old;
+      }
+      if (k + 1 == s->groups[g].levels.size()) s->gsize[g] = tot;
+    }
+  s->state = FINAL_SHARD;  // sizes global; decode needs the whole tree (not available)
+  return ATF_OK;
+}
+
+atf_status atf_test_exclusive_scan_u32(const uint32_t* d_in, uint64_t* d_out, int64_t n, void* stream) {
+  if ((!d_in && n > 0) || !d_out || n < 0) return ATF_ERR_INVALID_ARG;
+  cudaStream_t st = (cudaStream_t)stream;
+  const int64_t tiles = n > 0 ? (n + 1023) / 1024 : 1;
+  unsigned long long* status = nullptr;
+  unsigned int* counter = nullptr;
+  if (cudaMallocAsync((void**)&status, tiles * 8, st) != cudaSuccess) return ATF_ERR_OOM;
+  if (cudaMallocAsync((void**)&counter, 4, st) != cudaSuccess) return ATF_ERR_OOM;
+  cudaMemsetAsync(status, 0, tiles * 8, st);
+  cudaMemsetAsync(counter, 0, 4, st);
+  if (n == 0) cudaMemsetAsync(d_out, 0, 8, st);
+  else if (launch_scan_u32(d_in, d_out, n, status, counter, st)) return ATF_ERR_CUDA;
+  cudaFreeAsync(status, st);
+  cudaFreeAsync(counter, st);
+  return cudaStreamSynchronize(st) == cudaSuccess ? ATF_OK : ATF_ERR_CUDA;
+}
+
+void atf_space_destroy(atf_space* s) {
+  if (!s) return;
+  if (s->dev_ready) {
+    cudaSetDevice(s->opts.device);
+    release_device(s);
+    cudaStreamSynchronize((cudaStream_t)s->opts.stream);
+  }
+  delete s;
+}
+
+}  // extern "C"

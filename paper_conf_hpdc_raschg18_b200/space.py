@@ -1,0 +1,212 @@
+"""Thin Python front end over the C ABI (argument marshalling only).
+
+``Space`` builds an ``atf_space`` from an :class:`atfspec.Spec` (names, ranges,
+constraint bytecode — PAPER.md P:49-59), lets PyTorch provide device memory
+(caching allocator) and the CUDA stream, and exposes generate / size / decode.
+"""
+from __future__ import annotations
+
+import ctypes as C
+import json
+from typing import Dict, List, Optional
+
+from . import _lib as L
+
+
+def _range_struct(rng: dict):
+    kind = rng["kind"]
+    if kind == "interval":
+        return L.atf_range(L.ATF_RANGE_INTERVAL, rng["begin"], rng["end"], rng.get("step", 1), None, 0), None
+    if kind == "pow2":
+        return L.atf_range(L.ATF_RANGE_POW2, rng["begin"], rng["end"], rng.get("step", 1), None, 0), None
+    if kind == "set":
+        vals = (C.c_int32 * max(1, len(rng["values"])))(*rng["values"])
+        return L.atf_range(L.ATF_RANGE_SET, 0, 0, 0, C.cast(vals, C.POINTER(C.c_int32)), len(rng["values"])), vals
+    raise ValueError(f"unknown range kind {kind}")
+
+
+class Space:
+    """One search space on one device.
+
+    flags: L.ATF_FLAG_TIMING (per-level device times) | L.ATF_FLAG_GENERIC_ONLY
+    (interpret every candidate with the generic bytecode interpreter).
+    """
+
+    def __init__(self, spec=None, device: int = 0, stream=None, flags: int = 0, torch_alloc: bool = True):
+        self._h = C.c_void_p()
+        self._bufs: Dict[int, object] = {}
+        self._device = device
+        self._stream_obj = stream
+        stream_ptr = None
+        self._alloc_cb = L.ALLOC_FN()
+        self._free_cb = L.FREE_FN()
+        if torch_alloc or stream is not None:
+            import torch
+            if torch.cuda.is_available():
+                if stream is None:
+                    stream = torch.cuda.current_stream(device)
+                self._stream_obj = stream
+                stream_ptr = stream.cuda_stream
+                if torch_alloc:
+                    dev = torch.device("cuda", device)
+
+                    def _alloc(nbytes, _stream, _ctx):
+                        try:
+                            with torch.cuda.stream(self._stream_obj):
+                                t = torch.empty(int(nbytes), dtype=torch.uint8, device=dev)
+                        except RuntimeError:
+                            return None
+                        p = t.data_ptr()
+                        self._bufs[p] = t
+                        return p
+
+                    def _free(ptr, _nbytes, _stream, _ctx):
+                        self._bufs.pop(ptr, None)
+
+                    self._alloc_cb = L.ALLOC_FN(_alloc)
+                    self._free_cb = L.FREE_FN(_free)
+        opts = L.atf_space_opts(device, stream_ptr, self._alloc_cb, self._free_cb, None, flags)
+        L.check(L.atf_space_create(C.byref(opts), C.byref(self._h)))
+        self.names: List[str] = []
+        if spec is not None:
+            self.add_spec(spec)
+
+    # ---- building
+    def add_spec(self, spec) -> None:
+        for p in spec.params:
+            pid = self.add_param(p.name, p.range)
+            for code in p.constraints:
+                self.add_constraint(pid, code)
+
+    def add_param(self, name: str, rng: dict) -> int:
+        st, keep = _range_struct(rng)
+        out = C.c_int32()
+        L.check(L.atf_space_add_param(self._h, name.encode(), C.byref(st), C.byref(out)), self._h)
+        self.names.append(name)
+        return out.value
+
+    def add_constraint(self, pid: int, code) -> None:
+        arr = (C.c_int32 * len(code))(*[int(w) for w in code])
+        L.check(L.atf_space_add_constraint(self._h, pid, arr, len(code)), self._h)
+
+    # ---- planning
+    def plan(self) -> None:
+        L.check(L.atf_space_plan(self._h), self._h)
+
+    def num_groups(self) -> int:
+        out = C.c_int32()
+        L.check(L.atf_space_num_groups(self._h, C.byref(out)), self._h)
+        return out.value
+
+    def groups(self) -> List[List[int]]:
+        res = []
+        for g in range(self.num_groups()):
+            buf = (C.c_int32 * 64)()
+            n = C.c_int32()
+            L.check(L.atf_space_group_members(self._h, g, buf, 64, C.byref(n)), self._h)
+            res.append(list(buf[: n.value]))
+        return res
+
+    def plan_json(self) -> dict:
+        n = C.c_size_t()
+        L.check(L.atf_space_plan_json(self._h, None, 0, C.byref(n)), self._h)
+        buf = C.create_string_buffer(n.value + 1)
+        L.check(L.atf_space_plan_json(self._h, buf, n.value + 1, None), self._h)
+        return json.loads(buf.value.decode())
+
+    # ---- generation
+    def generate(self) -> None:
+        L.check(L.atf_space_generate(self._h), self._h)
+
+    def generate_shard(self, rank: int, world: int) -> List[int]:
+        cap = 64 * 64
+        buf = (C.c_int64 * cap)()
+        n = C.c_int32()
+        L.check(L.atf_space_generate_shard(self._h, rank, world, buf, cap, C.byref(n)), self._h)
+        return list(buf[: n.value])
+
+    def finalize_shard(self, all_counts: List[List[int]]) -> None:
+        world = len(all_counts)
+        n = len(all_counts[0])
+        flat = (C.c_int64 * (world * n))(*[int(c) for row in all_counts for c in row])
+        L.check(L.atf_space_finalize_shard(self._h, flat, world, n), self._h)
+
+    def size(self) -> int:
+        lo, hi = C.c_uint64(), C.c_uint64()
+        L.check(L.atf_space_size(self._h, C.byref(lo), C.byref(hi)), self._h)
+        return (hi.value << 64) | lo.value
+
+    def group_sizes(self) -> List[int]:
+        out = []
+        for g in range(self.num_groups()):
+            v = C.c_uint64()
+            L.check(L.atf_space_group_size(self._h, g, C.byref(v)), self._h)
+            out.append(v.value)
+        return out
+
+    def num_levels(self, g: int) -> int:
+        v = C.c_int32()
+        L.check(L.atf_space_num_levels(self._h, g, C.byref(v)), self._h)
+        return v.value
+
+    def level_sizes(self, g: int) -> List[int]:
+        out = []
+        for k in range(self.num_levels(g)):
+            v = C.c_uint64()
+            L.check(L.atf_space_level_size(self._h, g, k, C.byref(v)), self._h)
+            out.append(v.value)
+        return out
+
+    def level_view(self, g: int, k: int) -> dict:
+        v = L.atf_level_view()
+        L.check(L.atf_space_level_view(self._h, g, k, C.byref(v)), self._h)
+        return {f: getattr(v, f) for f, _ in L.atf_level_view._fields_}
+
+    def stats(self) -> List[dict]:
+        n = C.c_int32()
+        L.check(L.atf_space_stats(self._h, None, 0, C.byref(n)), self._h)
+        arr = (L.atf_level_stats * max(1, n.value))()
+        L.check(L.atf_space_stats(self._h, arr, n.value, C.byref(n)), self._h)
+        return [{f: getattr(arr[i], f) for f, _ in L.atf_level_stats._fields_} for i in range(n.value)]
+
+    # ---- decode (device tensors in, device tensor out)
+    def decode(self, idx, out=None, stream=None):
+        """idx: CUDA tensor of uint64/int64 indices [n] -> int32 tensor [P, n] (SoA)."""
+        import torch
+        n = idx.numel()
+        P = len(self.names)
+        if out is None:
+            out = torch.empty((P, n), dtype=torch.int32, device=idx.device)
+        sp = stream.cuda_stream if stream is not None else None
+        L.check(L.atf_space_decode_indices(self._h, idx.data_ptr(), n, out.data_ptr(), out.stride(0), sp), self._h)
+        return out
+
+    def decode_digits(self, digits, out=None, stream=None):
+        """digits: CUDA tensor [G, n] of per-group indices -> int32 tensor [P, n]."""
+        import torch
+        n = digits.shape[1]
+        P = len(self.names)
+        if out is None:
+            out = torch.empty((P, n), dtype=torch.int32, device=digits.device)
+        digits = digits.contiguous()
+        sp = stream.cuda_stream if stream is not None else None
+        L.check(L.atf_space_decode_digits(self._h, digits.data_ptr(), n, out.data_ptr(), out.stride(0), sp), self._h)
+        return out
+
+    def close(self) -> None:
+        if self._h:
+            L.atf_space_destroy(self._h)
+            self._h = C.c_void_p()
+            self._bufs.clear()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()

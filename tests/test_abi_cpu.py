@@ -1,0 +1,185 @@
+"""CPU-side tests of the C ABI: the library loads and exports every symbol the headers
+declare; the host planner (validation, static analysis, group partition, atom
+compilation) behaves as documented.  No CUDA device is needed (no compute calls)."""
+import os
+import re
+import subprocess
+
+import pytest
+
+import atfspec as A
+from atfspec import Spec, X, C, P, interval, set_, divides
+from oracle import run as orc
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def L():
+    from paper_conf_hpdc_raschg18_b200 import _lib
+    return _lib
+
+
+def _declared(header):
+    txt = open(os.path.join(ROOT, "include", header)).read()
+    txt = re.sub(r"/\*.*?\*/", "", txt, flags=re.S)
+    return set(re.findall(r"\b(atf_\w+)\s*\(", txt)) - {"atf_alloc_fn", "atf_free_fn"}
+
+
+def test_library_exports_every_declared_symbol(L):
+    declared = _declared("atfgen.h") | _declared("atfgen_test.h")
+    assert declared, "no declarations parsed"
+    out = subprocess.run(["nm", "-D", "--defined-only", L.LIB_PATH], capture_output=True, text=True).stdout
+    exported = set(re.findall(r" T (atf_\w+)", out))
+    assert declared <= exported, declared - exported
+    assert declared <= set(L.EXPORTED) | {"atf_test_exclusive_scan_u32"}
+    for name in declared:
+        assert hasattr(L, name)
+
+
+def test_library_is_sm100a(L):
+    out = subprocess.run(["cuobjdump", "--list-elf", L.LIB_PATH], capture_output=True, text=True).stdout
+    assert "sm_100a" in out
+
+
+def _space(spec, **kw):
+    from paper_conf_hpdc_raschg18_b200 import Space
+    return Space(spec, torch_alloc=False, **kw)
+
+
+@pytest.mark.parametrize("mk", [A.fig1, A.c1_toy, lambda: A.c2_xgemm_direct(64), lambda: A.c3_xgemm("IS3"),
+                                lambda: A.c5_chains(32, 4)] + [lambda s=s: A.random_spec(s) for s in range(25)])
+def test_group_partition_matches_oracle(oracle_bin, mk):
+    spec = mk()
+    sp = _space(spec)
+    sp.plan()
+    try:
+        ref = orc.info(spec)
+    except ValueError:
+        return
+    assert sp.groups() == [g["members"] for g in ref["groups"]]
+
+
+def test_named_partitions():
+    # SURVEY.md §8(a) A2
+    for spec, want in [(A.fig1(), [[0, 1], [2, 3]]), (A.c2_xgemm_direct(256), [list(range(8)), [8], [9]]),
+                       (A.c3_xgemm("IS2"), [list(range(10)), [10], [11], [12], [13]]),
+                       (A.c5_chains(), [list(range(8)), list(range(8, 16)), list(range(16, 24))])]:
+        sp = _space(spec)
+        sp.plan()
+        assert sp.groups() == want
+
+
+def test_atoms_for_the_hot_levels():
+    """The C3 NDIMB level (the dominant one) compiles to the divisibility
+    atom x|NWG and the computed-divisor atom KWG mod (MDIMC*NDIMC/x) == 0, both 16-bit."""
+    sp = _space(A.c3_xgemm("IS2"))
+    sp.plan()
+    lv = sp.plan_json()["groups"][0]["levels"]
+    kinds = [[t["kind"] for t in l["terms"]] for l in lv]
+    assert kinds[6] == [2, 5] and all(t["variant"] == 0 for t in lv[6]["terms"])
+    assert lv[6]["terms"][1]["qtable"] == 1
+    assert kinds[8] == [4, 4] and kinds[9] == [4, 4]
+    assert lv[6]["cost"] == 9.0 and lv[9]["cost"] == 5.0
+    sp = _space(A.c5_chains())
+    sp.plan()
+    pj = sp.plan_json()
+    assert all(l["terms"][0]["kind"] == (2 if g != 1 else 3) for g in range(3)
+               for l in pj["groups"][g]["levels"][1:])
+    assert [g["words"] for g in pj["groups"]] == [4, 4, 4]
+
+
+def test_generic_only_flag_compiles_generic_terms(L):
+    sp = _space(A.c3_xgemm("IS2"), flags=L.ATF_FLAG_GENERIC_ONLY)
+    sp.plan()
+    lv = sp.plan_json()["groups"][0]["levels"]
+    assert all(t["kind"] == 6 for l in lv for t in l["terms"])
+
+
+def test_record_packing_two_words():
+    sp = _space(A.c3_xgemm("IS2"))
+    sp.plan()
+    g0 = sp.plan_json()["groups"][0]
+    assert g0["words"] == 2        # 59 bits packed first-fit-decreasing into two words
+    used = {}
+    for l in g0["levels"]:
+        used.setdefault(l["word"], []).append((l["shift"], l["bits"]))
+    for w, fields in used.items():
+        fields.sort()
+        for (s0, b0), (s1, _) in zip(fields, fields[1:]):
+            assert s0 + b0 <= s1
+        assert fields[-1][0] + fields[-1][1] <= 32
+
+
+def _err(fn):
+    from paper_conf_hpdc_raschg18_b200 import AtfError
+    with pytest.raises(AtfError) as e:
+        fn()
+    return e.value.status
+
+
+def test_validation_errors():
+    from paper_conf_hpdc_raschg18_b200 import Space
+    sp = Space(None, torch_alloc=False)
+    a = sp.add_param("a", interval(1, 8))
+    b = sp.add_param("b", interval(1, 8))
+    assert _err(lambda: sp.add_param("a", interval(1, 2))) == -9                    # duplicate name
+    assert _err(lambda: sp.add_param("s", set_(1, 2, 2))) == -9                      # duplicate set value
+    assert _err(lambda: sp.add_param("t", {"kind": "interval", "begin": 1, "end": 4, "step": 0})) == -1
+    assert _err(lambda: sp.add_param("u", {"kind": "pow2", "begin": 0, "end": 31, "step": 1})) == -1
+    assert _err(lambda: sp.add_constraint(a, P(1).code + [1, 17])) == -6           # forward reference
+    assert _err(lambda: sp.add_constraint(b, [1, 17])) == -5                         # stack underflow
+    assert _err(lambda: sp.add_constraint(b, [1, 1])) == -5                          # two results
+    assert _err(lambda: sp.add_constraint(b, [99])) == -5                            # bad opcode
+    assert _err(lambda: sp.add_constraint(b, [1] * 17 + [4] * 16)) == -5           # depth > 16
+    sp.add_constraint(b, divides(P(a)).code)
+    assert _err(lambda: sp.size()) == -4                                             # state
+    sp.plan()
+    assert _err(lambda: sp.add_param("c", interval(1, 2))) == -4
+    assert sp.groups() == [[0, 1]]
+
+
+def test_static_overflow_rejected():
+    s = Spec("ovf")
+    s.add("x", interval(1, 4), (C(2 ** 62) * X) > 0)
+    sp = _space(s)
+    assert _err(sp.plan) == -7
+    s = Spec("ok")
+    s.add("x", interval(1, 4), (C(2 ** 60) * X) > 0)
+    _space(s).plan()
+
+
+def test_magic_formulas_exhaustive(tmp_path):
+    """The kernel's divisibility / quotient magics (Lemire, Kaser & Kurz 2019) restated in C and
+    checked exhaustively over all 16-bit pairs and on random 32-bit pairs against % and /."""
+    src = tmp_path / "magic.c"
+    src.write_text(r'''
+#include <stdint.h>
+#include <stdio.h>
+int main(void) {
+  unsigned long long bad = 0;
+  for (uint32_t d = 1; d < 65536; d++) {
+    uint32_t m = 0xffffffffu / d + 1u;            /* ceil(2^32/d) mod 2^32 */
+    for (uint32_t n = 0; n < 65536; n++) {
+      int div = (uint32_t)(n * m) <= m - 1u;       /* V16 divisibility test */
+      uint32_t q = d == 1 ? n : (uint32_t)(((uint64_t)n * m) >> 32);  /* V16 quotient */
+      bad += (div != (n % d == 0)) + (q != n / d);
+    }
+  }
+  uint64_t s = 88172645463325252ull;
+  for (int i = 0; i < 20000000; i++) {
+    s ^= s << 13; s ^= s >> 7; s ^= s << 17;
+    uint32_t n = (uint32_t)s, d = (uint32_t)(s >> 32) >> (s & 31);
+    if (!d) d = 1;
+    uint64_t m = ~0ull / d + 1ull;                 /* ceil(2^64/d) mod 2^64 */
+    int div = (uint64_t)n * m <= m - 1ull;         /* V32 divisibility test */
+    uint64_t q = d == 1 ? n : (uint64_t)(((unsigned __int128)m * n) >> 64);  /* V32 quotient */
+    bad += (div != (n % d == 0)) + (q != n / d);
+  }
+  printf("%llu\n", bad);
+  return 0;
+}
+''')
+    exe = tmp_path / "magic"
+    subprocess.check_call(["gcc", "-O2", "-o", str(exe), str(src)])
+    assert subprocess.check_output([str(exe)], timeout=300).strip() == b"0"

@@ -1,0 +1,236 @@
+"""GPU parity: the CUDA path (through the C ABI) vs the CPU oracle, bit-exact.
+
+Integer work throughout: sizes (u128), per-level node counts f_k, every decoded
+configuration (small spaces, all indices) and order-dependent hashes of whole
+groups / sampled decodes at full size (goldens written by tests/golden/make_golden.py,
+which calls only oracle/).  Every input is a deterministic spec from atfspec or a
+seeded fuzz spec.
+"""
+import json
+import os
+
+import numpy as np
+import pytest
+
+import atfspec as A
+from atfspec.fuzz import splitmix64_indices
+from oracle import closed_forms as cf
+from oracle import run as orc
+
+torch = pytest.importorskip("torch")
+pytestmark = pytest.mark.gpu
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+@pytest.fixture(scope="module")
+def Space():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_hpdc_raschg18_b200 import Space as S
+    return S
+
+
+def _flags(generic):
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    return L.ATF_FLAG_GENERIC_ONLY if generic else 0
+
+
+def torch_rowhash(rows_pm: "torch.Tensor", base: int = 0) -> int:
+    """Same definition as the oracle's: H = sum_i rowhash(row_i) * (2 (base+i) + 1) mod 2^64.
+    rows_pm: int32 [P, n] (SoA), computed on the GPU with wrapping int64 arithmetic."""
+    P, n = rows_pm.shape
+    M32 = 0xFFFFFFFF
+    z = torch.full((n,), 0x243F6A8885A308D3, dtype=torch.int64, device=rows_pm.device)
+    K = torch.tensor(0x9E3779B97F4A7C15 - (1 << 64), dtype=torch.int64, device=rows_pm.device)
+    for p in range(P):
+        z = z ^ (rows_pm[p].to(torch.int64) & M32)
+        z = z * K
+        z = z ^ ((z >> 32) & M32)
+    w = torch.arange(base, base + n, dtype=torch.int64, device=rows_pm.device) * 2 + 1
+    s = (z * w).sum()  # wraps mod 2^64
+    return int(s.item()) & ((1 << 64) - 1)
+
+
+def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000):
+    ref = orc.info(spec, threads=8)
+    with Space(spec, flags=_flags(generic)) as sp:
+        sp.generate()
+        assert sp.groups() == [g["members"] for g in ref["groups"]]
+        assert sp.size() == int(ref["S"])
+        assert sp.group_sizes() == [g["size"] for g in ref["groups"]]
+        for g, grp in enumerate(ref["groups"]):
+            assert sp.level_sizes(g) == [lv["f"] for lv in grp["levels"]], (spec.name, g)
+        st = sp.stats()
+        evals = [lv["evals"] for grp in ref["groups"] for lv in grp["levels"]]
+        assert [x["evals"] for x in st] == evals
+        S = sp.size()
+        if 0 < S <= decode_all_max:
+            idx = torch.arange(S, dtype=torch.int64, device="cuda")
+            got = sp.decode(idx).cpu().numpy()
+            _, want = orc.decode(spec, np.arange(S, dtype=np.uint64))
+            assert np.array_equal(got, want), spec.name
+
+
+SMALL = {
+    "C1": A.c1_toy,
+    "fig1": A.fig1,
+    "saxpy64": lambda: A.saxpy(64),
+    "saxpy360": lambda: A.saxpy(360),
+    "saxpy1": lambda: A.saxpy(1),
+    "C2-32": lambda: A.c2_xgemm_direct(32),
+    "C2-256": lambda: A.c2_xgemm_direct(256),
+    "C2-64-noimplied": lambda: A.c2_xgemm_direct(64, implied=False),
+    "C3-12x30x8": lambda: A.c3_xgemm((12, 30, 8)),
+    "C3-IS1": lambda: A.c3_xgemm("IS1"),
+    "C3-IS3": lambda: A.c3_xgemm("IS3"),
+    "C3-IS4-anch": lambda: A.c3_xgemm("IS4", anchored=True),
+    "C5-60x5": lambda: A.c5_chains(60, 5),
+    "C5-300x4": lambda: A.c5_chains(300, 4),
+}
+
+
+@pytest.mark.parametrize("name", list(SMALL))
+@pytest.mark.parametrize("generic", [False, True])
+def test_small_specs(Space, name, generic):
+    _check_against_oracle(Space, SMALL[name](), generic=generic)
+
+
+@pytest.mark.parametrize("seed", range(80))
+def test_fuzz_specs(Space, seed):
+    _check_against_oracle(Space, A.random_spec(seed))
+
+
+@pytest.mark.parametrize("seed", range(0, 80, 4))
+def test_fuzz_specs_generic(Space, seed):
+    _check_against_oracle(Space, A.random_spec(seed), generic=True)
+
+
+def test_wide_ranges_chunked(Space):
+    """r > 4096 candidates per level -> several candidate chunks per frontier node."""
+    _check_against_oracle(Space, A.saxpy(5040 * 4))
+    s = A.Spec("wide")
+    s.add("a", A.interval(1, 12))
+    s.add("b", A.interval(1, 20000), A.divides(A.P(0) * 1000) | (A.X > 19990))
+    _check_against_oracle(Space, s)
+
+
+def test_empty_space(Space):
+    s = A.Spec("cltune_wgd")
+    s.add("WGD", A.set_(8, 16, 32), A.divides(20) & A.divides(576))
+    s.add("KWID", A.interval(1, 32), A.divides(A.P(0)))
+    with Space(s) as sp:
+        sp.generate()
+        assert sp.size() == 0 and sp.level_sizes(0) == [0, 0]
+        from paper_conf_hpdc_raschg18_b200 import AtfError
+        with pytest.raises(AtfError):
+            sp.decode(torch.zeros(3, dtype=torch.int64, device="cuda"))
+
+
+def test_decode_out_of_range_rows(Space):
+    from paper_conf_hpdc_raschg18_b200 import AtfError
+    with Space(A.fig1()) as sp:
+        sp.generate()
+        idx = torch.tensor([0, 8, 9, 1 << 40], dtype=torch.int64, device="cuda")
+        out = torch.empty((4, 4), dtype=torch.int32, device="cuda")
+        with pytest.raises(AtfError) as e:
+            sp.decode(idx, out=out)
+        assert e.value.status == -8
+        o = out.cpu().numpy()
+        assert (o[:, 2:] == np.iinfo(np.int32).min).all()
+        assert o[:, 0].tolist() == [1, 1, 1, 1] and o[:, 1].tolist() == [2, 2, 2, 2]
+
+
+def test_csr_and_records_consistent(Space):
+    spec = A.c3_xgemm((12, 30, 8))
+    with Space(spec) as sp:
+        sp.generate()
+        L = sp.num_levels(0)
+        for k in range(L - 1):
+            v, nv = sp.level_view(0, k), sp.level_view(0, k + 1)
+            n, W = v["n_nodes"], v["words"]
+            csr = torch.empty(n + 1, dtype=torch.int64, device="cuda")
+            torch.cuda.cudart().cudaMemcpy(csr.data_ptr(), v["csr"], (n + 1) * 8, 3)
+            csr = csr.cpu().numpy()
+            assert csr[0] == 0 and csr[-1] == nv["n_nodes"] and (np.diff(csr) >= 0).all()
+
+
+@pytest.mark.parametrize("n", [0, 1, 31, 1024, 1025, 1 << 20, 3_000_001])
+def test_lookback_scan(Space, n):
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    g = torch.Generator().manual_seed(n)
+    for kind in ("rand", "zeros", "max", "one_huge"):
+        if kind == "rand":
+            x = torch.randint(0, 1000, (n,), generator=g, dtype=torch.int64)
+        elif kind == "zeros":
+            x = torch.zeros(n, dtype=torch.int64)
+        elif kind == "max":
+            x = torch.full((n,), 0xFFFFFFFF, dtype=torch.int64)
+        else:
+            x = torch.zeros(n, dtype=torch.int64)
+            if n:
+                x[n // 2] = 0xFFFFFFFF
+        d_in = x.to(torch.int32).cuda() if n else torch.zeros(1, dtype=torch.int32, device="cuda")
+        d_out = torch.empty(n + 1, dtype=torch.int64, device="cuda")
+        L.check(L.atf_test_exclusive_scan_u32(d_in.data_ptr(), d_out.data_ptr(), n, None))
+        want = np.concatenate([[0], np.cumsum(x.numpy().astype(np.uint64))]).astype(np.uint64)
+        assert np.array_equal(d_out.cpu().numpy().view(np.uint64), want), kind
+
+
+# ---------------------------------------------------------------- full sizes (goldens)
+def _golden(name):
+    with open(os.path.join(GOLDEN, f"{name}.json")) as f:
+        return json.load(f)
+
+
+def _group_hash(sp, g, size, n_params, chunk=1 << 24):
+    """Hash of group g's leaves (values of its members) in canonical order, via decode_digits."""
+    G = sp.num_groups()
+    members = sp.groups()[g]
+    H = 0
+    for s0 in range(0, size, chunk):
+        n = min(chunk, size - s0)
+        dig = torch.zeros((G, n), dtype=torch.int64, device="cuda")
+        dig[g] = torch.arange(s0, s0 + n, dtype=torch.int64, device="cuda")
+        out = sp.decode_digits(dig)
+        H = (H + torch_rowhash(out[members], base=s0)) & ((1 << 64) - 1)
+        del out, dig
+    return H
+
+
+@pytest.mark.parametrize("name", ["C2", "C2-1024", "C3-IS1", "C3-IS3", "C3-IS2", "C3-IS4", "C3-IS4-anchored", "C5-512"])
+def test_full_size_against_golden(Space, name):
+    from tests.golden.make_golden import SPECS
+    gold = _golden(name)
+    spec = SPECS[name]()
+    with Space(spec) as sp:
+        sp.generate()
+        assert sp.size() == int(gold["S"])
+        for g, grp in enumerate(gold["groups"]):
+            assert sp.level_sizes(g) == [lv["f"] for lv in grp["levels"]]
+            assert _group_hash(sp, g, grp["size"], len(spec.params)) == int(grp["hash"]), (name, g)
+        if "decode" in gold:
+            d = gold["decode"]
+            idx = torch.from_numpy(splitmix64_indices(d["n"], int(gold["S"]), d["seed"]).view(np.int64)).cuda()
+            out = sp.decode(idx)
+            assert torch_rowhash(out) == int(d["hash"])
+            assert out[:, :8].T.cpu().tolist() == d["first_rows"]
+
+
+def test_c5_full_closed_form(Space):
+    """C5 at full size (configs[4]): f_k = D_k(4096) for the x/y chains and D_k(2048) for z
+    (Piltz; oracle/closed_forms.py), S = product of the leaf levels (u128)."""
+    spec = A.c5_chains(4096, 8)
+    want = cf.c5_level_sizes(4096, 8)
+    with Space(spec) as sp:
+        sp.generate()
+        assert [sp.level_sizes(g) for g in range(3)] == want
+        assert sp.size() == want[0][-1] * want[1][-1] * want[2][-1]
+        # sampled decode: rows are valid configurations (checked by the oracle's constraint test)
+        dig = torch.stack([torch.randint(0, want[g][-1], (4096,), device="cuda") for g in range(3)])
+        rows = sp.decode_digits(dig).T.contiguous().cpu().numpy()
+        chk = orc.check(spec, rows)
+        assert chk["valid"] == chk["rows"] == 4096
+        # lexicographic extremes: digit 0 = the first valid tuple in range-position order
+        first = sp.decode_digits(torch.zeros((3, 1), dtype=torch.int64, device="cuda")).flatten().tolist()
+        assert first == [1] * 16 + [2] * 8
