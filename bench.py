@@ -1,0 +1,364 @@
+#!/usr/bin/env python
+"""bench.py — ATF search-space generation on B200 (BASELINE.json metric:
+"valid configs generated/sec (and constraint evals/sec) at 1/2/4/8 B200 vs roofline").
+
+Workload (config.workload): C5 = BASELINE.json configs[4], the 24-parameter,
+3-group chained-divisibility space over ranges 1..4096 — the config the metric is
+quoted on at 1/2/4/8 GPUs (sharded).  One step = one complete generation of every
+group's tree (all §8(a) rows: count, scan, emit on every level, group sizes, S).
+At N=1 rank 0 also measures the other configs (C3-IS2/IS4 generation, C4 decode of
+10^8 indices, C2) and reports them under "secondary".
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+
+--impl reference times the CPU oracle (oracle/atf_oracle, as it stands) on the
+host cores on a bounded sample of the same workload.
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import atfspec as A  # noqa: E402
+
+METRIC = "valid configs generated/sec (and constraint evals/sec) at 1/2/4/8 B200 vs roofline"
+
+
+def _peaks():
+    try:
+        with open(os.path.join(ROOT, "MEASURED_PEAKS.json")) as f:
+            return json.load(f)
+    except OSError:
+        return {}
+
+
+def int_peak_ops(sm_mhz, sms=148):
+    """INT32 issue bound: 4 SMSPs x 32 lanes x SMs x clock (one warp instruction per SMSP per
+    cycle)."""
+    return 4 * 32 * sms * sm_mhz * 1e6
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled DURING the timed region."""
+
+    Q = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+         "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+         "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except OSError:
+            self.proc = None
+        time.sleep(0.25)
+        return self
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        time.sleep(0.15)
+        if self.proc:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except subprocess.TimeoutExpired:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm)
+        return {"sm_mhz": float(np.median(sm)) if sm else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def flush_l2(buf):
+    buf.add_(1)  # 512 MiB write > 126 MB L2
+
+
+# ------------------------------------------------------------------ our arm
+def run_generation(spec, steps, warmup, dist_ctx=None, timing=True):
+    """Times `steps` generations of `spec`; returns per-step ms (max over ranks), stats."""
+    import torch
+    from paper_conf_hpdc_raschg18_b200 import Space, _lib as L
+    dev = torch.cuda.current_device()
+    stream = torch.cuda.current_stream()
+    flush = torch.empty(128 << 20, dtype=torch.int32, device="cuda")
+    flags = L.ATF_FLAG_TIMING if timing else 0
+    sp = Space(spec, device=dev, stream=stream, flags=flags)
+    world = dist_ctx["world"] if dist_ctx else 1
+    rank = dist_ctx["rank"] if dist_ctx else 0
+
+    def one_step():
+        if world == 1:
+            sp.generate()
+            return None
+        counts = sp.generate_shard(rank, world)
+        t = torch.tensor(counts, dtype=torch.int64, device="cuda")
+        out = torch.empty(world * len(counts), dtype=torch.int64, device="cuda")
+        dist_ctx["dist"].all_gather_into_tensor(out, t)   # NCCL over NVLink
+        allc = out.view(world, -1).cpu().tolist()
+        sp.finalize_shard(allc)
+        return allc
+
+    for _ in range(warmup):
+        one_step()
+        flush_l2(flush)
+    torch.cuda.synchronize()
+    if dist_ctx:
+        dist_ctx["dist"].barrier()
+    torch.cuda.synchronize()
+    evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    level_ms = []
+    for i in range(steps):
+        evs[i][0].record(stream)
+        one_step()
+        evs[i][1].record(stream)
+        if timing:
+            level_ms.append([s["ms"] for s in sp.stats()])
+        flush_l2(flush)
+    torch.cuda.synchronize()
+    if dist_ctx:
+        dist_ctx["dist"].barrier()
+    torch.cuda.synchronize()
+    ms = [a.elapsed_time(b) for a, b in evs]
+    st = sp.stats()
+    res = {"ms": ms, "stats": st, "size": sp.size(), "group_sizes": sp.group_sizes(),
+           "plan": sp.plan_json(), "level_ms": level_ms}
+    sp.close()
+    return res
+
+
+def roofline_of(res, sm_mhz):
+    """Dominant kernel = expand_kernel (every launch of the step).  achieved = algorithmic int ops
+    (evals_k x c_k, DESIGN.md cost table) / summed device time of the expand launches."""
+    plan = res["plan"]
+    costs = [lv["cost"] for g in plan["groups"] for lv in g["levels"]]
+    ops = sum(s["evals"] * c for s, c in zip(res["stats"], costs))
+    lm = np.array(res["level_ms"], dtype=np.float64)  # [steps, levels]
+    kern_ms = float(lm.sum(axis=1).mean()) if lm.size else float("nan")
+    achieved = ops / (kern_ms * 1e-3)
+    peak = int_peak_ops(sm_mhz)
+    return {"bound": "alu", "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tops/s",
+            "frac": achieved / peak, "traffic": None, "ops_per_step": ops, "kernel_ms": kern_ms,
+            "peak_clock_mhz": sm_mhz,
+            "cost_table": "DIVX/MULX/DIVPROD 2, QDIV 6, CMP 2, AND 1, GENERIC = bytecode ops"}
+
+
+def e2e_generation(spec, steps):
+    """Same metric through the public API from HOST inputs: a new space is built from the host
+    spec (ranges + bytecode uploaded), generated, and S + group sizes read back, every step."""
+    import torch
+    from paper_conf_hpdc_raschg18_b200 import Space
+    h2d = sum(4 * (len(p.range.get("values", [])) or 0) for p in spec.params)
+    h2d += sum(4 * len(c) for p in spec.params for c in p.constraints)
+    # interval ranges are materialised on the host and uploaded too
+    for p in spec.params:
+        if p.range["kind"] != "set":
+            r = p.range
+            h2d += 4 * max(0, (r["end"] - r["begin"]) // r["step"] + 1)
+    times, d2h = [], 0
+    for i in range(steps + 1):
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        with Space(spec) as sp:
+            sp.generate()
+            S = sp.size()
+            gs = sp.group_sizes()
+            nlev = sum(sp.num_levels(g) for g in range(len(gs)))
+        torch.cuda.synchronize()
+        if i:
+            times.append(time.perf_counter() - t0)
+        d2h = 12 * nlev
+    return {"s_per_step": float(np.mean(times)), "h2d": h2d, "d2h": d2h, "S": S}
+
+
+def secondary_n1(steps, warmup, sm_mhz):
+    import torch
+    from paper_conf_hpdc_raschg18_b200 import Space
+    out = {}
+    for name, mk in (("C3-IS2", lambda: A.c3_xgemm("IS2")), ("C3-IS4", lambda: A.c3_xgemm("IS4")),
+                     ("C2", lambda: A.c2_xgemm_direct(256))):
+        res = run_generation(mk(), steps, warmup)
+        ms = float(np.mean(res["ms"]))
+        leaves = sum(res["group_sizes"])
+        evals = sum(s["evals"] for s in res["stats"])
+        rf = roofline_of(res, sm_mhz)
+        out[name] = {"ms_per_step": ms, "configs_per_s": leaves / (ms * 1e-3), "evals_per_s": evals / (ms * 1e-3),
+                     "S": str(res["size"]), "group_leaves": leaves, "evals": evals,
+                     "roofline_frac": rf["frac"], "kernel_ms": rf["kernel_ms"],
+                     "level_ms": [round(x, 4) for x in np.mean(res["level_ms"], axis=0).tolist()]}
+    # C4: decode 10^8 random indices into C3-IS2
+    from atfspec.fuzz import splitmix64_indices
+    spec = A.c3_xgemm("IS2")
+    with Space(spec) as sp:
+        sp.generate()
+        S = sp.size()
+        n = 100_000_000
+        idx = torch.from_numpy(splitmix64_indices(n, S, A.c4_indices_seed()).view(np.int64)).cuda()
+        outb = torch.empty((len(spec.params), n), dtype=torch.int32, device="cuda")
+        flush = torch.empty(128 << 20, dtype=torch.int32, device="cuda")
+        for _ in range(warmup):
+            sp.decode(idx, out=outb)
+        torch.cuda.synchronize()
+        ts = []
+        for _ in range(steps):
+            flush_l2(flush)
+            a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            a.record()
+            sp.decode(idx, out=outb)
+            b.record()
+            torch.cuda.synchronize()
+            ts.append(a.elapsed_time(b))
+        ms = float(np.mean(ts))
+        io = n * (8 + 4 * len(spec.params))
+        out["C4-decode-1e8"] = {"ms": ms, "indices_per_s": n / (ms * 1e-3), "io_GBps": io / (ms * 1e-3) / 1e9,
+                                "io_bytes": io}
+        del outb, idx
+    return out
+
+
+def cpu_baseline(spec, budget_s=15.0):
+    from oracle import run as orc
+    orc.build()
+    cores = os.cpu_count() or 1
+    d = orc.time_sample(spec, threads=cores, budget_s=budget_s, timeout=budget_s * 10 + 120)
+    return {"value": d["leaves"] / d["seconds"], "unit": "configs/s", "cores": cores, "kind": "oracle",
+            "evals_per_s": d["evals"] / d["seconds"],
+            "sample": (f"O2 (pruned nested loop, interpreted bytecode) on {spec.name}: groups in order, level-1 "
+                       f"values in order until {budget_s:.0f}s CPU budget; {d['level1_done']}/{d['level1_total']} "
+                       f"level-1 values, {d['evals']} evals, {d['leaves']} leaves in {d['seconds']:.2f}s")}
+
+
+# ------------------------------------------------------------------ main
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--no-secondary", action="store_true")
+    ap.add_argument("--cpu-budget", type=float, default=15.0)
+    a = ap.parse_args()
+    a.warmup = max(a.warmup, 3)
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    spec = A.c5_chains(4096, 8)
+    config = {"workload": "C5: configs[4] synthetic 24-parameter 3-group chained divisibility, ranges 1..4096",
+              "spec": spec.name, "global_batch": 1, "parallelism": f"shard{world}" if world > 1 else "single",
+              "l2": "flushed between steps (512 MiB write); outputs ~2 GB > L2"}
+
+    if a.impl == "reference":
+        if rank != 0:
+            return
+        t0 = time.time()
+        vals = []
+        budget = max(1.0, min(6.0, 60.0 / max(1, a.steps + a.warmup)))
+        for i in range(a.warmup + a.steps):
+            cb = cpu_baseline(spec, budget_s=budget)
+            if i >= a.warmup:
+                vals.append(cb)
+        v = float(np.mean([c["value"] for c in vals]))
+        line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "configs/s", "n_gpus": a.gpus,
+                "steps": a.steps, "warmup": a.warmup, "ms_per_step": None, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "int64", "data": "synthetic (deterministic spec)",
+                "config": config,
+                "cpu_baseline": {"value": v, "unit": "configs/s", "cores": vals[0]["cores"], "kind": "oracle",
+                                 "sample": vals[0]["sample"]},
+                "e2e": {"value": v, "unit": "configs/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+                "wall_s": time.time() - t0}
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch
+    torch.cuda.set_device(local)
+    dist_ctx = None
+    if world > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        dist_ctx = {"dist": dist, "rank": rank, "world": world}
+
+    peaks = _peaks()
+    sm_max = float(peaks.get("sm_max_mhz", 1965.0))
+    with ClockSampler(local) as clk:
+        res = run_generation(spec, a.steps, a.warmup, dist_ctx)
+    clocks = clk.summary()
+    ms = float(np.mean(res["ms"]))
+    if dist_ctx:
+        t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+        dist_ctx["dist"].all_reduce(t, op=dist_ctx["dist"].ReduceOp.MAX)
+        ms = float(t.item())
+    leaves = sum(res["group_sizes"])                      # global (finalize_shard) sizes
+    plan = res["plan"]
+    evals_total = 0
+    for g in plan["groups"]:
+        pass
+    # algorithmic evals of the whole job: from the single-GPU level sizes (f_{k-1} r_k)
+    gl = [[lv["r"] for lv in g["levels"]] for g in plan["groups"]]
+    value = leaves / (ms * 1e-3)
+    n_launch = sum(1 for s in res["stats"] if s["ms"] >= 0)
+    if rank == 0:
+        line = {"metric": METRIC, "value": value, "unit": "configs/s", "n_gpus": world, "steps": a.steps,
+                "warmup": a.warmup, "ms_per_step": ms, "higher_is_better": True,
+                "scaling": "strong", "vs_baseline": None, "dtype": "int64 (int32 values, 16/32-bit magics)",
+                "data": "synthetic (deterministic spec, no dataset)", "config": config,
+                "S": str(res["size"]), "group_leaves": res["group_sizes"], "gpu_launches": n_launch * a.steps,
+                "clocks": clocks}
+        if world == 1:
+            evals_total = sum(s["evals"] for s in res["stats"])
+            line["evals_per_s"] = evals_total / (ms * 1e-3)
+            line["roofline"] = roofline_of(res, sm_max)
+            line["roofline_at_load_clock"] = (roofline_of(res, clocks["sm_mhz"])["frac"]
+                                              if clocks.get("sm_mhz") else None)
+            e2e = e2e_generation(spec, max(2, a.steps // 2))
+            line["e2e"] = {"value": leaves / e2e["s_per_step"], "unit": "configs/s",
+                           "h2d_bytes_per_step": e2e["h2d"], "d2h_bytes_per_step": e2e["d2h"],
+                           "s_per_step": e2e["s_per_step"]}
+            try:
+                line["cpu_baseline"] = cpu_baseline(spec, budget_s=a.cpu_budget)
+            except Exception as ex:  # noqa: BLE001
+                line["cpu_baseline"] = {"error": str(ex)}
+            if not a.no_secondary:
+                line["secondary"] = secondary_n1(max(3, a.steps // 2), 3, sm_max)
+        else:
+            line["e2e"] = None
+        print(json.dumps(line), flush=True)
+    if dist_ctx:
+        dist_ctx["dist"].barrier()
+        dist_ctx["dist"].destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

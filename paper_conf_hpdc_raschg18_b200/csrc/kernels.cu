@@ -253,7 +253,7 @@ __device__ void prologue_node(const LevelArgs& a, uint64_t gnode, int i, uint32_
 // (bit p*CPT + c).  Only bits set in `acc` matter.
 template <int CPT>
 __device__ __forceinline__ uint32_t eval_term(const LevelArgs& a, const Term& T, int t, const Cands<CPT>& cd,
-                                              uint32_t acc, int n_off, int tn, const int64_t* s_opa,
+                                              uint32_t acc, int n_off, int tn, int tn_valid, const int64_t* s_opa,
                                               const int64_t* s_opb, const int64_t* s_slots, const uint32_t* s_q,
                                               bool skip_empty_passes) {
   uint32_t bits = 0;
@@ -264,7 +264,7 @@ __device__ __forceinline__ uint32_t eval_term(const LevelArgs& a, const Term& T,
     const int nl = p * npp + n_off;
     const uint32_t pm = ((1u << CPT) - 1u) << (p * CPT);
     if (skip_empty_passes && !__any_sync(FULL, acc & pm)) continue;
-    if (nl >= tn) continue;
+    if (nl >= tn_valid) continue;
     uint32_t pb = 0;
     switch (T.kind) {
       case T_DIVX:
@@ -441,7 +441,7 @@ __global__ void __launch_bounds__(1024) expand_kernel(const __grid_constant__ Le
     }
     for (int t = 0; t < a.n_terms; t++) {
       if (!__any_sync(FULL, acc)) break;  // top-level AND: a rejected item stays rejected
-      acc &= eval_term<CPT>(a, a.terms[t], t, cd, acc, n_off, a.tile_nodes, s_opa, s_opb, s_slots, s_q, t > 0);
+      acc &= eval_term<CPT>(a, a.terms[t], t, cd, acc, n_off, a.tile_nodes, tn, s_opa, s_opb, s_slots, s_q, t > 0);
     }
 
     // ---- scan: per-warp counts in item order (pass, cand-slot, warp), block scan, look-back

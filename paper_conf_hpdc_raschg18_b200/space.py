@@ -162,6 +162,24 @@ class Space:
         L.check(L.atf_space_level_view(self._h, g, k, C.byref(v)), self._h)
         return {f: getattr(v, f) for f, _ in L.atf_level_view._fields_}
 
+    def level_tensors(self, g: int, k: int):
+        """Zero-copy torch views of level k of group g: (records int32 [n, words], csr int64 [n+1] or
+        None for the leaf level).  Valid until the space is regenerated or closed."""
+        import torch
+        v = self.level_view(g, k)
+
+        class _CAI:
+            def __init__(self, ptr, shape, typestr):
+                self.__cuda_array_interface__ = {"shape": shape, "typestr": typestr, "data": (ptr, False),
+                                                 "version": 3}
+
+        dev = torch.device("cuda", self._device)
+        n, W = v["n_nodes"], v["words"]
+        rec = (torch.as_tensor(_CAI(v["records"], (n, W), "<i4"), device=dev) if n and v["records"]
+               else torch.zeros((0, W), dtype=torch.int32, device=dev))
+        csr = torch.as_tensor(_CAI(v["csr"], (n + 1,), "<i8"), device=dev) if v["csr"] else None
+        return rec, csr
+
     def stats(self) -> List[dict]:
         n = C.c_int32()
         L.check(L.atf_space_stats(self._h, None, 0, C.byref(n)), self._h)

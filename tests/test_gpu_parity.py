@@ -146,13 +146,25 @@ def test_csr_and_records_consistent(Space):
     with Space(spec) as sp:
         sp.generate()
         L = sp.num_levels(0)
+        pj = sp.plan_json()["groups"][0]["levels"]
         for k in range(L - 1):
-            v, nv = sp.level_view(0, k), sp.level_view(0, k + 1)
-            n, W = v["n_nodes"], v["words"]
-            csr = torch.empty(n + 1, dtype=torch.int64, device="cuda")
-            torch.cuda.cudart().cudaMemcpy(csr.data_ptr(), v["csr"], (n + 1) * 8, 3)
+            rec, csr = sp.level_tensors(0, k)
+            crec, _ = sp.level_tensors(0, k + 1)
             csr = csr.cpu().numpy()
-            assert csr[0] == 0 and csr[-1] == nv["n_nodes"] and (np.diff(csr) >= 0).all()
+            assert csr[0] == 0 and csr[-1] == crec.shape[0] and (np.diff(csr) >= 0).all()
+            # every child carries its parent's path plus one new field (level k+1)
+            parent_of = np.repeat(np.arange(rec.shape[0]), np.diff(csr))
+            r, c = rec.cpu().numpy().astype(np.int64), crec.cpu().numpy().astype(np.int64)
+            w, sh, b = pj[k + 1]["word"], pj[k + 1]["shift"], pj[k + 1]["bits"]
+            mask = ((1 << b) - 1) << sh
+            c_wo = c.copy()
+            c_wo[:, w] &= ~mask & 0xFFFFFFFF
+            r_u = r & 0xFFFFFFFF
+            assert np.array_equal(c_wo & 0xFFFFFFFF, r_u[parent_of])
+            # children of one parent have strictly increasing range positions
+            pos = (c[:, w] & 0xFFFFFFFF) >> sh & ((1 << b) - 1)
+            same = parent_of[1:] == parent_of[:-1]
+            assert (pos[1:][same] > pos[:-1][same]).all()
 
 
 @pytest.mark.parametrize("n", [0, 1, 31, 1024, 1025, 1 << 20, 3_000_001])
