@@ -123,13 +123,8 @@ def run_generation(spec, steps, warmup, dist_ctx=None, timing=True):
         if world == 1:
             sp.generate()
             return None
-        counts = sp.generate_shard(rank, world)
-        t = torch.tensor(counts, dtype=torch.int64, device="cuda")
-        out = torch.empty(world * len(counts), dtype=torch.int64, device="cuda")
-        dist_ctx["dist"].all_gather_into_tensor(out, t)   # NCCL over NVLink
-        allc = out.view(world, -1).cpu().tolist()
-        sp.finalize_shard(allc)
-        return allc
+        from paper_conf_hpdc_raschg18_b200.shard import generate_sharded
+        return generate_sharded(sp)   # counts all-gathered over NCCL (NVLink)
 
     for _ in range(warmup):
         one_step()

@@ -6,6 +6,14 @@
  * against std::exclusive_scan on adversarial count arrays.
  *   d_in:  device uint32[n]; d_out: device uint64[n + 1]; d_out[n] = total.
  *   Scratch is allocated internally (cudaMallocAsync on `stream`).  Synchronous.
+ *
+ * atf_test_shard_slice / atf_test_shard_offsets: the host logic of the multi-GPU shard
+ * layer (atf_space_generate_shard / atf_space_finalize_shard use the
+ * same functions), callable without a GPU.
+ *   shard_slice:   h_csr[0..ncut] (host) = child-count prefix of the cut level; writes the
+ *                  rank's contiguous slice [*lo, *hi) balanced by children.
+ *   shard_offsets: h_all[world][n] (host, rank-major) per-rank counts; writes, per entry,
+ *                  before[i] = sum over ranks < rank and tot[i] = sum over all ranks.
  */
 #ifndef ATFGEN_TEST_H
 #define ATFGEN_TEST_H
@@ -14,6 +22,10 @@
 extern "C" {
 #endif
 atf_status atf_test_exclusive_scan_u32(const uint32_t* d_in, uint64_t* d_out, int64_t n, void* stream);
+atf_status atf_test_shard_slice(const uint64_t* h_csr, uint64_t ncut, int32_t rank, int32_t world, uint64_t* lo,
+                                uint64_t* hi);
+atf_status atf_test_shard_offsets(const int64_t* h_all, int32_t world, int32_t n, int32_t rank, uint64_t* before,
+                                  uint64_t* tot);
 #ifdef __cplusplus
 }
 #endif

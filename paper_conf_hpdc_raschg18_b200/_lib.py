@@ -81,6 +81,10 @@ _SIGS = {
     "atf_space_last_error": (C.c_char_p, [SP]),
     # include/atfgen_test.h
     "atf_test_exclusive_scan_u32": (_st, [C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p]),
+    "atf_test_shard_slice": (_st, [C.POINTER(C.c_uint64), C.c_uint64, C.c_int32, C.c_int32,
+                                   C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
+    "atf_test_shard_offsets": (_st, [C.POINTER(C.c_int64), C.c_int32, C.c_int32, C.c_int32,
+                                     C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
 }
 
 EXPORTED = tuple(_SIGS)

@@ -77,14 +77,29 @@ struct LevelArgs {
   unsigned long long* total_out;
   uint64_t child_cap;       // capacity of child_rec in records
   unsigned int* overflow_flag;
-  // geometry
-  int32_t block, cpt, npp, np;
-  int32_t tile_nodes;       // nodes per tile (np * npp), 1 if n_chunks > 1
-  int64_t n_chunks;         // candidate chunks per node (r > block*cpt)
+  // geometry (host choose_geometry)
+  int32_t kind;             // K_NARROW: one thread per frontier node, r <= 64 candidates each
+                            // K_WIDE:   each thread owns cpt consecutive candidates of a chunk
+  int32_t block, cpt;
+  int32_t hot, hot_term;    // wide: HOT_* filter of term hot_term evaluated in the hot loop
+  int32_t tile_nodes;       // frontier nodes per tile (wide: multiple of 4)
+  int32_t chunk;            // wide: candidates per chunk (= block * cpt)
+  int32_t rw, sw;           // wide: bitmap words per node (chunk/32), summary words (ceil(rw/32))
+  int32_t qcap;             // wide: slow-path queue entries per tile
+  int64_t n_chunks;         // candidate chunks per node (r > chunk); tile_nodes == 4 padded, 1 real
   uint64_t n_tiles;
   uint32_t qmax;            // T_QDIV table covers quotients [0, qmax]
   int32_t smem_bytes;
 };
+enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1 };
+// Hot-loop filter of the wide kernel: a superset test of one conjunct, 2 instructions per
+// (node, candidate) pair (IMAD + ISETP.OR into a per-node predicate).
+enum HotKind : int32_t {
+  HOT_NONE = 0,  // no filter: every (node, candidate) is evaluated exactly ("dense")
+  HOT_DIVX = 1,  // x | n   (T_DIVX / T_DIVPROD, V16): n * ceil(2^32/x) <= ceil(2^32/x) - 1
+  HOT_MULX = 2,  // d | x   (T_MULX, V16):            x * ceil(2^32/d) <= ceil(2^32/d) - 1
+};
+constexpr uint32_t kHotSentinel = 65521;  // largest 16-bit prime: hot operand of rejected nodes
 
 // Decode: index -> per-group digit (mixed radix, group 0 most significant) ->
 // leaf record -> range positions -> values.
@@ -100,24 +115,38 @@ struct DecodeArgs {
   const int32_t* lvl_range[kMaxLevels];
 };
 
-// Dynamic shared-memory layout of the expand kernel (byte offsets; -1 = absent).
+// Dynamic shared-memory layouts of the expand kernels (byte offsets; -1 = absent).
 struct SmemLayout {
-  int ctl, ok, rec, opa, opb, slots, wcnt, wtot, qtab, total;
+  int ctl, ok, rec, opa, opb, slots, hot, hot2, cnt, off, sum, bm, q, cx, cm, qtab, wtot, total;
 };
 ATF_HD int align16(int x) { return (x + 15) & ~15; }
 ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
   SmemLayout L;
   const int tn = a.tile_nodes;
+  const bool wide = a.kind == K_WIDE;
+  const int nc = wide ? a.chunk : a.r;  // candidate table entries
   int o = 0;
-  L.ctl = o; o += 32;
+  L.ctl = o; o += 64;
   L.ok = o; o = align16(o + 4 * tn);
   L.rec = o; o = align16(o + 4 * words * tn);
   L.opa = o; o = align16(o + 8 * a.n_terms * tn);
   L.opb = o; o = align16(o + 8 * a.n_terms * tn);
   if (a.need_slots_smem) { L.slots = o; o = align16(o + 8 * a.n_slots * tn); } else { L.slots = -1; }
-  L.wcnt = o; o = align16(o + 4 * (a.np * a.cpt * (a.block / 32) + 1));
-  L.wtot = o; o = align16(o + 4 * 33);
+  if (wide) {
+    L.hot = o; o = align16(o + 4 * tn);
+    L.hot2 = o; o = align16(o + 4 * tn);
+    L.cnt = o; o = align16(o + 4 * tn);
+    L.off = o; o = align16(o + 4 * tn);
+    L.sum = o; o = align16(o + 4 * tn * a.sw);
+    L.bm = o; o = align16(o + 4 * tn * a.rw);
+    L.q = o; o = align16(o + 4 * a.qcap);
+  } else {
+    L.hot = L.hot2 = L.cnt = L.off = L.sum = L.bm = L.q = -1;
+  }
+  L.cx = o; o = align16(o + 4 * (nc > 0 ? nc : 1));
+  L.cm = o; o = align16(o + 4 * (nc > 0 ? nc : 1));
   if (a.qmax > 0) { L.qtab = o; o = align16(o + 4 * ((int)a.qmax + 1)); } else { L.qtab = -1; }
+  L.wtot = o; o = align16(o + 8 * 34);
   L.total = o;
   return L;
 }

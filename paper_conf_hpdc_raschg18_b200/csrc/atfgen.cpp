@@ -698,50 +698,47 @@ static atf_status plan(atf_space* s) {
 }
 
 // ---------------------------------------------------------------- geometry
+// r <= 64 -> narrow kernel (thread per node); otherwise the wide
+// kernel with cpt candidates per thread, a hot filter when a conjunct allows one, and
+// ~2^18 (node, candidate) pairs per tile.
 static void choose_geometry(LevelArgs& a, int words) {
   const int r = a.r;
-  int B, cpt = 1, npp = 1;
-  int64_t n_chunks = 1;
-  if (r <= 1024) {
-    int best = -1;
-    double bu = -1;
-    for (int b = 32; b <= 1024; b += 32) {
-      if (b < r) continue;
-      int k = b / r;
-      double u = (double)k * r / b;
-      // prefer utilisation, then ~512 threads
-      double score = u - 1e-4 * std::abs(b - 512) / 512.0;
-      if (b < 256 && r < 256) score -= 1e-3;
-      if (score > bu) { bu = score; best = b; }
-    }
-    B = best;
-    npp = B / r;
+  a.hot = HOT_NONE;
+  a.hot_term = 0;
+  a.n_chunks = 1;
+  a.rw = a.sw = a.qcap = 0;
+  if (r <= 64) {
+    a.kind = K_NARROW;
+    a.block = 256;
+    a.cpt = 1;
+    a.tile_nodes = 256;
+    a.chunk = r;
   } else {
-    cpt = 2;
-    while (cpt < 8 && (r + cpt - 1) / cpt > 512) cpt *= 2;
-    int per = (r + cpt - 1) / cpt;
-    if (per > 512) per = 512;
-    B = (per + 31) / 32 * 32;
-    n_chunks = ((int64_t)r + (int64_t)B * cpt - 1) / ((int64_t)B * cpt);
+    a.kind = K_WIDE;
+    for (int t = 0; t < a.n_terms; t++) {
+      const Term& T = a.terms[t];
+      if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) { a.hot = HOT_DIVX; a.hot_term = t; break; }
+      if (T.kind == T_MULX && T.variant == V16) { a.hot = HOT_MULX; a.hot_term = t; break; }
+    }
+    double best = 1e30;
+    for (int cpt : {4, 8, 16}) {
+      int64_t per = ((int64_t)r + cpt - 1) / cpt;
+      int B = (int)std::min<int64_t>(512, (per + 31) / 32 * 32);
+      int64_t nch = ((int64_t)r + (int64_t)B * cpt - 1) / ((int64_t)B * cpt);
+      double cost = (2.0 + 6.0 / (4.0 * cpt)) * (double)((int64_t)B * cpt * nch) / r;
+      if (cost < best - 1e-9) { best = cost; a.cpt = cpt; a.block = B; a.n_chunks = nch; }
+    }
+    a.chunk = a.block * a.cpt;
+    a.rw = a.chunk / 32;
+    a.sw = (a.rw + 31) / 32;
+    int nt = a.n_chunks > 1 ? 4 : std::max(4, std::min(256, ((1 << 18) / a.chunk + 3) / 4 * 4));
+    for (;;) {
+      a.tile_nodes = nt;
+      a.qcap = std::min(4096, nt / 4 * a.block);
+      if (nt <= 4 || expand_layout(a, words).total <= 72 * 1024) break;
+      nt = std::max(4, (nt / 2 + 3) / 4 * 4);
+    }
   }
-  a.block = B;
-  a.cpt = cpt;
-  a.npp = npp;
-  a.n_chunks = n_chunks;
-  // passes per tile: bounded by 32 bits per thread and ~96 KB of shared memory
-  int per_node = 4 + 4 * words + 16 * a.n_terms + (a.need_slots_smem ? 8 * a.n_slots : 0);
-  int NW = B / 32;
-  int np = n_chunks > 1 ? 1 : 32 / cpt;
-  while (np > 1) {
-    a.np = np;
-    a.tile_nodes = np * npp;
-    if (expand_layout(a, words).total <= 96 * 1024) break;
-    np--;
-  }
-  (void)per_node;
-  (void)NW;
-  a.np = np;
-  a.tile_nodes = n_chunks > 1 ? 1 : np * npp;
   a.smem_bytes = expand_layout(a, words).total;
 }
 
@@ -871,6 +868,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   choose_geometry(a, gp.words);
   a.n_tiles = a.n_chunks > 1 ? n_parents * (uint64_t)a.n_chunks
                              : (n_parents + (uint64_t)a.tile_nodes - 1) / (uint64_t)a.tile_nodes;
+  if (a.smem_bytes > 227 * 1024)
+    return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %d bytes of shared memory", k, g, a.smem_bytes);
   if (a.n_tiles >= 0xffffffffull) return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %llu tiles", k, g,
                                               (unsigned long long)a.n_tiles);
   atf_status e = ensure_status(s, a.n_tiles);
@@ -1038,6 +1037,34 @@ static atf_status make_decode_args(const atf_space* s, DecodeArgs& a) {
   }
   a.lvl_begin[a.n_groups] = l;
   return ATF_OK;
+}
+
+// ---------------------------------------------------------------- shard host logic
+// S§8(e).  Rank `rank` of `world` takes the contiguous slice [lo, hi) of the cut level
+// whose child-count prefix (csr[0..ncut], csr[ncut] = T children) lies in
+// [rank*T/world, (rank+1)*T/world): contiguity keeps each rank's leaves a contiguous range
+// of the canonical order; balancing by children evens out the expansion below the cut.
+static void shard_slice(const uint64_t* csr, uint64_t ncut, int rank, int world, uint64_t* lo, uint64_t* hi) {
+  const uint64_t T = csr[ncut];
+  auto bound = [&](int r_) -> uint64_t {  // first cut node whose child prefix >= r T / world
+    u128 target = (u128)T * (u128)r_ / (u128)world;
+    return (uint64_t)(std::lower_bound(csr, csr + ncut + 1, (uint64_t)target) - csr);
+  };
+  *lo = rank == 0 ? 0 : std::min<uint64_t>(bound(rank), ncut);
+  *hi = rank == world - 1 ? ncut : std::min<uint64_t>(bound(rank + 1), ncut);
+  if (*hi < *lo) *hi = *lo;
+}
+// all: [world][n] per-rank counts (rank-major).  Entry idx: the global offset of rank's
+// part (exclusive scan over ranks) and the global total.
+static void shard_offsets(const int64_t* all, int world, int n, int idx, int rank, uint64_t* before,
+                          uint64_t* tot) {
+  *before = 0;
+  *tot = 0;
+  for (int r = 0; r < world; r++) {
+    const uint64_t c = (uint64_t)all[(size_t)r * n + idx];
+    if (r < rank) *before += c;
+    *tot += c;
+  }
 }
 
 // ================================================================= C ABI
@@ -1424,14 +1451,8 @@ atf_status atf_space_generate_shard(atf_space* s, int32_t rank, int32_t world, i
     std::vector<uint64_t> csr(ncut + 1);
     CUDA_TRY(s, cudaMemcpyAsync(csr.data(), cutd.csr, (ncut + 1) * 8, cudaMemcpyDeviceToHost, st));
     CUDA_TRY(s, cudaStreamSynchronize(st));
-    const uint64_t T = csr[ncut];
-    auto bound = [&](int r_) -> uint64_t {  // first cut node whose child prefix >= r T / world
-      u128 target = (u128)T * (u128)r_ / (u128)world;
-      return (uint64_t)(std::lower_bound(csr.begin(), csr.end(), (uint64_t)target) - csr.begin());
-    };
-    uint64_t lo = rank == 0 ? 0 : std::min<uint64_t>(bound(rank), ncut);
-    uint64_t hi = rank == world - 1 ? ncut : std::min<uint64_t>(bound(rank + 1), ncut);
-    if (hi < lo) hi = lo;
+    uint64_t lo = 0, hi = 0;
+    shard_slice(csr.data(), ncut, rank, world, &lo, &hi);
     // slice of level k*+1 = children of cut nodes [lo, hi)
     LevelData& nd = s->data[g][kc + 1];
     uint64_t c0 = csr[lo], c1 = csr[hi];
@@ -1475,11 +1496,7 @@ atf_status atf_space_finalize_shard(atf_space* s, const int64_t* all, int32_t wo
     for (size_t k = 0; k < s->groups[g].levels.size(); k++, idx++) {
       if (idx >= n) return fail(s, ATF_ERR_INVALID_ARG, "counts too short");
       uint64_t before = 0, tot = 0;
-      for (int r = 0; r < world; r++) {
-        uint64_t c = (uint64_t)all[(size_t)r * n + idx];
-        if (r < s->shard_rank) before += c;
-        tot += c;
-      }
+      shard_offsets(all, world, n, idx, s->shard_rank, &before, &tot);
       LevelData& d = s->data[g][k];
       if ((int)k >= s->shard_cut[g]) {
         uint64_t old = d.offset;
@@ -1516,6 +1533,20 @@ atf_status atf_test_exclusive_scan_u32(const uint32_t* d_in, uint64_t* d_out, in
   cudaFreeAsync(status, st);
   cudaFreeAsync(counter, st);
   return cudaStreamSynchronize(st) == cudaSuccess ? ATF_OK : ATF_ERR_CUDA;
+}
+
+atf_status atf_test_shard_slice(const uint64_t* h_csr, uint64_t ncut, int32_t rank, int32_t world, uint64_t* lo,
+                                uint64_t* hi) {
+  if (!h_csr || !lo || !hi || world < 1 || rank < 0 || rank >= world) return ATF_ERR_INVALID_ARG;
+  shard_slice(h_csr, ncut, rank, world, lo, hi);
+  return ATF_OK;
+}
+
+atf_status atf_test_shard_offsets(const int64_t* h_all, int32_t world, int32_t n, int32_t rank, uint64_t* before,
+                                  uint64_t* tot) {
+  if (!h_all || !before || !tot || world < 1 || n < 0 || rank < 0 || rank >= world) return ATF_ERR_INVALID_ARG;
+  for (int i = 0; i < n; i++) shard_offsets(h_all, world, n, i, rank, before + i, tot + i);
+  return ATF_OK;
 }
 
 void atf_space_destroy(atf_space* s) {

@@ -1,0 +1,593 @@
+// expand.cuh — the level-expansion kernels (SURVEY.md §8(a) A4-A6 fused: count, scan,
+// emit), instantiated per record width W in expand_w{1,2,4,8}.cu.
+#pragma once
+#include "dev_common.cuh"
+
+namespace atf {
+
+// ---------------------------------------------------------------- exact term evaluation
+// One (frontier node, candidate) pair against conjunct T (SURVEY.md §8(b) semantics; the
+// planner's atoms are exact rewrites of the bytecode).  A, Bv: the
+// node's operands of T (prologue); x: candidate value, ax = |x|, m32 = ceil(2^32/ax)
+// (0 for ax <= 1).  slots/stride: the node's slot column (generic terms only).
+__device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, int64_t A, int64_t Bv, int32_t x,
+                                             uint32_t ax, uint32_t m32, const uint32_t* s_q, const int64_t* slots,
+                                             int stride) {
+  switch (T.kind) {
+    case T_DIVX:
+    case T_DIVPROD: {  // x | n   (n = A = |m| or |b/a|); x == 0 -> poison -> reject
+      if (ax == 0) return false;
+      const uint64_t n = (uint64_t)A;
+      if (T.variant == V16) return (uint32_t)n * m32 <= m32 - 1u;
+      if (T.variant == V32) {
+        const uint64_t m64 = ~0ull / ax + 1ull;
+        return n * m64 <= m64 - 1ull;
+      }
+      return n % ax == 0;
+    }
+    case T_MULX: {  // d | x  (d = A != 0 checked by the node gate, Bv = magic(d))
+      const uint64_t d = (uint64_t)A, md = (uint64_t)Bv;
+      if (T.variant == V16) return ax * (uint32_t)md <= (uint32_t)md - 1u;
+      if (T.variant == V32) return (uint64_t)ax * md <= md - 1ull;
+      return d != 0 && (uint64_t)ax % d == 0;
+    }
+    case T_QDIV: {  // (num / x) | nb; x == 0 or quotient 0 -> poison -> reject
+      if (ax == 0) return false;
+      const uint64_t num = (uint64_t)A, nb = (uint64_t)Bv;
+      if (T.variant == V16) {
+        const uint32_t q = ax == 1 ? (uint32_t)num : __umulhi((uint32_t)num, m32);
+        if (q == 0) return false;
+        if (T.use_qtable) {
+          const uint32_t mq = s_q[q];
+          return (uint32_t)nb * mq <= mq - 1u;
+        }
+        return (uint32_t)nb % q == 0;
+      }
+      const uint64_t q = num / ax;
+      return q != 0 && nb % q == 0;
+    }
+    case T_CMP:
+      if (T.variant == V32) return rel_holds32(T.rel, (int32_t)A * x, (int32_t)Bv);
+      return rel_holds(T.rel, A * (int64_t)x, Bv);
+    default: {  // T_GENERIC: interpret the conjunct
+      bool poison = false;
+      const int64_t v = run_code(a.code + T.code_off, T.code_len, x, slots, stride, poison);
+      return !poison && v != 0;
+    }
+  }
+}
+
+// Candidate-table entries: value and 32-bit divisibility magic.
+__device__ __forceinline__ uint32_t cand_magic(int32_t x) {
+  const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+  return ax ? 0xffffffffu / ax + 1u : 0u;
+}
+
+// Exact acceptance of candidate (x, m32) by node i of the tile (all conjuncts, node gate).
+static __device__ __noinline__ bool node_accepts(const LevelArgs& a, int i, int tn, int32_t x, uint32_t m32,
+                                             const uint32_t* s_ok, const int64_t* s_opa, const int64_t* s_opb,
+                                             const int64_t* s_slots, const uint32_t* s_q) {
+  if (!s_ok[i]) return false;
+  const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+  for (int t = 0; t < a.n_terms; t++)
+    if (!term_accepts(a, a.terms[t], s_opa[t * tn + i], s_opb[t * tn + i], x, ax, m32, s_q,
+                      s_slots ? s_slots + i : nullptr, tn))
+      return false;
+  return true;
+}
+
+// ---------------------------------------------------------------- records
+template <int W>
+__device__ __forceinline__ void store_record(uint32_t* dst, const uint32_t* rec) {
+  if constexpr (W == 1) {
+    dst[0] = rec[0];
+  } else if constexpr (W == 2) {
+    *reinterpret_cast<uint2*>(dst) = make_uint2(rec[0], rec[1]);
+  } else if constexpr (W == 4) {
+    *reinterpret_cast<uint4*>(dst) = make_uint4(rec[0], rec[1], rec[2], rec[3]);
+  } else {
+    *reinterpret_cast<uint4*>(dst) = make_uint4(rec[0], rec[1], rec[2], rec[3]);
+    *reinterpret_cast<uint4*>(dst + 4) = make_uint4(rec[4], rec[5], rec[6], rec[7]);
+  }
+}
+
+template <int W>
+__device__ __forceinline__ void load_record(const uint32_t* src, uint32_t* rec) {
+  if constexpr (W == 1) {
+    rec[0] = __ldg(src);
+  } else if constexpr (W == 2) {
+    const uint2 v = __ldg(reinterpret_cast<const uint2*>(src));
+    rec[0] = v.x; rec[1] = v.y;
+  } else {
+#pragma unroll
+    for (int q = 0; q < W / 4; q++) {
+      const uint4 v = __ldg(reinterpret_cast<const uint4*>(src) + q);
+      rec[4 * q] = v.x; rec[4 * q + 1] = v.y; rec[4 * q + 2] = v.z; rec[4 * q + 3] = v.w;
+    }
+  }
+}
+
+// Per-node prologue: unpack ancestor values from the parent's path record, evaluate the
+// hoisted node-invariant expressions, the node gates and every conjunct's operands into
+// shared memory (node `i` of the tile, global index gnode).  Returns the gate result.
+template <int W>
+__device__ __noinline__ bool prologue_node(const LevelArgs& a, uint64_t gnode, int i, int tn, uint32_t* s_ok, uint32_t* s_rec,
+                              int64_t* s_opa, int64_t* s_opb, int64_t* s_slots) {
+  uint32_t rec[W];
+  if (a.level == 0) {
+#pragma unroll
+    for (int w = 0; w < W; w++) rec[w] = 0;
+  } else {
+    load_record<W>(a.parent_rec + gnode * W, rec);
+  }
+#pragma unroll
+  for (int w = 0; w < W; w++) s_rec[i * W + w] = rec[w];
+  int64_t slots[kMaxSlots];
+  for (int s = 0; s < a.n_pv; s++) {
+    uint32_t word = 0;
+#pragma unroll
+    for (int w = 0; w < W; w++)
+      if (w == a.pv_word[s]) word = rec[w];
+    const uint32_t bits = (uint32_t)a.pv_bits[s];
+    const uint32_t pos = bits ? (word >> a.pv_shift[s]) & ((bits >= 32) ? 0xffffffffu : ((1u << bits) - 1u)) : 0u;
+    slots[s] = a.pv_range[s][pos];
+  }
+  bool poison = false;
+  for (int s = a.n_pv; s < a.n_slots; s++)
+    slots[s] = run_code(a.code + a.inv_off[s], a.inv_len[s], 0, slots, 1, poison);
+  bool ok = !poison;
+  for (int g = 0; g < a.n_gates; g++) ok = ok && (slots[a.gate_slot[g]] != 0);
+  for (int t = 0; t < a.n_terms; t++) {
+    const Term& T = a.terms[t];
+    int64_t A = 0, B = 0;
+    switch (T.kind) {
+      case T_CMP: A = slots[T.slot_a]; B = slots[T.slot_b]; break;
+      case T_DIVX: A = (int64_t)uabs64(slots[T.slot_a]); break;
+      case T_MULX: {
+        const uint64_t d = uabs64(slots[T.slot_a]);
+        if (d == 0) ok = false;
+        A = (int64_t)d;
+        if (T.variant == V16) B = d ? (int64_t)(0xffffffffu / (uint32_t)d + 1u) : 0;
+        else if (T.variant == V32) B = d ? (int64_t)(~0ull / d + 1ull) : 0;
+        break;
+      }
+      case T_DIVPROD: {
+        const uint64_t av = uabs64(slots[T.slot_a]), bv = uabs64(slots[T.slot_b]);
+        if (av == 0) { ok = false; A = 0; }
+        else if (bv % av != 0) { ok = false; A = 0; }
+        else A = (int64_t)(bv / av);
+        break;
+      }
+      case T_QDIV: A = (int64_t)uabs64(slots[T.slot_a]); B = (int64_t)uabs64(slots[T.slot_b]); break;
+      default: break;
+    }
+    s_opa[t * tn + i] = A;
+    s_opb[t * tn + i] = B;
+  }
+  if (s_slots)
+    for (int s = 0; s < a.n_slots; s++) s_slots[s * tn + i] = slots[s];
+  s_ok[i] = ok ? 1u : 0u;
+  return ok;
+}
+
+// Block-wide exclusive scan of one u32 per thread (B <= 1024); returns the exclusive
+// prefix, *total = block sum.  s_w: >= 33 u64 of shared scratch.  Ends with a barrier.
+__device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* total, unsigned long long* s_w) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, NW = blockDim.x >> 5;
+  uint32_t incl = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, incl, o);
+    if (lane >= o) incl += y;
+  }
+  if (lane == 31) s_w[warp] = incl;
+  __syncthreads();
+  if (warp == 0) {
+    const uint32_t wt = lane < NW ? (uint32_t)s_w[lane] : 0u;
+    uint32_t wi = wt;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, wi, o);
+      if (lane >= o) wi += y;
+    }
+    if (lane < NW) s_w[lane] = wi - wt;
+    if (lane == 31) s_w[32] = wi;
+  }
+  __syncthreads();
+  *total = (uint32_t)s_w[32];
+  return incl - v + (uint32_t)s_w[warp];
+}
+
+// ---------------------------------------------------------------- narrow expand kernel
+// One launch = one tree level of one group, for ranges of r <= 64 candidates.  One
+// thread per frontier node (tile = blockDim.x nodes): prologue -> exact evaluation of the
+// r candidates into a 64-bit accept mask (count, A4) -> block scan + decoupled look-back
+// (A5) -> CSR + the node's children records in candidate order (emit, A6).
+template <int W>
+__global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ LevelArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const SmemLayout L = expand_layout(a, W);
+  uint32_t* ctl = reinterpret_cast<uint32_t*>(smem + L.ctl);
+  uint32_t* s_ok = reinterpret_cast<uint32_t*>(smem + L.ok);
+  uint32_t* s_rec = reinterpret_cast<uint32_t*>(smem + L.rec);
+  int64_t* s_opa = reinterpret_cast<int64_t*>(smem + L.opa);
+  int64_t* s_opb = reinterpret_cast<int64_t*>(smem + L.opb);
+  int64_t* s_slots = L.slots >= 0 ? reinterpret_cast<int64_t*>(smem + L.slots) : nullptr;
+  int32_t* s_cx = reinterpret_cast<int32_t*>(smem + L.cx);
+  uint32_t* s_cm = reinterpret_cast<uint32_t*>(smem + L.cm);
+  uint32_t* s_q = L.qtab >= 0 ? reinterpret_cast<uint32_t*>(smem + L.qtab) : nullptr;
+  unsigned long long* s_w = reinterpret_cast<unsigned long long*>(smem + L.wtot);
+
+  const int tid = threadIdx.x, lane = tid & 31, B = blockDim.x;
+  const int r = a.r, tn_max = a.tile_nodes;
+  for (int j = tid; j < r; j += B) {
+    const int32_t x = __ldg(a.cand + j);
+    s_cx[j] = x;
+    s_cm[j] = cand_magic(x);
+  }
+  if (s_q)
+    for (uint32_t q = tid; q <= a.qmax; q += B) s_q[q] = q ? (0xffffffffu / q + 1u) : 0u;
+
+  for (;;) {
+    if (tid == 0) ctl[0] = atomicAdd(a.tile_counter, 1u);
+    __syncthreads();
+    const uint64_t tile = ctl[0];
+    if (tile >= a.n_tiles) break;
+    const uint64_t node0 = tile * (uint64_t)tn_max;
+    const uint64_t rem = a.n_parents - node0;
+    const int tn = rem < (uint64_t)tn_max ? (int)rem : tn_max;
+    const int i = tid;
+    uint64_t mask = 0;
+    if (i < tn && prologue_node<W>(a, node0 + i, i, tn_max, s_ok, s_rec, s_opa, s_opb, s_slots)) {
+      mask = r >= 64 ? ~0ull : ((1ull << r) - 1ull);
+      for (int t = 0; t < a.n_terms && mask; t++) {
+        const Term& T = a.terms[t];
+        const int64_t A = s_opa[t * tn_max + i], Bv = s_opb[t * tn_max + i];
+        uint64_t mt = 0;
+        for (int c = 0; c < r; c++) {
+          if (!((mask >> c) & 1ull)) continue;
+          const int32_t x = s_cx[c];
+          const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+          if (term_accepts(a, T, A, Bv, x, ax, s_cm[c], s_q, s_slots ? s_slots + i : nullptr, tn_max))
+            mt |= 1ull << c;
+        }
+        mask &= mt;
+      }
+    }
+    uint32_t total;
+    const uint32_t excl = block_excl_scan((uint32_t)__popcll(mask), &total, s_w);
+    if (tid < 32) {
+      const unsigned long long base = lookback(a.status, tile, total, lane);
+      if (lane == 0) {
+        s_w[33] = base;
+        if (tile == a.n_tiles - 1) {
+          *a.total_out = base + total;
+          a.csr[a.n_parents] = base + total;
+        }
+      }
+    }
+    __syncthreads();
+    const uint64_t base = s_w[33];
+    if (i < tn) {
+      uint64_t rank = base + excl;
+      a.csr[node0 + i] = rank;
+      uint32_t rec[W];
+#pragma unroll
+      for (int w = 0; w < W; w++) rec[w] = s_rec[i * W + w];
+      uint64_t m = mask;
+      while (m) {
+        const int c = __ffsll((long long)m) - 1;
+        m &= m - 1;
+        if (rank < a.child_cap) {
+          uint32_t out[W];
+#pragma unroll
+          for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? (uint32_t)c << a.field_shift : 0u);
+          store_record<W>(a.child_rec + rank * W, out);
+        } else {
+          atomicOr(a.overflow_flag, 1u);
+        }
+        rank++;
+      }
+    }
+    __syncthreads();
+  }
+}
+
+// ---------------------------------------------------------------- wide expand kernel
+// One launch = one tree level of one group, for ranges of r > 64 candidates.  Tile =
+// tile_nodes frontier nodes x one chunk of `chunk` candidates; thread t owns candidate
+// positions [t*CPT, t*CPT + CPT) of the chunk for the whole launch (values/magics in
+// registers).  Per tile:
+//   prologue  one thread per node: path record -> ancestor values -> operands (smem)
+//   hot loop  (A4) every (node, candidate) pair through the HOT filter: IMAD + ISETP.OR,
+//             a superset of the accepted pairs; a thread whose CPT candidates pass for any
+//             of 4 consecutive nodes queues (node quad, thread) in shared memory
+//   slow path the queued pairs are re-evaluated exactly (all conjuncts), flattened over
+//             the block; accepted pairs set bits of a per-node candidate bitmap (smem)
+//             and bump the node's count.  Queue overflow -> the tile is evaluated densely.
+//   scan      (A5) block scan of node counts + decoupled look-back -> CSR offsets
+//   emit      (A6) per node, set bitmap words in order: lane b writes the child of bit b
+//             (coalesced), records = parent record | position; consumed words are zeroed.
+template <int W, int CPT, int HOT>
+__global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ LevelArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  const SmemLayout L = expand_layout(a, W);
+  uint32_t* ctl = reinterpret_cast<uint32_t*>(smem + L.ctl);
+  uint32_t* s_ok = reinterpret_cast<uint32_t*>(smem + L.ok);
+  uint32_t* s_rec = reinterpret_cast<uint32_t*>(smem + L.rec);
+  int64_t* s_opa = reinterpret_cast<int64_t*>(smem + L.opa);
+  int64_t* s_opb = reinterpret_cast<int64_t*>(smem + L.opb);
+  int64_t* s_slots = L.slots >= 0 ? reinterpret_cast<int64_t*>(smem + L.slots) : nullptr;
+  uint32_t* s_hot = reinterpret_cast<uint32_t*>(smem + L.hot);
+  uint32_t* s_hot2 = reinterpret_cast<uint32_t*>(smem + L.hot2);
+  uint32_t* s_cnt = reinterpret_cast<uint32_t*>(smem + L.cnt);
+  uint32_t* s_off = reinterpret_cast<uint32_t*>(smem + L.off);
+  uint32_t* s_sum = reinterpret_cast<uint32_t*>(smem + L.sum);
+  uint32_t* s_bm = reinterpret_cast<uint32_t*>(smem + L.bm);
+  uint32_t* s_qe = reinterpret_cast<uint32_t*>(smem + L.q);
+  int32_t* s_cx = reinterpret_cast<int32_t*>(smem + L.cx);
+  uint32_t* s_cm = reinterpret_cast<uint32_t*>(smem + L.cm);
+  uint32_t* s_q = L.qtab >= 0 ? reinterpret_cast<uint32_t*>(smem + L.qtab) : nullptr;
+  unsigned long long* s_w = reinterpret_cast<unsigned long long*>(smem + L.wtot);
+
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int B = blockDim.x, NW = B >> 5;
+  const int r = a.r, NT = a.tile_nodes, RW = a.rw, SW = a.sw, chunk = a.chunk;
+  const int hot_t = a.hot_term;
+
+  for (int k = tid; k < NT * RW; k += B) s_bm[k] = 0u;
+  for (int k = tid; k < NT * SW; k += B) s_sum[k] = 0u;
+  for (int k = tid; k < NT; k += B) s_cnt[k] = 0u;
+  if (s_q)
+    for (uint32_t q = tid; q <= a.qmax; q += B) s_q[q] = q ? (0xffffffffu / q + 1u) : 0u;
+
+  // candidate table of the current chunk: value and 32-bit divisibility magic
+  auto load_chunk = [&](int64_t ch) {
+    const int64_t j0 = ch * (int64_t)chunk;
+    for (int k = tid; k < chunk; k += B) {
+      const int64_t j = j0 + k;
+      const int32_t x = j < r ? __ldg(a.cand + j) : 0;
+      s_cx[k] = x;
+      s_cm[k] = cand_magic(x);
+    }
+  };
+  if (a.n_chunks == 1) load_chunk(0);
+
+  for (;;) {
+    if (tid == 0) {
+      ctl[0] = atomicAdd(a.tile_counter, 1u);
+      ctl[1] = 0u;  // queue length
+    }
+    __syncthreads();
+    const uint64_t tile = ctl[0];
+    if (tile >= a.n_tiles) break;
+    uint64_t node0;
+    int64_t ch = 0;
+    int tn;
+    if (a.n_chunks == 1) {
+      node0 = tile * (uint64_t)NT;
+      const uint64_t rem = a.n_parents - node0;
+      tn = rem < (uint64_t)NT ? (int)rem : NT;
+    } else {
+      node0 = tile / (uint64_t)a.n_chunks;
+      ch = (int64_t)(tile % (uint64_t)a.n_chunks);
+      tn = 1;
+      load_chunk(ch);
+    }
+    const int64_t j0 = ch * (int64_t)chunk;
+    // ---- prologue
+    for (int i = tid; i < NT; i += B) {
+      if (i < tn) {
+        const bool ok = prologue_node<W>(a, node0 + i, i, NT, s_ok, s_rec, s_opa, s_opb, s_slots);
+        if (HOT == HOT_DIVX) {
+          s_hot[i] = ok ? (uint32_t)s_opa[hot_t * NT + i] : kHotSentinel;
+        } else if (HOT == HOT_MULX) {
+          const uint32_t md = ok ? (uint32_t)s_opb[hot_t * NT + i] : (0xffffffffu / kHotSentinel + 1u);
+          s_hot[i] = md;
+          s_hot2[i] = md - 1u;
+        }
+      } else {
+        s_ok[i] = 0u;
+        s_hot[i] = HOT == HOT_MULX ? (0xffffffffu / kHotSentinel + 1u) : kHotSentinel;
+        s_hot2[i] = (0xffffffffu / kHotSentinel);
+      }
+    }
+    __syncthreads();
+
+    // ---- hot loop (A4): superset filter, queue (node quad, thread) on a possible accept
+    bool dense = HOT == HOT_NONE;
+    if (HOT != HOT_NONE) {
+      // registers (reloaded per tile so they are not live across the prologue):
+      // HOT_DIVX: hm = ceil(2^32/|x|), hm1 = hm - 1; HOT_MULX: hm = |x|.  Invalid slots
+      // and x == 0 get values that flag at most n == 0 / d == 1 (the slow path rejects).
+      uint32_t hm[CPT], hm1[CPT];
+#pragma unroll
+      for (int c = 0; c < CPT; c++) {
+        const int jl = tid * CPT + c;
+        const bool v = j0 + jl < r;
+        const int32_t x = s_cx[jl];
+        const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+        if (HOT == HOT_DIVX) {
+          hm[c] = (v && ax) ? s_cm[jl] : 1u;
+          hm1[c] = (v && ax) ? s_cm[jl] - 1u : 0u;
+        } else {
+          hm[c] = v ? ax : 1u;
+          hm1[c] = 0u;
+        }
+      }
+      for (int g = 0; g < tn; g += 4) {
+        const uint4 n4 = *reinterpret_cast<const uint4*>(s_hot + g);
+        bool h0 = false, h1 = false, h2 = false, h3 = false;
+        if (HOT == HOT_DIVX) {
+#pragma unroll
+          for (int c = 0; c < CPT; c++) {
+            h0 |= n4.x * hm[c] <= hm1[c];
+            h1 |= n4.y * hm[c] <= hm1[c];
+            h2 |= n4.z * hm[c] <= hm1[c];
+            h3 |= n4.w * hm[c] <= hm1[c];
+          }
+        } else {
+          const uint4 d4 = *reinterpret_cast<const uint4*>(s_hot2 + g);
+#pragma unroll
+          for (int c = 0; c < CPT; c++) {
+            h0 |= hm[c] * n4.x <= d4.x;
+            h1 |= hm[c] * n4.y <= d4.y;
+            h2 |= hm[c] * n4.z <= d4.z;
+            h3 |= hm[c] * n4.w <= d4.w;
+          }
+        }
+        if (h0 | h1 | h2 | h3) {
+          const uint32_t slot = atomicAdd(&ctl[1], 1u);
+          if (slot < (uint32_t)a.qcap) s_qe[slot] = ((uint32_t)(g >> 2) << 16) | (uint32_t)tid;
+        }
+      }
+      __syncthreads();
+      const uint32_t nq = ctl[1];
+      if (nq > (uint32_t)a.qcap) {
+        dense = true;
+      } else {
+        // ---- slow path: exact evaluation of the queued pairs, flattened over the block
+        const uint32_t items = nq * 4u * CPT;
+        for (uint32_t k = tid; k < items; k += B) {
+          const uint32_t e = s_qe[k / (4 * CPT)];
+          const uint32_t w4 = k % (4 * CPT);
+          const int i = (int)((e >> 16) * 4u + w4 / CPT);
+          const int jl = (int)((e & 0xffffu) * CPT + w4 % CPT);
+          if (i < tn && j0 + jl < r &&
+              node_accepts(a, i, NT, s_cx[jl], s_cm[jl], s_ok, s_opa, s_opb, s_slots, s_q)) {
+            atomicOr(&s_bm[i * RW + (jl >> 5)], 1u << (jl & 31));
+            atomicOr(&s_sum[i * SW + (jl >> 10)], 1u << ((jl >> 5) & 31));
+            atomicAdd(&s_cnt[i], 1u);
+          }
+        }
+      }
+    }
+    if (dense) {
+      // every (node, candidate) pair of the tile exactly; thread-owned candidates
+      const int jl0 = tid * CPT;
+      for (int i = 0; i < tn; i++) {
+        if (!s_ok[i]) continue;
+        uint32_t m = 0;
+#pragma unroll
+        for (int c = 0; c < CPT; c++)
+          if (j0 + jl0 + c < r &&
+              node_accepts(a, i, NT, s_cx[jl0 + c], s_cm[jl0 + c], s_ok, s_opa, s_opb, s_slots, s_q))
+            m |= 1u << c;
+        if (m) {
+          atomicOr(&s_bm[i * RW + (jl0 >> 5)], m << (jl0 & 31));
+          atomicOr(&s_sum[i * SW + (jl0 >> 10)], 1u << ((jl0 >> 5) & 31));
+          atomicAdd(&s_cnt[i], (uint32_t)__popc(m));
+        }
+      }
+    }
+    __syncthreads();
+
+    // ---- scan (A5): node counts -> tile offsets; look-back -> tile base
+    if (warp == 0) {
+      uint32_t run = 0;
+      for (int i0 = 0; i0 < tn; i0 += 32) {
+        const int i = i0 + lane;
+        const uint32_t v = i < tn ? s_cnt[i] : 0u;
+        uint32_t incl = v;
+#pragma unroll
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t y = __shfl_up_sync(FULL, incl, o);
+          if (lane >= o) incl += y;
+        }
+        if (i < tn) s_off[i] = run + incl - v;
+        run += __shfl_sync(FULL, incl, 31);
+      }
+      const unsigned long long base = lookback(a.status, tile, run, lane);
+      if (lane == 0) {
+        s_w[33] = base;
+        if (tile == a.n_tiles - 1) {
+          *a.total_out = base + run;
+          a.csr[a.n_parents] = base + run;
+        }
+      }
+    }
+    __syncthreads();
+    const uint64_t base = s_w[33];
+
+    // ---- emit (A6)
+    if (ch == 0)
+      for (int i = tid; i < tn; i += B) a.csr[node0 + i] = base + s_off[i];
+    const unsigned lt = (1u << lane) - 1u;
+    for (int i = warp; i < tn; i += NW) {
+      const uint32_t cnt = s_cnt[i];
+      if (cnt == 0) continue;
+      uint64_t rank = base + s_off[i];
+      uint32_t rec[W];
+#pragma unroll
+      for (int w = 0; w < W; w++) rec[w] = s_rec[i * W + w];
+      for (int sw = 0; sw < SW; sw++) {
+        uint32_t sm = s_sum[i * SW + sw];
+        while (sm) {
+          const int wi = sw * 32 + __ffs(sm) - 1;
+          sm &= sm - 1;
+          const uint32_t word = s_bm[i * RW + wi];
+          if ((word >> lane) & 1u) {
+            const uint64_t rk = rank + __popc(word & lt);
+            if (rk < a.child_cap) {
+              const uint32_t pos = (uint32_t)(j0 + wi * 32 + lane);
+              uint32_t out[W];
+#pragma unroll
+              for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? pos << a.field_shift : 0u);
+              store_record<W>(a.child_rec + rk * W, out);
+            } else {
+              atomicOr(a.overflow_flag, 1u);
+            }
+          }
+          rank += __popc(word);
+          __syncwarp();
+          if (lane == 0) s_bm[i * RW + wi] = 0u;
+        }
+        if (lane == 0) s_sum[i * SW + sw] = 0u;
+      }
+      if (lane == 0) s_cnt[i] = 0u;
+    }
+    __syncthreads();
+  }
+}
+
+template <typename K>
+static int launch_persistent(K k, const LevelArgs& a, int block, void* stream) {
+  const int smem = a.smem_bytes;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return (int)e;
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, block, smem);
+  if (e != cudaSuccess) return (int)e;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (per_sm < 1) return (int)cudaErrorInvalidConfiguration;
+  uint64_t grid = (uint64_t)sms * per_sm;  // persistent: one wave, tiles by ticket
+  if (grid > a.n_tiles) grid = a.n_tiles;
+  if (grid < 1) grid = 1;
+  k<<<(unsigned)grid, block, smem, (cudaStream_t)stream>>>(a);
+  return (int)cudaGetLastError();
+}
+
+template <int W, int CPT>
+static int launch_wide_wc(const LevelArgs& a, void* stream) {
+  switch (a.hot) {
+    case HOT_NONE: return launch_persistent(expand_wide<W, CPT, HOT_NONE>, a, a.block, stream);
+    case HOT_DIVX: return launch_persistent(expand_wide<W, CPT, HOT_DIVX>, a, a.block, stream);
+    case HOT_MULX: return launch_persistent(expand_wide<W, CPT, HOT_MULX>, a, a.block, stream);
+    default: return (int)cudaErrorInvalidValue;
+  }
+}
+
+template <int W>
+static int launch_w(const LevelArgs& a, void* stream) {
+  if (a.kind == K_NARROW) return launch_persistent(expand_narrow<W>, a, a.block, stream);
+  switch (a.cpt) {
+    case 4: return launch_wide_wc<W, 4>(a, stream);
+    case 8: return launch_wide_wc<W, 8>(a, stream);
+    case 16: return launch_wide_wc<W, 16>(a, stream);
+    default: return (int)cudaErrorInvalidValue;
+  }
+}
+
+}  // namespace atf

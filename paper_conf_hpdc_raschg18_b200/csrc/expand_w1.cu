@@ -1,0 +1,7 @@
+// expand_w1.cu — expand kernels for 1-word path records (one TU per width keeps the
+// sm_100a build parallel).
+#include "expand.cuh"
+
+namespace atf {
+int launch_expand_w1(const LevelArgs& a, void* stream) { return launch_w<1>(a, stream); }
+}  // namespace atf

@@ -1,0 +1,7 @@
+// expand_w2.cu — expand kernels for 2-word path records (one TU per width keeps the
+// sm_100a build parallel).
+#include "expand.cuh"
+
+namespace atf {
+int launch_expand_w2(const LevelArgs& a, void* stream) { return launch_w<2>(a, stream); }
+}  // namespace atf

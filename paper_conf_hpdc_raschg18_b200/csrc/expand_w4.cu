@@ -1,0 +1,7 @@
+// expand_w4.cu — expand kernels for 4-word path records (one TU per width keeps the
+// sm_100a build parallel).
+#include "expand.cuh"
+
+namespace atf {
+int launch_expand_w4(const LevelArgs& a, void* stream) { return launch_w<4>(a, stream); }
+}  // namespace atf

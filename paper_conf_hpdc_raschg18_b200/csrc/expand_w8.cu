@@ -1,0 +1,7 @@
+// expand_w8.cu — expand kernels for 8-word path records (one TU per width keeps the
+// sm_100a build parallel).
+#include "expand.cuh"
+
+namespace atf {
+int launch_expand_w8(const LevelArgs& a, void* stream) { return launch_w<8>(a, stream); }
+}  // namespace atf

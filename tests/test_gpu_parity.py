@@ -185,7 +185,7 @@ def test_lookback_scan(Space, n):
         d_in = x.to(torch.int32).cuda() if n else torch.zeros(1, dtype=torch.int32, device="cuda")
         d_out = torch.empty(n + 1, dtype=torch.int64, device="cuda")
         L.check(L.atf_test_exclusive_scan_u32(d_in.data_ptr(), d_out.data_ptr(), n, None))
-        want = np.concatenate([[0], np.cumsum(x.numpy().astype(np.uint64))]).astype(np.uint64)
+        want = np.concatenate([np.zeros(1, np.uint64), np.cumsum(x.numpy().astype(np.uint64))])  # exact u64 (no float64 promotion)
         assert np.array_equal(d_out.cpu().numpy().view(np.uint64), want), kind
 
 
