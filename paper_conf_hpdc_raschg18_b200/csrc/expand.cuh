@@ -293,6 +293,70 @@ __global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ Lev
   }
 }
 
+// Conjuncts other than the hot one, for the candidates still set in `mask` (bit c =
+// candidate jl0 + c of the chunk).  Out of line: only reached on hot-filter survivors.
+static __device__ __noinline__ uint32_t other_terms_mask(const LevelArgs& a, int i, int tn, int jl0, uint32_t mask,
+                                                        int skip, const int64_t* s_opa, const int64_t* s_opb,
+                                                        const int64_t* s_slots, const uint32_t* s_q,
+                                                        const int32_t* s_cx, const uint32_t* s_cm) {
+  for (int t = 0; t < a.n_terms && mask; t++) {
+    if (t == skip) continue;
+    const Term& T = a.terms[t];
+    const int64_t A = s_opa[t * tn + i], Bv = s_opb[t * tn + i];
+    uint32_t m = mask;
+    while (m) {
+      const int c = __ffs(m) - 1;
+      m &= m - 1;
+      const int32_t x = s_cx[jl0 + c];
+      const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+      if (!term_accepts(a, T, A, Bv, x, ax, s_cm[jl0 + c], s_q, s_slots ? s_slots + i : nullptr, tn))
+        mask &= ~(1u << c);
+    }
+  }
+  return mask;
+}
+
+// Exact accept mask of node i over candidates [jl0, jl0 + CPT) of the chunk, recorded in
+// the node's bitmap, summary and count (shared-memory atomics, once per call).
+template <int CPT, int HOT>
+__device__ __forceinline__ void record_mask(const LevelArgs& a, int i, int tn, int jl0, int64_t j0,
+                                            const uint32_t* s_ok, const uint32_t* s_hot, const uint32_t* s_hot2,
+                                            const int64_t* s_opa, const int64_t* s_opb, const int64_t* s_slots,
+                                            const uint32_t* s_q, const int32_t* s_cx, const uint32_t* s_cm,
+                                            uint32_t* s_bm, uint32_t* s_sum, uint32_t* s_cnt, int RW, int SW) {
+  if (!s_ok[i]) return;
+  uint32_t mask = 0;
+  if (HOT == HOT_NONE) {
+#pragma unroll
+    for (int c = 0; c < CPT; c++)
+      if (j0 + jl0 + c < a.r &&
+          node_accepts(a, i, tn, s_cx[jl0 + c], s_cm[jl0 + c], s_ok, s_opa, s_opb, s_slots, s_q))
+        mask |= 1u << c;
+  } else {
+    const uint32_t n = s_hot[i], d1 = s_hot2[i];
+#pragma unroll
+    for (int c = 0; c < CPT; c++) {
+      const int32_t x = s_cx[jl0 + c];
+      const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+      bool ok = j0 + jl0 + c < a.r;
+      if (HOT == HOT_DIVX) {
+        const uint32_t m = s_cm[jl0 + c];
+        ok = ok && ax != 0 && n * m <= m - 1u;  // exact for 16-bit operands (V16)
+      } else {
+        ok = ok && ax * n <= d1;  // n = ceil(2^32/d), d1 = n - 1
+      }
+      mask |= (uint32_t)ok << c;
+    }
+    if (mask && a.n_terms > 1)
+      mask = other_terms_mask(a, i, tn, jl0, mask, a.hot_term, s_opa, s_opb, s_slots, s_q, s_cx, s_cm);
+  }
+  if (mask) {
+    atomicOr(&s_bm[i * RW + (jl0 >> 5)], mask << (jl0 & 31));
+    atomicOr(&s_sum[i * SW + (jl0 >> 10)], 1u << ((jl0 >> 5) & 31));
+    atomicAdd(&s_cnt[i], (uint32_t)__popc(mask));
+  }
+}
+
 // ---------------------------------------------------------------- wide expand kernel
 // One launch = one tree level of one group, for ranges of r > 64 candidates.  Tile =
 // tile_nodes frontier nodes x one chunk of `chunk` candidates; thread t owns candidate
@@ -398,43 +462,39 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
     bool dense = HOT == HOT_NONE;
     if (HOT != HOT_NONE) {
       // registers (reloaded per tile so they are not live across the prologue):
-      // HOT_DIVX: hm = ceil(2^32/|x|), hm1 = hm - 1; HOT_MULX: hm = |x|.  Invalid slots
-      // and x == 0 get values that flag at most n == 0 / d == 1 (the slow path rejects).
-      uint32_t hm[CPT], hm1[CPT];
+      //   HOT_DIVX: hm = ceil(2^32/|x|).  For 16-bit n and x, (n * hm mod 2^32) < 2^16
+      //             iff x | n (exhaustively verified, tests/test_abi_cpu.py), so the
+      //             per-node test is min over the candidates < 2^16: one IMAD per pair
+      //             plus half a 3-input VIMNMX3.  Invalid slots and x == 0: hm = 2^16,
+      //             which flags only n == 0 (the slow path rejects).
+      //   HOT_MULX: hm = |x|; x * ceil(2^32/d) <= ceil(2^32/d) - 1 iff d | x, again a
+      //             min over the candidates against a per-node bound.  Invalid: hm = 1.
+      uint32_t hm[CPT];
 #pragma unroll
       for (int c = 0; c < CPT; c++) {
         const int jl = tid * CPT + c;
         const bool v = j0 + jl < r;
         const int32_t x = s_cx[jl];
         const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-        if (HOT == HOT_DIVX) {
-          hm[c] = (v && ax) ? s_cm[jl] : 1u;
-          hm1[c] = (v && ax) ? s_cm[jl] - 1u : 0u;
-        } else {
-          hm[c] = v ? ax : 1u;
-          hm1[c] = 0u;
-        }
+        if (HOT == HOT_DIVX) hm[c] = (v && ax) ? s_cm[jl] : 0x10000u;
+        else hm[c] = v ? ax : 1u;
       }
       for (int g = 0; g < tn; g += 4) {
         const uint4 n4 = *reinterpret_cast<const uint4*>(s_hot + g);
-        bool h0 = false, h1 = false, h2 = false, h3 = false;
-        if (HOT == HOT_DIVX) {
+        uint32_t m0 = 0xffffffffu, m1 = 0xffffffffu, m2 = 0xffffffffu, m3 = 0xffffffffu;
 #pragma unroll
-          for (int c = 0; c < CPT; c++) {
-            h0 |= n4.x * hm[c] <= hm1[c];
-            h1 |= n4.y * hm[c] <= hm1[c];
-            h2 |= n4.z * hm[c] <= hm1[c];
-            h3 |= n4.w * hm[c] <= hm1[c];
-          }
+        for (int c = 0; c < CPT; c++) {
+          m0 = min(m0, n4.x * hm[c]);
+          m1 = min(m1, n4.y * hm[c]);
+          m2 = min(m2, n4.z * hm[c]);
+          m3 = min(m3, n4.w * hm[c]);
+        }
+        bool h0, h1, h2, h3;
+        if (HOT == HOT_DIVX) {
+          h0 = m0 < 0x10000u; h1 = m1 < 0x10000u; h2 = m2 < 0x10000u; h3 = m3 < 0x10000u;
         } else {
           const uint4 d4 = *reinterpret_cast<const uint4*>(s_hot2 + g);
-#pragma unroll
-          for (int c = 0; c < CPT; c++) {
-            h0 |= hm[c] * n4.x <= d4.x;
-            h1 |= hm[c] * n4.y <= d4.y;
-            h2 |= hm[c] * n4.z <= d4.z;
-            h3 |= hm[c] * n4.w <= d4.w;
-          }
+          h0 = m0 <= d4.x; h1 = m1 <= d4.y; h2 = m2 <= d4.z; h3 = m3 <= d4.w;
         }
         if (h0 | h1 | h2 | h3) {
           const uint32_t slot = atomicAdd(&ctl[1], 1u);
@@ -446,39 +506,25 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
       if (nq > (uint32_t)a.qcap) {
         dense = true;
       } else {
-        // ---- slow path: exact evaluation of the queued pairs, flattened over the block
-        const uint32_t items = nq * 4u * CPT;
+        // ---- slow path: the queued (node, thread) pairs, flattened over the block; each
+        // item = one node x the thread's CPT candidates, exact (hot conjunct inline,
+        // the other conjuncts only for its survivors), one set of smem atomics per item
+        const uint32_t items = nq * 4u;
         for (uint32_t k = tid; k < items; k += B) {
-          const uint32_t e = s_qe[k / (4 * CPT)];
-          const uint32_t w4 = k % (4 * CPT);
-          const int i = (int)((e >> 16) * 4u + w4 / CPT);
-          const int jl = (int)((e & 0xffffu) * CPT + w4 % CPT);
-          if (i < tn && j0 + jl < r &&
-              node_accepts(a, i, NT, s_cx[jl], s_cm[jl], s_ok, s_opa, s_opb, s_slots, s_q)) {
-            atomicOr(&s_bm[i * RW + (jl >> 5)], 1u << (jl & 31));
-            atomicOr(&s_sum[i * SW + (jl >> 10)], 1u << ((jl >> 5) & 31));
-            atomicAdd(&s_cnt[i], 1u);
-          }
+          const uint32_t e = s_qe[k >> 2];
+          const int i = (int)((e >> 16) * 4u + (k & 3u));
+          const int jl0 = (int)((e & 0xffffu) * CPT);
+          if (i < tn) record_mask<CPT, HOT>(a, i, NT, jl0, j0, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q, s_cx,
+                                           s_cm, s_bm, s_sum, s_cnt, RW, SW);
         }
       }
     }
     if (dense) {
       // every (node, candidate) pair of the tile exactly; thread-owned candidates
       const int jl0 = tid * CPT;
-      for (int i = 0; i < tn; i++) {
-        if (!s_ok[i]) continue;
-        uint32_t m = 0;
-#pragma unroll
-        for (int c = 0; c < CPT; c++)
-          if (j0 + jl0 + c < r &&
-              node_accepts(a, i, NT, s_cx[jl0 + c], s_cm[jl0 + c], s_ok, s_opa, s_opb, s_slots, s_q))
-            m |= 1u << c;
-        if (m) {
-          atomicOr(&s_bm[i * RW + (jl0 >> 5)], m << (jl0 & 31));
-          atomicOr(&s_sum[i * SW + (jl0 >> 10)], 1u << ((jl0 >> 5) & 31));
-          atomicAdd(&s_cnt[i], (uint32_t)__popc(m));
-        }
-      }
+      for (int i = 0; i < tn; i++)
+        record_mask<CPT, HOT>(a, i, NT, jl0, j0, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q, s_cx, s_cm, s_bm,
+                              s_sum, s_cnt, RW, SW);
     }
     __syncthreads();
 

@@ -1,0 +1,35 @@
+"""Per-CUDA-line warp-stall samples and executed instructions from an ncu report
+(--page source --print-source cuda,sass): python tools/ncu_source.py rep [top]"""
+import csv
+import io
+import subprocess
+import sys
+
+rep = sys.argv[1]
+top = int(sys.argv[2]) if len(sys.argv) > 2 else 25
+out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+                     capture_output=True, text=True).stdout
+rows = list(csv.reader(io.StringIO(out)))
+agg, src, fname = {}, {}, None
+hdr = None
+for r in rows:
+    if len(r) == 2 and r[0] == "File Path":
+        fname = r[1].split("/")[-1]
+        continue
+    if r and r[0] == "Line No":
+        hdr = r
+        continue
+    if hdr is None or len(r) != len(hdr) or not r[0].strip():
+        continue
+    key = (fname, int(r[0]))
+    src[key] = r[1]
+    s = float(r[4] or 0)
+    ins = float(r[7] or 0)
+    a = agg.setdefault(key, [0.0, 0.0])
+    a[0] += s
+    a[1] += ins
+tot_s = sum(v[0] for v in agg.values()) or 1
+tot_i = sum(v[1] for v in agg.values()) or 1
+print(f"total stall samples {tot_s:.0f}, warp instructions {tot_i:.3g}")
+for k, v in sorted(agg.items(), key=lambda kv: -kv[1][0])[:top]:
+    print(f"{k[0]:>16}:{k[1]:<5d} stall {100*v[0]/tot_s:5.1f}%  inst {100*v[1]/tot_i:5.1f}%  {src[k].strip()[:80]}")
