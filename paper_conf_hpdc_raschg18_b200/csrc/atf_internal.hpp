@@ -51,6 +51,7 @@ struct LevelArgs {
   uint64_t n_parents;
   // candidates = materialised range of the level's parameter
   const int32_t* cand;
+  const uint32_t* cand_magic;  // ceil(2^32/|x|) per candidate (0 for |x| <= 1), host-computed
   int32_t r;
   int32_t level;
   int32_t field_word, field_shift;  // where the child's range position goes
@@ -127,11 +128,12 @@ ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
   const int nc = wide ? a.chunk : a.r;  // candidate table entries
   int o = 0;
   L.ctl = o; o += 64;
-  L.ok = o; o = align16(o + 4 * tn);
-  L.rec = o; o = align16(o + 4 * words * tn);
-  L.opa = o; o = align16(o + 8 * a.n_terms * tn);
-  L.opb = o; o = align16(o + 8 * a.n_terms * tn);
-  if (a.need_slots_smem) { L.slots = o; o = align16(o + 8 * a.n_slots * tn); } else { L.slots = -1; }
+  const int cols = wide ? tn : a.block;  // narrow: one operand column per thread, reused
+  L.ok = o; o = align16(o + 4 * cols);
+  L.rec = o; o = align16(o + 4 * words * cols);
+  L.opa = o; o = align16(o + 8 * a.n_terms * cols);
+  L.opb = o; o = align16(o + 8 * a.n_terms * cols);
+  if (a.need_slots_smem) { L.slots = o; o = align16(o + 8 * a.n_slots * cols); } else { L.slots = -1; }
   if (wide) {
     L.hot = o; o = align16(o + 4 * tn);
     L.hot2 = o; o = align16(o + 4 * tn);
@@ -143,8 +145,12 @@ ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
   } else {
     L.hot = L.hot2 = L.cnt = L.off = L.sum = L.bm = L.q = -1;
   }
-  L.cx = o; o = align16(o + 4 * (nc > 0 ? nc : 1));
-  L.cm = o; o = align16(o + 4 * (nc > 0 ? nc : 1));
+  if (!wide) {  // the wide kernel reads candidates and magics from global (L1)
+    L.cx = o; o = align16(o + 4 * (nc > 0 ? nc : 1));
+    L.cm = o; o = align16(o + 4 * (nc > 0 ? nc : 1));
+  } else {
+    L.cx = L.cm = -1;
+  }
   if (a.qmax > 0) { L.qtab = o; o = align16(o + 4 * ((int)a.qmax + 1)); } else { L.qtab = -1; }
   L.wtot = o; o = align16(o + 8 * 34);
   L.total = o;

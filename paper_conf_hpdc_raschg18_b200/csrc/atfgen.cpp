@@ -711,7 +711,7 @@ static void choose_geometry(LevelArgs& a, int words) {
     a.kind = K_NARROW;
     a.block = 256;
     a.cpt = 1;
-    a.tile_nodes = 256;
+    a.tile_nodes = 256 * 4;  // kNarrowNPT nodes per thread
     a.chunk = r;
   } else {
     a.kind = K_WIDE;
@@ -720,23 +720,27 @@ static void choose_geometry(LevelArgs& a, int words) {
       if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) { a.hot = HOT_DIVX; a.hot_term = t; break; }
       if (T.kind == T_MULX && T.variant == V16) { a.hot = HOT_MULX; a.hot_term = t; break; }
     }
+    // cost per useful pair ~ (1.6 instructions + queue/loop overhead per node quad) x
+    // padding waste; blocks under 256 threads lose latency hiding at the tile barriers
     double best = 1e30;
     for (int cpt : {4, 8, 16}) {
       int64_t per = ((int64_t)r + cpt - 1) / cpt;
-      int B = (int)std::min<int64_t>(512, (per + 31) / 32 * 32);
+      int B = (int)std::min<int64_t>(256, (per + 31) / 32 * 32);
       int64_t nch = ((int64_t)r + (int64_t)B * cpt - 1) / ((int64_t)B * cpt);
-      double cost = (2.0 + 6.0 / (4.0 * cpt)) * (double)((int64_t)B * cpt * nch) / r;
+      double cost = (1.6 + 6.0 / (4.0 * cpt)) * (double)((int64_t)B * cpt * nch) / r;
+      if (B < 256) cost *= 1.1;
       if (cost < best - 1e-9) { best = cost; a.cpt = cpt; a.block = B; a.n_chunks = nch; }
     }
     a.chunk = a.block * a.cpt;
     a.rw = a.chunk / 32;
     a.sw = (a.rw + 31) / 32;
+    // the slow-path queue holds one entry per (node quad, thread): it cannot overflow
     int nt = a.n_chunks > 1 ? 4 : std::max(4, std::min(256, ((1 << 18) / a.chunk + 3) / 4 * 4));
     for (;;) {
       a.tile_nodes = nt;
-      a.qcap = std::min(4096, nt / 4 * a.block);
-      if (nt <= 4 || expand_layout(a, words).total <= 72 * 1024) break;
-      nt = std::max(4, (nt / 2 + 3) / 4 * 4);
+      a.qcap = nt / 4 * a.block;
+      if (nt <= 4 || expand_layout(a, words).total <= 48 * 1024) break;
+      nt -= 4;
     }
   }
   a.smem_bytes = expand_layout(a, words).total;
@@ -749,12 +753,23 @@ static atf_status ensure_device(atf_space* s) {
   size_t np = s->params.size();
   s->d_range.assign(np, nullptr);
   for (size_t p = 0; p < np; p++) {
+    // [values r][divisibility magics r]: magic(x) = ceil(2^32/|x|) mod 2^32 (0 for |x| == 1);
+    // magic(0) = 2^16, which no 16-bit x != 0 has, so that the wide kernel's uniform test
+    // (n * magic mod 2^32) < 2^16 never accepts x == 0 for n != 0
     auto& v = s->params[p].values;
-    s->d_range[p] = (int32_t*)dalloc(s, std::max<size_t>(4, v.size() * 4));
+    s->d_range[p] = (int32_t*)dalloc(s, std::max<size_t>(8, v.size() * 8));
     if (!s->d_range[p]) return fail(s, ATF_ERR_OOM, "range upload");
-    if (!v.empty())
-      CUDA_TRY(s, cudaMemcpyAsync(s->d_range[p], v.data(), v.size() * 4, cudaMemcpyHostToDevice,
+    if (!v.empty()) {
+      std::vector<int32_t> buf(v.begin(), v.end());
+      buf.resize(2 * v.size());
+      for (size_t j = 0; j < v.size(); j++) {
+        uint32_t ax = v[j] < 0 ? 0u - (uint32_t)v[j] : (uint32_t)v[j];
+        buf[v.size() + j] = (int32_t)(ax ? 0xffffffffu / ax + 1u : 0x10000u);
+      }
+      // pageable source: the call returns once `buf` has been staged
+      CUDA_TRY(s, cudaMemcpyAsync(s->d_range[p], buf.data(), buf.size() * 4, cudaMemcpyHostToDevice,
                                   (cudaStream_t)s->opts.stream));
+    }
   }
   s->d_counter = (unsigned int*)dalloc(s, 4 * kMaxGroups);
   s->d_totals = (unsigned long long*)dalloc(s, 8 * kMaxGroups);
@@ -817,7 +832,7 @@ static void release_device(atf_space* s) {
   for (size_t g = 0; g < s->arena.size(); g++)
     for (auto& c : s->arena[g]) dfree(s, c.p, c.size);
   s->arena.clear();
-  for (size_t p = 0; p < s->d_range.size(); p++) dfree(s, s->d_range[p], 4 * s->params[p].values.size());
+  for (size_t p = 0; p < s->d_range.size(); p++) dfree(s, s->d_range[p], 8 * s->params[p].values.size());
   s->d_range.clear();
   dfree(s, s->d_status, s->status_cap * 8);
   dfree(s, s->d_counter, 4 * kMaxGroups);
@@ -863,6 +878,7 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   a.parent_rec = parents;
   a.n_parents = n_parents;
   a.cand = s->d_range[lp.param];
+  a.cand_magic = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + lp.r;  // see ensure_device
   a.r = lp.r;
   for (int i = 0; i < a.n_pv; i++) a.pv_range[i] = s->d_range[lp.pv_param[i]];
   choose_geometry(a, gp.words);

@@ -13,6 +13,47 @@ namespace atf {
 
 #define FULL 0xffffffffu
 
+// ---------------------------------------------------------------- division helpers
+// 64-bit '/' and '%' compile to a called subroutine on sm_100a, and a call in a kernel
+// caps its register allocation.  Operands that fit 32 bits (every C1-C5 value) take the
+// inlined 32-bit path; wider ones a restoring long division (rare, call-free).
+__device__ __forceinline__ uint64_t udivmod64_slow(uint64_t n, uint64_t d, uint64_t* rem) {
+  uint64_t q = 0, r = 0;
+  for (int i = 63; i >= 0; i--) {
+    const bool carry = (r >> 63) != 0;
+    r = (r << 1) | ((n >> i) & 1ull);
+    if (carry || r >= d) {
+      r -= d;
+      q |= 1ull << i;
+    }
+  }
+  *rem = r;
+  return q;
+}
+__device__ __forceinline__ uint64_t udiv64f(uint64_t a, uint64_t b) {
+  if (((a | b) >> 32) == 0) return (uint64_t)((uint32_t)a / (uint32_t)b);
+  uint64_t r;
+  return udivmod64_slow(a, b, &r);
+}
+__device__ __forceinline__ uint64_t umod64f(uint64_t a, uint64_t b) {
+  if (((a | b) >> 32) == 0) return (uint64_t)((uint32_t)a % (uint32_t)b);
+  uint64_t r;
+  udivmod64_slow(a, b, &r);
+  return r;
+}
+// signed, C truncation (quotient toward zero, remainder has the sign of a); b != 0 and
+// not (a == INT64_MIN && b == -1) (the interpreter handles b == -1 before calling)
+__device__ __forceinline__ int64_t sdiv64f(int64_t a, int64_t b) {
+  const uint64_t ua = a < 0 ? 0ull - (uint64_t)a : (uint64_t)a, ub = b < 0 ? 0ull - (uint64_t)b : (uint64_t)b;
+  const uint64_t q = udiv64f(ua, ub);
+  return ((a < 0) != (b < 0)) ? (int64_t)(0ull - q) : (int64_t)q;
+}
+__device__ __forceinline__ int64_t smod64f(int64_t a, int64_t b) {
+  const uint64_t ua = a < 0 ? 0ull - (uint64_t)a : (uint64_t)a, ub = b < 0 ? 0ull - (uint64_t)b : (uint64_t)b;
+  const uint64_t r = umod64f(ua, ub);
+  return a < 0 ? (int64_t)(0ull - r) : (int64_t)r;
+}
+
 // ---------------------------------------------------------------- generic interpreter
 // Semantics of SURVEY.md §8(b) (same as the C ABI doc in include/atfgen.h); int64
 // stack, poison on a zero divisor; strict evaluation.
@@ -37,8 +78,8 @@ __device__ __forceinline__ int64_t run_code(const int32_t* code, int len, int64_
       case 4: r = (int64_t)((uint64_t)a + (uint64_t)b); break;
       case 5: r = (int64_t)((uint64_t)a - (uint64_t)b); break;
       case 6: r = (int64_t)((uint64_t)a * (uint64_t)b); break;
-      case 7: if (b == 0) { poison = true; r = 0; } else if (b == -1) { r = (int64_t)(0ull - (uint64_t)a); } else { r = a / b; } break;
-      case 8: if (b == 0) { poison = true; r = 0; } else if (b == -1) { r = 0; } else { r = a % b; } break;
+      case 7: if (b == 0) { poison = true; r = 0; } else if (b == -1) { r = (int64_t)(0ull - (uint64_t)a); } else { r = sdiv64f(a, b); } break;
+      case 8: if (b == 0) { poison = true; r = 0; } else if (b == -1) { r = 0; } else { r = smod64f(a, b); } break;
       case 9: r = a < b ? a : b; break;
       case 10: r = a > b ? a : b; break;
       case 11: r = (a == b); break;
@@ -47,8 +88,8 @@ __device__ __forceinline__ int64_t run_code(const int32_t* code, int len, int64_
       case 14: r = (a <= b); break;
       case 15: r = (a > b); break;
       case 16: r = (a >= b); break;
-      case 17: if (a == 0) { poison = true; r = 0; } else if (a == -1) { r = 1; } else { r = (b % a == 0); } break;
-      case 18: if (b == 0) { poison = true; r = 0; } else if (b == -1) { r = 1; } else { r = (a % b == 0); } break;
+      case 17: if (a == 0) { poison = true; r = 0; } else if (a == -1) { r = 1; } else { r = (smod64f(b, a) == 0); } break;
+      case 18: if (b == 0) { poison = true; r = 0; } else if (b == -1) { r = 1; } else { r = (smod64f(a, b) == 0); } break;
       case 19: r = (a != 0) & (b != 0); break;
       case 20: r = (a != 0) | (b != 0); break;
       default: poison = true; break;

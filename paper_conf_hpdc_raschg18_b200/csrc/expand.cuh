@@ -20,16 +20,16 @@ __device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, 
       const uint64_t n = (uint64_t)A;
       if (T.variant == V16) return (uint32_t)n * m32 <= m32 - 1u;
       if (T.variant == V32) {
-        const uint64_t m64 = ~0ull / ax + 1ull;
+        const uint64_t m64 = udiv64f(~0ull, ax) + 1ull;
         return n * m64 <= m64 - 1ull;
       }
-      return n % ax == 0;
+      return umod64f(n, ax) == 0;
     }
     case T_MULX: {  // d | x  (d = A != 0 checked by the node gate, Bv = magic(d))
       const uint64_t d = (uint64_t)A, md = (uint64_t)Bv;
       if (T.variant == V16) return ax * (uint32_t)md <= (uint32_t)md - 1u;
       if (T.variant == V32) return (uint64_t)ax * md <= md - 1ull;
-      return d != 0 && (uint64_t)ax % d == 0;
+      return d != 0 && umod64f(ax, d) == 0;
     }
     case T_QDIV: {  // (num / x) | nb; x == 0 or quotient 0 -> poison -> reject
       if (ax == 0) return false;
@@ -43,8 +43,8 @@ __device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, 
         }
         return (uint32_t)nb % q == 0;
       }
-      const uint64_t q = num / ax;
-      return q != 0 && nb % q == 0;
+      const uint64_t q = udiv64f(num, ax);
+      return q != 0 && umod64f(nb, q) == 0;
     }
     case T_CMP:
       if (T.variant == V32) return rel_holds32(T.rel, (int32_t)A * x, (int32_t)Bv);
@@ -55,12 +55,6 @@ __device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, 
       return !poison && v != 0;
     }
   }
-}
-
-// Candidate-table entries: value and 32-bit divisibility magic.
-__device__ __forceinline__ uint32_t cand_magic(int32_t x) {
-  const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-  return ax ? 0xffffffffu / ax + 1u : 0u;
 }
 
 // Exact acceptance of candidate (x, m32) by node i of the tile (all conjuncts, node gate).
@@ -111,7 +105,7 @@ __device__ __forceinline__ void load_record(const uint32_t* src, uint32_t* rec) 
 // hoisted node-invariant expressions, the node gates and every conjunct's operands into
 // shared memory (node `i` of the tile, global index gnode).  Returns the gate result.
 template <int W>
-__device__ __noinline__ bool prologue_node(const LevelArgs& a, uint64_t gnode, int i, int tn, uint32_t* s_ok, uint32_t* s_rec,
+__device__ __forceinline__ bool prologue_node_impl(const LevelArgs& a, uint64_t gnode, int i, int tn, uint32_t* s_ok, uint32_t* s_rec,
                               int64_t* s_opa, int64_t* s_opb, int64_t* s_slots) {
   uint32_t rec[W];
   if (a.level == 0) {
@@ -148,14 +142,14 @@ __device__ __noinline__ bool prologue_node(const LevelArgs& a, uint64_t gnode, i
         if (d == 0) ok = false;
         A = (int64_t)d;
         if (T.variant == V16) B = d ? (int64_t)(0xffffffffu / (uint32_t)d + 1u) : 0;
-        else if (T.variant == V32) B = d ? (int64_t)(~0ull / d + 1ull) : 0;
+        else if (T.variant == V32) B = d ? (int64_t)(udiv64f(~0ull, d) + 1ull) : 0;
         break;
       }
       case T_DIVPROD: {
         const uint64_t av = uabs64(slots[T.slot_a]), bv = uabs64(slots[T.slot_b]);
         if (av == 0) { ok = false; A = 0; }
-        else if (bv % av != 0) { ok = false; A = 0; }
-        else A = (int64_t)(bv / av);
+        else if (umod64f(bv, av) != 0) { ok = false; A = 0; }
+        else A = (int64_t)udiv64f(bv, av);
         break;
       }
       case T_QDIV: A = (int64_t)uabs64(slots[T.slot_a]); B = (int64_t)uabs64(slots[T.slot_b]); break;
@@ -168,6 +162,13 @@ __device__ __noinline__ bool prologue_node(const LevelArgs& a, uint64_t gnode, i
     for (int s = 0; s < a.n_slots; s++) s_slots[s * tn + i] = slots[s];
   s_ok[i] = ok ? 1u : 0u;
   return ok;
+}
+
+// Out-of-line copy for the wide kernel (keeps the hot loop's registers free).
+template <int W>
+__device__ __noinline__ bool prologue_node(const LevelArgs& a, uint64_t gnode, int i, int tn, uint32_t* s_ok,
+                                           uint32_t* s_rec, int64_t* s_opa, int64_t* s_opb, int64_t* s_slots) {
+  return prologue_node_impl<W>(a, gnode, i, tn, s_ok, s_rec, s_opa, s_opb, s_slots);
 }
 
 // Block-wide exclusive scan of one u32 per thread (B <= 1024); returns the exclusive
@@ -199,10 +200,15 @@ __device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* total,
 }
 
 // ---------------------------------------------------------------- narrow expand kernel
-// One launch = one tree level of one group, for ranges of r <= 64 candidates.  One
-// thread per frontier node (tile = blockDim.x nodes): prologue -> exact evaluation of the
-// r candidates into a 64-bit accept mask (count, A4) -> block scan + decoupled look-back
-// (A5) -> CSR + the node's children records in candidate order (emit, A6).
+// One launch = one tree level of one group, for ranges of r <= 64 candidates.  Tile =
+// blockDim.x * NPT frontier nodes; thread t owns the NPT consecutive nodes
+// [t*NPT, t*NPT + NPT) of the tile (thread order = node order).  Per node: prologue ->
+// exact term-major evaluation of the r candidates into a 64-bit accept mask (count, A4);
+// per tile: block scan of the per-thread child counts + decoupled look-back (A5); then
+// every thread writes its nodes' CSR entries and children records in candidate order
+// (emit, A6).  The prologue's operand columns are per thread and reused node by node.
+constexpr int kNarrowNPT = 4;
+
 template <int W>
 __global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ LevelArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -219,14 +225,14 @@ __global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ Lev
   unsigned long long* s_w = reinterpret_cast<unsigned long long*>(smem + L.wtot);
 
   const int tid = threadIdx.x, lane = tid & 31, B = blockDim.x;
-  const int r = a.r, tn_max = a.tile_nodes;
+  const int r = a.r, tn_max = a.tile_nodes;  // = B * kNarrowNPT
   for (int j = tid; j < r; j += B) {
-    const int32_t x = __ldg(a.cand + j);
-    s_cx[j] = x;
-    s_cm[j] = cand_magic(x);
+    s_cx[j] = __ldg(a.cand + j);
+    s_cm[j] = __ldg(a.cand_magic + j);
   }
   if (s_q)
     for (uint32_t q = tid; q <= a.qmax; q += B) s_q[q] = q ? (0xffffffffu / q + 1u) : 0u;
+  const uint64_t full = r >= 64 ? ~0ull : ((1ull << r) - 1ull);
 
   for (;;) {
     if (tid == 0) ctl[0] = atomicAdd(a.tile_counter, 1u);
@@ -236,26 +242,39 @@ __global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ Lev
     const uint64_t node0 = tile * (uint64_t)tn_max;
     const uint64_t rem = a.n_parents - node0;
     const int tn = rem < (uint64_t)tn_max ? (int)rem : tn_max;
-    const int i = tid;
-    uint64_t mask = 0;
-    if (i < tn && prologue_node<W>(a, node0 + i, i, tn_max, s_ok, s_rec, s_opa, s_opb, s_slots)) {
-      mask = r >= 64 ? ~0ull : ((1ull << r) - 1ull);
-      for (int t = 0; t < a.n_terms && mask; t++) {
-        const Term& T = a.terms[t];
-        const int64_t A = s_opa[t * tn_max + i], Bv = s_opb[t * tn_max + i];
-        uint64_t mt = 0;
-        for (int c = 0; c < r; c++) {
-          if (!((mask >> c) & 1ull)) continue;
-          const int32_t x = s_cx[c];
-          const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-          if (term_accepts(a, T, A, Bv, x, ax, s_cm[c], s_q, s_slots ? s_slots + i : nullptr, tn_max))
-            mt |= 1ull << c;
+    uint64_t mask[kNarrowNPT];
+    uint32_t rec[kNarrowNPT][W];
+    uint32_t cnt = 0;
+#pragma unroll
+    for (int k = 0; k < kNarrowNPT; k++) {
+      const int i = tid * kNarrowNPT + k;
+      mask[k] = 0;
+      // the operand column of this thread (index tid) is reused for each of its nodes
+      if (i < tn && prologue_node_impl<W>(a, node0 + i, tid, B, s_ok, s_rec, s_opa, s_opb, s_slots)) {
+        uint64_t m = full;
+        for (int t = 0; t < a.n_terms && m; t++) {
+          const Term& T = a.terms[t];
+          const int64_t A = s_opa[t * B + tid], Bv = s_opb[t * B + tid];
+          uint64_t mt = 0;
+          for (int c = 0; c < r; c++) {
+            if (!((m >> c) & 1ull)) continue;
+            const int32_t x = s_cx[c];
+            const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+            if (term_accepts(a, T, A, Bv, x, ax, s_cm[c], s_q, s_slots ? s_slots + tid : nullptr, B))
+              mt |= 1ull << c;
+          }
+          m &= mt;
         }
-        mask &= mt;
+        mask[k] = m;
       }
+      if (i < tn) {
+#pragma unroll
+        for (int w = 0; w < W; w++) rec[k][w] = s_rec[tid * W + w];
+      }
+      cnt += (uint32_t)__popcll(mask[k]);
     }
     uint32_t total;
-    const uint32_t excl = block_excl_scan((uint32_t)__popcll(mask), &total, s_w);
+    const uint32_t excl = block_excl_scan(cnt, &total, s_w);
     if (tid < 32) {
       const unsigned long long base = lookback(a.status, tile, total, lane);
       if (lane == 0) {
@@ -267,21 +286,20 @@ __global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ Lev
       }
     }
     __syncthreads();
-    const uint64_t base = s_w[33];
-    if (i < tn) {
-      uint64_t rank = base + excl;
-      a.csr[node0 + i] = rank;
-      uint32_t rec[W];
+    uint64_t rank = s_w[33] + excl;
 #pragma unroll
-      for (int w = 0; w < W; w++) rec[w] = s_rec[i * W + w];
-      uint64_t m = mask;
+    for (int k = 0; k < kNarrowNPT; k++) {
+      const int i = tid * kNarrowNPT + k;
+      if (i >= tn) break;
+      a.csr[node0 + i] = rank;
+      uint64_t m = mask[k];
       while (m) {
         const int c = __ffsll((long long)m) - 1;
         m &= m - 1;
         if (rank < a.child_cap) {
           uint32_t out[W];
 #pragma unroll
-          for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? (uint32_t)c << a.field_shift : 0u);
+          for (int w = 0; w < W; w++) out[w] = rec[k][w] | (w == a.field_word ? (uint32_t)c << a.field_shift : 0u);
           store_record<W>(a.child_rec + rank * W, out);
         } else {
           atomicOr(a.overflow_flag, 1u);
@@ -294,11 +312,11 @@ __global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ Lev
 }
 
 // Conjuncts other than the hot one, for the candidates still set in `mask` (bit c =
-// candidate jl0 + c of the chunk).  Out of line: only reached on hot-filter survivors.
-static __device__ __noinline__ uint32_t other_terms_mask(const LevelArgs& a, int i, int tn, int jl0, uint32_t mask,
-                                                        int skip, const int64_t* s_opa, const int64_t* s_opb,
-                                                        const int64_t* s_slots, const uint32_t* s_q,
-                                                        const int32_t* s_cx, const uint32_t* s_cm) {
+// candidate jg0 + c of the range).  Out of line: only reached on hot-filter survivors.
+static __device__ __noinline__ uint32_t other_terms_mask(const LevelArgs& a, int i, int tn, int64_t jg0,
+                                                        uint32_t mask, int skip, const int64_t* s_opa,
+                                                        const int64_t* s_opb, const int64_t* s_slots,
+                                                        const uint32_t* s_q) {
   for (int t = 0; t < a.n_terms && mask; t++) {
     if (t == skip) continue;
     const Term& T = a.terms[t];
@@ -307,48 +325,52 @@ static __device__ __noinline__ uint32_t other_terms_mask(const LevelArgs& a, int
     while (m) {
       const int c = __ffs(m) - 1;
       m &= m - 1;
-      const int32_t x = s_cx[jl0 + c];
+      const int32_t x = __ldg(a.cand + jg0 + c);
       const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-      if (!term_accepts(a, T, A, Bv, x, ax, s_cm[jl0 + c], s_q, s_slots ? s_slots + i : nullptr, tn))
+      if (!term_accepts(a, T, A, Bv, x, ax, __ldg(a.cand_magic + jg0 + c), s_q, s_slots ? s_slots + i : nullptr, tn))
         mask &= ~(1u << c);
     }
   }
   return mask;
 }
 
-// Exact accept mask of node i over candidates [jl0, jl0 + CPT) of the chunk, recorded in
-// the node's bitmap, summary and count (shared-memory atomics, once per call).
+// Exact accept mask of node i over chunk candidates [jl0, jl0 + CPT), recorded in the
+// node's bitmap, summary and count (shared-memory atomics, once per call).
 template <int CPT, int HOT>
 __device__ __forceinline__ void record_mask(const LevelArgs& a, int i, int tn, int jl0, int64_t j0,
                                             const uint32_t* s_ok, const uint32_t* s_hot, const uint32_t* s_hot2,
                                             const int64_t* s_opa, const int64_t* s_opb, const int64_t* s_slots,
-                                            const uint32_t* s_q, const int32_t* s_cx, const uint32_t* s_cm,
-                                            uint32_t* s_bm, uint32_t* s_sum, uint32_t* s_cnt, int RW, int SW) {
+                                            const uint32_t* s_q, uint32_t* s_bm, uint32_t* s_sum, uint32_t* s_cnt,
+                                            int RW, int SW) {
   if (!s_ok[i]) return;
+  const int64_t jg0 = j0 + jl0;
   uint32_t mask = 0;
   if (HOT == HOT_NONE) {
 #pragma unroll
     for (int c = 0; c < CPT; c++)
-      if (j0 + jl0 + c < a.r &&
-          node_accepts(a, i, tn, s_cx[jl0 + c], s_cm[jl0 + c], s_ok, s_opa, s_opb, s_slots, s_q))
+      if (jg0 + c < a.r &&
+          node_accepts(a, i, tn, __ldg(a.cand + jg0 + c), __ldg(a.cand_magic + jg0 + c), s_ok, s_opa, s_opb,
+                       s_slots, s_q))
         mask |= 1u << c;
   } else {
     const uint32_t n = s_hot[i], d1 = s_hot2[i];
 #pragma unroll
     for (int c = 0; c < CPT; c++) {
-      const int32_t x = s_cx[jl0 + c];
-      const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-      bool ok = j0 + jl0 + c < a.r;
-      if (HOT == HOT_DIVX) {
-        const uint32_t m = s_cm[jl0 + c];
-        ok = ok && ax != 0 && n * m <= m - 1u;  // exact for 16-bit operands (V16)
-      } else {
-        ok = ok && ax * n <= d1;  // n = ceil(2^32/d), d1 = n - 1
+      if (jg0 + c < a.r) {
+        bool ok;
+        if (HOT == HOT_DIVX) {
+          // exact for 16-bit operands; magic(0) = 2^16 excludes x == 0 (host table)
+          const uint32_t m = __ldg(a.cand_magic + jg0 + c);
+          ok = n * m < 0x10000u && m != 0x10000u;
+        } else {
+          const int32_t x = __ldg(a.cand + jg0 + c);
+          const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+          ok = ax * n <= d1;  // n = ceil(2^32/d), d1 = n - 1
+        }
+        mask |= (uint32_t)ok << c;
       }
-      mask |= (uint32_t)ok << c;
     }
-    if (mask && a.n_terms > 1)
-      mask = other_terms_mask(a, i, tn, jl0, mask, a.hot_term, s_opa, s_opb, s_slots, s_q, s_cx, s_cm);
+    if (mask && a.n_terms > 1) mask = other_terms_mask(a, i, tn, jg0, mask, a.hot_term, s_opa, s_opb, s_slots, s_q);
   }
   if (mask) {
     atomicOr(&s_bm[i * RW + (jl0 >> 5)], mask << (jl0 & 31));
@@ -357,23 +379,55 @@ __device__ __forceinline__ void record_mask(const LevelArgs& a, int i, int tn, i
   }
 }
 
+// Children of node i with a large count, emitted by the whole warp: set bitmap words in
+// order, lane b writes the child of bit b (coalesced); consumed words are zeroed.
+template <int W>
+__device__ __forceinline__ void emit_node_warp(const LevelArgs& a, int i, uint64_t rank, int64_t j0, const uint32_t* rec,
+                                               uint32_t* s_bm, uint32_t* s_sum, int RW, int SW, int lane) {
+  const unsigned lt = (1u << lane) - 1u;
+  for (int sw = 0; sw < SW; sw++) {
+    uint32_t sm = s_sum[i * SW + sw];
+    while (sm) {
+      const int wi = sw * 32 + __ffs(sm) - 1;
+      sm &= sm - 1;
+      const uint32_t word = s_bm[i * RW + wi];
+      if ((word >> lane) & 1u) {
+        const uint64_t rk = rank + __popc(word & lt);
+        if (rk < a.child_cap) {
+          const uint32_t pos = (uint32_t)(j0 + wi * 32 + lane);
+          uint32_t out[W];
+#pragma unroll
+          for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? pos << a.field_shift : 0u);
+          store_record<W>(a.child_rec + rk * W, out);
+        } else {
+          atomicOr(a.overflow_flag, 1u);
+        }
+      }
+      rank += __popc(word);
+      __syncwarp();
+      if (lane == 0) s_bm[i * RW + wi] = 0u;
+    }
+    __syncwarp();
+    if (lane == 0) s_sum[i * SW + sw] = 0u;
+  }
+}
+
 // ---------------------------------------------------------------- wide expand kernel
 // One launch = one tree level of one group, for ranges of r > 64 candidates.  Tile =
 // tile_nodes frontier nodes x one chunk of `chunk` candidates; thread t owns candidate
-// positions [t*CPT, t*CPT + CPT) of the chunk for the whole launch (values/magics in
-// registers).  Per tile:
+// positions [t*CPT, t*CPT + CPT) of the chunk.  Per tile:
 //   prologue  one thread per node: path record -> ancestor values -> operands (smem)
-//   hot loop  (A4) every (node, candidate) pair through the HOT filter: IMAD + ISETP.OR,
-//             a superset of the accepted pairs; a thread whose CPT candidates pass for any
-//             of 4 consecutive nodes queues (node quad, thread) in shared memory
-//   slow path the queued pairs are re-evaluated exactly (all conjuncts), flattened over
-//             the block; accepted pairs set bits of a per-node candidate bitmap (smem)
-//             and bump the node's count.  Queue overflow -> the tile is evaluated densely.
-//   scan      (A5) block scan of node counts + decoupled look-back -> CSR offsets
-//   emit      (A6) per node, set bitmap words in order: lane b writes the child of bit b
-//             (coalesced), records = parent record | position; consumed words are zeroed.
+//   hot loop  (A4) every (node, candidate) pair through the HOT filter (one IMAD + half a
+//             VIMNMX3 per pair, min over the thread's candidates per node); a thread whose
+//             candidates may pass for any of 4 consecutive nodes queues (node quad, thread)
+//   slow path the queued pairs are evaluated exactly, one item = node x CPT candidates,
+//             flattened over the block; accepted pairs set bits of a per-node candidate
+//             bitmap (smem) and bump the node's count.  Queue overflow -> dense tile.
+//   scan      (A5) warp scan of node counts + decoupled look-back -> CSR offsets
+//   emit      (A6) lane-per-node for nodes with few children, warp-per-node (coalesced)
+//             for many; records = parent record | position; consumed words are zeroed.
 template <int W, int CPT, int HOT>
-__global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ LevelArgs a) {
+__global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ LevelArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   const SmemLayout L = expand_layout(a, W);
   uint32_t* ctl = reinterpret_cast<uint32_t*>(smem + L.ctl);
@@ -389,8 +443,6 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
   uint32_t* s_sum = reinterpret_cast<uint32_t*>(smem + L.sum);
   uint32_t* s_bm = reinterpret_cast<uint32_t*>(smem + L.bm);
   uint32_t* s_qe = reinterpret_cast<uint32_t*>(smem + L.q);
-  int32_t* s_cx = reinterpret_cast<int32_t*>(smem + L.cx);
-  uint32_t* s_cm = reinterpret_cast<uint32_t*>(smem + L.cm);
   uint32_t* s_q = L.qtab >= 0 ? reinterpret_cast<uint32_t*>(smem + L.qtab) : nullptr;
   unsigned long long* s_w = reinterpret_cast<unsigned long long*>(smem + L.wtot);
 
@@ -398,24 +450,13 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
   const int B = blockDim.x, NW = B >> 5;
   const int r = a.r, NT = a.tile_nodes, RW = a.rw, SW = a.sw, chunk = a.chunk;
   const int hot_t = a.hot_term;
+  constexpr uint32_t kBig = 48;  // children above which a node is emitted by the whole warp
 
   for (int k = tid; k < NT * RW; k += B) s_bm[k] = 0u;
   for (int k = tid; k < NT * SW; k += B) s_sum[k] = 0u;
   for (int k = tid; k < NT; k += B) s_cnt[k] = 0u;
   if (s_q)
     for (uint32_t q = tid; q <= a.qmax; q += B) s_q[q] = q ? (0xffffffffu / q + 1u) : 0u;
-
-  // candidate table of the current chunk: value and 32-bit divisibility magic
-  auto load_chunk = [&](int64_t ch) {
-    const int64_t j0 = ch * (int64_t)chunk;
-    for (int k = tid; k < chunk; k += B) {
-      const int64_t j = j0 + k;
-      const int32_t x = j < r ? __ldg(a.cand + j) : 0;
-      s_cx[k] = x;
-      s_cm[k] = cand_magic(x);
-    }
-  };
-  if (a.n_chunks == 1) load_chunk(0);
 
   for (;;) {
     if (tid == 0) {
@@ -433,10 +474,9 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
       const uint64_t rem = a.n_parents - node0;
       tn = rem < (uint64_t)NT ? (int)rem : NT;
     } else {
-      node0 = tile / (uint64_t)a.n_chunks;
-      ch = (int64_t)(tile % (uint64_t)a.n_chunks);
+      node0 = udiv64f(tile, (uint64_t)a.n_chunks);
+      ch = (int64_t)umod64f(tile, (uint64_t)a.n_chunks);
       tn = 1;
-      load_chunk(ch);
     }
     const int64_t j0 = ch * (int64_t)chunk;
     // ---- prologue
@@ -459,9 +499,8 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
     __syncthreads();
 
     // ---- hot loop (A4): superset filter, queue (node quad, thread) on a possible accept
-    bool dense = HOT == HOT_NONE;
+    const bool dense = HOT == HOT_NONE;
     if (HOT != HOT_NONE) {
-      // registers (reloaded per tile so they are not live across the prologue):
       //   HOT_DIVX: hm = ceil(2^32/|x|).  For 16-bit n and x, (n * hm mod 2^32) < 2^16
       //             iff x | n (exhaustively verified, tests/test_abi_cpu.py), so the
       //             per-node test is min over the candidates < 2^16: one IMAD per pair
@@ -472,11 +511,11 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
       uint32_t hm[CPT];
 #pragma unroll
       for (int c = 0; c < CPT; c++) {
-        const int jl = tid * CPT + c;
-        const bool v = j0 + jl < r;
-        const int32_t x = s_cx[jl];
+        const int64_t j = j0 + tid * CPT + c;
+        const bool v = j < r;
+        const int32_t x = v ? __ldg(a.cand + j) : 0;
         const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-        if (HOT == HOT_DIVX) hm[c] = (v && ax) ? s_cm[jl] : 0x10000u;
+        if (HOT == HOT_DIVX) hm[c] = v ? __ldg(a.cand_magic + j) : 0x10000u;  // magic(0) = 2^16
         else hm[c] = v ? ax : 1u;
       }
       for (int g = 0; g < tn; g += 4) {
@@ -496,35 +535,32 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
           const uint4 d4 = *reinterpret_cast<const uint4*>(s_hot2 + g);
           h0 = m0 <= d4.x; h1 = m1 <= d4.y; h2 = m2 <= d4.z; h3 = m3 <= d4.w;
         }
-        if (h0 | h1 | h2 | h3) {
+        const uint32_t hq = (uint32_t)h0 | ((uint32_t)h1 << 1) | ((uint32_t)h2 << 2) | ((uint32_t)h3 << 3);
+        if (hq) {  // entry: node quad << 16 | flagged nodes << 12 | thread
           const uint32_t slot = atomicAdd(&ctl[1], 1u);
-          if (slot < (uint32_t)a.qcap) s_qe[slot] = ((uint32_t)(g >> 2) << 16) | (uint32_t)tid;
+          s_qe[slot] = ((uint32_t)(g >> 2) << 16) | (hq << 12) | (uint32_t)tid;
         }
       }
       __syncthreads();
-      const uint32_t nq = ctl[1];
-      if (nq > (uint32_t)a.qcap) {
-        dense = true;
-      } else {
-        // ---- slow path: the queued (node, thread) pairs, flattened over the block; each
-        // item = one node x the thread's CPT candidates, exact (hot conjunct inline,
-        // the other conjuncts only for its survivors), one set of smem atomics per item
-        const uint32_t items = nq * 4u;
-        for (uint32_t k = tid; k < items; k += B) {
-          const uint32_t e = s_qe[k >> 2];
-          const int i = (int)((e >> 16) * 4u + (k & 3u));
-          const int jl0 = (int)((e & 0xffffu) * CPT);
-          if (i < tn) record_mask<CPT, HOT>(a, i, NT, jl0, j0, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q, s_cx,
-                                           s_cm, s_bm, s_sum, s_cnt, RW, SW);
-        }
+      // ---- slow path: queued (node, thread) pairs flattened over the block; one item =
+      // one flagged node x the thread's CPT candidates, exact.  (qcap = one entry per
+      // node quad and thread, so the queue cannot overflow.)
+      const uint32_t items = ctl[1] * 4u;
+      for (uint32_t k = tid; k < items; k += B) {
+        const uint32_t e = s_qe[k >> 2];
+        if (!((e >> (12 + (k & 3u))) & 1u)) continue;
+        const int i = (int)((e >> 16) * 4u + (k & 3u));
+        const int jl0 = (int)((e & 0xfffu) * CPT);
+        record_mask<CPT, HOT>(a, i, NT, jl0, j0, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q, s_bm, s_sum,
+                              s_cnt, RW, SW);
       }
     }
     if (dense) {
       // every (node, candidate) pair of the tile exactly; thread-owned candidates
       const int jl0 = tid * CPT;
       for (int i = 0; i < tn; i++)
-        record_mask<CPT, HOT>(a, i, NT, jl0, j0, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q, s_cx, s_cm, s_bm,
-                              s_sum, s_cnt, RW, SW);
+        record_mask<CPT, HOT>(a, i, NT, jl0, j0, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q, s_bm, s_sum,
+                              s_cnt, RW, SW);
     }
     __syncthreads();
 
@@ -558,39 +594,52 @@ __global__ void __launch_bounds__(512) expand_wide(const __grid_constant__ Level
     // ---- emit (A6)
     if (ch == 0)
       for (int i = tid; i < tn; i += B) a.csr[node0 + i] = base + s_off[i];
-    const unsigned lt = (1u << lane) - 1u;
-    for (int i = warp; i < tn; i += NW) {
-      const uint32_t cnt = s_cnt[i];
-      if (cnt == 0) continue;
-      uint64_t rank = base + s_off[i];
-      uint32_t rec[W];
+    for (int i0 = warp * 32; i0 < tn; i0 += NW * 32) {
+      const int i = i0 + lane;
+      const uint32_t cnt = i < tn ? s_cnt[i] : 0u;
+      if (cnt && cnt <= kBig) {
+        // lane per node: its set words in order, its bits in order
+        uint64_t rank = base + s_off[i];
+        uint32_t rec[W];
 #pragma unroll
-      for (int w = 0; w < W; w++) rec[w] = s_rec[i * W + w];
-      for (int sw = 0; sw < SW; sw++) {
-        uint32_t sm = s_sum[i * SW + sw];
-        while (sm) {
-          const int wi = sw * 32 + __ffs(sm) - 1;
-          sm &= sm - 1;
-          const uint32_t word = s_bm[i * RW + wi];
-          if ((word >> lane) & 1u) {
-            const uint64_t rk = rank + __popc(word & lt);
-            if (rk < a.child_cap) {
-              const uint32_t pos = (uint32_t)(j0 + wi * 32 + lane);
-              uint32_t out[W];
+        for (int w = 0; w < W; w++) rec[w] = s_rec[i * W + w];
+        for (int sw = 0; sw < SW; sw++) {
+          uint32_t sm = s_sum[i * SW + sw];
+          if (!sm) continue;
+          s_sum[i * SW + sw] = 0u;
+          while (sm) {
+            const int wi = sw * 32 + __ffs(sm) - 1;
+            sm &= sm - 1;
+            uint32_t word = s_bm[i * RW + wi];
+            s_bm[i * RW + wi] = 0u;
+            while (word) {
+              const int b = __ffs(word) - 1;
+              word &= word - 1;
+              if (rank < a.child_cap) {
+                const uint32_t pos = (uint32_t)(j0 + wi * 32 + b);
+                uint32_t out[W];
 #pragma unroll
-              for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? pos << a.field_shift : 0u);
-              store_record<W>(a.child_rec + rk * W, out);
-            } else {
-              atomicOr(a.overflow_flag, 1u);
+                for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? pos << a.field_shift : 0u);
+                store_record<W>(a.child_rec + rank * W, out);
+              } else {
+                atomicOr(a.overflow_flag, 1u);
+              }
+              rank++;
             }
           }
-          rank += __popc(word);
-          __syncwarp();
-          if (lane == 0) s_bm[i * RW + wi] = 0u;
         }
-        if (lane == 0) s_sum[i * SW + sw] = 0u;
       }
-      if (lane == 0) s_cnt[i] = 0u;
+      unsigned big = __ballot_sync(FULL, cnt > kBig);
+      while (big) {
+        const int src = __ffs(big) - 1;
+        big &= big - 1;
+        const int ib = i0 + src;
+        uint32_t rec[W];
+#pragma unroll
+        for (int w = 0; w < W; w++) rec[w] = s_rec[ib * W + w];
+        emit_node_warp<W>(a, ib, base + s_off[ib], j0, rec, s_bm, s_sum, RW, SW, lane);
+      }
+      if (i < tn) s_cnt[i] = 0u;
     }
     __syncthreads();
   }

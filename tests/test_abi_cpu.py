@@ -151,7 +151,9 @@ def test_static_overflow_rejected():
 
 def test_magic_formulas_exhaustive(tmp_path):
     """The kernel's divisibility / quotient magics (Lemire, Kaser & Kurz 2019) restated in C and
-    checked exhaustively over all 16-bit pairs and on random 32-bit pairs against % and /."""
+    checked exhaustively over all 16-bit pairs and on random 32-bit pairs against % and /.
+    Includes the wide kernel's hot filter: for 16-bit n and d, (n * ceil(2^32/d) mod 2^32) <
+    2^16 iff d | n, which lets the hot loop take a min over candidates against one bound."""
     src = tmp_path / "magic.c"
     src.write_text(r'''
 #include <stdint.h>
@@ -162,8 +164,9 @@ int main(void) {
     uint32_t m = 0xffffffffu / d + 1u;            /* ceil(2^32/d) mod 2^32 */
     for (uint32_t n = 0; n < 65536; n++) {
       int div = (uint32_t)(n * m) <= m - 1u;       /* V16 divisibility test */
+      int hot = (uint32_t)(n * m) < 65536u;         /* wide kernel's HOT_DIVX filter: uniform bound */
       uint32_t q = d == 1 ? n : (uint32_t)(((uint64_t)n * m) >> 32);  /* V16 quotient */
-      bad += (div != (n % d == 0)) + (q != n / d);
+      bad += (div != (n % d == 0)) + (hot != (n % d == 0)) + (q != n / d);
     }
   }
   uint64_t s = 88172645463325252ull;

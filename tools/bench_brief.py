@@ -1,0 +1,12 @@
+"""One-screen summary of a bench.py JSON line: python tools/bench_brief.py file.json"""
+import json
+import sys
+
+d = json.loads(open(sys.argv[1]).read().strip().splitlines()[-1])
+print(f"C5 ms/step {d['ms_per_step']:.2f}  configs/s {d['value']:.3g}  evals/s {d.get('evals_per_s', 0):.3g}  "
+      f"roofline frac {d['roofline']['frac']:.3f}  e2e {d['e2e']['value']:.3g}  clocks {d['clocks']}")
+for k, v in d.get("secondary", {}).items():
+    if "ms_per_step" in v:
+        print(f"{k:8s} ms {v['ms_per_step']:.3f} frac {v['roofline_frac']:.3f} levels {v['level_ms']}")
+    else:
+        print(k, v)
