@@ -78,6 +78,14 @@ struct LevelArgs {
   unsigned long long* total_out;
   uint64_t child_cap;       // capacity of child_rec in records
   unsigned int* overflow_flag;
+  // wide levels: children go to per-tile stash segments first (no cross-tile wait),
+  // then wide_emit_kernel copies them to their final positions
+  uint32_t* stash;          // [stash_cap][W]
+  uint64_t stash_cap;
+  unsigned long long* stash_top;
+  uint32_t* tile_total;     // [n_tiles] children per tile
+  unsigned long long* tile_seg;  // [n_tiles] stash segment (records)
+  const uint64_t* tile_base;     // [n_tiles + 1] exclusive scan of tile_total
   // geometry (host choose_geometry)
   int32_t kind;             // K_NARROW: one thread per frontier node, r <= 64 candidates each
                             // K_WIDE:   each thread owns cpt consecutive candidates of a chunk
@@ -161,6 +169,7 @@ ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
 // All return a cudaError_t value as int (0 = success).
 int launch_expand(const LevelArgs& a, int words, void* stream);
 int expand_smem_bytes(const LevelArgs& a, int words);
+int launch_wide_emit(const LevelArgs& a, int words, void* stream);
 int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out,
                           int64_t ld, unsigned int* bad_flag, void* stream);
 int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,

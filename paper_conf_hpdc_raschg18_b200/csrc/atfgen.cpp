@@ -104,6 +104,11 @@ struct atf_space {
   std::vector<uint64_t> gsize;
   unsigned long long* d_status = nullptr;
   size_t status_cap = 0;
+  uint64_t stash_hint = 0;     // records: exact size of the last level that overflowed
+  char* d_scratch = nullptr;   // wide levels: per-tile totals, segments, bases, scan state
+  size_t scratch_cap = 0;
+  uint32_t* d_stash = nullptr; // wide levels: children in tile segments before the final copy
+  size_t stash_cap = 0;        // bytes
   unsigned int* d_counter = nullptr;     // [kMaxGroups] tile counters
   unsigned long long* d_totals = nullptr;  // [kMaxGroups]
   unsigned int* d_ovf = nullptr;         // [kMaxGroups]
@@ -750,6 +755,16 @@ static void choose_geometry(LevelArgs& a, int words) {
 static atf_status ensure_device(atf_space* s) {
   CUDA_TRY(s, cudaSetDevice(s->opts.device));
   if (s->dev_ready) return ATF_OK;
+  if (!s->opts.alloc) {
+    // cudaMallocAsync path: keep freed blocks in the device's default pool so that a new
+    // space (e.g. one per request) does not re-map its arenas
+    cudaMemPool_t pool;
+    if (cudaDeviceGetDefaultMemPool(&pool, s->opts.device) == cudaSuccess) {
+      uint64_t keep = UINT64_MAX;
+      cudaMemPoolSetAttribute(pool, cudaMemPoolAttrReleaseThreshold, &keep);
+    }
+    cudaGetLastError();
+  }
   size_t np = s->params.size();
   s->d_range.assign(np, nullptr);
   for (size_t p = 0; p < np; p++) {
@@ -795,6 +810,16 @@ static atf_status ensure_status(atf_space* s, size_t tiles) {
   return ATF_OK;
 }
 
+static atf_status ensure_buf(atf_space* s, char** p, size_t* cap, size_t bytes, const char* what) {
+  if (bytes <= *cap) return ATF_OK;
+  dfree(s, *p, *cap);
+  size_t c = std::max<size_t>(bytes, *cap * 2);
+  *p = (char*)dalloc(s, c);
+  if (!*p) { *cap = 0; return fail(s, ATF_ERR_OOM, "%s (%zu bytes)", what, c); }
+  *cap = c;
+  return ATF_OK;
+}
+
 // bump allocation inside group g's arena; nullptr if no chunk has room
 static char* arena_alloc(atf_space* s, int g, size_t bytes) {
   bytes = (bytes + 255) & ~(size_t)255;
@@ -835,6 +860,11 @@ static void release_device(atf_space* s) {
   for (size_t p = 0; p < s->d_range.size(); p++) dfree(s, s->d_range[p], 8 * s->params[p].values.size());
   s->d_range.clear();
   dfree(s, s->d_status, s->status_cap * 8);
+  dfree(s, s->d_scratch, s->scratch_cap);
+  dfree(s, (char*)s->d_stash, s->stash_cap);
+  s->d_scratch = nullptr;
+  s->d_stash = nullptr;
+  s->scratch_cap = s->stash_cap = 0;
   dfree(s, s->d_counter, 4 * kMaxGroups);
   dfree(s, s->d_totals, 8 * kMaxGroups);
   dfree(s, s->d_ovf, 4 * kMaxGroups);
@@ -897,10 +927,25 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     if ((e = arena_grow(s, g, csr_bytes + n_parents * gp.words * 4))) return e;
     csr = arena_alloc(s, g, csr_bytes);
   }
+  // child region: the largest free tail, grown up front to an estimate of the level's
+  // size (the exact bound n_parents * r when small, else the previous level's branching
+  // factor x 2) so that a fresh space rarely re-runs a level after an overflow
+  uint64_t est;
+  const uint64_t exact = n_parents * (uint64_t)lp.r;
+  if (exact <= (1ull << 24)) {
+    est = exact;
+  } else if (k >= 2 && s->data[g][k - 2].n > 0) {
+    const double bf = (double)s->data[g][k - 1].n / (double)s->data[g][k - 2].n;
+    est = (uint64_t)std::min<double>((double)exact, 2.0 * bf * (double)n_parents + 1024.0);
+  } else {
+    est = std::min<uint64_t>(exact, 16 * n_parents + 1024);
+  }
+  est = std::min<uint64_t>(est, (4ull << 30) / (gp.words * 4));  // at most 4 GB up front
   int which = -1;
   size_t tail = arena_tail(s, g, &which);
-  if (tail < (size_t)gp.words * 4 * 64) {
-    if ((e = arena_grow(s, g, std::max<size_t>(n_parents * gp.words * 4, 1 << 20)))) return e;
+  const size_t want = std::max<size_t>((size_t)est * gp.words * 4, (size_t)gp.words * 4 * 64);
+  if (tail < want) {
+    if ((e = arena_grow(s, g, want))) return e;
     tail = arena_tail(s, g, &which);
   }
   Chunk& c = s->arena[g][which];
@@ -914,13 +959,47 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   a.tile_counter = s->d_counter + g;
   a.total_out = s->d_totals + g;
   a.overflow_flag = s->d_ovf + g;
-  CUDA_TRY(s, cudaMemsetAsync(s->d_status, 0, a.n_tiles * 8, st));
+  const bool wide = a.kind == K_WIDE;
+  uint64_t* scan_out = nullptr;
+  unsigned long long* scan_status = nullptr;
+  unsigned int* scan_counter = nullptr;
+  if (wide) {
+    // scratch: tile_seg u64[n] | tile_base u64[n+1] | tile_total u32[n] (pad) |
+    //          scan status u64[ceil(n/1024)+1] | scan counter u32 | stash_top u64
+    const size_t n = a.n_tiles, nscan = (n + 1023) / 1024 + 1;
+    const size_t o_seg = 0, o_base = o_seg + 8 * n, o_tot = o_base + 8 * (n + 1);
+    const size_t o_scan = (o_tot + 4 * n + 15) & ~(size_t)15, o_cnt = o_scan + 8 * nscan, o_top = o_cnt + 16;
+    if ((e = ensure_buf(s, &s->d_scratch, &s->scratch_cap, o_top + 16, "tile scratch"))) return e;
+    // stash: the level's estimated size (or the exact size after an overflow), not the
+    // whole arena tail
+    const uint64_t stash_recs = std::min<uint64_t>(cap, std::max<uint64_t>({est + est / 4, (uint64_t)1 << 16,
+                                                                             s->stash_hint}));
+    if ((e = ensure_buf(s, (char**)&s->d_stash, &s->stash_cap, (size_t)stash_recs * gp.words * 4, "stash")))
+      return e;
+    a.tile_seg = (unsigned long long*)(s->d_scratch + o_seg);
+    scan_out = (uint64_t*)(s->d_scratch + o_base);
+    a.tile_base = scan_out;
+    a.tile_total = (uint32_t*)(s->d_scratch + o_tot);
+    scan_status = (unsigned long long*)(s->d_scratch + o_scan);
+    scan_counter = (unsigned int*)(s->d_scratch + o_cnt);
+    a.stash_top = (unsigned long long*)(s->d_scratch + o_top);
+    a.stash = s->d_stash;
+    a.stash_cap = s->stash_cap / (gp.words * 4);
+    CUDA_TRY(s, cudaMemsetAsync(s->d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
+  } else {
+    CUDA_TRY(s, cudaMemsetAsync(s->d_status, 0, a.n_tiles * 8, st));
+  }
   CUDA_TRY(s, cudaMemsetAsync(s->d_counter + g, 0, 4, st));
   CUDA_TRY(s, cudaMemsetAsync(s->d_ovf + g, 0, 4, st));
   bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].first, st));
   int ce = launch_expand(a, gp.words, st);
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
+  if (wide) {
+    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st);
+    if (!ce) ce = launch_wide_emit(a, gp.words, st);
+    if (ce) return fail(s, ATF_ERR_CUDA, "wide scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
+  }
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].second, st));
   pd = Pending{g, k, n_parents, parents, (uint64_t*)csr, child, cap, which, off};
   return ATF_OK;
@@ -975,7 +1054,8 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       uint64_t total = s->h_totals[pd.g];
       GroupPlan& gp = s->groups[pd.g];
       if (s->h_flags[pd.g] || total > pd.cap) {
-        // child region too small: grow the arena and redo this level next round
+        // child region or stash too small: grow and redo this level next round
+        s->stash_hint = std::max<uint64_t>(s->stash_hint, total);
         atf_status e = arena_grow(s, pd.g, total * gp.words * 4 + (pd.n_parents + 1) * 8);
         if (e) return e;
         continue;

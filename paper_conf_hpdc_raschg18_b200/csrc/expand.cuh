@@ -57,6 +57,45 @@ __device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, 
   }
 }
 
+// Narrow kernel: conjunct T over all r <= 64 candidates of one node, restricted to the
+// candidates still set in m.  The kind/variant dispatch is hoisted out of the candidate
+// loop; the 16-bit divisibility atoms are evaluated branch-free for every candidate.
+__device__ __forceinline__ uint64_t term_mask_narrow(const LevelArgs& a, const Term& T, int64_t A, int64_t Bv,
+                                                     uint64_t m, int r, const int32_t* s_cx, const uint32_t* s_cm,
+                                                     const uint32_t* s_q, const int64_t* slots, int stride) {
+  if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) {
+    // x | n  iff  n * magic(x) mod 2^32 < 2^16 (magic(0) = 2^16 excludes x == 0)
+    const uint32_t n = (uint32_t)A;
+    uint32_t lo = 0, hi = 0;
+    for (int c = 0; c < r; c++) {
+      const uint32_t mg = s_cm[c];
+      const uint32_t ok = (uint32_t)((n * mg < 0x10000u) & (mg != 0x10000u));
+      if (c < 32) lo |= ok << c; else hi |= ok << (c - 32);
+    }
+    return m & (((uint64_t)hi << 32) | lo);
+  }
+  if (T.kind == T_MULX && T.variant == V16) {
+    const uint32_t md = (uint32_t)Bv, md1 = md - 1u;
+    uint32_t lo = 0, hi = 0;
+    for (int c = 0; c < r; c++) {
+      const int32_t x = s_cx[c];
+      const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+      const uint32_t ok = (uint32_t)(ax * md <= md1);
+      if (c < 32) lo |= ok << c; else hi |= ok << (c - 32);
+    }
+    return m & (((uint64_t)hi << 32) | lo);
+  }
+  uint64_t out = 0, mm = m;
+  while (mm) {
+    const int c = __ffsll((long long)mm) - 1;
+    mm &= mm - 1;
+    const int32_t x = s_cx[c];
+    const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
+    if (term_accepts(a, T, A, Bv, x, ax, s_cm[c], s_q, slots, stride)) out |= 1ull << c;
+  }
+  return out;
+}
+
 // Exact acceptance of candidate (x, m32) by node i of the tile (all conjuncts, node gate).
 static __device__ __noinline__ bool node_accepts(const LevelArgs& a, int i, int tn, int32_t x, uint32_t m32,
                                              const uint32_t* s_ok, const int64_t* s_opa, const int64_t* s_opb,
@@ -252,19 +291,9 @@ __global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ Lev
       // the operand column of this thread (index tid) is reused for each of its nodes
       if (i < tn && prologue_node_impl<W>(a, node0 + i, tid, B, s_ok, s_rec, s_opa, s_opb, s_slots)) {
         uint64_t m = full;
-        for (int t = 0; t < a.n_terms && m; t++) {
-          const Term& T = a.terms[t];
-          const int64_t A = s_opa[t * B + tid], Bv = s_opb[t * B + tid];
-          uint64_t mt = 0;
-          for (int c = 0; c < r; c++) {
-            if (!((m >> c) & 1ull)) continue;
-            const int32_t x = s_cx[c];
-            const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-            if (term_accepts(a, T, A, Bv, x, ax, s_cm[c], s_q, s_slots ? s_slots + tid : nullptr, B))
-              mt |= 1ull << c;
-          }
-          m &= mt;
-        }
+        for (int t = 0; t < a.n_terms && m; t++)
+          m = term_mask_narrow(a, a.terms[t], s_opa[t * B + tid], s_opb[t * B + tid], m, r, s_cx, s_cm, s_q,
+                               s_slots ? s_slots + tid : nullptr, B);
         mask[k] = m;
       }
       if (i < tn) {
@@ -379,8 +408,9 @@ __device__ __forceinline__ void record_mask(const LevelArgs& a, int i, int tn, i
   }
 }
 
-// Children of node i with a large count, emitted by the whole warp: set bitmap words in
-// order, lane b writes the child of bit b (coalesced); consumed words are zeroed.
+// Children of node i with a large count, emitted by the whole warp into the stash: set
+// bitmap words in order, lane b writes the child of bit b (coalesced); consumed words are
+// zeroed.
 template <int W>
 __device__ __forceinline__ void emit_node_warp(const LevelArgs& a, int i, uint64_t rank, int64_t j0, const uint32_t* rec,
                                                uint32_t* s_bm, uint32_t* s_sum, int RW, int SW, int lane) {
@@ -393,14 +423,12 @@ __device__ __forceinline__ void emit_node_warp(const LevelArgs& a, int i, uint64
       const uint32_t word = s_bm[i * RW + wi];
       if ((word >> lane) & 1u) {
         const uint64_t rk = rank + __popc(word & lt);
-        if (rk < a.child_cap) {
+        if (rk < a.stash_cap) {
           const uint32_t pos = (uint32_t)(j0 + wi * 32 + lane);
           uint32_t out[W];
 #pragma unroll
           for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? pos << a.field_shift : 0u);
-          store_record<W>(a.child_rec + rk * W, out);
-        } else {
-          atomicOr(a.overflow_flag, 1u);
+          store_record<W>(a.stash + rk * W, out);
         }
       }
       rank += __popc(word);
@@ -564,7 +592,10 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
     }
     __syncthreads();
 
-    // ---- scan (A5): node counts -> tile offsets; look-back -> tile base
+    // ---- scan (A5, tile part): node counts -> tile-local offsets; the tile's children
+    // go to a stash segment claimed with one atomic (no wait on other tiles); the
+    // device-wide scan of tile totals and the copy to final positions follow in
+    // scan_kernel + wide_emit_kernel.
     if (warp == 0) {
       uint32_t run = 0;
       for (int i0 = 0; i0 < tn; i0 += 32) {
@@ -579,27 +610,26 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
         if (i < tn) s_off[i] = run + incl - v;
         run += __shfl_sync(FULL, incl, 31);
       }
-      const unsigned long long base = lookback(a.status, tile, run, lane);
       if (lane == 0) {
-        s_w[33] = base;
-        if (tile == a.n_tiles - 1) {
-          *a.total_out = base + run;
-          a.csr[a.n_parents] = base + run;
-        }
+        const unsigned long long seg = run ? atomicAdd(a.stash_top, (unsigned long long)run) : 0ull;
+        if (run && seg + run > a.stash_cap) atomicOr(a.overflow_flag, 1u);
+        a.tile_total[tile] = run;
+        a.tile_seg[tile] = seg;
+        s_w[33] = seg;
       }
     }
     __syncthreads();
-    const uint64_t base = s_w[33];
+    const uint64_t seg = s_w[33];
 
-    // ---- emit (A6)
+    // ---- emit (A6, into the stash segment in final order); CSR gets tile-local offsets
     if (ch == 0)
-      for (int i = tid; i < tn; i += B) a.csr[node0 + i] = base + s_off[i];
+      for (int i = tid; i < tn; i += B) a.csr[node0 + i] = s_off[i];
     for (int i0 = warp * 32; i0 < tn; i0 += NW * 32) {
       const int i = i0 + lane;
       const uint32_t cnt = i < tn ? s_cnt[i] : 0u;
       if (cnt && cnt <= kBig) {
         // lane per node: its set words in order, its bits in order
-        uint64_t rank = base + s_off[i];
+        uint64_t rank = seg + s_off[i];
         uint32_t rec[W];
 #pragma unroll
         for (int w = 0; w < W; w++) rec[w] = s_rec[i * W + w];
@@ -615,14 +645,12 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
             while (word) {
               const int b = __ffs(word) - 1;
               word &= word - 1;
-              if (rank < a.child_cap) {
+              if (rank < a.stash_cap) {
                 const uint32_t pos = (uint32_t)(j0 + wi * 32 + b);
                 uint32_t out[W];
 #pragma unroll
                 for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? pos << a.field_shift : 0u);
-                store_record<W>(a.child_rec + rank * W, out);
-              } else {
-                atomicOr(a.overflow_flag, 1u);
+                store_record<W>(a.stash + rank * W, out);
               }
               rank++;
             }
@@ -637,7 +665,7 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
         uint32_t rec[W];
 #pragma unroll
         for (int w = 0; w < W; w++) rec[w] = s_rec[ib * W + w];
-        emit_node_warp<W>(a, ib, base + s_off[ib], j0, rec, s_bm, s_sum, RW, SW, lane);
+        emit_node_warp<W>(a, ib, seg + s_off[ib], j0, rec, s_bm, s_sum, RW, SW, lane);
       }
       if (i < tn) s_cnt[i] = 0u;
     }

@@ -22,6 +22,78 @@ int launch_expand(const LevelArgs& a, int words, void* stream) {
 
 int expand_smem_bytes(const LevelArgs& a, int words) { return expand_layout(a, words).total; }
 
+// ---------------------------------------------------------------- wide level, second half
+// Second half of a wide level: tile_base = exclusive scan of the tile totals (scan_kernel);
+// each tile's stash segment is copied to its final position and the tile's CSR entries
+// get the tile base added.  Grid-stride over tiles, one warp per tile; records move as
+// W-word vectors, 4 loads in flight per lane.
+template <int W>
+struct RecVec;
+template <> struct RecVec<1> { using T = uint32_t; };
+template <> struct RecVec<2> { using T = uint2; };
+template <> struct RecVec<4> { using T = uint4; };
+template <> struct RecVec<8> { using T = uint4; };  // two uint4 per record
+
+template <int W>
+__global__ void __launch_bounds__(256) wide_emit_kernel(const __grid_constant__ LevelArgs a) {
+  using V = typename RecVec<W>::T;
+  constexpr int VPR = W == 8 ? 2 : 1;  // vectors per record
+  const int lane = threadIdx.x & 31;
+  const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t t = gw; t < a.n_tiles; t += nw) {
+    const uint64_t base = a.tile_base[t];
+    const uint64_t cnt = a.tile_total[t];
+    const uint64_t seg = a.tile_seg[t];
+    if (cnt) {
+      if (base + cnt > a.child_cap || seg + cnt > a.stash_cap) {
+        if (lane == 0) atomicOr(a.overflow_flag, 1u);
+      } else {
+        const V* __restrict__ src = reinterpret_cast<const V*>(a.stash + seg * W);
+        V* __restrict__ dst = reinterpret_cast<V*>(a.child_rec + base * W);
+        const uint64_t nv = cnt * VPR;
+        uint64_t k = lane;
+        for (; k + 96 < nv; k += 128) {
+          const V v0 = __ldcs(src + k), v1 = __ldcs(src + k + 32), v2 = __ldcs(src + k + 64), v3 = __ldcs(src + k + 96);
+          dst[k] = v0; dst[k + 32] = v1; dst[k + 64] = v2; dst[k + 96] = v3;
+        }
+        for (; k < nv; k += 32) dst[k] = __ldcs(src + k);
+      }
+    }
+    if (a.n_chunks == 1) {
+      const uint64_t n0 = t * (uint64_t)a.tile_nodes;
+      const uint64_t n1 = min(n0 + (uint64_t)a.tile_nodes, a.n_parents);
+      for (uint64_t n = n0 + lane; n < n1; n += 32) a.csr[n] += base;
+    } else if (lane == 0 && umod64f(t, (uint64_t)a.n_chunks) == 0) {
+      a.csr[udiv64f(t, (uint64_t)a.n_chunks)] += base;
+    }
+    if (t == a.n_tiles - 1 && lane == 0) {
+      const uint64_t total = a.tile_base[a.n_tiles];
+      *a.total_out = total;
+      a.csr[a.n_parents] = total;
+    }
+  }
+}
+
+int launch_wide_emit(const LevelArgs& a, int words, void* stream) {
+  if (a.n_tiles == 0) return 0;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  uint64_t blocks = (a.n_tiles + 7) / 8;  // 8 warps (tiles) per block
+  const uint64_t cap = (uint64_t)sms * 16;
+  if (blocks > cap) blocks = cap;
+  cudaStream_t st = (cudaStream_t)stream;
+  switch (words) {
+    case 1: wide_emit_kernel<1><<<(unsigned)blocks, 256, 0, st>>>(a); break;
+    case 2: wide_emit_kernel<2><<<(unsigned)blocks, 256, 0, st>>>(a); break;
+    case 4: wide_emit_kernel<4><<<(unsigned)blocks, 256, 0, st>>>(a); break;
+    case 8: wide_emit_kernel<8><<<(unsigned)blocks, 256, 0, st>>>(a); break;
+    default: return (int)cudaErrorInvalidValue;
+  }
+  return (int)cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- decode
 // index -> mixed-radix digits (group 0 most significant, P:229-231 reading #11) ->
 // per group: leaf record -> positions -> values; int32 SoA output.

@@ -20,12 +20,21 @@ def main():
     ap.add_argument("config")
     ap.add_argument("--reps", type=int, default=1)
     ap.add_argument("--decode", type=int, default=0)
+    ap.add_argument("--profile-last", action="store_true",
+                    help="cudaProfilerStart/Stop around the last rep (ncu --profile-from-start off)")
     a = ap.parse_args()
     spec = A.config_spec(a.config)
     torch.cuda.set_device(0)
     with Space(spec, device=0) as sp:
-        for _ in range(a.reps):
+        for i in range(a.reps):
+            last = i == a.reps - 1
+            if last and a.profile_last:
+                torch.cuda.synchronize()
+                torch.cuda.profiler.start()
             sp.generate()
+            if last and a.profile_last:
+                torch.cuda.synchronize()
+                torch.cuda.profiler.stop()
         print(a.config, "S =", sp.size(), "groups =", sp.group_sizes(), flush=True)
         if a.decode:
             from atfspec.fuzz import splitmix64_indices
