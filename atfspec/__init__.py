@@ -221,4 +221,4 @@ class Spec:
 
 
 from .configs import *  # noqa: E402,F401,F403
-from .fuzz import random_spec  # noqa: E402,F401
+from .fuzz import random_spec, random_wide_spec  # noqa: E402,F401

@@ -76,6 +76,57 @@ def random_spec(seed: int, n_params: int | None = None) -> Spec:
     return s
 
 
+def _rand_wide_range(rng: random.Random) -> dict:
+    """65..6000 values: the wide expansion kernel's territory (r > 64), sometimes with 0 and
+    negatives, steps, or r > 4096 (several candidate chunks)."""
+    k = rng.random()
+    n = rng.randint(65, 6000)
+    if k < 0.6:
+        b = rng.randint(1, 3) if rng.random() < 0.7 else rng.randint(-40, 0)
+        step = rng.choice([1, 1, 1, 2, 3])
+        return interval(b, b + (n - 1) * step, step)
+    vals = rng.sample(range(-50, 9000), n)
+    return set_(*vals)
+
+
+def _rand_div_atom(rng: random.Random, refs) -> E:
+    """A divisibility conjunct of the shapes the planner compiles to hot atoms (or not)."""
+    j = rng.choice(refs)
+    c = rng.random()
+    if c < 0.35:
+        return E(X.code + P(j).code + [OP_DIVIDES])                      # x | p_j
+    if c < 0.55:
+        return E(X.code + P(j).code + [OP_MULOF])                        # p_j | x
+    if c < 0.7:
+        return E(X.code + (P(j) * rng.randint(1, 12)).code + [OP_DIVIDES])  # x | c p_j
+    if c < 0.8:
+        return E((X * rng.randint(1, 4)).code + P(j).code + [OP_DIVIDES])   # (a x) | p_j
+    if c < 0.9:
+        return E(P(j).code + (C(rng.randint(1, 50)) // X).code + [OP_MULOF])  # (c / x) | p_j
+    return E(X.code + (P(j) + rng.randint(-2, 5)).code + [OP_DIVIDES])   # x | (p_j + c)
+
+
+def random_wide_spec(seed: int) -> Spec:
+    """2-3 parameters whose later ranges have 65..6000 values, constrained by divisibility
+    atoms (kept selective so the oracle finishes in seconds), optionally ANDed / ORed with a
+    random expression.  Pure input generation."""
+    rng = random.Random(1_000_003 + seed)
+    n = rng.randint(2, 3)
+    s = Spec(f"fuzzw_{seed}")
+    s.add("p0", interval(rng.randint(-3, 2), rng.randint(3, 200)))
+    for i in range(1, n):
+        refs = list(range(i))
+        cons = _rand_div_atom(rng, refs)
+        k = rng.random()
+        if k < 0.3:
+            cons = cons & _rand_expr(rng, 2, refs, True)
+        elif k < 0.4:
+            cons = cons | (X.eq(rng.randint(-5, 100)))
+        extra = [_rand_div_atom(rng, refs)] if rng.random() < 0.3 else []
+        s.add(f"p{i}", _rand_wide_range(rng), cons, *extra)
+    return s
+
+
 def splitmix64_indices(n: int, modulus: int, seed: int, start: int = 0) -> np.ndarray:
     """idx_i = splitmix64(seed + i) mod modulus, i in [start, start+n) (C4 input recipe)."""
     if modulus <= 0:

@@ -155,8 +155,9 @@ def run_generation(spec, steps, warmup, dist_ctx=None, timing=True):
 
 
 def roofline_of(res, sm_mhz):
-    """Dominant kernel = expand_kernel (every launch of the step).  achieved = algorithmic int ops
-    (evals_k x c_k, DESIGN.md cost table) / summed device time of the expand launches."""
+    """Dominant kernels = the level expansion (expand_wide + scan + wide_emit, expand_narrow; every
+    launch of the step).  achieved = algorithmic int ops (evals_k x c_k, DESIGN.md cost table) /
+    summed device time of the levels (CUDA events on the launch stream around each level)."""
     plan = res["plan"]
     costs = [lv["cost"] for g in plan["groups"] for lv in g["levels"]]
     ops = sum(s["evals"] * c for s, c in zip(res["stats"], costs))
@@ -175,13 +176,13 @@ def e2e_generation(spec, steps):
     spec (ranges + bytecode uploaded), generated, and S + group sizes read back, every step."""
     import torch
     from paper_conf_hpdc_raschg18_b200 import Space
-    h2d = sum(4 * (len(p.range.get("values", [])) or 0) for p in spec.params)
-    h2d += sum(4 * len(c) for p in spec.params for c in p.constraints)
-    # interval ranges are materialised on the host and uploaded too
+    # per parameter the library uploads [values][magics][|values|], each padded to 128
+    # entries (ensure_device); constraint programs travel as kernel parameters
+    h2d = sum(4 * len(c) for p in spec.params for c in p.constraints)
     for p in spec.params:
-        if p.range["kind"] != "set":
-            r = p.range
-            h2d += 4 * max(0, (r["end"] - r["begin"]) // r["step"] + 1)
+        r = p.range
+        n = len(r["values"]) if r["kind"] == "set" else max(0, (r["end"] - r["begin"]) // r["step"] + 1)
+        h2d += 12 * ((n + 127) // 128 * 128)
     times, d2h = [], 0
     for i in range(steps + 1):
         torch.cuda.synchronize()
@@ -323,7 +324,9 @@ def main():
     # algorithmic evals of the whole job: from the single-GPU level sizes (f_{k-1} r_k)
     gl = [[lv["r"] for lv in g["levels"]] for g in plan["groups"]]
     value = leaves / (ms * 1e-3)
-    n_launch = sum(1 for s in res["stats"] if s["ms"] >= 0)
+    # our kernels per step: every non-empty level launches expand_narrow (r <= 64) or
+    # expand_wide, then scan_kernel and level_emit_kernel
+    n_launch = 3 * sum(1 for s in res["stats"] if s["ms"] >= 0)
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "configs/s", "n_gpus": world, "steps": a.steps,
                 "warmup": a.warmup, "ms_per_step": ms, "higher_is_better": True,

@@ -51,7 +51,8 @@ struct LevelArgs {
   uint64_t n_parents;
   // candidates = materialised range of the level's parameter
   const int32_t* cand;
-  const uint32_t* cand_magic;  // ceil(2^32/|x|) per candidate (0 for |x| <= 1), host-computed
+  const uint32_t* cand_magic;  // ceil(2^32/|x|) mod 2^32 per candidate (2^16 for x == 0), host-computed
+  const uint32_t* cand_abs;    // |x| per candidate; both padded to a multiple of 128
   int32_t r;
   int32_t level;
   int32_t field_word, field_shift;  // where the child's range position goes
@@ -79,7 +80,7 @@ struct LevelArgs {
   uint64_t child_cap;       // capacity of child_rec in records
   unsigned int* overflow_flag;
   // wide levels: children go to per-tile stash segments first (no cross-tile wait),
-  // then wide_emit_kernel copies them to their final positions
+  // then level_emit_kernel copies them to their final positions
   uint32_t* stash;          // [stash_cap][W]
   uint64_t stash_cap;
   unsigned long long* stash_top;
@@ -116,6 +117,7 @@ struct DecodeArgs {
   int32_t n_groups;
   int32_t n_params;
   uint64_t gsize[kMaxGroups];
+  uint64_t gmagic[kMaxGroups];  // floor((2^64 - 1) / gsize) (0 if gsize == 0): mixed-radix division
   const uint32_t* leaves[kMaxGroups];
   int32_t words[kMaxGroups];
   int32_t lvl_begin[kMaxGroups + 1];   // levels of group g: [lvl_begin[g], lvl_begin[g+1])
@@ -169,7 +171,7 @@ ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
 // All return a cudaError_t value as int (0 = success).
 int launch_expand(const LevelArgs& a, int words, void* stream);
 int expand_smem_bytes(const LevelArgs& a, int words);
-int launch_wide_emit(const LevelArgs& a, int words, void* stream);
+int launch_level_emit(const LevelArgs& a, int words, void* stream);
 int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out,
                           int64_t ld, unsigned int* bad_flag, void* stream);
 int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,

@@ -515,8 +515,10 @@ static atf_status compile_level(const std::vector<ParamDef>& P, int p, const std
           i128 nu = absmax(t.nodes[D.a].iv), nb = absmax(t.nodes[m].iv);
           if (xabs < 65536 && nu < 65536 && nb < 65536) {
             T.variant = V16;
-            T.use_qtable = nu <= kQTableMax ? 1 : 0;
-            if (T.use_qtable) a.qmax = std::max<uint32_t>(a.qmax, (uint32_t)nu);
+            // the quotient's divisibility test divides inline (32-bit): QDIV is only reached
+            // by survivors of the cheaper conjuncts, and a per-CTA magic table of the
+            // quotients would cost shared memory that bounds the tile size
+            T.use_qtable = 0;
           } else {
             T.variant = (nu < ((i128)1 << 32) && nb < ((i128)1 << 32)) ? V32 : V64;
           }
@@ -736,15 +738,23 @@ static void choose_geometry(LevelArgs& a, int words) {
       if (B < 256) cost *= 1.1;
       if (cost < best - 1e-9) { best = cost; a.cpt = cpt; a.block = B; a.n_chunks = nch; }
     }
+    if (r >= 2048 && r <= 4096) {
+      // wide ranges: 128-thread CTAs with 16-32 candidates per thread, so that 8 CTAs fit
+      // an SM (64 registers, <= 26 KB shared) and cover each other's tile barriers
+      a.cpt = r > 2048 ? 32 : 16;
+      a.block = (int)(((int64_t)r + a.cpt * 32 - 1) / (a.cpt * 32) * 32);
+      a.n_chunks = 1;
+    }
     a.chunk = a.block * a.cpt;
     a.rw = a.chunk / 32;
     a.sw = (a.rw + 31) / 32;
+    const int smem_budget = a.block <= 128 ? 26 * 1024 : 48 * 1024;
     // the slow-path queue holds one entry per (node quad, thread): it cannot overflow
     int nt = a.n_chunks > 1 ? 4 : std::max(4, std::min(256, ((1 << 18) / a.chunk + 3) / 4 * 4));
     for (;;) {
       a.tile_nodes = nt;
       a.qcap = nt / 4 * a.block;
-      if (nt <= 4 || expand_layout(a, words).total <= 48 * 1024) break;
+      if (nt <= 4 || expand_layout(a, words).total <= smem_budget) break;
       nt -= 4;
     }
   }
@@ -768,18 +778,23 @@ static atf_status ensure_device(atf_space* s) {
   size_t np = s->params.size();
   s->d_range.assign(np, nullptr);
   for (size_t p = 0; p < np; p++) {
-    // [values r][divisibility magics r]: magic(x) = ceil(2^32/|x|) mod 2^32 (0 for |x| == 1);
-    // magic(0) = 2^16, which no 16-bit x != 0 has, so that the wide kernel's uniform test
-    // (n * magic mod 2^32) < 2^16 never accepts x == 0 for n != 0
+    // [values rp][divisibility magics rp][|values| rp], rp = r rounded up to 128 (the wide
+    // kernel reads 16-byte vectors of the last two straight from global memory on chunked
+    // ranges).  magic(x) = ceil(2^32/|x|) mod 2^32 (0 for |x| == 1); magic(0) = 2^16, which
+    // no 16-bit x != 0 has, so the wide kernel's uniform test (n * magic mod 2^32) < 2^16
+    // never accepts x == 0 for n != 0.  Padding: value 1, magic 2^16, |value| 1.
     auto& v = s->params[p].values;
-    s->d_range[p] = (int32_t*)dalloc(s, std::max<size_t>(8, v.size() * 8));
+    const size_t rp = (v.size() + 127) / 128 * 128;
+    s->d_range[p] = (int32_t*)dalloc(s, std::max<size_t>(16, rp * 12));
     if (!s->d_range[p]) return fail(s, ATF_ERR_OOM, "range upload");
     if (!v.empty()) {
-      std::vector<int32_t> buf(v.begin(), v.end());
-      buf.resize(2 * v.size());
-      for (size_t j = 0; j < v.size(); j++) {
-        uint32_t ax = v[j] < 0 ? 0u - (uint32_t)v[j] : (uint32_t)v[j];
-        buf[v.size() + j] = (int32_t)(ax ? 0xffffffffu / ax + 1u : 0x10000u);
+      std::vector<int32_t> buf(3 * rp, 1);
+      for (size_t j = 0; j < rp; j++) {
+        const bool real = j < v.size();
+        const uint32_t ax = real ? (v[j] < 0 ? 0u - (uint32_t)v[j] : (uint32_t)v[j]) : 1u;
+        if (real) buf[j] = v[j];
+        buf[rp + j] = (int32_t)(real ? (ax ? 0xffffffffu / ax + 1u : 0x10000u) : 0x10000u);
+        buf[2 * rp + j] = (int32_t)ax;
       }
       // pageable source: the call returns once `buf` has been staged
       CUDA_TRY(s, cudaMemcpyAsync(s->d_range[p], buf.data(), buf.size() * 4, cudaMemcpyHostToDevice,
@@ -800,15 +815,6 @@ static atf_status ensure_device(atf_space* s) {
   return ATF_OK;
 }
 
-static atf_status ensure_status(atf_space* s, size_t tiles) {
-  if (tiles <= s->status_cap) return ATF_OK;
-  dfree(s, s->d_status, s->status_cap * 8);
-  size_t cap = std::max<size_t>(tiles, s->status_cap * 2);
-  s->d_status = (unsigned long long*)dalloc(s, cap * 8);
-  if (!s->d_status) { s->status_cap = 0; return fail(s, ATF_ERR_OOM, "tile status (%zu tiles)", cap); }
-  s->status_cap = cap;
-  return ATF_OK;
-}
 
 static atf_status ensure_buf(atf_space* s, char** p, size_t* cap, size_t bytes, const char* what) {
   if (bytes <= *cap) return ATF_OK;
@@ -857,7 +863,8 @@ static void release_device(atf_space* s) {
   for (size_t g = 0; g < s->arena.size(); g++)
     for (auto& c : s->arena[g]) dfree(s, c.p, c.size);
   s->arena.clear();
-  for (size_t p = 0; p < s->d_range.size(); p++) dfree(s, s->d_range[p], 8 * s->params[p].values.size());
+  for (size_t p = 0; p < s->d_range.size(); p++)
+    dfree(s, s->d_range[p], 12 * ((s->params[p].values.size() + 127) / 128 * 128));
   s->d_range.clear();
   dfree(s, s->d_status, s->status_cap * 8);
   dfree(s, s->d_scratch, s->scratch_cap);
@@ -908,7 +915,11 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   a.parent_rec = parents;
   a.n_parents = n_parents;
   a.cand = s->d_range[lp.param];
-  a.cand_magic = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + lp.r;  // see ensure_device
+  {  // see ensure_device: [values rp][magic rp][abs rp]
+    const size_t rp = ((size_t)lp.r + 127) / 128 * 128;
+    a.cand_magic = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + rp;
+    a.cand_abs = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + 2 * rp;
+  }
   a.r = lp.r;
   for (int i = 0; i < a.n_pv; i++) a.pv_range[i] = s->d_range[lp.pv_param[i]];
   choose_geometry(a, gp.words);
@@ -918,8 +929,7 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %d bytes of shared memory", k, g, a.smem_bytes);
   if (a.n_tiles >= 0xffffffffull) return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %llu tiles", k, g,
                                               (unsigned long long)a.n_tiles);
-  atf_status e = ensure_status(s, a.n_tiles);
-  if (e) return e;
+  atf_status e = ATF_OK;
   // CSR of the parent level (exact size), then the child region = largest free tail
   size_t csr_bytes = (n_parents + 1) * 8;
   char* csr = arena_alloc(s, g, csr_bytes);
@@ -959,11 +969,12 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   a.tile_counter = s->d_counter + g;
   a.total_out = s->d_totals + g;
   a.overflow_flag = s->d_ovf + g;
-  const bool wide = a.kind == K_WIDE;
+  // every level: the expand kernel writes tile stash segments; scan_kernel turns the tile
+  // totals into tile bases; level_emit_kernel places the segments and fixes the CSR
   uint64_t* scan_out = nullptr;
   unsigned long long* scan_status = nullptr;
   unsigned int* scan_counter = nullptr;
-  if (wide) {
+  {
     // scratch: tile_seg u64[n] | tile_base u64[n+1] | tile_total u32[n] (pad) |
     //          scan status u64[ceil(n/1024)+1] | scan counter u32 | stash_top u64
     const size_t n = a.n_tiles, nscan = (n + 1023) / 1024 + 1;
@@ -986,8 +997,6 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     a.stash = s->d_stash;
     a.stash_cap = s->stash_cap / (gp.words * 4);
     CUDA_TRY(s, cudaMemsetAsync(s->d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
-  } else {
-    CUDA_TRY(s, cudaMemsetAsync(s->d_status, 0, a.n_tiles * 8, st));
   }
   CUDA_TRY(s, cudaMemsetAsync(s->d_counter + g, 0, 4, st));
   CUDA_TRY(s, cudaMemsetAsync(s->d_ovf + g, 0, 4, st));
@@ -995,10 +1004,10 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].first, st));
   int ce = launch_expand(a, gp.words, st);
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
-  if (wide) {
+  {
     ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st);
-    if (!ce) ce = launch_wide_emit(a, gp.words, st);
-    if (ce) return fail(s, ATF_ERR_CUDA, "wide scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
+    if (!ce) ce = launch_level_emit(a, gp.words, st);
+    if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   }
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].second, st));
   pd = Pending{g, k, n_parents, parents, (uint64_t*)csr, child, cap, which, off};
@@ -1119,6 +1128,7 @@ static atf_status make_decode_args(const atf_space* s, DecodeArgs& a) {
   for (int g = 0; g < a.n_groups; g++) {
     const GroupPlan& gp = s->groups[g];
     a.gsize[g] = s->gsize[g];
+    a.gmagic[g] = s->gsize[g] ? ~0ull / s->gsize[g] : 0ull;
     a.leaves[g] = s->data[g].back().rec;
     a.words[g] = gp.words;
     a.lvl_begin[g] = l;

@@ -145,11 +145,14 @@ __device__ __forceinline__ void load_record(const uint32_t* src, uint32_t* rec) 
 // shared memory (node `i` of the tile, global index gnode).  Returns the gate result.
 template <int W>
 __device__ __forceinline__ bool prologue_node_impl(const LevelArgs& a, uint64_t gnode, int i, int tn, uint32_t* s_ok, uint32_t* s_rec,
-                              int64_t* s_opa, int64_t* s_opb, int64_t* s_slots) {
+                              int64_t* s_opa, int64_t* s_opb, int64_t* s_slots, bool rec_staged = false) {
   uint32_t rec[W];
   if (a.level == 0) {
 #pragma unroll
     for (int w = 0; w < W; w++) rec[w] = 0;
+  } else if (rec_staged) {  // the caller prefetched the record into s_rec
+#pragma unroll
+    for (int w = 0; w < W; w++) rec[w] = s_rec[i * W + w];
   } else {
     load_record<W>(a.parent_rec + gnode * W, rec);
   }
@@ -206,8 +209,9 @@ __device__ __forceinline__ bool prologue_node_impl(const LevelArgs& a, uint64_t 
 // Out-of-line copy for the wide kernel (keeps the hot loop's registers free).
 template <int W>
 __device__ __noinline__ bool prologue_node(const LevelArgs& a, uint64_t gnode, int i, int tn, uint32_t* s_ok,
-                                           uint32_t* s_rec, int64_t* s_opa, int64_t* s_opb, int64_t* s_slots) {
-  return prologue_node_impl<W>(a, gnode, i, tn, s_ok, s_rec, s_opa, s_opb, s_slots);
+                                           uint32_t* s_rec, int64_t* s_opa, int64_t* s_opb, int64_t* s_slots,
+                                           bool rec_staged) {
+  return prologue_node_impl<W>(a, gnode, i, tn, s_ok, s_rec, s_opa, s_opb, s_slots, rec_staged);
 }
 
 // Block-wide exclusive scan of one u32 per thread (B <= 1024); returns the exclusive
@@ -243,9 +247,10 @@ __device__ __forceinline__ uint32_t block_excl_scan(uint32_t v, uint32_t* total,
 // blockDim.x * NPT frontier nodes; thread t owns the NPT consecutive nodes
 // [t*NPT, t*NPT + NPT) of the tile (thread order = node order).  Per node: prologue ->
 // exact term-major evaluation of the r candidates into a 64-bit accept mask (count, A4);
-// per tile: block scan of the per-thread child counts + decoupled look-back (A5); then
-// every thread writes its nodes' CSR entries and children records in candidate order
-// (emit, A6).  The prologue's operand columns are per thread and reused node by node.
+// per tile: block scan of the per-thread child counts (A5, tile part); every thread
+// writes its nodes' tile-local CSR entries and its children records, in candidate order,
+// into the tile's stash segment (emit, A6); scan_kernel + level_emit_kernel then place
+// the segments.  The prologue's operand columns are per thread and reused node by node.
 constexpr int kNarrowNPT = 4;
 
 template <int W>
@@ -304,36 +309,35 @@ __global__ void __launch_bounds__(256) expand_narrow(const __grid_constant__ Lev
     }
     uint32_t total;
     const uint32_t excl = block_excl_scan(cnt, &total, s_w);
-    if (tid < 32) {
-      const unsigned long long base = lookback(a.status, tile, total, lane);
-      if (lane == 0) {
-        s_w[33] = base;
-        if (tile == a.n_tiles - 1) {
-          *a.total_out = base + total;
-          a.csr[a.n_parents] = base + total;
-        }
-      }
+    // the tile's children go to a stash segment claimed with one atomic (no wait on other
+    // tiles); scan_kernel + level_emit_kernel place the segments (as for wide levels)
+    if (tid == 0) {
+      const unsigned long long sg = total ? atomicAdd(a.stash_top, (unsigned long long)total) : 0ull;
+      if (total && sg + total > a.stash_cap) atomicOr(a.overflow_flag, 1u);
+      a.tile_total[tile] = total;
+      a.tile_seg[tile] = sg;
+      s_w[33] = sg;
     }
     __syncthreads();
-    uint64_t rank = s_w[33] + excl;
+    const uint64_t seg = s_w[33];
+    uint32_t local = excl;  // tile-local child index (CSR gets it; the emit kernel adds the tile base)
 #pragma unroll
     for (int k = 0; k < kNarrowNPT; k++) {
       const int i = tid * kNarrowNPT + k;
       if (i >= tn) break;
-      a.csr[node0 + i] = rank;
+      a.csr[node0 + i] = local;
       uint64_t m = mask[k];
       while (m) {
         const int c = __ffsll((long long)m) - 1;
         m &= m - 1;
-        if (rank < a.child_cap) {
+        const uint64_t rank = seg + local;
+        if (rank < a.stash_cap) {
           uint32_t out[W];
 #pragma unroll
           for (int w = 0; w < W; w++) out[w] = rec[k][w] | (w == a.field_word ? (uint32_t)c << a.field_shift : 0u);
-          store_record<W>(a.child_rec + rank * W, out);
-        } else {
-          atomicOr(a.overflow_flag, 1u);
+          store_record<W>(a.stash + rank * W, out);
         }
-        rank++;
+        local++;
       }
     }
     __syncthreads();
@@ -486,31 +490,45 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
   if (s_q)
     for (uint32_t q = tid; q <= a.qmax; q += B) s_q[q] = q ? (0xffffffffu / q + 1u) : 0u;
 
-  for (;;) {
-    if (tid == 0) {
-      ctl[0] = atomicAdd(a.tile_counter, 1u);
-      ctl[1] = 0u;  // queue length
+  // tiles by ticket, one ahead: ctl[2] = this tile, ctl[3] = the next one, whose parent
+  // records are prefetched into registers during this tile's hot loop
+  auto tile_nodes = [&](uint64_t t, uint64_t& n0, int64_t& c, int& cnt) {
+    if (a.n_chunks == 1) {
+      n0 = t * (uint64_t)NT;
+      const uint64_t rem = a.n_parents - n0;
+      cnt = rem < (uint64_t)NT ? (int)rem : NT;
+      c = 0;
+    } else {
+      n0 = udiv64f(t, (uint64_t)a.n_chunks);
+      c = (int64_t)umod64f(t, (uint64_t)a.n_chunks);
+      cnt = 1;
     }
-    __syncthreads();
-    const uint64_t tile = ctl[0];
+  };
+  if (tid == 0) {
+    ctl[1] = 0u;  // slow-path queue length (reset again after each tile's slow path)
+    ctl[2] = atomicAdd(a.tile_counter, 1u);
+    ctl[3] = atomicAdd(a.tile_counter, 1u);
+  }
+  __syncthreads();
+  uint32_t pre[W];
+  uint64_t pre_tile = ~0ull;
+  for (;;) {
+    const uint64_t tile = ctl[2], nxt = ctl[3];
     if (tile >= a.n_tiles) break;
     uint64_t node0;
-    int64_t ch = 0;
+    int64_t ch;
     int tn;
-    if (a.n_chunks == 1) {
-      node0 = tile * (uint64_t)NT;
-      const uint64_t rem = a.n_parents - node0;
-      tn = rem < (uint64_t)NT ? (int)rem : NT;
-    } else {
-      node0 = udiv64f(tile, (uint64_t)a.n_chunks);
-      ch = (int64_t)umod64f(tile, (uint64_t)a.n_chunks);
-      tn = 1;
-    }
+    tile_nodes(tile, node0, ch, tn);
     const int64_t j0 = ch * (int64_t)chunk;
     // ---- prologue
     for (int i = tid; i < NT; i += B) {
       if (i < tn) {
-        const bool ok = prologue_node<W>(a, node0 + i, i, NT, s_ok, s_rec, s_opa, s_opb, s_slots);
+        const bool staged = a.level > 0 && i == tid && pre_tile == tile;
+        if (staged) {
+#pragma unroll
+          for (int w = 0; w < W; w++) s_rec[i * W + w] = pre[w];
+        }
+        const bool ok = prologue_node<W>(a, node0 + i, i, NT, s_ok, s_rec, s_opa, s_opb, s_slots, staged);
         if (HOT == HOT_DIVX) {
           s_hot[i] = ok ? (uint32_t)s_opa[hot_t * NT + i] : kHotSentinel;
         } else if (HOT == HOT_MULX) {
@@ -525,6 +543,20 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
       }
     }
     __syncthreads();
+    if (tid == 0) {  // every thread has read ctl[2..3]; claim the tile after next
+      ctl[2] = (uint32_t)nxt;
+      ctl[3] = nxt < a.n_tiles ? atomicAdd(a.tile_counter, 1u) : (uint32_t)nxt;
+    }
+    if (a.level > 0 && nxt < a.n_tiles) {  // prefetch the next tile's parent records
+      uint64_t n0;
+      int64_t c2;
+      int cnt2;
+      tile_nodes(nxt, n0, c2, cnt2);
+      if (tid < cnt2) {
+        load_record<W>(a.parent_rec + (n0 + tid) * W, pre);
+        pre_tile = nxt;
+      }
+    }
 
     // ---- hot loop (A4): superset filter, queue (node quad, thread) on a possible accept
     const bool dense = HOT == HOT_NONE;
@@ -611,6 +643,7 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
         run += __shfl_sync(FULL, incl, 31);
       }
       if (lane == 0) {
+        ctl[1] = 0u;  // queue consumed (barrier after the slow path); next tile's hot loop is 2 barriers away
         const unsigned long long seg = run ? atomicAdd(a.stash_top, (unsigned long long)run) : 0ull;
         if (run && seg + run > a.stash_cap) atomicOr(a.overflow_flag, 1u);
         a.tile_total[tile] = run;
@@ -709,6 +742,7 @@ static int launch_w(const LevelArgs& a, void* stream) {
     case 4: return launch_wide_wc<W, 4>(a, stream);
     case 8: return launch_wide_wc<W, 8>(a, stream);
     case 16: return launch_wide_wc<W, 16>(a, stream);
+    case 32: return launch_wide_wc<W, 32>(a, stream);
     default: return (int)cudaErrorInvalidValue;
   }
 }

@@ -23,7 +23,7 @@ int launch_expand(const LevelArgs& a, int words, void* stream) {
 int expand_smem_bytes(const LevelArgs& a, int words) { return expand_layout(a, words).total; }
 
 // ---------------------------------------------------------------- wide level, second half
-// Second half of a wide level: tile_base = exclusive scan of the tile totals (scan_kernel);
+// Second half of a level (wide and narrow kernels alike): tile_base = exclusive scan of the tile totals (scan_kernel);
 // each tile's stash segment is copied to its final position and the tile's CSR entries
 // get the tile base added.  Grid-stride over tiles, one warp per tile; records move as
 // W-word vectors, 4 loads in flight per lane.
@@ -35,7 +35,7 @@ template <> struct RecVec<4> { using T = uint4; };
 template <> struct RecVec<8> { using T = uint4; };  // two uint4 per record
 
 template <int W>
-__global__ void __launch_bounds__(256) wide_emit_kernel(const __grid_constant__ LevelArgs a) {
+__global__ void __launch_bounds__(256) level_emit_kernel(const __grid_constant__ LevelArgs a) {
   using V = typename RecVec<W>::T;
   constexpr int VPR = W == 8 ? 2 : 1;  // vectors per record
   const int lane = threadIdx.x & 31;
@@ -75,7 +75,7 @@ __global__ void __launch_bounds__(256) wide_emit_kernel(const __grid_constant__ 
   }
 }
 
-int launch_wide_emit(const LevelArgs& a, int words, void* stream) {
+int launch_level_emit(const LevelArgs& a, int words, void* stream) {
   if (a.n_tiles == 0) return 0;
   int dev = 0, sms = 0;
   cudaGetDevice(&dev);
@@ -85,10 +85,10 @@ int launch_wide_emit(const LevelArgs& a, int words, void* stream) {
   if (blocks > cap) blocks = cap;
   cudaStream_t st = (cudaStream_t)stream;
   switch (words) {
-    case 1: wide_emit_kernel<1><<<(unsigned)blocks, 256, 0, st>>>(a); break;
-    case 2: wide_emit_kernel<2><<<(unsigned)blocks, 256, 0, st>>>(a); break;
-    case 4: wide_emit_kernel<4><<<(unsigned)blocks, 256, 0, st>>>(a); break;
-    case 8: wide_emit_kernel<8><<<(unsigned)blocks, 256, 0, st>>>(a); break;
+    case 1: level_emit_kernel<1><<<(unsigned)blocks, 256, 0, st>>>(a); break;
+    case 2: level_emit_kernel<2><<<(unsigned)blocks, 256, 0, st>>>(a); break;
+    case 4: level_emit_kernel<4><<<(unsigned)blocks, 256, 0, st>>>(a); break;
+    case 8: level_emit_kernel<8><<<(unsigned)blocks, 256, 0, st>>>(a); break;
     default: return (int)cudaErrorInvalidValue;
   }
   return (int)cudaGetLastError();
@@ -116,10 +116,16 @@ __global__ void decode_kernel(const __grid_constant__ DecodeArgs a, const uint64
     }
     for (int g = a.n_groups - 1; g >= 0; g--) {
       uint64_t d;
-      if (idx) {
+      if (idx) {  // rem / sz by multiply-high with floor((2^64-1)/sz) + at most 2 corrections
         const uint64_t sz = a.gsize[g];
-        d = rem % sz;
-        rem /= sz;
+        uint64_t q = __umul64hi(rem, a.gmagic[g]);
+        uint64_t rr = rem - q * sz;
+        while (rr >= sz) {
+          q++;
+          rr -= sz;
+        }
+        d = rr;
+        rem = q;
       } else {
         d = __ldg(digits + (int64_t)g * n + i);
       }

@@ -78,7 +78,7 @@ def test_atoms_for_the_hot_levels():
     lv = sp.plan_json()["groups"][0]["levels"]
     kinds = [[t["kind"] for t in l["terms"]] for l in lv]
     assert kinds[6] == [2, 5] and all(t["variant"] == 0 for t in lv[6]["terms"])
-    assert lv[6]["terms"][1]["qtable"] == 1
+    assert lv[6]["terms"][1]["qtable"] == 0  # quotient divisibility divides inline
     assert kinds[8] == [4, 4] and kinds[9] == [4, 4]
     assert lv[6]["cost"] == 9.0 and lv[9]["cost"] == 5.0
     sp = _space(A.c5_chains())

@@ -106,6 +106,18 @@ def test_fuzz_specs_generic(Space, seed):
     _check_against_oracle(Space, A.random_spec(seed), generic=True)
 
 
+@pytest.mark.parametrize("seed", range(40))
+def test_fuzz_wide_specs(Space, seed):
+    """Ranges of 65..6000 values (the wide kernel: hot filters x|n, d|x, (a x)|n, generic
+    conjuncts, chunked ranges > 4096, zero and negative candidates) vs the oracle."""
+    _check_against_oracle(Space, A.random_wide_spec(seed))
+
+
+@pytest.mark.parametrize("seed", range(0, 40, 5))
+def test_fuzz_wide_specs_generic(Space, seed):
+    _check_against_oracle(Space, A.random_wide_spec(seed), generic=True)
+
+
 def test_wide_ranges_chunked(Space):
     """r > 4096 candidates per level -> several candidate chunks per frontier node."""
     _check_against_oracle(Space, A.saxpy(5040 * 4))
