@@ -94,6 +94,8 @@ typedef struct {
 #define ATF_FLAG_TIMING 1u        /* record per-level CUDA-event times (atf_space_stats)  */
 #define ATF_FLAG_GENERIC_ONLY 2u  /* disable the hoisted fast atoms: interpret every
                                      candidate with the generic bytecode interpreter     */
+#define ATF_FLAG_LEGACY_WIDE 8u   /* levels with r > 64 use the block-tile kernel instead of
+                                     the warp-tile kernel (kept for parity coverage)      */
 #define ATF_FLAG_KEEP_LEVELS 4u   /* keep inner-level arrays (CSR + records); default
                                      keeps them too — reserved                          */
 

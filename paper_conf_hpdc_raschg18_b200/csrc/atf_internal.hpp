@@ -87,6 +87,7 @@ struct LevelArgs {
   uint32_t* tile_total;     // [n_tiles] children per tile
   unsigned long long* tile_seg;  // [n_tiles] stash segment (records)
   const uint64_t* tile_base;     // [n_tiles + 1] exclusive scan of tile_total
+  const uint32_t* piece_tile;    // [total / kPiece + 1] tile holding output record p * kPiece
   // geometry (host choose_geometry)
   int32_t kind;             // K_NARROW: one thread per frontier node, r <= 64 candidates each
                             // K_WIDE:   each thread owns cpt consecutive candidates of a chunk
@@ -96,12 +97,16 @@ struct LevelArgs {
   int32_t chunk;            // wide: candidates per chunk (= block * cpt)
   int32_t rw, sw;           // wide: bitmap words per node (chunk/32), summary words (ceil(rw/32))
   int32_t qcap;             // wide: slow-path queue entries per tile
+  int32_t nseg;             // warp-tile: candidate segments of 32*cpt per node (<= kMaxSeg)
   int64_t n_chunks;         // candidate chunks per node (r > chunk); tile_nodes == 4 padded, 1 real
   uint64_t n_tiles;
   uint32_t qmax;            // T_QDIV table covers quotients [0, qmax]
   int32_t smem_bytes;
 };
-enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1 };
+enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1, K_WTILE = 2 };
+constexpr int kWT = 32;        // warp-tile kernel: frontier nodes per warp tile (one per lane)
+constexpr int kMaxSeg = 8;     // warp-tile kernel: candidate segments per node
+constexpr int kPieceShift = 10;  // level_emit_kernel copies the level in pieces of 2^10 records
 // Hot-loop filter of the wide kernel: a superset test of one conjunct, 2 instructions per
 // (node, candidate) pair (IMAD + ISETP.OR into a per-node predicate).
 enum HotKind : int32_t {
@@ -167,6 +172,35 @@ ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
   return L;
 }
 
+// Warp-tile kernel layout: a CTA-wide candidate table (hot operand per candidate,
+// transposed [seg][c][lane] so that lane b's CPT candidates are conflict-free) and one
+// private region per warp (its tile's records, gates, hot operands, item words, operands).
+struct WarpLayout {
+  int tab, qtab, warp0, wstride;            // CTA part; warp w's region at warp0 + w * wstride
+  int rec, ok, hot, hot2, cnt, items, opa, opb, slots;  // offsets inside a warp region
+  int total;
+};
+ATF_HD WarpLayout wtile_layout(const LevelArgs& a, int words) {
+  WarpLayout L;
+  int o = 0;
+  if (a.hot != HOT_NONE) { L.tab = o; o = align16(o + 4 * a.nseg * 32 * a.cpt); } else { L.tab = -1; }
+  if (a.qmax > 0) { L.qtab = o; o = align16(o + 4 * ((int)a.qmax + 1)); } else { L.qtab = -1; }
+  L.warp0 = o;
+  int w = 0;
+  L.rec = w; w = align16(w + 4 * words * kWT);
+  L.ok = w; w += 4 * kWT;
+  L.hot = w; w += 4 * kWT;
+  L.hot2 = w; w += 4 * kWT;
+  L.cnt = w; w += 4 * kWT;
+  L.items = w; w = align16(w + 4 * kWT * a.nseg);
+  L.opa = w; w = align16(w + 8 * kWT * a.n_terms);
+  L.opb = w; w = align16(w + 8 * kWT * a.n_terms);
+  if (a.need_slots_smem) { L.slots = w; w = align16(w + 8 * kWT * a.n_slots); } else { L.slots = -1; }
+  L.wstride = w;
+  L.total = o + w * (a.block / 32);
+  return L;
+}
+
 // ---- launch wrappers (kernels.cu) ------------------------------------------------
 // All return a cudaError_t value as int (0 = success).
 int launch_expand(const LevelArgs& a, int words, void* stream);
@@ -177,7 +211,8 @@ int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, i
 int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,
                          int64_t ld, unsigned int* bad_flag, void* stream);
 int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long long* status,
-                    unsigned int* counter, void* stream);
+                    unsigned int* counter, void* stream, uint32_t* piece_tile = nullptr,
+                    uint64_t piece_cap = 0);
 int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
 
 }  // namespace atf

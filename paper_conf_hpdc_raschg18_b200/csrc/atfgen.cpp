@@ -708,12 +708,44 @@ static atf_status plan(atf_space* s) {
 // r <= 64 -> narrow kernel (thread per node); otherwise the wide
 // kernel with cpt candidates per thread, a hot filter when a conjunct allows one, and
 // ~2^18 (node, candidate) pairs per tile.
-static void choose_geometry(LevelArgs& a, int words) {
+static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
   const int r = a.r;
   a.hot = HOT_NONE;
   a.hot_term = 0;
   a.n_chunks = 1;
   a.rw = a.sw = a.qcap = 0;
+  a.nseg = 0;
+  if (r > 64 && !legacy_wide) {
+    // warp-tile kernel: segments of 32*cpt candidates; cost per node quad
+    // ~ nseg * (6 cpt + 12) instructions (hot loop + per-quad ballots / loop overhead)
+    int best_cpt = 0, best_nseg = 0;
+    double best = 1e30;
+    for (int cpt : {4, 8, 12, 16, 20, 24, 32}) {
+      const int64_t seg = 32 * (int64_t)cpt;
+      const int64_t nseg = ((int64_t)r + seg - 1) / seg;
+      if (nseg > kMaxSeg) continue;
+      const double cost = (double)nseg * (6.0 * cpt + 12.0);
+      if (cost < best - 1e-9) { best = cost; best_cpt = cpt; best_nseg = (int)nseg; }
+    }
+    if (best_cpt) {
+      for (int t = 0; t < a.n_terms; t++) {
+        const Term& T = a.terms[t];
+        if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) { a.hot = HOT_DIVX; a.hot_term = t; break; }
+        if (T.kind == T_MULX && T.variant == V16) { a.hot = HOT_MULX; a.hot_term = t; break; }
+      }
+      a.kind = K_WTILE;
+      a.cpt = best_cpt;
+      a.nseg = best_nseg;
+      a.chunk = 32 * best_cpt * best_nseg;
+      a.tile_nodes = kWT;
+      // 8 warps per CTA unless the level has too few tiles to give every SM a full CTA
+      const uint64_t tiles = (a.n_parents + kWT - 1) / kWT;
+      const uint64_t per_sm = (tiles + 147) / 148;
+      a.block = 32 * (int)std::min<uint64_t>(8, std::max<uint64_t>(1, per_sm));
+      a.smem_bytes = wtile_layout(a, words).total;
+      return;
+    }
+  }
   if (r <= 64) {
     a.kind = K_NARROW;
     a.block = 256;
@@ -922,7 +954,7 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   }
   a.r = lp.r;
   for (int i = 0; i < a.n_pv; i++) a.pv_range[i] = s->d_range[lp.pv_param[i]];
-  choose_geometry(a, gp.words);
+  choose_geometry(a, gp.words, (s->opts.flags & ATF_FLAG_LEGACY_WIDE) != 0);
   a.n_tiles = a.n_chunks > 1 ? n_parents * (uint64_t)a.n_chunks
                              : (n_parents + (uint64_t)a.tile_nodes - 1) / (uint64_t)a.tile_nodes;
   if (a.smem_bytes > 227 * 1024)
@@ -974,19 +1006,26 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   uint64_t* scan_out = nullptr;
   unsigned long long* scan_status = nullptr;
   unsigned int* scan_counter = nullptr;
+  uint32_t* piece_tile = nullptr;
+  uint64_t piece_cap = 0;
   {
-    // scratch: tile_seg u64[n] | tile_base u64[n+1] | tile_total u32[n] (pad) |
-    //          scan status u64[ceil(n/1024)+1] | scan counter u32 | stash_top u64
-    const size_t n = a.n_tiles, nscan = (n + 1023) / 1024 + 1;
-    const size_t o_seg = 0, o_base = o_seg + 8 * n, o_tot = o_base + 8 * (n + 1);
-    const size_t o_scan = (o_tot + 4 * n + 15) & ~(size_t)15, o_cnt = o_scan + 8 * nscan, o_top = o_cnt + 16;
-    if ((e = ensure_buf(s, &s->d_scratch, &s->scratch_cap, o_top + 16, "tile scratch"))) return e;
     // stash: the level's estimated size (or the exact size after an overflow), not the
     // whole arena tail
     const uint64_t stash_recs = std::min<uint64_t>(cap, std::max<uint64_t>({est + est / 4, (uint64_t)1 << 16,
                                                                              s->stash_hint}));
     if ((e = ensure_buf(s, (char**)&s->d_stash, &s->stash_cap, (size_t)stash_recs * gp.words * 4, "stash")))
       return e;
+    a.stash = s->d_stash;
+    a.stash_cap = s->stash_cap / (gp.words * 4);
+    // scratch: tile_seg u64[n] | tile_base u64[n+1] | tile_total u32[n] (pad) |
+    //          scan status u64[ceil(n/1024)+1] | scan counter u32 | stash_top u64 |
+    //          piece_tile u32[stash_cap / 2^kPieceShift + 2]
+    const size_t n = a.n_tiles, nscan = (n + 1023) / 1024 + 1;
+    const size_t o_seg = 0, o_base = o_seg + 8 * n, o_tot = o_base + 8 * (n + 1);
+    const size_t o_scan = (o_tot + 4 * n + 15) & ~(size_t)15, o_cnt = o_scan + 8 * nscan, o_top = o_cnt + 16;
+    const size_t o_piece = o_top + 16;
+    piece_cap = (a.stash_cap >> kPieceShift) + 2;
+    if ((e = ensure_buf(s, &s->d_scratch, &s->scratch_cap, o_piece + 4 * piece_cap, "tile scratch"))) return e;
     a.tile_seg = (unsigned long long*)(s->d_scratch + o_seg);
     scan_out = (uint64_t*)(s->d_scratch + o_base);
     a.tile_base = scan_out;
@@ -994,8 +1033,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     scan_status = (unsigned long long*)(s->d_scratch + o_scan);
     scan_counter = (unsigned int*)(s->d_scratch + o_cnt);
     a.stash_top = (unsigned long long*)(s->d_scratch + o_top);
-    a.stash = s->d_stash;
-    a.stash_cap = s->stash_cap / (gp.words * 4);
+    piece_tile = (uint32_t*)(s->d_scratch + o_piece);
+    a.piece_tile = piece_tile;
     CUDA_TRY(s, cudaMemsetAsync(s->d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
   }
   CUDA_TRY(s, cudaMemsetAsync(s->d_counter + g, 0, 4, st));
@@ -1005,7 +1044,7 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   int ce = launch_expand(a, gp.words, st);
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   {
-    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st);
+    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st, piece_tile, piece_cap);
     if (!ce) ce = launch_level_emit(a, gp.words, st);
     if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   }

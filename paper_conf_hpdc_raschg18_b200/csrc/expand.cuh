@@ -706,6 +706,315 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
   }
 }
 
+// ---------------------------------------------------------------- warp-tile expand kernel
+// One launch = one tree level of one group, for 64 < r <= kMaxSeg * 32 * CPT.  Every warp
+// works alone on tiles of kWT = 32 consecutive frontier nodes x all r candidates (no block
+// barrier after the candidate table is staged), so the scheduler always has independent
+// warps to issue from.  Candidate position j = seg * 32 * CPT + b * CPT + c: lane b owns
+// CPT consecutive candidates of every segment.  Per tile:
+//   prologue  lane i: node i's path record -> ancestor values -> operands (warp region)
+//   hot loop  (A4) per segment, per node quad: one IMAD + half a VIMNMX3 per pair (the
+//             expand_wide filter); the per-node ballot of "some candidate of lane b may
+//             pass" is the node's item word for the segment (item = node x seg x lane)
+//   items     the tile's items in canonical order (node, seg, lane) = candidate order;
+//             rounds of 32 items, one per lane: exact accept mask of the item's CPT
+//             candidates (hot conjunct from the table, other conjuncts on survivors)
+//   scan      (A5) warp scan of node counts -> tile-local CSR; one atomicAdd claims the
+//             tile's stash segment (no wait on other tiles)
+//   emit      (A6) warp scan of item counts -> each lane writes its item's children
+//             (records = parent record | position) in final order into the segment
+// scan_kernel + level_emit_kernel then place the segments (as for the other kernels).
+
+// position of the (n+1)-th set bit of w (n < popc(w))
+__device__ __forceinline__ int nth_set_bit(uint32_t w, int n) {
+  int pos = 0;
+#pragma unroll
+  for (int s = 16; s > 0; s >>= 1) {
+    const int c = __popc(w & ((1u << s) - 1u));
+    if (n >= c) { n -= c; w >>= s; pos += s; }
+  }
+  return pos;
+}
+
+template <int CPT, int HOT>
+__device__ __forceinline__ uint32_t wtile_item_mask(const LevelArgs& a, int i, int sg, int b, const uint32_t* s_tab,
+                                                    const uint32_t* s_ok, const uint32_t* s_hot,
+                                                    const uint32_t* s_hot2, const int64_t* s_opa,
+                                                    const int64_t* s_opb, const int64_t* s_slots,
+                                                    const uint32_t* s_q) {
+  constexpr int SEG = 32 * CPT;
+  const int64_t jl = (int64_t)sg * SEG + (int64_t)b * CPT;
+  const int64_t left = (int64_t)a.r - jl;
+  const uint32_t valid = left >= CPT ? (CPT == 32 ? 0xffffffffu : ((1u << CPT) - 1u))
+                                     : (left > 0 ? ((1u << left) - 1u) : 0u);
+  uint32_t mask = 0;
+  if (HOT == HOT_NONE) {
+#pragma unroll 4
+    for (int c = 0; c < CPT; c++)
+      if (((valid >> c) & 1u) &&
+          node_accepts(a, i, kWT, __ldg(a.cand + jl + c), __ldg(a.cand_magic + jl + c), s_ok, s_opa, s_opb, s_slots,
+                       s_q))
+        mask |= 1u << c;
+    return mask;
+  }
+  const uint32_t n = s_hot[i], d1 = s_hot2[i];
+  const uint32_t* tp = s_tab + sg * SEG + b;
+#pragma unroll
+  for (int c = 0; c < CPT; c++) {
+    const uint32_t t = tp[c * 32];
+    bool ok;
+    if (HOT == HOT_DIVX) ok = n * t < 0x10000u && t != 0x10000u;  // x | n, exact for 16-bit operands
+    else ok = t * n <= d1;                                          // d | x, n = ceil(2^32/d)
+    mask |= (uint32_t)ok << c;
+  }
+  mask &= valid;
+  if (mask && a.n_terms > 1) mask = other_terms_mask(a, i, kWT, jl, mask, a.hot_term, s_opa, s_opb, s_slots, s_q);
+  return mask;
+}
+
+// Item k of the tile -> (node, segment, lane b).  ie: this lane's exclusive item prefix
+// (lane = node); nodes without items share the next node's prefix, so the largest node
+// whose prefix is <= k owns item k.
+template <int HOT>
+__device__ __forceinline__ void wtile_decode_item(uint32_t k, uint32_t ie, const uint32_t* s_items, int nseg,
+                                                  uint32_t vword_last, int& node, int& sg, int& b) {
+  int nd = 0;
+#pragma unroll
+  for (int s = 16; s > 0; s >>= 1) {
+    const uint32_t e = __shfl_sync(FULL, ie, (nd + s) & 31);
+    if (nd + s < 32 && e <= k) nd += s;
+  }
+  int rr = (int)(k - __shfl_sync(FULL, ie, nd));
+  node = nd;
+  sg = 0;
+  b = 0;
+  for (int q = 0; q < nseg; q++) {
+    const uint32_t w = HOT == HOT_NONE ? (q == nseg - 1 ? vword_last : 0xffffffffu) : s_items[q * kWT + nd];
+    const int p = __popc(w);
+    if (rr < p) {
+      sg = q;
+      b = nth_set_bit(w, rr);
+      break;
+    }
+    rr -= p;
+  }
+}
+
+template <int W, int CPT, int HOT>
+__global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ LevelArgs a) {
+  extern __shared__ __align__(16) unsigned char smem[];
+  constexpr int SEG = 32 * CPT;
+  const WarpLayout L = wtile_layout(a, W);
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int nseg = a.nseg, r = a.r, hot_t = a.hot_term;
+  uint32_t* s_tab = L.tab >= 0 ? reinterpret_cast<uint32_t*>(smem + L.tab) : nullptr;
+  uint32_t* s_q = L.qtab >= 0 ? reinterpret_cast<uint32_t*>(smem + L.qtab) : nullptr;
+  if (HOT != HOT_NONE) {
+    // hot operand per candidate slot, transposed [seg][c][lane]; padding: magic(0) = 2^16
+    // (DIVX) / |x| = 1 (MULX), rejected by the exact test's validity mask
+    const uint32_t* src = HOT == HOT_DIVX ? a.cand_magic : a.cand_abs;
+    const uint32_t pad = HOT == HOT_DIVX ? 0x10000u : 1u;
+    for (int j = threadIdx.x; j < nseg * SEG; j += blockDim.x) {
+      const int sg = j / SEG, rem = j - sg * SEG, b = rem / CPT, c = rem - b * CPT;
+      s_tab[sg * SEG + c * 32 + b] = j < r ? __ldg(src + j) : pad;
+    }
+  }
+  if (s_q)
+    for (uint32_t q = threadIdx.x; q <= a.qmax; q += blockDim.x) s_q[q] = q ? (0xffffffffu / q + 1u) : 0u;
+  __syncthreads();  // the only block barrier: everything below is per warp
+
+  unsigned char* wb = smem + L.warp0 + warp * L.wstride;
+  uint32_t* s_rec = reinterpret_cast<uint32_t*>(wb + L.rec);
+  uint32_t* s_ok = reinterpret_cast<uint32_t*>(wb + L.ok);
+  uint32_t* s_hot = reinterpret_cast<uint32_t*>(wb + L.hot);
+  uint32_t* s_hot2 = reinterpret_cast<uint32_t*>(wb + L.hot2);
+  uint32_t* s_cnt = reinterpret_cast<uint32_t*>(wb + L.cnt);
+  uint32_t* s_items = reinterpret_cast<uint32_t*>(wb + L.items);
+  int64_t* s_opa = reinterpret_cast<int64_t*>(wb + L.opa);
+  int64_t* s_opb = reinterpret_cast<int64_t*>(wb + L.opb);
+  int64_t* s_slots = L.slots >= 0 ? reinterpret_cast<int64_t*>(wb + L.slots) : nullptr;
+  s_cnt[lane] = 0u;
+  // valid-lane word of the last segment (dense levels: every valid pair is an item)
+  const int64_t last_left = (int64_t)r - (int64_t)(nseg - 1) * SEG;  // candidates in the last segment
+  const int last_lanes = (int)((last_left + CPT - 1) / CPT);
+  const uint32_t vword_last = last_lanes >= 32 ? 0xffffffffu : ((1u << last_lanes) - 1u);
+
+  uint32_t cur = 0, nxt = 0;
+  if (lane == 0) {
+    cur = atomicAdd(a.tile_counter, 1u);
+    nxt = atomicAdd(a.tile_counter, 1u);
+  }
+  cur = __shfl_sync(FULL, cur, 0);
+  nxt = __shfl_sync(FULL, nxt, 0);
+  uint32_t pre[W];
+  uint64_t pre_tile = ~0ull;
+  while ((uint64_t)cur < a.n_tiles) {
+    const uint64_t node0 = (uint64_t)cur * kWT;
+    const uint64_t remn = a.n_parents - node0;
+    const int tn = remn < (uint64_t)kWT ? (int)remn : kWT;
+    // ---- prologue: lane = node
+    bool ok = false;
+    if (lane < tn) {
+      const bool staged = a.level > 0 && pre_tile == cur;
+      if (staged) {
+#pragma unroll
+        for (int w = 0; w < W; w++) s_rec[lane * W + w] = pre[w];
+      }
+      ok = prologue_node<W>(a, node0 + lane, lane, kWT, s_ok, s_rec, s_opa, s_opb, s_slots, staged);
+    } else {
+      s_ok[lane] = 0u;
+    }
+    if (HOT == HOT_DIVX) {
+      s_hot[lane] = ok ? (uint32_t)s_opa[hot_t * kWT + lane] : kHotSentinel;
+    } else if (HOT == HOT_MULX) {
+      const uint32_t md = ok ? (uint32_t)s_opb[hot_t * kWT + lane] : (0xffffffffu / kHotSentinel + 1u);
+      s_hot[lane] = md;
+      s_hot2[lane] = md - 1u;
+    }
+    // claim the tile after next; prefetch the next tile's parent records
+    uint32_t nn = nxt;
+    if (lane == 0 && (uint64_t)nxt < a.n_tiles) nn = atomicAdd(a.tile_counter, 1u);
+    nn = __shfl_sync(FULL, nn, 0);
+    if (a.level > 0 && (uint64_t)nxt < a.n_tiles) {
+      const uint64_t n1 = (uint64_t)nxt * kWT + lane;
+      if (n1 < a.n_parents) {
+        load_record<W>(a.parent_rec + n1 * W, pre);
+        pre_tile = nxt;
+      }
+    }
+    __syncwarp();
+
+    // ---- hot loop (A4): item words = per-node ballots of the superset filter
+    const int nq = (tn + 3) >> 2;
+    if (HOT != HOT_NONE) {
+      for (int sg = 0; sg < nseg; sg++) {
+        uint32_t hm[CPT];
+        const uint32_t* tp = s_tab + sg * SEG + lane;
+#pragma unroll
+        for (int c = 0; c < CPT; c++) hm[c] = tp[c * 32];
+        for (int q = 0; q < nq; q++) {
+          const uint4 n4 = *reinterpret_cast<const uint4*>(s_hot + 4 * q);
+          uint32_t m0 = 0xffffffffu, m1 = 0xffffffffu, m2 = 0xffffffffu, m3 = 0xffffffffu;
+#pragma unroll
+          for (int c = 0; c < CPT; c++) {
+            m0 = min(m0, n4.x * hm[c]);
+            m1 = min(m1, n4.y * hm[c]);
+            m2 = min(m2, n4.z * hm[c]);
+            m3 = min(m3, n4.w * hm[c]);
+          }
+          bool h0, h1, h2, h3;
+          if (HOT == HOT_DIVX) {
+            h0 = m0 < 0x10000u; h1 = m1 < 0x10000u; h2 = m2 < 0x10000u; h3 = m3 < 0x10000u;
+          } else {
+            const uint4 d4 = *reinterpret_cast<const uint4*>(s_hot2 + 4 * q);
+            h0 = m0 <= d4.x; h1 = m1 <= d4.y; h2 = m2 <= d4.z; h3 = m3 <= d4.w;
+          }
+          const uint32_t b0 = __ballot_sync(FULL, h0), b1 = __ballot_sync(FULL, h1);
+          const uint32_t b2 = __ballot_sync(FULL, h2), b3 = __ballot_sync(FULL, h3);
+          if (lane == 0) *reinterpret_cast<uint4*>(s_items + sg * kWT + 4 * q) = make_uint4(b0, b1, b2, b3);
+        }
+      }
+      __syncwarp();
+    }
+
+    // ---- items: per-node item counts (lane = node) -> exclusive item prefix
+    uint32_t ic = 0;
+    if (lane < tn && s_ok[lane]) {
+      if (HOT == HOT_NONE) {
+        ic = (uint32_t)(nseg - 1) * 32u + (uint32_t)__popc(vword_last);
+      } else {
+        for (int sg = 0; sg < nseg; sg++) ic += (uint32_t)__popc(s_items[sg * kWT + lane]);
+      }
+    }
+    uint32_t ie = ic;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, ie, o);
+      if (lane >= o) ie += y;
+    }
+    const uint32_t T = __shfl_sync(FULL, ie, 31);
+    ie -= ic;
+    // pass 1: exact masks -> node counts; the first 4 rounds keep their masks in registers
+    uint32_t km0 = 0, km1 = 0, km2 = 0, km3 = 0;
+    for (uint32_t R = 0; R < T; R += 32) {
+      const uint32_t k = R + lane;
+      int node, sg, b;
+      wtile_decode_item<HOT>(k < T ? k : T - 1, ie, s_items, nseg, vword_last, node, sg, b);
+      uint32_t m = 0;
+      if (k < T)
+        m = wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q);
+      if (R == 0) km0 = m;
+      else if (R == 32) km1 = m;
+      else if (R == 64) km2 = m;
+      else if (R == 96) km3 = m;
+      if (m) atomicAdd(&s_cnt[node], (uint32_t)__popc(m));
+    }
+    __syncwarp();
+    // ---- scan (A5, tile part): node counts -> tile-local CSR offsets, stash segment
+    const uint32_t cn = lane < tn ? s_cnt[lane] : 0u;
+    uint32_t co = cn;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t y = __shfl_up_sync(FULL, co, o);
+      if (lane >= o) co += y;
+    }
+    const uint32_t total = __shfl_sync(FULL, co, 31);
+    if (lane < tn) a.csr[node0 + lane] = co - cn;
+    s_cnt[lane] = 0u;  // for the next tile (read above by this lane only)
+    unsigned long long sgb = 0;
+    if (lane == 0) {
+      sgb = total ? atomicAdd(a.stash_top, (unsigned long long)total) : 0ull;
+      if (total && sgb + total > a.stash_cap) atomicOr(a.overflow_flag, 1u);
+      a.tile_total[cur] = total;
+      a.tile_seg[cur] = sgb;
+    }
+    sgb = __shfl_sync(FULL, sgb, 0);
+    // ---- emit (A6): items in order; lane writes its item's children at their final rank
+    uint64_t carry = sgb;
+    for (uint32_t R = 0; R < T; R += 32) {
+      const uint32_t k = R + lane;
+      int node, sg, b;
+      wtile_decode_item<HOT>(k < T ? k : T - 1, ie, s_items, nseg, vword_last, node, sg, b);
+      uint32_t m;
+      if (R == 0) m = km0;
+      else if (R == 32) m = km1;
+      else if (R == 64) m = km2;
+      else if (R == 96) m = km3;
+      else m = k < T ? wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q)
+                     : 0u;
+      const uint32_t pc = (uint32_t)__popc(m);
+      uint32_t incl = pc;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+      }
+      uint64_t rank = carry + (incl - pc);
+      carry += __shfl_sync(FULL, incl, 31);
+      if (m) {
+        uint32_t rec[W];
+#pragma unroll
+        for (int w = 0; w < W; w++) rec[w] = s_rec[node * W + w];
+        const uint32_t pos0 = (uint32_t)(sg * SEG + b * CPT);
+        while (m) {
+          const int c = __ffs(m) - 1;
+          m &= m - 1;
+          if (rank < a.stash_cap) {
+            uint32_t out[W];
+#pragma unroll
+            for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? (pos0 + c) << a.field_shift : 0u);
+            store_record<W>(a.stash + rank * W, out);
+          }
+          rank++;
+        }
+      }
+    }
+    __syncwarp();
+    cur = nxt;
+    nxt = nn;
+  }
+}
+
 template <typename K>
 static int launch_persistent(K k, const LevelArgs& a, int block, void* stream) {
   const int smem = a.smem_bytes;
@@ -735,9 +1044,53 @@ static int launch_wide_wc(const LevelArgs& a, void* stream) {
   }
 }
 
+// warp-tile levels: one wave of CTAs, never more warps than tiles
+template <typename K>
+static int launch_wtile_k(K k, const LevelArgs& a, void* stream) {
+  const int smem = a.smem_bytes;
+  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return (int)e;
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, a.block, smem);
+  if (e != cudaSuccess) return (int)e;
+  if (per_sm < 1) return (int)cudaErrorInvalidConfiguration;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const uint64_t nw = (uint64_t)(a.block / 32);
+  uint64_t grid = (uint64_t)sms * per_sm;
+  const uint64_t need = (a.n_tiles + nw - 1) / nw;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  k<<<(unsigned)grid, a.block, smem, (cudaStream_t)stream>>>(a);
+  return (int)cudaGetLastError();
+}
+
+template <int W, int CPT>
+static int launch_wtile_wc(const LevelArgs& a, void* stream) {
+  switch (a.hot) {
+    case HOT_NONE: return launch_wtile_k(expand_wtile<W, CPT, HOT_NONE>, a, stream);
+    case HOT_DIVX: return launch_wtile_k(expand_wtile<W, CPT, HOT_DIVX>, a, stream);
+    case HOT_MULX: return launch_wtile_k(expand_wtile<W, CPT, HOT_MULX>, a, stream);
+    default: return (int)cudaErrorInvalidValue;
+  }
+}
+
 template <int W>
 static int launch_w(const LevelArgs& a, void* stream) {
   if (a.kind == K_NARROW) return launch_persistent(expand_narrow<W>, a, a.block, stream);
+  if (a.kind == K_WTILE) {
+    switch (a.cpt) {
+      case 4: return launch_wtile_wc<W, 4>(a, stream);
+      case 8: return launch_wtile_wc<W, 8>(a, stream);
+      case 12: return launch_wtile_wc<W, 12>(a, stream);
+      case 16: return launch_wtile_wc<W, 16>(a, stream);
+      case 20: return launch_wtile_wc<W, 20>(a, stream);
+      case 24: return launch_wtile_wc<W, 24>(a, stream);
+      case 32: return launch_wtile_wc<W, 32>(a, stream);
+      default: return (int)cudaErrorInvalidValue;
+    }
+  }
   switch (a.cpt) {
     case 4: return launch_wide_wc<W, 4>(a, stream);
     case 8: return launch_wide_wc<W, 8>(a, stream);

@@ -1,6 +1,8 @@
 // kernels.cu — sm_100a kernels of the ATF search-space generator other than the level
 // expansion (expand.cuh): the batched decoder, the standalone
 // look-back scan used by the tests, and the shard offset fix-up.
+#include <algorithm>
+
 #include "dev_common.cuh"
 
 namespace atf {
@@ -22,11 +24,15 @@ int launch_expand(const LevelArgs& a, int words, void* stream) {
 
 int expand_smem_bytes(const LevelArgs& a, int words) { return expand_layout(a, words).total; }
 
-// ---------------------------------------------------------------- wide level, second half
-// Second half of a level (wide and narrow kernels alike): tile_base = exclusive scan of the tile totals (scan_kernel);
-// each tile's stash segment is copied to its final position and the tile's CSR entries
-// get the tile base added.  Grid-stride over tiles, one warp per tile; records move as
-// W-word vectors, 4 loads in flight per lane.
+// ---------------------------------------------------------------- level, second half
+// After the expand kernel (every kind): tile_base = exclusive scan of the tile totals
+// (scan_kernel, which also records piece_tile[p] = the tile holding output record
+// p << kPieceShift).  Then (1) every parent's tile-local CSR entry gets its tile's base
+// (grid-stride, coalesced) and (2) the level's records are copied from the tiles' stash
+// segments to their final positions in pieces of 2^kPieceShift output records, one warp
+// per piece (a piece may span several small tiles; a large tile spans many pieces), so
+// the copy is balanced whatever the tile sizes.  Records move as W-word vectors, 4 loads
+// in flight per lane.
 template <int W>
 struct RecVec;
 template <> struct RecVec<1> { using T = uint32_t; };
@@ -38,39 +44,48 @@ template <int W>
 __global__ void __launch_bounds__(256) level_emit_kernel(const __grid_constant__ LevelArgs a) {
   using V = typename RecVec<W>::T;
   constexpr int VPR = W == 8 ? 2 : 1;  // vectors per record
+  constexpr uint64_t P = 1ull << kPieceShift;
   const int lane = threadIdx.x & 31;
-  const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
-  for (uint64_t t = gw; t < a.n_tiles; t += nw) {
-    const uint64_t base = a.tile_base[t];
-    const uint64_t cnt = a.tile_total[t];
-    const uint64_t seg = a.tile_seg[t];
-    if (cnt) {
-      if (base + cnt > a.child_cap || seg + cnt > a.stash_cap) {
-        if (lane == 0) atomicOr(a.overflow_flag, 1u);
-      } else {
-        const V* __restrict__ src = reinterpret_cast<const V*>(a.stash + seg * W);
-        V* __restrict__ dst = reinterpret_cast<V*>(a.child_rec + base * W);
-        const uint64_t nv = cnt * VPR;
+  const uint64_t gt = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t nt = (uint64_t)gridDim.x * blockDim.x;
+  const uint64_t total = a.tile_base[a.n_tiles];
+  const bool over = total > a.child_cap || total > a.stash_cap;
+  if (gt == 0) {
+    if (over) atomicOr(a.overflow_flag, 1u);
+    *a.total_out = total;
+    a.csr[a.n_parents] = total;
+  }
+  // (1) CSR fix-up
+  if (a.n_chunks == 1) {
+    const uint64_t tn = (uint64_t)a.tile_nodes;
+    for (uint64_t n = gt; n < a.n_parents; n += nt) a.csr[n] += a.tile_base[n / tn];
+  } else {
+    for (uint64_t n = gt; n < a.n_parents; n += nt) a.csr[n] += a.tile_base[n * (uint64_t)a.n_chunks];
+  }
+  if (over) return;
+  // (2) pieces
+  const uint64_t gw = gt >> 5, nw = nt >> 5;
+  const uint64_t n_pieces = (total + P - 1) >> kPieceShift;
+  for (uint64_t p = gw; p < n_pieces; p += nw) {
+    uint64_t o = p << kPieceShift;
+    const uint64_t o_end = min(o + P, total);
+    uint64_t t = a.piece_tile[p];
+    while (o < o_end) {
+      const uint64_t base = a.tile_base[t], cnt = a.tile_total[t];
+      const uint64_t e = min(o_end, base + cnt);
+      if (e > o) {
+        const V* __restrict__ src = reinterpret_cast<const V*>(a.stash + (a.tile_seg[t] + (o - base)) * W);
+        V* __restrict__ dst = reinterpret_cast<V*>(a.child_rec + o * W);
+        const uint64_t nv = (e - o) * VPR;
         uint64_t k = lane;
         for (; k + 96 < nv; k += 128) {
           const V v0 = __ldcs(src + k), v1 = __ldcs(src + k + 32), v2 = __ldcs(src + k + 64), v3 = __ldcs(src + k + 96);
           dst[k] = v0; dst[k + 32] = v1; dst[k + 64] = v2; dst[k + 96] = v3;
         }
         for (; k < nv; k += 32) dst[k] = __ldcs(src + k);
+        o = e;
       }
-    }
-    if (a.n_chunks == 1) {
-      const uint64_t n0 = t * (uint64_t)a.tile_nodes;
-      const uint64_t n1 = min(n0 + (uint64_t)a.tile_nodes, a.n_parents);
-      for (uint64_t n = n0 + lane; n < n1; n += 32) a.csr[n] += base;
-    } else if (lane == 0 && umod64f(t, (uint64_t)a.n_chunks) == 0) {
-      a.csr[udiv64f(t, (uint64_t)a.n_chunks)] += base;
-    }
-    if (t == a.n_tiles - 1 && lane == 0) {
-      const uint64_t total = a.tile_base[a.n_tiles];
-      *a.total_out = total;
-      a.csr[a.n_parents] = total;
+      t++;
     }
   }
 }
@@ -80,9 +95,13 @@ int launch_level_emit(const LevelArgs& a, int words, void* stream) {
   int dev = 0, sms = 0;
   cudaGetDevice(&dev);
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  uint64_t blocks = (a.n_tiles + 7) / 8;  // 8 warps (tiles) per block
-  const uint64_t cap = (uint64_t)sms * 16;
+  // enough warps for the larger of the parents (CSR) and the records (pieces); the
+  // record count is only known on the device, so the grid covers the stash capacity
+  const uint64_t pieces = (a.stash_cap >> kPieceShift) + 1;
+  uint64_t blocks = std::max<uint64_t>((a.n_parents + 255) / 256, (pieces + 7) / 8);
+  const uint64_t cap = (uint64_t)sms * 8;
   if (blocks > cap) blocks = cap;
+  if (blocks < 1) blocks = 1;
   cudaStream_t st = (cudaStream_t)stream;
   switch (words) {
     case 1: level_emit_kernel<1><<<(unsigned)blocks, 256, 0, st>>>(a); break;
@@ -184,7 +203,8 @@ int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n,
 // ---------------------------------------------------------------- standalone scan (tests)
 // Exclusive scan u32 -> u64 with the same look-back as expand_kernel; out[n] = total.
 __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restrict__ out, int64_t n,
-                            unsigned long long* status, unsigned int* counter, uint64_t n_tiles) {
+                            unsigned long long* status, unsigned int* counter, uint64_t n_tiles,
+                            uint32_t* __restrict__ piece_tile, uint64_t piece_cap) {
   __shared__ uint32_t s_tile;
   __shared__ unsigned long long s_wt[33];
   __shared__ unsigned long long s_base;
@@ -226,7 +246,14 @@ __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restric
     __syncthreads();
     unsigned long long run = s_base + s_wt[warp] + incl - sum;
     for (int q = 0; q < ITEMS; q++) {
-      if (i0 + q < n) out[i0 + q] = run;
+      if (i0 + q < n) {
+        out[i0 + q] = run;
+        if (piece_tile && v[q]) {  // pieces whose first record lies in element i0 + q
+          constexpr uint64_t P = 1ull << kPieceShift;
+          for (uint64_t p = (run + P - 1) >> kPieceShift; (p << kPieceShift) < run + v[q] && p < piece_cap; p++)
+            piece_tile[p] = (uint32_t)(i0 + q);
+        }
+      }
       run += v[q];
     }
     __syncthreads();
@@ -234,7 +261,7 @@ __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restric
 }
 
 int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long long* status, unsigned int* counter,
-                    void* stream) {
+                    void* stream, uint32_t* piece_tile, uint64_t piece_cap) {
   const int B = 256;
   const uint64_t n_tiles = n > 0 ? (uint64_t)((n + B * 4 - 1) / (B * 4)) : 1;
   int dev = 0, sms = 0;
@@ -242,7 +269,7 @@ int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long 
   cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   uint64_t grid = (uint64_t)sms * 4;
   if (grid > n_tiles) grid = n_tiles;
-  scan_kernel<<<(unsigned)grid, B, 0, (cudaStream_t)stream>>>(in, out, n, status, counter, n_tiles);
+  scan_kernel<<<(unsigned)grid, B, 0, (cudaStream_t)stream>>>(in, out, n, status, counter, n_tiles, piece_tile, piece_cap);
   return (int)cudaGetLastError();
 }
 

@@ -52,9 +52,10 @@ def torch_rowhash(rows_pm: "torch.Tensor", base: int = 0) -> int:
     return int(s.item()) & ((1 << 64) - 1)
 
 
-def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000):
+def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, legacy=False):
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
     ref = orc.info(spec, threads=8)
-    with Space(spec, flags=_flags(generic)) as sp:
+    with Space(spec, flags=_flags(generic) | (L.ATF_FLAG_LEGACY_WIDE if legacy else 0)) as sp:
         sp.generate()
         assert sp.groups() == [g["members"] for g in ref["groups"]]
         assert sp.size() == int(ref["S"])
@@ -87,6 +88,8 @@ SMALL = {
     "C3-IS4-anch": lambda: A.c3_xgemm("IS4", anchored=True),
     "C5-60x5": lambda: A.c5_chains(60, 5),
     "C5-300x4": lambda: A.c5_chains(300, 4),
+    # full-width ranges: nodes with 4096 children (y-chain value 1), heavy first tiles
+    "C5-4096x3": lambda: A.c5_chains(4096, 3),
 }
 
 
@@ -111,6 +114,17 @@ def test_fuzz_wide_specs(Space, seed):
     """Ranges of 65..6000 values (the wide kernel: hot filters x|n, d|x, (a x)|n, generic
     conjuncts, chunked ranges > 4096, zero and negative candidates) vs the oracle."""
     _check_against_oracle(Space, A.random_wide_spec(seed))
+
+
+@pytest.mark.parametrize("seed", range(0, 40, 3))
+def test_fuzz_wide_specs_legacy_kernel(Space, seed):
+    """The block-tile wide kernel (ATF_FLAG_LEGACY_WIDE) on the same specs."""
+    _check_against_oracle(Space, A.random_wide_spec(seed), legacy=True)
+
+
+@pytest.mark.parametrize("name", ["C3-IS1", "C5-300x4", "C5-4096x3", "C2-256"])
+def test_small_specs_legacy_kernel(Space, name):
+    _check_against_oracle(Space, SMALL[name](), legacy=True)
 
 
 @pytest.mark.parametrize("seed", range(0, 40, 5))

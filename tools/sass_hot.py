@@ -8,7 +8,7 @@ obj = sys.argv[1]
 sass = subprocess.run(["cuobjdump", "-sass", obj], capture_output=True, text=True).stdout
 for f in re.split(r"\n\s*Function : ", sass)[1:]:
     name = f.split("\n", 1)[0].strip()
-    if "expand_wide" not in name:
+    if "expand_wide" not in name and "expand_wtile" not in name:
         continue
     L = [re.sub(r"/\* 0x[0-9a-f]+ \*/", "", l) for l in f.split("\n") if l.strip().startswith("/*")]
     # densest window of VIMNMX3 = the unrolled body
