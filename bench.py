@@ -134,13 +134,15 @@ def run_generation(spec, steps, warmup, dist_ctx=None, timing=True):
         dist_ctx["dist"].barrier()
     torch.cuda.synchronize()
     evs = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
-    level_ms = []
+    level_ms, level_exp_ms = [], []
     for i in range(steps):
         evs[i][0].record(stream)
         one_step()
         evs[i][1].record(stream)
         if timing:
-            level_ms.append([s["ms"] for s in sp.stats()])
+            sts = sp.stats()
+            level_ms.append([s["ms"] for s in sts])
+            level_exp_ms.append([s["expand_ms"] for s in sts])
         flush_l2(flush)
     torch.cuda.synchronize()
     if dist_ctx:
@@ -149,26 +151,56 @@ def run_generation(spec, steps, warmup, dist_ctx=None, timing=True):
     ms = [a.elapsed_time(b) for a, b in evs]
     st = sp.stats()
     res = {"ms": ms, "stats": st, "size": sp.size(), "group_sizes": sp.group_sizes(),
-           "plan": sp.plan_json(), "level_ms": level_ms}
+           "plan": sp.plan_json(), "level_ms": level_ms, "level_exp_ms": level_exp_ms}
     sp.close()
     return res
 
 
-def roofline_of(res, sm_mhz):
-    """Dominant kernels = the level expansion (expand_wide + scan + wide_emit, expand_narrow; every
-    launch of the step).  achieved = algorithmic int ops (evals_k x c_k, DESIGN.md cost table) /
-    summed device time of the levels (CUDA events on the launch stream around each level)."""
+def _traffic_db():
+    """ncu-measured DRAM bytes per launch (dram__bytes_read.sum + dram__bytes_write.sum from one
+    `ncu --set full` capture), keyed "spec:g<group>:l<level>"; written by tools/traffic_db.py
+    from the committed profiles/ captures."""
+    try:
+        with open(os.path.join(ROOT, "profiles", "traffic.json")) as f:
+            return json.load(f)
+    except OSError:
+        return {}
+
+
+def roofline_of(res, sm_mhz, spec_name=None):
+    """Roofline of the dominant kernel: the level-expansion launch with the largest
+    device time.  achieved = its algorithmic integer ops (evals_k x c_k, the planner's cost table)
+    / its average launch duration (CUDA events around the expand kernel alone, on the launch
+    stream); peak = 4 SMSP x 32 lanes x SMs x clock (bound "alu").  "step" aggregates every
+    launch of a generation (expand + scan + emit of every level)."""
     plan = res["plan"]
-    costs = [lv["cost"] for g in plan["groups"] for lv in g["levels"]]
-    ops = sum(s["evals"] * c for s, c in zip(res["stats"], costs))
-    lm = np.array(res["level_ms"], dtype=np.float64)  # [steps, levels]
-    kern_ms = float(lm.sum(axis=1).mean()) if lm.size else float("nan")
-    achieved = ops / (kern_ms * 1e-3)
+    lv = [(gi, k, l) for gi, g in enumerate(plan["groups"]) for k, l in enumerate(g["levels"])]
+    costs = [l["cost"] for _, _, l in lv]
+    st = res["stats"]
+    ops = [s["evals"] * c for s, c in zip(st, costs)]
+    exp_ms = np.array(res["level_exp_ms"], dtype=np.float64).mean(axis=0)
+    lvl_ms = np.array(res["level_ms"], dtype=np.float64).mean(axis=0)
+    d = int(np.argmax(exp_ms))
+    g, k, _ = lv[d]
     peak = int_peak_ops(sm_mhz)
+    achieved = ops[d] / (exp_ms[d] * 1e-3)
+    W = plan["groups"][g].get("words", 4)
+    f_prev = st[d]["evals"] // max(1, st[d]["r"])
+    alg_bytes = f_prev * W * 4 + st[d]["f"] * W * 4 + (f_prev + 1) * 8
+    tdb = _traffic_db()
+    tr = tdb.get(f"{spec_name}:g{g}:l{k}") if spec_name else None
+    kname = {0: "expand_narrow", 1: "expand_wide", 2: "expand_wtile"}.get(st[d].get("kernel", -1), "expand")
+    step_ops = float(sum(ops))
+    step_ms = float(lvl_ms.sum())
     return {"bound": "alu", "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tops/s",
-            "frac": achieved / peak, "traffic": None, "ops_per_step": ops, "kernel_ms": kern_ms,
-            "peak_clock_mhz": sm_mhz,
-            "cost_table": "DIVX/MULX/DIVPROD 2, QDIV 6, CMP 2, AND 1, GENERIC = bytecode ops"}
+            "frac": achieved / peak, "traffic": tr["dram_bytes"] if tr else None,
+            "traffic_source": tr["source"] if tr else None,
+            "kernel": kname, "launch": f"group {g} level {k + 1} (r={st[d]['r']}, evals={st[d]['evals']})",
+            "ops_per_launch": ops[d], "launch_ms": float(exp_ms[d]), "algorithmic_bytes_per_launch": int(alg_bytes),
+            "peak_clock_mhz": sm_mhz, "peak_source": "4 SMSP x 32 lanes x 148 SMs x clock (B200_PROFILING.md unit counts)",
+            "cost_table": "DIVX/MULX/DIVPROD 2, QDIV 6, CMP 2, AND 1, GENERIC = bytecode ops",
+            "step": {"ops": step_ops, "ms": step_ms, "achieved": step_ops / (step_ms * 1e-3) / 1e12,
+                     "frac": step_ops / (step_ms * 1e-3) / peak}}
 
 
 def e2e_generation(spec, steps):
@@ -209,10 +241,11 @@ def secondary_n1(steps, warmup, sm_mhz):
         ms = float(np.mean(res["ms"]))
         leaves = sum(res["group_sizes"])
         evals = sum(s["evals"] for s in res["stats"])
-        rf = roofline_of(res, sm_mhz)
+        rf = roofline_of(res, sm_mhz, mk().name)
         out[name] = {"ms_per_step": ms, "configs_per_s": leaves / (ms * 1e-3), "evals_per_s": evals / (ms * 1e-3),
                      "S": str(res["size"]), "group_leaves": leaves, "evals": evals,
-                     "roofline_frac": rf["frac"], "kernel_ms": rf["kernel_ms"],
+                     "roofline_frac_step": rf["step"]["frac"], "dominant_launch": rf["launch"],
+                     "dominant_frac": rf["frac"], "kernel_ms": rf["step"]["ms"],
                      "level_ms": [round(x, 4) for x in np.mean(res["level_ms"], axis=0).tolist()]}
     # C4: decode 10^8 random indices into C3-IS2
     from atfspec.fuzz import splitmix64_indices
@@ -318,11 +351,6 @@ def main():
         ms = float(t.item())
     leaves = sum(res["group_sizes"])                      # global (finalize_shard) sizes
     plan = res["plan"]
-    evals_total = 0
-    for g in plan["groups"]:
-        pass
-    # algorithmic evals of the whole job: from the single-GPU level sizes (f_{k-1} r_k)
-    gl = [[lv["r"] for lv in g["levels"]] for g in plan["groups"]]
     value = leaves / (ms * 1e-3)
     # our kernels per step: every non-empty level launches expand_narrow (r <= 64) or
     # expand_wide, then scan_kernel and level_emit_kernel
@@ -337,8 +365,8 @@ def main():
         if world == 1:
             evals_total = sum(s["evals"] for s in res["stats"])
             line["evals_per_s"] = evals_total / (ms * 1e-3)
-            line["roofline"] = roofline_of(res, sm_max)
-            line["roofline_at_load_clock"] = (roofline_of(res, clocks["sm_mhz"])["frac"]
+            line["roofline"] = roofline_of(res, sm_max, spec.name)
+            line["roofline_at_load_clock"] = (roofline_of(res, clocks["sm_mhz"], spec.name)["frac"]
                                               if clocks.get("sm_mhz") else None)
             e2e = e2e_generation(spec, max(2, a.steps // 2))
             line["e2e"] = {"value": leaves / e2e["s_per_step"], "unit": "configs/s",

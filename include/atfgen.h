@@ -225,6 +225,8 @@ typedef struct {
   uint64_t f;       /* nodes f_k                              */
   float ms;         /* device time of the level (ATF_FLAG_TIMING), else -1 */
   int32_t path;     /* 0 = fast atoms, 1 = generic interpreter */
+  float expand_ms;  /* device time of the level's expand kernel alone (ATF_FLAG_TIMING), else -1 */
+  int32_t kernel;   /* expand kernel: 0 = narrow (r <= 64), 1 = block-tile wide, 2 = warp-tile wide */
 } atf_level_stats;
 atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap, int32_t* n_out);
 

@@ -84,7 +84,9 @@ struct LevelData {
   uint64_t n = 0;
   uint64_t offset = 0;      // global index of rec[0] (shards)
   uint64_t evals = 0;
-  float ms = -1.f;
+  float ms = -1.f;         // expand + scan + emit of the level (ATF_FLAG_TIMING)
+  float expand_ms = -1.f;  // the expand kernel alone
+  int32_t kernel = -1;     // KernelKind of the expand launch
 };
 
 }  // namespace
@@ -116,7 +118,8 @@ struct atf_space {
   uint32_t* d_root = nullptr;            // 8 zero words
   unsigned long long* h_totals = nullptr;  // pinned
   unsigned int* h_flags = nullptr;         // pinned
-  std::vector<std::vector<std::pair<cudaEvent_t, cudaEvent_t>>> events;
+  struct EvTriple { cudaEvent_t first = nullptr, mid = nullptr, second = nullptr; };
+  std::vector<std::vector<EvTriple>> events;
   // shards
   int shard_rank = 0, shard_world = 1;
   std::vector<int> shard_cut;  // per group: first level expanded on a slice (L = none)
@@ -914,6 +917,7 @@ static void release_device(atf_space* s) {
   for (auto& ev : s->events)
     for (auto& e : ev) {
       cudaEventDestroy(e.first);
+      cudaEventDestroy(e.mid);
       cudaEventDestroy(e.second);
     }
   s->events.clear();
@@ -1043,6 +1047,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].first, st));
   int ce = launch_expand(a, gp.words, st);
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].mid, st));
+  s->data[g][k].kernel = a.kind;
   {
     ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st, piece_tile, piece_cap);
     if (!ce) ce = launch_level_emit(a, gp.words, st);
@@ -1116,7 +1122,10 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       d.evals = pd.n_parents * (uint64_t)gp.levels[pd.k].r;
       if (pd.k > 0) s->data[pd.g][pd.k - 1].csr = pd.csr;
       if (s->opts.flags & ATF_FLAG_TIMING)
+      {
         cudaEventElapsedTime(&d.ms, s->events[pd.g][pd.k].first, s->events[pd.g][pd.k].second);
+        cudaEventElapsedTime(&d.expand_ms, s->events[pd.g][pd.k].first, s->events[pd.g][pd.k].mid);
+      }
       frontier[i] = pd.child;
       fsize[i] = total;
       k[i]++;
@@ -1142,6 +1151,7 @@ static atf_status generate_impl(atf_space* s) {
         s->events[g].resize(s->groups[g].levels.size());
         for (auto& ev : s->events[g]) {
           CUDA_TRY(s, cudaEventCreate(&ev.first));
+          CUDA_TRY(s, cudaEventCreate(&ev.mid));
           CUDA_TRY(s, cudaEventCreate(&ev.second));
         }
       }
@@ -1511,6 +1521,8 @@ atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap
         o.f = d.n;
         o.ms = d.ms;
         o.path = lp.generic ? 1 : 0;
+        o.expand_ms = d.expand_ms;
+        o.kernel = d.kernel;
       }
       n++;
     }

@@ -935,7 +935,8 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
     const uint32_t T = __shfl_sync(FULL, ie, 31);
     ie -= ic;
     // pass 1: exact masks -> node counts; the first 4 rounds keep their masks in registers
-    uint32_t km0 = 0, km1 = 0, km2 = 0, km3 = 0;
+    // (mask, item code = node | seg << 5 | lane << 8)
+    uint32_t km0 = 0, km1 = 0, km2 = 0, km3 = 0, kc0 = 0, kc1 = 0, kc2 = 0, kc3 = 0;
     for (uint32_t R = 0; R < T; R += 32) {
       const uint32_t k = R + lane;
       int node, sg, b;
@@ -943,10 +944,11 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
       uint32_t m = 0;
       if (k < T)
         m = wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q);
-      if (R == 0) km0 = m;
-      else if (R == 32) km1 = m;
-      else if (R == 64) km2 = m;
-      else if (R == 96) km3 = m;
+      const uint32_t code = (uint32_t)node | ((uint32_t)sg << 5) | ((uint32_t)b << 8);
+      if (R == 0) { km0 = m; kc0 = code; }
+      else if (R == 32) { km1 = m; kc1 = code; }
+      else if (R == 64) { km2 = m; kc2 = code; }
+      else if (R == 96) { km3 = m; kc3 = code; }
       if (m) atomicAdd(&s_cnt[node], (uint32_t)__popc(m));
     }
     __syncwarp();
@@ -974,14 +976,18 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
     for (uint32_t R = 0; R < T; R += 32) {
       const uint32_t k = R + lane;
       int node, sg, b;
-      wtile_decode_item<HOT>(k < T ? k : T - 1, ie, s_items, nseg, vword_last, node, sg, b);
       uint32_t m;
-      if (R == 0) m = km0;
-      else if (R == 32) m = km1;
-      else if (R == 64) m = km2;
-      else if (R == 96) m = km3;
-      else m = k < T ? wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q)
-                     : 0u;
+      if (R < 128) {
+        const uint32_t code = R == 0 ? kc0 : R == 32 ? kc1 : R == 64 ? kc2 : kc3;
+        m = R == 0 ? km0 : R == 32 ? km1 : R == 64 ? km2 : km3;
+        node = (int)(code & 31u);
+        sg = (int)((code >> 5) & 7u);
+        b = (int)(code >> 8);
+      } else {
+        wtile_decode_item<HOT>(k < T ? k : T - 1, ie, s_items, nseg, vword_last, node, sg, b);
+        m = k < T ? wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q)
+                  : 0u;
+      }
       const uint32_t pc = (uint32_t)__popc(m);
       uint32_t incl = pc;
 #pragma unroll

@@ -58,34 +58,65 @@ __global__ void __launch_bounds__(256) level_emit_kernel(const __grid_constant__
   // (1) CSR fix-up
   if (a.n_chunks == 1) {
     const uint64_t tn = (uint64_t)a.tile_nodes;
-    for (uint64_t n = gt; n < a.n_parents; n += nt) a.csr[n] += a.tile_base[n / tn];
+    if ((tn & (tn - 1)) == 0) {
+      const int sh = __ffsll((long long)tn) - 1;
+      for (uint64_t n = gt; n < a.n_parents; n += nt) a.csr[n] += a.tile_base[n >> sh];
+    } else {
+      for (uint64_t n = gt; n < a.n_parents; n += nt) a.csr[n] += a.tile_base[udiv64f(n, tn)];
+    }
   } else {
     for (uint64_t n = gt; n < a.n_parents; n += nt) a.csr[n] += a.tile_base[n * (uint64_t)a.n_chunks];
   }
   if (over) return;
-  // (2) pieces
+  // (2) pieces.  A window of 32 consecutive tiles (lane j holds tile t0 + j's base, count
+  // and stash segment); each output record finds its tile by a 5-step shuffle search of
+  // the window; 4 records per lane in flight.
   const uint64_t gw = gt >> 5, nw = nt >> 5;
   const uint64_t n_pieces = (total + P - 1) >> kPieceShift;
   for (uint64_t p = gw; p < n_pieces; p += nw) {
     uint64_t o = p << kPieceShift;
     const uint64_t o_end = min(o + P, total);
-    uint64_t t = a.piece_tile[p];
+    uint64_t t0 = a.piece_tile[p];
     while (o < o_end) {
-      const uint64_t base = a.tile_base[t], cnt = a.tile_total[t];
-      const uint64_t e = min(o_end, base + cnt);
-      if (e > o) {
-        const V* __restrict__ src = reinterpret_cast<const V*>(a.stash + (a.tile_seg[t] + (o - base)) * W);
-        V* __restrict__ dst = reinterpret_cast<V*>(a.child_rec + o * W);
-        const uint64_t nv = (e - o) * VPR;
-        uint64_t k = lane;
-        for (; k + 96 < nv; k += 128) {
-          const V v0 = __ldcs(src + k), v1 = __ldcs(src + k + 32), v2 = __ldcs(src + k + 64), v3 = __ldcs(src + k + 96);
-          dst[k] = v0; dst[k + 32] = v1; dst[k + 64] = v2; dst[k + 96] = v3;
+      const uint64_t tt = t0 + lane;
+      const bool tv = tt < a.n_tiles;
+      const uint64_t bj = tv ? a.tile_base[tt] : ~0ull;
+      const uint64_t ej = tv ? bj + a.tile_total[tt] : ~0ull;
+      const uint64_t sj = tv ? a.tile_seg[tt] : 0ull;
+      // records of this window: [o, lim)
+      const uint64_t e31 = __shfl_sync(FULL, ej, 31);
+      const uint64_t lim = min(o_end, e31);
+      for (uint64_t ob = o; ob < lim; ob += 128) {
+        V v[4][VPR];
+        uint64_t dsto[4];
+#pragma unroll
+        for (int u = 0; u < 4; u++) {
+          const uint64_t oo = ob + (uint64_t)u * 32 + lane;
+          int j = 0;
+#pragma unroll
+          for (int s = 16; s > 0; s >>= 1) {
+            const uint64_t bb = __shfl_sync(FULL, bj, j + s);
+            if (bb <= oo) j += s;
+          }
+          const uint64_t bsel = __shfl_sync(FULL, bj, j), ssel = __shfl_sync(FULL, sj, j);
+          dsto[u] = oo;
+          if (oo < lim) {
+            const V* src = reinterpret_cast<const V*>(a.stash + (ssel + (oo - bsel)) * W);
+#pragma unroll
+            for (int q = 0; q < VPR; q++) v[u][q] = __ldcs(src + q);
+          }
         }
-        for (; k < nv; k += 32) dst[k] = __ldcs(src + k);
-        o = e;
+#pragma unroll
+        for (int u = 0; u < 4; u++)
+          if (dsto[u] < lim) {
+            V* dst = reinterpret_cast<V*>(a.child_rec + dsto[u] * W);
+#pragma unroll
+            for (int q = 0; q < VPR; q++) dst[q] = v[u][q];
+          }
       }
-      t++;
+      o = lim;
+      t0 += 31;  // tile t0 + 31 holds record lim - 1 (or the window ended inside it)
+      while (o < o_end && a.tile_base[t0] + a.tile_total[t0] <= o) t0++;
     }
   }
 }
