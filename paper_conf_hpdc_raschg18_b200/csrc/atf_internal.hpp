@@ -44,6 +44,15 @@ struct Term {
   int32_t use_qtable;          // T_QDIV V16: divisibility magic of the quotient from smem
 };
 
+// Operand of a term on the narrow fast path (expand_nfast): an ancestor value, a constant
+// or the product of two ancestor values, read straight from the parent record.
+enum NfKind : int16_t { NF_PV = 0, NF_CONST = 1, NF_PROD = 2 };
+struct NfOp {
+  int16_t kind, s1, s2, pad;
+  int32_t c;     // NF_CONST value
+  uint32_t cm;   // NF_CONST: ceil(2^32/|c|) mod 2^32 (divisor magic)
+};
+
 // Per-level program + geometry, passed by value to the expand kernel.
 struct LevelArgs {
   // frontier = level k-1 of this group (k == 0: a single empty root record)
@@ -69,6 +78,11 @@ struct LevelArgs {
   int32_t n_terms;
   Term terms[kMaxTerms];
   int32_t need_slots_smem;  // a generic term reads slots per candidate
+  void* masks;              // nfast: per-parent accept masks (pass 1 -> pass 2)
+  int32_t mask_bytes;       // 1, 2 or 4
+  int32_t nf_ok;            // narrow fast path possible (no gates / generic terms / wide variants)
+  NfOp nf_op[kMaxTerms][2];
+  const uint32_t* pv_magic[kMaxSlots];  // divisor magics of each ancestor's range
   int32_t need_m64;         // some term needs the 64-bit candidate magic
   int32_t code[kMaxCode];
   // outputs
@@ -103,7 +117,8 @@ struct LevelArgs {
   uint32_t qmax;            // T_QDIV table covers quotients [0, qmax]
   int32_t smem_bytes;
 };
-enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1, K_WTILE = 2 };
+enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1, K_WTILE = 2, K_NFAST = 3 };
+constexpr int kNfNPL = 4;  // narrow fast kernel: frontier nodes per lane (warp tile = 128 nodes)
 constexpr int kWT = 32;        // warp-tile kernel: frontier nodes per warp tile (one per lane)
 constexpr int kMaxSeg = 8;     // warp-tile kernel: candidate segments per node
 constexpr int kPieceShift = 10;  // level_emit_kernel copies the level in pieces of 2^10 records
@@ -206,6 +221,7 @@ ATF_HD WarpLayout wtile_layout(const LevelArgs& a, int words) {
 int launch_expand(const LevelArgs& a, int words, void* stream);
 int expand_smem_bytes(const LevelArgs& a, int words);
 int launch_level_emit(const LevelArgs& a, int words, void* stream);
+int launch_nfast_emit(const LevelArgs& a, int words, void* stream);
 int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out,
                           int64_t ld, unsigned int* bad_flag, void* stream);
 int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,

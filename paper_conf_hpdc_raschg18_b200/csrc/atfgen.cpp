@@ -106,6 +106,8 @@ struct atf_space {
   std::vector<uint64_t> gsize;
   unsigned long long* d_status = nullptr;
   size_t status_cap = 0;
+  char* d_masks = nullptr;  // nfast accept masks
+  size_t masks_cap = 0;
   uint64_t stash_hint = 0;     // records: exact size of the last level that overflowed
   char* d_scratch = nullptr;   // wide levels: per-tile totals, segments, bases, scan state
   size_t scratch_cap = 0;
@@ -623,6 +625,46 @@ static atf_status compile_level(const std::vector<ParamDef>& P, int p, const std
   a.n_slots = lc.n_slots;
   if (lc.code.size() > (size_t)kMaxCode) { *why = "level program too long"; return ATF_ERR_LIMIT; }
   std::copy(lc.code.begin(), lc.code.end(), a.code);
+  // narrow fast path (expand_nfast): no gates, every conjunct a 16-bit divisibility atom or a
+  // 32-bit comparison whose operands are ancestor values, constants or ancestor products
+  {
+    auto opdesc = [&](int slot, NfOp& o) -> bool {
+      o = NfOp{};
+      if (slot < 0) return false;
+      if (slot < a.n_pv) { o.kind = NF_PV; o.s1 = (int16_t)slot; return true; }
+      const int32_t* c = a.code + a.inv_off[slot];
+      const int len = a.inv_len[slot];
+      if (len == 3 && c[0] == ATF_OP_CONST) {
+        const int64_t v = (int64_t)(((uint64_t)(uint32_t)c[2] << 32) | (uint32_t)c[1]);
+        if (v < INT32_MIN || v > INT32_MAX) return false;
+        o.kind = NF_CONST;
+        o.c = (int32_t)v;
+        const uint32_t av = v < 0 ? 0u - (uint32_t)v : (uint32_t)v;
+        o.cm = av > 1 ? 0xffffffffu / av + 1u : 0u;
+        return true;
+      }
+      if (len == 5 && c[0] == OP_SLOT && c[2] == OP_SLOT && c[4] == ATF_OP_MUL && c[1] < a.n_pv && c[3] < a.n_pv) {
+        o.kind = NF_PROD;
+        o.s1 = (int16_t)c[1];
+        o.s2 = (int16_t)c[3];
+        return true;
+      }
+      return false;
+    };
+    bool ok = a.n_gates == 0 && !lp.generic;
+    for (int t = 0; ok && t < a.n_terms; t++) {
+      const Term& T = a.terms[t];
+      switch (T.kind) {
+        case T_DIVX: case T_MULX: ok = T.variant == V16 && opdesc(T.slot_a, a.nf_op[t][0]); break;
+        case T_DIVPROD: case T_QDIV:
+          ok = T.variant == V16 && !T.use_qtable && opdesc(T.slot_a, a.nf_op[t][0]) && opdesc(T.slot_b, a.nf_op[t][1]);
+          break;
+        case T_CMP: ok = T.variant == V32 && opdesc(T.slot_a, a.nf_op[t][0]) && opdesc(T.slot_b, a.nf_op[t][1]); break;
+        default: ok = false;
+      }
+    }
+    a.nf_ok = ok ? 1 : 0;
+  }
   lp.desc = d.empty() ? "TRUE" : d;
   return ATF_OK;
 }
@@ -748,6 +790,15 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
       a.smem_bytes = wtile_layout(a, words).total;
       return;
     }
+  }
+  if (r <= 32 && a.nf_ok && !legacy_wide) {
+    a.kind = K_NFAST;
+    a.block = 256;
+    a.cpt = 1;
+    a.tile_nodes = 32 * kNfNPL;
+    a.chunk = r;
+    a.smem_bytes = 0;
+    return;
   }
   if (r <= 64) {
     a.kind = K_NARROW;
@@ -904,6 +955,9 @@ static void release_device(atf_space* s) {
   dfree(s, s->d_status, s->status_cap * 8);
   dfree(s, s->d_scratch, s->scratch_cap);
   dfree(s, (char*)s->d_stash, s->stash_cap);
+  dfree(s, s->d_masks, s->masks_cap);
+  s->d_masks = nullptr;
+  s->masks_cap = 0;
   s->d_scratch = nullptr;
   s->d_stash = nullptr;
   s->scratch_cap = s->stash_cap = 0;
@@ -957,7 +1011,12 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     a.cand_abs = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + 2 * rp;
   }
   a.r = lp.r;
-  for (int i = 0; i < a.n_pv; i++) a.pv_range[i] = s->d_range[lp.pv_param[i]];
+  for (int i = 0; i < a.n_pv; i++) {
+    a.pv_range[i] = s->d_range[lp.pv_param[i]];
+    // see ensure_device: [values rp][magic rp][abs rp]
+    const size_t rpi = (s->params[lp.pv_param[i]].values.size() + 127) / 128 * 128;
+    a.pv_magic[i] = reinterpret_cast<const uint32_t*>(s->d_range[lp.pv_param[i]]) + rpi;
+  }
   choose_geometry(a, gp.words, (s->opts.flags & ATF_FLAG_LEGACY_WIDE) != 0);
   a.n_tiles = a.n_chunks > 1 ? n_parents * (uint64_t)a.n_chunks
                              : (n_parents + (uint64_t)a.tile_nodes - 1) / (uint64_t)a.tile_nodes;
@@ -1041,6 +1100,13 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     a.piece_tile = piece_tile;
     CUDA_TRY(s, cudaMemsetAsync(s->d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
   }
+  // narrow fast levels: pass 1 writes per-parent accept masks, pass 2 the children in place
+  if (a.kind == K_NFAST) {
+    a.mask_bytes = a.r <= 8 ? 1 : (a.r <= 16 ? 2 : 4);
+    if ((e = ensure_buf(s, &s->d_masks, &s->masks_cap, (size_t)n_parents * a.mask_bytes + 16, "accept masks")))
+      return e;
+    a.masks = s->d_masks;
+  }
   CUDA_TRY(s, cudaMemsetAsync(s->d_counter + g, 0, 4, st));
   CUDA_TRY(s, cudaMemsetAsync(s->d_ovf + g, 0, 4, st));
   bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
@@ -1049,7 +1115,11 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].mid, st));
   s->data[g][k].kernel = a.kind;
-  {
+  if (a.kind == K_NFAST) {
+    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st);
+    if (!ce) ce = launch_nfast_emit(a, gp.words, st);
+    if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
+  } else {
     ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st, piece_tile, piece_cap);
     if (!ce) ce = launch_level_emit(a, gp.words, st);
     if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));

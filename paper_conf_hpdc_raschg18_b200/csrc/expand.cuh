@@ -1050,6 +1050,251 @@ static int launch_wide_wc(const LevelArgs& a, void* stream) {
   }
 }
 
+// ---------------------------------------------------------------- narrow fast kernel
+// r <= 32 candidates and a level whose conjuncts are all 16/32-bit atoms over ancestor
+// values, constants or products of two ancestors (host: nf_ok; every C1-C3 narrow level).
+// Warp-autonomous tiles of 32 x kNfNPL frontier nodes (lane l: nodes l, l+32, ...); per
+// node the operands come straight from the parent record (field -> range value, and the
+// range's divisor magic where a quotient or a d | x test needs one: no division, no
+// per-node slot array), each conjunct is a bit-parallel mask over the r candidates
+// (candidate values / magics in shared memory), children are written by their node's
+// lane in candidate order into the tile's stash segment.  No block barrier after staging.
+template <int W>
+__device__ __forceinline__ uint32_t nf_field(const LevelArgs& a, const uint32_t* rec, int s) {
+  uint32_t word = rec[0];
+#pragma unroll
+  for (int w = 1; w < W; w++)
+    if (a.pv_word[s] == w) word = rec[w];
+  const uint32_t bits = (uint32_t)a.pv_bits[s];
+  return bits ? (word >> a.pv_shift[s]) & ((1u << bits) - 1u) : 0u;
+}
+// signed value of operand o
+template <int W>
+__device__ __forceinline__ int64_t nf_sval(const LevelArgs& a, const NfOp& o, const uint32_t* rec) {
+  if (o.kind == NF_CONST) return o.c;
+  const int64_t v1 = __ldg(a.pv_range[o.s1] + nf_field<W>(a, rec, o.s1));
+  if (o.kind == NF_PV) return v1;
+  return v1 * (int64_t)__ldg(a.pv_range[o.s2] + nf_field<W>(a, rec, o.s2));
+}
+// |value| of operand o and its divisor magic ceil(2^32/|v|) mod 2^32 (0 for |v| <= 1)
+template <int W>
+__device__ __forceinline__ uint32_t nf_abs(const LevelArgs& a, const NfOp& o, const uint32_t* rec, uint32_t* mag) {
+  if (o.kind == NF_CONST) {
+    if (mag) *mag = o.cm;
+    return o.c < 0 ? 0u - (uint32_t)o.c : (uint32_t)o.c;
+  }
+  if (o.kind == NF_PV) {
+    const uint32_t pos = nf_field<W>(a, rec, o.s1);
+    const int32_t v = __ldg(a.pv_range[o.s1] + pos);
+    const uint32_t av = v < 0 ? 0u - (uint32_t)v : (uint32_t)v;
+    if (mag) *mag = av == 0 ? 0u : __ldg(a.pv_magic[o.s1] + pos);
+    return av;
+  }
+  const int64_t p = nf_sval<W>(a, o, rec);
+  const uint32_t av = (uint32_t)(p < 0 ? -p : p);
+  if (mag) *mag = av > 1 ? 0xffffffffu / av + 1u : 0u;
+  return av;
+}
+
+template <int W>
+__device__ __forceinline__ uint32_t nf_node_mask(const LevelArgs& a, const uint32_t* rec, int r, uint32_t m,
+                                                 uint32_t nz, const int32_t* s_cx, const uint32_t* s_cm,
+                                                 const uint32_t* s_ca) {
+  for (int t = 0; t < a.n_terms && m; t++) {
+    const Term& T = a.terms[t];
+    const NfOp& oa = a.nf_op[t][0];
+    const NfOp& ob = a.nf_op[t][1];
+    uint32_t mm = 0;
+    switch (T.kind) {
+      case T_DIVX:
+      case T_DIVPROD: {  // x | n; DIVPROD: gate a != 0 && a | b, n = b / a (magic quotient)
+        uint32_t n;
+        if (T.kind == T_DIVX) {
+          n = nf_abs<W>(a, oa, rec, nullptr);
+        } else {
+          uint32_t ma;
+          const uint32_t av = nf_abs<W>(a, oa, rec, &ma), bv = nf_abs<W>(a, ob, rec, nullptr);
+          if (av == 0) return 0u;
+          n = av == 1 ? bv : __umulhi(bv, ma);
+          if (n * av != bv) return 0u;
+        }
+#pragma unroll 4
+        for (int c = 0; c < r; c++) mm |= (uint32_t)(n * s_cm[c] < 0x10000u) << c;
+        mm &= nz;  // x == 0 rejects (poison)
+        break;
+      }
+      case T_MULX: {  // d | x, d != 0
+        uint32_t md;
+        const uint32_t d = nf_abs<W>(a, oa, rec, &md);
+        if (d == 0) return 0u;
+        const uint32_t md1 = md - 1u;
+#pragma unroll 4
+        for (int c = 0; c < r; c++) mm |= (uint32_t)(s_ca[c] * md <= md1) << c;
+        break;
+      }
+      case T_QDIV: {  // (num / x) | nb; x == 0 or quotient 0 rejects
+        const uint32_t num = nf_abs<W>(a, oa, rec, nullptr), nb = nf_abs<W>(a, ob, rec, nullptr);
+        uint32_t rest = m;
+        while (rest) {
+          const int c = __ffs(rest) - 1;
+          rest &= rest - 1;
+          const uint32_t ax = s_ca[c];
+          if (ax == 0) continue;
+          const uint32_t q = ax == 1 ? num : __umulhi(num, s_cm[c]);
+          if (q != 0 && nb % q == 0) mm |= 1u << c;
+        }
+        break;
+      }
+      default: {  // T_CMP, 32-bit: (A * x) rel B
+        const int32_t A = (int32_t)nf_sval<W>(a, oa, rec), Bv = (int32_t)nf_sval<W>(a, ob, rec);
+#pragma unroll 4
+        for (int c = 0; c < r; c++) mm |= (uint32_t)rel_holds32(T.rel, A * s_cx[c], Bv) << c;
+        break;
+      }
+    }
+    m &= mm;
+  }
+  return m;
+}
+
+// Pass 1 (A4): accept masks of every frontier node (mask_bytes = 1/2/4 per node) and the
+// child count of every warp tile (tile_total).  Tiles are static: warp w of the grid takes
+// tiles w, w + nwarps, ...
+template <int W>
+__global__ void __launch_bounds__(256, 4) expand_nfast(const __grid_constant__ LevelArgs a) {
+  __shared__ int32_t s_cx[32];
+  __shared__ uint32_t s_cm[32], s_ca[32];
+  const int lane = threadIdx.x & 31;
+  const int r = a.r;
+  if (threadIdx.x < 32) {
+    const bool v = threadIdx.x < r;
+    s_cx[threadIdx.x] = v ? __ldg(a.cand + threadIdx.x) : 0;
+    s_cm[threadIdx.x] = v ? __ldg(a.cand_magic + threadIdx.x) : 0x10000u;
+    s_ca[threadIdx.x] = v ? __ldg(a.cand_abs + threadIdx.x) : 0u;
+  }
+  __syncthreads();
+  const uint32_t full = r >= 32 ? 0xffffffffu : ((1u << r) - 1u);
+  uint32_t nz = 0;
+  for (int c = 0; c < r; c++) nz |= (uint32_t)(s_cx[c] != 0) << c;
+  constexpr int TN = 32 * kNfNPL;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t t = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; t < a.n_tiles; t += nw) {
+    const uint64_t node0 = t * TN;
+    uint32_t rec[kNfNPL][W];
+#pragma unroll
+    for (int q = 0; q < kNfNPL; q++) {
+      const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
+      if (nd < a.n_parents) {
+        if (a.level == 0) {
+#pragma unroll
+          for (int w = 0; w < W; w++) rec[q][w] = 0u;
+        } else {
+          load_record<W>(a.parent_rec + nd * W, rec[q]);
+        }
+      }
+    }
+    uint32_t cnt = 0;
+#pragma unroll
+    for (int q = 0; q < kNfNPL; q++) {
+      const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
+      if (nd < a.n_parents) {
+        const uint32_t m = nf_node_mask<W>(a, rec[q], r, full, nz, s_cx, s_cm, s_ca);
+        cnt += (uint32_t)__popc(m);
+        if (a.mask_bytes == 1) reinterpret_cast<uint8_t*>(a.masks)[nd] = (uint8_t)m;
+        else if (a.mask_bytes == 2) reinterpret_cast<uint16_t*>(a.masks)[nd] = (uint16_t)m;
+        else reinterpret_cast<uint32_t*>(a.masks)[nd] = m;
+      }
+    }
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(FULL, cnt, o);
+    if (lane == 0) a.tile_total[t] = cnt;
+  }
+}
+
+// Pass 2 (A6, after scan_kernel turned tile_total into tile_base): children written at
+// their final index, CSR entries final; no stash.
+template <int W>
+__global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelArgs a) {
+  const int lane = threadIdx.x & 31;
+  constexpr int TN = 32 * kNfNPL;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t total = a.tile_base[a.n_tiles];
+  if (gw == 0 && lane == 0) {
+    if (total > a.child_cap) atomicOr(a.overflow_flag, 1u);
+    *a.total_out = total;
+    a.csr[a.n_parents] = total;
+  }
+  if (total > a.child_cap) return;
+  for (uint64_t t = gw; t < a.n_tiles; t += nw) {
+    const uint64_t node0 = t * TN;
+    uint32_t mask[kNfNPL], rec[kNfNPL][W];
+#pragma unroll
+    for (int q = 0; q < kNfNPL; q++) {
+      const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
+      mask[q] = 0;
+      if (nd < a.n_parents) {
+        if (a.mask_bytes == 1) mask[q] = reinterpret_cast<const uint8_t*>(a.masks)[nd];
+        else if (a.mask_bytes == 2) mask[q] = reinterpret_cast<const uint16_t*>(a.masks)[nd];
+        else mask[q] = reinterpret_cast<const uint32_t*>(a.masks)[nd];
+      }
+    }
+#pragma unroll
+    for (int q = 0; q < kNfNPL; q++) {
+      const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
+      if (mask[q]) {
+        if (a.level == 0) {
+#pragma unroll
+          for (int w = 0; w < W; w++) rec[q][w] = 0u;
+        } else {
+          load_record<W>(a.parent_rec + nd * W, rec[q]);
+        }
+      }
+    }
+    uint64_t run = a.tile_base[t];
+#pragma unroll
+    for (int q = 0; q < kNfNPL; q++) {
+      const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
+      const uint32_t c = (uint32_t)__popc(mask[q]);
+      uint32_t incl = c;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+      }
+      uint64_t rank = run + (incl - c);
+      run += __shfl_sync(FULL, incl, 31);
+      if (nd < a.n_parents) a.csr[nd] = rank;
+      uint32_t m = mask[q];
+      while (m) {
+        const int cc = __ffs(m) - 1;
+        m &= m - 1;
+        uint32_t out[W];
+#pragma unroll
+        for (int w = 0; w < W; w++) out[w] = rec[q][w] | (w == a.field_word ? (uint32_t)cc << a.field_shift : 0u);
+        store_record<W>(a.child_rec + rank * W, out);
+        rank++;
+      }
+    }
+  }
+}
+
+template <typename K>
+static int launch_grid_warps(K k, const LevelArgs& a, void* stream) {
+  int per_sm = 0;
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, 256, 0);
+  if (e != cudaSuccess) return (int)e;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  uint64_t grid = (uint64_t)sms * (per_sm > 0 ? per_sm : 1);
+  const uint64_t need = (a.n_tiles + 7) / 8;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  k<<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>(a);
+  return (int)cudaGetLastError();
+}
+
 // warp-tile levels: one wave of CTAs, never more warps than tiles
 template <typename K>
 static int launch_wtile_k(K k, const LevelArgs& a, void* stream) {
@@ -1083,8 +1328,14 @@ static int launch_wtile_wc(const LevelArgs& a, void* stream) {
 }
 
 template <int W>
+static int launch_nfast_emit_w(const LevelArgs& a, void* stream) {
+  return launch_grid_warps(nfast_emit<W>, a, stream);
+}
+
+template <int W>
 static int launch_w(const LevelArgs& a, void* stream) {
   if (a.kind == K_NARROW) return launch_persistent(expand_narrow<W>, a, a.block, stream);
+  if (a.kind == K_NFAST) return launch_grid_warps(expand_nfast<W>, a, stream);
   if (a.kind == K_WTILE) {
     switch (a.cpt) {
       case 4: return launch_wtile_wc<W, 4>(a, stream);

@@ -4,4 +4,5 @@
 
 namespace atf {
 int launch_expand_w1(const LevelArgs& a, void* stream) { return launch_w<1>(a, stream); }
+int launch_nfast_emit_w1(const LevelArgs& a, void* stream) { return launch_nfast_emit_w<1>(a, stream); }
 }  // namespace atf

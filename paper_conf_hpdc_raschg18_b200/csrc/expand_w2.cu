@@ -4,4 +4,5 @@
 
 namespace atf {
 int launch_expand_w2(const LevelArgs& a, void* stream) { return launch_w<2>(a, stream); }
+int launch_nfast_emit_w2(const LevelArgs& a, void* stream) { return launch_nfast_emit_w<2>(a, stream); }
 }  // namespace atf

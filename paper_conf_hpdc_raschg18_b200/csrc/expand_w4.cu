@@ -4,4 +4,5 @@
 
 namespace atf {
 int launch_expand_w4(const LevelArgs& a, void* stream) { return launch_w<4>(a, stream); }
+int launch_nfast_emit_w4(const LevelArgs& a, void* stream) { return launch_nfast_emit_w<4>(a, stream); }
 }  // namespace atf

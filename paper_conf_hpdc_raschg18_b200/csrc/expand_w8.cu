@@ -4,4 +4,5 @@
 
 namespace atf {
 int launch_expand_w8(const LevelArgs& a, void* stream) { return launch_w<8>(a, stream); }
+int launch_nfast_emit_w8(const LevelArgs& a, void* stream) { return launch_nfast_emit_w<8>(a, stream); }
 }  // namespace atf

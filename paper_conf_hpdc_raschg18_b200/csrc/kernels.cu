@@ -11,6 +11,20 @@ int launch_expand_w1(const LevelArgs& a, void* stream);
 int launch_expand_w2(const LevelArgs& a, void* stream);
 int launch_expand_w4(const LevelArgs& a, void* stream);
 int launch_expand_w8(const LevelArgs& a, void* stream);
+int launch_nfast_emit_w1(const LevelArgs& a, void* stream);
+int launch_nfast_emit_w2(const LevelArgs& a, void* stream);
+int launch_nfast_emit_w4(const LevelArgs& a, void* stream);
+int launch_nfast_emit_w8(const LevelArgs& a, void* stream);
+
+int launch_nfast_emit(const LevelArgs& a, int words, void* stream) {
+  switch (words) {
+    case 1: return launch_nfast_emit_w1(a, stream);
+    case 2: return launch_nfast_emit_w2(a, stream);
+    case 4: return launch_nfast_emit_w4(a, stream);
+    case 8: return launch_nfast_emit_w8(a, stream);
+    default: return (int)cudaErrorInvalidValue;
+  }
+}
 
 int launch_expand(const LevelArgs& a, int words, void* stream) {
   switch (words) {
