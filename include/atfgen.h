@@ -217,6 +217,33 @@ atf_status atf_space_decode_indices(const atf_space* s, const uint64_t* d_idx, i
 atf_status atf_space_decode_digits(const atf_space* s, const uint64_t* d_digits, int64_t n,
                                    int32_t* d_out, int64_t ld, void* stream);
 
+/* Encode = inverse of decode (the index access of P:229-231 read
+ * backwards, which also answers membership): d_values is a batch of n configurations,
+ * int32 SoA (value of parameter p at d_values + p*ld, ld >= n).  Each row is located by a
+ * top-down walk of every group's tree.  d_digits ([G][n] uint64, device) receives the
+ * per-group leaf indices; a group whose values are not a valid prefix path gets
+ * UINT64_MAX (the row is not in the space: not an error).  encode_indices also writes the
+ * mixed-radix index d_idx[n] (group 0 most significant; UINT64_MAX for rows not in the
+ * space) and needs S < 2^64 (else ATF_ERR_OVERFLOW).  Asynchronous on `stream`
+ * (NULL = the space's stream); device buffers are borrowed until the work completes.
+ * ATF_ERR_STATE before generate and on shard spaces. */
+atf_status atf_space_encode_digits(const atf_space* s, const int32_t* d_values, int64_t n, int64_t ld,
+                                   uint64_t* d_digits, void* stream);
+atf_status atf_space_encode_indices(const atf_space* s, const int32_t* d_values, int64_t n, int64_t ld,
+                                    uint64_t* d_digits, uint64_t* d_idx, void* stream);
+
+/* Random neighbours for simulated annealing ("a random neighbor c' of the
+ * current configuration c"; SURVEY.md §8(f) NEXT-1 reading: c' = c with ONE parameter
+ * re-drawn uniformly from its range such that c' is again a valid configuration).
+ * d_in / d_out: n configurations, int32 SoA (ld_in / ld_out >= n; d_out may not alias
+ * d_in).  Per row up to max_tries draws (counter-based splitmix64 of seed, row, draw);
+ * the first draw whose row is in the space (tree walk of the changed parameter's group)
+ * is kept.  d_moved[i] = the changed parameter id, or -1 (row copied unchanged).  Rows of
+ * d_in must be valid configurations.  Asynchronous on `stream`.  ATF_ERR_STATE before
+ * generate and on shard spaces. */
+atf_status atf_space_neighbors(const atf_space* s, const int32_t* d_in, int64_t ld_in, int64_t n, uint64_t seed,
+                               int32_t max_tries, int32_t* d_out, int64_t ld_out, int32_t* d_moved, void* stream);
+
 /* Per (group, level) statistics, in (group, level) order. */
 typedef struct {
   int32_t group, level, param;

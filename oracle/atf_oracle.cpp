@@ -669,9 +669,10 @@ static int cmd_decode(const Spec& s, const char* idxfile, const char* out, int t
 }
 
 // check: rows of values (int32 [n][P]) -> how many satisfy every constraint
-static int cmd_check(const Spec& s, const char* rowfile) {
+static int cmd_check(const Spec& s, const char* rowfile, const char* flagfile) {
   size_t P = s.params.size();
   FILE* f = std::fopen(rowfile, "rb");
+  FILE* ff = flagfile ? std::fopen(flagfile, "wb") : nullptr;  // optional: one byte per row
   std::vector<int32_t> row(P);
   std::vector<i64> vals(P);
   u64 n = 0, ok = 0, in_range = 0;
@@ -686,8 +687,10 @@ static int cmd_check(const Spec& s, const char* rowfile) {
     for (size_t p = 0; p < P; p++) good = constraint_holds(s, (int)p, vals[p], vals.data()) && good;
     ok += (good && inr);
     in_range += inr;
+    if (ff) std::fputc((good && inr) ? 1 : 0, ff);
   }
   std::fclose(f);
+  if (ff) std::fclose(ff);
   std::printf("{\"rows\":%" PRIu64 ",\"valid\":%" PRIu64 ",\"in_range\":%" PRIu64 "}\n", n, ok, in_range);
   return 0;
 }
@@ -769,7 +772,7 @@ int main(int argc, char** argv) {
     if (cmd == "o1") return cmd_o1(s, pos.size() > 1 ? pos[1].c_str() : nullptr);
     if (cmd == "leaves") return cmd_leaves(s, std::atoi(pos.at(1).c_str()), pos.at(2).c_str());
     if (cmd == "decode") return cmd_decode(s, pos.at(1).c_str(), pos.at(2).c_str(), threads);
-    if (cmd == "check") return cmd_check(s, pos.at(1).c_str());
+    if (cmd == "check") return cmd_check(s, pos.at(1).c_str(), pos.size() > 2 ? pos.at(2).c_str() : nullptr);
     if (cmd == "time") return cmd_time(s, threads, budget);
     std::fprintf(stderr, "unknown command %s\n", cmd.c_str());
     return 2;

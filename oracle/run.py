@@ -84,11 +84,20 @@ def decode(spec, indices: np.ndarray, threads: int = 1, want_rows: bool = True, 
         return d, np.fromfile(out, dtype=np.int32).reshape(P, -1)
 
 
-def check(spec, rows: np.ndarray, timeout=None) -> dict:
+def check(spec, rows: np.ndarray, timeout=None, per_row: bool = False) -> dict:
+    """Constraint check of configurations rows[n][P] (valid iff every parameter's
+    value is in its range and every constraint holds).  per_row: also return "flags", a
+    uint8 array with 1 for each valid row."""
     with tempfile.TemporaryDirectory() as td:
         f = os.path.join(td, "rows.bin")
         np.ascontiguousarray(rows, dtype=np.int32).tofile(f)
-        return _run(["check", _spec_path(spec, td), f], timeout)
+        args = ["check", _spec_path(spec, td), f]
+        if per_row:
+            args.append(os.path.join(td, "flags.bin"))
+        out = _run(args, timeout)
+        if per_row:
+            out["flags"] = np.fromfile(os.path.join(td, "flags.bin"), dtype=np.uint8)
+        return out
 
 
 def time_sample(spec, threads: int, budget_s: float, timeout=None) -> dict:

@@ -76,6 +76,10 @@ _SIGS = {
     "atf_space_level_view": (_st, [SP, C.c_int32, C.c_int32, C.POINTER(atf_level_view)]),
     "atf_space_decode_indices": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_space_decode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
+    "atf_space_encode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p]),
+    "atf_space_encode_indices": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p, C.c_void_p]),
+    "atf_space_neighbors": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_uint64, C.c_int32, C.c_void_p, C.c_int64,
+                                  C.c_void_p, C.c_void_p]),
     "atf_space_stats": (_st, [SP, C.POINTER(atf_level_stats), C.c_int32, C.POINTER(C.c_int32)]),
     "atf_space_destroy": (None, [SP]),
     "atf_status_str": (C.c_char_p, [_st]),

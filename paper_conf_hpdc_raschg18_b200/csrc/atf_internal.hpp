@@ -146,6 +146,28 @@ struct DecodeArgs {
   const int32_t* lvl_range[kMaxLevels];
 };
 
+// Encode (inverse decode): configuration -> per-group leaf index by
+// a top-down walk of each group's tree (value -> range position by binary search in the
+// parameter's sorted value table, position -> child by binary search among the node's
+// children, which are sorted by position).
+struct EncodeArgs {
+  int32_t n_groups;
+  uint64_t gsize[kMaxGroups];
+  int32_t lvl_begin[kMaxGroups + 1];
+  int16_t lvl_param[kMaxLevels], lvl_word[kMaxLevels], lvl_shift[kMaxLevels], lvl_bits[kMaxLevels];
+  int32_t lvl_words[kMaxLevels];         // record words of the level's group
+  const uint32_t* lvl_rec[kMaxLevels];   // level records [n][words]
+  const uint64_t* lvl_csr[kMaxLevels];   // CSR of level l into level l + 1 (null at the leaves)
+  uint64_t lvl_n[kMaxLevels];
+  const int32_t* lvl_sorted[kMaxLevels]; // the parameter's [sorted values r][their positions r]
+  int32_t lvl_r[kMaxLevels];
+  // per parameter (neighbour proposals)
+  int32_t n_params;
+  int32_t param_group[kMaxLevels];
+  int32_t param_r[kMaxLevels];
+  const int32_t* param_range[kMaxLevels];  // values in range order
+};
+
 // Dynamic shared-memory layouts of the expand kernels (byte offsets; -1 = absent).
 struct SmemLayout {
   int ctl, ok, rec, opa, opb, slots, hot, hot2, cnt, off, sum, bm, q, cx, cm, qtab, wtot, total;
@@ -230,5 +252,9 @@ int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long 
                     unsigned int* counter, void* stream, uint32_t* piece_tile = nullptr,
                     uint64_t piece_cap = 0);
 int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
+int launch_encode(const EncodeArgs& a, const int32_t* vals, int64_t ld, int64_t n, uint64_t* digits, uint64_t* idx,
+                  void* stream);
+int launch_neighbors(const EncodeArgs& a, const int32_t* in, int64_t ld_in, int32_t* out, int64_t ld_out, int64_t n,
+                     uint64_t seed, int max_tries, int32_t* moved, void* stream);
 
 }  // namespace atf

@@ -101,6 +101,7 @@ struct atf_space {
   // device state
   bool dev_ready = false;
   std::vector<int32_t*> d_range;
+  std::vector<int32_t*> d_sorted;  // per parameter: [values sorted ascending][their positions] (encode)
   std::vector<std::vector<Chunk>> arena;  // per group
   std::vector<std::vector<LevelData>> data;
   std::vector<uint64_t> gsize;
@@ -887,6 +888,24 @@ static atf_status ensure_device(atf_space* s) {
                                   (cudaStream_t)s->opts.stream));
     }
   }
+  s->d_sorted.assign(np, nullptr);
+  for (size_t p = 0; p < np; p++) {
+    auto& v = s->params[p].values;
+    s->d_sorted[p] = (int32_t*)dalloc(s, std::max<size_t>(16, v.size() * 8));
+    if (!s->d_sorted[p]) return fail(s, ATF_ERR_OOM, "sorted range upload");
+    if (!v.empty()) {
+      std::vector<int32_t> idx(v.size());
+      std::iota(idx.begin(), idx.end(), 0);
+      std::sort(idx.begin(), idx.end(), [&](int32_t x, int32_t y) { return v[x] < v[y]; });
+      std::vector<int32_t> buf(2 * v.size());
+      for (size_t j = 0; j < v.size(); j++) {
+        buf[j] = v[idx[j]];
+        buf[v.size() + j] = idx[j];
+      }
+      CUDA_TRY(s, cudaMemcpyAsync(s->d_sorted[p], buf.data(), buf.size() * 4, cudaMemcpyHostToDevice,
+                                  (cudaStream_t)s->opts.stream));
+    }
+  }
   s->d_counter = (unsigned int*)dalloc(s, 4 * kMaxGroups);
   s->d_totals = (unsigned long long*)dalloc(s, 8 * kMaxGroups);
   s->d_ovf = (unsigned int*)dalloc(s, 4 * kMaxGroups);
@@ -952,6 +971,9 @@ static void release_device(atf_space* s) {
   for (size_t p = 0; p < s->d_range.size(); p++)
     dfree(s, s->d_range[p], 12 * ((s->params[p].values.size() + 127) / 128 * 128));
   s->d_range.clear();
+  for (size_t p = 0; p < s->d_sorted.size(); p++)
+    dfree(s, s->d_sorted[p], std::max<size_t>(16, s->params[p].values.size() * 8));
+  s->d_sorted.clear();
   dfree(s, s->d_status, s->status_cap * 8);
   dfree(s, s->d_scratch, s->scratch_cap);
   dfree(s, (char*)s->d_stash, s->stash_cap);
@@ -1559,6 +1581,86 @@ static atf_status decode_common(const atf_space* cs, const uint64_t* idx, const 
   CUDA_TRY(s, cudaStreamSynchronize(st));
   if (s->h_flags[0]) return fail(s, ATF_ERR_INDEX, "index/digit out of range (rows set to INT32_MIN)");
   return ATF_OK;
+}
+
+static void make_encode_args(const atf_space* s, EncodeArgs& a) {
+  std::memset(&a, 0, sizeof a);
+  a.n_groups = (int)s->groups.size();
+  int l = 0;
+  for (int g = 0; g < a.n_groups; g++) {
+    const GroupPlan& gp = s->groups[g];
+    a.gsize[g] = s->gsize[g];
+    a.lvl_begin[g] = l;
+    for (size_t k = 0; k < gp.levels.size(); k++, l++) {
+      const LevelPlan& lp = gp.levels[k];
+      const LevelData& d = s->data[g][k];
+      a.lvl_param[l] = (int16_t)lp.param;
+      a.lvl_word[l] = (int16_t)lp.field_word;
+      a.lvl_shift[l] = (int16_t)lp.field_shift;
+      a.lvl_bits[l] = (int16_t)lp.field_bits;
+      a.lvl_words[l] = gp.words;
+      a.lvl_rec[l] = d.rec;
+      a.lvl_csr[l] = d.csr;
+      a.lvl_n[l] = d.rec ? d.n : 0;
+      a.lvl_sorted[l] = s->d_sorted[lp.param];
+      a.lvl_r[l] = (int32_t)s->params[lp.param].values.size();
+    }
+  }
+  a.lvl_begin[a.n_groups] = l;
+  a.n_params = (int)s->params.size();
+  for (int g = 0; g < a.n_groups; g++)
+    for (int m : s->groups[g].members) a.param_group[m] = g;
+  for (int p = 0; p < a.n_params; p++) {
+    a.param_r[p] = (int32_t)s->params[p].values.size();
+    a.param_range[p] = s->d_range[p];
+  }
+}
+
+static atf_status encode_common(const atf_space* cs, const int32_t* vals, int64_t n, int64_t ld, uint64_t* digits,
+                                uint64_t* idx, void* stream) {
+  atf_space* s = (atf_space*)cs;
+  if (!s || !vals || !digits || n < 0 || ld < n) return fail(s, ATF_ERR_INVALID_ARG, "bad encode arguments");
+  if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "encode needs a generated (non-shard) space");
+  if (idx) {
+    u128 S = 1;
+    for (uint64_t z : s->gsize) S *= z;
+    if (S >> 64) return fail(s, ATF_ERR_OVERFLOW, "S >= 2^64: use atf_space_encode_digits");
+  }
+  if (n == 0) return ATF_OK;
+  EncodeArgs a;
+  make_encode_args(s, a);
+  CUDA_TRY(s, cudaSetDevice(s->opts.device));
+  cudaStream_t st = (cudaStream_t)(stream ? stream : s->opts.stream);
+  int ce = launch_encode(a, vals, ld, n, digits, idx, st);
+  if (ce) return fail(s, ATF_ERR_CUDA, "encode launch: %s", cudaGetErrorString((cudaError_t)ce));
+  return ATF_OK;
+}
+
+atf_status atf_space_neighbors(const atf_space* cs, const int32_t* d_in, int64_t ld_in, int64_t n, uint64_t seed,
+                               int32_t max_tries, int32_t* d_out, int64_t ld_out, int32_t* d_moved, void* stream) {
+  atf_space* s = (atf_space*)cs;
+  if (!s || !d_in || !d_out || !d_moved || n < 0 || ld_in < n || ld_out < n || max_tries < 0)
+    return fail(s, ATF_ERR_INVALID_ARG, "bad neighbour arguments");
+  if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "neighbours need a generated (non-shard) space");
+  if (n == 0) return ATF_OK;
+  EncodeArgs a;
+  make_encode_args(s, a);
+  CUDA_TRY(s, cudaSetDevice(s->opts.device));
+  cudaStream_t st = (cudaStream_t)(stream ? stream : s->opts.stream);
+  int ce = launch_neighbors(a, d_in, ld_in, d_out, ld_out, n, seed, max_tries, d_moved, st);
+  if (ce) return fail(s, ATF_ERR_CUDA, "neighbour launch: %s", cudaGetErrorString((cudaError_t)ce));
+  return ATF_OK;
+}
+
+atf_status atf_space_encode_indices(const atf_space* s, const int32_t* d_values, int64_t n, int64_t ld,
+                                    uint64_t* d_digits, uint64_t* d_idx, void* stream) {
+  if (!d_idx) return fail((atf_space*)s, ATF_ERR_INVALID_ARG, "null index output");
+  return encode_common(s, d_values, n, ld, d_digits, d_idx, stream);
+}
+
+atf_status atf_space_encode_digits(const atf_space* s, const int32_t* d_values, int64_t n, int64_t ld,
+                                   uint64_t* d_digits, void* stream) {
+  return encode_common(s, d_values, n, ld, d_digits, nullptr, stream);
 }
 
 atf_status atf_space_decode_indices(const atf_space* s, const uint64_t* d_idx, int64_t n, int32_t* d_out, int64_t ld,

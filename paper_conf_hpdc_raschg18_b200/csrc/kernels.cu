@@ -245,6 +245,124 @@ int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n,
   return launch_decode(a, nullptr, digits, n, out, ld, bad, stream);
 }
 
+// ---------------------------------------------------------------- encode
+// configuration (int32 SoA, column p at vals + p*ld) -> per-group digits [G][n] (UINT64_MAX:
+// the row is not a valid configuration, i.e. not in the space) and, if idx != null, the
+// mixed-radix index (group 0 most significant; UINT64_MAX when invalid).
+// Leaf index of group g for row i (UINT64_MAX if the group's values are not a valid path).
+__device__ uint64_t encode_group(const EncodeArgs& a, const int32_t* __restrict__ vals, int64_t ld, int64_t i, int g) {
+  const int l0 = a.lvl_begin[g], l1 = a.lvl_begin[g + 1];
+  if (l1 <= l0) return ~0ull;
+  uint64_t lo = 0, hi = a.lvl_n[l0], node = 0;
+  for (int l = l0; l < l1; l++) {
+    const int32_t v = vals[(int64_t)a.lvl_param[l] * ld + i];
+    // value -> range position
+    const int32_t* sv = a.lvl_sorted[l];
+    const int r = a.lvl_r[l];
+    int b = 0, e = r;
+    while (b < e) {
+      const int m = (b + e) >> 1;
+      if (__ldg(sv + m) < v) b = m + 1; else e = m;
+    }
+    if (b >= r || __ldg(sv + b) != v) return ~0ull;
+    const uint32_t pos = (uint32_t)__ldg(sv + r + b);
+    // position -> child among [lo, hi) (children sorted by their level-l field)
+    const int W = a.lvl_words[l];
+    const uint32_t* rec = a.lvl_rec[l] + a.lvl_word[l];
+    const uint32_t bits = (uint32_t)a.lvl_bits[l];
+    const uint32_t fm = bits >= 32 ? 0xffffffffu : ((1u << bits) - 1u);
+    const int sh = a.lvl_shift[l];
+    uint64_t cb = lo, ce = hi;
+    while (cb < ce) {
+      const uint64_t m = (cb + ce) >> 1;
+      const uint32_t f = bits ? (__ldg(rec + m * (uint64_t)W) >> sh) & fm : 0u;
+      if (f < pos) cb = m + 1; else ce = m;
+    }
+    if (cb >= hi || (bits ? (__ldg(rec + cb * (uint64_t)W) >> sh) & fm : 0u) != pos) return ~0ull;
+    node = cb;
+    if (l + 1 < l1) {
+      lo = __ldg(a.lvl_csr[l] + node);
+      hi = __ldg(a.lvl_csr[l] + node + 1);
+    }
+  }
+  return node;
+}
+
+__global__ void encode_kernel(const __grid_constant__ EncodeArgs a, const int32_t* __restrict__ vals, int64_t ld,
+                              int64_t n, uint64_t* __restrict__ digits, uint64_t* __restrict__ idx) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    bool ok = true;
+    uint64_t index = 0;
+    for (int g = 0; g < a.n_groups; g++) {
+      const uint64_t d = encode_group(a, vals, ld, i, g);
+      digits[(int64_t)g * n + i] = d;
+      ok = ok && d != ~0ull;
+      index = index * a.gsize[g] + d;
+    }
+    if (idx) idx[i] = ok ? index : ~0ull;
+  }
+}
+
+// counter-based generator shared by nothing else: splitmix64 of (seed, row, draw)
+__device__ __forceinline__ uint64_t nb_rand(uint64_t seed, uint64_t row, uint64_t k) {
+  uint64_t z = seed + 0x9E3779B97F4A7C15ull * (row * 0x100000001B3ull + k + 1);
+  z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+  z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+  return z ^ (z >> 31);
+}
+
+// Random neighbours (simulated annealing P:217-223): row i of
+// `out` = row i of `in` with one parameter re-drawn uniformly from its range, retried up
+// to max_tries times until the changed row is a valid configuration (only the changed
+// parameter's group is re-walked: the other groups are untouched).  moved[i] = the changed
+// parameter, or -1 if no valid neighbour was found (row copied unchanged).
+__global__ void neighbor_kernel(const __grid_constant__ EncodeArgs a, const int32_t* __restrict__ in, int64_t ld_in,
+                                int32_t* __restrict__ out, int64_t ld_out, int64_t n, uint64_t seed, int max_tries,
+                                int32_t* __restrict__ moved) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    for (int p = 0; p < a.n_params; p++) out[(int64_t)p * ld_out + i] = in[(int64_t)p * ld_in + i];
+    int32_t mv = -1;
+    for (int t = 0; t < max_tries && mv < 0; t++) {
+      const uint64_t r1 = nb_rand(seed, (uint64_t)i, 2 * (uint64_t)t), r2 = nb_rand(seed, (uint64_t)i, 2 * (uint64_t)t + 1);
+      const int p = (int)(r1 % (uint64_t)a.n_params);
+      const int rp = a.param_r[p];
+      if (rp <= 1) continue;
+      const int32_t old = out[(int64_t)p * ld_out + i];
+      const int32_t v = __ldg(a.param_range[p] + (int64_t)(r2 % (uint64_t)rp));
+      if (v == old) continue;
+      out[(int64_t)p * ld_out + i] = v;
+      if (encode_group(a, out, ld_out, i, a.param_group[p]) != ~0ull) mv = p;
+      else out[(int64_t)p * ld_out + i] = old;
+    }
+    moved[i] = mv;
+  }
+}
+
+int launch_neighbors(const EncodeArgs& a, const int32_t* in, int64_t ld_in, int32_t* out, int64_t ld_out, int64_t n,
+                     uint64_t seed, int max_tries, int32_t* moved, void* stream) {
+  if (n <= 0) return 0;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  int64_t blocks = (n + 255) / 256;
+  if (blocks > (int64_t)sms * 8) blocks = (int64_t)sms * 8;
+  neighbor_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, in, ld_in, out, ld_out, n, seed, max_tries,
+                                                                        moved);
+  return (int)cudaGetLastError();
+}
+
+int launch_encode(const EncodeArgs& a, const int32_t* vals, int64_t ld, int64_t n, uint64_t* digits, uint64_t* idx,
+                  void* stream) {
+  if (n <= 0) return 0;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  int64_t blocks = (n + 255) / 256;
+  if (blocks > (int64_t)sms * 8) blocks = (int64_t)sms * 8;
+  encode_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, vals, ld, n, digits, idx);
+  return (int)cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- standalone scan (tests)
 // Exclusive scan u32 -> u64 with the same look-back as expand_kernel; out[n] = total.
 __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restrict__ out, int64_t n,

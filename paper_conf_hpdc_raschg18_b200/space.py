@@ -211,6 +211,53 @@ class Space:
         L.check(L.atf_space_decode_digits(self._h, digits.data_ptr(), n, out.data_ptr(), out.stride(0), sp), self._h)
         return out
 
+    # ---- encode (inverse of decode; membership)
+    def encode(self, values, stream=None):
+        """values: int32 CUDA tensor [P, n] (SoA, one configuration per column) -> int64
+        tensor [n] of 0-based indices, -1 where the configuration is not in the space
+        (requires S < 2^64)."""
+        import torch
+        values = values.to(torch.int32)
+        if values.stride(1) != 1:
+            values = values.contiguous()
+        n = values.shape[1]
+        G = self.num_groups()
+        dig = torch.empty((G, n), dtype=torch.int64, device=values.device)
+        idx = torch.empty(n, dtype=torch.int64, device=values.device)
+        sp = stream.cuda_stream if stream is not None else None
+        L.check(L.atf_space_encode_indices(self._h, values.data_ptr(), n, values.stride(0), dig.data_ptr(),
+                                           idx.data_ptr(), sp), self._h)
+        return idx  # UINT64_MAX reads as -1 in int64
+
+    def encode_digits(self, values, stream=None):
+        """values: int32 CUDA tensor [P, n] -> int64 tensor [G, n] of per-group leaf indices
+        (-1 where the group's values are not a valid path); works for any S."""
+        import torch
+        values = values.to(torch.int32)
+        if values.stride(1) != 1:
+            values = values.contiguous()
+        n = values.shape[1]
+        dig = torch.empty((self.num_groups(), n), dtype=torch.int64, device=values.device)
+        sp = stream.cuda_stream if stream is not None else None
+        L.check(L.atf_space_encode_digits(self._h, values.data_ptr(), n, values.stride(0), dig.data_ptr(), sp),
+                self._h)
+        return dig
+
+    def neighbors(self, values, seed: int, max_tries: int = 16, stream=None):
+        """values: int32 CUDA tensor [P, n] of valid configurations -> (int32 [P, n] neighbours,
+        int32 [n] changed parameter id or -1); one parameter re-drawn per row."""
+        import torch
+        values = values.to(torch.int32)
+        if values.stride(1) != 1:
+            values = values.contiguous()
+        P, n = values.shape
+        out = torch.empty((P, n), dtype=torch.int32, device=values.device)
+        moved = torch.empty(n, dtype=torch.int32, device=values.device)
+        sp = stream.cuda_stream if stream is not None else None
+        L.check(L.atf_space_neighbors(self._h, values.data_ptr(), values.stride(0), n, seed & ((1 << 64) - 1),
+                                      max_tries, out.data_ptr(), out.stride(0), moved.data_ptr(), sp), self._h)
+        return out, moved
+
     def close(self) -> None:
         if self._h:
             L.atf_space_destroy(self._h)

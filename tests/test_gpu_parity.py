@@ -272,3 +272,75 @@ def test_c5_full_closed_form(Space):
         # lexicographic extremes: digit 0 = the first valid tuple in range-position order
         first = sp.decode_digits(torch.zeros((3, 1), dtype=torch.int64, device="cuda")).flatten().tolist()
         assert first == [1] * 16 + [2] * 8
+
+
+# ---------------------------------------------------------------- encode (inverse decode)
+def _range_values(r):
+    """Range of a parameter as written in the spec: INTERVAL inclusive, POW2 = 2^i, SET listed."""
+    if r["kind"] == "interval":
+        return list(range(r["begin"], r["end"] + 1, r["step"]))
+    if r["kind"] == "pow2":
+        return [1 << i for i in range(r["begin"], r["end"] + 1, r["step"])]
+    return list(r["values"])
+
+
+def _perturb(spec, rows, gen):
+    """Each row with one parameter replaced by a random value of its range (or a value
+    outside every range): a mix of rows inside and outside the space."""
+    rows = rows.copy()
+    n, P = rows.shape
+    ranges = [np.array(_range_values(p.range), dtype=np.int64) for p in spec.params]
+    which = gen.integers(0, P, n)
+    for i in range(n):
+        R = ranges[which[i]]
+        rows[i, which[i]] = R[gen.integers(0, len(R))] if gen.random() < 0.85 else 1_000_003
+    return rows
+
+
+@pytest.mark.parametrize("name", ["C1", "fig1", "saxpy360", "C2-256", "C3-IS1", "C3-12x30x8", "C5-300x4",
+                                  "C3-IS4-anch"])
+def test_encode_inverts_decode_and_tests_membership(Space, name):
+    spec = SMALL[name]()
+    gen = np.random.default_rng(7)
+    with Space(spec) as sp:
+        sp.generate()
+        S = sp.size()
+        if S < (1 << 63):
+            n = min(S, 100_000)
+            idx = torch.from_numpy(gen.integers(0, S, n, dtype=np.int64)).cuda() if S > n else \
+                torch.arange(S, dtype=torch.int64, device="cuda")
+            rows = sp.decode(idx)
+            assert torch.equal(sp.encode(rows), idx)
+        else:
+            G = sp.num_groups()
+            sizes = sp.group_sizes()
+            n = 100_000
+            dig = torch.stack([torch.from_numpy(gen.integers(0, sizes[g], n, dtype=np.int64)) for g in range(G)]).cuda()
+            rows = sp.decode_digits(dig)
+            assert torch.equal(sp.encode_digits(rows), dig)
+        # membership of perturbed rows == the oracle's constraint check (P:49)
+        pert = _perturb(spec, rows.T.cpu().numpy(), gen)[:20_000]
+        got = sp.encode_digits(torch.from_numpy(pert.T.copy()).cuda())
+        got_valid = (got >= 0).all(dim=0).cpu().numpy()
+        want = orc.check(spec, pert, per_row=True)["flags"].astype(bool)
+        assert np.array_equal(got_valid, want)
+        assert 0 < want.sum() < len(want) or S == 0
+
+
+@pytest.mark.parametrize("seed", range(0, 80, 8))
+def test_encode_fuzz_membership(Space, seed):
+    spec = A.random_spec(seed)
+    gen = np.random.default_rng(seed)
+    with Space(spec) as sp:
+        sp.generate()
+        S = sp.size()
+        ranges = [np.array(_range_values(p.range), dtype=np.int64) for p in spec.params]
+        n = 5000
+        rows = np.stack([R[gen.integers(0, len(R), n)] if len(R) else np.zeros(n, np.int64) for R in ranges], 1)
+        got = sp.encode_digits(torch.from_numpy(rows.T.astype(np.int32).copy()).cuda())
+        got_valid = (got >= 0).all(dim=0).cpu().numpy()
+        want = orc.check(spec, rows.astype(np.int32), per_row=True)["flags"].astype(bool)
+        assert np.array_equal(got_valid, want)
+        if S and S < (1 << 63):
+            idx = torch.arange(min(S, 4096), dtype=torch.int64, device="cuda")
+            assert torch.equal(sp.encode(sp.decode(idx)), idx)
