@@ -247,6 +247,20 @@ def secondary_n1(steps, warmup, sm_mhz):
                      "roofline_frac_step": rf["step"]["frac"], "dominant_launch": rf["launch"],
                      "dominant_frac": rf["frac"], "kernel_ms": rf["step"]["ms"],
                      "level_ms": [round(x, 4) for x in np.mean(res["level_ms"], axis=0).tolist()]}
+    # P:280's 32x32 experiment: CLTune-style filtering of the full product (SURVEY.md §8(f)
+    # NEXT-4; 6.87e10 tuples, the paper's CLTune run was aborted after 3 hours) vs the tree
+    spec = A.c2_xgemm_direct(32)
+    with Space(spec) as sp:
+        sp.filter_product()  # warm-up (upload, module load)
+        torch.cuda.synchronize()
+        t0 = time.perf_counter()
+        cnt, tot = sp.filter_product()
+        t_filter = time.perf_counter() - t0
+        res = run_generation(spec, steps, warmup)
+        out["C2-32-full-product-filter"] = {
+            "tuples": tot, "valid": cnt, "filter_s": t_filter, "tuples_per_s": tot / t_filter,
+            "tree_ms_per_step": float(np.mean(res["ms"])), "tree_S": str(res["size"]),
+            "note": "P:280: CLTune-style generation of the 32x32 XgemmDirect space aborted after 3 h (CPU)"}
     # C4: decode 10^8 random indices into C3-IS2
     from atfspec.fuzz import splitmix64_indices
     spec = A.c3_xgemm("IS2")

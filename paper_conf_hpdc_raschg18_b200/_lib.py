@@ -78,6 +78,7 @@ _SIGS = {
     "atf_space_decode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_space_encode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p]),
     "atf_space_encode_indices": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p, C.c_void_p]),
+    "atf_space_filter_product": (_st, [SP, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),
     "atf_space_neighbors": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_uint64, C.c_int32, C.c_void_p, C.c_int64,
                                   C.c_void_p, C.c_void_p]),
     "atf_space_stats": (_st, [SP, C.POINTER(atf_level_stats), C.c_int32, C.POINTER(C.c_int32)]),

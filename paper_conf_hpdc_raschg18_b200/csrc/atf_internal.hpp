@@ -168,6 +168,19 @@ struct EncodeArgs {
   const int32_t* param_range[kMaxLevels];  // values in range order
 };
 
+// CLTune-style baseline (SURVEY.md §8(f) NEXT-4, P:183 / P:280): enumerate the FULL
+// cartesian product and test every constraint of every tuple.
+struct ProductArgs {
+  int32_t n_params;
+  int32_t r[kMaxLevels];
+  const int32_t* range[kMaxLevels];
+  int32_t prog_first[kMaxLevels], prog_count[kMaxLevels];  // the parameter's programs in `progs`
+  const int32_t* progs;    // [n_progs][2] (offset, length) into `code`
+  const int32_t* code;     // device bytecode, OP_SLOT j = value of parameter j
+  uint64_t total;          // product of the r (< 2^64)
+  uint64_t chunk;          // tuples per thread (odometer)
+};
+
 // Dynamic shared-memory layouts of the expand kernels (byte offsets; -1 = absent).
 struct SmemLayout {
   int ctl, ok, rec, opa, opb, slots, hot, hot2, cnt, off, sum, bm, q, cx, cm, qtab, wtot, total;
@@ -254,6 +267,7 @@ int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long 
 int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
 int launch_encode(const EncodeArgs& a, const int32_t* vals, int64_t ld, int64_t n, uint64_t* digits, uint64_t* idx,
                   void* stream);
+int launch_filter_product(const ProductArgs& a, unsigned long long* count, void* stream);
 int launch_neighbors(const EncodeArgs& a, const int32_t* in, int64_t ld_in, int32_t* out, int64_t ld_out, int64_t n,
                      uint64_t seed, int max_tries, int32_t* moved, void* stream);
 

@@ -1636,6 +1636,66 @@ static atf_status encode_common(const atf_space* cs, const int32_t* vals, int64_
   return ATF_OK;
 }
 
+atf_status atf_space_filter_product(atf_space* s, uint64_t* h_count, uint64_t* h_tuples) {
+  if (!s || !h_count) return ATF_ERR_INVALID_ARG;
+  atf_status e = plan(s);  // validation + static analysis (the product path needs no tree)
+  if (e) return e;
+  if ((e = ensure_device(s))) return e;
+  ProductArgs a;
+  std::memset(&a, 0, sizeof a);
+  a.n_params = (int)s->params.size();
+  u128 total = 1;
+  std::vector<int32_t> code, progs;
+  for (int p = 0; p < a.n_params; p++) {
+    const ParamDef& pd = s->params[p];
+    a.r[p] = (int32_t)pd.values.size();
+    a.range[p] = s->d_range[p];
+    total *= (u128)pd.values.size();
+    // the parameter's programs (ANDed), PARAM j -> SLOT j (slots = the tuple's values)
+    a.prog_first[p] = (int32_t)progs.size() / 2;
+    a.prog_count[p] = (int32_t)pd.programs.size();
+    for (const auto& pr : pd.programs) {
+      progs.push_back((int32_t)code.size());
+      for (size_t i = 0; i < pr.size();) {
+        const int op = pr[i];
+        if (op == ATF_OP_PARAM) { code.push_back(OP_SLOT); code.push_back(pr[i + 1]); i += 2; }
+        else if (op == ATF_OP_CONST) { code.insert(code.end(), pr.begin() + i, pr.begin() + i + 3); i += 3; }
+        else { code.push_back(op); i += 1; }
+      }
+      progs.push_back((int32_t)code.size() - progs.back());
+    }
+  }
+  if (total >> 64) return fail(s, ATF_ERR_OVERFLOW, "full product >= 2^64");
+  a.total = (uint64_t)total;
+  if (h_tuples) *h_tuples = a.total;
+  if (a.total == 0) { *h_count = 0; return ATF_OK; }
+  a.chunk = std::max<uint64_t>(1, std::min<uint64_t>(4096, a.total / (148ull * 2048)));
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  const size_t cbytes = std::max<size_t>(16, (code.size() + progs.size()) * 4);
+  int32_t* d_code = (int32_t*)dalloc(s, cbytes);
+  unsigned long long* d_cnt = (unsigned long long*)dalloc(s, 16);
+  if (!d_code || !d_cnt) return fail(s, ATF_ERR_OOM, "product filter scratch");
+  a.code = d_code;
+  a.progs = d_code + code.size();
+  std::vector<int32_t> up(code);
+  up.insert(up.end(), progs.begin(), progs.end());
+  atf_status out = ATF_OK;
+  if (!up.empty() && cudaMemcpyAsync(d_code, up.data(), up.size() * 4, cudaMemcpyHostToDevice, st) != cudaSuccess)
+    out = fail(s, ATF_ERR_CUDA, "product filter upload");
+  if (!out && cudaMemsetAsync(d_cnt, 0, 8, st) != cudaSuccess) out = fail(s, ATF_ERR_CUDA, "memset");
+  if (!out) {
+    int ce = launch_filter_product(a, d_cnt, st);
+    if (ce) out = fail(s, ATF_ERR_CUDA, "product filter launch: %s", cudaGetErrorString((cudaError_t)ce));
+  }
+  if (!out && (cudaMemcpyAsync(s->h_totals, d_cnt, 8, cudaMemcpyDeviceToHost, st) != cudaSuccess ||
+               cudaStreamSynchronize(st) != cudaSuccess))
+    out = fail(s, ATF_ERR_CUDA, "product filter readback");
+  if (!out) *h_count = s->h_totals[0];
+  dfree(s, d_code, cbytes);
+  dfree(s, d_cnt, 16);
+  return out;
+}
+
 atf_status atf_space_neighbors(const atf_space* cs, const int32_t* d_in, int64_t ld_in, int64_t n, uint64_t seed,
                                int32_t max_tries, int32_t* d_out, int64_t ld_out, int32_t* d_moved, void* stream) {
   atf_space* s = (atf_space*)cs;

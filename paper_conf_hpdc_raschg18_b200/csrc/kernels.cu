@@ -363,6 +363,60 @@ int launch_encode(const EncodeArgs& a, const int32_t* vals, int64_t ld, int64_t 
   return (int)cudaGetLastError();
 }
 
+// ---------------------------------------------------------------- CLTune-style baseline
+// Thread t takes tuples [t*chunk, (t+1)*chunk) of the full product in declaration order
+// (last parameter fastest): one mixed-radix decode of its first tuple, then an odometer.
+// A tuple is valid iff every parameter's constraint holds (strict bytecode semantics; a
+// tuple is rejected at its first failing parameter).  Valid tuples are counted.
+__global__ void filter_product_kernel(const __grid_constant__ ProductArgs a, unsigned long long* count) {
+  const uint64_t t = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const uint64_t b = t * a.chunk;
+  unsigned long long ok = 0;
+  if (b < a.total) {
+    const uint64_t e = min(b + a.chunk, a.total);
+    const int P = a.n_params;
+    int32_t pos[kMaxLevels];
+    int64_t val[kMaxLevels];
+    uint64_t rem = b;
+    for (int p = P - 1; p >= 0; p--) {
+      const uint64_t rp = (uint64_t)a.r[p];
+      pos[p] = (int32_t)(rem % rp);
+      rem /= rp;
+      val[p] = __ldg(a.range[p] + pos[p]);
+    }
+    for (uint64_t i = b; i < e; i++) {
+      bool good = true;
+      for (int p = 0; p < P && good; p++) {
+        for (int q = a.prog_first[p]; q < a.prog_first[p] + a.prog_count[p] && good; q++) {  // ANDed
+          bool poison = false;
+          const int64_t v = run_code(a.code + __ldg(a.progs + 2 * q), __ldg(a.progs + 2 * q + 1), val[p], val, 1, poison);
+          good = !poison && v != 0;
+        }
+      }
+      ok += good;
+      for (int p = P - 1; p >= 0; p--) {  // odometer
+        if (++pos[p] < a.r[p]) {
+          val[p] = __ldg(a.range[p] + pos[p]);
+          break;
+        }
+        pos[p] = 0;
+        val[p] = __ldg(a.range[p]);
+      }
+    }
+  }
+  ok = warp_sum_u64(ok);
+  if ((threadIdx.x & 31) == 0 && ok) atomicAdd(count, ok);
+}
+
+int launch_filter_product(const ProductArgs& a, unsigned long long* count, void* stream) {
+  if (a.total == 0) return 0;
+  const uint64_t threads = (a.total + a.chunk - 1) / a.chunk;
+  const uint64_t blocks = (threads + 255) / 256;
+  if (blocks > 0x7fffffffull) return (int)cudaErrorInvalidValue;
+  filter_product_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, count);
+  return (int)cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- standalone scan (tests)
 // Exclusive scan u32 -> u64 with the same look-back as expand_kernel; out[n] = total.
 __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restrict__ out, int64_t n,

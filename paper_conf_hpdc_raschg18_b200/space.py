@@ -243,6 +243,14 @@ class Space:
                 self._h)
         return dig
 
+    def filter_product(self):
+        """CLTune-style baseline: count the valid tuples of the FULL cartesian
+        product on the GPU (every tuple enumerated, every constraint interpreted).
+        Returns (valid tuples = S, product size)."""
+        cnt, tot = C.c_uint64(), C.c_uint64()
+        L.check(L.atf_space_filter_product(self._h, C.byref(cnt), C.byref(tot)), self._h)
+        return cnt.value, tot.value
+
     def neighbors(self, values, seed: int, max_tries: int = 16, stream=None):
         """values: int32 CUDA tensor [P, n] of valid configurations -> (int32 [P, n] neighbours,
         int32 [n] changed parameter id or -1); one parameter re-drawn per row."""

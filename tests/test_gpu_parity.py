@@ -344,3 +344,29 @@ def test_encode_fuzz_membership(Space, seed):
         if S and S < (1 << 63):
             idx = torch.arange(min(S, 4096), dtype=torch.int64, device="cuda")
             assert torch.equal(sp.encode(sp.decode(idx)), idx)
+
+
+# ---------------------------------------------------------------- CLTune-style full-product filter
+@pytest.mark.parametrize("name", ["C1", "fig1", "saxpy360", "C2-8", "C3-4x5x3", "C3-3x4x2-anch"])
+def test_filter_product_counts_the_space(Space, name):
+    """P:183: filtering the full product yields the same set as ATF's constrained ranges;
+    here its size, against the oracle's O1 (literal brute force) and the tree generator."""
+    spec = {"C1": A.c1_toy, "fig1": A.fig1, "saxpy360": lambda: A.saxpy(360),
+            "C2-8": lambda: A.c2_xgemm_direct(8), "C3-4x5x3": lambda: A.c3_xgemm((4, 5, 3)),
+            "C3-3x4x2-anch": lambda: A.c3_xgemm((3, 4, 2), anchored=True)}[name]()
+    with Space(spec) as sp:
+        cnt, tot = sp.filter_product()
+        sp.generate()
+        assert cnt == sp.size()
+    o1, _ = orc.o1(spec)
+    assert cnt == int(o1["S"])
+    assert tot == int(np.prod([len(_range_values(p.range)) for p in spec.params], dtype=object))
+
+
+@pytest.mark.parametrize("seed", range(0, 80, 5))
+def test_filter_product_fuzz(Space, seed):
+    spec = A.random_spec(seed)
+    with Space(spec) as sp:
+        cnt, _ = sp.filter_product()
+        sp.generate()
+        assert cnt == sp.size()
