@@ -203,30 +203,43 @@ def roofline_of(res, sm_mhz, spec_name=None):
                      "frac": step_ops / (step_ms * 1e-3) / peak}}
 
 
-def e2e_generation(spec, steps):
-    """Same metric through the public API from HOST inputs: a new space is built from the host
-    spec (ranges + bytecode uploaded), generated, and S + group sizes read back, every step."""
+def e2e_generation(spec, steps, dist_ctx=None):
+    """Same metric through the public API from HOST inputs: every step builds a new space from
+    the host spec (ranges + bytecode uploaded), generates it (sharded over the ranks when
+    world > 1, counts all-gathered over NCCL) and reads S + the group sizes back.  Timed by the
+    host clock around device-synchronised steps; max over ranks."""
     import torch
     from paper_conf_hpdc_raschg18_b200 import Space
-    # per parameter the library uploads [values][magics][|values|], each padded to 128
-    # entries (ensure_device); constraint programs travel as kernel parameters
+    # per parameter the library uploads [values][magics][|values|] padded to 128 entries plus
+    # the sorted value table (encode); constraint programs travel as kernel parameters
     h2d = sum(4 * len(c) for p in spec.params for c in p.constraints)
     for p in spec.params:
         r = p.range
         n = len(r["values"]) if r["kind"] == "set" else max(0, (r["end"] - r["begin"]) // r["step"] + 1)
-        h2d += 12 * ((n + 127) // 128 * 128)
+        h2d += 12 * ((n + 127) // 128 * 128) + 8 * n
     times, d2h = [], 0
     for i in range(steps + 1):
         torch.cuda.synchronize()
+        if dist_ctx:
+            dist_ctx["dist"].barrier()
         t0 = time.perf_counter()
         with Space(spec) as sp:
-            sp.generate()
+            if dist_ctx:
+                from paper_conf_hpdc_raschg18_b200.shard import generate_sharded
+                generate_sharded(sp)
+            else:
+                sp.generate()
             S = sp.size()
             gs = sp.group_sizes()
             nlev = sum(sp.num_levels(g) for g in range(len(gs)))
         torch.cuda.synchronize()
+        dt = time.perf_counter() - t0
+        if dist_ctx:
+            t = torch.tensor([dt], dtype=torch.float64, device="cuda")
+            dist_ctx["dist"].all_reduce(t, op=dist_ctx["dist"].ReduceOp.MAX)
+            dt = float(t.item())
         if i:
-            times.append(time.perf_counter() - t0)
+            times.append(dt)
         d2h = 12 * nlev
     return {"s_per_step": float(np.mean(times)), "h2d": h2d, "d2h": d2h, "S": S}
 
@@ -369,31 +382,30 @@ def main():
     # our kernels per step: every non-empty level launches expand_narrow (r <= 64) or
     # expand_wide, then scan_kernel and level_emit_kernel
     n_launch = 3 * sum(1 for s in res["stats"] if s["ms"] >= 0)
+    e2e = e2e_generation(spec, max(2, a.steps // 2), dist_ctx)
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "configs/s", "n_gpus": world, "steps": a.steps,
                 "warmup": a.warmup, "ms_per_step": ms, "higher_is_better": True,
                 "scaling": "strong", "vs_baseline": None, "dtype": "int64 (int32 values, 16/32-bit magics)",
                 "data": "synthetic (deterministic spec, no dataset)", "config": config,
                 "S": str(res["size"]), "group_leaves": res["group_sizes"], "gpu_launches": n_launch * a.steps,
-                "clocks": clocks}
+                "clocks": clocks,
+                "e2e": {"value": leaves / e2e["s_per_step"], "unit": "configs/s",
+                        "h2d_bytes_per_step": e2e["h2d"], "d2h_bytes_per_step": e2e["d2h"],
+                        "s_per_step": e2e["s_per_step"]}}
         if world == 1:
             evals_total = sum(s["evals"] for s in res["stats"])
             line["evals_per_s"] = evals_total / (ms * 1e-3)
             line["roofline"] = roofline_of(res, sm_max, spec.name)
             line["roofline_at_load_clock"] = (roofline_of(res, clocks["sm_mhz"], spec.name)["frac"]
                                               if clocks.get("sm_mhz") else None)
-            e2e = e2e_generation(spec, max(2, a.steps // 2))
-            line["e2e"] = {"value": leaves / e2e["s_per_step"], "unit": "configs/s",
-                           "h2d_bytes_per_step": e2e["h2d"], "d2h_bytes_per_step": e2e["d2h"],
-                           "s_per_step": e2e["s_per_step"]}
+
             try:
                 line["cpu_baseline"] = cpu_baseline(spec, budget_s=a.cpu_budget)
             except Exception as ex:  # noqa: BLE001
                 line["cpu_baseline"] = {"error": str(ex)}
             if not a.no_secondary:
                 line["secondary"] = secondary_n1(max(3, a.steps // 2), 3, sm_max)
-        else:
-            line["e2e"] = None
         print(json.dumps(line), flush=True)
     if dist_ctx:
         dist_ctx["dist"].barrier()

@@ -370,3 +370,45 @@ def test_filter_product_fuzz(Space, seed):
         cnt, _ = sp.filter_product()
         sp.generate()
         assert cnt == sp.size()
+
+
+# ---------------------------------------------------------------- multi-GPU protocol, virtual ranks
+@pytest.mark.parametrize("world", [2, 3, 8])
+@pytest.mark.parametrize("name", ["C5-300x4", "C3-IS1", "C2-256", "C5-4096x3"])
+def test_virtual_shards_concatenate_to_single_gpu(Space, world, name):
+    """S§8(e) on one GPU: `world` spaces each expand their rank's slice (generate_shard), the
+    counts are exchanged (here in-process instead of NCCL) and finalize_shard fixes global
+    offsets.  Every rank reports the global group sizes, and the rank slices of every level,
+    in rank order, are the single-GPU arrays bit for bit."""
+    spec = SMALL[name]()
+    with Space(spec) as one:
+        one.generate()
+        G = one.num_groups()
+        ref = {(g, k): one.level_tensors(g, k)[0].clone() for g in range(G) for k in range(one.num_levels(g))}
+        sizes = one.group_sizes()
+    shards = [Space(spec) for _ in range(world)]
+    try:
+        counts = [sp.generate_shard(r, world) for r, sp in enumerate(shards)]
+        for sp in shards:
+            sp.finalize_shard(counts)
+        for sp in shards:
+            assert sp.group_sizes() == sizes
+        for (g, k), want in ref.items():
+            parts = []
+            for sp in shards:
+                v = sp.level_view(g, k)
+                rec, _ = sp.level_tensors(g, k)
+                parts.append((v["offset"], rec))
+            if all(off == 0 and rec.shape[0] == want.shape[0] for off, rec in parts):
+                for _, rec in parts:          # replicated prefix level
+                    assert torch.equal(rec, want)
+                continue
+            parts.sort(key=lambda t: t[0])
+            pos = 0
+            for off, rec in parts:
+                assert off == pos, (g, k)
+                pos += rec.shape[0]
+            assert torch.equal(torch.cat([rec for _, rec in parts]), want), (g, k)
+    finally:
+        for sp in shards:
+            sp.close()
