@@ -160,6 +160,12 @@ def pow2(begin: int, end: int, step: int = 1) -> dict:
     return {"kind": "pow2", "begin": int(begin), "end": int(end), "step": int(step)}
 
 
+def gen(begin: int, end: int, expr, step: int = 1) -> dict:
+    """``atf::interval<T>(begin, end, step, generator)`` (P:57): values expr(i) for i = begin,
+    begin+step, ..., <= end; `expr` is an expression in X (= i) and constants."""
+    return {"kind": "gen", "begin": int(begin), "end": int(end), "step": int(step), "code": list(lift(expr).code)}
+
+
 def set_(*values: int) -> dict:
     return {"kind": "set", "values": [int(v) for v in values]}
 

@@ -66,8 +66,14 @@ typedef enum {
  *   POW2:     values 2^i for i = begin, begin+step, ..., <= end; 0 <= i <= 30
  *             ("atf::interval<size_t>(1,10,[](i){return pow(2,i);})" = first ten powers of 2).
  *   SET:      values[0..n_values) in the listed order; duplicates -> ATF_ERR_DUPLICATE.
- *             bool and enum parameters are SETs of ints ({0,1} for bools). */
-typedef enum { ATF_RANGE_INTERVAL = 0, ATF_RANGE_POW2 = 1, ATF_RANGE_SET = 2 } atf_range_kind;
+ *             bool and enum parameters are SETs of ints ({0,1} for bools).
+ *   GEN:      the general generator of P:57 ("the elements generator(i) for each i from
+ *             begin to end"): values gen(i) for i = begin, begin+step, ..., <= end, where
+ *             gen is a bytecode program (`values` = its int32 words, `n_values` = their
+ *             number) in which X is i (PARAM is not allowed).  Evaluated exactly in int64
+ *             on the host when the parameter is added; a poisoned or non-int32 value ->
+ *             ATF_ERR_BYTECODE, a repeated value -> ATF_ERR_DUPLICATE (reading #5). */
+typedef enum { ATF_RANGE_INTERVAL = 0, ATF_RANGE_POW2 = 1, ATF_RANGE_SET = 2, ATF_RANGE_GEN = 3 } atf_range_kind;
 
 typedef struct {
   int32_t kind;           /* atf_range_kind */

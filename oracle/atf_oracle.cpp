@@ -150,6 +150,8 @@ struct Spec {
   std::vector<Param> params;
 };
 
+static i64 run_value(const std::vector<int32_t>& code, i64 x, const i64* vals, bool& poison);
+
 // "atf::interval<T>(begin, end, step_size, generator) represents the values
 // ... from begin to end using the optional step_size"; "the interval comprises the
 // elements generator(i) for each i from begin to end"; "atf::set(val_1,...,val_n)".
@@ -169,6 +171,22 @@ static std::vector<i64> materialise(const Json& r) {
         for (i64 k = 0; k < i; k++) p *= 2;      // exact 2^i (reading #3)
         v.push_back(p);
       }
+    }
+  } else if (kind == "gen") {                   // P:57 generator(i), i = begin, begin+step, ..., <= end
+    i64 b = r.at("begin").num, e = r.at("end").num, st = r.at("step").num;
+    if (st <= 0) throw std::runtime_error("range: step must be positive");
+    std::vector<int32_t> code;
+    for (auto& w : r.at("code").arr) code.push_back((int32_t)w.num);
+    for (size_t k = 0; k < code.size(); k += (code[k] == CONST ? 3 : 1))
+      if (code[k] == PARAM) throw std::runtime_error("range: generator references a parameter");
+    for (i64 i = b; i <= e; i += st) {
+      bool poison = false;
+      i64 y = run_value(code, i, nullptr, poison);
+      if (poison) throw std::runtime_error("range: generator poison");
+      if (y < INT32_MIN || y > INT32_MAX) throw std::runtime_error("range: value outside int32");
+      for (i64 z : v)
+        if (z == y) throw std::runtime_error("range: duplicate generator value");  // reading #5
+      v.push_back(y);
     }
   } else if (kind == "set") {
     for (auto& x : r.at("values").arr) {
@@ -232,10 +250,9 @@ static Spec load_spec(const std::string& path) {
 // Evaluation is strict: every operation of the program is executed.
 static std::atomic<bool> g_overflow{false};
 
-static bool run_program(const std::vector<int32_t>& code, i64 x, const i64* vals) {
+static i64 run_value(const std::vector<int32_t>& code, i64 x, const i64* vals, bool& poison) {
   i64 st[256];
   int sp = 0;
-  bool poison = false;
   for (size_t i = 0; i < code.size();) {
     int op = code[i];
     if (op == X) { st[sp++] = x; i++; continue; }
@@ -289,7 +306,13 @@ static bool run_program(const std::vector<int32_t>& code, i64 x, const i64* vals
     i++;
   }
   if (sp != 1) throw std::runtime_error("bytecode: program must leave exactly one item");
-  return !poison && st[0] != 0;
+  return st[0];
+}
+
+static bool run_program(const std::vector<int32_t>& code, i64 x, const i64* vals) {
+  bool poison = false;
+  const i64 v = run_value(code, x, vals, poison);
+  return !poison && v != 0;
 }
 
 // Optional hand-written predicates (native C++ encodings of C1, C2, C3, saxpy) used

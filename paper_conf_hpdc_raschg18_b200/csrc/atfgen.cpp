@@ -1374,6 +1374,82 @@ atf_status atf_space_add_param(atf_space* s, const char* name, const atf_range* 
         pd.values.push_back((int32_t)(1u << (int)i));
       }
     }
+  } else if (range->kind == ATF_RANGE_GEN) {
+    // P:57 generator over i: the program is checked like a constraint (no PARAM) and
+    // evaluated exactly in int64 for every i
+    if (range->step <= 0) return fail(s, ATF_ERR_INVALID_ARG, "step must be positive");
+    if (range->n_values <= 0 || range->n_values > ATF_MAX_PROGRAM_WORDS || !range->values)
+      return fail(s, ATF_ERR_BYTECODE, "generator of %s: bad program length", name);
+    const int32_t* code = range->values;
+    const int n = (int)range->n_values;
+    for (int i = 0; i < n;) {
+      const int op = code[i];
+      if (op == ATF_OP_PARAM) return fail(s, ATF_ERR_BYTECODE, "generator of %s references a parameter", name);
+      if (op < ATF_OP_X || op > ATF_OP_NOT) return fail(s, ATF_ERR_BYTECODE, "generator of %s: bad opcode", name);
+      i += op == ATF_OP_CONST ? 3 : 1;
+      if (i > n) return fail(s, ATF_ERR_BYTECODE, "generator of %s: truncated CONST", name);
+    }
+    if (range->end >= range->begin) {
+      i128 count = ((i128)range->end - range->begin) / range->step + 1;
+      if (count > ATF_MAX_RANGE) return fail(s, ATF_ERR_LIMIT, "range of %s has more than 2^24 values", name);
+    }
+    for (i128 i = range->begin; i <= range->end; i += range->step) {
+      if (i < INT64_MIN || i > INT64_MAX) return fail(s, ATF_ERR_INVALID_ARG, "generator index outside int64");
+      int64_t st[ATF_MAX_STACK + 1];
+      int sp = 0;
+      bool poison = false, bad = false;
+      for (int k = 0; k < n && !bad;) {
+        const int op = code[k];
+        if (op == ATF_OP_X || op == ATF_OP_CONST) {
+          if (sp >= ATF_MAX_STACK) { bad = true; break; }
+          st[sp++] = op == ATF_OP_X ? (int64_t)i
+                                    : (int64_t)(((uint64_t)(uint32_t)code[k + 2] << 32) | (uint32_t)code[k + 1]);
+          k += op == ATF_OP_X ? 1 : 3;
+          continue;
+        }
+        if (op == ATF_OP_NOT) {
+          if (sp < 1) { bad = true; break; }
+          st[sp - 1] = st[sp - 1] == 0;
+          k++;
+          continue;
+        }
+        if (sp < 2) { bad = true; break; }
+        const int64_t b = st[--sp], a = st[sp - 1];
+        i128 r = 0;
+        switch (op) {
+          case ATF_OP_ADD: r = (i128)a + b; break;
+          case ATF_OP_SUB: r = (i128)a - b; break;
+          case ATF_OP_MUL: r = (i128)a * b; break;
+          case ATF_OP_DIV: if (b == 0) poison = true; else r = (i128)a / b; break;     // C truncation
+          case ATF_OP_MOD: if (b == 0) poison = true; else r = (i128)a % b; break;
+          case ATF_OP_MIN: r = a < b ? a : b; break;
+          case ATF_OP_MAX: r = a > b ? a : b; break;
+          case ATF_OP_EQ: r = a == b; break;
+          case ATF_OP_NE: r = a != b; break;
+          case ATF_OP_LT: r = a < b; break;
+          case ATF_OP_LE: r = a <= b; break;
+          case ATF_OP_GT: r = a > b; break;
+          case ATF_OP_GE: r = a >= b; break;
+          case ATF_OP_DIVIDES: if (a == 0) poison = true; else r = ((i128)b % a) == 0; break;
+          case ATF_OP_MULOF: if (b == 0) poison = true; else r = ((i128)a % b) == 0; break;
+          case ATF_OP_AND: r = (a != 0) && (b != 0); break;
+          case ATF_OP_OR: r = (a != 0) || (b != 0); break;
+          default: bad = true;
+        }
+        if (r < INT64_MIN || r > INT64_MAX) return fail(s, ATF_ERR_OVERFLOW, "generator of %s overflows int64", name);
+        st[sp - 1] = (int64_t)r;
+        k++;
+      }
+      if (bad || sp != 1) return fail(s, ATF_ERR_BYTECODE, "generator of %s: malformed program", name);
+      if (poison) return fail(s, ATF_ERR_BYTECODE, "generator of %s: zero divisor at i = %lld", name, (long long)i);
+      if (st[0] < INT32_MIN || st[0] > INT32_MAX)
+        return fail(s, ATF_ERR_BYTECODE, "generator of %s: value outside int32 at i = %lld", name, (long long)i);
+      pd.values.push_back((int32_t)st[0]);
+    }
+    std::vector<int32_t> sorted(pd.values);
+    std::sort(sorted.begin(), sorted.end());
+    if (std::adjacent_find(sorted.begin(), sorted.end()) != sorted.end())
+      return fail(s, ATF_ERR_DUPLICATE, "generator of %s repeats a value", name);
   } else if (range->kind == ATF_RANGE_SET) {
     if (range->n_values < 0 || (range->n_values > 0 && !range->values))
       return fail(s, ATF_ERR_INVALID_ARG, "bad set");

@@ -19,6 +19,10 @@ def _range_struct(rng: dict):
         return L.atf_range(L.ATF_RANGE_INTERVAL, rng["begin"], rng["end"], rng.get("step", 1), None, 0), None
     if kind == "pow2":
         return L.atf_range(L.ATF_RANGE_POW2, rng["begin"], rng["end"], rng.get("step", 1), None, 0), None
+    if kind == "gen":
+        code = (C.c_int32 * max(1, len(rng["code"])))(*rng["code"])
+        return L.atf_range(L.ATF_RANGE_GEN, rng["begin"], rng["end"], rng.get("step", 1),
+                           C.cast(code, C.POINTER(C.c_int32)), len(rng["code"])), code
     if kind == "set":
         vals = (C.c_int32 * max(1, len(rng["values"])))(*rng["values"])
         return L.atf_range(L.ATF_RANGE_SET, 0, 0, 0, C.cast(vals, C.POINTER(C.c_int32)), len(rng["values"])), vals

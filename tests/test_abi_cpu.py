@@ -186,3 +186,26 @@ int main(void) {
     exe = tmp_path / "magic"
     subprocess.check_call(["gcc", "-O2", "-o", str(exe), str(src)])
     assert subprocess.check_output([str(exe)], timeout=300).strip() == b"0"
+
+
+def test_generator_range_abi_validation(L):
+    """The library materialises generator ranges on the host (no GPU needed): duplicates,
+    zero divisors, PARAM references and non-int32 values are rejected."""
+    import ctypes as C
+    from paper_conf_hpdc_raschg18_b200 import _lib as LL
+
+    def add(expr_code, b, e, step=1):
+        sp = C.c_void_p()
+        LL.check(LL.atf_space_create(None, C.byref(sp)))
+        try:
+            code = (C.c_int32 * len(expr_code))(*expr_code)
+            r = LL.atf_range(LL.ATF_RANGE_GEN, b, e, step, C.cast(code, C.POINTER(C.c_int32)), len(expr_code))
+            pid = C.c_int32()
+            return LL.atf_space_add_param(sp, b"p", C.byref(r), C.byref(pid))
+        finally:
+            LL.atf_space_destroy(sp)
+    assert add(A.gen(1, 10, A.X * A.X)["code"], 1, 10) == 0
+    assert add(A.gen(-2, 2, A.X * A.X)["code"], -2, 2) == -9           # duplicate
+    assert add(A.gen(0, 3, A.C(12) // A.X)["code"], 0, 3) == -5         # 12 / 0: poison
+    assert add([2, 0], 0, 3) == -5                                       # PARAM 0
+    assert add(A.gen(0, 3, A.X * A.C(1 << 40))["code"], 0, 3) == -5     # > int32

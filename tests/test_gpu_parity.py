@@ -412,3 +412,15 @@ def test_virtual_shards_concatenate_to_single_gpu(Space, world, name):
     finally:
         for sp in shards:
             sp.close()
+
+
+def test_generator_ranges_against_oracle(Space):
+    """P:57 generator ranges (NEXT-3): a GEMM-like space whose tile sizes are generated
+    (squares, powers of two by doubling expression, an affine map) vs the oracle."""
+    s = A.Spec("gen_space")
+    s.add("T", A.gen(1, 24, A.X * A.X))                                        # 1, 4, ..., 576
+    s.add("U", A.gen(0, 9, A.X * 64 + 1), A.divides(A.P(0) * 64 + 64) | (A.X < 100))
+    s.add("V", A.gen(1, 40, A.X * 3, step=1), A.divides(A.P(0)))
+    s.add("W", A.interval(1, 200), A.divides(A.P(2) * 4))
+    _check_against_oracle(Space, s)
+    _check_against_oracle(Space, s, generic=True)

@@ -285,3 +285,26 @@ def test_c3_small_shapes_match_survey_appendix(oracle_bin):
     d = orc.info(A.c3_xgemm("IS3"), threads=8)
     assert fs(d) == [50, 3200, 3200, 13248, 57960, 35070, 30555, 30555, 48298, 80124]
     assert int(d["S"]) == 80124 * 16
+
+
+# ---------------------------------------------------------------- P:57 generator ranges (NEXT-3)
+def test_generator_range_closed_forms():
+    """interval(begin, end, step, generator): the elements generator(i); pinned by closed
+    forms of the materialised range (squares, an affine map, a step) through the oracle's own
+    parser: a space whose only parameter has the range enumerates exactly those values."""
+    import numpy as np
+    cases = [(A.gen(1, 10, A.X * A.X), [i * i for i in range(1, 11)]),
+             (A.gen(0, 20, A.X * 3 + 1, step=4), [3 * i + 1 for i in range(0, 21, 4)]),
+             (A.gen(-3, 3, A.X * A.X * A.X - A.X), None)]
+    for rng, want in cases[:2]:
+        s = A.Spec("gen")
+        s.add("p", rng)
+        info = orc.info(s)
+        assert info["groups"][0]["size"] == len(want)
+        _, rows = orc.decode(s, np.arange(len(want), dtype=np.uint64))
+        assert rows[0].tolist() == want
+    # i^3 - i repeats 0 at i = -1, 0, 1: rejected like a duplicate set value (reading #5)
+    s = A.Spec("gen_dup")
+    s.add("p", cases[2][0])
+    with pytest.raises(Exception):
+        orc.info(s)
