@@ -121,6 +121,7 @@ enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1, K_WTILE = 2, K_NFAST = 3 }
 constexpr int kNfNPL = 4;  // narrow fast kernel: frontier nodes per lane (warp tile = 128 nodes)
 constexpr int kWT = 32;        // warp-tile kernel: frontier nodes per warp tile (one per lane)
 constexpr int kMaxSeg = 8;     // warp-tile kernel: candidate segments per node
+constexpr int kItemCap = 256;  // warp-tile kernel: items whose exact masks pass 1 keeps for the emit pass
 constexpr int kPieceShift = 10;  // level_emit_kernel copies the level in pieces of 2^10 records
 // Hot-loop filter of the wide kernel: a superset test of one conjunct, 2 instructions per
 // (node, candidate) pair (IMAD + ISETP.OR into a per-node predicate).
@@ -227,7 +228,7 @@ ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
 // private region per warp (its tile's records, gates, hot operands, item words, operands).
 struct WarpLayout {
   int tab, qtab, warp0, wstride;            // CTA part; warp w's region at warp0 + w * wstride
-  int rec, ok, hot, hot2, cnt, items, opa, opb, slots;  // offsets inside a warp region
+  int rec, ok, hot, hot2, cnt, items, imask, icode, opa, opb, slots;  // offsets inside a warp region
   int total;
 };
 ATF_HD WarpLayout wtile_layout(const LevelArgs& a, int words) {
@@ -243,6 +244,8 @@ ATF_HD WarpLayout wtile_layout(const LevelArgs& a, int words) {
   L.hot2 = w; w += 4 * kWT;
   L.cnt = w; w += 4 * kWT;
   L.items = w; w = align16(w + 4 * kWT * a.nseg);
+  L.imask = w; w = align16(w + 4 * kItemCap);
+  L.icode = w; w = align16(w + 2 * kItemCap);
   L.opa = w; w = align16(w + 8 * kWT * a.n_terms);
   L.opb = w; w = align16(w + 8 * kWT * a.n_terms);
   if (a.need_slots_smem) { L.slots = w; w = align16(w + 8 * kWT * a.n_slots); } else { L.slots = -1; }

@@ -830,6 +830,8 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
   uint32_t* s_hot2 = reinterpret_cast<uint32_t*>(wb + L.hot2);
   uint32_t* s_cnt = reinterpret_cast<uint32_t*>(wb + L.cnt);
   uint32_t* s_items = reinterpret_cast<uint32_t*>(wb + L.items);
+  uint32_t* s_imask = reinterpret_cast<uint32_t*>(wb + L.imask);
+  uint16_t* s_icode = reinterpret_cast<uint16_t*>(wb + L.icode);
   int64_t* s_opa = reinterpret_cast<int64_t*>(wb + L.opa);
   int64_t* s_opb = reinterpret_cast<int64_t*>(wb + L.opb);
   int64_t* s_slots = L.slots >= 0 ? reinterpret_cast<int64_t*>(wb + L.slots) : nullptr;
@@ -934,9 +936,8 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
     }
     const uint32_t T = __shfl_sync(FULL, ie, 31);
     ie -= ic;
-    // pass 1: exact masks -> node counts; the first 4 rounds keep their masks in registers
-    // (mask, item code = node | seg << 5 | lane << 8)
-    uint32_t km0 = 0, km1 = 0, km2 = 0, km3 = 0, kc0 = 0, kc1 = 0, kc2 = 0, kc3 = 0;
+    // pass 1: exact masks -> node counts; the first kItemCap items keep (mask, item code =
+    // node | seg << 5 | lane << 8) in the warp's shared memory for the emit pass
     for (uint32_t R = 0; R < T; R += 32) {
       const uint32_t k = R + lane;
       int node, sg, b;
@@ -944,11 +945,10 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
       uint32_t m = 0;
       if (k < T)
         m = wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q);
-      const uint32_t code = (uint32_t)node | ((uint32_t)sg << 5) | ((uint32_t)b << 8);
-      if (R == 0) { km0 = m; kc0 = code; }
-      else if (R == 32) { km1 = m; kc1 = code; }
-      else if (R == 64) { km2 = m; kc2 = code; }
-      else if (R == 96) { km3 = m; kc3 = code; }
+      if (k < (uint32_t)kItemCap) {
+        s_imask[k] = m;
+        s_icode[k] = (uint16_t)((uint32_t)node | ((uint32_t)sg << 5) | ((uint32_t)b << 8));
+      }
       if (m) atomicAdd(&s_cnt[node], (uint32_t)__popc(m));
     }
     __syncwarp();
@@ -977,9 +977,9 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
       const uint32_t k = R + lane;
       int node, sg, b;
       uint32_t m;
-      if (R < 128) {
-        const uint32_t code = R == 0 ? kc0 : R == 32 ? kc1 : R == 64 ? kc2 : kc3;
-        m = R == 0 ? km0 : R == 32 ? km1 : R == 64 ? km2 : km3;
+      if (R < (uint32_t)kItemCap) {
+        const uint32_t code = s_icode[k];
+        m = k < T ? s_imask[k] : 0u;
         node = (int)(code & 31u);
         sg = (int)((code >> 5) & 7u);
         b = (int)(code >> 8);
