@@ -783,9 +783,13 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
       a.cpt = best_cpt;
       a.nseg = best_nseg;
       a.chunk = 32 * best_cpt * best_nseg;
-      a.tile_nodes = kWT;
+      // small frontiers: fewer nodes per warp tile (power of two, >= 4 = one node quad of
+      // the hot loop) so that at least ~4 warp tiles per SM exist
+      int tnodes = kWT;
+      while (tnodes > 4 && (a.n_parents + tnodes - 1) / tnodes < 148ull * 4) tnodes >>= 1;
+      a.tile_nodes = tnodes;
       // 8 warps per CTA unless the level has too few tiles to give every SM a full CTA
-      const uint64_t tiles = (a.n_parents + kWT - 1) / kWT;
+      const uint64_t tiles = (a.n_parents + tnodes - 1) / tnodes;
       const uint64_t per_sm = (tiles + 147) / 148;
       a.block = 32 * (int)std::min<uint64_t>(8, std::max<uint64_t>(1, per_sm));
       a.smem_bytes = wtile_layout(a, words).total;

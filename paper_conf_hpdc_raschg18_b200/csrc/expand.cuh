@@ -749,6 +749,7 @@ __device__ __forceinline__ uint32_t wtile_item_mask(const LevelArgs& a, int i, i
                                      : (left > 0 ? ((1u << left) - 1u) : 0u);
   uint32_t mask = 0;
   if (HOT == HOT_NONE) {
+    if (a.n_terms == 0) return valid;  // unconstrained level (node gates already applied)
 #pragma unroll 4
     for (int c = 0; c < CPT; c++)
       if (((valid >> c) & 1u) &&
@@ -807,6 +808,7 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
   const WarpLayout L = wtile_layout(a, W);
   const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
   const int nseg = a.nseg, r = a.r, hot_t = a.hot_term;
+  const int TN = a.tile_nodes;  // nodes per warp tile (power of two <= kWT; small levels use fewer)
   uint32_t* s_tab = L.tab >= 0 ? reinterpret_cast<uint32_t*>(smem + L.tab) : nullptr;
   uint32_t* s_q = L.qtab >= 0 ? reinterpret_cast<uint32_t*>(smem + L.qtab) : nullptr;
   if (HOT != HOT_NONE) {
@@ -851,9 +853,9 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
   uint32_t pre[W];
   uint64_t pre_tile = ~0ull;
   while ((uint64_t)cur < a.n_tiles) {
-    const uint64_t node0 = (uint64_t)cur * kWT;
+    const uint64_t node0 = (uint64_t)cur * TN;
     const uint64_t remn = a.n_parents - node0;
-    const int tn = remn < (uint64_t)kWT ? (int)remn : kWT;
+    const int tn = remn < (uint64_t)TN ? (int)remn : TN;
     // ---- prologue: lane = node
     bool ok = false;
     if (lane < tn) {
@@ -878,8 +880,8 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
     if (lane == 0 && (uint64_t)nxt < a.n_tiles) nn = atomicAdd(a.tile_counter, 1u);
     nn = __shfl_sync(FULL, nn, 0);
     if (a.level > 0 && (uint64_t)nxt < a.n_tiles) {
-      const uint64_t n1 = (uint64_t)nxt * kWT + lane;
-      if (n1 < a.n_parents) {
+      const uint64_t n1 = (uint64_t)nxt * TN + lane;
+      if (lane < TN && n1 < a.n_parents) {
         load_record<W>(a.parent_rec + n1 * W, pre);
         pre_tile = nxt;
       }
