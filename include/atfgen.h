@@ -102,6 +102,8 @@ typedef struct {
                                      candidate with the generic bytecode interpreter     */
 #define ATF_FLAG_LEGACY_WIDE 8u   /* levels with r > 64 use the block-tile kernel instead of
                                      the warp-tile kernel (kept for parity coverage)      */
+#define ATF_FLAG_NO_JIT 16u       /* narrow fast levels use the generic kernel instead of the
+                                     NVRTC-specialised one (kept for parity coverage)     */
 #define ATF_FLAG_KEEP_LEVELS 4u   /* keep inner-level arrays (CSR + records); default
                                      keeps them too — reserved                          */
 
@@ -267,7 +269,8 @@ typedef struct {
   float ms;         /* device time of the level (ATF_FLAG_TIMING), else -1 */
   int32_t path;     /* 0 = fast atoms, 1 = generic interpreter */
   float expand_ms;  /* device time of the level's expand kernel alone (ATF_FLAG_TIMING), else -1 */
-  int32_t kernel;   /* expand kernel: 0 = narrow (r <= 64), 1 = block-tile wide, 2 = warp-tile wide */
+  int32_t kernel;   /* expand kernel: 0 = narrow (r <= 64), 1 = block-tile wide, 2 = warp-tile wide,
+                       3 = narrow fast, 4 = narrow fast specialised at run time (NVRTC) */
 } atf_level_stats;
 atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap, int32_t* n_out);
 

@@ -26,6 +26,9 @@ atf_status atf_test_shard_slice(const uint64_t* h_csr, uint64_t ncut, int32_t ra
                                 uint64_t* hi);
 atf_status atf_test_shard_offsets(const int64_t* h_all, int32_t world, int32_t n, int32_t rank, uint64_t* before,
                                   uint64_t* tot);
+/* Source text of the NVRTC-specialised pass-1 kernel of level k of group g (empty when the
+ * level is not a narrow fast level); plans the space if needed.  Host only. */
+atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, size_t cap, size_t* len_out);
 #ifdef __cplusplus
 }
 #endif

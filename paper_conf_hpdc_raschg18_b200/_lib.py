@@ -24,7 +24,7 @@ STATUS = {0: "ATF_OK", -1: "ATF_ERR_INVALID_ARG", -2: "ATF_ERR_OOM", -3: "ATF_ER
           -5: "ATF_ERR_BYTECODE", -6: "ATF_ERR_FORWARD_REF", -7: "ATF_ERR_OVERFLOW", -8: "ATF_ERR_INDEX",
           -9: "ATF_ERR_DUPLICATE", -10: "ATF_ERR_LIMIT"}
 ATF_RANGE_INTERVAL, ATF_RANGE_POW2, ATF_RANGE_SET, ATF_RANGE_GEN = 0, 1, 2, 3
-ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE = 1, 2, 8
+ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT = 1, 2, 8, 16
 
 
 class atf_range(C.Structure):
@@ -86,6 +86,7 @@ _SIGS = {
     "atf_status_str": (C.c_char_p, [_st]),
     "atf_space_last_error": (C.c_char_p, [SP]),
     # include/atfgen_test.h
+    "atf_test_jit_source": (_st, [SP, C.c_int32, C.c_int32, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "atf_test_exclusive_scan_u32": (_st, [C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_test_shard_slice": (_st, [C.POINTER(C.c_uint64), C.c_uint64, C.c_int32, C.c_int32,
                                    C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),

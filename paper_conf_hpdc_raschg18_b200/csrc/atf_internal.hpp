@@ -260,6 +260,18 @@ int launch_expand(const LevelArgs& a, int words, void* stream);
 int expand_smem_bytes(const LevelArgs& a, int words);
 int launch_level_emit(const LevelArgs& a, int words, void* stream);
 int launch_nfast_emit(const LevelArgs& a, int words, void* stream);
+}  // namespace atf
+#include <vector>
+namespace atf {
+// jit.cpp: level-specialised pass-1 kernel of narrow fast levels (NVRTC, sm_100a)
+void* jit_nfast_kernel(const LevelArgs& a, int words, const std::vector<int32_t>& cand_values,
+                       const std::vector<uint32_t>& cand_magics);
+int jit_nfast_launch(void* kernel, const LevelArgs& a, void* stream);
+}  // namespace atf
+#include <string>
+namespace atf {
+std::string jit_nfast_source(const LevelArgs& a, int words, const std::vector<int32_t>& cand_values,
+                             const std::vector<uint32_t>& cand_magics);
 int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out,
                           int64_t ld, unsigned int* bad_flag, void* stream);
 int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,

@@ -65,6 +65,8 @@ struct LevelPlan {
   double cost = 0;           // algorithmic int ops per candidate evaluation (roofline)
   bool generic = false;
   std::string desc;
+  void* jit = nullptr;       // NVRTC-specialised narrow kernel (jit.cpp), if any
+  bool jit_tried = false;
 };
 
 struct GroupPlan {
@@ -1137,10 +1139,22 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   CUDA_TRY(s, cudaMemsetAsync(s->d_ovf + g, 0, 4, st));
   bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].first, st));
-  int ce = launch_expand(a, gp.words, st);
+  if (a.kind == K_NFAST && !lp.jit_tried && !(s->opts.flags & (ATF_FLAG_NO_JIT | ATF_FLAG_LEGACY_WIDE))) {
+    const auto& vals = s->params[lp.param].values;
+    std::vector<uint32_t> mags(vals.size());
+    for (size_t j = 0; j < vals.size(); j++) {
+      const uint32_t ax = vals[j] < 0 ? 0u - (uint32_t)vals[j] : (uint32_t)vals[j];
+      mags[j] = ax ? 0xffffffffu / ax + 1u : 0x10000u;  // ceil(2^32/|x|) mod 2^32 (see ensure_device)
+    }
+    lp.jit = jit_nfast_kernel(a, gp.words, vals, mags);
+    lp.jit_tried = true;
+  }
+  const bool use_jit = a.kind == K_NFAST && lp.jit && !(s->opts.flags & (ATF_FLAG_NO_JIT | ATF_FLAG_LEGACY_WIDE));
+  int ce = use_jit ? jit_nfast_launch(lp.jit, a, st) : launch_expand(a, gp.words, st);
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
+  if (use_jit) s->data[g][k].kernel = 4;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].mid, st));
-  s->data[g][k].kernel = a.kind;
+  if (!use_jit) s->data[g][k].kernel = a.kind;
   if (a.kind == K_NFAST) {
     ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st);
     if (!ce) ce = launch_nfast_emit(a, gp.words, st);
@@ -1984,6 +1998,34 @@ atf_status atf_space_finalize_shard(atf_space* s, const int64_t* all, int32_t wo
       if (k + 1 == s->groups[g].levels.size()) s->gsize[g] = tot;
     }
   s->state = FINAL_SHARD;  // sizes global; decode needs the whole tree (not available)
+  return ATF_OK;
+}
+
+atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, size_t cap, size_t* len_out) {
+  if (!s) return ATF_ERR_INVALID_ARG;
+  atf_status e = plan(s);
+  if (e) return e;
+  if (g < 0 || g >= (int)s->groups.size() || k < 0 || k >= (int)s->groups[g].levels.size()) return ATF_ERR_INVALID_ARG;
+  const GroupPlan& gp = s->groups[g];
+  const LevelPlan& lp = gp.levels[k];
+  LevelArgs a = lp.proto;
+  a.r = lp.r;
+  a.n_parents = 1;
+  choose_geometry(a, gp.words, false);
+  a.mask_bytes = a.r <= 8 ? 1 : (a.r <= 16 ? 2 : 4);
+  const auto& vals = s->params[lp.param].values;
+  std::vector<uint32_t> mags(vals.size());
+  for (size_t j = 0; j < vals.size(); j++) {
+    const uint32_t ax = vals[j] < 0 ? 0u - (uint32_t)vals[j] : (uint32_t)vals[j];
+    mags[j] = ax ? 0xffffffffu / ax + 1u : 0x10000u;
+  }
+  const std::string src = jit_nfast_source(a, gp.words, vals, mags);
+  if (len_out) *len_out = src.size();
+  if (buf && cap) {
+    const size_t n = std::min(cap - 1, src.size());
+    memcpy(buf, src.data(), n);
+    buf[n] = 0;
+  }
   return ATF_OK;
 }
 

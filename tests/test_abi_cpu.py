@@ -209,3 +209,59 @@ def test_generator_range_abi_validation(L):
     assert add(A.gen(0, 3, A.C(12) // A.X)["code"], 0, 3) == -5         # 12 / 0: poison
     assert add([2, 0], 0, 3) == -5                                       # PARAM 0
     assert add(A.gen(0, 3, A.X * A.C(1 << 40))["code"], 0, 3) == -5     # > int32
+
+
+def test_jit_level_sources_compile_for_sm100a(L, tmp_path):
+    """Narrow fast levels are specialised at run time (jit.cpp, NVRTC on the GPU box); here the
+    generated sources of every C1-C3 narrow level (+ fuzz specs) compile with nvcc for sm_100a."""
+    import ctypes as C
+    from paper_conf_hpdc_raschg18_b200 import _lib as LL
+    specs = [A.c1_toy(), A.c2_xgemm_direct(256), A.c3_xgemm("IS2"), A.c3_xgemm("IS4"), A.saxpy(360)]
+    specs += [A.random_spec(s) for s in range(0, 40, 3)]
+    srcs = []
+    for spec in specs:
+        sp = C.c_void_p()
+        LL.check(LL.atf_space_create(None, C.byref(sp)))
+        try:
+            keep = []
+            for p in spec.params:
+                from paper_conf_hpdc_raschg18_b200.space import _range_struct
+                rs, k = _range_struct(p.range)
+                keep.append(k)
+                pid = C.c_int32()
+                LL.check(LL.atf_space_add_param(sp, p.name.encode(), C.byref(rs), C.byref(pid)), sp)
+                for code in p.constraints:
+                    arr = (C.c_int32 * len(code))(*code)
+                    LL.check(LL.atf_space_add_constraint(sp, pid.value, arr, len(code)), sp)
+            LL.check(LL.atf_space_plan(sp), sp)
+            G = C.c_int32()
+            LL.check(LL.atf_space_num_groups(sp, C.byref(G)), sp)
+            for g in range(G.value):
+                nl = C.c_int32()
+                LL.check(LL.atf_space_num_levels(sp, g, C.byref(nl)), sp)
+                for k in range(nl.value):
+                    n = C.c_size_t()
+                    LL.check(LL.atf_test_jit_source(sp, g, k, None, 0, C.byref(n)), sp)
+                    if n.value:
+                        buf = C.create_string_buffer(n.value + 1)
+                        LL.check(LL.atf_test_jit_source(sp, g, k, buf, n.value + 1, None), sp)
+                        srcs.append(buf.value.decode())
+        finally:
+            LL.atf_space_destroy(sp)
+    assert len(srcs) >= 6
+    # one translation unit per source (kernel names collide), compiled in parallel
+    procs = []
+    for i, src in enumerate(srcs):
+        f = tmp_path / f"lvl{i}.cu"
+        f.write_text(src)
+        procs.append(subprocess.Popen(["/usr/local/cuda/bin/nvcc", "-gencode", "arch=compute_100a,code=sm_100a",
+                                       "-std=c++17", "-c", str(f), "-o", str(tmp_path / f"lvl{i}.o")],
+                                      stdout=subprocess.PIPE, stderr=subprocess.STDOUT, text=True))
+        if len(procs) >= 8:
+            for p in procs:
+                out, _ = p.communicate()
+                assert p.returncode == 0, out
+            procs = []
+    for p in procs:
+        out, _ = p.communicate()
+        assert p.returncode == 0, out

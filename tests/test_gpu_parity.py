@@ -52,10 +52,11 @@ def torch_rowhash(rows_pm: "torch.Tensor", base: int = 0) -> int:
     return int(s.item()) & ((1 << 64) - 1)
 
 
-def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, legacy=False):
+def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, legacy=False, no_jit=False):
     from paper_conf_hpdc_raschg18_b200 import _lib as L
     ref = orc.info(spec, threads=8)
-    with Space(spec, flags=_flags(generic) | (L.ATF_FLAG_LEGACY_WIDE if legacy else 0)) as sp:
+    flags = _flags(generic) | (L.ATF_FLAG_LEGACY_WIDE if legacy else 0) | (L.ATF_FLAG_NO_JIT if no_jit else 0)
+    with Space(spec, flags=flags) as sp:
         sp.generate()
         assert sp.groups() == [g["members"] for g in ref["groups"]]
         assert sp.size() == int(ref["S"])
@@ -120,6 +121,26 @@ def test_fuzz_wide_specs(Space, seed):
 def test_fuzz_wide_specs_legacy_kernel(Space, seed):
     """The block-tile wide kernel (ATF_FLAG_LEGACY_WIDE) on the same specs."""
     _check_against_oracle(Space, A.random_wide_spec(seed), legacy=True)
+
+
+@pytest.mark.parametrize("name", ["C1", "C2-256", "C3-IS1", "C3-IS3", "C3-12x30x8", "saxpy360"])
+def test_small_specs_generic_narrow_kernel(Space, name):
+    """The generic (not NVRTC-specialised) narrow fast kernel on the same specs."""
+    _check_against_oracle(Space, SMALL[name](), no_jit=True)
+
+
+@pytest.mark.parametrize("seed", range(0, 80, 9))
+def test_fuzz_specs_generic_narrow_kernel(Space, seed):
+    _check_against_oracle(Space, A.random_spec(seed), no_jit=True)
+
+
+def test_jit_kernels_run(Space):
+    """The narrow levels of C3 run the NVRTC-specialised kernel (kernel id 4) on the GPU box."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    with Space(A.c3_xgemm("IS1"), flags=L.ATF_FLAG_TIMING) as sp:
+        sp.generate()
+        kinds = [st["kernel"] for st in sp.stats()]
+        assert 4 in kinds, kinds
 
 
 @pytest.mark.parametrize("name", ["C3-IS1", "C5-300x4", "C5-4096x3", "C2-256"])
