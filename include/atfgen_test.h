@@ -28,6 +28,9 @@ atf_status atf_test_shard_offsets(const int64_t* h_all, int32_t world, int32_t n
                                   uint64_t* tot);
 /* Source text of the NVRTC-specialised pass-1 kernel of level k of group g (empty when the
  * level is not a narrow fast level); plans the space if needed.  Host only. */
+/* Exhaustive device check of the float-reciprocal divisibility test used for 16-bit quotient
+ * divisors (dev_common.cuh divisible16) against integer modulo: *h_mismatches must be 0. */
+atf_status atf_test_divisible16(uint64_t* h_mismatches);
 atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, size_t cap, size_t* len_out);
 #ifdef __cplusplus
 }

@@ -86,6 +86,7 @@ _SIGS = {
     "atf_status_str": (C.c_char_p, [_st]),
     "atf_space_last_error": (C.c_char_p, [SP]),
     # include/atfgen_test.h
+    "atf_test_divisible16": (_st, [C.POINTER(C.c_uint64)]),
     "atf_test_jit_source": (_st, [SP, C.c_int32, C.c_int32, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "atf_test_exclusive_scan_u32": (_st, [C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_test_shard_slice": (_st, [C.POINTER(C.c_uint64), C.c_uint64, C.c_int32, C.c_int32,

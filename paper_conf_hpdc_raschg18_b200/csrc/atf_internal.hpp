@@ -280,6 +280,7 @@ int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long 
                     unsigned int* counter, void* stream, uint32_t* piece_tile = nullptr,
                     uint64_t piece_cap = 0);
 int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
+int launch_divisible16_check(unsigned long long* mismatches, void* stream);
 int launch_encode(const EncodeArgs& a, const int32_t* vals, int64_t ld, int64_t n, uint64_t* digits, uint64_t* idx,
                   void* stream);
 int launch_filter_product(const ProductArgs& a, unsigned long long* count, void* stream);

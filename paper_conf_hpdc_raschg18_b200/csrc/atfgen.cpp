@@ -2029,6 +2029,19 @@ atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, si
   return ATF_OK;
 }
 
+atf_status atf_test_divisible16(uint64_t* h_mismatches) {
+  if (!h_mismatches) return ATF_ERR_INVALID_ARG;
+  unsigned long long* d = nullptr;
+  if (cudaMalloc(&d, 8) != cudaSuccess) return ATF_ERR_CUDA;
+  cudaMemset(d, 0, 8);
+  int ce = launch_divisible16_check(d, nullptr);
+  unsigned long long h = ~0ull;
+  if (!ce) ce = (int)cudaMemcpy(&h, d, 8, cudaMemcpyDeviceToHost);
+  cudaFree(d);
+  *h_mismatches = h;
+  return ce ? ATF_ERR_CUDA : ATF_OK;
+}
+
 atf_status atf_test_exclusive_scan_u32(const uint32_t* d_in, uint64_t* d_out, int64_t n, void* stream) {
   if ((!d_in && n > 0) || !d_out || n < 0) return ATF_ERR_INVALID_ARG;
   cudaStream_t st = (cudaStream_t)stream;

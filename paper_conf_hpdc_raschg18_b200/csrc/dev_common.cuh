@@ -100,6 +100,17 @@ __device__ __forceinline__ int64_t run_code(const int32_t* code, int len, int64_
   return sp == 1 ? st[0] : (poison = true, 0);
 }
 
+// q | nb for 16-bit operands (nb < 2^16, 1 <= q < 2^16) without an integer division: k =
+// round(nb * rcp(q)) in fp32 (operands exact; approximate rcp within 2 ulp, so |nb/q - k| <
+// 2^-6 whenever q divides nb and k is then nb / q), divisible iff k * q == nb (exact integer
+// check: no false positives).
+__device__ __forceinline__ bool divisible16(uint32_t nb, uint32_t q) {
+  float rq;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(rq) : "f"((float)q));
+  const uint32_t k = __float2uint_rn((float)nb * rq);
+  return k * q == nb;
+}
+
 __device__ __forceinline__ uint64_t uabs64(int64_t v) { return v < 0 ? 0ull - (uint64_t)v : (uint64_t)v; }
 
 __device__ __forceinline__ bool rel_holds(int rel, int64_t l, int64_t r) {

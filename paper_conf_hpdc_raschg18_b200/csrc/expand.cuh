@@ -41,7 +41,7 @@ __device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, 
           const uint32_t mq = s_q[q];
           return (uint32_t)nb * mq <= mq - 1u;
         }
-        return (uint32_t)nb % q == 0;
+        return divisible16((uint32_t)nb, q);
       }
       const uint64_t q = udiv64f(num, ax);
       return q != 0 && umod64f(nb, q) == 0;
@@ -355,6 +355,32 @@ static __device__ __noinline__ uint32_t other_terms_mask(const LevelArgs& a, int
     const Term& T = a.terms[t];
     const int64_t A = s_opa[t * tn + i], Bv = s_opb[t * tn + i];
     uint32_t m = mask;
+    if (T.kind == T_QDIV && T.variant == V16 && !T.use_qtable) {
+      // (num / x) | nb, the 16-bit case hoisted out of the generic dispatch
+      const uint32_t num = (uint32_t)A, nb = (uint32_t)Bv;
+      while (m) {
+        const int c = __ffs(m) - 1;
+        m &= m - 1;
+        const uint32_t ax = __ldg(a.cand_abs + jg0 + c);
+        bool ok = false;
+        if (ax != 0) {
+          const uint32_t q = ax == 1 ? num : __umulhi(num, __ldg(a.cand_magic + jg0 + c));
+          ok = q != 0 && divisible16(nb, q);
+        }
+        if (!ok) mask &= ~(1u << c);
+      }
+      continue;
+    }
+    if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) {
+      const uint32_t n = (uint32_t)A;
+      while (m) {
+        const int c = __ffs(m) - 1;
+        m &= m - 1;
+        const uint32_t mg = __ldg(a.cand_magic + jg0 + c);
+        if (!(n * mg < 0x10000u && mg != 0x10000u)) mask &= ~(1u << c);
+      }
+      continue;
+    }
     while (m) {
       const int c = __ffs(m) - 1;
       m &= m - 1;
@@ -1143,7 +1169,7 @@ __device__ __forceinline__ uint32_t nf_node_mask(const LevelArgs& a, const uint3
           const uint32_t ax = s_ca[c];
           if (ax == 0) continue;
           const uint32_t q = ax == 1 ? num : __umulhi(num, s_cm[c]);
-          if (q != 0 && nb % q == 0) mm |= 1u << c;
+          if (q != 0 && divisible16(nb, q)) mm |= 1u << c;
         }
         break;
       }

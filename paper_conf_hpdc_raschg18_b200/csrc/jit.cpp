@@ -73,6 +73,12 @@ typedef unsigned int u32; typedef unsigned long long u64; typedef int i32; typed
 struct JitArgs { const u32* parent_rec; u64 n_parents, n_tiles; void* masks; u32* tile_total;
                  const i32* pv_range[24]; const u32* pv_magic[24]; };
 __device__ __forceinline__ u32 uabs(i64 v) { return (u32)(v < 0 ? -v : v); }
+__device__ __forceinline__ bool divisible16(u32 nb, u32 q) {  // as in dev_common.cuh
+  float rq;
+  asm("rcp.approx.ftz.f32 %0, %1;" : "=f"(rq) : "f"((float)q));
+  const u32 k = __float2uint_rn((float)nb * rq);
+  return k * q == nb;
+}
 )";
 
 std::string hex(uint32_t v) {
@@ -178,7 +184,7 @@ std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx
           if (ax == 0) continue;  // x == 0 rejects
           const std::string q = ax == 1 ? std::string("num") : "__umulhi(num, " + hex(cm[c]) + ")";
           s += "        if ((m >> " + std::to_string(c) + ") & 1u) { const u32 q = " + q +
-               "; if (q != 0u && nb % q == 0u) mm |= 1u << " + std::to_string(c) + "; }\n";
+               "; if (q != 0u && divisible16(nb, q)) mm |= 1u << " + std::to_string(c) + "; }\n";
         }
         s += "        m &= mm;\n";
         break;

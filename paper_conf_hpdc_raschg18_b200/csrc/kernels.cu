@@ -417,6 +417,20 @@ int launch_filter_product(const ProductArgs& a, unsigned long long* count, void*
   return (int)cudaGetLastError();
 }
 
+// ---------------------------------------------------------------- divisible16 check (tests)
+// Exhaustive: every (nb, q) with nb < 2^16, 1 <= q < 2^16 against integer modulo.
+__global__ void divisible16_check_kernel(unsigned long long* mismatches) {
+  unsigned long long bad = 0;
+  for (uint32_t q = blockIdx.x + 1; q < 65536u; q += gridDim.x)
+    for (uint32_t nb = threadIdx.x; nb < 65536u; nb += blockDim.x) bad += divisible16(nb, q) != (nb % q == 0);
+  bad = warp_sum_u64(bad);
+  if ((threadIdx.x & 31) == 0 && bad) atomicAdd(mismatches, bad);
+}
+int launch_divisible16_check(unsigned long long* mismatches, void* stream) {
+  divisible16_check_kernel<<<4096, 256, 0, (cudaStream_t)stream>>>(mismatches);
+  return (int)cudaGetLastError();
+}
+
 // ---------------------------------------------------------------- standalone scan (tests)
 // Exclusive scan u32 -> u64 with the same look-back as expand_kernel; out[n] = total.
 __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restrict__ out, int64_t n,

@@ -445,3 +445,12 @@ def test_generator_ranges_against_oracle(Space):
     s.add("W", A.interval(1, 200), A.divides(A.P(2) * 4))
     _check_against_oracle(Space, s)
     _check_against_oracle(Space, s, generic=True)
+
+
+def test_divisible16_exhaustive(Space):
+    """q | nb through an fp32 reciprocal (16-bit quotient divisors) = integer modulo on all 2^32 pairs."""
+    import ctypes as C
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    bad = C.c_uint64(1)
+    L.check(L.atf_test_divisible16(C.byref(bad)))
+    assert bad.value == 0
