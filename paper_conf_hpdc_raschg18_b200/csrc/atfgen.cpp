@@ -798,7 +798,7 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
       return;
     }
   }
-  if (r <= 32 && a.nf_ok && !legacy_wide) {
+  if (r <= 64 && a.nf_ok && !legacy_wide) {
     a.kind = K_NFAST;
     a.block = 256;
     a.cpt = 1;
@@ -1130,7 +1130,7 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   }
   // narrow fast levels: pass 1 writes per-parent accept masks, pass 2 the children in place
   if (a.kind == K_NFAST) {
-    a.mask_bytes = a.r <= 8 ? 1 : (a.r <= 16 ? 2 : 4);
+    a.mask_bytes = a.r <= 8 ? 1 : (a.r <= 16 ? 2 : (a.r <= 32 ? 4 : 8));
     if ((e = ensure_buf(s, &s->d_masks, &s->masks_cap, (size_t)n_parents * a.mask_bytes + 16, "accept masks")))
       return e;
     a.masks = s->d_masks;
@@ -2012,7 +2012,7 @@ atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, si
   a.r = lp.r;
   a.n_parents = 1;
   choose_geometry(a, gp.words, false);
-  a.mask_bytes = a.r <= 8 ? 1 : (a.r <= 16 ? 2 : 4);
+  a.mask_bytes = a.r <= 8 ? 1 : (a.r <= 16 ? 2 : (a.r <= 32 ? 4 : 8));
   const auto& vals = s->params[lp.param].values;
   std::vector<uint32_t> mags(vals.size());
   for (size_t j = 0; j < vals.size(); j++) {

@@ -1124,15 +1124,14 @@ __device__ __forceinline__ uint32_t nf_abs(const LevelArgs& a, const NfOp& o, co
   return av;
 }
 
-template <int W>
-__device__ __forceinline__ uint32_t nf_node_mask(const LevelArgs& a, const uint32_t* rec, int r, uint32_t m,
-                                                 uint32_t nz, const int32_t* s_cx, const uint32_t* s_cm,
+template <int W, typename M>
+__device__ __forceinline__ M nf_node_mask(const LevelArgs& a, const uint32_t* rec, int r, M m, M nz, const int32_t* s_cx, const uint32_t* s_cm,
                                                  const uint32_t* s_ca) {
   for (int t = 0; t < a.n_terms && m; t++) {
     const Term& T = a.terms[t];
     const NfOp& oa = a.nf_op[t][0];
     const NfOp& ob = a.nf_op[t][1];
-    uint32_t mm = 0;
+    M mm = 0;
     switch (T.kind) {
       case T_DIVX:
       case T_DIVPROD: {  // x | n; DIVPROD: gate a != 0 && a | b, n = b / a (magic quotient)
@@ -1142,41 +1141,41 @@ __device__ __forceinline__ uint32_t nf_node_mask(const LevelArgs& a, const uint3
         } else {
           uint32_t ma;
           const uint32_t av = nf_abs<W>(a, oa, rec, &ma), bv = nf_abs<W>(a, ob, rec, nullptr);
-          if (av == 0) return 0u;
+          if (av == 0) return 0;
           n = av == 1 ? bv : __umulhi(bv, ma);
-          if (n * av != bv) return 0u;
+          if (n * av != bv) return 0;
         }
 #pragma unroll 4
-        for (int c = 0; c < r; c++) mm |= (uint32_t)(n * s_cm[c] < 0x10000u) << c;
+        for (int c = 0; c < r; c++) mm |= (M)(n * s_cm[c] < 0x10000u) << c;
         mm &= nz;  // x == 0 rejects (poison)
         break;
       }
       case T_MULX: {  // d | x, d != 0
         uint32_t md;
         const uint32_t d = nf_abs<W>(a, oa, rec, &md);
-        if (d == 0) return 0u;
+        if (d == 0) return 0;
         const uint32_t md1 = md - 1u;
 #pragma unroll 4
-        for (int c = 0; c < r; c++) mm |= (uint32_t)(s_ca[c] * md <= md1) << c;
+        for (int c = 0; c < r; c++) mm |= (M)(s_ca[c] * md <= md1) << c;
         break;
       }
       case T_QDIV: {  // (num / x) | nb; x == 0 or quotient 0 rejects
         const uint32_t num = nf_abs<W>(a, oa, rec, nullptr), nb = nf_abs<W>(a, ob, rec, nullptr);
-        uint32_t rest = m;
+        M rest = m;
         while (rest) {
-          const int c = __ffs(rest) - 1;
+          const int c = (sizeof(M) == 8 ? __ffsll((long long)rest) : __ffs((int)rest)) - 1;
           rest &= rest - 1;
           const uint32_t ax = s_ca[c];
           if (ax == 0) continue;
           const uint32_t q = ax == 1 ? num : __umulhi(num, s_cm[c]);
-          if (q != 0 && divisible16(nb, q)) mm |= 1u << c;
+          if (q != 0 && divisible16(nb, q)) mm |= (M)1 << c;
         }
         break;
       }
       default: {  // T_CMP, 32-bit: (A * x) rel B
         const int32_t A = (int32_t)nf_sval<W>(a, oa, rec), Bv = (int32_t)nf_sval<W>(a, ob, rec);
 #pragma unroll 4
-        for (int c = 0; c < r; c++) mm |= (uint32_t)rel_holds32(T.rel, A * s_cx[c], Bv) << c;
+        for (int c = 0; c < r; c++) mm |= (M)rel_holds32(T.rel, A * s_cx[c], Bv) << c;
         break;
       }
     }
@@ -1185,25 +1184,25 @@ __device__ __forceinline__ uint32_t nf_node_mask(const LevelArgs& a, const uint3
   return m;
 }
 
-// Pass 1 (A4): accept masks of every frontier node (mask_bytes = 1/2/4 per node) and the
+// Pass 1 (A4): accept masks of every frontier node (mask_bytes = 1/2/4/8 per node) and the
 // child count of every warp tile (tile_total).  Tiles are static: warp w of the grid takes
 // tiles w, w + nwarps, ...
-template <int W>
+template <int W, typename M>
 __global__ void __launch_bounds__(256, 4) expand_nfast(const __grid_constant__ LevelArgs a) {
-  __shared__ int32_t s_cx[32];
-  __shared__ uint32_t s_cm[32], s_ca[32];
+  __shared__ int32_t s_cx[64];
+  __shared__ uint32_t s_cm[64], s_ca[64];
   const int lane = threadIdx.x & 31;
   const int r = a.r;
-  if (threadIdx.x < 32) {
+  if (threadIdx.x < 64) {
     const bool v = threadIdx.x < r;
     s_cx[threadIdx.x] = v ? __ldg(a.cand + threadIdx.x) : 0;
     s_cm[threadIdx.x] = v ? __ldg(a.cand_magic + threadIdx.x) : 0x10000u;
     s_ca[threadIdx.x] = v ? __ldg(a.cand_abs + threadIdx.x) : 0u;
   }
   __syncthreads();
-  const uint32_t full = r >= 32 ? 0xffffffffu : ((1u << r) - 1u);
-  uint32_t nz = 0;
-  for (int c = 0; c < r; c++) nz |= (uint32_t)(s_cx[c] != 0) << c;
+  const M full = r >= (int)(8 * sizeof(M)) ? ~(M)0 : (((M)1 << r) - 1);
+  M nz = 0;
+  for (int c = 0; c < r; c++) nz |= (M)(s_cx[c] != 0) << c;
   constexpr int TN = 32 * kNfNPL;
   const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   for (uint64_t t = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; t < a.n_tiles; t += nw) {
@@ -1226,11 +1225,12 @@ __global__ void __launch_bounds__(256, 4) expand_nfast(const __grid_constant__ L
     for (int q = 0; q < kNfNPL; q++) {
       const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
       if (nd < a.n_parents) {
-        const uint32_t m = nf_node_mask<W>(a, rec[q], r, full, nz, s_cx, s_cm, s_ca);
-        cnt += (uint32_t)__popc(m);
+        const M m = nf_node_mask<W, M>(a, rec[q], r, full, nz, s_cx, s_cm, s_ca);
+        cnt += (uint32_t)__popcll((unsigned long long)m);
         if (a.mask_bytes == 1) reinterpret_cast<uint8_t*>(a.masks)[nd] = (uint8_t)m;
         else if (a.mask_bytes == 2) reinterpret_cast<uint16_t*>(a.masks)[nd] = (uint16_t)m;
-        else reinterpret_cast<uint32_t*>(a.masks)[nd] = m;
+        else if (a.mask_bytes == 4) reinterpret_cast<uint32_t*>(a.masks)[nd] = (uint32_t)m;
+        else reinterpret_cast<unsigned long long*>(a.masks)[nd] = (unsigned long long)m;
       }
     }
 #pragma unroll
@@ -1256,7 +1256,8 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
   if (total > a.child_cap) return;
   for (uint64_t t = gw; t < a.n_tiles; t += nw) {
     const uint64_t node0 = t * TN;
-    uint32_t mask[kNfNPL], rec[kNfNPL][W];
+    unsigned long long mask[kNfNPL];
+    uint32_t rec[kNfNPL][W];
 #pragma unroll
     for (int q = 0; q < kNfNPL; q++) {
       const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
@@ -1264,7 +1265,8 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
       if (nd < a.n_parents) {
         if (a.mask_bytes == 1) mask[q] = reinterpret_cast<const uint8_t*>(a.masks)[nd];
         else if (a.mask_bytes == 2) mask[q] = reinterpret_cast<const uint16_t*>(a.masks)[nd];
-        else mask[q] = reinterpret_cast<const uint32_t*>(a.masks)[nd];
+        else if (a.mask_bytes == 4) mask[q] = reinterpret_cast<const uint32_t*>(a.masks)[nd];
+        else mask[q] = reinterpret_cast<const unsigned long long*>(a.masks)[nd];
       }
     }
 #pragma unroll
@@ -1283,7 +1285,7 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
 #pragma unroll
     for (int q = 0; q < kNfNPL; q++) {
       const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
-      const uint32_t c = (uint32_t)__popc(mask[q]);
+      const uint32_t c = (uint32_t)__popcll(mask[q]);
       uint32_t incl = c;
 #pragma unroll
       for (int o = 1; o < 32; o <<= 1) {
@@ -1293,9 +1295,9 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
       uint64_t rank = run + (incl - c);
       run += __shfl_sync(FULL, incl, 31);
       if (nd < a.n_parents) a.csr[nd] = rank;
-      uint32_t m = mask[q];
+      unsigned long long m = mask[q];
       while (m) {
-        const int cc = __ffs(m) - 1;
+        const int cc = __ffsll((long long)m) - 1;
         m &= m - 1;
         uint32_t out[W];
 #pragma unroll
@@ -1363,7 +1365,9 @@ static int launch_nfast_emit_w(const LevelArgs& a, void* stream) {
 template <int W>
 static int launch_w(const LevelArgs& a, void* stream) {
   if (a.kind == K_NARROW) return launch_persistent(expand_narrow<W>, a, a.block, stream);
-  if (a.kind == K_NFAST) return launch_grid_warps(expand_nfast<W>, a, stream);
+  if (a.kind == K_NFAST)
+    return a.r <= 32 ? launch_grid_warps(expand_nfast<W, uint32_t>, a, stream)
+                     : launch_grid_warps(expand_nfast<W, unsigned long long>, a, stream);
   if (a.kind == K_WTILE) {
     switch (a.cpt) {
       case 4: return launch_wtile_wc<W, 4>(a, stream);

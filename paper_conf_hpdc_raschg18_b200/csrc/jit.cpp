@@ -90,8 +90,10 @@ std::string hex(uint32_t v) {
 // Source of the level kernel, or "" if the level uses something the generator does not
 // cover (then the generic kernel runs).
 std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx, const std::vector<uint32_t>& cm) {
-  if (a.kind != K_NFAST || a.n_terms == 0 || a.r > 32 || (int)cx.size() != a.r) return "";
+  if (a.kind != K_NFAST || a.n_terms == 0 || a.r > 64 || (int)cx.size() != a.r) return "";
   const int r = a.r;
+  const bool wide = r > 32;  // 64-bit masks
+  const std::string MT = wide ? "u64" : "u32";
   std::string s = kPrelude;
   s += "extern \"C\" __global__ void __launch_bounds__(256) atf_nfast_jit(const __grid_constant__ JitArgs a) {\n";
   s += "  const int lane = threadIdx.x & 31;\n";
@@ -138,9 +140,10 @@ std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx
     if (o.kind == NF_PV) return "(" + absname + " == 0u ? 0u : g" + std::to_string(o.s1) + ")";
     return "(" + absname + " > 1u ? 0xffffffffu / " + absname + " + 1u : 0u)";
   };
-  uint32_t full = r >= 32 ? 0xffffffffu : ((1u << r) - 1u), nz = 0;
-  for (int c = 0; c < r; c++) nz |= (uint32_t)(cx[c] != 0) << c;
-  s += "      u32 m = " + hex(full) + ";\n";
+  const unsigned long long full = r >= 64 ? ~0ull : ((1ull << r) - 1ull);
+  char fb[32];
+  snprintf(fb, sizeof fb, "0x%llxull", full);
+  s += "      " + MT + " m = (" + MT + ")" + fb + ";\n";
   for (int t = 0; t < a.n_terms; t++) {
     const Term& T = a.terms[t];
     const NfOp& oa = a.nf_op[t][0];
@@ -148,9 +151,9 @@ std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx
     const std::string ts = std::to_string(t);
     s += "      if (m) {  // term " + ts + "\n";
     auto divx_bits = [&](const std::string& n) {
-      std::string b = "        u32 mm = 0u;\n";
+      std::string b = "        " + MT + " mm = 0u;\n";
       for (int c = 0; c < r; c++)
-        if (cx[c] != 0) b += "        mm |= (u32)(" + n + " * " + hex(cm[c]) + " < 0x10000u) << " + std::to_string(c) + ";\n";
+        if (cx[c] != 0) b += "        mm |= (" + MT + ")(" + n + " * " + hex(cm[c]) + " < 0x10000u) << " + std::to_string(c) + ";\n";
       b += "        m &= mm;\n";
       return b;
     };
@@ -168,23 +171,23 @@ std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx
       case T_MULX: {
         s += "        const u32 d = uabs(" + sval(oa) + ");\n";
         s += "        const u32 md = " + magic(oa, "d") + ", md1 = md - 1u;\n";
-        s += "        if (d == 0u) m = 0u;\n        else {\n          u32 mm = 0u;\n";
+        s += "        if (d == 0u) m = 0u;\n        else {\n          " + MT + " mm = 0u;\n";
         for (int c = 0; c < r; c++) {
           const uint32_t ax = cx[c] < 0 ? 0u - (uint32_t)cx[c] : (uint32_t)cx[c];
-          s += "          mm |= (u32)(" + hex(ax) + " * md <= md1) << " + std::to_string(c) + ";\n";
+          s += "          mm |= (" + MT + ")(" + hex(ax) + " * md <= md1) << " + std::to_string(c) + ";\n";
         }
         s += "          m &= mm;\n        }\n";
         break;
       }
       case T_QDIV: {
         s += "        const u32 num = uabs(" + sval(oa) + "), nb = uabs(" + sval(ob) + ");\n";
-        s += "        u32 mm = 0u;\n";
+        s += "        " + MT + " mm = 0u;\n";
         for (int c = 0; c < r; c++) {
           const uint32_t ax = cx[c] < 0 ? 0u - (uint32_t)cx[c] : (uint32_t)cx[c];
           if (ax == 0) continue;  // x == 0 rejects
           const std::string q = ax == 1 ? std::string("num") : "__umulhi(num, " + hex(cm[c]) + ")";
           s += "        if ((m >> " + std::to_string(c) + ") & 1u) { const u32 q = " + q +
-               "; if (q != 0u && divisible16(nb, q)) mm |= 1u << " + std::to_string(c) + "; }\n";
+               "; if (q != 0u && divisible16(nb, q)) mm |= (" + MT + ")1u << " + std::to_string(c) + "; }\n";
         }
         s += "        m &= mm;\n";
         break;
@@ -192,9 +195,9 @@ std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx
       case T_CMP: {
         static const char* rel[] = {"==", "!=", "<", "<=", ">", ">="};
         if (T.rel < R_EQ || T.rel > R_GE) return "";
-        s += "        const i32 A = (i32)" + sval(oa) + ", B = (i32)" + sval(ob) + ";\n        u32 mm = 0u;\n";
+        s += "        const i32 A = (i32)" + sval(oa) + ", B = (i32)" + sval(ob) + ";\n        " + MT + " mm = 0u;\n";
         for (int c = 0; c < r; c++)
-          s += "        mm |= (u32)(A * " + std::to_string(cx[c]) + " " + rel[T.rel - R_EQ] + " B) << " +
+          s += "        mm |= (" + MT + ")(A * " + std::to_string(cx[c]) + " " + rel[T.rel - R_EQ] + " B) << " +
                std::to_string(c) + ";\n";
         s += "        m &= mm;\n";
         break;
@@ -203,9 +206,9 @@ std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx
     }
     s += "      }\n";
   }
-  (void)nz;  // x == 0 candidates get no bit in the DIVX / DIVPROD / QDIV loops
-  s += "      cnt += __popc(m);\n";
-  const char* mt = a.mask_bytes == 1 ? "unsigned char" : (a.mask_bytes == 2 ? "unsigned short" : "u32");
+  // x == 0 candidates get no bit in the DIVX / DIVPROD / QDIV loops
+  s += "      cnt += __popcll((u64)m);\n";
+  const char* mt = a.mask_bytes == 1 ? "unsigned char" : (a.mask_bytes == 2 ? "unsigned short" : (a.mask_bytes == 4 ? "u32" : "u64"));
   s += std::string("      reinterpret_cast<") + mt + "*>(a.masks)[nd] = (" + mt + ")m;\n";
   s += "    }\n";
   s += "#pragma unroll\n    for (int o = 16; o > 0; o >>= 1) cnt += __shfl_xor_sync(0xffffffffu, cnt, o);\n";
