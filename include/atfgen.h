@@ -104,6 +104,9 @@ typedef struct {
                                      the warp-tile kernel (kept for parity coverage)      */
 #define ATF_FLAG_NO_JIT 16u       /* narrow fast levels use the generic kernel instead of the
                                      NVRTC-specialised one (kept for parity coverage)     */
+#define ATF_FLAG_SERIAL_GROUPS 32u /* run the groups' levels one after another on the space's
+                                     stream (default: concurrently, one stream per group) —
+                                     isolates per-launch times for roofline measurements    */
 #define ATF_FLAG_KEEP_LEVELS 4u   /* keep inner-level arrays (CSR + records); default
                                      keeps them too — reserved                          */
 

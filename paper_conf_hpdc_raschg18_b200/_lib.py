@@ -24,7 +24,7 @@ STATUS = {0: "ATF_OK", -1: "ATF_ERR_INVALID_ARG", -2: "ATF_ERR_OOM", -3: "ATF_ER
           -5: "ATF_ERR_BYTECODE", -6: "ATF_ERR_FORWARD_REF", -7: "ATF_ERR_OVERFLOW", -8: "ATF_ERR_INDEX",
           -9: "ATF_ERR_DUPLICATE", -10: "ATF_ERR_LIMIT"}
 ATF_RANGE_INTERVAL, ATF_RANGE_POW2, ATF_RANGE_SET, ATF_RANGE_GEN = 0, 1, 2, 3
-ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT = 1, 2, 8, 16
+ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT, ATF_FLAG_SERIAL_GROUPS = 1, 2, 8, 16, 32
 
 
 class atf_range(C.Structure):

@@ -109,13 +109,19 @@ struct atf_space {
   std::vector<uint64_t> gsize;
   unsigned long long* d_status = nullptr;
   size_t status_cap = 0;
-  char* d_masks = nullptr;  // nfast accept masks
-  size_t masks_cap = 0;
+  // per group (levels of different groups in one round run concurrently, one stream each)
+  struct GroupBufs {
+    char* masks = nullptr;      // nfast accept masks
+    size_t masks_cap = 0;
+    char* scratch = nullptr;    // per-tile totals, segments, bases, scan state
+    size_t scratch_cap = 0;
+    uint32_t* stash = nullptr;  // wide levels: children in tile segments before the final copy
+    size_t stash_cap = 0;       // bytes
+    cudaStream_t stream = nullptr;
+    cudaEvent_t fork = nullptr, join = nullptr;
+  };
+  std::vector<GroupBufs> gb;
   uint64_t stash_hint = 0;     // records: exact size of the last level that overflowed
-  char* d_scratch = nullptr;   // wide levels: per-tile totals, segments, bases, scan state
-  size_t scratch_cap = 0;
-  uint32_t* d_stash = nullptr; // wide levels: children in tile segments before the final copy
-  size_t stash_cap = 0;        // bytes
   unsigned int* d_counter = nullptr;     // [kMaxGroups] tile counters
   unsigned long long* d_totals = nullptr;  // [kMaxGroups]
   unsigned int* d_ovf = nullptr;         // [kMaxGroups]
@@ -922,6 +928,12 @@ static atf_status ensure_device(atf_space* s) {
   CUDA_TRY(s, cudaMallocHost(&s->h_totals, 8 * kMaxGroups));
   CUDA_TRY(s, cudaMallocHost(&s->h_flags, 4 * kMaxGroups));
   s->arena.assign(s->groups.size(), {});
+  s->gb.assign(s->groups.size(), {});
+  for (auto& b : s->gb) {
+    CUDA_TRY(s, cudaStreamCreateWithFlags(&b.stream, cudaStreamNonBlocking));
+    CUDA_TRY(s, cudaEventCreateWithFlags(&b.fork, cudaEventDisableTiming));
+    CUDA_TRY(s, cudaEventCreateWithFlags(&b.join, cudaEventDisableTiming));
+  }
   s->dev_ready = true;
   return ATF_OK;
 }
@@ -981,14 +993,18 @@ static void release_device(atf_space* s) {
     dfree(s, s->d_sorted[p], std::max<size_t>(16, s->params[p].values.size() * 8));
   s->d_sorted.clear();
   dfree(s, s->d_status, s->status_cap * 8);
-  dfree(s, s->d_scratch, s->scratch_cap);
-  dfree(s, (char*)s->d_stash, s->stash_cap);
-  dfree(s, s->d_masks, s->masks_cap);
-  s->d_masks = nullptr;
-  s->masks_cap = 0;
-  s->d_scratch = nullptr;
-  s->d_stash = nullptr;
-  s->scratch_cap = s->stash_cap = 0;
+  for (auto& b : s->gb) {
+    dfree(s, b.scratch, b.scratch_cap);
+    dfree(s, (char*)b.stash, b.stash_cap);
+    dfree(s, b.masks, b.masks_cap);
+    if (b.stream) {
+      cudaStreamSynchronize(b.stream);
+      cudaStreamDestroy(b.stream);
+    }
+    if (b.fork) cudaEventDestroy(b.fork);
+    if (b.join) cudaEventDestroy(b.join);
+  }
+  s->gb.clear();
   dfree(s, s->d_counter, 4 * kMaxGroups);
   dfree(s, s->d_totals, 8 * kMaxGroups);
   dfree(s, s->d_ovf, 4 * kMaxGroups);
@@ -1028,7 +1044,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   (void)tile_base_unused;
   GroupPlan& gp = s->groups[g];
   LevelPlan& lp = gp.levels[k];
-  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  cudaStream_t st = (cudaStream_t)s->opts.stream;  // allocations, memsets
+  auto& gbf = s->gb[g];                            // this group's buffers and launch stream
   LevelArgs a = lp.proto;
   a.parent_rec = parents;
   a.n_parents = n_parents;
@@ -1104,10 +1121,10 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     // whole arena tail
     const uint64_t stash_recs = std::min<uint64_t>(cap, std::max<uint64_t>({est + est / 4, (uint64_t)1 << 16,
                                                                              s->stash_hint}));
-    if ((e = ensure_buf(s, (char**)&s->d_stash, &s->stash_cap, (size_t)stash_recs * gp.words * 4, "stash")))
+    if ((e = ensure_buf(s, (char**)&gbf.stash, &gbf.stash_cap, (size_t)stash_recs * gp.words * 4, "stash")))
       return e;
-    a.stash = s->d_stash;
-    a.stash_cap = s->stash_cap / (gp.words * 4);
+    a.stash = gbf.stash;
+    a.stash_cap = gbf.stash_cap / (gp.words * 4);
     // scratch: tile_seg u64[n] | tile_base u64[n+1] | tile_total u32[n] (pad) |
     //          scan status u64[ceil(n/1024)+1] | scan counter u32 | stash_top u64 |
     //          piece_tile u32[stash_cap / 2^kPieceShift + 2]
@@ -1116,29 +1133,38 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     const size_t o_scan = (o_tot + 4 * n + 15) & ~(size_t)15, o_cnt = o_scan + 8 * nscan, o_top = o_cnt + 16;
     const size_t o_piece = o_top + 16;
     piece_cap = (a.stash_cap >> kPieceShift) + 2;
-    if ((e = ensure_buf(s, &s->d_scratch, &s->scratch_cap, o_piece + 4 * piece_cap, "tile scratch"))) return e;
-    a.tile_seg = (unsigned long long*)(s->d_scratch + o_seg);
-    scan_out = (uint64_t*)(s->d_scratch + o_base);
+    if ((e = ensure_buf(s, &gbf.scratch, &gbf.scratch_cap, o_piece + 4 * piece_cap, "tile scratch"))) return e;
+    char* const d_scratch = gbf.scratch;
+    a.tile_seg = (unsigned long long*)(d_scratch + o_seg);
+    scan_out = (uint64_t*)(d_scratch + o_base);
     a.tile_base = scan_out;
-    a.tile_total = (uint32_t*)(s->d_scratch + o_tot);
-    scan_status = (unsigned long long*)(s->d_scratch + o_scan);
-    scan_counter = (unsigned int*)(s->d_scratch + o_cnt);
-    a.stash_top = (unsigned long long*)(s->d_scratch + o_top);
-    piece_tile = (uint32_t*)(s->d_scratch + o_piece);
+    a.tile_total = (uint32_t*)(d_scratch + o_tot);
+    scan_status = (unsigned long long*)(d_scratch + o_scan);
+    scan_counter = (unsigned int*)(d_scratch + o_cnt);
+    a.stash_top = (unsigned long long*)(d_scratch + o_top);
+    piece_tile = (uint32_t*)(d_scratch + o_piece);
     a.piece_tile = piece_tile;
-    CUDA_TRY(s, cudaMemsetAsync(s->d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
+    CUDA_TRY(s, cudaMemsetAsync(d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
   }
   // narrow fast levels: pass 1 writes per-parent accept masks, pass 2 the children in place
   if (a.kind == K_NFAST) {
     a.mask_bytes = a.r <= 8 ? 1 : (a.r <= 16 ? 2 : (a.r <= 32 ? 4 : 8));
-    if ((e = ensure_buf(s, &s->d_masks, &s->masks_cap, (size_t)n_parents * a.mask_bytes + 16, "accept masks")))
+    if ((e = ensure_buf(s, &gbf.masks, &gbf.masks_cap, (size_t)n_parents * a.mask_bytes + 16, "accept masks")))
       return e;
-    a.masks = s->d_masks;
+    a.masks = gbf.masks;
   }
   CUDA_TRY(s, cudaMemsetAsync(s->d_counter + g, 0, 4, st));
   CUDA_TRY(s, cudaMemsetAsync(s->d_ovf + g, 0, 4, st));
+  // the level's kernels run on the group's stream after the allocations / memsets above;
+  // run_levels joins the group streams back into the space's stream
+  const bool serial = (s->opts.flags & ATF_FLAG_SERIAL_GROUPS) != 0;
+  cudaStream_t ls = serial ? st : gbf.stream;
+  if (!serial) {
+    CUDA_TRY(s, cudaEventRecord(gbf.fork, st));
+    CUDA_TRY(s, cudaStreamWaitEvent(gbf.stream, gbf.fork, 0));
+  }
   bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
-  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].first, st));
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].first, ls));
   if (a.kind == K_NFAST && !lp.jit_tried && !(s->opts.flags & (ATF_FLAG_NO_JIT | ATF_FLAG_LEGACY_WIDE))) {
     const auto& vals = s->params[lp.param].values;
     std::vector<uint32_t> mags(vals.size());
@@ -1150,21 +1176,22 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     lp.jit_tried = true;
   }
   const bool use_jit = a.kind == K_NFAST && lp.jit && !(s->opts.flags & (ATF_FLAG_NO_JIT | ATF_FLAG_LEGACY_WIDE));
-  int ce = use_jit ? jit_nfast_launch(lp.jit, a, st) : launch_expand(a, gp.words, st);
+  int ce = use_jit ? jit_nfast_launch(lp.jit, a, ls) : launch_expand(a, gp.words, ls);
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   if (use_jit) s->data[g][k].kernel = 4;
-  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].mid, st));
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].mid, ls));
   if (!use_jit) s->data[g][k].kernel = a.kind;
   if (a.kind == K_NFAST) {
-    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st);
-    if (!ce) ce = launch_nfast_emit(a, gp.words, st);
+    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, ls);
+    if (!ce) ce = launch_nfast_emit(a, gp.words, ls);
     if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   } else {
-    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, st, piece_tile, piece_cap);
-    if (!ce) ce = launch_level_emit(a, gp.words, st);
+    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, ls, piece_tile, piece_cap);
+    if (!ce) ce = launch_level_emit(a, gp.words, ls);
     if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   }
-  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].second, st));
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].second, ls));
+  if (!serial) CUDA_TRY(s, cudaEventRecord(gbf.join, ls));
   pd = Pending{g, k, n_parents, parents, (uint64_t*)csr, child, cap, which, off};
   return ATF_OK;
 }
@@ -1208,6 +1235,8 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       pend.push_back(pd);
     }
     if (pend.empty()) break;
+    if (!(s->opts.flags & ATF_FLAG_SERIAL_GROUPS))
+      for (auto& pd : pend) CUDA_TRY(s, cudaStreamWaitEvent(st, s->gb[pd.g].join, 0));  // join the group streams
     for (auto& pd : pend) {
       CUDA_TRY(s, cudaMemcpyAsync(s->h_totals + pd.g, s->d_totals + pd.g, 8, cudaMemcpyDeviceToHost, st));
       CUDA_TRY(s, cudaMemcpyAsync(s->h_flags + pd.g, s->d_ovf + pd.g, 4, cudaMemcpyDeviceToHost, st));
