@@ -318,7 +318,7 @@ def cpu_baseline(spec, budget_s=15.0):
     return {"value": d["leaves"] / d["seconds"], "unit": "configs/s", "cores": cores, "kind": "oracle",
             "evals_per_s": d["evals"] / d["seconds"],
             "sample": (f"O2 (pruned nested loop, interpreted bytecode) on {spec.name}: groups in order, level-1 "
-                       f"values in order until {budget_s:.0f}s CPU budget; {d['level1_done']}/{d['level1_total']} "
+                       f"values in a strided order (spanning the range) until {budget_s:.0f}s CPU budget; {d['level1_done']}/{d['level1_total']} "
                        f"level-1 values, {d['evals']} evals, {d['leaves']} leaves in {d['seconds']:.2f}s")}
 
 

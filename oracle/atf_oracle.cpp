@@ -49,6 +49,7 @@
 #include <sstream>
 #include <stdexcept>
 #include <string>
+#include <numeric>
 #include <thread>
 #include <vector>
 
@@ -732,6 +733,11 @@ static int cmd_time(const Spec& s, int threads, double budget_s) {
     std::atomic<size_t> next{0};
     std::atomic<u64> ev{0}, lf{0}, done{0};
     std::atomic<bool> halt{false};
+    // level-1 positions in a strided order (stride coprime to r1) so that a bounded sample
+    // spans the whole range instead of its first values
+    size_t stride = r1 > 1 ? (size_t)(2654435761ull % r1) : 1;
+    if (stride == 0) stride = 1;
+    while (r1 > 1 && std::gcd(stride, r1) != 1) stride++;
     auto worker = [&]() {
       GroupRun gr;
       gr.s = &s;
@@ -742,6 +748,7 @@ static int cmd_time(const Spec& s, int threads, double budget_s) {
         if (halt.load()) break;
         size_t j = next.fetch_add(1);
         if (j >= r1) break;
+        j = (size_t)(((unsigned __int128)j * stride) % r1);
         gr.run(j, j + 1);
         u64 e = 0;
         for (auto& l : gr.lv) e += l.evals;
