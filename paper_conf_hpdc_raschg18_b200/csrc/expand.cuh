@@ -1,6 +1,8 @@
 // expand.cuh — the level-expansion kernels (SURVEY.md §8(a) A4-A6 fused: count, scan,
 // emit), instantiated per record width W in expand_w{1,2,4,8}.cu.
 #pragma once
+#include <type_traits>
+
 #include "dev_common.cuh"
 
 namespace atf {
@@ -1240,10 +1242,19 @@ __global__ void __launch_bounds__(256, 4) expand_nfast(const __grid_constant__ L
 }
 
 // Pass 2 (A6, after scan_kernel turned tile_total into tile_base): children written at
-// their final index, CSR entries final; no stash.
+// their final index, CSR entries final; no stash.  A warp tile's children (<= 4 KB) are
+// assembled in the warp's shared-memory buffer in order and written out as coalesced
+// vectors; larger tiles write each child directly.
+constexpr int kNfEmitBufBytes = 4096;  // per warp
+
 template <int W>
 __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelArgs a) {
+  extern __shared__ __align__(16) unsigned char nf_smem[];
+  using V = typename std::conditional<W == 1, uint32_t, typename std::conditional<W == 2, uint2, uint4>::type>::type;
+  constexpr int VPR = W == 8 ? 2 : 1;                        // vectors per record
+  constexpr int CAP = kNfEmitBufBytes / (4 * W);             // records per warp buffer
   const int lane = threadIdx.x & 31;
+  uint32_t* buf = reinterpret_cast<uint32_t*>(nf_smem + (threadIdx.x >> 5) * kNfEmitBufBytes);
   constexpr int TN = 32 * kNfNPL;
   const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
   const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
@@ -1281,7 +1292,10 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
         }
       }
     }
-    uint64_t run = a.tile_base[t];
+    const uint64_t base = a.tile_base[t];
+    const uint32_t tt = (uint32_t)(a.tile_base[t + 1] - base);  // the tile's children
+    const bool staged = tt <= (uint32_t)CAP;
+    uint32_t run = 0;
 #pragma unroll
     for (int q = 0; q < kNfNPL; q++) {
       const uint64_t nd = node0 + (uint64_t)q * 32 + lane;
@@ -1292,9 +1306,9 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
         const uint32_t y = __shfl_up_sync(FULL, incl, o);
         if (lane >= o) incl += y;
       }
-      uint64_t rank = run + (incl - c);
+      uint32_t rank = run + (incl - c);  // tile-local
       run += __shfl_sync(FULL, incl, 31);
-      if (nd < a.n_parents) a.csr[nd] = rank;
+      if (nd < a.n_parents) a.csr[nd] = base + rank;
       unsigned long long m = mask[q];
       while (m) {
         const int cc = __ffsll((long long)m) - 1;
@@ -1302,9 +1316,21 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
         uint32_t out[W];
 #pragma unroll
         for (int w = 0; w < W; w++) out[w] = rec[q][w] | (w == a.field_word ? (uint32_t)cc << a.field_shift : 0u);
-        store_record<W>(a.child_rec + rank * W, out);
+        if (staged) {
+#pragma unroll
+          for (int w = 0; w < W; w++) buf[rank * W + w] = out[w];
+        } else {
+          store_record<W>(a.child_rec + (base + rank) * W, out);
+        }
         rank++;
       }
+    }
+    if (staged) {
+      __syncwarp();
+      const V* src = reinterpret_cast<const V*>(buf);
+      V* dst = reinterpret_cast<V*>(a.child_rec + base * W);
+      for (uint32_t v = lane; v < tt * VPR; v += 32) dst[v] = src[v];
+      __syncwarp();
     }
   }
 }
@@ -1359,7 +1385,21 @@ static int launch_wtile_wc(const LevelArgs& a, void* stream) {
 
 template <int W>
 static int launch_nfast_emit_w(const LevelArgs& a, void* stream) {
-  return launch_grid_warps(nfast_emit<W>, a, stream);
+  const int smem = 8 * kNfEmitBufBytes;  // 8 warps per block
+  cudaError_t e = cudaFuncSetAttribute(nfast_emit<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+  if (e != cudaSuccess) return (int)e;
+  int per_sm = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, nfast_emit<W>, 256, smem);
+  if (e != cudaSuccess) return (int)e;
+  int dev = 0, sms = 0;
+  cudaGetDevice(&dev);
+  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  uint64_t grid = (uint64_t)sms * (per_sm > 0 ? per_sm : 1);
+  const uint64_t need = (a.n_tiles + 7) / 8;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  nfast_emit<W><<<(unsigned)grid, 256, smem, (cudaStream_t)stream>>>(a);
+  return (int)cudaGetLastError();
 }
 
 template <int W>

@@ -100,14 +100,30 @@ std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx
   s += "  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n";
   s += "  for (u64 t = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5; t < a.n_tiles; t += nw) {\n";
   s += "    u32 cnt = 0;\n";
-  s += "#pragma unroll\n    for (int q = 0; q < " + std::to_string(kNfNPL) + "; q++) {\n";
-  s += "      const u64 nd = t * " + std::to_string(32 * kNfNPL) + "ull + (u64)q * 32 + lane;\n";
-  s += "      if (nd >= a.n_parents) continue;\n";
-  for (int w = 0; w < W; w++) {
-    if (a.level == 0) s += "      const u32 w" + std::to_string(w) + " = 0u;\n";
-    else s += "      const u32 w" + std::to_string(w) + " = __ldg(a.parent_rec + nd * " + std::to_string(W) + " + " +
-              std::to_string(w) + ");\n";
+  // all parent records of the lane first (vector loads, independent), then the nodes
+  const std::string NPL = std::to_string(kNfNPL), TNs = std::to_string(32 * kNfNPL), Ws = std::to_string(W);
+  s += "    u32 rq[" + NPL + "][" + Ws + "];\n";
+  s += "#pragma unroll\n    for (int q = 0; q < " + NPL + "; q++) {\n";
+  s += "      const u64 nd = t * " + TNs + "ull + (u64)q * 32 + lane;\n";
+  if (a.level == 0) {
+    s += "      for (int w = 0; w < " + Ws + "; w++) rq[q][w] = 0u;\n";
+  } else {
+    s += "      if (nd < a.n_parents) {\n";
+    if (W == 1) s += "        rq[q][0] = __ldg(a.parent_rec + nd);\n";
+    else if (W == 2) s += "        const uint2 v = __ldg(reinterpret_cast<const uint2*>(a.parent_rec) + nd);\n"
+                          "        rq[q][0] = v.x; rq[q][1] = v.y;\n";
+    else
+      for (int h = 0; h < W / 4; h++)
+        s += "        { const uint4 v = __ldg(reinterpret_cast<const uint4*>(a.parent_rec) + nd * " + std::to_string(W / 4) +
+             " + " + std::to_string(h) + "); rq[q][" + std::to_string(4 * h) + "] = v.x; rq[q][" + std::to_string(4 * h + 1) +
+             "] = v.y; rq[q][" + std::to_string(4 * h + 2) + "] = v.z; rq[q][" + std::to_string(4 * h + 3) + "] = v.w; }\n";
+    s += "      }\n";
   }
+  s += "    }\n";
+  s += "#pragma unroll\n    for (int q = 0; q < " + NPL + "; q++) {\n";
+  s += "      const u64 nd = t * " + TNs + "ull + (u64)q * 32 + lane;\n";
+  s += "      if (nd >= a.n_parents) continue;\n";
+  for (int w = 0; w < W; w++) s += "      const u32 w" + std::to_string(w) + " = rq[q][" + std::to_string(w) + "];\n";
   // ancestor values (and magics) used by the terms
   std::vector<int> need_v(a.n_pv, 0), need_m(a.n_pv, 0);
   auto mark = [&](const NfOp& o, bool mag) {

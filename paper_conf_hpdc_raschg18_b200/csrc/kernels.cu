@@ -195,21 +195,29 @@ __global__ void decode_kernel(const __grid_constant__ DecodeArgs a, const uint64
       }
       const int W = a.words[g];
       const uint32_t* rp = a.leaves[g] + d * (uint64_t)W;
-      uint32_t rec[8];
+      // record words in registers (static indices only: no local-memory array)
+      uint32_t rec[8] = {0, 0, 0, 0, 0, 0, 0, 0};
       if (W == 1) {
         rec[0] = __ldg(rp);
       } else if (W == 2) {
         const uint2 v = __ldg(reinterpret_cast<const uint2*>(rp));
         rec[0] = v.x; rec[1] = v.y;
       } else {
-        for (int q = 0; q < W / 4; q++) {
-          const uint4 v = __ldg(reinterpret_cast<const uint4*>(rp) + q);
-          rec[4 * q] = v.x; rec[4 * q + 1] = v.y; rec[4 * q + 2] = v.z; rec[4 * q + 3] = v.w;
+        const uint4 v = __ldg(reinterpret_cast<const uint4*>(rp));
+        rec[0] = v.x; rec[1] = v.y; rec[2] = v.z; rec[3] = v.w;
+        if (W == 8) {
+          const uint4 u = __ldg(reinterpret_cast<const uint4*>(rp) + 1);
+          rec[4] = u.x; rec[5] = u.y; rec[6] = u.z; rec[7] = u.w;
         }
       }
       for (int l = a.lvl_begin[g]; l < a.lvl_begin[g + 1]; l++) {
+        const int lw = a.lvl_word[l];
+        uint32_t word = rec[0];
+#pragma unroll
+        for (int w = 1; w < 8; w++)
+          if (lw == w) word = rec[w];
         const uint32_t bits = (uint32_t)a.lvl_bits[l];
-        const uint32_t pos = bits ? (rec[a.lvl_word[l]] >> a.lvl_shift[l]) & ((1u << bits) - 1u) : 0u;
+        const uint32_t pos = bits ? (word >> a.lvl_shift[l]) & ((1u << bits) - 1u) : 0u;
         out[(int64_t)a.lvl_param[l] * ld + i] = __ldg(a.lvl_range[l] + pos);
       }
     }
