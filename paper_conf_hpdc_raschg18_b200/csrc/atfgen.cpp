@@ -127,8 +127,12 @@ struct atf_space {
   unsigned int* d_ovf = nullptr;         // [kMaxGroups]
   unsigned int* d_bad = nullptr;         // decode flag
   uint32_t* d_root = nullptr;            // 8 zero words
-  unsigned long long* h_totals = nullptr;  // pinned
-  unsigned int* h_flags = nullptr;         // pinned
+  unsigned long long* h_totals = nullptr;  // -> h_totals_v
+  unsigned int* h_flags = nullptr;         // -> h_flags_v
+  std::vector<unsigned long long> h_totals_v;
+  std::vector<unsigned int> h_flags_v;
+  int32_t* d_table = nullptr;              // all parameter tables + scratch words (ensure_device)
+  size_t table_bytes = 0;
   struct EvTriple { cudaEvent_t first = nullptr, mid = nullptr, second = nullptr; };
   std::vector<std::vector<EvTriple>> events;
   // shards
@@ -874,59 +878,69 @@ static atf_status ensure_device(atf_space* s) {
     }
     cudaGetLastError();
   }
+  // one device block for every parameter's tables and the small scratch words, filled by
+  // one host -> device copy: per parameter [values rp][divisibility magics rp][|values| rp]
+  // (rp = r rounded up to 128; the wide kernel reads 16-byte vectors of the last two on
+  // chunked ranges), then [values sorted ascending r][their positions r] (encode).
+  // magic(x) = ceil(2^32/|x|) mod 2^32 (0 for |x| == 1); magic(0) = 2^16, which no 16-bit
+  // x != 0 has, so the wide kernel's uniform test (n * magic mod 2^32) < 2^16 never accepts
+  // x == 0 for n != 0.  Padding: value 1, magic 2^16, |value| 1.
   size_t np = s->params.size();
-  s->d_range.assign(np, nullptr);
+  std::vector<size_t> off_range(np), off_sorted(np);
+  size_t words = 0;
   for (size_t p = 0; p < np; p++) {
-    // [values rp][divisibility magics rp][|values| rp], rp = r rounded up to 128 (the wide
-    // kernel reads 16-byte vectors of the last two straight from global memory on chunked
-    // ranges).  magic(x) = ceil(2^32/|x|) mod 2^32 (0 for |x| == 1); magic(0) = 2^16, which
-    // no 16-bit x != 0 has, so the wide kernel's uniform test (n * magic mod 2^32) < 2^16
-    // never accepts x == 0 for n != 0.  Padding: value 1, magic 2^16, |value| 1.
+    const size_t r = s->params[p].values.size(), rp = (r + 127) / 128 * 128;
+    off_range[p] = words;
+    words += 3 * rp;
+    off_sorted[p] = words;
+    words += (2 * r + 3) / 4 * 4;
+  }
+  const size_t off_scr = words;  // counter[kMaxGroups] | totals u64[kMaxGroups] | ovf[kMaxGroups] | bad[4] | root[16]
+  words += kMaxGroups + 2 * kMaxGroups + kMaxGroups + 4 + 16;
+  std::vector<int32_t> host(words, 0);
+  for (size_t p = 0; p < np; p++) {
     auto& v = s->params[p].values;
-    const size_t rp = (v.size() + 127) / 128 * 128;
-    s->d_range[p] = (int32_t*)dalloc(s, std::max<size_t>(16, rp * 12));
-    if (!s->d_range[p]) return fail(s, ATF_ERR_OOM, "range upload");
-    if (!v.empty()) {
-      std::vector<int32_t> buf(3 * rp, 1);
-      for (size_t j = 0; j < rp; j++) {
-        const bool real = j < v.size();
-        const uint32_t ax = real ? (v[j] < 0 ? 0u - (uint32_t)v[j] : (uint32_t)v[j]) : 1u;
-        if (real) buf[j] = v[j];
-        buf[rp + j] = (int32_t)(real ? (ax ? 0xffffffffu / ax + 1u : 0x10000u) : 0x10000u);
-        buf[2 * rp + j] = (int32_t)ax;
-      }
-      // pageable source: the call returns once `buf` has been staged
-      CUDA_TRY(s, cudaMemcpyAsync(s->d_range[p], buf.data(), buf.size() * 4, cudaMemcpyHostToDevice,
-                                  (cudaStream_t)s->opts.stream));
+    const size_t r = v.size(), rp = (r + 127) / 128 * 128;
+    int32_t* buf = host.data() + off_range[p];
+    for (size_t j = 0; j < rp; j++) {
+      const bool real = j < r;
+      const uint32_t ax = real ? (v[j] < 0 ? 0u - (uint32_t)v[j] : (uint32_t)v[j]) : 1u;
+      buf[j] = real ? v[j] : 1;
+      buf[rp + j] = (int32_t)(real ? (ax ? 0xffffffffu / ax + 1u : 0x10000u) : 0x10000u);
+      buf[2 * rp + j] = (int32_t)ax;
+    }
+    std::vector<int32_t> idx(r);
+    std::iota(idx.begin(), idx.end(), 0);
+    std::sort(idx.begin(), idx.end(), [&](int32_t x, int32_t y) { return v[x] < v[y]; });
+    int32_t* sb = host.data() + off_sorted[p];
+    for (size_t j = 0; j < r; j++) {
+      sb[j] = v[idx[j]];
+      sb[r + j] = idx[j];
     }
   }
+  s->table_bytes = words * 4;
+  s->d_table = (int32_t*)dalloc(s, s->table_bytes);
+  if (!s->d_table) return fail(s, ATF_ERR_OOM, "parameter tables (%zu bytes)", s->table_bytes);
+  // pageable source: the call returns once `host` has been staged
+  CUDA_TRY(s, cudaMemcpyAsync(s->d_table, host.data(), s->table_bytes, cudaMemcpyHostToDevice,
+                              (cudaStream_t)s->opts.stream));
+  s->d_range.assign(np, nullptr);
   s->d_sorted.assign(np, nullptr);
   for (size_t p = 0; p < np; p++) {
-    auto& v = s->params[p].values;
-    s->d_sorted[p] = (int32_t*)dalloc(s, std::max<size_t>(16, v.size() * 8));
-    if (!s->d_sorted[p]) return fail(s, ATF_ERR_OOM, "sorted range upload");
-    if (!v.empty()) {
-      std::vector<int32_t> idx(v.size());
-      std::iota(idx.begin(), idx.end(), 0);
-      std::sort(idx.begin(), idx.end(), [&](int32_t x, int32_t y) { return v[x] < v[y]; });
-      std::vector<int32_t> buf(2 * v.size());
-      for (size_t j = 0; j < v.size(); j++) {
-        buf[j] = v[idx[j]];
-        buf[v.size() + j] = idx[j];
-      }
-      CUDA_TRY(s, cudaMemcpyAsync(s->d_sorted[p], buf.data(), buf.size() * 4, cudaMemcpyHostToDevice,
-                                  (cudaStream_t)s->opts.stream));
-    }
+    s->d_range[p] = s->d_table + off_range[p];
+    s->d_sorted[p] = s->d_table + off_sorted[p];
   }
-  s->d_counter = (unsigned int*)dalloc(s, 4 * kMaxGroups);
-  s->d_totals = (unsigned long long*)dalloc(s, 8 * kMaxGroups);
-  s->d_ovf = (unsigned int*)dalloc(s, 4 * kMaxGroups);
-  s->d_bad = (unsigned int*)dalloc(s, 16);
-  s->d_root = (uint32_t*)dalloc(s, 64);
-  if (!s->d_counter || !s->d_totals || !s->d_ovf || !s->d_bad || !s->d_root) return fail(s, ATF_ERR_OOM, "scratch");
-  CUDA_TRY(s, cudaMemsetAsync(s->d_root, 0, 64, (cudaStream_t)s->opts.stream));
-  CUDA_TRY(s, cudaMallocHost(&s->h_totals, 8 * kMaxGroups));
-  CUDA_TRY(s, cudaMallocHost(&s->h_flags, 4 * kMaxGroups));
+  int32_t* scr = s->d_table + off_scr;
+  s->d_counter = (unsigned int*)scr;
+  s->d_totals = (unsigned long long*)(scr + kMaxGroups);
+  s->d_ovf = (unsigned int*)(scr + 3 * kMaxGroups);
+  s->d_bad = (unsigned int*)(scr + 4 * kMaxGroups);
+  s->d_root = (uint32_t*)(scr + 4 * kMaxGroups + 4);
+  // level totals and flags come back with the round's synchronisation (pageable is enough)
+  s->h_totals_v.assign(kMaxGroups, 0);
+  s->h_flags_v.assign(kMaxGroups, 0);
+  s->h_totals = s->h_totals_v.data();
+  s->h_flags = s->h_flags_v.data();
   s->arena.assign(s->groups.size(), {});
   s->gb.assign(s->groups.size(), {});
   for (auto& b : s->gb) {
@@ -986,11 +1000,10 @@ static void release_device(atf_space* s) {
   for (size_t g = 0; g < s->arena.size(); g++)
     for (auto& c : s->arena[g]) dfree(s, c.p, c.size);
   s->arena.clear();
-  for (size_t p = 0; p < s->d_range.size(); p++)
-    dfree(s, s->d_range[p], 12 * ((s->params[p].values.size() + 127) / 128 * 128));
+  dfree(s, s->d_table, s->table_bytes);
+  s->d_table = nullptr;
+  s->table_bytes = 0;
   s->d_range.clear();
-  for (size_t p = 0; p < s->d_sorted.size(); p++)
-    dfree(s, s->d_sorted[p], std::max<size_t>(16, s->params[p].values.size() * 8));
   s->d_sorted.clear();
   dfree(s, s->d_status, s->status_cap * 8);
   for (auto& b : s->gb) {
@@ -1005,13 +1018,11 @@ static void release_device(atf_space* s) {
     if (b.join) cudaEventDestroy(b.join);
   }
   s->gb.clear();
-  dfree(s, s->d_counter, 4 * kMaxGroups);
-  dfree(s, s->d_totals, 8 * kMaxGroups);
-  dfree(s, s->d_ovf, 4 * kMaxGroups);
-  dfree(s, s->d_bad, 16);
-  dfree(s, s->d_root, 64);
-  if (s->h_totals) cudaFreeHost(s->h_totals);
-  if (s->h_flags) cudaFreeHost(s->h_flags);
+  s->d_counter = nullptr;
+  s->d_totals = nullptr;
+  s->d_ovf = nullptr;
+  s->d_bad = nullptr;
+  s->d_root = nullptr;
   for (auto& ev : s->events)
     for (auto& e : ev) {
       cudaEventDestroy(e.first);
