@@ -6,9 +6,49 @@
 #include <cuda/atomic>
 #include <stdint.h>
 
+#include <map>
+#include <mutex>
+#include <tuple>
+
 #include "atf_internal.hpp"
 
 namespace atf {
+
+// ---------------------------------------------------------------- host launch helpers
+// Launch-configuration queries cached per process: the per-level host time sits between two
+// device-idle synchronisations, so attribute / occupancy queries are paid once, not per launch.
+inline int cached_sm_count() {
+  static int n = 0;
+  if (!n) {
+    int d = 0, c = 0;
+    cudaGetDevice(&d);
+    cudaDeviceGetAttribute(&c, cudaDevAttrMultiProcessorCount, d);
+    n = c > 0 ? c : 148;
+  }
+  return n;
+}
+// resident blocks per SM of kernel k (raises its dynamic shared-memory limit when needed);
+// returns < 0 (a cudaError_t, negated) on failure
+inline int cached_occupancy(const void* k, int block, int smem) {
+  static std::mutex mu;
+  static std::map<std::tuple<const void*, int, int>, int> occ;
+  static std::map<const void*, int> smem_limit;
+  std::lock_guard<std::mutex> lk(mu);
+  const auto key = std::make_tuple(k, block, smem);
+  auto it = occ.find(key);
+  if (it != occ.end()) return it->second;
+  int& lim = smem_limit[k];
+  if (smem > lim) {
+    cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    if (e != cudaSuccess) return -(int)e;
+    lim = smem;
+  }
+  int per_sm = 0;
+  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, block, smem);
+  if (e != cudaSuccess) return -(int)e;
+  occ[key] = per_sm;
+  return per_sm;
+}
 
 
 #define FULL 0xffffffffu

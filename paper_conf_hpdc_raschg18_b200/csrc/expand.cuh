@@ -1054,16 +1054,10 @@ __global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ L
 template <typename K>
 static int launch_persistent(K k, const LevelArgs& a, int block, void* stream) {
   const int smem = a.smem_bytes;
-  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e != cudaSuccess) return (int)e;
-  int per_sm = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, block, smem);
-  if (e != cudaSuccess) return (int)e;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int per_sm = cached_occupancy((const void*)k, block, smem);
+  if (per_sm < 0) return -per_sm;
   if (per_sm < 1) return (int)cudaErrorInvalidConfiguration;
-  uint64_t grid = (uint64_t)sms * per_sm;  // persistent: one wave, tiles by ticket
+  uint64_t grid = (uint64_t)cached_sm_count() * per_sm;  // persistent: one wave, tiles by ticket
   if (grid > a.n_tiles) grid = a.n_tiles;
   if (grid < 1) grid = 1;
   k<<<(unsigned)grid, block, smem, (cudaStream_t)stream>>>(a);
@@ -1336,18 +1330,14 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
 }
 
 template <typename K>
-static int launch_grid_warps(K k, const LevelArgs& a, void* stream) {
-  int per_sm = 0;
-  cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, 256, 0);
-  if (e != cudaSuccess) return (int)e;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  uint64_t grid = (uint64_t)sms * (per_sm > 0 ? per_sm : 1);
+static int launch_grid_warps(K k, const LevelArgs& a, void* stream, int smem = 0) {
+  const int per_sm = cached_occupancy((const void*)k, 256, smem);
+  if (per_sm < 0) return -per_sm;
+  uint64_t grid = (uint64_t)cached_sm_count() * (per_sm > 0 ? per_sm : 1);
   const uint64_t need = (a.n_tiles + 7) / 8;
   if (grid > need) grid = need;
   if (grid < 1) grid = 1;
-  k<<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>(a);
+  k<<<(unsigned)grid, 256, smem, (cudaStream_t)stream>>>(a);
   return (int)cudaGetLastError();
 }
 
@@ -1355,17 +1345,11 @@ static int launch_grid_warps(K k, const LevelArgs& a, void* stream) {
 template <typename K>
 static int launch_wtile_k(K k, const LevelArgs& a, void* stream) {
   const int smem = a.smem_bytes;
-  cudaError_t e = cudaFuncSetAttribute(k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e != cudaSuccess) return (int)e;
-  int per_sm = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, k, a.block, smem);
-  if (e != cudaSuccess) return (int)e;
+  const int per_sm = cached_occupancy((const void*)k, a.block, smem);
+  if (per_sm < 0) return -per_sm;
   if (per_sm < 1) return (int)cudaErrorInvalidConfiguration;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   const uint64_t nw = (uint64_t)(a.block / 32);
-  uint64_t grid = (uint64_t)sms * per_sm;
+  uint64_t grid = (uint64_t)cached_sm_count() * per_sm;
   const uint64_t need = (a.n_tiles + nw - 1) / nw;
   if (grid > need) grid = need;
   if (grid < 1) grid = 1;
@@ -1385,21 +1369,7 @@ static int launch_wtile_wc(const LevelArgs& a, void* stream) {
 
 template <int W>
 static int launch_nfast_emit_w(const LevelArgs& a, void* stream) {
-  const int smem = 8 * kNfEmitBufBytes;  // 8 warps per block
-  cudaError_t e = cudaFuncSetAttribute(nfast_emit<W>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-  if (e != cudaSuccess) return (int)e;
-  int per_sm = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, nfast_emit<W>, 256, smem);
-  if (e != cudaSuccess) return (int)e;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-  uint64_t grid = (uint64_t)sms * (per_sm > 0 ? per_sm : 1);
-  const uint64_t need = (a.n_tiles + 7) / 8;
-  if (grid > need) grid = need;
-  if (grid < 1) grid = 1;
-  nfast_emit<W><<<(unsigned)grid, 256, smem, (cudaStream_t)stream>>>(a);
-  return (int)cudaGetLastError();
+  return launch_grid_warps(nfast_emit<W>, a, stream, 8 * kNfEmitBufBytes);  // 8 warps per block
 }
 
 template <int W>

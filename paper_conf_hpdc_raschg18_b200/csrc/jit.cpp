@@ -302,9 +302,12 @@ int jit_nfast_launch(void* kernel, const LevelArgs& a, void* stream) {
     j.pv_range[i] = a.pv_range[i];
     j.pv_magic[i] = a.pv_magic[i];
   }
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
   uint64_t grid = (uint64_t)sms * 8;
   const uint64_t need = (a.n_tiles + 7) / 8;
   if (grid > need) grid = need;

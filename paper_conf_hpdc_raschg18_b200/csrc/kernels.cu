@@ -137,9 +137,7 @@ __global__ void __launch_bounds__(256) level_emit_kernel(const __grid_constant__
 
 int launch_level_emit(const LevelArgs& a, int words, void* stream) {
   if (a.n_tiles == 0) return 0;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int sms = cached_sm_count();
   // enough warps for the larger of the parents (CSR) and the records (pieces); the
   // record count is only known on the device, so the grid covers the stash capacity
   const uint64_t pieces = (a.stash_cap >> kPieceShift) + 1;
@@ -234,9 +232,7 @@ static int launch_decode(const DecodeArgs& a, const uint64_t* idx, const uint64_
     if (t >> 64) fits = 0;
     S = (uint64_t)t;
   }
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int sms = cached_sm_count();
   int64_t blocks = (n + 255) / 256;
   const int64_t cap = (int64_t)sms * 8;
   if (blocks > cap) blocks = cap;
@@ -349,9 +345,7 @@ __global__ void neighbor_kernel(const __grid_constant__ EncodeArgs a, const int3
 int launch_neighbors(const EncodeArgs& a, const int32_t* in, int64_t ld_in, int32_t* out, int64_t ld_out, int64_t n,
                      uint64_t seed, int max_tries, int32_t* moved, void* stream) {
   if (n <= 0) return 0;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int sms = cached_sm_count();
   int64_t blocks = (n + 255) / 256;
   if (blocks > (int64_t)sms * 8) blocks = (int64_t)sms * 8;
   neighbor_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, in, ld_in, out, ld_out, n, seed, max_tries,
@@ -362,9 +356,7 @@ int launch_neighbors(const EncodeArgs& a, const int32_t* in, int64_t ld_in, int3
 int launch_encode(const EncodeArgs& a, const int32_t* vals, int64_t ld, int64_t n, uint64_t* digits, uint64_t* idx,
                   void* stream) {
   if (n <= 0) return 0;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int sms = cached_sm_count();
   int64_t blocks = (n + 255) / 256;
   if (blocks > (int64_t)sms * 8) blocks = (int64_t)sms * 8;
   encode_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, vals, ld, n, digits, idx);
@@ -503,9 +495,7 @@ int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long 
                     void* stream, uint32_t* piece_tile, uint64_t piece_cap) {
   const int B = 256;
   const uint64_t n_tiles = n > 0 ? (uint64_t)((n + B * 4 - 1) / (B * 4)) : 1;
-  int dev = 0, sms = 0;
-  cudaGetDevice(&dev);
-  cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  const int sms = cached_sm_count();
   uint64_t grid = (uint64_t)sms * 4;
   if (grid > n_tiles) grid = n_tiles;
   scan_kernel<<<(unsigned)grid, B, 0, (cudaStream_t)stream>>>(in, out, n, status, counter, n_tiles, piece_tile, piece_cap);
