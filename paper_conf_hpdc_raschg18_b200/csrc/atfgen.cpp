@@ -795,10 +795,11 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
       a.cpt = best_cpt;
       a.nseg = best_nseg;
       a.chunk = 32 * best_cpt * best_nseg;
-      // small frontiers: fewer nodes per warp tile (power of two, >= 4 = one node quad of
-      // the hot loop) so that at least ~4 warp tiles per SM exist
+      // small and mid-size frontiers: fewer nodes per warp tile (power of two, >= 4 = one
+      // node quad of the hot loop) until ~256 tiles per SM exist: more tiles shorten the tail
+      // of heavy tiles (nodes with thousands of children); measured sweet spot on C5
       int tnodes = kWT;
-      while (tnodes > 4 && (a.n_parents + tnodes - 1) / tnodes < 148ull * 4) tnodes >>= 1;
+      while (tnodes > 4 && (a.n_parents + tnodes - 1) / tnodes < 148ull * 256) tnodes >>= 1;
       a.tile_nodes = tnodes;
       // 8 warps per CTA unless the level has too few tiles to give every SM a full CTA
       const uint64_t tiles = (a.n_parents + tnodes - 1) / tnodes;
