@@ -830,7 +830,7 @@ __device__ __forceinline__ void wtile_decode_item(uint32_t k, uint32_t ie, const
 }
 
 template <int W, int CPT, int HOT>
-__global__ void __launch_bounds__(256, 4) expand_wtile(const __grid_constant__ LevelArgs a) {
+__global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ LevelArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
   constexpr int SEG = 32 * CPT;
   const WarpLayout L = wtile_layout(a, W);
