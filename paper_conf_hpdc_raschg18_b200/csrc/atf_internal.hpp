@@ -121,7 +121,7 @@ enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1, K_WTILE = 2, K_NFAST = 3 }
 constexpr int kNfNPL = 4;  // narrow fast kernel: frontier nodes per lane (warp tile = 128 nodes)
 constexpr int kWT = 32;        // warp-tile kernel: frontier nodes per warp tile (one per lane)
 constexpr int kMaxSeg = 8;     // warp-tile kernel: candidate segments per node
-constexpr int kItemCap = 256;  // warp-tile kernel: items whose exact masks pass 1 keeps for the emit pass
+constexpr int kItemCap = 512;  // warp-tile kernel: items whose exact masks pass 1 keeps for the emit pass
 constexpr int kPieceShift = 10;  // level_emit_kernel copies the level in pieces of 2^10 records
 // Hot-loop filter of the wide kernel: a superset test of one conjunct, 2 instructions per
 // (node, candidate) pair (IMAD + ISETP.OR into a per-node predicate).
