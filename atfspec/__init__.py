@@ -170,6 +170,19 @@ def set_(*values: int) -> dict:
     return {"kind": "set", "values": [int(v) for v in values]}
 
 
+def enum(*names: str) -> dict:
+    """A named enumeration (S§8(f) NEXT-3): a SET of the integer codes 0..n-1 in the listed
+    order (reading #4), with the names kept for display; constraints compare codes
+    (e.g. ``equal(enum_code(rng, "local"))``)."""
+    if len(set(names)) != len(names):
+        raise ValueError("duplicate enum name")  # reading #5
+    return {"kind": "set", "values": list(range(len(names))), "names": [str(n) for n in names]}
+
+
+def enum_code(rng: dict, name: str) -> int:
+    return rng["names"].index(name)
+
+
 @dataclass
 class Param:
     name: str

@@ -72,6 +72,7 @@ class Space:
         opts = L.atf_space_opts(device, stream_ptr, self._alloc_cb, self._free_cb, None, flags)
         L.check(L.atf_space_create(C.byref(opts), C.byref(self._h)))
         self.names: List[str] = []
+        self._labels: List[Optional[List[str]]] = []  # enum names per parameter (atfspec.enum)
         if spec is not None:
             self.add_spec(spec)
 
@@ -87,6 +88,7 @@ class Space:
         out = C.c_int32()
         L.check(L.atf_space_add_param(self._h, name.encode(), C.byref(st), C.byref(out)), self._h)
         self.names.append(name)
+        self._labels.append(rng.get("names"))
         return out.value
 
     def add_constraint(self, pid: int, code) -> None:
@@ -269,6 +271,21 @@ class Space:
         L.check(L.atf_space_neighbors(self._h, values.data_ptr(), values.stride(0), n, seed & ((1 << 64) - 1),
                                       max_tries, out.data_ptr(), out.stride(0), moved.data_ptr(), sp), self._h)
         return out, moved
+
+    def to_named(self, configs) -> List[dict]:
+        """Decoded configurations (int32 [P, n]) -> one dict per configuration, parameter name ->
+        value, with the names of enum parameters (atfspec.enum) in place of their codes.
+        Host-side formatting for display / logging."""
+        cols = configs.cpu().numpy() if hasattr(configs, "cpu") else configs
+        names = self._labels
+        out = []
+        for j in range(cols.shape[1]):
+            row = {}
+            for p, nm in enumerate(self.names):
+                v = int(cols[p, j])
+                row[nm] = names[p][v] if names[p] is not None else v
+            out.append(row)
+        return out
 
     def close(self) -> None:
         if self._h:

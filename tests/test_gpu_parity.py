@@ -454,3 +454,21 @@ def test_divisible16_exhaustive(Space):
     bad = C.c_uint64(1)
     L.check(L.atf_test_divisible16(C.byref(bad)))
     assert bad.value == 0
+
+
+def test_enum_parameters(Space):
+    """Named enumerations (NEXT-3): SETs of codes in listed order; constraints compare codes;
+    decode + to_named give the names; the space equals the oracle's."""
+    s = A.Spec("enum_space")
+    mem = A.enum("global", "local", "private")
+    s.add("MEM", mem)
+    s.add("TS", A.interval(1, 64), A.divides(64) & ((A.P(0).eq(A.enum_code(mem, "local"))) | (A.X <= 8)))
+    s.add("VEC", A.enum("scalar", "vec2", "vec4"), A.X <= A.P(1))
+    _check_against_oracle(Space, s)
+    with Space(s) as sp:
+        sp.generate()
+        rows = sp.decode(torch.arange(sp.size(), dtype=torch.int64, device="cuda"))
+        named = sp.to_named(rows)
+        assert named[0] == {"MEM": "global", "TS": 1, "VEC": "scalar"}
+        assert {r["MEM"] for r in named} == {"global", "local", "private"}
+        assert all(r["TS"] <= 8 or r["MEM"] == "local" for r in named)
