@@ -1775,6 +1775,11 @@ atf_status atf_space_filter_product(atf_space* s, uint64_t* h_count, uint64_t* h
   if (!s || !h_count) return ATF_ERR_INVALID_ARG;
   atf_status e = plan(s);  // validation + static analysis (the product path needs no tree)
   if (e) return e;
+  {
+    u128 prod = 1;
+    for (auto& p : s->params) prod *= (u128)p.values.size();
+    if (prod >> 64) return fail(s, ATF_ERR_OVERFLOW, "full product >= 2^64");
+  }
   if ((e = ensure_device(s))) return e;
   ProductArgs a;
   std::memset(&a, 0, sizeof a);

@@ -265,3 +265,30 @@ def test_jit_level_sources_compile_for_sm100a(L, tmp_path):
     for p in procs:
         out, _ = p.communicate()
         assert p.returncode == 0, out
+
+
+def test_new_entry_points_validate_without_a_gpu(L):
+    """encode / neighbours before generate -> ATF_ERR_STATE; the full-product filter of a
+    product >= 2^64 -> ATF_ERR_OVERFLOW; bad arguments -> ATF_ERR_INVALID_ARG (no CUDA work)."""
+    import ctypes as C
+    from paper_conf_hpdc_raschg18_b200 import _lib as LL
+    from paper_conf_hpdc_raschg18_b200.space import _range_struct
+    sp = C.c_void_p()
+    LL.check(LL.atf_space_create(None, C.byref(sp)))
+    try:
+        keep = []
+        for i in range(5):  # 5 parameters of 2^14 values: product 2^70
+            rs, k = _range_struct(A.interval(1, 1 << 14))
+            keep.append(k)
+            pid = C.c_int32()
+            LL.check(LL.atf_space_add_param(sp, f"p{i}".encode(), C.byref(rs), C.byref(pid)), sp)
+        dummy = C.c_void_p(16)
+        assert LL.atf_space_encode_digits(sp, dummy, 4, 4, dummy, None) == -4      # STATE
+        assert LL.atf_space_encode_indices(sp, dummy, 4, 4, dummy, dummy, None) == -4
+        assert LL.atf_space_neighbors(sp, dummy, 4, 4, 1, 8, dummy, 4, dummy, None) == -4
+        assert LL.atf_space_encode_digits(sp, None, 4, 4, dummy, None) == -1       # INVALID_ARG
+        assert LL.atf_space_neighbors(sp, dummy, 2, 4, 1, 8, dummy, 4, dummy, None) == -1  # ld < n
+        cnt, tot = C.c_uint64(), C.c_uint64()
+        assert LL.atf_space_filter_product(sp, C.byref(cnt), C.byref(tot)) == -7  # OVERFLOW
+    finally:
+        LL.atf_space_destroy(sp)
