@@ -129,8 +129,7 @@ struct atf_space {
   uint32_t* d_root = nullptr;            // 8 zero words
   unsigned long long* h_totals = nullptr;  // -> h_totals_v
   unsigned int* h_flags = nullptr;         // -> h_flags_v
-  std::vector<unsigned long long> h_totals_v;
-  std::vector<unsigned int> h_flags_v;
+  std::vector<unsigned int> h_ctl;          // [totals u64 x kMaxGroups | ovf u32 x kMaxGroups]
   int32_t* d_table = nullptr;              // all parameter tables + scratch words (ensure_device)
   size_t table_bytes = 0;
   struct EvTriple { cudaEvent_t first = nullptr, mid = nullptr, second = nullptr; };
@@ -896,8 +895,10 @@ static atf_status ensure_device(atf_space* s) {
     off_sorted[p] = words;
     words += (2 * r + 3) / 4 * 4;
   }
-  const size_t off_scr = words;  // counter[kMaxGroups] | totals u64[kMaxGroups] | ovf[kMaxGroups] | bad[4] | root[16]
-  words += kMaxGroups + 2 * kMaxGroups + kMaxGroups + 4 + 16;
+  // totals u64[kMaxGroups] | ovf[kMaxGroups] | tile counters[kMaxGroups] | bad[4] | root[16]:
+  // one memset per level round resets [totals, ovf, counters], one copy reads [totals, ovf]
+  const size_t off_scr = words;
+  words += 2 * kMaxGroups + kMaxGroups + kMaxGroups + 4 + 16;
   std::vector<int32_t> host(words, 0);
   for (size_t p = 0; p < np; p++) {
     auto& v = s->params[p].values;
@@ -932,16 +933,16 @@ static atf_status ensure_device(atf_space* s) {
     s->d_sorted[p] = s->d_table + off_sorted[p];
   }
   int32_t* scr = s->d_table + off_scr;
-  s->d_counter = (unsigned int*)scr;
-  s->d_totals = (unsigned long long*)(scr + kMaxGroups);
-  s->d_ovf = (unsigned int*)(scr + 3 * kMaxGroups);
+  s->d_totals = (unsigned long long*)scr;
+  s->d_ovf = (unsigned int*)(scr + 2 * kMaxGroups);
+  s->d_counter = (unsigned int*)(scr + 3 * kMaxGroups);
   s->d_bad = (unsigned int*)(scr + 4 * kMaxGroups);
   s->d_root = (uint32_t*)(scr + 4 * kMaxGroups + 4);
-  // level totals and flags come back with the round's synchronisation (pageable is enough)
-  s->h_totals_v.assign(kMaxGroups, 0);
-  s->h_flags_v.assign(kMaxGroups, 0);
-  s->h_totals = s->h_totals_v.data();
-  s->h_flags = s->h_flags_v.data();
+  // level totals and flags come back with the round's synchronisation (pageable is enough):
+  // host mirror of [totals u64[kMaxGroups] | ovf u32[kMaxGroups]]
+  s->h_ctl.assign(3 * kMaxGroups, 0);
+  s->h_totals = reinterpret_cast<unsigned long long*>(s->h_ctl.data());
+  s->h_flags = s->h_ctl.data() + 2 * kMaxGroups;
   s->arena.assign(s->groups.size(), {});
   s->gb.assign(s->groups.size(), {});
   for (auto& b : s->gb) {
@@ -1049,11 +1050,11 @@ struct Pending {
   uint64_t cap;
   int chunk;  // arena chunk holding the child region
   size_t child_off;
+  bool joined = false;  // ran on the group's own stream (join event recorded)
 };
 
 static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parents, uint64_t n_parents, Pending& pd,
-                              uint64_t tile_base_unused = 0) {
-  (void)tile_base_unused;
+                              bool own_stream) {
   GroupPlan& gp = s->groups[g];
   LevelPlan& lp = gp.levels[k];
   cudaStream_t st = (cudaStream_t)s->opts.stream;  // allocations, memsets
@@ -1165,11 +1166,10 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
       return e;
     a.masks = gbf.masks;
   }
-  CUDA_TRY(s, cudaMemsetAsync(s->d_counter + g, 0, 4, st));
-  CUDA_TRY(s, cudaMemsetAsync(s->d_ovf + g, 0, 4, st));
+  // (tile counter, overflow flag and total of the group were reset by run_levels' round memset)
   // the level's kernels run on the group's stream after the allocations / memsets above;
   // run_levels joins the group streams back into the space's stream
-  const bool serial = (s->opts.flags & ATF_FLAG_SERIAL_GROUPS) != 0;
+  const bool serial = !own_stream || (s->opts.flags & ATF_FLAG_SERIAL_GROUPS) != 0;
   cudaStream_t ls = serial ? st : gbf.stream;
   if (!serial) {
     CUDA_TRY(s, cudaEventRecord(gbf.fork, st));
@@ -1204,7 +1204,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   }
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].second, ls));
   if (!serial) CUDA_TRY(s, cudaEventRecord(gbf.join, ls));
-  pd = Pending{g, k, n_parents, parents, (uint64_t*)csr, child, cap, which, off};
+  pd.joined = !serial;
+  pd = Pending{g, k, n_parents, parents, (uint64_t*)csr, child, cap, which, off, pd.joined};
   return ATF_OK;
 }
 
@@ -1215,6 +1216,12 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
   std::vector<int> k = k_from;
   for (;;) {
     std::vector<Pending> pend;
+    // levels launched this round: more than one -> one stream per group (concurrent)
+    int active = 0;
+    for (size_t i = 0; i < gs.size(); i++)
+      if (k[i] < (int)s->groups[gs[i]].levels.size() && fsize[i] > 0 && s->groups[gs[i]].levels[k[i]].r > 0) active++;
+    // one memset resets every group's level total, overflow flag and tile counter
+    if (active) CUDA_TRY(s, cudaMemsetAsync(s->d_totals, 0, 16 * kMaxGroups, st));
     for (size_t i = 0; i < gs.size(); i++) {
       int g = gs[i];
       int L = (int)s->groups[g].levels.size();
@@ -1242,17 +1249,15 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
         continue;
       }
       Pending pd;
-      atf_status e = queue_level(s, g, k[i], frontier[i], fsize[i], pd);
+      atf_status e = queue_level(s, g, k[i], frontier[i], fsize[i], pd, active > 1);
       if (e) return e;
       pend.push_back(pd);
     }
     if (pend.empty()) break;
-    if (!(s->opts.flags & ATF_FLAG_SERIAL_GROUPS))
-      for (auto& pd : pend) CUDA_TRY(s, cudaStreamWaitEvent(st, s->gb[pd.g].join, 0));  // join the group streams
-    for (auto& pd : pend) {
-      CUDA_TRY(s, cudaMemcpyAsync(s->h_totals + pd.g, s->d_totals + pd.g, 8, cudaMemcpyDeviceToHost, st));
-      CUDA_TRY(s, cudaMemcpyAsync(s->h_flags + pd.g, s->d_ovf + pd.g, 4, cudaMemcpyDeviceToHost, st));
-    }
+    for (auto& pd : pend)
+      if (pd.joined) CUDA_TRY(s, cudaStreamWaitEvent(st, s->gb[pd.g].join, 0));  // join the group streams
+    // one copy brings back [totals | overflow flags] of every group
+    CUDA_TRY(s, cudaMemcpyAsync(s->h_ctl.data(), s->d_totals, 12 * kMaxGroups, cudaMemcpyDeviceToHost, st));
     CUDA_TRY(s, cudaStreamSynchronize(st));
     for (auto& pd : pend) {
       size_t i = std::find(gs.begin(), gs.end(), pd.g) - gs.begin();
