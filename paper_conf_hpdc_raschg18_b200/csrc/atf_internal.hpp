@@ -79,7 +79,8 @@ struct LevelArgs {
   Term terms[kMaxTerms];
   int32_t need_slots_smem;  // a generic term reads slots per candidate
   void* masks;              // nfast: per-parent accept masks (pass 1 -> pass 2)
-  int32_t mask_bytes;       // 1, 2 or 4
+  int32_t mask_bytes;       // 1, 2, 4 or 8
+  int32_t direct;           // warp-tile: tiny level written in place (look-back over <= 16 tiles)
   int32_t nf_ok;            // narrow fast path possible (no gates / generic terms / wide variants)
   NfOp nf_op[kMaxTerms][2];
   const uint32_t* pv_magic[kMaxSlots];  // divisor magics of each ancestor's range

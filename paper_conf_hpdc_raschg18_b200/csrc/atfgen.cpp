@@ -117,6 +117,8 @@ struct atf_space {
     size_t scratch_cap = 0;
     uint32_t* stash = nullptr;  // wide levels: children in tile segments before the final copy
     size_t stash_cap = 0;       // bytes
+    unsigned long long* status = nullptr;  // tiny wide levels: look-back tile status words
+    size_t status_cap = 0;                 // entries
     cudaStream_t stream = nullptr;
     cudaEvent_t fork = nullptr, join = nullptr;
   };
@@ -1012,6 +1014,7 @@ static void release_device(atf_space* s) {
     dfree(s, b.scratch, b.scratch_cap);
     dfree(s, (char*)b.stash, b.stash_cap);
     dfree(s, b.masks, b.masks_cap);
+    dfree(s, (char*)b.status, b.status_cap * 8);
     if (b.stream) {
       cudaStreamSynchronize(b.stream);
       cudaStreamDestroy(b.stream);
@@ -1159,6 +1162,20 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     a.piece_tile = piece_tile;
     CUDA_TRY(s, cudaMemsetAsync(d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
   }
+  // tiny wide levels: one launch, in place (decoupled look-back over <= 16 warp tiles; with
+  // more tiles the waits cost more than the two saved launches)
+  a.direct = (a.kind == K_WTILE && a.n_tiles <= 16 && !(s->opts.flags & ATF_FLAG_LEGACY_WIDE)) ? 1 : 0;
+  if (a.direct) {
+    const size_t need = (size_t)a.n_tiles + 1;
+    if (need > gbf.status_cap) {
+      dfree(s, (char*)gbf.status, gbf.status_cap * 8);
+      gbf.status_cap = std::max<size_t>(need, 64);
+      gbf.status = (unsigned long long*)dalloc(s, gbf.status_cap * 8);
+      if (!gbf.status) { gbf.status_cap = 0; return fail(s, ATF_ERR_OOM, "tile status"); }
+    }
+    a.status = gbf.status;
+    CUDA_TRY(s, cudaMemsetAsync(gbf.status, 0, need * 8, st));
+  }
   // narrow fast levels: pass 1 writes per-parent accept masks, pass 2 the children in place
   if (a.kind == K_NFAST) {
     a.mask_bytes = a.r <= 8 ? 1 : (a.r <= 16 ? 2 : (a.r <= 32 ? 4 : 8));
@@ -1193,7 +1210,9 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   if (use_jit) s->data[g][k].kernel = 4;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].mid, ls));
   if (!use_jit) s->data[g][k].kernel = a.kind;
-  if (a.kind == K_NFAST) {
+  if (a.direct) {
+    // nothing more: the expand kernel placed the level
+  } else if (a.kind == K_NFAST) {
     ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, ls);
     if (!ce) ce = launch_nfast_emit(a, gp.words, ls);
     if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));

@@ -991,16 +991,35 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
       if (lane >= o) co += y;
     }
     const uint32_t total = __shfl_sync(FULL, co, 31);
-    if (lane < tn) a.csr[node0 + lane] = co - cn;
     s_cnt[lane] = 0u;  // for the next tile (read above by this lane only)
     unsigned long long sgb = 0;
-    if (lane == 0) {
-      sgb = total ? atomicAdd(a.stash_top, (unsigned long long)total) : 0ull;
-      if (total && sgb + total > a.stash_cap) atomicOr(a.overflow_flag, 1u);
-      a.tile_total[cur] = total;
-      a.tile_seg[cur] = sgb;
+    uint32_t* dst = a.stash;
+    uint64_t cap = a.stash_cap;
+    if (a.direct) {
+      // tiny level (a handful of tiles, all resident): the tile's final base by decoupled
+      // look-back; children and CSR entries go straight to their final place (no scan /
+      // copy launches)
+      sgb = lookback(a.status, cur, total, lane);
+      dst = a.child_rec;
+      cap = a.child_cap;
+      if (lane < tn) a.csr[node0 + lane] = sgb + co - cn;
+      if (lane == 0) {
+        if (sgb + total > cap) atomicOr(a.overflow_flag, 1u);
+        if ((uint64_t)cur == a.n_tiles - 1) {
+          *a.total_out = sgb + total;
+          a.csr[a.n_parents] = sgb + total;
+        }
+      }
+    } else {
+      if (lane < tn) a.csr[node0 + lane] = co - cn;
+      if (lane == 0) {
+        sgb = total ? atomicAdd(a.stash_top, (unsigned long long)total) : 0ull;
+        if (total && sgb + total > a.stash_cap) atomicOr(a.overflow_flag, 1u);
+        a.tile_total[cur] = total;
+        a.tile_seg[cur] = sgb;
+      }
+      sgb = __shfl_sync(FULL, sgb, 0);
     }
-    sgb = __shfl_sync(FULL, sgb, 0);
     // ---- emit (A6): items in order; lane writes its item's children at their final rank
     uint64_t carry = sgb;
     for (uint32_t R = 0; R < T; R += 32) {
@@ -1035,11 +1054,11 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
         while (m) {
           const int c = __ffs(m) - 1;
           m &= m - 1;
-          if (rank < a.stash_cap) {
+          if (rank < cap) {
             uint32_t out[W];
 #pragma unroll
             for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? (pos0 + c) << a.field_shift : 0u);
-            store_record<W>(a.stash + rank * W, out);
+            store_record<W>(dst + rank * W, out);
           }
           rank++;
         }
