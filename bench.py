@@ -239,7 +239,7 @@ def e2e_generation(spec, steps, dist_ctx=None):
         torch.cuda.synchronize()
         dt = time.perf_counter() - t0
         if dist_ctx:
-            t = torch.tensor([dt], dtype=torch.float64, device="cuda")
+            t = torch.tensor([dt], dtype=torch.float64, device=dist_ctx["dev"])
             dist_ctx["dist"].all_reduce(t, op=dist_ctx["dist"].ReduceOp.MAX)
             dt = float(t.item())
         if i:
@@ -365,12 +365,21 @@ def main():
         return
 
     import torch
-    torch.cuda.set_device(local)
+    # one process per GPU; ATF_DIST_BACKEND=gloo (ranks may then share a GPU) only exercises the
+    # sharded path on a single-GPU box — its timings are not a scaling measurement
+    backend = os.environ.get("ATF_DIST_BACKEND", "nccl")
+    dev_index = local % max(1, torch.cuda.device_count()) if backend != "nccl" else local
+    torch.cuda.set_device(dev_index)
+    local = dev_index
     dist_ctx = None
     if world > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
-        dist_ctx = {"dist": dist, "rank": rank, "world": world}
+        if backend == "nccl":
+            dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+        else:
+            dist.init_process_group(backend)
+        dist_ctx = {"dist": dist, "rank": rank, "world": world,
+                    "dev": torch.device("cuda", local) if backend == "nccl" else torch.device("cpu")}
 
     peaks = _peaks()
     sm_max = float(peaks.get("sm_max_mhz", 1965.0))
@@ -379,7 +388,7 @@ def main():
     clocks = clk.summary()
     ms = float(np.mean(res["ms"]))
     if dist_ctx:
-        t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+        t = torch.tensor([ms], dtype=torch.float64, device=dist_ctx["dev"])
         dist_ctx["dist"].all_reduce(t, op=dist_ctx["dist"].ReduceOp.MAX)
         ms = float(t.item())
     leaves = sum(res["group_sizes"])                      # global (finalize_shard) sizes
