@@ -181,7 +181,9 @@ def roofline_of(res, sm_mhz, spec_name=None, step_ms=None):
     lv = [(gi, k, l) for gi, g in enumerate(plan["groups"]) for k, l in enumerate(g["levels"])]
     costs = [l["cost"] for _, _, l in lv]
     st = res["stats"]
-    ops = [s["evals"] * c for s, c in zip(st, costs)]
+    # evaluated pairs: the spec's f_{k-1} x r_k, less the pairs the warp-tile hot loop rejects
+    # wholesale by its per-segment |x| bounds (stats "pairs", ATF_FLAG_TIMING)
+    ops = [(s["pairs"] or s["evals"]) * c for s, c in zip(st, costs)]
     exp_ms = np.array(res["level_exp_ms"], dtype=np.float64).mean(axis=0)
     lvl_ms = np.array(res["level_ms"], dtype=np.float64).mean(axis=0)
     d = int(np.argmax(exp_ms))
@@ -199,7 +201,8 @@ def roofline_of(res, sm_mhz, spec_name=None, step_ms=None):
     return {"bound": "alu", "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tops/s",
             "frac": achieved / peak, "traffic": tr["dram_bytes"] if tr else None,
             "traffic_source": tr["source"] if tr else None,
-            "kernel": kname, "launch": f"group {g} level {k + 1} (r={st[d]['r']}, evals={st[d]['evals']})",
+            "kernel": kname, "launch": f"group {g} level {k + 1} (r={st[d]['r']}, evals={st[d]['evals']}, "
+                                       f"evaluated pairs={st[d]['pairs'] or st[d]['evals']})",
             "ops_per_launch": ops[d], "launch_ms": float(exp_ms[d]), "algorithmic_bytes_per_launch": int(alg_bytes),
             "peak_clock_mhz": sm_mhz, "peak_source": "4 SMSP x 32 lanes x 148 SMs x clock (B200_PROFILING.md unit counts)",
             "cost_table": "DIVX/MULX/DIVPROD 2, QDIV 6, CMP 2, AND 1, GENERIC = bytecode ops",

@@ -274,6 +274,10 @@ typedef struct {
   float expand_ms;  /* device time of the level's expand kernel alone (ATF_FLAG_TIMING), else -1 */
   int32_t kernel;   /* expand kernel: 0 = narrow (r <= 64), 1 = block-tile wide, 2 = warp-tile wide,
                        3 = narrow fast, 4 = narrow fast specialised at run time (NVRTC) */
+  uint64_t pairs;   /* ATF_FLAG_TIMING: (node, candidate) pairs evaluated = evals, except on
+                       warp-tile levels with a hot filter: the pairs the hot loop tested (the rest
+                       are rejected by the per-segment |x| bounds: x | n needs |x| <= |n|, d | x
+                       needs |x| >= |d|).  0 without ATF_FLAG_TIMING */
 } atf_level_stats;
 atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap, int32_t* n_out);
 

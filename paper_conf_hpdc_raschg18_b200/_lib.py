@@ -50,7 +50,8 @@ class atf_level_view(C.Structure):
 class atf_level_stats(C.Structure):
     _fields_ = [("group", C.c_int32), ("level", C.c_int32), ("param", C.c_int32), ("r", C.c_int64),
                 ("evals", C.c_uint64), ("f", C.c_uint64), ("ms", C.c_float), ("path", C.c_int32),
-                ("expand_ms", C.c_float), ("kernel", C.c_int32)]
+                ("expand_ms", C.c_float), ("kernel", C.c_int32),
+                ("pairs", C.c_uint64)]
 
 
 SP = C.c_void_p  # atf_space*

@@ -54,6 +54,7 @@ struct NfOp {
 };
 
 // Per-level program + geometry, passed by value to the expand kernel.
+constexpr int kMaxSeg = 8;     // warp-tile kernel: candidate segments per node
 struct LevelArgs {
   // frontier = level k-1 of this group (k == 0: a single empty root record)
   const uint32_t* parent_rec;
@@ -113,6 +114,11 @@ struct LevelArgs {
   int32_t rw, sw;           // wide: bitmap words per node (chunk/32), summary words (ceil(rw/32))
   int32_t qcap;             // wide: slow-path queue entries per tile
   int32_t nseg;             // warp-tile: candidate segments of 32*cpt per node (<= kMaxSeg)
+  // warp-tile hot filter, per segment: min / max |x| over its candidates (0 / 0xffffffff
+  // when a candidate is 0).  x | n with n != 0 needs |x| <= |n|, d | x with x != 0 needs
+  // |x| >= |d|: a node quad outside a segment's bounds has no item there
+  uint32_t seg_lo[kMaxSeg], seg_hi[kMaxSeg];
+  unsigned long long* pairs_out;  // ATF_FLAG_TIMING: (node, candidate) pairs the hot loop tested
   int64_t n_chunks;         // candidate chunks per node (r > chunk); tile_nodes == 4 padded, 1 real
   uint64_t n_tiles;
   uint32_t qmax;            // T_QDIV table covers quotients [0, qmax]
@@ -121,7 +127,6 @@ struct LevelArgs {
 enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1, K_WTILE = 2, K_NFAST = 3 };
 constexpr int kNfNPL = 4;  // narrow fast kernel: frontier nodes per lane (warp tile = 128 nodes)
 constexpr int kWT = 32;        // warp-tile kernel: frontier nodes per warp tile (one per lane)
-constexpr int kMaxSeg = 8;     // warp-tile kernel: candidate segments per node
 constexpr int kItemCap = 512;  // warp-tile kernel: items whose exact masks pass 1 keeps for the emit pass
 constexpr int kPieceShift = 10;  // level_emit_kernel copies the level in pieces of 2^10 records
 // Hot-loop filter of the wide kernel: a superset test of one conjunct, 2 instructions per

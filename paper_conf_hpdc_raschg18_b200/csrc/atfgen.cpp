@@ -66,6 +66,8 @@ struct LevelPlan {
   bool generic = false;
   std::string desc;
   void* jit = nullptr;       // NVRTC-specialised narrow kernel (jit.cpp), if any
+  int seg_cpt = -1;          // cpt the cached warp-tile segment bounds were computed for
+  uint32_t seg_lo[kMaxSeg], seg_hi[kMaxSeg];
   bool jit_tried = false;
 };
 
@@ -89,6 +91,9 @@ struct LevelData {
   float ms = -1.f;         // expand + scan + emit of the level (ATF_FLAG_TIMING)
   float expand_ms = -1.f;  // the expand kernel alone
   int32_t kernel = -1;     // KernelKind of the expand launch
+  uint64_t pairs = 0;      // (node, candidate) pairs evaluated (ATF_FLAG_TIMING; = evals unless
+                           // the warp-tile hot loop skipped segments by their |x| bounds)
+  bool seg_skip = false;   // the level's hot loop applies the segment bounds
 };
 
 }  // namespace
@@ -128,6 +133,7 @@ struct atf_space {
   unsigned long long* d_totals = nullptr;  // [kMaxGroups]
   unsigned int* d_ovf = nullptr;         // [kMaxGroups]
   unsigned int* d_bad = nullptr;         // decode flag
+  unsigned long long* d_pairs = nullptr;  // [kMaxGroups] hot-loop pairs tested (ATF_FLAG_TIMING)
   uint32_t* d_root = nullptr;            // 8 zero words
   unsigned long long* h_totals = nullptr;  // -> h_totals_v
   unsigned int* h_flags = nullptr;         // -> h_flags_v
@@ -900,7 +906,7 @@ static atf_status ensure_device(atf_space* s) {
   // totals u64[kMaxGroups] | ovf[kMaxGroups] | tile counters[kMaxGroups] | bad[4] | root[16]:
   // one memset per level round resets [totals, ovf, counters], one copy reads [totals, ovf]
   const size_t off_scr = words;
-  words += 2 * kMaxGroups + kMaxGroups + kMaxGroups + 4 + 16;
+  words += 2 * kMaxGroups + kMaxGroups + kMaxGroups + 4 + 16 + 2 * kMaxGroups;  // + pairs u64 (timing)
   std::vector<int32_t> host(words, 0);
   for (size_t p = 0; p < np; p++) {
     auto& v = s->params[p].values;
@@ -940,6 +946,7 @@ static atf_status ensure_device(atf_space* s) {
   s->d_counter = (unsigned int*)(scr + 3 * kMaxGroups);
   s->d_bad = (unsigned int*)(scr + 4 * kMaxGroups);
   s->d_root = (uint32_t*)(scr + 4 * kMaxGroups + 4);
+  s->d_pairs = (unsigned long long*)(scr + 4 * kMaxGroups + 20);
   // level totals and flags come back with the round's synchronisation (pageable is enough):
   // host mirror of [totals u64[kMaxGroups] | ovf u32[kMaxGroups]]
   s->h_ctl.assign(3 * kMaxGroups, 0);
@@ -1027,6 +1034,7 @@ static void release_device(atf_space* s) {
   s->d_totals = nullptr;
   s->d_ovf = nullptr;
   s->d_bad = nullptr;
+  s->d_pairs = nullptr;
   s->d_root = nullptr;
   for (auto& ev : s->events)
     for (auto& e : ev) {
@@ -1079,6 +1087,27 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     a.pv_magic[i] = reinterpret_cast<const uint32_t*>(s->d_range[lp.pv_param[i]]) + rpi;
   }
   choose_geometry(a, gp.words, (s->opts.flags & ATF_FLAG_LEGACY_WIDE) != 0);
+  if (a.kind == K_WTILE && a.hot != HOT_NONE) {
+    if (lp.seg_cpt != a.cpt) {  // per-segment |x| bounds of the hot filter (cached per level)
+      const std::vector<int32_t>& v = s->params[lp.param].values;
+      const int seg = 32 * a.cpt;
+      for (int sg = 0; sg < kMaxSeg; sg++) {
+        uint32_t lo = 0xffffffffu, hi = 0u;
+        for (int j = sg * seg; j < std::min((int)v.size(), (sg + 1) * seg); j++) {
+          const uint32_t ax = (uint32_t)(v[j] < 0 ? -(int64_t)v[j] : (int64_t)v[j]);
+          if (ax == 0) { lo = 0u; hi = 0xffffffffu; break; }
+          lo = std::min(lo, ax);
+          hi = std::max(hi, ax);
+        }
+        lp.seg_lo[sg] = lo;
+        lp.seg_hi[sg] = hi;
+      }
+      lp.seg_cpt = a.cpt;
+    }
+    for (int sg = 0; sg < kMaxSeg; sg++) { a.seg_lo[sg] = lp.seg_lo[sg]; a.seg_hi[sg] = lp.seg_hi[sg]; }
+  }
+  a.pairs_out = (s->opts.flags & ATF_FLAG_TIMING) ? s->d_pairs + g : nullptr;
+  s->data[g][k].seg_skip = a.kind == K_WTILE && a.hot != HOT_NONE;
   a.n_tiles = a.n_chunks > 1 ? n_parents * (uint64_t)a.n_chunks
                              : (n_parents + (uint64_t)a.tile_nodes - 1) / (uint64_t)a.tile_nodes;
   if (a.smem_bytes > 227 * 1024)
@@ -1241,6 +1270,7 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       if (k[i] < (int)s->groups[gs[i]].levels.size() && fsize[i] > 0 && s->groups[gs[i]].levels[k[i]].r > 0) active++;
     // one memset resets every group's level total, overflow flag and tile counter
     if (active) CUDA_TRY(s, cudaMemsetAsync(s->d_totals, 0, 16 * kMaxGroups, st));
+    if (active && (s->opts.flags & ATF_FLAG_TIMING)) CUDA_TRY(s, cudaMemsetAsync(s->d_pairs, 0, 8 * kMaxGroups, st));
     for (size_t i = 0; i < gs.size(); i++) {
       int g = gs[i];
       int L = (int)s->groups[g].levels.size();
@@ -1278,6 +1308,9 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
     // one copy brings back [totals | overflow flags] of every group
     CUDA_TRY(s, cudaMemcpyAsync(s->h_ctl.data(), s->d_totals, 12 * kMaxGroups, cudaMemcpyDeviceToHost, st));
     CUDA_TRY(s, cudaStreamSynchronize(st));
+    unsigned long long h_pairs[kMaxGroups] = {};
+    if (s->opts.flags & ATF_FLAG_TIMING)
+      CUDA_TRY(s, cudaMemcpy(h_pairs, s->d_pairs, sizeof(h_pairs), cudaMemcpyDeviceToHost));
     for (auto& pd : pend) {
       size_t i = std::find(gs.begin(), gs.end(), pd.g) - gs.begin();
       uint64_t total = s->h_totals[pd.g];
@@ -1300,6 +1333,7 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       {
         cudaEventElapsedTime(&d.ms, s->events[pd.g][pd.k].first, s->events[pd.g][pd.k].second);
         cudaEventElapsedTime(&d.expand_ms, s->events[pd.g][pd.k].first, s->events[pd.g][pd.k].mid);
+        d.pairs = d.seg_skip ? h_pairs[pd.g] : d.evals;
       }
       frontier[i] = pd.child;
       fsize[i] = total;
@@ -1919,6 +1953,7 @@ atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap
         o.path = lp.generic ? 1 : 0;
         o.expand_ms = d.expand_ms;
         o.kernel = d.kernel;
+        o.pairs = d.pairs;
       }
       n++;
     }

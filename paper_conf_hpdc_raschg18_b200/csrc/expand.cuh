@@ -880,6 +880,7 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
   nxt = __shfl_sync(FULL, nxt, 0);
   uint32_t pre[W];
   uint64_t pre_tile = ~0ull;
+  uint64_t pairs = 0;  // hot-loop pairs tested (ATF_FLAG_TIMING statistics)
   while ((uint64_t)cur < a.n_tiles) {
     const uint64_t node0 = (uint64_t)cur * TN;
     const uint64_t remn = a.n_parents - node0;
@@ -903,6 +904,20 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
       s_hot[lane] = md;
       s_hot2[lane] = md - 1u;
     }
+    // segment bounds of the hot filter (A4): x | n (n != 0) needs |x| <= n, d | x (x != 0)
+    // needs |x| >= d, so a node quad whose largest n (smallest d) lies outside a segment's
+    // [seg_lo, seg_hi] has no item there.  Lane 4q holds quad q's bound; rejected nodes
+    // bound nothing, n == 0 (divisible by every x) bounds everything.
+    uint32_t qb = 0;
+    if (HOT == HOT_DIVX) {
+      qb = ok ? (s_hot[lane] ? s_hot[lane] : 0xffffffffu) : 0u;
+      qb = max(qb, __shfl_xor_sync(FULL, qb, 1));
+      qb = max(qb, __shfl_xor_sync(FULL, qb, 2));
+    } else if (HOT == HOT_MULX) {
+      qb = ok ? (uint32_t)s_opa[hot_t * kWT + lane] : 0xffffffffu;
+      qb = min(qb, __shfl_xor_sync(FULL, qb, 1));
+      qb = min(qb, __shfl_xor_sync(FULL, qb, 2));
+    }
     // claim the tile after next; prefetch the next tile's parent records
     uint32_t nn = nxt;
     if (lane == 0 && (uint64_t)nxt < a.n_tiles) nn = atomicAdd(a.tile_counter, 1u);
@@ -924,7 +939,17 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
         const uint32_t* tp = s_tab + sg * SEG + lane;
 #pragma unroll
         for (int c = 0; c < CPT; c++) hm[c] = tp[c * 32];
+        uint32_t sb = HOT == HOT_DIVX ? a.seg_lo[0] : a.seg_hi[0];  // no dynamic param indexing
+#pragma unroll
+        for (int i = 1; i < kMaxSeg; i++)
+          if (sg == i) sb = HOT == HOT_DIVX ? a.seg_lo[i] : a.seg_hi[i];
         for (int q = 0; q < nq; q++) {
+          const uint32_t qv = __shfl_sync(FULL, qb, 4 * q);
+          if (HOT == HOT_DIVX ? qv < sb : qv > sb) {
+            if (lane == 0) *reinterpret_cast<uint4*>(s_items + sg * kWT + 4 * q) = make_uint4(0u, 0u, 0u, 0u);
+            continue;
+          }
+          pairs += (uint64_t)min(4, tn - 4 * q) * (uint64_t)min(SEG, r - sg * SEG);
           const uint4 n4 = *reinterpret_cast<const uint4*>(s_hot + 4 * q);
           uint32_t m0 = 0xffffffffu, m1 = 0xffffffffu, m2 = 0xffffffffu, m3 = 0xffffffffu;
 #pragma unroll
@@ -1068,6 +1093,7 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
     cur = nxt;
     nxt = nn;
   }
+  if (a.pairs_out && lane == 0 && pairs) atomicAdd(a.pairs_out, (unsigned long long)pairs);
 }
 
 template <typename K>

@@ -472,3 +472,44 @@ def test_enum_parameters(Space):
         assert named[0] == {"MEM": "global", "TS": 1, "VEC": "scalar"}
         assert {r["MEM"] for r in named} == {"global", "local", "private"}
         assert all(r["TS"] <= 8 or r["MEM"] == "local" for r in named)
+
+
+def _seg_bound_spec(kind, order):
+    """Wide divisibility chains whose candidate sets put 0, negatives and large values in
+    different warp-tile segments (sorted, reversed, shuffled): the per-segment |x| bounds of
+    the hot filter (x | n needs |x| <= |n|, d | x needs |x| >= |d|, 0 passes both) must not
+    drop an accepted pair."""
+    import random
+    vals = list(range(-40, 0)) + [0] + list(range(1, 1500))
+    if order == "reversed":
+        vals = vals[::-1]
+    elif order == "shuffled":
+        random.Random(7).shuffle(vals)
+    s = A.Spec(f"segbound_{kind}_{order}")
+    alias = A.divides if kind == "divx" else A.is_multiple_of
+    s.add("a", A.interval(-3, 40))
+    s.add("b", A.set_(*vals), alias(s.P("a")))
+    s.add("c", A.set_(*vals), alias(s.P("b")))
+    return s
+
+
+@pytest.mark.parametrize("kind", ["divx", "mulx"])
+@pytest.mark.parametrize("order", ["sorted", "reversed", "shuffled"])
+def test_segment_bounds_parity(Space, kind, order):
+    _check_against_oracle(Space, _seg_bound_spec(kind, order), decode_all_max=200_000)
+
+
+def test_segment_bounds_skip_work_not_results(Space):
+    """ATF_FLAG_TIMING statistics: evaluated pairs never exceed the spec's f_{k-1} r_k, equal it
+    on levels without the filter, and fall below it where nodes' values exclude whole segments
+    (C5's divisor chain: deep levels hold small values).  Level sizes stay the oracle's
+    (C5 closed form, Piltz divisor sums)."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    spec = A.c5_chains(4096, 4)
+    with Space(spec, flags=L.ATF_FLAG_TIMING | L.ATF_FLAG_SERIAL_GROUPS) as sp:
+        sp.generate()
+        st = sp.stats()
+        assert all(0 < x["pairs"] <= x["evals"] for x in st if x["evals"])
+        g0 = [x for x in st if x["group"] == 0]
+        assert g0[-1]["pairs"] < g0[-1]["evals"] // 2
+        assert sp.level_sizes(0) == cf.piltz_D(4096, 4)
