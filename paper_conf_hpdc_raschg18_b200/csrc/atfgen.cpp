@@ -798,6 +798,15 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
         if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) { a.hot = HOT_DIVX; a.hot_term = t; break; }
         if (T.kind == T_MULX && T.variant == V16) { a.hot = HOT_MULX; a.hot_term = t; break; }
       }
+      static const int fine = [] { const char* e = getenv("ATF_SEG_FINE"); return e ? atoi(e) : 0; }();
+      if (fine && a.hot != HOT_NONE) {
+        // finer segments: more node quads fall outside a segment's |x| bounds
+        for (int cpt : {4, 8, 12, 16, 20, 24, 32}) {
+          if (cpt < fine) continue;
+          const int64_t seg = 32 * (int64_t)cpt, nseg = ((int64_t)r + seg - 1) / seg;
+          if (nseg <= kMaxSeg) { best_cpt = cpt; best_nseg = (int)nseg; break; }
+        }
+      }
       a.kind = K_WTILE;
       a.cpt = best_cpt;
       a.nseg = best_nseg;
