@@ -7,6 +7,6 @@ print(f"C5 ms/step {d['ms_per_step']:.2f}  configs/s {d['value']:.3g}  evals/s {
       f"roofline frac {d['roofline']['frac']:.3f}  e2e {d['e2e']['value']:.3g}  clocks {d['clocks']}")
 for k, v in d.get("secondary", {}).items():
     if "ms_per_step" in v:
-        print(f"{k:8s} ms {v['ms_per_step']:.3f} frac {v['roofline_frac']:.3f} levels {v['level_ms']}")
+        print(f"{k:8s} ms {v['ms_per_step']:.3f} frac {v.get('dominant_frac', 0):.3f} levels {v['level_ms']}")
     else:
         print(k, v)
