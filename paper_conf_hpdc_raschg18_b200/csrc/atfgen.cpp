@@ -798,7 +798,15 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
         if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) { a.hot = HOT_DIVX; a.hot_term = t; break; }
         if (T.kind == T_MULX && T.variant == V16) { a.hot = HOT_MULX; a.hot_term = t; break; }
       }
-      static const int fine = [] { const char* e = getenv("ATF_SEG_FINE"); return e ? atoi(e) : 0; }();
+      // Divisor filters over ranges that already span several segments: finer segments (the
+      // smallest cpt >= 8 that fits kMaxSeg) let small node values skip more candidates
+      // (C5 9.44 -> 9.33 ms measured; multiples filters and single-segment levels lose, so
+      // they keep the cost-model choice).  ATF_SEG_FINE / ATF_SEG_FINE_KIND override (A/B).
+      static const int fine_env = [] { const char* e = getenv("ATF_SEG_FINE"); return e ? atoi(e) : -1; }();
+      static const int fine_kind = [] { const char* e = getenv("ATF_SEG_FINE_KIND"); return e ? atoi(e) : 0; }();
+      int fine = 0;
+      if (fine_env >= 0) fine = (fine_kind == 0 || fine_kind == a.hot) ? fine_env : 0;
+      else if (a.hot == HOT_DIVX && best_nseg >= 2) fine = 8;
       if (fine && a.hot != HOT_NONE) {
         // finer segments: more node quads fall outside a segment's |x| bounds
         for (int cpt : {4, 8, 12, 16, 20, 24, 32}) {
