@@ -107,7 +107,16 @@ def flush_l2(buf):
 
 
 # ------------------------------------------------------------------ our arm
-def run_generation(spec, steps, warmup, dist_ctx=None, timing=False, serial=False):
+# The headline evaluates EVERY (frontier node, candidate) pair: all f_{k-1} r_k candidate
+# evaluations of the spec as written ("iterating over the constrained
+# ranges").  The segment-bound variant (whole candidate segments of a divisibility filter
+# rejected by their |x| bounds, same space) is reported as a secondary line.
+def headline_flags():
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    return L.ATF_FLAG_NO_SEG_BOUNDS
+
+
+def run_generation(spec, steps, warmup, dist_ctx=None, timing=False, serial=False, flags=None):
     """Times `steps` generations of `spec`; returns per-step ms (max over ranks), stats.
     The production configuration runs the groups' levels concurrently (one stream per group)
     without per-level events; `timing` + `serial` is the roofline pass: the same kernels,
@@ -117,7 +126,8 @@ def run_generation(spec, steps, warmup, dist_ctx=None, timing=False, serial=Fals
     dev = torch.cuda.current_device()
     stream = torch.cuda.current_stream()
     flush = torch.empty(128 << 20, dtype=torch.int32, device="cuda")
-    flags = (L.ATF_FLAG_TIMING if timing else 0) | (L.ATF_FLAG_SERIAL_GROUPS if serial else 0)
+    flags = (headline_flags() if flags is None else flags) | (L.ATF_FLAG_TIMING if timing else 0) | \
+        (L.ATF_FLAG_SERIAL_GROUPS if serial else 0)
     sp = Space(spec, device=dev, stream=stream, flags=flags)
     world = dist_ctx["world"] if dist_ctx else 1
     rank = dist_ctx["rank"] if dist_ctx else 0
@@ -153,8 +163,9 @@ def run_generation(spec, steps, warmup, dist_ctx=None, timing=False, serial=Fals
     torch.cuda.synchronize()
     ms = [a.elapsed_time(b) for a, b in evs]
     st = sp.stats()
+    launches = sum(x["launches"] for x in st)
     res = {"ms": ms, "stats": st, "size": sp.size(), "group_sizes": sp.group_sizes(),
-           "plan": sp.plan_json(), "level_ms": level_ms, "level_exp_ms": level_exp_ms}
+           "plan": sp.plan_json(), "level_ms": level_ms, "level_exp_ms": level_exp_ms, "launches": launches}
     sp.close()
     return res
 
@@ -183,7 +194,7 @@ def roofline_of(res, sm_mhz, spec_name=None, step_ms=None):
     st = res["stats"]
     # evaluated pairs: the spec's f_{k-1} x r_k, less the pairs the warp-tile hot loop rejects
     # wholesale by its per-segment |x| bounds (stats "pairs", ATF_FLAG_TIMING)
-    ops = [(s["pairs"] or s["evals"]) * c for s, c in zip(st, costs)]
+    ops = [s["pairs"] * c for s, c in zip(st, costs)]   # timing pass: pairs = evaluated pairs
     exp_ms = np.array(res["level_exp_ms"], dtype=np.float64).mean(axis=0)
     lvl_ms = np.array(res["level_ms"], dtype=np.float64).mean(axis=0)
     d = int(np.argmax(exp_ms))
@@ -195,19 +206,22 @@ def roofline_of(res, sm_mhz, spec_name=None, step_ms=None):
     alg_bytes = f_prev * W * 4 + st[d]["f"] * W * 4 + (f_prev + 1) * 8
     tdb = _traffic_db()
     tr = tdb.get(f"{spec_name}:g{g}:l{k}") if spec_name else None
-    kname = {0: "expand_narrow", 1: "expand_wide", 2: "expand_wtile"}.get(st[d].get("kernel", -1), "expand")
+    kname = {0: "expand_narrow", 1: "expand_wide", 2: "expand_wtile", 3: "expand_nfast", 4: "atf_nfast_jit",
+             5: "tail_count+tail_emit"}.get(st[d].get("kernel", -1), "expand")
     step_ops = float(sum(ops))
     step_ms = float(step_ms) if step_ms else float(lvl_ms.sum())
     return {"bound": "alu", "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tops/s",
             "frac": achieved / peak, "traffic": tr["dram_bytes"] if tr else None,
             "traffic_source": tr["source"] if tr else None,
             "kernel": kname, "launch": f"group {g} level {k + 1} (r={st[d]['r']}, evals={st[d]['evals']}, "
-                                       f"evaluated pairs={st[d]['pairs'] or st[d]['evals']})",
+                                       f"evaluated pairs={st[d]['pairs']})",
             "ops_per_launch": ops[d], "launch_ms": float(exp_ms[d]), "algorithmic_bytes_per_launch": int(alg_bytes),
             "peak_clock_mhz": sm_mhz, "peak_source": "4 SMSP x 32 lanes x 148 SMs x clock (B200_PROFILING.md unit counts)",
             "cost_table": "DIVX/MULX/DIVPROD 2, QDIV 6, CMP 2, AND 1, GENERIC = bytecode ops",
             "step": {"ops": step_ops, "ms": step_ms, "achieved": step_ops / (step_ms * 1e-3) / 1e12,
-                     "frac": step_ops / (step_ms * 1e-3) / peak}}
+                     "frac": step_ops / (step_ms * 1e-3) / peak,
+                     "pairs_evaluated": int(sum(s["pairs"] for s in st)),
+                     "pairs_decided": int(sum(s["evals"] for s in st))}}
 
 
 def e2e_generation(spec, steps, dist_ctx=None):
@@ -230,7 +244,7 @@ def e2e_generation(spec, steps, dist_ctx=None):
         if dist_ctx:
             dist_ctx["dist"].barrier()
         t0 = time.perf_counter()
-        with Space(spec) as sp:
+        with Space(spec, flags=headline_flags()) as sp:
             if dist_ctx:
                 from paper_conf_hpdc_raschg18_b200.shard import generate_sharded
                 generate_sharded(sp)
@@ -255,6 +269,27 @@ def secondary_n1(steps, warmup, sm_mhz):
     import torch
     from paper_conf_hpdc_raschg18_b200 import Space
     out = {}
+    # C5 with the per-segment |x| bounds (same space; pairs decided without evaluation)
+    spec = A.c5_chains(4096, 8)
+    res = run_generation(spec, steps, warmup, flags=0)
+    ms = float(np.mean(res["ms"]))
+    leaves = sum(res["group_sizes"])
+    res_t = run_generation(spec, steps, 2, timing=True, serial=True, flags=0)
+    rf = roofline_of(res_t, sm_mhz, spec.name + ":segbounds", step_ms=ms)
+    out["C5-segment-bounds"] = {
+        "ms_per_step": ms, "configs_per_s": leaves / (ms * 1e-3),
+        "pairs_decided_per_s": rf["step"]["pairs_decided"] / (ms * 1e-3),
+        "pairs_evaluated_per_s": rf["step"]["pairs_evaluated"] / (ms * 1e-3),
+        "pairs_evaluated": rf["step"]["pairs_evaluated"], "pairs_decided": rf["step"]["pairs_decided"],
+        "roofline_frac_step_on_evaluated_pairs": rf["step"]["frac"], "dominant_launch": rf["launch"],
+        "dominant_frac_on_evaluated_pairs": rf["frac"],
+        "note": "flags 0: warp-tile hot loop rejects candidate segments by their |x| bounds (DESIGN.md §5)"}
+    for name, mk in (("C1", A.c1_toy), ("C3-IS1", lambda: A.c3_xgemm("IS1")), ("C3-IS3", lambda: A.c3_xgemm("IS3"))):
+        res = run_generation(mk(), steps, warmup)
+        ms = float(np.mean(res["ms"]))
+        out[name] = {"ms_per_step": ms, "S": str(res["size"]), "group_leaves": sum(res["group_sizes"]),
+                     "configs_per_s": sum(res["group_sizes"]) / (ms * 1e-3),
+                     "note": "launch-latency bound (SURVEY.md §8(d)); device time of one generation"}
     for name, mk in (("C3-IS2", lambda: A.c3_xgemm("IS2")), ("C3-IS4", lambda: A.c3_xgemm("IS4")),
                      ("C2", lambda: A.c2_xgemm_direct(256))):
         res = run_generation(mk(), steps, warmup)
@@ -399,7 +434,7 @@ def main():
     value = leaves / (ms * 1e-3)
     # our kernels per step: every non-empty level launches expand_narrow (r <= 64) or
     # expand_wide, then scan_kernel and level_emit_kernel
-    n_launch = 3 * sum(1 for s in res["stats"] if s["evals"] > 0)
+    n_launch = res["launches"]  # library-counted kernel launches of one generation
     e2e = e2e_generation(spec, max(2, a.steps // 2), dist_ctx)
     if rank == 0:
         line = {"metric": METRIC, "value": value, "unit": "configs/s", "n_gpus": world, "steps": a.steps,
@@ -413,10 +448,14 @@ def main():
                         "s_per_step": e2e["s_per_step"]}}
         if world == 1:
             evals_total = sum(s["evals"] for s in res["stats"])
-            line["evals_per_s"] = evals_total / (ms * 1e-3)
+            # every pair evaluated (headline flags): evaluated = decided = f_{k-1} r_k
+            line["pairs_decided_per_s"] = evals_total / (ms * 1e-3)
+            line["flags"] = "ATF_FLAG_NO_SEG_BOUNDS (every f_{k-1} r_k pair evaluated)"
             # roofline: a serialized timing pass of the same generation (per-launch events)
             res_t = run_generation(spec, max(3, a.steps // 2), 2, timing=True, serial=True)
             line["roofline"] = roofline_of(res_t, sm_max, spec.name, step_ms=ms)
+            # evaluated pairs counted on the device (ATF_FLAG_TIMING statistics of the timing pass)
+            line["pairs_evaluated_per_s"] = line["roofline"]["step"]["pairs_evaluated"] / (ms * 1e-3)
             line["roofline"]["timing_pass"] = ("serialized groups, CUDA events per level / expand kernel, "
                                                f"{max(3, a.steps // 2)} steps after the timed region")
             line["roofline_at_load_clock"] = (roofline_of(res_t, clocks["sm_mhz"], spec.name, step_ms=ms)["frac"]

@@ -109,6 +109,17 @@ typedef struct {
                                      isolates per-launch times for roofline measurements    */
 #define ATF_FLAG_KEEP_LEVELS 4u   /* keep inner-level arrays (CSR + records); default
                                      keeps them too — reserved                          */
+#define ATF_FLAG_NO_SEG_BOUNDS 64u /* evaluate EVERY (frontier node, candidate) pair, i.e. all
+                                     f_{k-1} * r_k candidate evaluations of the spec as written
+                                     ("must not skip candidates"; P:280
+                                     "iterating over the constrained ranges").  Without it the
+                                     warp-tile kernel rejects whole candidate segments of a
+                                     divisibility filter by their |x| bounds (x | n needs
+                                     |x| <= |n|) without evaluating their pairs; the result is
+                                     identical, the evaluated-pair count is not */
+#define ATF_FLAG_NO_TAIL 128u     /* expand a group's trailing narrow levels one at a time instead
+                                     of the fused narrow tail (two launches for up to 4 levels,
+                                     DESIGN.md §5); kept for parity coverage and A/B timing    */
 
 /* Bytecode: postfix int32 words, int64 stack.
  *   1 X            push the candidate value
@@ -278,6 +289,10 @@ typedef struct {
                        warp-tile levels with a hot filter: the pairs the hot loop tested (the rest
                        are rejected by the per-segment |x| bounds: x | n needs |x| <= |n|, d | x
                        needs |x| >= |d|).  0 without ATF_FLAG_TIMING */
+  int32_t cpt;      /* warp-tile levels: candidates per lane per segment (else 0)          */
+  int32_t nseg;     /* warp-tile levels: candidate segments of 32 * cpt per node (else 0)  */
+  int32_t launches; /* kernels the library launched for this level in the last generation
+                       (expand + scan + emit, a re-run after an arena overflow included)    */
 } atf_level_stats;
 atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap, int32_t* n_out);
 

@@ -25,6 +25,8 @@ STATUS = {0: "ATF_OK", -1: "ATF_ERR_INVALID_ARG", -2: "ATF_ERR_OOM", -3: "ATF_ER
           -9: "ATF_ERR_DUPLICATE", -10: "ATF_ERR_LIMIT"}
 ATF_RANGE_INTERVAL, ATF_RANGE_POW2, ATF_RANGE_SET, ATF_RANGE_GEN = 0, 1, 2, 3
 ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT, ATF_FLAG_SERIAL_GROUPS = 1, 2, 8, 16, 32
+ATF_FLAG_NO_SEG_BOUNDS = 64
+ATF_FLAG_NO_TAIL = 128
 
 
 class atf_range(C.Structure):
@@ -51,7 +53,7 @@ class atf_level_stats(C.Structure):
     _fields_ = [("group", C.c_int32), ("level", C.c_int32), ("param", C.c_int32), ("r", C.c_int64),
                 ("evals", C.c_uint64), ("f", C.c_uint64), ("ms", C.c_float), ("path", C.c_int32),
                 ("expand_ms", C.c_float), ("kernel", C.c_int32),
-                ("pairs", C.c_uint64)]
+                ("pairs", C.c_uint64), ("cpt", C.c_int32), ("nseg", C.c_int32), ("launches", C.c_int32)]
 
 
 SP = C.c_void_p  # atf_space*

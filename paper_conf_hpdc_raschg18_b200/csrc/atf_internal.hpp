@@ -125,6 +125,29 @@ struct LevelArgs {
   int32_t smem_bytes;
 };
 enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1, K_WTILE = 2, K_NFAST = 3 };
+
+// Fused narrow tail (DESIGN.md §5 "Narrow tail"): the last nl (2..kMaxTail) levels of a group,
+// every one a narrow fast level (nf_ok, 1 <= r <= 32), expanded from the frontier of level
+// t0 - 1 in two launches: tail_count (per warp tile of 32 frontier nodes: the tile's node
+// count at every tail level) and, after an exclusive scan of those tile counts per level,
+// tail_emit (the same masks again; every level's records and CSR written at their final
+// positions through per-warp shared-memory buffers).  No intermediate level is re-read.
+constexpr int kMaxTail = 4;
+constexpr int kTailWarps = 4;  // warps per CTA of tail_emit
+struct TailArgs {
+  int32_t nl;
+  const uint32_t* parent_rec;  // frontier (level t0 - 1); nullptr at t0 == 0 (root)
+  uint64_t n_parents;
+  uint64_t n_tiles;            // ceil(n_parents / 32)
+  uint32_t* tile_total;        // [nl][n_tiles] (tail_count)
+  const uint64_t* tile_base;   // [nl][n_tiles + 1] exclusive scans of tile_total per level
+  uint64_t* csr[kMaxTail];     // csr[0]: CSR of the frontier level [n_parents + 1];
+                               // csr[d] (d >= 1): CSR of tail level d - 1
+  uint32_t* rec[kMaxTail];     // records of tail level d (tail_emit)
+  int32_t buf_off[kMaxTail];   // tail_emit: per-warp shared-memory buffer of level d (bytes)
+  int32_t warp_bytes;          // tail_emit: shared memory per warp
+  LevelArgs lv[kMaxTail];      // the levels' programs (narrow fast atoms) and candidates
+};
 constexpr int kNfNPL = 4;  // narrow fast kernel: frontier nodes per lane (warp tile = 128 nodes)
 constexpr int kWT = 32;        // warp-tile kernel: frontier nodes per warp tile (one per lane)
 constexpr int kItemCap = 512;  // warp-tile kernel: items whose exact masks pass 1 keeps for the emit pass
@@ -266,6 +289,8 @@ int launch_expand(const LevelArgs& a, int words, void* stream);
 int expand_smem_bytes(const LevelArgs& a, int words);
 int launch_level_emit(const LevelArgs& a, int words, void* stream);
 int launch_nfast_emit(const LevelArgs& a, int words, void* stream);
+int launch_tail_count(const TailArgs& t, int words, void* stream);
+int launch_tail_emit(const TailArgs& t, int words, void* stream);
 }  // namespace atf
 #include <vector>
 namespace atf {

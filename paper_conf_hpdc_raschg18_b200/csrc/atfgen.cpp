@@ -94,6 +94,8 @@ struct LevelData {
   uint64_t pairs = 0;      // (node, candidate) pairs evaluated (ATF_FLAG_TIMING; = evals unless
                            // the warp-tile hot loop skipped segments by their |x| bounds)
   bool seg_skip = false;   // the level's hot loop applies the segment bounds
+  int32_t cpt = 0, nseg = 0;  // warp-tile geometry of the level's last launch
+  int32_t launches = 0;    // kernels launched for the level (re-runs included)
 };
 
 }  // namespace
@@ -142,6 +144,14 @@ struct atf_space {
   size_t table_bytes = 0;
   struct EvTriple { cudaEvent_t first = nullptr, mid = nullptr, second = nullptr; };
   std::vector<std::vector<EvTriple>> events;
+  // fused narrow tails (one per group at most): count round -> emit round
+  struct Tail {
+    int k0 = -1, nl = 0;         // tail levels [k0, k0 + nl) of the group (k0 = -1: none)
+    int phase = 0;               // 0 idle, 1 counted (totals known), 2 emitted
+    TailArgs t;                  // kernel arguments (count and emit)
+    uint64_t tot[kMaxTail] = {};  // node count of every tail level
+  };
+  std::vector<Tail> tails;
   // shards
   int shard_rank = 0, shard_world = 1;
   std::vector<int> shard_cut;  // per group: first level expanded on a slice (L = none)
@@ -773,7 +783,7 @@ static atf_status plan(atf_space* s) {
 // r <= 64 -> narrow kernel (thread per node); otherwise the wide
 // kernel with cpt candidates per thread, a hot filter when a conjunct allows one, and
 // ~2^18 (node, candidate) pairs per tile.
-static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
+static void choose_geometry(LevelArgs& a, int words, bool legacy_wide, bool seg_bounds = true) {
   const int r = a.r;
   a.hot = HOT_NONE;
   a.hot_term = 0;
@@ -801,13 +811,10 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide) {
       // Divisor filters over ranges that already span several segments: finer segments (the
       // smallest cpt >= 8 that fits kMaxSeg) let small node values skip more candidates
       // (C5 9.44 -> 9.33 ms measured; multiples filters and single-segment levels lose, so
-      // they keep the cost-model choice).  ATF_SEG_FINE / ATF_SEG_FINE_KIND override (A/B).
-      static const int fine_env = [] { const char* e = getenv("ATF_SEG_FINE"); return e ? atoi(e) : -1; }();
-      static const int fine_kind = [] { const char* e = getenv("ATF_SEG_FINE_KIND"); return e ? atoi(e) : 0; }();
-      int fine = 0;
-      if (fine_env >= 0) fine = (fine_kind == 0 || fine_kind == a.hot) ? fine_env : 0;
-      else if (a.hot == HOT_DIVX && best_nseg >= 2) fine = 8;
-      if (fine && a.hot != HOT_NONE) {
+      // they keep the cost-model choice).  Without segment bounds (ATF_FLAG_NO_SEG_BOUNDS)
+      // finer segments only add loop overhead.
+      const int fine = (seg_bounds && a.hot == HOT_DIVX && best_nseg >= 2) ? 8 : 0;
+      if (fine) {
         // finer segments: more node quads fall outside a segment's |x| bounds
         for (int cpt : {4, 8, 12, 16, 20, 24, 32}) {
           if (cpt < fine) continue;
@@ -1079,7 +1086,23 @@ struct Pending {
   int chunk;  // arena chunk holding the child region
   size_t child_off;
   bool joined = false;  // ran on the group's own stream (join event recorded)
+  int kind = 0;         // 0 one level, 1 tail count, 2 tail emit
 };
+
+// device tables of a level: candidate values / magics / |values| and every referenced
+// ancestor's value and magic table (see ensure_device: [values rp][magic rp][abs rp])
+static void fill_level_ptrs(atf_space* s, const LevelPlan& lp, LevelArgs& a) {
+  a.cand = s->d_range[lp.param];
+  const size_t rp = ((size_t)lp.r + 127) / 128 * 128;
+  a.cand_magic = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + rp;
+  a.cand_abs = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + 2 * rp;
+  a.r = lp.r;
+  for (int i = 0; i < a.n_pv; i++) {
+    a.pv_range[i] = s->d_range[lp.pv_param[i]];
+    const size_t rpi = (s->params[lp.pv_param[i]].values.size() + 127) / 128 * 128;
+    a.pv_magic[i] = reinterpret_cast<const uint32_t*>(s->d_range[lp.pv_param[i]]) + rpi;
+  }
+}
 
 static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parents, uint64_t n_parents, Pending& pd,
                               bool own_stream) {
@@ -1090,21 +1113,13 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   LevelArgs a = lp.proto;
   a.parent_rec = parents;
   a.n_parents = n_parents;
-  a.cand = s->d_range[lp.param];
-  {  // see ensure_device: [values rp][magic rp][abs rp]
-    const size_t rp = ((size_t)lp.r + 127) / 128 * 128;
-    a.cand_magic = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + rp;
-    a.cand_abs = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + 2 * rp;
-  }
-  a.r = lp.r;
-  for (int i = 0; i < a.n_pv; i++) {
-    a.pv_range[i] = s->d_range[lp.pv_param[i]];
-    // see ensure_device: [values rp][magic rp][abs rp]
-    const size_t rpi = (s->params[lp.pv_param[i]].values.size() + 127) / 128 * 128;
-    a.pv_magic[i] = reinterpret_cast<const uint32_t*>(s->d_range[lp.pv_param[i]]) + rpi;
-  }
-  choose_geometry(a, gp.words, (s->opts.flags & ATF_FLAG_LEGACY_WIDE) != 0);
-  if (a.kind == K_WTILE && a.hot != HOT_NONE) {
+  fill_level_ptrs(s, lp, a);
+  const bool seg_bounds = (s->opts.flags & ATF_FLAG_NO_SEG_BOUNDS) == 0;
+  choose_geometry(a, gp.words, (s->opts.flags & ATF_FLAG_LEGACY_WIDE) != 0, seg_bounds);
+  if (a.kind == K_WTILE && a.hot != HOT_NONE && !seg_bounds) {
+    // every pair is evaluated: bounds that no node quad can fall outside of
+    for (int sg = 0; sg < kMaxSeg; sg++) { a.seg_lo[sg] = 0u; a.seg_hi[sg] = 0xffffffffu; }
+  } else if (a.kind == K_WTILE && a.hot != HOT_NONE) {
     if (lp.seg_cpt != a.cpt) {  // per-segment |x| bounds of the hot filter (cached per level)
       const std::vector<int32_t>& v = s->params[lp.param].values;
       const int seg = 32 * a.cpt;
@@ -1124,7 +1139,7 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     for (int sg = 0; sg < kMaxSeg; sg++) { a.seg_lo[sg] = lp.seg_lo[sg]; a.seg_hi[sg] = lp.seg_hi[sg]; }
   }
   a.pairs_out = (s->opts.flags & ATF_FLAG_TIMING) ? s->d_pairs + g : nullptr;
-  s->data[g][k].seg_skip = a.kind == K_WTILE && a.hot != HOT_NONE;
+  s->data[g][k].seg_skip = a.kind == K_WTILE && a.hot != HOT_NONE && seg_bounds;
   a.n_tiles = a.n_chunks > 1 ? n_parents * (uint64_t)a.n_chunks
                              : (n_parents + (uint64_t)a.tile_nodes - 1) / (uint64_t)a.tile_nodes;
   if (a.smem_bytes > 227 * 1024)
@@ -1252,6 +1267,10 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   }
   const bool use_jit = a.kind == K_NFAST && lp.jit && !(s->opts.flags & (ATF_FLAG_NO_JIT | ATF_FLAG_LEGACY_WIDE));
   int ce = use_jit ? jit_nfast_launch(lp.jit, a, ls) : launch_expand(a, gp.words, ls);
+  LevelData& ld = s->data[g][k];
+  ld.cpt = a.kind == K_WTILE ? a.cpt : 0;
+  ld.nseg = a.kind == K_WTILE ? a.nseg : 0;
+  ld.launches += a.direct ? 1 : 3;
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   if (use_jit) s->data[g][k].kernel = 4;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].mid, ls));
@@ -1272,6 +1291,177 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   pd.joined = !serial;
   pd = Pending{g, k, n_parents, parents, (uint64_t*)csr, child, cap, which, off, pd.joined};
   return ATF_OK;
+}
+
+// ---------------------------------------------------------------- fused narrow tail
+// First level of group g's fused narrow tail: the longest run of trailing
+// levels (2..kMaxTail) that are all narrow fast levels with 1 <= r <= 32 and whose per-warp
+// emit buffers (32 * r * words * 4 bytes per level) fit 16 KB; -1 if none.
+static int tail_start(const atf_space* s, int g) {
+  if (s->opts.flags & (ATF_FLAG_NO_TAIL | ATF_FLAG_LEGACY_WIDE | ATF_FLAG_GENERIC_ONLY)) return -1;
+  const GroupPlan& gp = s->groups[g];
+  const int L = (int)gp.levels.size();
+  int k0 = L, bytes = 0;
+  while (k0 > 0 && L - k0 < kMaxTail) {
+    const LevelPlan& lp = gp.levels[k0 - 1];
+    if (!lp.proto.nf_ok || lp.generic || lp.r < 1 || lp.r > 32) break;
+    const int b = 32 * lp.r * gp.words * 4;
+    if (bytes + b > 16 * 1024) break;
+    bytes += b;
+    k0--;
+  }
+  return L - k0 >= 2 ? k0 : -1;
+}
+
+// Count round of the tail of group g from frontier `parents` (level k0 - 1, n_parents nodes):
+// tail_count, then one exclusive scan of the warp-tile counts per tail level.
+static atf_status queue_tail_count(atf_space* s, int g, int k0, const uint32_t* parents, uint64_t n_parents,
+                                   Pending& pd, bool own_stream) {
+  GroupPlan& gp = s->groups[g];
+  auto& T = s->tails[g];
+  auto& gbf = s->gb[g];
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  const int nl = (int)gp.levels.size() - k0;
+  T.k0 = k0;
+  T.nl = nl;
+  T.phase = 0;
+  TailArgs& t = T.t;
+  std::memset(&t, 0, sizeof t);
+  t.nl = nl;
+  t.parent_rec = parents;
+  t.n_parents = n_parents;
+  t.n_tiles = (n_parents + 31) / 32;
+  for (int d = 0; d < nl; d++) {
+    t.lv[d] = gp.levels[k0 + d].proto;
+    fill_level_ptrs(s, gp.levels[k0 + d], t.lv[d]);
+  }
+  // scratch: tile_total u32[nl][n] | tile_base u64[nl][n+1] | scan status u64[nl][ns] | counters u32[nl]
+  const size_t n = t.n_tiles, ns = (n + 1023) / 1024 + 1;
+  const size_t o_tot = 0, o_base = (o_tot + 4 * nl * n + 15) & ~(size_t)15, o_stat = o_base + 8 * nl * (n + 1);
+  const size_t o_cnt = o_stat + 8 * nl * ns, bytes = o_cnt + 4 * nl + 16;
+  atf_status e = ensure_buf(s, &gbf.scratch, &gbf.scratch_cap, bytes, "tail scratch");
+  if (e) return e;
+  t.tile_total = (uint32_t*)(gbf.scratch + o_tot);
+  t.tile_base = (const uint64_t*)(gbf.scratch + o_base);
+  CUDA_TRY(s, cudaMemsetAsync(gbf.scratch + o_stat, 0, bytes - o_stat, st));
+  const bool serial = !own_stream || (s->opts.flags & ATF_FLAG_SERIAL_GROUPS) != 0;
+  cudaStream_t ls = serial ? st : gbf.stream;
+  if (!serial) {
+    CUDA_TRY(s, cudaEventRecord(gbf.fork, st));
+    CUDA_TRY(s, cudaStreamWaitEvent(gbf.stream, gbf.fork, 0));
+  }
+  const bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0].first, ls));
+  int ce = launch_tail_count(t, gp.words, ls);
+  if (ce) return fail(s, ATF_ERR_CUDA, "tail count launch (group %d): %s", g, cudaGetErrorString((cudaError_t)ce));
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0].mid, ls));
+  for (int d = 0; d < nl && !ce; d++)
+    ce = launch_scan_u32(t.tile_total + d * n, (uint64_t*)t.tile_base + d * (n + 1), (int64_t)n,
+                         (unsigned long long*)(gbf.scratch + o_stat) + d * ns, (unsigned int*)(gbf.scratch + o_cnt) + d,
+                         ls);
+  if (ce) return fail(s, ATF_ERR_CUDA, "tail scan (group %d): %s", g, cudaGetErrorString((cudaError_t)ce));
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0].second, ls));
+  if (!serial) CUDA_TRY(s, cudaEventRecord(gbf.join, ls));
+  s->data[g][k0].launches += 1 + nl;
+  pd = Pending{};
+  pd.g = g;
+  pd.k = k0;
+  pd.n_parents = n_parents;
+  pd.parents = parents;
+  pd.joined = !serial;
+  pd.kind = 1;
+  return ATF_OK;
+}
+
+static char* arena_take(atf_space* s, int g, size_t bytes, atf_status* e) {
+  char* p = arena_alloc(s, g, bytes);
+  if (!p) {
+    if ((*e = arena_grow(s, g, bytes))) return nullptr;
+    p = arena_alloc(s, g, bytes);
+  }
+  return p;
+}
+
+// Emit round of group g's tail (level sizes known from the count round): exact allocations,
+// then tail_emit writes every tail level's records and the CSR of the levels above them.
+static atf_status queue_tail_emit(atf_space* s, int g, Pending& pd, bool own_stream) {
+  GroupPlan& gp = s->groups[g];
+  auto& T = s->tails[g];
+  auto& gbf = s->gb[g];
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  TailArgs& t = T.t;
+  const int nl = T.nl, k0 = T.k0;
+  atf_status e = ATF_OK;
+  // CSR of the frontier level (its size + 1), then per tail level its records and (but the
+  // last) its CSR
+  t.csr[0] = (uint64_t*)arena_take(s, g, (t.n_parents + 1) * 8, &e);
+  if (!t.csr[0]) return e ? e : fail(s, ATF_ERR_OOM, "tail CSR");
+  for (int d = 0; d < nl; d++) {
+    t.rec[d] = (uint32_t*)arena_take(s, g, std::max<uint64_t>(T.tot[d], 1) * gp.words * 4, &e);
+    if (!t.rec[d]) return e ? e : fail(s, ATF_ERR_OOM, "tail records");
+    if (d + 1 < nl) {
+      t.csr[d + 1] = (uint64_t*)arena_take(s, g, (T.tot[d] + 1) * 8, &e);
+      if (!t.csr[d + 1]) return e ? e : fail(s, ATF_ERR_OOM, "tail CSR");
+    }
+  }
+  int off = 0;
+  for (int d = 0; d < nl; d++) {
+    t.buf_off[d] = off;
+    off += (32 * t.lv[d].r * gp.words * 4 + 15) & ~15;
+  }
+  t.warp_bytes = off;
+  const bool serial = !own_stream || (s->opts.flags & ATF_FLAG_SERIAL_GROUPS) != 0;
+  cudaStream_t ls = serial ? st : gbf.stream;
+  if (!serial) {
+    CUDA_TRY(s, cudaEventRecord(gbf.fork, st));
+    CUDA_TRY(s, cudaStreamWaitEvent(gbf.stream, gbf.fork, 0));
+  }
+  const bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0 + 1].first, ls));
+  int ce = launch_tail_emit(t, gp.words, ls);
+  if (ce) return fail(s, ATF_ERR_CUDA, "tail emit launch (group %d): %s", g, cudaGetErrorString((cudaError_t)ce));
+  if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0 + 1].second, ls));
+  if (!serial) CUDA_TRY(s, cudaEventRecord(gbf.join, ls));
+  s->data[g][k0].launches += 1;
+  pd = Pending{};
+  pd.g = g;
+  pd.k = k0;
+  pd.n_parents = t.n_parents;
+  pd.parents = t.parent_rec;
+  pd.joined = !serial;
+  pd.kind = 2;
+  return ATF_OK;
+}
+
+// After the emit round: the tail levels become the group's level data.
+static void finish_tail(atf_space* s, int g) {
+  auto& T = s->tails[g];
+  const TailArgs& t = T.t;
+  GroupPlan& gp = s->groups[g];
+  const bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
+  float ms_count = 0.f, ms_count_k = 0.f, ms_emit = 0.f;
+  if (timing) {
+    cudaEventElapsedTime(&ms_count, s->events[g][T.k0].first, s->events[g][T.k0].second);
+    cudaEventElapsedTime(&ms_count_k, s->events[g][T.k0].first, s->events[g][T.k0].mid);
+    cudaEventElapsedTime(&ms_emit, s->events[g][T.k0 + 1].first, s->events[g][T.k0 + 1].second);
+  }
+  if (T.k0 > 0) s->data[g][T.k0 - 1].csr = t.csr[0];
+  for (int d = 0; d < T.nl; d++) {
+    LevelData& ld = s->data[g][T.k0 + d];
+    const uint64_t above = d == 0 ? t.n_parents : T.tot[d - 1];
+    ld.rec = T.tot[d] ? t.rec[d] : nullptr;
+    ld.n = T.tot[d];
+    ld.evals = above * (uint64_t)gp.levels[T.k0 + d].r;
+    ld.kernel = 5;
+    ld.cpt = ld.nseg = 0;
+    if (d + 1 < T.nl) ld.csr = t.csr[d + 1];
+    if (timing) {  // the whole tail is attributed to its first level
+      ld.ms = d == 0 ? ms_count + ms_emit : 0.f;
+      ld.expand_ms = d == 0 ? ms_count_k + ms_emit : 0.f;
+      ld.pairs = ld.evals;
+    }
+  }
+  T.phase = 2;
 }
 
 // Generate groups' levels [k_from, L) starting from the given frontiers; syncs once per round.
@@ -1315,7 +1505,14 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
         continue;
       }
       Pending pd;
-      atf_status e = queue_level(s, g, k[i], frontier[i], fsize[i], pd, active > 1);
+      atf_status e;
+      if (s->tails[g].phase == 1) {
+        e = queue_tail_emit(s, g, pd, active > 1);
+      } else if (k[i] == tail_start(s, g)) {
+        e = queue_tail_count(s, g, k[i], frontier[i], fsize[i], pd, active > 1);
+      } else {
+        e = queue_level(s, g, k[i], frontier[i], fsize[i], pd, active > 1);
+      }
       if (e) return e;
       pend.push_back(pd);
     }
@@ -1324,12 +1521,28 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       if (pd.joined) CUDA_TRY(s, cudaStreamWaitEvent(st, s->gb[pd.g].join, 0));  // join the group streams
     // one copy brings back [totals | overflow flags] of every group
     CUDA_TRY(s, cudaMemcpyAsync(s->h_ctl.data(), s->d_totals, 12 * kMaxGroups, cudaMemcpyDeviceToHost, st));
+    for (auto& pd : pend)
+      if (pd.kind == 1) {  // tail level sizes = the scans' totals
+        auto& T = s->tails[pd.g];
+        for (int d = 0; d < T.nl; d++)
+          CUDA_TRY(s, cudaMemcpyAsync(&T.tot[d], T.t.tile_base + d * (T.t.n_tiles + 1) + T.t.n_tiles, 8,
+                                      cudaMemcpyDeviceToHost, st));
+      }
     CUDA_TRY(s, cudaStreamSynchronize(st));
     unsigned long long h_pairs[kMaxGroups] = {};
     if (s->opts.flags & ATF_FLAG_TIMING)
       CUDA_TRY(s, cudaMemcpy(h_pairs, s->d_pairs, sizeof(h_pairs), cudaMemcpyDeviceToHost));
     for (auto& pd : pend) {
       size_t i = std::find(gs.begin(), gs.end(), pd.g) - gs.begin();
+      if (pd.kind == 1) {
+        s->tails[pd.g].phase = 1;
+        continue;
+      }
+      if (pd.kind == 2) {
+        finish_tail(s, pd.g);
+        k[i] = (int)s->groups[pd.g].levels.size();
+        continue;
+      }
       uint64_t total = s->h_totals[pd.g];
       GroupPlan& gp = s->groups[pd.g];
       if (s->h_flags[pd.g] || total > pd.cap) {
@@ -1366,6 +1579,7 @@ static atf_status generate_impl(atf_space* s) {
   if ((e = ensure_device(s))) return e;
   size_t G = s->groups.size();
   s->data.assign(G, {});
+  s->tails.assign(G, {});
   for (size_t g = 0; g < G; g++) {
     s->data[g].assign(s->groups[g].levels.size(), LevelData{});
     for (auto& c : s->arena[g]) c.used = 0;
@@ -1971,6 +2185,9 @@ atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap
         o.expand_ms = d.expand_ms;
         o.kernel = d.kernel;
         o.pairs = d.pairs;
+        o.cpt = d.cpt;
+        o.nseg = d.nseg;
+        o.launches = d.launches;
       }
       n++;
     }
@@ -1995,6 +2212,7 @@ atf_status atf_space_generate_shard(atf_space* s, int32_t rank, int32_t world, i
   if (e) return e;
   size_t G = s->groups.size();
   s->data.assign(G, {});
+  s->tails.assign(G, {});
   for (size_t g = 0; g < G; g++) {
     s->data[g].assign(s->groups[g].levels.size(), LevelData{});
     for (auto& c : s->arena[g]) c.used = 0;

@@ -1444,4 +1444,220 @@ static int launch_w(const LevelArgs& a, void* stream) {
   }
 }
 
+// ---------------------------------------------------------------- fused narrow tail
+// The last nl levels of a group when every one is a narrow fast level (r <= 32): one
+// count launch + one emit launch for all of them (atf_internal.hpp TailArgs).  The
+// candidate tables of every tail level live in shared memory; a node's accept mask is
+// nf_node_mask (the same exact atoms as expand_nfast), its children are its record with
+// the level's field set.
+struct TailTables {
+  int32_t cx[kMaxTail][32];
+  uint32_t cm[kMaxTail][32], ca[kMaxTail][32];
+  uint32_t full[kMaxTail], nz[kMaxTail];
+};
+
+__device__ __forceinline__ void tail_stage_tables(const TailArgs& t, TailTables& S) {
+  for (int i = threadIdx.x; i < kMaxTail * 32; i += blockDim.x) {
+    const int d = i >> 5, c = i & 31;
+    const bool v = d < t.nl && c < t.lv[d].r;
+    S.cx[d][c] = v ? __ldg(t.lv[d].cand + c) : 0;
+    S.cm[d][c] = v ? __ldg(t.lv[d].cand_magic + c) : 0x10000u;
+    S.ca[d][c] = v ? __ldg(t.lv[d].cand_abs + c) : 0u;
+  }
+  __syncthreads();
+  if (threadIdx.x < kMaxTail) {
+    const int d = threadIdx.x;
+    const int r = d < t.nl ? t.lv[d].r : 0;
+    uint32_t nz = 0;
+    for (int c = 0; c < r; c++) nz |= (uint32_t)(S.cx[d][c] != 0) << c;
+    S.full[d] = r >= 32 ? 0xffffffffu : ((1u << r) - 1u);
+    S.nz[d] = nz;
+  }
+  __syncthreads();
+}
+
+template <int W>
+__device__ __forceinline__ void tail_child(const LevelArgs& a, const uint32_t* rec, int c, uint32_t* out) {
+#pragma unroll
+  for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? (uint32_t)c << a.field_shift : 0u);
+}
+
+// subtree counts of one frontier node, depth-first (tail_count)
+template <int W, int D, int NL>
+__device__ __forceinline__ void tail_count_node(const TailArgs& t, const TailTables& S, const uint32_t* rec,
+                                                uint32_t (&cnt)[NL]) {
+  const LevelArgs& a = t.lv[D];
+  uint32_t m = nf_node_mask<W, uint32_t>(a, rec, a.r, S.full[D], S.nz[D], S.cx[D], S.cm[D], S.ca[D]);
+  cnt[D] += (uint32_t)__popc(m);
+  if constexpr (D + 1 < NL) {
+    while (m) {
+      const int c = __ffs(m) - 1;
+      m &= m - 1;
+      uint32_t cr[W];
+      tail_child<W>(a, rec, c, cr);
+      tail_count_node<W, D + 1, NL>(t, S, cr, cnt);
+    }
+  }
+}
+
+// Pass 1: warp tile = 32 consecutive frontier nodes (lane = node); tile_total[d][tile] =
+// the tile's node count at tail level d.
+template <int W, int NL>
+__global__ void __launch_bounds__(256, 4) tail_count(const __grid_constant__ TailArgs t) {
+  __shared__ TailTables S;
+  tail_stage_tables(t, S);
+  const int lane = threadIdx.x & 31;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  for (uint64_t tile = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile < t.n_tiles; tile += nw) {
+    const uint64_t nd = tile * 32 + lane;
+    uint32_t cnt[NL];
+#pragma unroll
+    for (int d = 0; d < NL; d++) cnt[d] = 0;
+    if (nd < t.n_parents) {
+      uint32_t rec[W];
+      if (t.parent_rec) load_record<W>(t.parent_rec + nd * W, rec);
+      else
+#pragma unroll
+        for (int w = 0; w < W; w++) rec[w] = 0u;
+      tail_count_node<W, 0, NL>(t, S, rec, cnt);
+    }
+#pragma unroll
+    for (int d = 0; d < NL; d++) {
+      uint32_t v = cnt[d];
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(FULL, v, o);
+      if (lane == 0) t.tile_total[(uint64_t)d * t.n_tiles + tile] = v;
+    }
+  }
+}
+
+// Pass 2, one tail level for a chunk of <= 32 nodes of the level above (lane = node, global
+// index gidx): accept masks -> warp scan -> the chunk's CSR entries; children into the
+// level's warp buffer at their chunk rank, then copied to the level's output as coalesced
+// vectors at cursor[D]; then the children, in chunks of 32, are expanded one level deeper.
+// Chunks are processed in node order at every depth, so every level's output is written in
+// its canonical (parent-major, candidate-order) order.
+template <int W, int D, int NL>
+__device__ __forceinline__ void tail_emit_chunk(const TailArgs& t, const TailTables& S, const uint32_t* rec, bool valid,
+                                                uint64_t gidx, uint64_t (&cursor)[NL], unsigned char* wbuf, int lane) {
+  using V = typename std::conditional<W == 1, uint32_t, typename std::conditional<W == 2, uint2, uint4>::type>::type;
+  constexpr int VPR = W == 8 ? 2 : 1;
+  const LevelArgs& a = t.lv[D];
+  uint32_t m = valid ? nf_node_mask<W, uint32_t>(a, rec, a.r, S.full[D], S.nz[D], S.cx[D], S.cm[D], S.ca[D]) : 0u;
+  const uint32_t c = (uint32_t)__popc(m);
+  uint32_t incl = c;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t y = __shfl_up_sync(FULL, incl, o);
+    if (lane >= o) incl += y;
+  }
+  const uint32_t T = __shfl_sync(FULL, incl, 31);
+  uint32_t k = incl - c;
+  const uint64_t first = cursor[D];
+  if (valid) t.csr[D][gidx] = first + k;
+  uint32_t* buf = reinterpret_cast<uint32_t*>(wbuf + t.buf_off[D]);
+  while (m) {
+    const int cc = __ffs(m) - 1;
+    m &= m - 1;
+    uint32_t out[W];
+    tail_child<W>(a, rec, cc, out);
+#pragma unroll
+    for (int w = 0; w < W; w++) buf[k * W + w] = out[w];
+    k++;
+  }
+  __syncwarp();
+  {
+    const V* src = reinterpret_cast<const V*>(buf);
+    V* dst = reinterpret_cast<V*>(t.rec[D] + first * W);
+    for (uint32_t v = lane; v < T * VPR; v += 32) dst[v] = src[v];
+  }
+  cursor[D] = first + T;
+  if constexpr (D + 1 < NL) {
+    for (uint32_t s0 = 0; s0 < T; s0 += 32) {
+      const bool v = s0 + lane < T;
+      uint32_t cr[W];
+#pragma unroll
+      for (int w = 0; w < W; w++) cr[w] = v ? buf[(s0 + lane) * W + w] : 0u;
+      tail_emit_chunk<W, D + 1, NL>(t, S, cr, v, first + s0 + lane, cursor, wbuf, lane);
+    }
+  }
+  __syncwarp();  // buf[D] is refilled by the next chunk at this depth
+}
+
+template <int W, int NL>
+__global__ void __launch_bounds__(32 * kTailWarps, 8) tail_emit(const __grid_constant__ TailArgs t) {
+  extern __shared__ __align__(16) unsigned char tail_smem[];
+  __shared__ TailTables S;
+  tail_stage_tables(t, S);
+  const int lane = threadIdx.x & 31;
+  unsigned char* wbuf = tail_smem + (threadIdx.x >> 5) * t.warp_bytes;
+  const uint64_t nw = ((uint64_t)gridDim.x * blockDim.x) >> 5;
+  const uint64_t gw = ((uint64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (gw == 0 && lane < NL) {  // closing CSR entries: csr[d][size of the level above] = level total
+    const uint64_t above = lane == 0 ? t.n_parents : t.tile_base[(uint64_t)(lane - 1) * (t.n_tiles + 1) + t.n_tiles];
+    t.csr[lane][above] = t.tile_base[(uint64_t)lane * (t.n_tiles + 1) + t.n_tiles];
+  }
+  for (uint64_t tile = gw; tile < t.n_tiles; tile += nw) {
+    uint64_t cursor[NL];
+#pragma unroll
+    for (int d = 0; d < NL; d++) cursor[d] = t.tile_base[(uint64_t)d * (t.n_tiles + 1) + tile];
+    const uint64_t nd = tile * 32 + lane;
+    const bool v = nd < t.n_parents;
+    uint32_t rec[W];
+    if (v && t.parent_rec) load_record<W>(t.parent_rec + nd * W, rec);
+    else
+#pragma unroll
+      for (int w = 0; w < W; w++) rec[w] = 0u;
+    tail_emit_chunk<W, 0, NL>(t, S, rec, v, nd, cursor, wbuf, lane);
+  }
+}
+
+template <int W>
+static int launch_tail_count_w(const TailArgs& t, void* stream) {
+  const void* k = nullptr;
+  switch (t.nl) {
+    case 2: k = (const void*)tail_count<W, 2>; break;
+    case 3: k = (const void*)tail_count<W, 3>; break;
+    case 4: k = (const void*)tail_count<W, 4>; break;
+    default: return (int)cudaErrorInvalidValue;
+  }
+  const int per_sm = cached_occupancy(k, 256, 0);
+  if (per_sm < 0) return -per_sm;
+  uint64_t grid = (uint64_t)cached_sm_count() * (per_sm > 0 ? per_sm : 1);
+  const uint64_t need = (t.n_tiles + 7) / 8;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  switch (t.nl) {
+    case 2: tail_count<W, 2><<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>(t); break;
+    case 3: tail_count<W, 3><<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>(t); break;
+    default: tail_count<W, 4><<<(unsigned)grid, 256, 0, (cudaStream_t)stream>>>(t); break;
+  }
+  return (int)cudaGetLastError();
+}
+
+template <int W>
+static int launch_tail_emit_w(const TailArgs& t, void* stream) {
+  const void* k = nullptr;
+  switch (t.nl) {
+    case 2: k = (const void*)tail_emit<W, 2>; break;
+    case 3: k = (const void*)tail_emit<W, 3>; break;
+    case 4: k = (const void*)tail_emit<W, 4>; break;
+    default: return (int)cudaErrorInvalidValue;
+  }
+  const int smem = kTailWarps * t.warp_bytes;
+  const int per_sm = cached_occupancy(k, 32 * kTailWarps, smem);
+  if (per_sm < 0) return -per_sm;
+  if (per_sm < 1) return (int)cudaErrorInvalidConfiguration;
+  uint64_t grid = (uint64_t)cached_sm_count() * per_sm;
+  const uint64_t need = (t.n_tiles + kTailWarps - 1) / kTailWarps;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  switch (t.nl) {
+    case 2: tail_emit<W, 2><<<(unsigned)grid, 32 * kTailWarps, smem, (cudaStream_t)stream>>>(t); break;
+    case 3: tail_emit<W, 3><<<(unsigned)grid, 32 * kTailWarps, smem, (cudaStream_t)stream>>>(t); break;
+    default: tail_emit<W, 4><<<(unsigned)grid, 32 * kTailWarps, smem, (cudaStream_t)stream>>>(t); break;
+  }
+  return (int)cudaGetLastError();
+}
+
 }  // namespace atf

@@ -6,3 +6,7 @@ namespace atf {
 int launch_expand_w1(const LevelArgs& a, void* stream) { return launch_w<1>(a, stream); }
 int launch_nfast_emit_w1(const LevelArgs& a, void* stream) { return launch_nfast_emit_w<1>(a, stream); }
 }  // namespace atf
+namespace atf {
+int launch_tail_count_w1(const TailArgs& t, void* stream) { return launch_tail_count_w<1>(t, stream); }
+int launch_tail_emit_w1(const TailArgs& t, void* stream) { return launch_tail_emit_w<1>(t, stream); }
+}  // namespace atf

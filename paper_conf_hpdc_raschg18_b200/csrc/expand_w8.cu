@@ -6,3 +6,7 @@ namespace atf {
 int launch_expand_w8(const LevelArgs& a, void* stream) { return launch_w<8>(a, stream); }
 int launch_nfast_emit_w8(const LevelArgs& a, void* stream) { return launch_nfast_emit_w<8>(a, stream); }
 }  // namespace atf
+namespace atf {
+int launch_tail_count_w8(const TailArgs& t, void* stream) { return launch_tail_count_w<8>(t, stream); }
+int launch_tail_emit_w8(const TailArgs& t, void* stream) { return launch_tail_emit_w<8>(t, stream); }
+}  // namespace atf

@@ -26,6 +26,35 @@ int launch_nfast_emit(const LevelArgs& a, int words, void* stream) {
   }
 }
 
+int launch_tail_count_w1(const TailArgs& t, void* stream);
+int launch_tail_count_w2(const TailArgs& t, void* stream);
+int launch_tail_count_w4(const TailArgs& t, void* stream);
+int launch_tail_count_w8(const TailArgs& t, void* stream);
+int launch_tail_emit_w1(const TailArgs& t, void* stream);
+int launch_tail_emit_w2(const TailArgs& t, void* stream);
+int launch_tail_emit_w4(const TailArgs& t, void* stream);
+int launch_tail_emit_w8(const TailArgs& t, void* stream);
+
+int launch_tail_count(const TailArgs& t, int words, void* stream) {
+  switch (words) {
+    case 1: return launch_tail_count_w1(t, stream);
+    case 2: return launch_tail_count_w2(t, stream);
+    case 4: return launch_tail_count_w4(t, stream);
+    case 8: return launch_tail_count_w8(t, stream);
+    default: return (int)cudaErrorInvalidValue;
+  }
+}
+
+int launch_tail_emit(const TailArgs& t, int words, void* stream) {
+  switch (words) {
+    case 1: return launch_tail_emit_w1(t, stream);
+    case 2: return launch_tail_emit_w2(t, stream);
+    case 4: return launch_tail_emit_w4(t, stream);
+    case 8: return launch_tail_emit_w8(t, stream);
+    default: return (int)cudaErrorInvalidValue;
+  }
+}
+
 int launch_expand(const LevelArgs& a, int words, void* stream) {
   switch (words) {
     case 1: return launch_expand_w1(a, stream);

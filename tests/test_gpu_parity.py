@@ -52,10 +52,16 @@ def torch_rowhash(rows_pm: "torch.Tensor", base: int = 0) -> int:
     return int(s.item()) & ((1 << 64) - 1)
 
 
-def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, legacy=False, no_jit=False):
+def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, legacy=False, no_jit=False,
+                          extra_flags=0, leaves_max=4_000_000):
+    """Sizes, groups, f_k and evals vs the oracle; then CONTENT: every configuration (decode of
+    all S indices) when S <= decode_all_max, else every group's leaves element by element
+    (decode_digits over all of the group's leaves vs the oracle's canonical leaf stream) for
+    groups of at most leaves_max leaves."""
     from paper_conf_hpdc_raschg18_b200 import _lib as L
     ref = orc.info(spec, threads=8)
-    flags = _flags(generic) | (L.ATF_FLAG_LEGACY_WIDE if legacy else 0) | (L.ATF_FLAG_NO_JIT if no_jit else 0)
+    flags = (_flags(generic) | (L.ATF_FLAG_LEGACY_WIDE if legacy else 0) | (L.ATF_FLAG_NO_JIT if no_jit else 0)
+             | extra_flags)
     with Space(spec, flags=flags) as sp:
         sp.generate()
         assert sp.groups() == [g["members"] for g in ref["groups"]]
@@ -72,6 +78,28 @@ def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, 
             got = sp.decode(idx).cpu().numpy()
             _, want = orc.decode(spec, np.arange(S, dtype=np.uint64))
             assert np.array_equal(got, want), spec.name
+        elif S > decode_all_max:
+            checked = 0
+            for g, grp in enumerate(ref["groups"]):
+                if grp["size"] > leaves_max:
+                    continue
+                assert _group_leaves(sp, g, grp["size"]).equal(
+                    torch.from_numpy(orc.leaves(spec, g, len(grp["members"])))), (spec.name, g)
+                checked += 1
+            assert checked, spec.name
+
+
+def _group_leaves(sp, g, size, start=0, chunk=1 << 22):
+    """Leaves [start, start+size) of group g as int32 [n][members] (host), via decode_digits."""
+    members = sp.groups()[g]
+    G = sp.num_groups()
+    parts = []
+    for s0 in range(start, start + size, chunk):
+        n = min(chunk, start + size - s0)
+        dig = torch.zeros((G, n), dtype=torch.int64, device="cuda")
+        dig[g] = torch.arange(s0, s0 + n, dtype=torch.int64, device="cuda")
+        parts.append(sp.decode_digits(dig)[members].T.cpu())
+    return torch.cat(parts) if parts else torch.zeros((0, len(members)), dtype=torch.int32)
 
 
 SMALL = {
@@ -98,6 +126,14 @@ SMALL = {
 @pytest.mark.parametrize("generic", [False, True])
 def test_small_specs(Space, name, generic):
     _check_against_oracle(Space, SMALL[name](), generic=generic)
+
+
+@pytest.mark.parametrize("name", ["C5-60x5", "C5-300x4", "C5-4096x3", "C2-256", "C3-IS1", "C3-12x30x8"])
+def test_small_specs_every_pair_evaluated(Space, name):
+    """ATF_FLAG_NO_SEG_BOUNDS (the bench headline's configuration: all f_{k-1} r_k pairs
+    evaluated) gives the same space."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    _check_against_oracle(Space, SMALL[name](), extra_flags=L.ATF_FLAG_NO_SEG_BOUNDS)
 
 
 @pytest.mark.parametrize("seed", range(80))
@@ -132,6 +168,32 @@ def test_small_specs_generic_narrow_kernel(Space, name):
 @pytest.mark.parametrize("seed", range(0, 80, 9))
 def test_fuzz_specs_generic_narrow_kernel(Space, seed):
     _check_against_oracle(Space, A.random_spec(seed), no_jit=True)
+
+
+@pytest.mark.parametrize("name", ["C1", "C2-256", "C3-IS1", "C3-IS3", "C3-12x30x8", "saxpy360", "C5-300x4"])
+def test_small_specs_without_tail(Space, name):
+    """ATF_FLAG_NO_TAIL: the trailing narrow levels one level at a time (expand_nfast +
+    nfast_emit) instead of the fused tail give the same space."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    _check_against_oracle(Space, SMALL[name](), extra_flags=L.ATF_FLAG_NO_TAIL)
+
+
+@pytest.mark.parametrize("seed", range(0, 80, 7))
+def test_fuzz_specs_without_tail(Space, seed):
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    _check_against_oracle(Space, A.random_spec(seed), extra_flags=L.ATF_FLAG_NO_TAIL)
+
+
+def test_tail_kernel_runs(Space):
+    """C3's trailing narrow levels KWI, VWM, VWN (and C2's VWMD, VWND) run as one fused tail
+    (kernel id 5), with every pair of those levels evaluated."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    for spec, want in ((A.c3_xgemm("IS1"), [7, 8, 9]), (A.c2_xgemm_direct(256), [6, 7])):
+        with Space(spec, flags=L.ATF_FLAG_TIMING) as sp:
+            sp.generate()
+            st = [x for x in sp.stats() if x["group"] == 0]
+            assert [x["level"] for x in st if x["kernel"] == 5] == want
+            assert all(x["pairs"] == x["evals"] for x in st if x["kernel"] == 5)
 
 
 def test_jit_kernels_run(Space):
@@ -257,23 +319,64 @@ def _group_hash(sp, g, size, n_params, chunk=1 << 24):
     return H
 
 
-@pytest.mark.parametrize("name", ["C2", "C2-1024", "C3-IS1", "C3-IS3", "C3-IS2", "C3-IS4", "C3-IS4-anchored", "C5-512"])
-def test_full_size_against_golden(Space, name):
+FULL = ["C2", "C2-1024", "C3-IS1", "C3-IS3", "C3-IS2", "C3-IS4", "C3-IS4-anchored", "C5-512", "C5"]
+
+
+@pytest.mark.parametrize("every_pair", [True, False])
+@pytest.mark.parametrize("name", FULL)
+def test_full_size_against_golden(Space, name, every_pair):
+    """Full-size configs (C5 = configs[4] at 4096 x 8, the bench workload) in both launch
+    configurations bench.py times (every pair evaluated = the headline; segment bounds = the
+    secondary line): S, every f_k, the order-dependent hash of every group's leaves (all of
+    them, in canonical order), element-wise windows of leaf rows (first / middle / last 1024
+    leaves of every group, where the golden has them) and the C4 sampled decodes."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
     from tests.golden.make_golden import SPECS
     gold = _golden(name)
     spec = SPECS[name]()
-    with Space(spec) as sp:
+    with Space(spec, flags=L.ATF_FLAG_NO_SEG_BOUNDS if every_pair else 0) as sp:
         sp.generate()
         assert sp.size() == int(gold["S"])
         for g, grp in enumerate(gold["groups"]):
             assert sp.level_sizes(g) == [lv["f"] for lv in grp["levels"]]
             assert _group_hash(sp, g, grp["size"], len(spec.params)) == int(grp["hash"]), (name, g)
+        for g, wins in enumerate(gold.get("windows", [])):
+            for w in wins:
+                want = torch.tensor(w["rows"], dtype=torch.int32)
+                got = _group_leaves(sp, g, want.shape[0], start=w["start"])
+                assert got.equal(want), (name, g, w["start"])
         if "decode" in gold:
             d = gold["decode"]
             idx = torch.from_numpy(splitmix64_indices(d["n"], int(gold["S"]), d["seed"]).view(np.int64)).cuda()
             out = sp.decode(idx)
             assert torch_rowhash(out) == int(d["hash"])
             assert out[:, :8].T.cpu().tolist() == d["first_rows"]
+
+
+def test_c4_decode_all_1e8_indices(Space):
+    """configs[3] in full: decode of all 10^8 splitmix indices into C3-IS2 (the bench's C4
+    launch: one decode_indices call over the whole batch), compared with the oracle's hash of
+    all 10^8 rows (tests/golden/C3-IS2.json "decode_full"), plus 2*10^6 rows element by element
+    against the oracle's own decode (a window at the start and one at the end of the batch)."""
+    from tests.golden.make_golden import SPECS
+    gold = _golden("C3-IS2")
+    d = gold["decode_full"]
+    spec = SPECS["C3-IS2"]()
+    S = int(gold["S"])
+    idx_h = splitmix64_indices(d["n"], S, d["seed"])
+    with Space(spec) as sp:
+        sp.generate()
+        idx = torch.from_numpy(idx_h.view(np.int64)).cuda()
+        out = sp.decode(idx)                       # [14][10^8] int32, 5.6 GB
+        del idx
+        H, chunk = 0, 1 << 24
+        for s0 in range(0, d["n"], chunk):
+            H = (H + torch_rowhash(out[:, s0:s0 + chunk], base=s0)) & ((1 << 64) - 1)
+        assert H == int(d["hash"])
+        for s0 in (0, d["n"] - 1_000_000):
+            sel = idx_h[s0:s0 + 1_000_000]
+            _, want = orc.decode(spec, sel, threads=8)
+            assert np.array_equal(out[:, s0:s0 + 1_000_000].cpu().numpy(), want), s0
 
 
 def test_c5_full_closed_form(Space):
@@ -474,18 +577,18 @@ def test_enum_parameters(Space):
         assert all(r["TS"] <= 8 or r["MEM"] == "local" for r in named)
 
 
-def _seg_bound_spec(kind, order):
+def _seg_bound_spec(kind, order, top=1500):
     """Wide divisibility chains whose candidate sets put 0, negatives and large values in
     different warp-tile segments (sorted, reversed, shuffled): the per-segment |x| bounds of
     the hot filter (x | n needs |x| <= |n|, d | x needs |x| >= |d|, 0 passes both) must not
     drop an accepted pair."""
     import random
-    vals = list(range(-40, 0)) + [0] + list(range(1, 1500))
+    vals = list(range(-40, 0)) + [0] + list(range(1, top))
     if order == "reversed":
         vals = vals[::-1]
     elif order == "shuffled":
         random.Random(7).shuffle(vals)
-    s = A.Spec(f"segbound_{kind}_{order}")
+    s = A.Spec(f"segbound_{kind}_{order}_{top}")
     alias = A.divides if kind == "divx" else A.is_multiple_of
     s.add("a", A.interval(-3, 40))
     s.add("b", A.set_(*vals), alias(s.P("a")))
@@ -497,6 +600,20 @@ def _seg_bound_spec(kind, order):
 @pytest.mark.parametrize("order", ["sorted", "reversed", "shuffled"])
 def test_segment_bounds_parity(Space, kind, order):
     _check_against_oracle(Space, _seg_bound_spec(kind, order), decode_all_max=200_000)
+
+
+@pytest.mark.parametrize("kind", ["divx", "mulx"])
+@pytest.mark.parametrize("order", ["sorted", "shuffled"])
+def test_segment_bounds_parity_eight_segments(Space, kind, order):
+    """r = 7341 candidates: both the divisor (x | n) and the multiples (d | x) hot filters run
+    8 segments of 1024 (the 8th, partial, segment included); leaves compared element-wise."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    spec = _seg_bound_spec(kind, order, top=7301)
+    with Space(spec) as sp:
+        sp.generate()
+        assert [x["nseg"] for x in sp.stats()] == [0, 8, 8]
+    _check_against_oracle(Space, spec, decode_all_max=200_000)
+    _check_against_oracle(Space, spec, decode_all_max=200_000, extra_flags=L.ATF_FLAG_NO_SEG_BOUNDS)
 
 
 def test_segment_bounds_skip_work_not_results(Space):

@@ -308,3 +308,115 @@ def test_generator_range_closed_forms():
     s.add("p", cases[2][0])
     with pytest.raises(Exception):
         orc.info(s)
+
+
+# ---------------------------------------------------------------- the oracle's constraint check
+# orc.check (oracle/atf_oracle.cpp cmd_check) decides "valid configuration" ("all valid
+# parameter configurations, i.e., for which the parameters' constraints are satisfied").
+# Pinned three ways, none of which is the oracle's own interpreter: (1) hand-written Python
+# predicates restated from the paper / CLBlast's constraint list on EVERY tuple of the full
+# product, plus values outside the ranges; (2) on fuzz specs, membership in O1's row set over the
+# full product (O1 is pinned by the closed forms above); (3) an out-of-range value in any column
+# makes a row invalid.
+def _product(ranges):
+    grids = np.meshgrid(*[np.asarray(r, dtype=np.int64) for r in ranges], indexing="ij")
+    return np.stack([g.ravel() for g in grids], 1)
+
+
+def _values(spec):
+    out = []
+    for p in spec.params:
+        r = p.range
+        if r["kind"] == "interval":
+            out.append(list(range(r["begin"], r["end"] + 1, r["step"])))
+        elif r["kind"] == "pow2":
+            out.append([1 << i for i in range(r["begin"], r["end"] + 1, r["step"])])
+        else:
+            out.append(list(r["values"]))
+    return out
+
+
+def _dv(a, b):
+    """a | b with the reading-#7 zero rule (a == 0 rejects)."""
+    return a != 0 and b % a == 0
+
+
+def _c2_pred(n):
+    def ok(WGD, MC, NC, MA, NB, KW, VM, VN, PA, PB):
+        return (_dv(WGD, n) and _dv(MC, WGD) and _dv(NC, WGD) and _dv(MA, WGD) and MA != 0
+                and (MC * NC) // MA != 0 and _dv((MC * NC) // MA, WGD) and _dv(NB, WGD) and NB != 0
+                and (MC * NC) // NB != 0 and _dv((MC * NC) // NB, WGD) and _dv(KW, WGD)
+                and _dv(MC * VM, WGD) and _dv(MA * VM, WGD) and _dv(NC * VN, WGD) and _dv(NB * VN, WGD))
+    return ok
+
+
+def _c3_pred(MWG, NWG, KWG, MC, NC, MA, NB, KWI, VM, VN, *_):
+    # CLBlast Xgemm c1-c7 (reading #13): every value >= 1 on these ranges
+    return (_dv(MC, MWG) and _dv(NC, NWG) and _dv(MA, MWG) and _dv(NB, NWG)
+            and (MC * NC) // MA != 0 and _dv((MC * NC) // MA, KWG)
+            and (MC * NC) // NB != 0 and _dv((MC * NC) // NB, KWG) and _dv(KWI, KWG)
+            and _dv(MC * VM, MWG) and _dv(MA * VM, MWG) and _dv(NC * VN, NWG) and _dv(NB * VN, NWG))
+
+
+CHECK_PREDICATES = {
+    # C1 (configs[0]): TS_M | 64, TS_N | 64, TS_M * TS_N <= 1024
+    "C1": (A.c1_toy, lambda m, n: _dv(m, 64) and _dv(n, 64) and m * n <= 1024),
+    # saxpy: WPT | N, LS | (N / WPT)
+    "saxpy12": (lambda: A.saxpy(12), lambda w, l: _dv(w, 12) and _dv(l, 12 // w)),
+    # Fig. 1: tp2 | tp1, tp4 | tp3
+    "fig1": (A.fig1, lambda a, b, c, d: _dv(b, a) and _dv(d, c)),
+    "C2-4": (lambda: A.c2_xgemm_direct(4), _c2_pred(4)),
+    "C3-2x3x2": (lambda: A.c3_xgemm((2, 3, 2)), _c3_pred),
+    # C5 chains: x_k | x_{k-1}, y_{k-1} | y_k
+    "C5-4x3": (lambda: A.c5_chains(4, 3),
+               lambda x0, x1, x2, y0, y1, y2, z0, z1, z2: _dv(x1, x0) and _dv(x2, x1) and _dv(y0, y1)
+               and _dv(y1, y2) and _dv(z1, z0) and _dv(z2, z1)),
+}
+
+
+@pytest.mark.parametrize("name", list(CHECK_PREDICATES))
+def test_check_matches_paper_predicates_on_full_product(oracle_bin, name):
+    mk, pred = CHECK_PREDICATES[name]
+    spec = mk()
+    vals = _values(spec)
+    rows = _product(vals)
+    assert 0 < rows.shape[0] <= 600_000
+    want = np.array([bool(pred(*map(int, r))) for r in rows])
+    got = orc.check(spec, rows.astype(np.int32), per_row=True)
+    assert np.array_equal(got["flags"].astype(bool), want), name
+    assert got["valid"] == int(want.sum()) and got["in_range"] == rows.shape[0]
+    assert 0 < want.sum() < len(want)
+    # the valid rows are exactly the space the oracle enumerates (its size and its rows)
+    d1, o1rows = orc.o1(spec)
+    assert int(d1["S"]) == int(want.sum())
+    assert {tuple(r) for r in o1rows.tolist()} == {tuple(r) for r in rows[want].tolist()}
+
+
+@pytest.mark.parametrize("seed", range(0, 60, 3))
+def test_check_is_o1_membership_on_fuzz_products(oracle_bin, seed):
+    spec = A.random_spec(seed)
+    vals = _values(spec)
+    if any(len(v) == 0 for v in vals) or np.prod([len(v) for v in vals], dtype=object) > 400_000:
+        pytest.skip("empty range or product too large for an exhaustive check")
+    rows = _product(vals)
+    _, o1rows = orc.o1(spec)
+    members = {tuple(r) for r in o1rows.tolist()}
+    want = np.array([tuple(r) in members for r in rows.tolist()])
+    got = orc.check(spec, rows.astype(np.int32), per_row=True)["flags"].astype(bool)
+    assert np.array_equal(got, want)
+
+
+def test_check_rejects_values_outside_the_ranges(oracle_bin):
+    """a configuration takes each parameter's value from its range; a row that is
+    valid except for one column replaced by a value outside that column's range is invalid."""
+    for spec in (A.c1_toy(), A.saxpy(64), A.c3_xgemm((4, 6, 2)), A.c5_chains(6, 3)):
+        _, rows = orc.o1(spec)
+        rows = rows[:200].astype(np.int64)
+        assert orc.check(spec, rows.astype(np.int32))["valid"] == rows.shape[0]
+        vals = _values(spec)
+        bad = rows.copy()
+        for i in range(bad.shape[0]):
+            p = i % bad.shape[1]
+            bad[i, p] = max(vals[p]) + 1 + i   # outside the range (every range here is bounded above)
+        got = orc.check(spec, bad.astype(np.int32), per_row=True)
+        assert got["valid"] == 0 and not got["flags"].any()
