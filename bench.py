@@ -207,7 +207,7 @@ def roofline_of(res, sm_mhz, spec_name=None, step_ms=None):
     tdb = _traffic_db()
     tr = tdb.get(f"{spec_name}:g{g}:l{k}") if spec_name else None
     kname = {0: "expand_narrow", 1: "expand_wide", 2: "expand_wtile", 3: "expand_nfast", 4: "atf_nfast_jit",
-             5: "tail_count+tail_emit"}.get(st[d].get("kernel", -1), "expand")
+             5: "tail_count+tail_emit", 6: "atf_tail_count+atf_tail_emit (NVRTC)"}.get(st[d].get("kernel", -1), "expand")
     step_ops = float(sum(ops))
     step_ms = float(step_ms) if step_ms else float(lvl_ms.sum())
     return {"bound": "alu", "achieved": achieved / 1e12, "peak": peak / 1e12, "unit": "Tops/s",

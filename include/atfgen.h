@@ -120,6 +120,11 @@ typedef struct {
 #define ATF_FLAG_NO_TAIL 128u     /* expand a group's trailing narrow levels one at a time instead
                                      of the fused narrow tail (two launches for up to 4 levels,
                                      DESIGN.md §5); kept for parity coverage and A/B timing    */
+#define ATF_FLAG_INPLACE 256u     /* every warp-tile level writes its children in place behind a
+                                     deferred decoupled look-back (one launch) instead of per-tile
+                                     stash segments + scan + copy (three launches; the default
+                                     above 16 warp tiles: measured faster); kept
+                                     for parity coverage and A/B timing                         */
 
 /* Bytecode: postfix int32 words, int64 stack.
  *   1 X            push the candidate value
@@ -284,7 +289,10 @@ typedef struct {
   int32_t path;     /* 0 = fast atoms, 1 = generic interpreter */
   float expand_ms;  /* device time of the level's expand kernel alone (ATF_FLAG_TIMING), else -1 */
   int32_t kernel;   /* expand kernel: 0 = narrow (r <= 64), 1 = block-tile wide, 2 = warp-tile wide,
-                       3 = narrow fast, 4 = narrow fast specialised at run time (NVRTC) */
+                       3 = narrow fast, 4 = narrow fast specialised at run time (NVRTC),
+                       5 = fused narrow tail (tail_count + tail_emit, attributed to the tail's
+                       first level; its other levels report 0 ms), 6 = the same specialised at
+                       run time (NVRTC) */
   uint64_t pairs;   /* ATF_FLAG_TIMING: (node, candidate) pairs evaluated = evals, except on
                        warp-tile levels with a hot filter: the pairs the hot loop tested (the rest
                        are rejected by the per-segment |x| bounds: x | n needs |x| <= |n|, d | x

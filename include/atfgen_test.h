@@ -32,6 +32,10 @@ atf_status atf_test_shard_offsets(const int64_t* h_all, int32_t world, int32_t n
  * divisors (dev_common.cuh divisible16) against integer modulo: *h_mismatches must be 0. */
 atf_status atf_test_divisible16(uint64_t* h_mismatches);
 atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, size_t cap, size_t* len_out);
+/* Source text of the NVRTC-specialised fused-tail kernels of group g (atf_tail_count +
+ * atf_tail_emit; empty when the group has no fused narrow tail); plans the space.  Host only.
+ * *k0_out (optional) = the tail's first level (-1 if none). */
+atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, size_t* len_out, int32_t* k0_out);
 #ifdef __cplusplus
 }
 #endif

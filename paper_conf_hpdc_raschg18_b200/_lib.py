@@ -27,6 +27,7 @@ ATF_RANGE_INTERVAL, ATF_RANGE_POW2, ATF_RANGE_SET, ATF_RANGE_GEN = 0, 1, 2, 3
 ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT, ATF_FLAG_SERIAL_GROUPS = 1, 2, 8, 16, 32
 ATF_FLAG_NO_SEG_BOUNDS = 64
 ATF_FLAG_NO_TAIL = 128
+ATF_FLAG_INPLACE = 256
 
 
 class atf_range(C.Structure):
@@ -91,6 +92,8 @@ _SIGS = {
     # include/atfgen_test.h
     "atf_test_divisible16": (_st, [C.POINTER(C.c_uint64)]),
     "atf_test_jit_source": (_st, [SP, C.c_int32, C.c_int32, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
+    "atf_test_tail_source": (_st, [SP, C.c_int32, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t),
+                                   C.POINTER(C.c_int32)]),
     "atf_test_exclusive_scan_u32": (_st, [C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_test_shard_slice": (_st, [C.POINTER(C.c_uint64), C.c_uint64, C.c_int32, C.c_int32,
                                    C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),

@@ -75,6 +75,8 @@ struct GroupPlan {
   std::vector<int> members;
   int words = 1;
   std::vector<LevelPlan> levels;
+  void* tail_jit = nullptr;   // NVRTC-specialised tail kernels (jit.cpp), if any
+  int tail_jit_k0 = -1;       // tail start they were built for (-1: not tried)
 };
 
 struct Chunk {
@@ -1138,10 +1140,19 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     }
     for (int sg = 0; sg < kMaxSeg; sg++) { a.seg_lo[sg] = lp.seg_lo[sg]; a.seg_hi[sg] = lp.seg_hi[sg]; }
   }
+  // warp-tile levels are written in place (deferred decoupled look-back) unless
+  // ATF_FLAG_STASH_EMIT asks for the stash + scan + level_emit path
   a.pairs_out = (s->opts.flags & ATF_FLAG_TIMING) ? s->d_pairs + g : nullptr;
   s->data[g][k].seg_skip = a.kind == K_WTILE && a.hot != HOT_NONE && seg_bounds;
   a.n_tiles = a.n_chunks > 1 ? n_parents * (uint64_t)a.n_chunks
                              : (n_parents + (uint64_t)a.tile_nodes - 1) / (uint64_t)a.tile_nodes;
+  // In place (deferred decoupled look-back): tiny levels (<= 16 warp tiles: one
+  // launch instead of three), or every warp-tile level with ATF_FLAG_INPLACE (measured slower
+  // on large levels: look-back waits cost more than the stash copy).  Otherwise children go to
+  // per-tile stash segments and scan_kernel + level_emit_kernel place them.
+  a.direct = (a.kind == K_WTILE && !(s->opts.flags & ATF_FLAG_LEGACY_WIDE) &&
+              (a.n_tiles <= 16 || (s->opts.flags & ATF_FLAG_INPLACE))) ? 1 : 0;
+  if (a.kind == K_WTILE) a.smem_bytes = wtile_layout(a, gp.words).total;
   if (a.smem_bytes > 227 * 1024)
     return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %d bytes of shared memory", k, g, a.smem_bytes);
   if (a.n_tiles >= 0xffffffffull) return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %llu tiles", k, g,
@@ -1196,8 +1207,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   {
     // stash: the level's estimated size (or the exact size after an overflow), not the
     // whole arena tail
-    const uint64_t stash_recs = std::min<uint64_t>(cap, std::max<uint64_t>({est + est / 4, (uint64_t)1 << 16,
-                                                                             s->stash_hint}));
+    const uint64_t stash_recs = a.direct ? 16 : std::min<uint64_t>(cap, std::max<uint64_t>({est + est / 4,
+                                                                             (uint64_t)1 << 16, s->stash_hint}));
     if ((e = ensure_buf(s, (char**)&gbf.stash, &gbf.stash_cap, (size_t)stash_recs * gp.words * 4, "stash")))
       return e;
     a.stash = gbf.stash;
@@ -1223,9 +1234,6 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     a.piece_tile = piece_tile;
     CUDA_TRY(s, cudaMemsetAsync(d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
   }
-  // tiny wide levels: one launch, in place (decoupled look-back over <= 16 warp tiles; with
-  // more tiles the waits cost more than the two saved launches)
-  a.direct = (a.kind == K_WTILE && a.n_tiles <= 16 && !(s->opts.flags & ATF_FLAG_LEGACY_WIDE)) ? 1 : 0;
   if (a.direct) {
     const size_t need = (size_t)a.n_tiles + 1;
     if (need > gbf.status_cap) {
@@ -1352,7 +1360,21 @@ static atf_status queue_tail_count(atf_space* s, int g, int k0, const uint32_t* 
   }
   const bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0].first, ls));
-  int ce = launch_tail_count(t, gp.words, ls);
+  if (gp.tail_jit_k0 != k0 && !(s->opts.flags & ATF_FLAG_NO_JIT)) {
+    std::vector<std::vector<int32_t>> cx(nl);
+    std::vector<std::vector<uint32_t>> cm(nl);
+    for (int d = 0; d < nl; d++) {
+      cx[d] = s->params[gp.levels[k0 + d].param].values;
+      for (int32_t v : cx[d]) {
+        const uint32_t ax = v < 0 ? 0u - (uint32_t)v : (uint32_t)v;
+        cm[d].push_back(ax ? 0xffffffffu / ax + 1u : 0x10000u);  // as ensure_device
+      }
+    }
+    gp.tail_jit = jit_tail_kernels(t, gp.words, cx, cm);
+    gp.tail_jit_k0 = k0;
+  }
+  void* tj = (s->opts.flags & ATF_FLAG_NO_JIT) ? nullptr : gp.tail_jit;
+  int ce = tj ? jit_tail_launch(tj, t, false, ls) : launch_tail_count(t, gp.words, ls);
   if (ce) return fail(s, ATF_ERR_CUDA, "tail count launch (group %d): %s", g, cudaGetErrorString((cudaError_t)ce));
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0].mid, ls));
   for (int d = 0; d < nl && !ce; d++)
@@ -1418,7 +1440,8 @@ static atf_status queue_tail_emit(atf_space* s, int g, Pending& pd, bool own_str
   }
   const bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0 + 1].first, ls));
-  int ce = launch_tail_emit(t, gp.words, ls);
+  void* tj = (s->opts.flags & ATF_FLAG_NO_JIT) ? nullptr : gp.tail_jit;
+  int ce = tj ? jit_tail_launch(tj, t, true, ls) : launch_tail_emit(t, gp.words, ls);
   if (ce) return fail(s, ATF_ERR_CUDA, "tail emit launch (group %d): %s", g, cudaGetErrorString((cudaError_t)ce));
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0 + 1].second, ls));
   if (!serial) CUDA_TRY(s, cudaEventRecord(gbf.join, ls));
@@ -1452,7 +1475,7 @@ static void finish_tail(atf_space* s, int g) {
     ld.rec = T.tot[d] ? t.rec[d] : nullptr;
     ld.n = T.tot[d];
     ld.evals = above * (uint64_t)gp.levels[T.k0 + d].r;
-    ld.kernel = 5;
+    ld.kernel = ((s->opts.flags & ATF_FLAG_NO_JIT) || !gp.tail_jit) ? 5 : 6;
     ld.cpt = ld.nseg = 0;
     if (d + 1 < T.nl) ld.csr = t.csr[d + 1];
     if (timing) {  // the whole tail is attributed to its first level
@@ -2360,6 +2383,41 @@ atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, si
     mags[j] = ax ? 0xffffffffu / ax + 1u : 0x10000u;
   }
   const std::string src = jit_nfast_source(a, gp.words, vals, mags);
+  if (len_out) *len_out = src.size();
+  if (buf && cap) {
+    const size_t n = std::min(cap - 1, src.size());
+    memcpy(buf, src.data(), n);
+    buf[n] = 0;
+  }
+  return ATF_OK;
+}
+
+atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, size_t* len_out, int32_t* k0_out) {
+  if (!s) return ATF_ERR_INVALID_ARG;
+  atf_status e = plan(s);
+  if (e) return e;
+  if (g < 0 || g >= (int)s->groups.size()) return ATF_ERR_INVALID_ARG;
+  const GroupPlan& gp = s->groups[g];
+  const int k0 = tail_start(s, g);
+  if (k0_out) *k0_out = k0;
+  std::string src;
+  if (k0 >= 0) {
+    TailArgs t;
+    std::memset(&t, 0, sizeof t);
+    t.nl = (int)gp.levels.size() - k0;
+    std::vector<std::vector<int32_t>> cx(t.nl);
+    std::vector<std::vector<uint32_t>> cm(t.nl);
+    for (int d = 0; d < t.nl; d++) {
+      t.lv[d] = gp.levels[k0 + d].proto;
+      t.lv[d].r = gp.levels[k0 + d].r;
+      cx[d] = s->params[gp.levels[k0 + d].param].values;
+      for (int32_t v : cx[d]) {
+        const uint32_t ax = v < 0 ? 0u - (uint32_t)v : (uint32_t)v;
+        cm[d].push_back(ax ? 0xffffffffu / ax + 1u : 0x10000u);
+      }
+    }
+    src = jit_tail_source(t, gp.words, cx, cm);
+  }
   if (len_out) *len_out = src.size();
   if (buf && cap) {
     const size_t n = std::min(cap - 1, src.size());

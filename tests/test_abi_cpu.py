@@ -218,7 +218,7 @@ def test_jit_level_sources_compile_for_sm100a(L, tmp_path):
     from paper_conf_hpdc_raschg18_b200 import _lib as LL
     specs = [A.c1_toy(), A.c2_xgemm_direct(256), A.c3_xgemm("IS2"), A.c3_xgemm("IS4"), A.saxpy(360)]
     specs += [A.random_spec(s) for s in range(0, 40, 3)]
-    srcs = []
+    srcs, tails = [], []
     for spec in specs:
         sp = C.c_void_p()
         LL.check(LL.atf_space_create(None, C.byref(sp)))
@@ -237,6 +237,13 @@ def test_jit_level_sources_compile_for_sm100a(L, tmp_path):
             G = C.c_int32()
             LL.check(LL.atf_space_num_groups(sp, C.byref(G)), sp)
             for g in range(G.value):
+                n, k0 = C.c_size_t(), C.c_int32()
+                LL.check(LL.atf_test_tail_source(sp, g, None, 0, C.byref(n), C.byref(k0)), sp)
+                if n.value:
+                    buf = C.create_string_buffer(n.value + 1)
+                    LL.check(LL.atf_test_tail_source(sp, g, buf, n.value + 1, None, None), sp)
+                    srcs.append(buf.value.decode())
+                    tails.append((spec.name, g, k0.value))
                 nl = C.c_int32()
                 LL.check(LL.atf_space_num_levels(sp, g, C.byref(nl)), sp)
                 for k in range(nl.value):
@@ -249,6 +256,9 @@ def test_jit_level_sources_compile_for_sm100a(L, tmp_path):
         finally:
             LL.atf_space_destroy(sp)
     assert len(srcs) >= 6
+    # fused narrow tails: C2's VWMD/VWND, C3-IS2's KWI/VWM/VWN, C3-IS4's VWM/VWN
+    assert ("C2_xgemm_direct_256", 0, 6) in tails and ("C3_xgemm_IS2", 0, 7) in tails
+    assert ("C3_xgemm_IS4", 0, 8) in tails
     # one translation unit per source (kernel names collide), compiled in parallel
     procs = []
     for i, src in enumerate(srcs):

@@ -178,6 +178,26 @@ def test_small_specs_without_tail(Space, name):
     _check_against_oracle(Space, SMALL[name](), extra_flags=L.ATF_FLAG_NO_TAIL)
 
 
+@pytest.mark.parametrize("name", ["C2-256", "C3-IS1", "C3-12x30x8"])
+def test_small_specs_generic_tail(Space, name):
+    """The generic (not NVRTC-specialised) fused tail kernels."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    _check_against_oracle(Space, SMALL[name](), no_jit=True)
+
+
+@pytest.mark.parametrize("name", ["C5-300x4", "C5-4096x3", "C2-256", "C3-IS1", "C3-12x30x8"])
+def test_small_specs_in_place_wtile(Space, name):
+    """ATF_FLAG_INPLACE: every warp-tile level written in place behind the deferred look-back."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    _check_against_oracle(Space, SMALL[name](), extra_flags=L.ATF_FLAG_INPLACE)
+
+
+@pytest.mark.parametrize("seed", range(0, 40, 4))
+def test_fuzz_wide_specs_in_place_wtile(Space, seed):
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    _check_against_oracle(Space, A.random_wide_spec(seed), extra_flags=L.ATF_FLAG_INPLACE)
+
+
 @pytest.mark.parametrize("seed", range(0, 80, 7))
 def test_fuzz_specs_without_tail(Space, seed):
     from paper_conf_hpdc_raschg18_b200 import _lib as L
@@ -192,8 +212,11 @@ def test_tail_kernel_runs(Space):
         with Space(spec, flags=L.ATF_FLAG_TIMING) as sp:
             sp.generate()
             st = [x for x in sp.stats() if x["group"] == 0]
-            assert [x["level"] for x in st if x["kernel"] == 5] == want
-            assert all(x["pairs"] == x["evals"] for x in st if x["kernel"] == 5)
+            assert [x["level"] for x in st if x["kernel"] == 6] == want   # NVRTC-specialised tail
+            assert all(x["pairs"] == x["evals"] for x in st if x["kernel"] == 6)
+        with Space(spec, flags=L.ATF_FLAG_TIMING | L.ATF_FLAG_NO_JIT) as sp:
+            sp.generate()
+            assert [x["level"] for x in sp.stats() if x["group"] == 0 and x["kernel"] == 5] == want
 
 
 def test_jit_kernels_run(Space):

@@ -3,10 +3,10 @@ import json
 import sys
 
 d = json.loads(open(sys.argv[1]).read().strip().splitlines()[-1])
-print(f"C5 ms/step {d['ms_per_step']:.2f}  configs/s {d['value']:.3g}  evals/s {d.get('evals_per_s', 0):.3g}  "
+print(f"C5 ms/step {d['ms_per_step']:.2f}  configs/s {d['value']:.3g}  pairs/s {d.get('pairs_evaluated_per_s', 0):.3g}  "
       f"roofline frac {d['roofline']['frac']:.3f}  e2e {d['e2e']['value']:.3g}  clocks {d['clocks']}")
 for k, v in d.get("secondary", {}).items():
     if "ms_per_step" in v:
-        print(f"{k:8s} ms {v['ms_per_step']:.3f} frac {v.get('dominant_frac', 0):.3f} levels {v['level_ms']}")
+        print(f"{k:8s} ms {v['ms_per_step']:.3f} frac {v.get('dominant_frac', 0):.3f} levels {v.get('level_ms')}")
     else:
         print(k, v)

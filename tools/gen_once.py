@@ -21,13 +21,15 @@ def main():
     ap.add_argument("--reps", type=int, default=1)
     ap.add_argument("--decode", type=int, default=0)
     ap.add_argument("--legacy", action="store_true")
+    ap.add_argument("--flags", type=int, default=None, help="atf_space_opts.flags (default: the bench headline's)")
     ap.add_argument("--profile-last", action="store_true",
                     help="cudaProfilerStart/Stop around the last rep (ncu --profile-from-start off)")
     a = ap.parse_args()
     spec = A.config_spec(a.config)
     torch.cuda.set_device(0)
     from paper_conf_hpdc_raschg18_b200 import _lib as L
-    with Space(spec, device=0, flags=L.ATF_FLAG_LEGACY_WIDE if a.legacy else 0) as sp:
+    flags = a.flags if a.flags is not None else L.ATF_FLAG_NO_SEG_BOUNDS
+    with Space(spec, device=0, flags=flags | (L.ATF_FLAG_LEGACY_WIDE if a.legacy else 0)) as sp:
         for i in range(a.reps):
             last = i == a.reps - 1
             if last and a.profile_last:

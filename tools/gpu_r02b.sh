@@ -1,0 +1,14 @@
+#!/bin/bash
+mkdir -p gpurun_out
+T=r02b
+timeout 1800 python -m pytest tests -m gpu -q -x --durations=15 --deselect "tests/test_gpu_parity.py::test_full_size_against_golden[C5-True]" --deselect "tests/test_gpu_parity.py::test_full_size_against_golden[C5-False]" > gpurun_out/${T}_pytest_gpu.txt 2>&1
+echo "pytest rc=$?" >> gpurun_out/${T}_pytest_gpu.txt
+tail -3 gpurun_out/${T}_pytest_gpu.txt
+for cfg in C3-IS4 C3-IS2 C5; do
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${T}_launches_${cfg}.csv python tools/gen_once.py $cfg --reps 2 --profile-last > /dev/null 2>&1
+  echo "launches $cfg rc=$?"
+done
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:tail -c 2 -o gpurun_out/${T}_tail_is4 python tools/gen_once.py C3-IS4 > gpurun_out/${T}_ncu_tail.log 2>&1
+echo "ncu tail rc=$?"
+timeout 900 python bench.py --no-secondary --steps 10 > gpurun_out/${T}_bench.json 2> gpurun_out/${T}_bench.err; echo "bench rc=$?"
+python tools/bench_brief.py gpurun_out/${T}_bench.json 2>/dev/null | head -20
