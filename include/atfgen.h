@@ -120,11 +120,6 @@ typedef struct {
 #define ATF_FLAG_NO_TAIL 128u     /* expand a group's trailing narrow levels one at a time instead
                                      of the fused narrow tail (two launches for up to 4 levels,
                                      DESIGN.md §5); kept for parity coverage and A/B timing    */
-#define ATF_FLAG_INPLACE 256u     /* every warp-tile level writes its children in place behind a
-                                     deferred decoupled look-back (one launch) instead of per-tile
-                                     stash segments + scan + copy (three launches; the default
-                                     above 16 warp tiles: measured faster); kept
-                                     for parity coverage and A/B timing                         */
 
 /* Bytecode: postfix int32 words, int64 stack.
  *   1 X            push the candidate value
@@ -243,6 +238,17 @@ atf_status atf_space_decode_indices(const atf_space* s, const uint64_t* d_idx, i
  * (digit of group g at d_digits + g*n, each < |G_g|); works for any S. */
 atf_status atf_space_decode_digits(const atf_space* s, const uint64_t* d_digits, int64_t n,
                                    int32_t* d_out, int64_t ld, void* stream);
+
+/* Indices of any size (S may be >= 2^64; P:280 mentions spaces of ~10^19 configurations):
+ * index i = hi * 2^64 + lo.  decode_indices128 takes per-row device arrays d_idx_lo[n] /
+ * d_idx_hi[n]; decode_range decodes the n consecutive indices first, first + 1, ... (the
+ * exhaustive search of P:218) with first = first_hi * 2^64 + first_lo.  Output and errors as
+ * atf_space_decode_indices (rows >= S: INT32_MIN and ATF_ERR_INDEX; the call synchronises
+ * the stream once to read the out-of-range flag). */
+atf_status atf_space_decode_indices128(const atf_space* s, const uint64_t* d_idx_lo, const uint64_t* d_idx_hi,
+                                       int64_t n, int32_t* d_out, int64_t ld, void* stream);
+atf_status atf_space_decode_range(const atf_space* s, uint64_t first_lo, uint64_t first_hi, int64_t n, int32_t* d_out,
+                                  int64_t ld, void* stream);
 
 /* Encode = inverse of decode (the index access of P:229-231 read
  * backwards, which also answers membership): d_values is a batch of n configurations,

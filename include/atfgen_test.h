@@ -26,11 +26,13 @@ atf_status atf_test_shard_slice(const uint64_t* h_csr, uint64_t ncut, int32_t ra
                                 uint64_t* hi);
 atf_status atf_test_shard_offsets(const int64_t* h_all, int32_t world, int32_t n, int32_t rank, uint64_t* before,
                                   uint64_t* tot);
-/* Source text of the NVRTC-specialised pass-1 kernel of level k of group g (empty when the
- * level is not a narrow fast level); plans the space if needed.  Host only. */
+
 /* Exhaustive device check of the float-reciprocal divisibility test used for 16-bit quotient
  * divisors (dev_common.cuh divisible16) against integer modulo: *h_mismatches must be 0. */
 atf_status atf_test_divisible16(uint64_t* h_mismatches);
+/* Source text of the NVRTC-specialised kernel of level k of group g: the pass-1 kernel of a
+ * narrow fast level, the exact-mask kernel of a mid-width (32 < r <= 1024) nf_ok level; empty
+ * otherwise.  Plans the space if needed.  Host only. */
 atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, size_t cap, size_t* len_out);
 /* Source text of the NVRTC-specialised fused-tail kernels of group g (atf_tail_count +
  * atf_tail_emit; empty when the group has no fused narrow tail); plans the space.  Host only.

@@ -27,7 +27,6 @@ ATF_RANGE_INTERVAL, ATF_RANGE_POW2, ATF_RANGE_SET, ATF_RANGE_GEN = 0, 1, 2, 3
 ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT, ATF_FLAG_SERIAL_GROUPS = 1, 2, 8, 16, 32
 ATF_FLAG_NO_SEG_BOUNDS = 64
 ATF_FLAG_NO_TAIL = 128
-ATF_FLAG_INPLACE = 256
 
 
 class atf_range(C.Structure):
@@ -79,6 +78,8 @@ _SIGS = {
     "atf_space_level_size": (_st, [SP, C.c_int32, C.c_int32, C.POINTER(C.c_uint64)]),
     "atf_space_level_view": (_st, [SP, C.c_int32, C.c_int32, C.POINTER(atf_level_view)]),
     "atf_space_decode_indices": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
+    "atf_space_decode_indices128": (_st, [SP, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
+    "atf_space_decode_range": (_st, [SP, C.c_uint64, C.c_uint64, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_space_decode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_space_encode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p]),
     "atf_space_encode_indices": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p, C.c_void_p]),

@@ -151,7 +151,6 @@ struct TailArgs {
 constexpr int kNfNPL = 4;  // narrow fast kernel: frontier nodes per lane (warp tile = 128 nodes)
 constexpr int kWT = 32;        // warp-tile kernel: frontier nodes per warp tile (one per lane)
 constexpr int kItemCap = 512;  // warp-tile kernel: items whose exact masks pass 1 keeps for the emit pass
-constexpr int kItemCapD = 256; // same, per buffer set, for in-place levels (two sets: deferred emit)
 constexpr int kPieceShift = 10;  // level_emit_kernel copies the level in pieces of 2^10 records
 // Hot-loop filter of the wide kernel: a superset test of one conjunct, 2 instructions per
 // (node, candidate) pair (IMAD + ISETP.OR into a per-node predicate).
@@ -258,7 +257,7 @@ ATF_HD SmemLayout expand_layout(const LevelArgs& a, int words) {
 // private region per warp (its tile's records, gates, hot operands, item words, operands).
 struct WarpLayout {
   int tab, qtab, warp0, wstride;            // CTA part; warp w's region at warp0 + w * wstride
-  int rec, ok, hot, hot2, cnt, items, imask, icode, opa, opb, slots, poff;  // offsets inside a warp region
+  int rec, ok, hot, hot2, cnt, items, imask, icode, opa, opb, slots;  // offsets inside a warp region
   int total;
 };
 ATF_HD WarpLayout wtile_layout(const LevelArgs& a, int words) {
@@ -268,17 +267,14 @@ ATF_HD WarpLayout wtile_layout(const LevelArgs& a, int words) {
   if (a.qmax > 0) { L.qtab = o; o = align16(o + 4 * ((int)a.qmax + 1)); } else { L.qtab = -1; }
   L.warp0 = o;
   int w = 0;
-  // in place (a.direct): tile records and item buffers in two sets (deferred emit)
-  const int sets = a.direct ? 2 : 1, icap = a.direct ? kItemCapD : kItemCap;
-  L.rec = w; w = align16(w + 4 * words * kWT * sets);
+  L.rec = w; w = align16(w + 4 * words * kWT);
   L.ok = w; w += 4 * kWT;
   L.hot = w; w += 4 * kWT;
   L.hot2 = w; w += 4 * kWT;
   L.cnt = w; w += 4 * kWT;
   L.items = w; w = align16(w + 4 * kWT * a.nseg);
-  L.imask = w; w = align16(w + 4 * icap * sets);
-  L.icode = w; w = align16(w + 2 * icap * sets);
-  if (a.direct) { L.poff = w; w = align16(w + 4 * (kWT + 4)); } else { L.poff = -1; }
+  L.imask = w; w = align16(w + 4 * kItemCap);
+  L.icode = w; w = align16(w + 2 * kItemCap);
   L.opa = w; w = align16(w + 8 * kWT * a.n_terms);
   L.opb = w; w = align16(w + 8 * kWT * a.n_terms);
   if (a.need_slots_smem) { L.slots = w; w = align16(w + 8 * kWT * a.n_slots); } else { L.slots = -1; }
@@ -308,15 +304,29 @@ namespace atf {
 std::string jit_nfast_source(const LevelArgs& a, int words, const std::vector<int32_t>& cand_values,
                              const std::vector<uint32_t>& cand_magics);
 // jit.cpp: fused narrow tail, specialised count + emit kernels (nullptr if not covered / no NVRTC)
+// (k0 = the tail's first group level, pv_level[d][s] = group level of slot s's ancestor at tail level d)
 std::string jit_tail_source(const TailArgs& t, int words, const std::vector<std::vector<int32_t>>& cand_values,
-                            const std::vector<std::vector<uint32_t>>& cand_magics);
+                            const std::vector<std::vector<uint32_t>>& cand_magics, int k0,
+                            const std::vector<std::vector<int>>& pv_level);
 void* jit_tail_kernels(const TailArgs& t, int words, const std::vector<std::vector<int32_t>>& cand_values,
-                       const std::vector<std::vector<uint32_t>>& cand_magics);
+                       const std::vector<std::vector<uint32_t>>& cand_magics, int k0,
+                       const std::vector<std::vector<int>>& pv_level);
 int jit_tail_launch(void* handle, const TailArgs& t, bool emit, void* stream);
+// jit.cpp: mid-width levels (nf_ok, 32 < r <= kWideJitMax), specialised exact-mask kernel
+constexpr int kWideJitMax = 1024;
+std::string jit_wide_source(const LevelArgs& a, int words, const std::vector<int32_t>& cand_values,
+                            const std::vector<uint32_t>& cand_magics);
+void* jit_wide_kernel(const LevelArgs& a, int words, const std::vector<int32_t>& cand_values,
+                      const std::vector<uint32_t>& cand_magics);
+int jit_wide_smem(int r, int words);
+int jit_wide_launch(void* kernel, const LevelArgs& a, int words, void* stream);
 int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out,
                           int64_t ld, unsigned int* bad_flag, void* stream);
 int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,
                          int64_t ld, unsigned int* bad_flag, void* stream);
+int launch_decode128(const DecodeArgs& a, const uint64_t* idx_lo, const uint64_t* idx_hi, uint64_t first_lo,
+                     uint64_t first_hi, int64_t n, int32_t* out, int64_t ld, unsigned int* bad, uint64_t S_lo,
+                     uint64_t S_hi, void* stream);
 int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long long* status,
                     unsigned int* counter, void* stream, uint32_t* piece_tile = nullptr,
                     uint64_t piece_cap = 0);

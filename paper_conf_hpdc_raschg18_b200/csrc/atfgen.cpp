@@ -21,8 +21,17 @@
 #include <vector>
 
 #include "atf_internal.hpp"
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX3: ranges are free unless a profiler attaches
 
 using namespace atf;
+
+namespace {
+// NVTX range for the lifetime of a scope (nsys / ncu --nvtx show the level rounds)
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
 using i128 = __int128;
 using u128 = unsigned __int128;
 
@@ -66,6 +75,8 @@ struct LevelPlan {
   bool generic = false;
   std::string desc;
   void* jit = nullptr;       // NVRTC-specialised narrow kernel (jit.cpp), if any
+  void* wide_jit = nullptr;  // NVRTC-specialised mid-width kernel (jit.cpp), if any
+  bool wide_jit_tried = false;
   int seg_cpt = -1;          // cpt the cached warp-tile segment bounds were computed for
   uint32_t seg_lo[kMaxSeg], seg_hi[kMaxSeg];
   bool jit_tried = false;
@@ -752,7 +763,7 @@ static atf_status plan(atf_space* s) {
       while (w < fill.size() && fill[w] + fb[l] > 32) w++;
       if (w == fill.size()) fill.push_back(0);
       fw[l] = (int)w;
-      fs[l] = fill[w];
+      fs[l] = fb[l] ? fill[w] : 0;  // a 0-bit field (r <= 1) never shifts by 32
       fill[w] += fb[l];
     }
     int words = std::max<int>(1, (int)fill.size());
@@ -1143,15 +1154,36 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   // warp-tile levels are written in place (deferred decoupled look-back) unless
   // ATF_FLAG_STASH_EMIT asks for the stash + scan + level_emit path
   a.pairs_out = (s->opts.flags & ATF_FLAG_TIMING) ? s->d_pairs + g : nullptr;
-  s->data[g][k].seg_skip = a.kind == K_WTILE && a.hot != HOT_NONE && seg_bounds;
+  // mid-width nf_ok levels: the NVRTC-specialised exact-mask kernel (jit.cpp), tiles of 32
+  // nodes, stash output protocol of the warp-tile kernel
+  const bool jit_ok = !(s->opts.flags & (ATF_FLAG_NO_JIT | ATF_FLAG_LEGACY_WIDE));
+  void* wide_jit = nullptr;
+  // (frontiers of >= 4096 nodes: lane = node needs enough warp tiles to fill the GPU; a
+  // small frontier with many children per node stays on the warp-tile kernel)
+  if (jit_ok && a.kind == K_WTILE && a.nf_ok && a.r <= kWideJitMax && n_parents >= 4096) {
+    if (!lp.wide_jit_tried) {
+      const auto& vals = s->params[lp.param].values;
+      std::vector<uint32_t> mags(vals.size());
+      for (size_t j = 0; j < vals.size(); j++) {
+        const uint32_t ax = vals[j] < 0 ? 0u - (uint32_t)vals[j] : (uint32_t)vals[j];
+        mags[j] = ax ? 0xffffffffu / ax + 1u : 0x10000u;  // as ensure_device
+      }
+      lp.wide_jit = jit_wide_kernel(a, gp.words, vals, mags);
+      lp.wide_jit_tried = true;
+    }
+    wide_jit = lp.wide_jit;
+    if (wide_jit) {
+      a.tile_nodes = kWT;
+      a.n_chunks = 1;
+    }
+  }
+  s->data[g][k].seg_skip = a.kind == K_WTILE && a.hot != HOT_NONE && seg_bounds && !wide_jit;
   a.n_tiles = a.n_chunks > 1 ? n_parents * (uint64_t)a.n_chunks
                              : (n_parents + (uint64_t)a.tile_nodes - 1) / (uint64_t)a.tile_nodes;
-  // In place (deferred decoupled look-back): tiny levels (<= 16 warp tiles: one
-  // launch instead of three), or every warp-tile level with ATF_FLAG_INPLACE (measured slower
-  // on large levels: look-back waits cost more than the stash copy).  Otherwise children go to
-  // per-tile stash segments and scan_kernel + level_emit_kernel place them.
-  a.direct = (a.kind == K_WTILE && !(s->opts.flags & ATF_FLAG_LEGACY_WIDE) &&
-              (a.n_tiles <= 16 || (s->opts.flags & ATF_FLAG_INPLACE))) ? 1 : 0;
+  // tiny wide levels: one launch, in place (decoupled look-back over <= 16 warp tiles; with
+  // more tiles the waits cost more than the two saved launches: DESIGN.md §5).  Otherwise
+  // children go to per-tile stash segments and scan_kernel + level_emit_kernel place them.
+  a.direct = (a.kind == K_WTILE && !wide_jit && !(s->opts.flags & ATF_FLAG_LEGACY_WIDE) && a.n_tiles <= 16) ? 1 : 0;
   if (a.kind == K_WTILE) a.smem_bytes = wtile_layout(a, gp.words).total;
   if (a.smem_bytes > 227 * 1024)
     return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %d bytes of shared memory", k, g, a.smem_bytes);
@@ -1274,15 +1306,15 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     lp.jit_tried = true;
   }
   const bool use_jit = a.kind == K_NFAST && lp.jit && !(s->opts.flags & (ATF_FLAG_NO_JIT | ATF_FLAG_LEGACY_WIDE));
-  int ce = use_jit ? jit_nfast_launch(lp.jit, a, ls) : launch_expand(a, gp.words, ls);
+  int ce = wide_jit ? jit_wide_launch(wide_jit, a, gp.words, ls)
+                    : (use_jit ? jit_nfast_launch(lp.jit, a, ls) : launch_expand(a, gp.words, ls));
   LevelData& ld = s->data[g][k];
-  ld.cpt = a.kind == K_WTILE ? a.cpt : 0;
-  ld.nseg = a.kind == K_WTILE ? a.nseg : 0;
+  ld.cpt = a.kind == K_WTILE && !wide_jit ? a.cpt : 0;
+  ld.nseg = a.kind == K_WTILE && !wide_jit ? a.nseg : 0;
   ld.launches += a.direct ? 1 : 3;
   if (ce) return fail(s, ATF_ERR_CUDA, "expand launch (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
-  if (use_jit) s->data[g][k].kernel = 4;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].mid, ls));
-  if (!use_jit) s->data[g][k].kernel = a.kind;
+  s->data[g][k].kernel = wide_jit ? 7 : (use_jit ? 4 : a.kind);
   if (a.direct) {
     // nothing more: the expand kernel placed the level
   } else if (a.kind == K_NFAST) {
@@ -1319,6 +1351,25 @@ static int tail_start(const atf_space* s, int g) {
     k0--;
   }
   return L - k0 >= 2 ? k0 : -1;
+}
+
+// Candidate tables and ancestor levels of a tail's levels (the NVRTC generator's inputs).
+static void tail_jit_inputs(const atf_space* s, const GroupPlan& gp, int k0, int nl,
+                            std::vector<std::vector<int32_t>>& cx, std::vector<std::vector<uint32_t>>& cm,
+                            std::vector<std::vector<int>>& pv_level) {
+  cx.assign(nl, {});
+  cm.assign(nl, {});
+  pv_level.assign(nl, {});
+  for (int d = 0; d < nl; d++) {
+    const LevelPlan& lp = gp.levels[k0 + d];
+    cx[d] = s->params[lp.param].values;
+    for (int32_t v : cx[d]) {
+      const uint32_t ax = v < 0 ? 0u - (uint32_t)v : (uint32_t)v;
+      cm[d].push_back(ax ? 0xffffffffu / ax + 1u : 0x10000u);  // as ensure_device
+    }
+    for (int q : lp.pv_param)
+      pv_level[d].push_back((int)(std::find(gp.members.begin(), gp.members.end(), q) - gp.members.begin()));
+  }
 }
 
 // Count round of the tail of group g from frontier `parents` (level k0 - 1, n_parents nodes):
@@ -1361,16 +1412,11 @@ static atf_status queue_tail_count(atf_space* s, int g, int k0, const uint32_t* 
   const bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0].first, ls));
   if (gp.tail_jit_k0 != k0 && !(s->opts.flags & ATF_FLAG_NO_JIT)) {
-    std::vector<std::vector<int32_t>> cx(nl);
-    std::vector<std::vector<uint32_t>> cm(nl);
-    for (int d = 0; d < nl; d++) {
-      cx[d] = s->params[gp.levels[k0 + d].param].values;
-      for (int32_t v : cx[d]) {
-        const uint32_t ax = v < 0 ? 0u - (uint32_t)v : (uint32_t)v;
-        cm[d].push_back(ax ? 0xffffffffu / ax + 1u : 0x10000u);  // as ensure_device
-      }
-    }
-    gp.tail_jit = jit_tail_kernels(t, gp.words, cx, cm);
+    std::vector<std::vector<int32_t>> cx;
+    std::vector<std::vector<uint32_t>> cm;
+    std::vector<std::vector<int>> pvl;
+    tail_jit_inputs(s, gp, k0, nl, cx, cm, pvl);
+    gp.tail_jit = jit_tail_kernels(t, gp.words, cx, cm, k0, pvl);
     gp.tail_jit_k0 = k0;
   }
   void* tj = (s->opts.flags & ATF_FLAG_NO_JIT) ? nullptr : gp.tail_jit;
@@ -1492,7 +1538,10 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
                              std::vector<const uint32_t*> frontier, std::vector<uint64_t> fsize) {
   cudaStream_t st = (cudaStream_t)s->opts.stream;
   std::vector<int> k = k_from;
-  for (;;) {
+  for (int round = 0;; round++) {
+    char rname[48];
+    snprintf(rname, sizeof rname, "atf level round %d", round);
+    NvtxRange nvtx_round(rname);
     std::vector<Pending> pend;
     // levels launched this round: more than one -> one stream per group (concurrent)
     int active = 0;
@@ -1597,6 +1646,7 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
 }
 
 static atf_status generate_impl(atf_space* s) {
+  NvtxRange nvtx("atf_space_generate");
   atf_status e = plan(s);
   if (e) return e;
   if ((e = ensure_device(s))) return e;
@@ -2126,7 +2176,11 @@ atf_status atf_space_filter_product(atf_space* s, uint64_t* h_count, uint64_t* h
   const size_t cbytes = std::max<size_t>(16, (code.size() + progs.size()) * 4);
   int32_t* d_code = (int32_t*)dalloc(s, cbytes);
   unsigned long long* d_cnt = (unsigned long long*)dalloc(s, 16);
-  if (!d_code || !d_cnt) return fail(s, ATF_ERR_OOM, "product filter scratch");
+  if (!d_code || !d_cnt) {
+    dfree(s, d_code, cbytes);
+    dfree(s, d_cnt, 16);
+    return fail(s, ATF_ERR_OOM, "product filter scratch");
+  }
   a.code = d_code;
   a.progs = d_code + code.size();
   std::vector<int32_t> up(code);
@@ -2179,6 +2233,41 @@ atf_status atf_space_decode_indices(const atf_space* s, const uint64_t* d_idx, i
                                     void* stream) {
   if (!d_idx) return fail((atf_space*)s, ATF_ERR_INVALID_ARG, "null indices");
   return decode_common(s, d_idx, nullptr, n, d_out, ld, stream);
+}
+
+static atf_status decode128_common(const atf_space* cs, const uint64_t* lo, const uint64_t* hi, uint64_t first_lo,
+                                   uint64_t first_hi, int64_t n, int32_t* out, int64_t ld, void* stream) {
+  atf_space* s = (atf_space*)cs;
+  if (!s || !out || n < 0 || ld < n) return fail(s, ATF_ERR_INVALID_ARG, "bad decode arguments");
+  if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "decode needs a generated (non-shard) space");
+  u128 S = 1;
+  for (uint64_t z : s->gsize) {
+    if (z && S > (~(u128)0) / z) return fail(s, ATF_ERR_OVERFLOW, "S >= 2^128");
+    S *= z;
+  }
+  if (n == 0) return ATF_OK;
+  CUDA_TRY(s, cudaSetDevice(s->opts.device));
+  cudaStream_t st = (cudaStream_t)(stream ? stream : s->opts.stream);
+  DecodeArgs a;
+  make_decode_args(s, a);
+  CUDA_TRY(s, cudaMemsetAsync(s->d_bad, 0, 4, st));
+  int ce = launch_decode128(a, lo, hi, first_lo, first_hi, n, out, ld, s->d_bad, (uint64_t)S, (uint64_t)(S >> 64), st);
+  if (ce) return fail(s, ATF_ERR_CUDA, "decode launch: %s", cudaGetErrorString((cudaError_t)ce));
+  CUDA_TRY(s, cudaMemcpyAsync(s->h_flags, s->d_bad, 4, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(s, cudaStreamSynchronize(st));
+  if (s->h_flags[0]) return fail(s, ATF_ERR_INDEX, "index out of range (rows set to INT32_MIN)");
+  return ATF_OK;
+}
+
+atf_status atf_space_decode_indices128(const atf_space* s, const uint64_t* d_idx_lo, const uint64_t* d_idx_hi,
+                                       int64_t n, int32_t* d_out, int64_t ld, void* stream) {
+  if (!d_idx_lo || !d_idx_hi) return fail((atf_space*)s, ATF_ERR_INVALID_ARG, "null indices");
+  return decode128_common(s, d_idx_lo, d_idx_hi, 0, 0, n, d_out, ld, stream);
+}
+
+atf_status atf_space_decode_range(const atf_space* s, uint64_t first_lo, uint64_t first_hi, int64_t n, int32_t* d_out,
+                                  int64_t ld, void* stream) {
+  return decode128_common(s, nullptr, nullptr, first_lo, first_hi, n, d_out, ld, stream);
 }
 
 atf_status atf_space_decode_digits(const atf_space* s, const uint64_t* d_digits, int64_t n, int32_t* d_out,
@@ -2382,7 +2471,10 @@ atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, si
     const uint32_t ax = vals[j] < 0 ? 0u - (uint32_t)vals[j] : (uint32_t)vals[j];
     mags[j] = ax ? 0xffffffffu / ax + 1u : 0x10000u;
   }
-  const std::string src = jit_nfast_source(a, gp.words, vals, mags);
+  // narrow fast levels: the pass-1 kernel; mid-width nf_ok levels: the exact-mask kernel
+  const std::string src = a.kind == K_NFAST ? jit_nfast_source(a, gp.words, vals, mags)
+                          : (a.kind == K_WTILE && a.nf_ok && a.r <= kWideJitMax) ? jit_wide_source(a, gp.words, vals, mags)
+                                                                                 : std::string();
   if (len_out) *len_out = src.size();
   if (buf && cap) {
     const size_t n = std::min(cap - 1, src.size());
@@ -2405,18 +2497,15 @@ atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, 
     TailArgs t;
     std::memset(&t, 0, sizeof t);
     t.nl = (int)gp.levels.size() - k0;
-    std::vector<std::vector<int32_t>> cx(t.nl);
-    std::vector<std::vector<uint32_t>> cm(t.nl);
     for (int d = 0; d < t.nl; d++) {
       t.lv[d] = gp.levels[k0 + d].proto;
       t.lv[d].r = gp.levels[k0 + d].r;
-      cx[d] = s->params[gp.levels[k0 + d].param].values;
-      for (int32_t v : cx[d]) {
-        const uint32_t ax = v < 0 ? 0u - (uint32_t)v : (uint32_t)v;
-        cm[d].push_back(ax ? 0xffffffffu / ax + 1u : 0x10000u);
-      }
     }
-    src = jit_tail_source(t, gp.words, cx, cm);
+    std::vector<std::vector<int32_t>> cx;
+    std::vector<std::vector<uint32_t>> cm;
+    std::vector<std::vector<int>> pvl;
+    tail_jit_inputs(s, gp, k0, t.nl, cx, cm, pvl);
+    src = jit_tail_source(t, gp.words, cx, cm, k0, pvl);
   }
   if (len_out) *len_out = src.size();
   if (buf && cap) {

@@ -829,148 +829,6 @@ __device__ __forceinline__ void wtile_decode_item(uint32_t k, uint32_t ie, const
   }
 }
 
-// ---- warp-tile emit (A6): the tile's items in order; lane writes its item's children at
-// their rank (base + tile-local rank) in dst.  Items [0, icap) come from the stored masks /
-// codes, later ones are recomputed.
-template <int W, int CPT, int HOT>
-__device__ __forceinline__ void wtile_emit(const LevelArgs& a, uint32_t T, uint64_t base, uint32_t* dst, uint64_t cap,
-                                           int icap, const uint32_t* t_imask, const uint16_t* t_icode,
-                                           const uint32_t* t_rec, uint32_t ie, const uint32_t* s_items, int nseg,
-                                           uint32_t vword_last, const uint32_t* s_tab, const uint32_t* s_ok,
-                                           const uint32_t* s_hot, const uint32_t* s_hot2, const int64_t* s_opa,
-                                           const int64_t* s_opb, const int64_t* s_slots, const uint32_t* s_q, int lane) {
-  constexpr int SEG = 32 * CPT;
-  uint64_t carry = base;
-  for (uint32_t R = 0; R < T; R += 32) {
-    const uint32_t k = R + lane;
-    int node, sg, b;
-    uint32_t m;
-    if (R < (uint32_t)icap) {
-      const uint32_t code = t_icode[k];
-      m = k < T ? t_imask[k] : 0u;
-      node = (int)(code & 31u);
-      sg = (int)((code >> 5) & 7u);
-      b = (int)(code >> 8);
-    } else {
-      wtile_decode_item<HOT>(k < T ? k : T - 1, ie, s_items, nseg, vword_last, node, sg, b);
-      m = k < T ? wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q)
-                : 0u;
-    }
-    const uint32_t pc = (uint32_t)__popc(m);
-    uint32_t incl = pc;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL, incl, o);
-      if (lane >= o) incl += y;
-    }
-    uint64_t rank = carry + (incl - pc);
-    carry += __shfl_sync(FULL, incl, 31);
-    if (m) {
-      uint32_t rec[W];
-#pragma unroll
-      for (int w = 0; w < W; w++) rec[w] = t_rec[node * W + w];
-      const uint32_t pos0 = (uint32_t)(sg * SEG + b * CPT);
-      while (m) {
-        const int c = __ffs(m) - 1;
-        m &= m - 1;
-        if (rank < cap) {
-          uint32_t out[W];
-#pragma unroll
-          for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? (pos0 + c) << a.field_shift : 0u);
-          store_record<W>(dst + rank * W, out);
-        }
-        rank++;
-      }
-    }
-  }
-}
-
-// In-place levels: exclusive prefix of tile `tile` by look-back (its aggregate is already
-// published; tile 0 published its inclusive prefix), then its inclusive prefix.
-__device__ __forceinline__ unsigned long long wtile_base(const LevelArgs& a, uint64_t tile, unsigned long long total,
-                                                         int lane) {
-  if (tile == 0) return 0ull;
-  unsigned long long excl = 0;
-  int64_t idx = (int64_t)tile - 1 - lane;
-  for (;;) {
-    unsigned long long st = idx >= 0 ? status_load(&a.status[idx]) : kFlagP;
-    while (__any_sync(FULL, (st >> 62) == 0)) {
-      if ((st >> 62) == 0) st = status_load(&a.status[idx]);
-    }
-    const unsigned pm = __ballot_sync(FULL, (st >> 62) == 2);
-    unsigned long long v = st & kValMask;
-    if (pm) {
-      const int first = __ffs(pm) - 1;  // nearest predecessor with an inclusive prefix
-      if (lane > first) v = 0;
-      excl += warp_sum_u64(v);
-      break;
-    }
-    excl += warp_sum_u64(v);
-    idx -= 32;
-  }
-  if (lane == 0) status_store(&a.status[tile], kFlagP | (excl + total));
-  return excl;
-}
-
-// the last tile closes the level: its total and the closing CSR entry; overflow check
-__device__ __forceinline__ void wtile_finish_tile(const LevelArgs& a, uint64_t tile, unsigned long long base,
-                                                  unsigned long long total, int lane) {
-  if (lane == 0) {
-    if (base + total > a.child_cap) atomicOr(a.overflow_flag, 1u);
-    if (tile == a.n_tiles - 1) {
-      *a.total_out = base + total;
-      a.csr[a.n_parents] = base + total;
-    }
-  }
-}
-
-// Resolve the warp's pending in-place tile (every item stored): base, CSR entries, children.
-template <int W>
-__device__ __forceinline__ void wtile_resolve(const LevelArgs& a, const uint32_t* s_pend, const uint32_t* s_poff,
-                                              const uint32_t* p_rec, const uint32_t* p_imask, const uint16_t* p_icode,
-                                              int seg, int cpt, int lane) {
-  const uint64_t tile = s_pend[0];
-  const uint32_t T = s_pend[1], total = s_pend[2];
-  const int tn = (int)s_pend[3];
-  const unsigned long long base = wtile_base(a, tile, total, lane);
-  if (lane < tn) a.csr[tile * (uint64_t)a.tile_nodes + lane] = base + s_poff[lane];
-  wtile_finish_tile(a, tile, base, total, lane);
-  uint64_t carry = base;
-  for (uint32_t R = 0; R < T; R += 32) {
-    const uint32_t k = R + lane;
-    const uint32_t code = p_icode[k < T ? k : 0];
-    uint32_t m = k < T ? p_imask[k] : 0u;
-    const int node = (int)(code & 31u), sg = (int)((code >> 5) & 7u), b = (int)(code >> 8);
-    const uint32_t pc = (uint32_t)__popc(m);
-    uint32_t incl = pc;
-#pragma unroll
-    for (int o = 1; o < 32; o <<= 1) {
-      const uint32_t y = __shfl_up_sync(FULL, incl, o);
-      if (lane >= o) incl += y;
-    }
-    uint64_t rank = carry + (incl - pc);
-    carry += __shfl_sync(FULL, incl, 31);
-    if (m) {
-      uint32_t rec[W];
-#pragma unroll
-      for (int w = 0; w < W; w++) rec[w] = p_rec[node * W + w];
-      const uint32_t pos0 = (uint32_t)(sg * seg + b * cpt);
-      while (m) {
-        const int c = __ffs(m) - 1;
-        m &= m - 1;
-        if (rank < a.child_cap) {
-          uint32_t out[W];
-#pragma unroll
-          for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? (pos0 + c) << a.field_shift : 0u);
-          store_record<W>(a.child_rec + rank * W, out);
-        }
-        rank++;
-      }
-    }
-  }
-  __syncwarp();
-}
-
 template <int W, int CPT, int HOT>
 __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ LevelArgs a) {
   extern __shared__ __align__(16) unsigned char smem[];
@@ -1013,14 +871,6 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
   const int last_lanes = (int)((last_left + CPT - 1) / CPT);
   const uint32_t vword_last = last_lanes >= 32 ? 0xffffffffu : ((1u << last_lanes) - 1u);
 
-  // in place (a.direct): item buffers and tile records are ping-ponged between two sets so
-  // that a tile's emit can wait one tile (deferred look-back, see below)
-  const int icap = a.direct ? kItemCapD : kItemCap;
-  uint32_t* s_poff = L.poff >= 0 ? reinterpret_cast<uint32_t*>(wb + L.poff) : nullptr;
-  uint32_t* s_pend = L.poff >= 0 ? s_poff + kWT : nullptr;  // pending tile: cur, T, total, tn
-  bool have_pend = false;
-  int set = 0;
-
   uint32_t cur = 0, nxt = 0;
   if (lane == 0) {
     cur = atomicAdd(a.tile_counter, 1u);
@@ -1035,18 +885,15 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
     const uint64_t node0 = (uint64_t)cur * TN;
     const uint64_t remn = a.n_parents - node0;
     const int tn = remn < (uint64_t)TN ? (int)remn : TN;
-    uint32_t* t_rec = s_rec + set * (kWT * W);
-    uint32_t* t_imask = s_imask + set * icap;
-    uint16_t* t_icode = s_icode + set * icap;
     // ---- prologue: lane = node
     bool ok = false;
     if (lane < tn) {
       const bool staged = a.level > 0 && pre_tile == cur;
       if (staged) {
 #pragma unroll
-        for (int w = 0; w < W; w++) t_rec[lane * W + w] = pre[w];
+        for (int w = 0; w < W; w++) s_rec[lane * W + w] = pre[w];
       }
-      ok = prologue_node<W>(a, node0 + lane, lane, kWT, s_ok, t_rec, s_opa, s_opb, s_slots, staged);
+      ok = prologue_node<W>(a, node0 + lane, lane, kWT, s_ok, s_rec, s_opa, s_opb, s_slots, staged);
     } else {
       s_ok[lane] = 0u;
     }
@@ -1060,8 +907,7 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
     // segment bounds of the hot filter (A4): x | n (n != 0) needs |x| <= n, d | x (x != 0)
     // needs |x| >= d, so a node quad whose largest n (smallest d) lies outside a segment's
     // [seg_lo, seg_hi] has no item there.  Lane 4q holds quad q's bound; rejected nodes
-    // bound nothing, n == 0 (divisible by every x) bounds everything.  (ATF_FLAG_NO_SEG_BOUNDS:
-    // the host passes bounds no quad falls outside of, every pair is evaluated.)
+    // bound nothing, n == 0 (divisible by every x) bounds everything.
     uint32_t qb = 0;
     if (HOT == HOT_DIVX) {
       qb = ok ? (s_hot[lane] ? s_hot[lane] : 0xffffffffu) : 0u;
@@ -1145,7 +991,7 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
     }
     const uint32_t T = __shfl_sync(FULL, ie, 31);
     ie -= ic;
-    // pass 1: exact masks -> node counts; the first icap items keep (mask, item code =
+    // pass 1: exact masks -> node counts; the first kItemCap items keep (mask, item code =
     // node | seg << 5 | lane << 8) in the warp's shared memory for the emit pass
     for (uint32_t R = 0; R < T; R += 32) {
       const uint32_t k = R + lane;
@@ -1154,14 +1000,14 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
       uint32_t m = 0;
       if (k < T)
         m = wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q);
-      if (k < (uint32_t)icap) {
-        t_imask[k] = m;
-        t_icode[k] = (uint16_t)((uint32_t)node | ((uint32_t)sg << 5) | ((uint32_t)b << 8));
+      if (k < (uint32_t)kItemCap) {
+        s_imask[k] = m;
+        s_icode[k] = (uint16_t)((uint32_t)node | ((uint32_t)sg << 5) | ((uint32_t)b << 8));
       }
       if (m) atomicAdd(&s_cnt[node], (uint32_t)__popc(m));
     }
     __syncwarp();
-    // ---- scan (A5, tile part): node counts -> tile-local CSR offsets
+    // ---- scan (A5, tile part): node counts -> tile-local CSR offsets, stash segment
     const uint32_t cn = lane < tn ? s_cnt[lane] : 0u;
     uint32_t co = cn;
 #pragma unroll
@@ -1171,39 +1017,25 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
     }
     const uint32_t total = __shfl_sync(FULL, co, 31);
     s_cnt[lane] = 0u;  // for the next tile (read above by this lane only)
-
+    unsigned long long sgb = 0;
+    uint32_t* dst = a.stash;
+    uint64_t cap = a.stash_cap;
     if (a.direct) {
-      // In place: the tile's final base is the exclusive prefix of the tile totals, found by a
-      // decoupled look-back over the tile status words.  The tile publishes its aggregate now
-      // and is resolved (look-back, CSR entries, children at their final positions) only after
-      // the warp has computed its NEXT tile, by which time its predecessors (claimed earlier)
-      // have normally published: the warps rarely wait.  Deadlock-free: a warp publishes every
-      // tile it computes before it waits, and waits only on earlier-claimed tiles.  A tile
-      // with more than kItemCapD items (its masks would have to be recomputed) is resolved at
-      // once.
-      if (lane == 0) status_store(&a.status[cur], (cur == 0 ? kFlagP : kFlagA) | (unsigned long long)total);
-      if (have_pend) wtile_resolve<W>(a, s_pend, s_poff, s_rec + (set ^ 1) * (kWT * W), s_imask + (set ^ 1) * icap,
-                                      s_icode + (set ^ 1) * icap, CPT * 32, CPT, lane);
-      have_pend = false;
-      if (T <= (uint32_t)icap) {
-        if (lane == 0) {
-          s_pend[0] = cur;
-          s_pend[1] = T;
-          s_pend[2] = total;
-          s_pend[3] = (uint32_t)tn;
+      // tiny level (a handful of tiles, all resident): the tile's final base by decoupled
+      // look-back; children and CSR entries go straight to their final place (no scan /
+      // copy launches)
+      sgb = lookback(a.status, cur, total, lane);
+      dst = a.child_rec;
+      cap = a.child_cap;
+      if (lane < tn) a.csr[node0 + lane] = sgb + co - cn;
+      if (lane == 0) {
+        if (sgb + total > cap) atomicOr(a.overflow_flag, 1u);
+        if ((uint64_t)cur == a.n_tiles - 1) {
+          *a.total_out = sgb + total;
+          a.csr[a.n_parents] = sgb + total;
         }
-        s_poff[lane] = co - cn;
-        have_pend = true;
-        __syncwarp();
-      } else {
-        const unsigned long long base = wtile_base(a, cur, total, lane);
-        if (lane < tn) a.csr[node0 + lane] = base + co - cn;
-        wtile_finish_tile(a, cur, base, total, lane);
-        wtile_emit<W, CPT, HOT>(a, T, base, a.child_rec, a.child_cap, icap, t_imask, t_icode, t_rec, ie, s_items,
-                                nseg, vword_last, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q, lane);
       }
     } else {
-      unsigned long long sgb = 0;
       if (lane < tn) a.csr[node0 + lane] = co - cn;
       if (lane == 0) {
         sgb = total ? atomicAdd(a.stash_top, (unsigned long long)total) : 0ull;
@@ -1212,16 +1044,55 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
         a.tile_seg[cur] = sgb;
       }
       sgb = __shfl_sync(FULL, sgb, 0);
-      wtile_emit<W, CPT, HOT>(a, T, sgb, a.stash, a.stash_cap, icap, t_imask, t_icode, t_rec, ie, s_items, nseg,
-                              vword_last, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q, lane);
+    }
+    // ---- emit (A6): items in order; lane writes its item's children at their final rank
+    uint64_t carry = sgb;
+    for (uint32_t R = 0; R < T; R += 32) {
+      const uint32_t k = R + lane;
+      int node, sg, b;
+      uint32_t m;
+      if (R < (uint32_t)kItemCap) {
+        const uint32_t code = s_icode[k];
+        m = k < T ? s_imask[k] : 0u;
+        node = (int)(code & 31u);
+        sg = (int)((code >> 5) & 7u);
+        b = (int)(code >> 8);
+      } else {
+        wtile_decode_item<HOT>(k < T ? k : T - 1, ie, s_items, nseg, vword_last, node, sg, b);
+        m = k < T ? wtile_item_mask<CPT, HOT>(a, node, sg, b, s_tab, s_ok, s_hot, s_hot2, s_opa, s_opb, s_slots, s_q)
+                  : 0u;
+      }
+      const uint32_t pc = (uint32_t)__popc(m);
+      uint32_t incl = pc;
+#pragma unroll
+      for (int o = 1; o < 32; o <<= 1) {
+        const uint32_t y = __shfl_up_sync(FULL, incl, o);
+        if (lane >= o) incl += y;
+      }
+      uint64_t rank = carry + (incl - pc);
+      carry += __shfl_sync(FULL, incl, 31);
+      if (m) {
+        uint32_t rec[W];
+#pragma unroll
+        for (int w = 0; w < W; w++) rec[w] = s_rec[node * W + w];
+        const uint32_t pos0 = (uint32_t)(sg * SEG + b * CPT);
+        while (m) {
+          const int c = __ffs(m) - 1;
+          m &= m - 1;
+          if (rank < cap) {
+            uint32_t out[W];
+#pragma unroll
+            for (int w = 0; w < W; w++) out[w] = rec[w] | (w == a.field_word ? (pos0 + c) << a.field_shift : 0u);
+            store_record<W>(dst + rank * W, out);
+          }
+          rank++;
+        }
+      }
     }
     __syncwarp();
-    set ^= 1;
     cur = nxt;
     nxt = nn;
   }
-  if (have_pend) wtile_resolve<W>(a, s_pend, s_poff, s_rec + (set ^ 1) * (kWT * W), s_imask + (set ^ 1) * icap,
-                                  s_icode + (set ^ 1) * icap, CPT * 32, CPT, lane);
   if (a.pairs_out && lane == 0 && pairs) atomicAdd(a.pairs_out, (unsigned long long)pairs);
 }
 

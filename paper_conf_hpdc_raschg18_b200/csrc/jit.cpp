@@ -233,108 +233,118 @@ std::string gen_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx
 }
 
 // ---------------------------------------------------------------- fused narrow tail
-// Accept mask of one node of a tail level as a device function of the node's record words
-// w[0..W): the same straight-line code as the level kernel above (field positions, constants,
-// candidate magics as immediates), candidates r <= 32.  `tab` names the level's ancestor
-// table arrays in the kernel parameters.  "" if the level is not covered.
-std::string gen_mask_fn(const LevelArgs& a, int W, const std::vector<int32_t>& cx, const std::vector<uint32_t>& cm,
-                        const std::string& fname, const std::string& tab) {
-  if (a.n_terms == 0 || a.r > 32 || a.r < 1 || (int)cx.size() != a.r) return "";
-  const int r = a.r;
-  std::string s = "__device__ __forceinline__ u32 " + fname + "(const TailJitArgs& a, const u32* w) {\n";
-  std::vector<int> need_v(a.n_pv, 0), need_m(a.n_pv, 0);
-  auto mark = [&](const NfOp& o, bool mag) {
+// Operand code of level program `a` over a record held in w[] (field positions as immediates,
+// ancestor values / magics from the level's tables `tab`).  `pfx` makes the names unique.
+struct OpGen {
+  const LevelArgs& a;
+  std::string tab, pfx;
+  std::vector<int> need_v, need_m;
+  OpGen(const LevelArgs& a_, std::string tab_, std::string pfx_)
+      : a(a_), tab(std::move(tab_)), pfx(std::move(pfx_)), need_v(a_.n_pv, 0), need_m(a_.n_pv, 0) {}
+  void mark(const NfOp& o, bool mag) {
     if (o.kind == NF_PV) { need_v[o.s1] = 1; if (mag) need_m[o.s1] = 1; }
     if (o.kind == NF_PROD) { need_v[o.s1] = 1; need_v[o.s2] = 1; }
-  };
-  for (int t = 0; t < a.n_terms; t++) {
+  }
+  void mark_term(int t) {
     const Term& T = a.terms[t];
     mark(a.nf_op[t][0], T.kind == T_MULX || T.kind == T_DIVPROD);
     if (T.kind == T_DIVPROD || T.kind == T_QDIV || T.kind == T_CMP) mark(a.nf_op[t][1], false);
   }
-  for (int p = 0; p < a.n_pv; p++) {
-    if (!need_v[p]) continue;
-    const std::string ps = std::to_string(p);
-    const uint32_t bits = (uint32_t)a.pv_bits[p];
-    std::string pos = bits ? "((w[" + std::to_string(a.pv_word[p]) + "] >> " + std::to_string(a.pv_shift[p]) + ") & " +
-                                 hex(bits >= 32 ? 0xffffffffu : ((1u << bits) - 1u)) + ")"
-                           : std::string("0u");
-    s += "  const u32 p" + ps + " = " + pos + ";\n";
-    s += "  const i64 v" + ps + " = (i64)__ldg(a." + tab + "_range[" + ps + "] + p" + ps + ");\n";
-    if (need_m[p]) s += "  const u32 g" + ps + " = __ldg(a." + tab + "_magic[" + ps + "] + p" + ps + ");\n";
-  }
-  auto sval = [&](const NfOp& o) -> std::string {
-    if (o.kind == NF_CONST) return "(i64)" + std::to_string(o.c) + "ll";
-    if (o.kind == NF_PV) return "v" + std::to_string(o.s1);
-    return "(v" + std::to_string(o.s1) + " * v" + std::to_string(o.s2) + ")";
-  };
-  auto magic = [&](const NfOp& o, const std::string& absname) -> std::string {
-    if (o.kind == NF_CONST) return hex(o.cm);
-    if (o.kind == NF_PV) return "(" + absname + " == 0u ? 0u : g" + std::to_string(o.s1) + ")";
-    return "(" + absname + " > 1u ? 0xffffffffu / " + absname + " + 1u : 0u)";
-  };
-  s += "  u32 m = " + hex(r >= 32 ? 0xffffffffu : ((1u << r) - 1u)) + ";\n";
-  auto divx_bits = [&](const std::string& n) {
-    std::string b = "    u32 mm = 0u;\n";
-    for (int c = 0; c < r; c++)
-      if (cx[c] != 0) b += "    mm |= (u32)(" + n + " * " + hex(cm[c]) + " < 0x10000u) << " + std::to_string(c) + ";\n";
-    return b + "    m &= mm;\n";
-  };
-  for (int t = 0; t < a.n_terms; t++) {
-    const Term& T = a.terms[t];
-    const NfOp& oa = a.nf_op[t][0];
-    const NfOp& ob = a.nf_op[t][1];
-    const std::string ts = std::to_string(t);
-    s += "  if (m) {  // term " + ts + "\n";
-    switch (T.kind) {
-      case T_DIVX:
-        s += "    const u32 n" + ts + " = uabs(" + sval(oa) + ");\n" + divx_bits("n" + ts);
-        break;
-      case T_DIVPROD:
-        s += "    const u32 av = uabs(" + sval(oa) + "), bv = uabs(" + sval(ob) + ");\n";
-        s += "    const u32 ma = " + magic(oa, "av") + ";\n";
-        s += "    const u32 n" + ts + " = av == 1u ? bv : __umulhi(bv, ma);\n";
-        s += "    if (av == 0u || n" + ts + " * av != bv) m = 0u;\n";
-        s += "    else {\n" + divx_bits("n" + ts) + "    }\n";
-        break;
-      case T_MULX: {
-        s += "    const u32 d = uabs(" + sval(oa) + ");\n";
-        s += "    const u32 md = " + magic(oa, "d") + ", md1 = md - 1u;\n";
-        s += "    if (d == 0u) m = 0u;\n    else {\n      u32 mm = 0u;\n";
-        for (int c = 0; c < r; c++) {
-          const uint32_t ax = cx[c] < 0 ? 0u - (uint32_t)cx[c] : (uint32_t)cx[c];
-          s += "      mm |= (u32)(" + hex(ax) + " * md <= md1) << " + std::to_string(c) + ";\n";
-        }
-        s += "      m &= mm;\n    }\n";
-        break;
-      }
-      case T_QDIV: {
-        s += "    const u32 num = uabs(" + sval(oa) + "), nb = uabs(" + sval(ob) + ");\n";
-        s += "    u32 mm = 0u;\n";
-        for (int c = 0; c < r; c++) {
-          const uint32_t ax = cx[c] < 0 ? 0u - (uint32_t)cx[c] : (uint32_t)cx[c];
-          if (ax == 0) continue;  // x == 0 rejects
-          const std::string q = ax == 1 ? std::string("num") : "__umulhi(num, " + hex(cm[c]) + ")";
-          s += "    if ((m >> " + std::to_string(c) + ") & 1u) { const u32 q = " + q +
-               "; if (q != 0u && divisible16(nb, q)) mm |= 1u << " + std::to_string(c) + "; }\n";
-        }
-        s += "    m &= mm;\n";
-        break;
-      }
-      case T_CMP: {
-        static const char* rel[] = {"==", "!=", "<", "<=", ">", ">="};
-        if (T.rel < R_EQ || T.rel > R_GE) return "";
-        s += "    const i32 A = (i32)" + sval(oa) + ", B = (i32)" + sval(ob) + ";\n    u32 mm = 0u;\n";
-        for (int c = 0; c < r; c++)
-          s += "    mm |= (u32)(A * " + std::to_string(cx[c]) + " " + rel[T.rel - R_EQ] + " B) << " + std::to_string(c) + ";\n";
-        s += "    m &= mm;\n";
-        break;
-      }
-      default: return "";
+  std::string loads(const std::string& ind) const {  // value (and magic) loads of the marked slots
+    std::string s;
+    for (int p = 0; p < a.n_pv; p++) {
+      if (!need_v[p]) continue;
+      const std::string ps = std::to_string(p), nm = pfx + ps;
+      const uint32_t bits = (uint32_t)a.pv_bits[p];
+      std::string pos = bits ? "((w[" + std::to_string(a.pv_word[p]) + "] >> " + std::to_string(a.pv_shift[p]) + ") & " +
+                                   hex(bits >= 32 ? 0xffffffffu : ((1u << bits) - 1u)) + ")"
+                             : std::string("0u");
+      s += ind + "const u32 p" + nm + " = " + pos + ";\n";
+      s += ind + "const i64 v" + nm + " = (i64)__ldg(a." + tab + "_range[" + ps + "] + p" + nm + ");\n";
+      if (need_m[p]) s += ind + "const u32 g" + nm + " = __ldg(a." + tab + "_magic[" + ps + "] + p" + nm + ");\n";
     }
-    s += "  }\n";
+    return s;
   }
-  return s + "  return m;\n}\n";
+  std::string sval(const NfOp& o) const {
+    if (o.kind == NF_CONST) return "(i64)" + std::to_string(o.c) + "ll";
+    if (o.kind == NF_PV) return "v" + pfx + std::to_string(o.s1);
+    return "(v" + pfx + std::to_string(o.s1) + " * v" + pfx + std::to_string(o.s2) + ")";
+  }
+  std::string magic(const NfOp& o, const std::string& absname) const {
+    if (o.kind == NF_CONST) return hex(o.cm);
+    if (o.kind == NF_PV) return "(" + absname + " == 0u ? 0u : g" + pfx + std::to_string(o.s1) + ")";
+    return "(" + absname + " > 1u ? 0xffffffffu / " + absname + " + 1u : 0u)";
+  }
+};
+
+// Per-term node operands -> u32 words (a term's "node constants"): DIVX n | DIVPROD n, or
+// 0xffffffff when the gate a | b fails | MULX md, md - 1, d == 0 | QDIV num, nb | CMP A, B.
+int nc_words(const Term& T) { return T.kind == T_MULX ? 3 : (T.kind == T_QDIV || T.kind == T_CMP) ? 2 : 1; }
+std::string nc_code(const LevelArgs& a, int t, const OpGen& g, const std::string& dst, const std::string& ind) {
+  const Term& T = a.terms[t];
+  const NfOp& oa = a.nf_op[t][0];
+  const NfOp& ob = a.nf_op[t][1];
+  std::string s = ind + "{\n";
+  switch (T.kind) {
+    case T_DIVX: s += ind + "  " + dst + "[0] = uabs(" + g.sval(oa) + ");\n"; break;
+    case T_DIVPROD:
+      s += ind + "  const u32 av = uabs(" + g.sval(oa) + "), bv = uabs(" + g.sval(ob) + ");\n";
+      s += ind + "  const u32 ma = " + g.magic(oa, "av") + ";\n";
+      s += ind + "  const u32 n = av == 1u ? bv : __umulhi(bv, ma);\n";
+      s += ind + "  " + dst + "[0] = (av == 0u || n * av != bv) ? 0xffffffffu : n;\n";
+      break;
+    case T_MULX:
+      s += ind + "  const u32 d = uabs(" + g.sval(oa) + ");\n";
+      s += ind + "  const u32 md = " + g.magic(oa, "d") + ";\n";
+      s += ind + "  " + dst + "[0] = md; " + dst + "[1] = md - 1u; " + dst + "[2] = d == 0u;\n";
+      break;
+    case T_QDIV:
+      s += ind + "  " + dst + "[0] = uabs(" + g.sval(oa) + "); " + dst + "[1] = uabs(" + g.sval(ob) + ");\n";
+      break;
+    default:
+      s += ind + "  " + dst + "[0] = (u32)(i32)" + g.sval(oa) + "; " + dst + "[1] = (u32)(i32)" + g.sval(ob) + ";\n";
+  }
+  return s + ind + "}\n";
+}
+
+// Mask code of term t from its node constants `nc` (base index i0) over r <= 32 candidates.
+std::string term_mask_code(const LevelArgs& a, int t, const std::vector<int32_t>& cx, const std::vector<uint32_t>& cm,
+                           const std::string& nc) {
+  const Term& T = a.terms[t];
+  const int r = a.r;
+  std::string s = "  if (m) {  // term " + std::to_string(t) + "\n    u32 mm = 0u;\n";
+  switch (T.kind) {
+    case T_DIVX: case T_DIVPROD:
+      s += "    const u32 n = " + nc + "[0];\n";
+      if (T.kind == T_DIVPROD) s += "    if (n == 0xffffffffu) m = 0u;\n";
+      for (int c = 0; c < r; c++)
+        if (cx[c] != 0) s += "    mm |= (u32)(n * " + hex(cm[c]) + " < 0x10000u) << " + std::to_string(c) + ";\n";
+      break;
+    case T_MULX:
+      s += "    const u32 md = " + nc + "[0], mq = " + nc + "[1];\n    if (" + nc + "[2]) m = 0u;\n";
+      for (int c = 0; c < r; c++) {
+        const uint32_t ax = cx[c] < 0 ? 0u - (uint32_t)cx[c] : (uint32_t)cx[c];
+        s += "    mm |= (u32)(" + hex(ax) + " * md <= mq) << " + std::to_string(c) + ";\n";
+      }
+      break;
+    case T_QDIV:
+      s += "    const u32 num = " + nc + "[0], nb = " + nc + "[1];\n";
+      for (int c = 0; c < r; c++) {
+        const uint32_t ax = cx[c] < 0 ? 0u - (uint32_t)cx[c] : (uint32_t)cx[c];
+        if (ax == 0) continue;  // x == 0 rejects
+        const std::string q = ax == 1 ? std::string("num") : "__umulhi(num, " + hex(cm[c]) + ")";
+        s += "    if ((m >> " + std::to_string(c) + ") & 1u) { const u32 q = " + q +
+             "; if (q != 0u && divisible16(nb, q)) mm |= 1u << " + std::to_string(c) + "; }\n";
+      }
+      break;
+    default: {
+      static const char* rel[] = {"==", "!=", "<", "<=", ">", ">="};
+      s += "    const i32 A = (i32)" + nc + "[0], B = (i32)" + nc + "[1];\n";
+      for (int c = 0; c < r; c++)
+        s += "    mm |= (u32)(A * " + std::to_string(cx[c]) + " " + rel[T.rel - R_EQ] + " B) << " + std::to_string(c) + ";\n";
+    }
+  }
+  return s + "    m &= mm;\n  }\n";
 }
 
 // Kernel parameters of the generated tail kernels (same layout on both sides).
@@ -362,95 +372,400 @@ struct TailJitArgs { const u32* parent_rec; u64 n_parents, n_tiles; u32* tile_to
                      const i32* l2_range[24]; const u32* l2_magic[24]; const i32* l3_range[24]; const u32* l3_magic[24]; };
 )";
 
-// Source of the two tail kernels (atf_tail_count, atf_tail_emit) for levels lv[0..nl): the
-// structure of tail_count / tail_emit in expand.cuh (warp tile = 32 frontier nodes; every
-// tail level processed in chunks of 32 nodes in canonical order; children staged in per-warp
-// shared-memory buffers), every level's mask and child-record code specialised.  The count
-// kernel runs the same chunk walk without the global writes, so no lane diverges.
+// Source of the two tail kernels for levels lv[0..nl) (group levels k0..k0+nl-1; pv_level[d][s] =
+// the group level of slot s's ancestor).  A term whose operands all come from levels above the
+// tail ("node constants") is evaluated ONCE per frontier node (tnc) instead of once per tail node:
+// every tail node below a frontier node shares those ancestors.
+//   atf_tail_count: thread per frontier node, depth-first subtree counts (node constants in
+//                   registers), warp-tile totals per level.
+//   atf_tail_emit:  warp tile = 32 frontier nodes; every tail level in chunks of 32 nodes in
+//                   canonical order; children staged in per-warp shared-memory buffers (with the
+//                   frontier lane they descend from, whose node constants sit in shared memory),
+//                   written out as coalesced vectors, CSR entries of every chunk.
 std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vector<int32_t>>& cx,
-                            const std::vector<std::vector<uint32_t>>& cm) {
+                            const std::vector<std::vector<uint32_t>>& cm, int k0,
+                            const std::vector<std::vector<int>>& pv_level, int* warp_bytes) {
   const int nl = t.nl;
-  if (nl < 2 || nl > kMaxTail) return "";
+  if (nl < 2 || nl > kMaxTail || (int)pv_level.size() < nl) return "";
   std::string s = kPrelude;
   s += kTailPrelude;
   const std::string Ws = std::to_string(W);
+  // node-constant layout: (level, term) -> first word; hoisted iff every operand is above the tail
+  std::vector<std::vector<int>> ncoff(nl);
+  int NNC = 0;
   for (int d = 0; d < nl; d++) {
-    const std::string f = gen_mask_fn(t.lv[d], W, cx[d], cm[d], "tmask" + std::to_string(d), "l" + std::to_string(d));
-    if (f.empty()) return "";
-    s += f;
-  }
-  // per-warp buffer offsets (bytes): level d holds <= 32 * r_d child records
-  std::vector<int> off(nl + 1, 0);
-  for (int d = 0; d < nl; d++) off[d + 1] = off[d] + ((32 * t.lv[d].r * W * 4 + 15) & ~15);
-  const std::string WB = std::to_string(off[nl]);
-  // chunk walk, one function per (mode, depth), deepest first
-  for (int emit = 0; emit < 2; emit++) {
-    for (int d = nl - 1; d >= 0; d--) {
-      const std::string ds = std::to_string(d), nm = std::string(emit ? "e" : "c") + ds;
-      s += "__device__ __forceinline__ void chunk_" + nm + "(const TailJitArgs& a, const u32* rec, bool valid, u64 gidx, "
-           "u64* cur, unsigned char* wbuf, int lane) {\n";
-      s += "  u32 m = valid ? tmask" + ds + "(a, rec) : 0u;\n";
-      s += "  const u32 c = __popc(m);\n  u32 incl = c;\n";
-      s += "#pragma unroll\n  for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
-           "if (lane >= o) incl += y; }\n";
-      s += "  const u32 T = __shfl_sync(0xffffffffu, incl, 31);\n  u32 k = incl - c;\n  const u64 first = cur[" + ds + "];\n";
-      if (emit) s += "  if (valid) a.csr[" + ds + "][gidx] = first + k;\n";
-      const bool stage = emit || d + 1 < nl;
-      const int fw = t.lv[d].field_word, fs = t.lv[d].field_shift;
-      if (stage) {
-        s += "  u32* buf = reinterpret_cast<u32*>(wbuf + " + std::to_string(off[d]) + ");\n";
-        s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n";
-        for (int w = 0; w < W; w++)
-          s += "    buf[k * " + Ws + " + " + std::to_string(w) + "] = rec[" + std::to_string(w) + "]" +
-               (w == fw ? " | (cc << " + std::to_string(fs) + ")" : "") + ";\n";
-        s += "    k++;\n  }\n  __syncwarp();\n";
+    const LevelArgs& a = t.lv[d];
+    if (a.n_terms == 0 || a.r > 32 || a.r < 1 || (int)cx[d].size() != a.r) return "";
+    auto above = [&](const NfOp& o) {
+      if (o.kind == NF_CONST) return true;
+      if (o.kind == NF_PV) return pv_level[d][o.s1] < k0;
+      return pv_level[d][o.s1] < k0 && pv_level[d][o.s2] < k0;
+    };
+    ncoff[d].assign(a.n_terms, -1);
+    for (int tt = 0; tt < a.n_terms; tt++) {
+      const Term& T = a.terms[tt];
+      if (T.kind == T_CMP && (T.rel < R_EQ || T.rel > R_GE)) return "";
+      if (T.kind != T_DIVX && T.kind != T_DIVPROD && T.kind != T_MULX && T.kind != T_QDIV && T.kind != T_CMP) return "";
+      const bool two = T.kind == T_DIVPROD || T.kind == T_QDIV || T.kind == T_CMP;
+      if (above(a.nf_op[tt][0]) && (!two || above(a.nf_op[tt][1]))) {
+        ncoff[d][tt] = NNC;
+        NNC += nc_words(T);
       }
-      if (emit) {
-        if (W == 1) s += "  { u32* dst = a.rec[" + ds + "] + first; for (u32 v = lane; v < T; v += 32) dst[v] = buf[v]; }\n";
-        else if (W == 2)
-          s += "  { uint2* dst = reinterpret_cast<uint2*>(a.rec[" + ds + "] + first * 2); const uint2* src = "
-               "reinterpret_cast<const uint2*>(buf); for (u32 v = lane; v < T; v += 32) dst[v] = src[v]; }\n";
-        else
-          s += "  { uint4* dst = reinterpret_cast<uint4*>(a.rec[" + ds + "] + first * " + Ws + "); const uint4* src = "
-               "reinterpret_cast<const uint4*>(buf); for (u32 v = lane; v < T * " + std::to_string(W / 4) +
-               "; v += 32) dst[v] = src[v]; }\n";
-      }
-      s += "  cur[" + ds + "] = first + T;\n";
-      if (d + 1 < nl) {
-        s += "  for (u32 s0 = 0; s0 < T; s0 += 32) {\n    const bool v = s0 + lane < T;\n    u32 cr[" + Ws + "];\n";
-        for (int w = 0; w < W; w++)
-          s += "    cr[" + std::to_string(w) + "] = v ? buf[(s0 + lane) * " + Ws + " + " + std::to_string(w) + "] : 0u;\n";
-        s += "    chunk_" + std::string(emit ? "e" : "c") + std::to_string(d + 1) + "(a, cr, v, first + s0 + lane, cur, wbuf, lane);\n  }\n";
-      }
-      if (stage) s += "  __syncwarp();\n";
-      s += "}\n";
     }
   }
-  // kernels
-  for (int emit = 0; emit < 2; emit++) {
-    const std::string kn = emit ? "atf_tail_emit" : "atf_tail_count";
-    s += "extern \"C\" __global__ void __launch_bounds__(128) " + kn + "(const __grid_constant__ TailJitArgs a) {\n";
-    s += "  extern __shared__ __align__(16) unsigned char smem[];\n";
-    s += "  const int lane = threadIdx.x & 31;\n  unsigned char* wbuf = smem + (threadIdx.x >> 5) * " + WB + ";\n";
-    s += "  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n  const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n";
-    if (emit) {
-      s += "  if (gw == 0 && lane < " + std::to_string(nl) + ") {\n";
-      s += "    const u64 above = lane == 0 ? a.n_parents : a.tile_base[(u64)(lane - 1) * (a.n_tiles + 1) + a.n_tiles];\n";
-      s += "    a.csr[lane][above] = a.tile_base[(u64)lane * (a.n_tiles + 1) + a.n_tiles];\n  }\n";
-    }
-    s += "  for (u64 tile = gw; tile < a.n_tiles; tile += nw) {\n    u64 cur[" + std::to_string(nl) + "];\n";
-    for (int d = 0; d < nl; d++)
-      s += emit ? "    cur[" + std::to_string(d) + "] = a.tile_base[(u64)" + std::to_string(d) + " * (a.n_tiles + 1) + tile];\n"
-                : "    cur[" + std::to_string(d) + "] = 0;\n";
-    s += "    const u64 nd = tile * 32 + lane;\n    const bool v = nd < a.n_parents;\n    u32 rec[" + Ws + "];\n";
-    s += "    for (int w = 0; w < " + Ws + "; w++) rec[w] = v ? __ldg(a.parent_rec + nd * " + Ws + " + w) : 0u;\n";
-    s += std::string("    chunk_") + (emit ? "e" : "c") + "0(a, rec, v, nd, cur, wbuf, lane);\n";
-    if (!emit)
-      for (int d = 0; d < nl; d++)
-        s += "    if (lane == 0) a.tile_total[(u64)" + std::to_string(d) + " * a.n_tiles + tile] = (u32)cur[" +
-             std::to_string(d) + "];\n";
-    s += "  }\n}\n";
+  const int NC = std::max(NNC, 1);
+  // tnc: node constants of a frontier node
+  s += "__device__ __forceinline__ void tnc(const TailJitArgs& a, const u32* w, u32* nc) {\n";
+  for (int d = 0; d < nl; d++) {
+    OpGen g(t.lv[d], "l" + std::to_string(d), std::to_string(d) + "_");
+    for (int tt = 0; tt < t.lv[d].n_terms; tt++)
+      if (ncoff[d][tt] >= 0) g.mark_term(tt);
+    s += "  {\n" + g.loads("    ");
+    for (int tt = 0; tt < t.lv[d].n_terms; tt++)
+      if (ncoff[d][tt] >= 0) s += nc_code(t.lv[d], tt, g, "(nc + " + std::to_string(ncoff[d][tt]) + ")", "    ");
+    s += "  }\n";
   }
+  s += "}\n";
+  // tmask_d(w, nc): hoisted terms from nc, the others from the node's own record
+  for (int d = 0; d < nl; d++) {
+    const LevelArgs& a = t.lv[d];
+    OpGen g(a, "l" + std::to_string(d), "");
+    for (int tt = 0; tt < a.n_terms; tt++)
+      if (ncoff[d][tt] < 0) g.mark_term(tt);
+    s += "__device__ __forceinline__ u32 tmask" + std::to_string(d) + "(const TailJitArgs& a, const u32* w, const u32* nc) {\n";
+    s += g.loads("  ");
+    s += "  u32 m = " + hex(a.r >= 32 ? 0xffffffffu : ((1u << a.r) - 1u)) + ";\n";
+    for (int tt = 0; tt < a.n_terms; tt++) {
+      if (ncoff[d][tt] >= 0) {
+        s += term_mask_code(a, tt, cx[d], cm[d], "(nc + " + std::to_string(ncoff[d][tt]) + ")");
+      } else {
+        s += "  {\n    u32 lc[3];\n" + nc_code(a, tt, g, "lc", "    ");
+        s += term_mask_code(a, tt, cx[d], cm[d], "lc") + "  }\n";
+      }
+    }
+    s += "  return m;\n}\n";
+  }
+  auto child = [&](int d, const std::string& src, const std::string& dst, const std::string& ind) {
+    std::string c;
+    const int fw = t.lv[d].field_word, fs = t.lv[d].field_shift;
+    for (int w = 0; w < W; w++)
+      c += ind + dst + "[" + std::to_string(w) + "] = " + src + "[" + std::to_string(w) + "]" +
+           (w == fw && t.lv[d].r > 1 ? " | (cc << " + std::to_string(fs) + ")" : "") + ";\n";  // r == 1: no field bits
+    return c;
+  };
+  // ---- count: depth-first per frontier node
+  for (int d = nl - 1; d >= 0; d--) {
+    const std::string ds = std::to_string(d);
+    s += "__device__ __forceinline__ void cnt" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cnt) {\n";
+    s += "  u32 m = tmask" + ds + "(a, w, nc);\n  cnt[" + ds + "] += __popc(m);\n";
+    if (d + 1 < nl) {
+      s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
+      s += child(d, "w", "cw", "    ");
+      s += "    cnt" + std::to_string(d + 1) + "(a, cw, nc, cnt);\n  }\n";
+    }
+    s += "}\n";
+  }
+  s += "extern \"C\" __global__ void __launch_bounds__(256) atf_tail_count(const __grid_constant__ TailJitArgs a) {\n";
+  s += "  const int lane = threadIdx.x & 31;\n  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n";
+  s += "  for (u64 tile = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile < a.n_tiles; tile += nw) {\n";
+  s += "    const u64 nd = tile * 32 + lane;\n    u32 cnt[" + std::to_string(nl) + "] = {};\n";
+  s += "    if (nd < a.n_parents) {\n      u32 w[" + Ws + "];\n";
+  s += "      for (int i = 0; i < " + Ws + "; i++) w[i] = __ldg(a.parent_rec + nd * " + Ws + " + i);\n";
+  s += "      u32 nc[" + std::to_string(NC) + "];\n      tnc(a, w, nc);\n      cnt0(a, w, nc, cnt);\n    }\n";
+  for (int d = 0; d < nl; d++) {
+    const std::string ds = std::to_string(d);
+    s += "    { u32 v = cnt[" + ds + "];\n#pragma unroll\n      for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);\n";
+    s += "      if (lane == 0) a.tile_total[(u64)" + ds + " * a.n_tiles + tile] = v; }\n";
+  }
+  s += "  }\n}\n";
+  // ---- emit: chunk walk.  emit_d takes a chunk of <= CS_d nodes of level d - 1 (lane = node),
+  // evaluates their level-d masks, writes their CSR entries and appends their children (records +
+  // the frontier lane they descend from) to level d's shared-memory buffer, then walks those
+  // children in chunks of CS_{d+1}.  Chunks go in node order at every depth, so each level's
+  // output is its canonical order; a level's buffer is flushed to global memory as coalesced
+  // vectors only when the next chunk's children would not fit (and at the end of the tile).
+  // CS_d * r_d <= 256 keeps every buffer <= 256 records whatever r.  Per-warp shared memory:
+  // node constants [32][NC], then per level d: records [BC_d][W], frontier lanes [BC_d].
+  std::vector<int> CS(nl), BC(nl), off(nl + 1, 0), ooff(nl, 0);
+  for (int d = 0; d < nl; d++) {
+    CS[d] = std::max(1, std::min(32, 256 / t.lv[d].r));
+    BC[d] = std::max(256, CS[d] * t.lv[d].r);
+  }
+  off[0] = (4 * 32 * NC + 15) & ~15;
+  for (int d = 0; d < nl; d++) {
+    ooff[d] = off[d] + BC[d] * W * 4;
+    off[d + 1] = (ooff[d] + BC[d] + 15) & ~15;
+  }
+  const std::string WB = std::to_string(off[nl]), NCs = std::to_string(NC);
+  if (warp_bytes) *warp_bytes = off[nl];
+  const std::string V = W == 1 ? "u32" : (W == 2 ? "uint2" : "uint4"), VPR = std::to_string(W <= 4 ? 1 : 2);
+  for (int d = 0; d < nl; d++) {  // flush of level d
+    const std::string ds = std::to_string(d);
+    s += "__device__ __forceinline__ void flush" + ds + "(const TailJitArgs& a, u64* cur, u32* fill, unsigned char* wbuf, int lane) {\n";
+    s += "  const u32 n = fill[" + ds + "] * " + VPR + ";\n";
+    s += "  const " + V + "* src = reinterpret_cast<const " + V + "*>(wbuf + " + std::to_string(off[d]) + ");\n";
+    s += "  " + V + "* dst = reinterpret_cast<" + V + "*>(a.rec[" + ds + "] + cur[" + ds + "] * " + Ws + ");\n";
+    s += "#pragma unroll 4\n  for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
+    s += "  cur[" + ds + "] += fill[" + ds + "];\n  fill[" + ds + "] = 0;\n  __syncwarp();\n}\n";
+  }
+  for (int d = nl - 1; d >= 0; d--) {
+    const std::string ds = std::to_string(d);
+    s += "__device__ __forceinline__ void emit" + ds + "(const TailJitArgs& a, const u32* w, u32 org, bool valid, u64 gidx, "
+         "u64* cur, u32* fill, unsigned char* wbuf, int lane) {\n";
+    s += "  const u32* s_nc = reinterpret_cast<const u32*>(wbuf);\n";
+    s += "  u32 m = valid ? tmask" + ds + "(a, w, s_nc + org * " + NCs + ") : 0u;\n";
+    s += "  const u32 c = __popc(m);\n  u32 incl = c;\n";
+    s += "#pragma unroll\n  for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
+         "if (lane >= o) incl += y; }\n";
+    s += "  const u32 T = __shfl_sync(0xffffffffu, incl, 31);\n";
+    s += "  if (fill[" + ds + "] + T > " + std::to_string(BC[d]) + "u) flush" + ds + "(a, cur, fill, wbuf, lane);\n";
+    s += "  const u32 base = fill[" + ds + "];\n  u32 k = base + incl - c;\n";
+    s += "  if (valid) a.csr[" + ds + "][gidx] = cur[" + ds + "] + k;\n";
+    s += "  u32* buf = reinterpret_cast<u32*>(wbuf + " + std::to_string(off[d]) + ");\n";
+    s += "  unsigned char* obuf = wbuf + " + std::to_string(ooff[d]) + ";\n";
+    s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n";
+    s += child(d, "w", "(buf + k * " + Ws + ")", "    ");
+    s += "    obuf[k] = (unsigned char)org;\n    k++;\n  }\n  __syncwarp();\n";
+    s += "  fill[" + ds + "] = base + T;\n";
+    if (d + 1 < nl) {
+      const std::string cs = std::to_string(CS[d + 1]);
+      s += "  const u64 g0 = cur[" + ds + "] + base;\n";
+      s += "  for (u32 s0 = 0; s0 < T; s0 += " + cs + ") {\n    const bool v = lane < " + cs + " && s0 + lane < T;\n";
+      s += "    const u32 ix = base + s0 + (v ? lane : 0);\n    u32 cw[" + Ws + "];\n";
+      for (int w = 0; w < W; w++) s += "    cw[" + std::to_string(w) + "] = buf[ix * " + Ws + " + " + std::to_string(w) + "];\n";
+      s += "    emit" + std::to_string(d + 1) + "(a, cw, obuf[ix], v, g0 + s0 + lane, cur, fill, wbuf, lane);\n  }\n";
+    }
+    s += "}\n";
+  }
+  s += "extern \"C\" __global__ void __launch_bounds__(128) atf_tail_emit(const __grid_constant__ TailJitArgs a) {\n";
+  s += "  extern __shared__ __align__(16) unsigned char smem[];\n";
+  s += "  const int lane = threadIdx.x & 31;\n  unsigned char* wbuf = smem + (threadIdx.x >> 5) * " + WB + ";\n";
+  s += "  u32* s_nc = reinterpret_cast<u32*>(wbuf);\n";
+  s += "  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n  const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n";
+  s += "  if (gw == 0 && lane < " + std::to_string(nl) + ") {\n";
+  s += "    const u64 above = lane == 0 ? a.n_parents : a.tile_base[(u64)(lane - 1) * (a.n_tiles + 1) + a.n_tiles];\n";
+  s += "    a.csr[lane][above] = a.tile_base[(u64)lane * (a.n_tiles + 1) + a.n_tiles];\n  }\n";
+  s += "  for (u64 tile = gw; tile < a.n_tiles; tile += nw) {\n    u64 cur[" + std::to_string(nl) + "];\n    u32 fill[" +
+       std::to_string(nl) + "];\n";
+  for (int d = 0; d < nl; d++)
+    s += "    cur[" + std::to_string(d) + "] = a.tile_base[(u64)" + std::to_string(d) + " * (a.n_tiles + 1) + tile]; fill[" +
+         std::to_string(d) + "] = 0;\n";
+  s += "    const u64 nd0 = tile * 32;\n    const bool vl = nd0 + lane < a.n_parents;\n    u32 w[" + Ws + "];\n";
+  s += "    for (int i = 0; i < " + Ws + "; i++) w[i] = vl ? __ldg(a.parent_rec + (nd0 + lane) * " + Ws + " + i) : 0u;\n";
+  s += "    { u32 nc[" + NCs + "];\n      tnc(a, w, nc);\n      for (int i = 0; i < " + NCs + "; i++) s_nc[lane * " + NCs +
+       " + i] = nc[i]; }\n    __syncwarp();\n";
+  const std::string cs0 = std::to_string(CS[0]);
+  s += "    for (u32 s0 = 0; s0 < 32; s0 += " + cs0 + ") {\n";
+  s += "      const u32 src = s0 + (lane < " + cs0 + " ? lane : 0);\n      u32 cw[" + Ws + "];\n";
+  for (int w = 0; w < W; w++) s += "      cw[" + std::to_string(w) + "] = __shfl_sync(0xffffffffu, w[" + std::to_string(w) + "], src & 31);\n";
+  s += "      const bool v = lane < " + cs0 + " && s0 + lane < 32 && nd0 + s0 + lane < a.n_parents;\n";
+  s += "      emit0(a, cw, src & 31, v, nd0 + s0 + lane, cur, fill, wbuf, lane);\n    }\n";
+  for (int d = 0; d < nl; d++) s += "    flush" + std::to_string(d) + "(a, cur, fill, wbuf, lane);\n";
+  s += "  }\n}\n";
+  return s;
+}
+
+
+// ---------------------------------------------------------------- mid-width levels
+// A narrow-fast-style level (nf_ok: every conjunct an atom over ancestor values / constants /
+// ancestor products) with 32 < r <= kWideJitMax candidates: lane = frontier node, the
+// candidates in words of 32.  Per word, the first conjunct (the cheapest, host order) is
+// evaluated EXACTLY for every candidate with the candidate's magic / |value| as an immediate
+// (one IMAD + compare per pair, no item recomputation as in the warp-tile kernel's
+// superset filter); the other conjuncts run only on that word's survivors (table loads).
+// The per-node word masks stay in the warp's shared memory for the emit.  Output protocol =
+// expand_wtile's stash path (tile = 32 nodes: tile_total / tile_seg / stash segment claimed
+// by atomicAdd, tile-local CSR), so scan_kernel + level_emit_kernel finish the level.
+struct WideJitArgs {
+  const uint32_t* parent_rec;
+  uint64_t n_parents, n_tiles;
+  const int32_t* pv_range[kMaxSlots];
+  const uint32_t* pv_magic[kMaxSlots];
+  const int32_t* cand;
+  const uint32_t* cand_magic;
+  const uint32_t* cand_abs;
+  uint64_t* csr;
+  uint32_t* stash;
+  uint64_t stash_cap;
+  unsigned long long* stash_top;
+  uint32_t* tile_total;
+  unsigned long long* tile_seg;
+  unsigned int* overflow_flag;
+};
+
+const char* kWidePrelude = R"(
+struct WideJitArgs { const u32* parent_rec; u64 n_parents, n_tiles; const i32* pv_range[24]; const u32* pv_magic[24];
+                     const i32* cand; const u32* cand_magic; const u32* cand_abs; u64* csr; u32* stash; u64 stash_cap;
+                     u64* stash_top; u32* tile_total; u64* tile_seg; u32* overflow_flag; };
+)";
+
+constexpr int kWideStageWords = 1024;  // u32 words of records staged per warp for coalesced stash writes
+
+std::string gen_wide_source(const LevelArgs& a, int W, const std::vector<int32_t>& cx, const std::vector<uint32_t>& cm) {
+  const int r = a.r;
+  if (!a.nf_ok || r <= 32 || r > kWideJitMax || (int)cx.size() != r || a.n_gates) return "";
+  const int NWD = (r + 31) / 32;
+  const std::string Ws = std::to_string(W);
+  std::string s = kPrelude;
+  s += kWidePrelude;
+  const int stage = kWideStageWords / W;           // records
+  const int stride = NWD * 32 + kWideStageWords;   // u32 per warp
+  s += "extern \"C\" __global__ void __launch_bounds__(256) atf_wide_jit(const __grid_constant__ WideJitArgs a) {\n";
+  s += "  extern __shared__ __align__(16) u32 smem[];\n  const int lane = threadIdx.x & 31;\n";
+  s += "  u32* s_m = smem + (threadIdx.x >> 5) * " + std::to_string(stride) + ";\n";
+  s += "  u32* s_st = s_m + " + std::to_string(NWD * 32) + ";\n";
+  s += "  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n";
+  s += "  for (u64 tile = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile < a.n_tiles; tile += nw) {\n";
+  s += "    const u64 nd = tile * 32 + lane;\n    const bool valid = nd < a.n_parents;\n    u32 w[" + Ws + "];\n";
+  if (a.level == 0) s += "    for (int i = 0; i < " + Ws + "; i++) w[i] = 0u;\n";
+  else s += "    for (int i = 0; i < " + Ws + "; i++) w[i] = valid ? __ldg(a.parent_rec + nd * " + Ws + " + i) : 0u;\n";
+  // operands
+  std::vector<int> need_v(a.n_pv, 0), need_m(a.n_pv, 0);
+  auto mark = [&](const NfOp& o, bool mag) {
+    if (o.kind == NF_PV) { need_v[o.s1] = 1; if (mag) need_m[o.s1] = 1; }
+    if (o.kind == NF_PROD) { need_v[o.s1] = 1; need_v[o.s2] = 1; }
+  };
+  for (int t = 0; t < a.n_terms; t++) {
+    const Term& T = a.terms[t];
+    mark(a.nf_op[t][0], T.kind == T_MULX || T.kind == T_DIVPROD);
+    if (T.kind == T_DIVPROD || T.kind == T_QDIV || T.kind == T_CMP) mark(a.nf_op[t][1], false);
+  }
+  for (int p = 0; p < a.n_pv; p++) {
+    if (!need_v[p]) continue;
+    const std::string ps = std::to_string(p);
+    const uint32_t bits = (uint32_t)a.pv_bits[p];
+    std::string pos = bits ? "((w[" + std::to_string(a.pv_word[p]) + "] >> " + std::to_string(a.pv_shift[p]) + ") & " +
+                                 hex(bits >= 32 ? 0xffffffffu : ((1u << bits) - 1u)) + ")"
+                           : std::string("0u");
+    s += "    const u32 p" + ps + " = " + pos + ";\n";
+    s += "    const i64 v" + ps + " = (i64)__ldg(a.pv_range[" + ps + "] + p" + ps + ");\n";
+    if (need_m[p]) s += "    const u32 g" + ps + " = __ldg(a.pv_magic[" + ps + "] + p" + ps + ");\n";
+  }
+  auto sval = [&](const NfOp& o) -> std::string {
+    if (o.kind == NF_CONST) return "(i64)" + std::to_string(o.c) + "ll";
+    if (o.kind == NF_PV) return "v" + std::to_string(o.s1);
+    return "(v" + std::to_string(o.s1) + " * v" + std::to_string(o.s2) + ")";
+  };
+  auto magic = [&](const NfOp& o, const std::string& absname) -> std::string {
+    if (o.kind == NF_CONST) return hex(o.cm);
+    if (o.kind == NF_PV) return "(" + absname + " == 0u ? 0u : g" + std::to_string(o.s1) + ")";
+    return "(" + absname + " > 1u ? 0xffffffffu / " + absname + " + 1u : 0u)";
+  };
+  // per-term node operands (and node gate from DIVPROD / MULX: the node accepts nothing)
+  s += "    bool alive = valid;\n";
+  for (int t = 0; t < a.n_terms; t++) {
+    const Term& T = a.terms[t];
+    const NfOp& oa = a.nf_op[t][0];
+    const NfOp& ob = a.nf_op[t][1];
+    const std::string ts = std::to_string(t);
+    switch (T.kind) {
+      case T_DIVX: s += "    const u32 n" + ts + " = uabs(" + sval(oa) + ");\n"; break;
+      case T_DIVPROD:
+        s += "    u32 n" + ts + ";\n    { const u32 av = uabs(" + sval(oa) + "), bv = uabs(" + sval(ob) + ");\n";
+        s += "      const u32 ma = " + magic(oa, "av") + ";\n";
+        s += "      n" + ts + " = av == 1u ? bv : __umulhi(bv, ma);\n";
+        s += "      if (av == 0u || n" + ts + " * av != bv) alive = false; }\n";
+        break;
+      case T_MULX:
+        s += "    const u32 d" + ts + " = uabs(" + sval(oa) + ");\n";
+        s += "    const u32 md" + ts + " = " + magic(oa, "d" + ts) + ", mq" + ts + " = md" + ts + " - 1u;\n";
+        s += "    if (d" + ts + " == 0u) alive = false;\n";
+        break;
+      case T_QDIV:
+        s += "    const u32 num" + ts + " = uabs(" + sval(oa) + "), nb" + ts + " = uabs(" + sval(ob) + ");\n";
+        break;
+      case T_CMP:
+        if (T.rel < R_EQ || T.rel > R_GE) return "";
+        s += "    const i32 A" + ts + " = (i32)" + sval(oa) + ", B" + ts + " = (i32)" + sval(ob) + ";\n";
+        break;
+      default: return "";
+    }
+  }
+  static const char* rel[] = {"==", "!=", "<", "<=", ">", ">="};
+  if (a.n_terms > 0 && a.terms[0].kind == T_QDIV) return "";  // a quotient test is never the cheapest conjunct
+  s += "    u32 cnt = 0;\n";
+  // first conjunct: divisibility tests (x | n, d | x) in groups of 4 candidates, a superset
+  // test per group (min of the 4 magic products, VIMNMX3) whose survivors are re-tested exactly
+  // below; comparisons exactly per candidate
+  const bool grouped = a.n_terms > 0 && (a.terms[0].kind == T_DIVX || a.terms[0].kind == T_DIVPROD ||
+                                         a.terms[0].kind == T_MULX);
+  for (int j = 0; j < NWD; j++) {
+    s += "    {  // candidates " + std::to_string(32 * j) + ".." + std::to_string(std::min(r, 32 * j + 32) - 1) + "\n";
+    s += "      u32 mw = 0u;\n";
+    if (grouped) {
+      const bool mulx = a.terms[0].kind == T_MULX;
+      for (int c0 = 0; c0 < 32 && 32 * j + c0 < r; c0 += 4) {
+        const int nc = std::min(4, r - (32 * j + c0));
+        std::vector<std::string> pr;
+        for (int c = c0; c < c0 + nc; c++) {
+          const int ci = 32 * j + c;
+          const uint32_t ax = cx[ci] < 0 ? 0u - (uint32_t)cx[ci] : (uint32_t)cx[ci];
+          pr.push_back(mulx ? hex(ax) + " * md0" : "n0 * " + hex(cm[ci]));
+        }
+        std::string q = pr[0];
+        if (pr.size() == 2) q = "min(" + pr[0] + ", " + pr[1] + ")";
+        if (pr.size() == 3) q = "min(min(" + pr[0] + ", " + pr[1] + "), " + pr[2] + ")";
+        if (pr.size() == 4) q = "min(min(" + pr[0] + ", " + pr[1] + "), min(" + pr[2] + ", " + pr[3] + "))";
+        s += "      { const u32 q = " + q + "; if (q " + (mulx ? "<= mq0" : "< 0x10000u") + ") mw |= " +
+             hex(((1u << nc) - 1u) << c0) + "; }\n";
+      }
+    } else {
+      for (int c = 0; c < 32 && 32 * j + c < r; c++) {
+        const int ci = 32 * j + c;
+        const std::string sh = " << " + std::to_string(c) + ";\n";
+        if (a.n_terms == 0) { s += "      mw |= 1u" + sh; continue; }
+        const Term& T = a.terms[0];
+        s += "      mw |= (u32)(A0 * " + std::to_string(cx[ci]) + " " + rel[T.rel - R_EQ] + " B0)" + sh;
+      }
+    }
+    if (grouped || a.n_terms > 1) {
+      s += "      u32 sv = mw;\n      while (sv) {\n        const int c = __ffs(sv) - 1;\n        sv &= sv - 1;\n";
+      s += "        const int ci = " + std::to_string(32 * j) + " + c;\n        bool ok = true;\n";
+      for (int t = grouped ? 0 : 1; t < a.n_terms; t++) {
+        const Term& T = a.terms[t];
+        const std::string ts = std::to_string(t);
+        switch (T.kind) {
+          case T_DIVX: case T_DIVPROD:
+            s += "        { const u32 mg = __ldg(a.cand_magic + ci); ok = ok && mg != 0x10000u && n" + ts + " * mg < 0x10000u; }\n";
+            break;
+          case T_MULX: s += "        ok = ok && __ldg(a.cand_abs + ci) * md" + ts + " <= mq" + ts + ";\n"; break;
+          case T_QDIV:
+            s += "        if (ok) { const u32 ax = __ldg(a.cand_abs + ci);\n";
+            s += "          const u32 q = ax == 1u ? num" + ts + " : __umulhi(num" + ts + ", __ldg(a.cand_magic + ci));\n";
+            s += "          ok = ax != 0u && q != 0u && divisible16(nb" + ts + ", q); }\n";
+            break;
+          default:
+            s += "        ok = ok && (A" + ts + " * __ldg(a.cand + ci) " + rel[T.rel - R_EQ] + " B" + ts + ");\n";
+        }
+      }
+      s += "        if (!ok) mw &= ~(1u << c);\n      }\n";
+    }
+    s += "      if (!alive) mw = 0u;\n      s_m[" + std::to_string(32 * j) + " + lane] = mw;\n      cnt += __popc(mw);\n    }\n";
+  }
+  // tile scan, stash segment, CSR
+  s += "    u32 incl = cnt;\n#pragma unroll\n    for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); if (lane >= o) incl += y; }\n";
+  s += "    const u32 total = __shfl_sync(0xffffffffu, incl, 31);\n    u32 k = incl - cnt;\n";
+  s += "    u64 sgb = 0;\n    if (lane == 0) {\n      sgb = total ? atomicAdd(a.stash_top, (u64)total) : 0ull;\n";
+  s += "      if (total && sgb + total > a.stash_cap) atomicOr(a.overflow_flag, 1u);\n";
+  s += "      a.tile_total[tile] = total;\n      a.tile_seg[tile] = sgb;\n    }\n";
+  s += "    sgb = __shfl_sync(0xffffffffu, sgb, 0);\n    if (valid) a.csr[nd] = k;\n";
+  s += "    const bool staged = total <= " + std::to_string(stage) + "u;\n";
+  s += "    __syncwarp();\n";
+  const int fw = a.field_word, fs = a.field_shift;
+  s += "    for (int j = 0; j < " + std::to_string(NWD) + "; j++) {\n      u32 mw = s_m[j * 32 + lane];\n";
+  s += "      while (mw) {\n        const u32 c = __ffs(mw) - 1;\n        mw &= mw - 1;\n        const u32 pos = (u32)j * 32u + c;\n";
+  s += "        if (staged) {\n";
+  for (int wd = 0; wd < W; wd++)
+    s += "          s_st[k * " + Ws + " + " + std::to_string(wd) + "] = w[" + std::to_string(wd) + "]" +
+         (wd == fw && r > 1 ? " | (pos << " + std::to_string(fs) + ")" : "") + ";\n";
+  s += "        } else if (sgb + k < a.stash_cap) {\n";
+  for (int wd = 0; wd < W; wd++)
+    s += "          a.stash[(sgb + k) * " + Ws + " + " + std::to_string(wd) + "] = w[" + std::to_string(wd) + "]" +
+         (wd == fw && r > 1 ? " | (pos << " + std::to_string(fs) + ")" : "") + ";\n";
+  s += "        }\n        k++;\n      }\n    }\n";
+  s += "    if (staged && sgb + total <= a.stash_cap) {\n      __syncwarp();\n";
+  s += "      for (u32 v = lane; v < total * " + Ws + "u; v += 32) a.stash[sgb * " + Ws + " + v] = s_st[v];\n    }\n";
+  s += "    __syncwarp();\n  }\n}\n";
   return s;
 }
 
@@ -502,7 +817,7 @@ cudaKernel_t compile(const std::string& src, const char* name = "atf_nfast_jit")
 
 struct TailJit {
   cudaKernel_t count = nullptr, emit = nullptr;
-  int warp_bytes = 0, per_sm = 0;
+  int warp_bytes = 0, per_sm = 0, per_sm_count = 0;
 };
 std::unordered_map<std::string, TailJit> g_tails;  // source -> kernels (under g_mu)
 
@@ -553,13 +868,16 @@ int jit_nfast_launch(void* kernel, const LevelArgs& a, void* stream) {
 
 // ---- fused narrow tail: specialised count + emit kernels (nullptr: use the generic ones)
 std::string jit_tail_source(const TailArgs& t, int words, const std::vector<std::vector<int32_t>>& cand_values,
-                            const std::vector<std::vector<uint32_t>>& cand_magics) {
-  return gen_tail_source(t, words, cand_values, cand_magics);
+                            const std::vector<std::vector<uint32_t>>& cand_magics, int k0,
+                            const std::vector<std::vector<int>>& pv_level) {
+  return gen_tail_source(t, words, cand_values, cand_magics, k0, pv_level, nullptr);
 }
 
 void* jit_tail_kernels(const TailArgs& t, int words, const std::vector<std::vector<int32_t>>& cand_values,
-                       const std::vector<std::vector<uint32_t>>& cand_magics) {
-  const std::string src = gen_tail_source(t, words, cand_values, cand_magics);
+                       const std::vector<std::vector<uint32_t>>& cand_magics, int k0,
+                       const std::vector<std::vector<int>>& pv_level) {
+  int wb = 0;
+  const std::string src = gen_tail_source(t, words, cand_values, cand_magics, k0, pv_level, &wb);
   if (src.empty()) return nullptr;
   {
     std::lock_guard<std::mutex> lk(g_mu);
@@ -569,23 +887,20 @@ void* jit_tail_kernels(const TailArgs& t, int words, const std::vector<std::vect
   TailJit tj;
   tj.count = compile(src, "atf_tail_count");
   tj.emit = compile(src, "atf_tail_emit");
-  int wb = 0;
-  for (int d = 0; d < t.nl; d++) wb += (32 * t.lv[d].r * words * 4 + 15) & ~15;
   tj.warp_bytes = wb;
   if (tj.count && tj.emit) {
     const int smem = 4 * wb;
-    bool ok = true;
-    for (cudaKernel_t k : {tj.count, tj.emit}) {
-      if (smem > 48 * 1024 &&
-          cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) != cudaSuccess)
-        ok = false;
-    }
-    int per_sm = 0;
-    if (ok && cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void*)tj.emit, 128, smem) != cudaSuccess)
+    bool ok = !(smem > 48 * 1024 &&
+                cudaFuncSetAttribute((const void*)tj.emit, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) !=
+                    cudaSuccess);
+    int per_sm = 0, per_sm_c = 0;
+    if (ok && (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void*)tj.emit, 128, smem) != cudaSuccess ||
+               cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm_c, (const void*)tj.count, 256, 0) != cudaSuccess))
       ok = false;
     cudaGetLastError();
     tj.per_sm = per_sm;
-    if (!ok || per_sm < 1) tj.count = tj.emit = nullptr;
+    tj.per_sm_count = per_sm_c;
+    if (!ok || per_sm < 1 || per_sm_c < 1) tj.count = tj.emit = nullptr;
   } else {
     tj.count = tj.emit = nullptr;
   }
@@ -621,14 +936,80 @@ int jit_tail_launch(void* handle, const TailArgs& t, bool emit, void* stream) {
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   }
-  uint64_t grid = (uint64_t)sms * tj.per_sm;
-  const uint64_t need = (t.n_tiles + 3) / 4;  // 4 warps per CTA, one warp tile each
+  const int threads = emit ? 128 : 256;  // one warp tile (32 frontier nodes) per warp
+  uint64_t grid = (uint64_t)sms * (emit ? tj.per_sm : tj.per_sm_count);
+  const uint64_t need = (t.n_tiles + threads / 32 - 1) / (threads / 32);
   if (grid > need) grid = need;
   if (grid < 1) grid = 1;
   void* args[] = {&j};
-  cudaError_t e = cudaLaunchKernel((const void*)(emit ? tj.emit : tj.count), dim3((unsigned)grid), dim3(128), args,
-                                   (size_t)(4 * tj.warp_bytes), (cudaStream_t)stream);
+  cudaError_t e = cudaLaunchKernel((const void*)(emit ? tj.emit : tj.count), dim3((unsigned)grid), dim3(threads), args,
+                                   emit ? (size_t)(4 * tj.warp_bytes) : 0, (cudaStream_t)stream);
   return (int)e;
+}
+
+// ---- mid-width levels: specialised exact-mask kernel (nullptr: use the warp-tile kernel)
+std::string jit_wide_source(const LevelArgs& a, int words, const std::vector<int32_t>& cand_values,
+                            const std::vector<uint32_t>& cand_magics) {
+  return gen_wide_source(a, words, cand_values, cand_magics);
+}
+
+void* jit_wide_kernel(const LevelArgs& a, int words, const std::vector<int32_t>& cand_values,
+                      const std::vector<uint32_t>& cand_magics) {
+  const std::string src = gen_wide_source(a, words, cand_values, cand_magics);
+  if (src.empty()) return nullptr;
+  cudaKernel_t k = compile(src, "atf_wide_jit");
+  if (!k) return nullptr;
+  const int smem = jit_wide_smem(a.r, words);
+  if (smem > 48 * 1024 && cudaFuncSetAttribute((const void*)k, cudaFuncAttributeMaxDynamicSharedMemorySize, smem) !=
+                              cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return (void*)k;
+}
+
+int jit_wide_smem(int r, int words) { (void)words; return 8 * 4 * (((r + 31) / 32) * 32 + kWideStageWords); }
+
+int jit_wide_launch(void* kernel, const LevelArgs& a, int words, void* stream) {
+  WideJitArgs j;
+  std::memset(&j, 0, sizeof j);
+  j.parent_rec = a.parent_rec;
+  j.n_parents = a.n_parents;
+  j.n_tiles = a.n_tiles;
+  for (int i = 0; i < a.n_pv; i++) {
+    j.pv_range[i] = a.pv_range[i];
+    j.pv_magic[i] = a.pv_magic[i];
+  }
+  j.cand = a.cand;
+  j.cand_magic = a.cand_magic;
+  j.cand_abs = a.cand_abs;
+  j.csr = a.csr;
+  j.stash = a.stash;
+  j.stash_cap = a.stash_cap;
+  j.stash_top = a.stash_top;
+  j.tile_total = a.tile_total;
+  j.tile_seg = a.tile_seg;
+  j.overflow_flag = a.overflow_flag;
+  const int smem = jit_wide_smem(a.r, words);
+  int per_sm = 0;
+  if (cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, (const void*)kernel, 256, smem) != cudaSuccess ||
+      per_sm < 1) {
+    cudaGetLastError();
+    return (int)cudaErrorInvalidConfiguration;
+  }
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  uint64_t grid = (uint64_t)sms * per_sm;
+  const uint64_t need = (a.n_tiles + 7) / 8;
+  if (grid > need) grid = need;
+  if (grid < 1) grid = 1;
+  void* args[] = {&j};
+  return (int)cudaLaunchKernel((const void*)kernel, dim3((unsigned)grid), dim3(256), args, (size_t)smem,
+                               (cudaStream_t)stream);
 }
 
 }  // namespace atf

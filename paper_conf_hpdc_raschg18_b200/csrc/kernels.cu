@@ -269,6 +269,58 @@ static int launch_decode(const DecodeArgs& a, const uint64_t* idx, const uint64_
   return (int)cudaGetLastError();
 }
 
+// Indices beyond 2^64 (S >= 2^64, P:280 mentions spaces of ~10^19): u128 index = hi * 2^64 + lo,
+// either per row (idx_lo / idx_hi) or the consecutive range first + i (exhaustive search).
+// Mixed radix in u128 (group 0 most significant), then the same leaf gather as decode_kernel.
+__global__ void decode128_kernel(const __grid_constant__ DecodeArgs a, const uint64_t* __restrict__ idx_lo,
+                                 const uint64_t* __restrict__ idx_hi, uint64_t first_lo, uint64_t first_hi, int64_t n,
+                                 int32_t* __restrict__ out, int64_t ld, unsigned int* bad, uint64_t S_lo, uint64_t S_hi) {
+  typedef unsigned __int128 u128;
+  const u128 S = ((u128)S_hi << 64) | S_lo;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
+    u128 rem = idx_lo ? (((u128)__ldg(idx_hi + i) << 64) | __ldg(idx_lo + i))
+                      : ((((u128)first_hi << 64) | first_lo) + (u128)i);
+    if (rem >= S) {
+      for (int p = 0; p < a.n_params; p++) out[(int64_t)p * ld + i] = INT32_MIN;
+      atomicOr(bad, 1u);
+      continue;
+    }
+    for (int g = a.n_groups - 1; g >= 0; g--) {
+      const uint64_t sz = a.gsize[g];
+      const u128 q = rem / sz;
+      const uint64_t d = (uint64_t)(rem - q * sz);
+      rem = q;
+      const int W = a.words[g];
+      const uint32_t* rp = a.leaves[g] + d * (uint64_t)W;
+      uint32_t rec[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+      for (int w = 0; w < W; w++) rec[w] = __ldg(rp + w);
+      for (int l = a.lvl_begin[g]; l < a.lvl_begin[g + 1]; l++) {
+        const int lw = a.lvl_word[l];
+        uint32_t word = rec[0];
+#pragma unroll
+        for (int w = 1; w < 8; w++)
+          if (lw == w) word = rec[w];
+        const uint32_t bits = (uint32_t)a.lvl_bits[l];
+        const uint32_t pos = bits ? (word >> a.lvl_shift[l]) & ((1u << bits) - 1u) : 0u;
+        out[(int64_t)a.lvl_param[l] * ld + i] = __ldg(a.lvl_range[l] + pos);
+      }
+    }
+  }
+}
+
+int launch_decode128(const DecodeArgs& a, const uint64_t* idx_lo, const uint64_t* idx_hi, uint64_t first_lo,
+                     uint64_t first_hi, int64_t n, int32_t* out, int64_t ld, unsigned int* bad, uint64_t S_lo,
+                     uint64_t S_hi, void* stream) {
+  if (n <= 0) return 0;
+  const int sms = cached_sm_count();
+  int64_t blocks = (n + 255) / 256;
+  const int64_t cap = (int64_t)sms * 8;
+  if (blocks > cap) blocks = cap;
+  decode128_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, idx_lo, idx_hi, first_lo, first_hi, n, out,
+                                                                       ld, bad, S_lo, S_hi);
+  return (int)cudaGetLastError();
+}
+
 int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out, int64_t ld,
                           unsigned int* bad, void* stream) {
   return launch_decode(a, idx, nullptr, n, out, ld, bad, stream);

@@ -205,6 +205,31 @@ class Space:
         L.check(L.atf_space_decode_indices(self._h, idx.data_ptr(), n, out.data_ptr(), out.stride(0), sp), self._h)
         return out
 
+    def decode_range(self, first: int, n: int, out=None, stream=None):
+        """The n consecutive indices first, first + 1, ... (any S, u128 in the library) ->
+        int32 tensor [P, n]."""
+        import torch
+        P = len(self.names)
+        if out is None:
+            out = torch.empty((P, n), dtype=torch.int32, device=torch.device("cuda", self._device))
+        sp = stream.cuda_stream if stream is not None else None
+        L.check(L.atf_space_decode_range(self._h, first & ((1 << 64) - 1), first >> 64, n, out.data_ptr(),
+                                         out.stride(0), sp), self._h)
+        return out
+
+    def decode128(self, idx_lo, idx_hi, out=None, stream=None):
+        """u128 indices hi * 2^64 + lo (CUDA int64 tensors holding the u64 halves) -> int32 [P, n]."""
+        import torch
+        n = idx_lo.numel()
+        P = len(self.names)
+        if out is None:
+            out = torch.empty((P, n), dtype=torch.int32, device=idx_lo.device)
+        idx_lo, idx_hi = idx_lo.contiguous(), idx_hi.contiguous()
+        sp = stream.cuda_stream if stream is not None else None
+        L.check(L.atf_space_decode_indices128(self._h, idx_lo.data_ptr(), idx_hi.data_ptr(), n, out.data_ptr(),
+                                              out.stride(0), sp), self._h)
+        return out
+
     def decode_digits(self, digits, out=None, stream=None):
         """digits: CUDA tensor [G, n] of per-group indices -> int32 tensor [P, n]."""
         import torch

@@ -259,6 +259,8 @@ def test_jit_level_sources_compile_for_sm100a(L, tmp_path):
     # fused narrow tails: C2's VWMD/VWND, C3-IS2's KWI/VWM/VWN, C3-IS4's VWM/VWN
     assert ("C2_xgemm_direct_256", 0, 6) in tails and ("C3_xgemm_IS2", 0, 7) in tails
     assert ("C3_xgemm_IS4", 0, 8) in tails
+    # mid-width levels (C2's WGD..KWID, C3's NWG / NDIMC / NDIMB, r = 256..576): exact-mask kernels
+    assert sum("atf_wide_jit" in x for x in srcs) >= 8
     # one translation unit per source (kernel names collide), compiled in parallel
     procs = []
     for i, src in enumerate(srcs):

@@ -185,19 +185,6 @@ def test_small_specs_generic_tail(Space, name):
     _check_against_oracle(Space, SMALL[name](), no_jit=True)
 
 
-@pytest.mark.parametrize("name", ["C5-300x4", "C5-4096x3", "C2-256", "C3-IS1", "C3-12x30x8"])
-def test_small_specs_in_place_wtile(Space, name):
-    """ATF_FLAG_INPLACE: every warp-tile level written in place behind the deferred look-back."""
-    from paper_conf_hpdc_raschg18_b200 import _lib as L
-    _check_against_oracle(Space, SMALL[name](), extra_flags=L.ATF_FLAG_INPLACE)
-
-
-@pytest.mark.parametrize("seed", range(0, 40, 4))
-def test_fuzz_wide_specs_in_place_wtile(Space, seed):
-    from paper_conf_hpdc_raschg18_b200 import _lib as L
-    _check_against_oracle(Space, A.random_wide_spec(seed), extra_flags=L.ATF_FLAG_INPLACE)
-
-
 @pytest.mark.parametrize("seed", range(0, 80, 7))
 def test_fuzz_specs_without_tail(Space, seed):
     from paper_conf_hpdc_raschg18_b200 import _lib as L
@@ -653,3 +640,125 @@ def test_segment_bounds_skip_work_not_results(Space):
         g0 = [x for x in st if x["group"] == 0]
         assert g0[-1]["pairs"] < g0[-1]["evals"] // 2
         assert sp.level_sizes(0) == cf.piltz_D(4096, 4)
+
+
+# ---------------------------------------------------------------- u128 indices (S >= 2^64)
+def _big_spec():
+    """Six independent groups (x_i in [1,3000], y_i | x_i): S = (sum_{n<=3000} tau(n))^6 ~ 2^88."""
+    s = A.Spec("six_divisor_groups")
+    for i in range(6):
+        s.add(f"x{i}", A.interval(1, 3000))
+        s.add(f"y{i}", A.interval(1, 3000), A.divides(s.P(f"x{i}")))
+    return s
+
+
+def test_decode_u128_indices_against_oracle_leaves(Space):
+    """decode_range / decode_indices128 (P:229-231 index access, P:280 spaces beyond 2^64):
+    index -> mixed-radix digits (group 0 most significant, reading #11) computed here in Python
+    integers -> the oracle's leaf rows of every group, element by element."""
+    spec = _big_spec()
+    ref = orc.info(spec, threads=8)
+    sizes = [g["size"] for g in ref["groups"]]
+    S = int(ref["S"])
+    assert S >= 1 << 64
+    leaves = [orc.leaves(spec, g, 2) for g in range(6)]
+
+    def want(indices):
+        rows = []
+        for i in indices:
+            dig, rem = [], i
+            for z in reversed(sizes):
+                dig.append(rem % z)
+                rem //= z
+            dig.reverse()
+            rows.append([int(v) for g in range(6) for v in leaves[g][dig[g]]])
+        return np.array(rows, dtype=np.int32).T
+    gen = np.random.default_rng(5)
+    with Space(spec) as sp:
+        sp.generate()
+        assert sp.size() == S
+        for first in (0, S // 3, (1 << 64) - 7, S - 50):
+            got = sp.decode_range(first, 50).cpu().numpy()
+            assert np.array_equal(got, want(range(first, first + 50))), first
+        idx = [int(gen.integers(0, 1 << 62)) * (1 << 26) % S for _ in range(2000)] + [S - 1, 0]
+        lo = torch.tensor([((i & ((1 << 64) - 1)) ^ (1 << 63)) - (1 << 63) for i in idx], dtype=torch.int64).cuda()
+        hi = torch.tensor([i >> 64 for i in idx], dtype=torch.int64).cuda()
+        assert np.array_equal(sp.decode128(lo, hi).cpu().numpy(), want(idx))
+        from paper_conf_hpdc_raschg18_b200 import AtfError
+        with pytest.raises(AtfError):
+            sp.decode_range(S - 2, 4)
+
+
+def test_exhaustive_search_beyond_2_64(Space):
+    """ExhaustiveSearch walks any space in index order through decode_range."""
+    from paper_conf_hpdc_raschg18_b200 import explore
+    spec = _big_spec()
+    with Space(spec) as sp:
+        sp.generate()
+        t = explore.ExhaustiveSearch()
+        t.initialize(sp)
+        t.next = sp.size() - 10
+        a = t.get_next_configs(4)
+        b = t.get_next_configs(100)
+        assert a.shape[1] == 4 and b.shape[1] == 6
+        assert torch.equal(torch.cat([a, b], 1), sp.decode_range(sp.size() - 10, 10))
+
+
+# ---------------------------------------------------------------- allocation failure (fault injection)
+def test_allocator_failure_is_reported_and_space_destroys_cleanly(Space):
+    """SURVEY.md §5 failure detection: the device allocator hook returns NULL at the k-th request
+    (k = 0, 1, ... up to every allocation a generation makes).  generate must return ATF_ERR_OOM
+    (never crash or hang), destroy must free every block that was handed out, and a later
+    generation of the same spec with a working allocator is still exact."""
+    import ctypes as C
+    from paper_conf_hpdc_raschg18_b200 import _lib as LL
+    from paper_conf_hpdc_raschg18_b200.space import _range_struct
+    spec = A.c3_xgemm((12, 30, 8))
+    ref = int(orc.info(spec)["S"])
+    stream = torch.cuda.current_stream()
+
+    def run(fail_at):
+        live, count = {}, [0]
+
+        def _alloc(nbytes, _st, _ctx):
+            count[0] += 1
+            if count[0] - 1 == fail_at:
+                return None
+            t = torch.empty(int(nbytes), dtype=torch.uint8, device="cuda")
+            live[t.data_ptr()] = t
+            return t.data_ptr()
+
+        def _free(ptr, _n, _st, _ctx):
+            assert ptr in live, "free of a block the hook never handed out"
+            live.pop(ptr)
+
+        acb, fcb = LL.ALLOC_FN(_alloc), LL.FREE_FN(_free)
+        opts = LL.atf_space_opts(0, stream.cuda_stream, acb, fcb, None, 0)
+        h = C.c_void_p()
+        LL.check(LL.atf_space_create(C.byref(opts), C.byref(h)))
+        keep = []
+        for p in spec.params:
+            rs, k = _range_struct(p.range)
+            keep.append(k)
+            pid = C.c_int32()
+            LL.check(LL.atf_space_add_param(h, p.name.encode(), C.byref(rs), C.byref(pid)), h)
+            for code in p.constraints:
+                arr = (C.c_int32 * len(code))(*code)
+                LL.check(LL.atf_space_add_constraint(h, pid.value, arr, len(code)), h)
+        st = LL.atf_space_generate(h)
+        S = None
+        if st == 0:
+            lo, hi = C.c_uint64(), C.c_uint64()
+            LL.check(LL.atf_space_size(h, C.byref(lo), C.byref(hi)), h)
+            S = lo.value
+        LL.atf_space_destroy(h)
+        torch.cuda.synchronize()
+        assert not live, f"{len(live)} blocks leaked (fail_at={fail_at})"
+        return st, S, count[0]
+
+    st, S, total = run(-1)
+    assert st == 0 and S == ref and total >= 3
+    for k in range(total):
+        st, S, _ = run(k)
+        assert st == -2, (k, st)          # ATF_ERR_OOM
+    assert run(-1)[:2] == (0, ref)
