@@ -201,6 +201,22 @@ atf_status atf_space_generate_shard(atf_space* s, int32_t rank, int32_t world, i
 atf_status atf_space_finalize_shard(atf_space* s, const int64_t* h_all_counts, int32_t world,
                                     int32_t n);
 
+/* Multi-GPU, balanced per level: called by every rank
+ * (one process per GPU, or several spaces of one process).  Every level is redistributed: rank
+ * r expands the parents [r F / N, (r + 1) F / N) of the previous level (F = its global size),
+ * so each rank evaluates f_{k-1} r_k / N candidate pairs per level however unbalanced the tree.
+ * After each level round the library calls `allgather` once: it must copy `bytes` from `send`
+ * (host memory) of every rank into recv + rank * bytes on every rank and return 0 (e.g.
+ * torch.distributed.all_gather_into_tensor over NCCL).  The record holds the level counts and
+ * where the new level's records live; the next parent slice is then copied from the owning ranks
+ * (CUDA IPC over NVLink / NVSwitch; plain device pointers between spaces of one process).  In
+ * this mode the space allocates its arenas with cudaMalloc (exportable), not the allocator hooks.
+ * -> state FINAL_SHARD: size / group_size / level_size global-local as after finalize_shard;
+ * level_view gives this rank's slice of every level (offset, csr_offset).  Every rank must call
+ * with the same spec; errors are local (a failing rank makes the others fail in the callback). */
+typedef int (*atf_allgather_fn)(const void* send, void* recv, size_t bytes, void* ctx);
+atf_status atf_space_generate_dist(atf_space* s, int32_t rank, int32_t world, atf_allgather_fn allgather, void* ctx);
+
 /* ---- results (state GENERATED) ---------------------------------------------------- */
 
 /* S = prod_g |G_g| as u128: *lo = low 64 bits, *hi = high 64 bits. */
@@ -224,6 +240,10 @@ typedef struct {
   int32_t words;
   int32_t param;     /* parameter id of level k */
   int32_t field_word, field_shift, field_bits;
+  uint64_t csr_offset;  /* global index of the level-k node whose entry is csr[0]          */
+  uint64_t csr_nodes;   /* level-k nodes the csr array covers (csr has csr_nodes + 1 entries;
+                           = n_nodes / offset except after atf_space_generate_dist, where a
+                           rank's CSR covers the parent slice it expanded)                   */
 } atf_level_view;
 atf_status atf_space_level_view(const atf_space* s, int32_t g, int32_t k, atf_level_view* out);
 

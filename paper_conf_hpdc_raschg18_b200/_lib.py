@@ -36,6 +36,7 @@ class atf_range(C.Structure):
 
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
 FREE_FN = C.CFUNCTYPE(None, C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
+ALLGATHER_FN = C.CFUNCTYPE(C.c_int, C.c_void_p, C.c_void_p, C.c_size_t, C.c_void_p)
 
 
 class atf_space_opts(C.Structure):
@@ -46,7 +47,8 @@ class atf_space_opts(C.Structure):
 class atf_level_view(C.Structure):
     _fields_ = [("records", C.c_void_p), ("csr", C.c_void_p), ("n_nodes", C.c_uint64), ("offset", C.c_uint64),
                 ("words", C.c_int32), ("param", C.c_int32), ("field_word", C.c_int32),
-                ("field_shift", C.c_int32), ("field_bits", C.c_int32)]
+                ("field_shift", C.c_int32), ("field_bits", C.c_int32), ("csr_offset", C.c_uint64),
+                ("csr_nodes", C.c_uint64)]
 
 
 class atf_level_stats(C.Structure):
@@ -87,6 +89,7 @@ _SIGS = {
     "atf_space_neighbors": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_uint64, C.c_int32, C.c_void_p, C.c_int64,
                                   C.c_void_p, C.c_void_p]),
     "atf_space_stats": (_st, [SP, C.POINTER(atf_level_stats), C.c_int32, C.POINTER(C.c_int32)]),
+    "atf_space_generate_dist": (_st, [SP, C.c_int32, C.c_int32, ALLGATHER_FN, C.c_void_p]),
     "atf_space_destroy": (None, [SP]),
     "atf_status_str": (C.c_char_p, [_st]),
     "atf_space_last_error": (C.c_char_p, [SP]),

@@ -9,6 +9,8 @@
 
 #include <cuda_runtime.h>
 
+#include <unistd.h>
+
 #include <algorithm>
 #include <cstdarg>
 #include <cstdio>
@@ -100,6 +102,8 @@ struct LevelData {
   uint64_t* csr = nullptr;  // [n + 1], written when the next level is expanded
   uint64_t n = 0;
   uint64_t offset = 0;      // global index of rec[0] (shards)
+  uint64_t csr_offset = 0;  // global index of the node whose CSR entry is csr[0] (shards)
+  uint64_t csr_n = UINT64_MAX;  // csr entries - 1 (the nodes it covers); UINT64_MAX: the level's own nodes
   uint64_t evals = 0;
   float ms = -1.f;         // expand + scan + emit of the level (ATF_FLAG_TIMING)
   float expand_ms = -1.f;  // the expand kernel alone
@@ -139,6 +143,8 @@ struct atf_space {
     size_t stash_cap = 0;       // bytes
     unsigned long long* status = nullptr;  // tiny wide levels: look-back tile status words
     size_t status_cap = 0;                 // entries
+    char* pbuf = nullptr;                  // generate_dist: this rank's parent slice, assembled
+    size_t pbuf_cap = 0;                   // from the ranks' level arrays (P2P copies)
     cudaStream_t stream = nullptr;
     cudaEvent_t fork = nullptr, join = nullptr;
   };
@@ -166,6 +172,9 @@ struct atf_space {
   };
   std::vector<Tail> tails;
   // shards
+  bool ipc_alloc = false;      // arena chunks from cudaMalloc (exported by CUDA IPC to peer ranks)
+  struct PeerMap { int rank; char handle[64]; char* base; };
+  std::vector<PeerMap> peers;  // opened IPC allocations of other ranks (generate_dist)
   int shard_rank = 0, shard_world = 1;
   std::vector<int> shard_cut;  // per group: first level expanded on a slice (L = none)
 };
@@ -192,7 +201,12 @@ static atf_status fail(atf_space* s, atf_status st, const char* fmt, ...) {
 static void* dalloc(atf_space* s, size_t bytes) {
   if (bytes == 0) bytes = 16;
   void* p = nullptr;
-  if (s->opts.alloc) {
+  if (s->ipc_alloc) {  // generate_dist: peers map the arena through CUDA IPC
+    if (cudaMalloc(&p, bytes) != cudaSuccess) {
+      cudaGetLastError();
+      p = nullptr;
+    }
+  } else if (s->opts.alloc) {
     p = s->opts.alloc(bytes, s->opts.stream, s->opts.alloc_ctx);
   } else {
     if (cudaMallocAsync(&p, bytes, (cudaStream_t)s->opts.stream) != cudaSuccess) {
@@ -204,7 +218,10 @@ static void* dalloc(atf_space* s, size_t bytes) {
 }
 static void dfree(atf_space* s, void* p, size_t bytes) {
   if (!p) return;
-  if (s->opts.alloc) {
+  if (s->ipc_alloc) {
+    cudaStreamSynchronize((cudaStream_t)s->opts.stream);
+    cudaFree(p);
+  } else if (s->opts.alloc) {
     if (s->opts.free) s->opts.free(p, bytes, s->opts.stream, s->opts.alloc_ctx);
   } else {
     cudaFreeAsync(p, (cudaStream_t)s->opts.stream);
@@ -1059,6 +1076,7 @@ static void release_device(atf_space* s) {
     dfree(s, (char*)b.stash, b.stash_cap);
     dfree(s, b.masks, b.masks_cap);
     dfree(s, (char*)b.status, b.status_cap * 8);
+    dfree(s, b.pbuf, b.pbuf_cap);
     if (b.stream) {
       cudaStreamSynchronize(b.stream);
       cudaStreamDestroy(b.stream);
@@ -1067,6 +1085,8 @@ static void release_device(atf_space* s) {
     if (b.join) cudaEventDestroy(b.join);
   }
   s->gb.clear();
+  for (auto& pm : s->peers) cudaIpcCloseMemHandle(pm.base);
+  s->peers.clear();
   s->d_counter = nullptr;
   s->d_totals = nullptr;
   s->d_ovf = nullptr;
@@ -1645,6 +1665,273 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
   return ATF_OK;
 }
 
+// ---------------------------------------------------------------- balanced multi-GPU generation
+// SURVEY.md §8(e), DESIGN.md §6.  Every level is distributed afresh: rank r expands the parents
+// [r F / N, (r + 1) F / N) of the previous level (F = its global size), so every rank evaluates
+// the same number of (node, candidate) pairs at every level (f_{k-1} r_k / N), whatever the
+// shape of the tree.  Rank r's children are a contiguous slice of the level in canonical order
+// (children of a contiguous parent slice).  After each level round the ranks all-gather a small
+// record per group (level counts + where the new level's records live), fix their CSR entries to
+// global child indices, and copy their next parent slice from the owning ranks: CUDA IPC
+// pointers (one process per GPU: peer memory over NVLink / NVSwitch) or plain pointers (ranks
+// in one process).
+namespace {
+struct DistDesc {       // where a rank's slice of a level lives
+  int64_t pid;          // owning process
+  uint64_t base, off;   // allocation base (device pointer in the owner) and byte offset
+  char handle[64];      // cudaIpcMemHandle_t of the allocation
+};
+struct DistGroup {      // per group, per round
+  uint32_t nd, pad;     // levels completed this round (0, 1 or a tail's nl)
+  uint64_t cnt[kMaxTail];
+  DistDesc desc;        // records of the last completed level
+};
+}  // namespace
+
+static atf_status dist_desc(atf_space* s, int g, const uint32_t* rec, DistDesc& d) {
+  std::memset(&d, 0, sizeof d);
+  d.pid = (int64_t)getpid();
+  if (!rec) return ATF_OK;
+  for (auto& c : s->arena[g])
+    if ((const char*)rec >= c.p && (const char*)rec < c.p + c.size) {
+      d.base = (uint64_t)(uintptr_t)c.p;
+      d.off = (uint64_t)((const char*)rec - c.p);
+      cudaIpcMemHandle_t h;
+      CUDA_TRY(s, cudaIpcGetMemHandle(&h, c.p));
+      std::memcpy(d.handle, &h, sizeof h);
+      return ATF_OK;
+    }
+  return fail(s, ATF_ERR_STATE, "internal: level records outside the arena");
+}
+
+static atf_status dist_peer_ptr(atf_space* s, int q, const DistDesc& d, const char** out) {
+  if (d.pid == (int64_t)getpid()) {  // ranks in one process (tests, the one-GPU prediction)
+    *out = (const char*)(uintptr_t)d.base + d.off;
+    return ATF_OK;
+  }
+  for (auto& pm : s->peers)
+    if (pm.rank == q && std::memcmp(pm.handle, d.handle, 64) == 0) {
+      *out = pm.base + d.off;
+      return ATF_OK;
+    }
+  cudaIpcMemHandle_t h;
+  std::memcpy(&h, d.handle, sizeof h);
+  void* p = nullptr;
+  CUDA_TRY(s, cudaIpcOpenMemHandle(&p, h, cudaIpcMemLazyEnablePeerAccess));
+  atf_space::PeerMap pm;
+  pm.rank = q;
+  std::memcpy(pm.handle, d.handle, 64);
+  pm.base = (char*)p;
+  s->peers.push_back(pm);
+  *out = pm.base + d.off;
+  return ATF_OK;
+}
+
+static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allgather_fn ag, void* ctx) {
+  NvtxRange nvtx("atf_space_generate_dist");
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  const size_t G = s->groups.size();
+  std::vector<int> k(G, 0);
+  std::vector<uint64_t> F(G, 1);                 // global size of the frontier (level k - 1)
+  std::vector<uint64_t> lo(G, 0), hi(G, 0);      // this rank's parent slice of the frontier
+  std::vector<const uint32_t*> frontier(G, s->d_root);
+  std::vector<DistGroup> mine(G), all((size_t)world * G);
+  for (size_t g = 0; g < G; g++) {  // level 0: the root (one parent), expanded by rank 0
+    lo[g] = 0;
+    hi[g] = rank == 0 ? 1 : 0;
+  }
+  for (int round = 0;; round++) {
+    char rname[48];
+    snprintf(rname, sizeof rname, "atf dist round %d", round);
+    NvtxRange nvtx_round(rname);
+    std::vector<Pending> pend;
+    int active = 0;
+    for (size_t g = 0; g < G; g++)
+      if (k[g] < (int)s->groups[g].levels.size() && hi[g] > lo[g] && s->groups[g].levels[k[g]].r > 0) active++;
+    bool any_open = false;
+    for (size_t g = 0; g < G; g++) mine[g] = DistGroup{};
+    for (int attempt = 0;; attempt++) {
+      pend.clear();
+      CUDA_TRY(s, cudaMemsetAsync(s->d_totals, 0, 16 * kMaxGroups, st));
+      if (s->opts.flags & ATF_FLAG_TIMING) CUDA_TRY(s, cudaMemsetAsync(s->d_pairs, 0, 8 * kMaxGroups, st));
+      for (size_t g = 0; g < G; g++) {
+        const int L = (int)s->groups[g].levels.size();
+        if (k[g] >= L || mine[g].nd) continue;
+        any_open = true;
+        const uint64_t np = hi[g] - lo[g];
+        const bool empty_range = s->groups[g].levels[k[g]].r == 0;
+        if (np == 0 || empty_range) {
+          // no local parents (or an empty range): this rank's part of the level is empty; the
+          // parents' CSR entries are all zero
+          LevelData& d = s->data[g][k[g]];
+          d.rec = nullptr;
+          d.n = 0;
+          d.evals = np * (uint64_t)s->groups[g].levels[k[g]].r;
+          d.pairs = d.evals;
+          if (k[g] > 0) {
+            char* csr = arena_alloc(s, (int)g, (np + 1) * 8);
+            if (!csr) {
+              atf_status e = arena_grow(s, (int)g, (np + 1) * 8);
+              if (e) return e;
+              csr = arena_alloc(s, (int)g, (np + 1) * 8);
+            }
+            CUDA_TRY(s, cudaMemsetAsync(csr, 0, (np + 1) * 8, st));
+            LevelData& pdl = s->data[g][k[g] - 1];
+            pdl.csr = (uint64_t*)csr;
+            pdl.csr_offset = lo[g];
+            pdl.csr_n = np;
+          }
+          mine[g].nd = 1;
+          mine[g].cnt[0] = 0;
+          continue;
+        }
+        Pending pd;
+        atf_status e;
+        if (s->tails[g].phase == 1) {
+          e = queue_tail_emit(s, (int)g, pd, active > 1);
+        } else if (k[g] == tail_start(s, (int)g)) {
+          e = queue_tail_count(s, (int)g, k[g], frontier[g], np, pd, active > 1);
+        } else {
+          e = queue_level(s, (int)g, k[g], frontier[g], np, pd, active > 1);
+        }
+        if (e) return e;
+        pend.push_back(pd);
+      }
+      if (pend.empty()) break;
+      for (auto& pd : pend)
+        if (pd.joined) CUDA_TRY(s, cudaStreamWaitEvent(st, s->gb[pd.g].join, 0));
+      CUDA_TRY(s, cudaMemcpyAsync(s->h_ctl.data(), s->d_totals, 12 * kMaxGroups, cudaMemcpyDeviceToHost, st));
+      for (auto& pd : pend)
+        if (pd.kind == 1) {
+          auto& T = s->tails[pd.g];
+          for (int d = 0; d < T.nl; d++)
+            CUDA_TRY(s, cudaMemcpyAsync(&T.tot[d], T.t.tile_base + d * (T.t.n_tiles + 1) + T.t.n_tiles, 8,
+                                        cudaMemcpyDeviceToHost, st));
+        }
+      CUDA_TRY(s, cudaStreamSynchronize(st));
+      unsigned long long h_pairs[kMaxGroups] = {};
+      if (s->opts.flags & ATF_FLAG_TIMING)
+        CUDA_TRY(s, cudaMemcpy(h_pairs, s->d_pairs, sizeof(h_pairs), cudaMemcpyDeviceToHost));
+      bool redo = false;
+      for (auto& pd : pend) {
+        const int g = pd.g;
+        if (pd.kind == 1) {  // tail counted: its emit runs in the same round (sizes known)
+          s->tails[g].phase = 1;
+          redo = true;
+          continue;
+        }
+        if (pd.kind == 2) {
+          finish_tail(s, g);
+          auto& T = s->tails[g];
+          s->data[g][T.k0 > 0 ? T.k0 - 1 : 0].csr_offset = lo[g];
+          if (T.k0 > 0) s->data[g][T.k0 - 1].csr_n = hi[g] - lo[g];
+          mine[g].nd = (uint32_t)T.nl;
+          for (int d = 0; d < T.nl; d++) mine[g].cnt[d] = T.tot[d];
+          continue;
+        }
+        const uint64_t total = s->h_totals[g];
+        GroupPlan& gp = s->groups[g];
+        if (s->h_flags[g] || total > pd.cap) {  // overflow: grow and redo within this round
+          s->stash_hint = std::max<uint64_t>(s->stash_hint, total);
+          atf_status e = arena_grow(s, g, total * gp.words * 4 + (pd.n_parents + 1) * 8);
+          if (e) return e;
+          redo = true;
+          continue;
+        }
+        Chunk& c = s->arena[g][pd.chunk];
+        c.used = pd.child_off + ((total * gp.words * 4 + 255) & ~(uint64_t)255);
+        LevelData& d = s->data[g][pd.k];
+        d.rec = pd.child;
+        d.n = total;
+        d.evals = pd.n_parents * (uint64_t)gp.levels[pd.k].r;
+        if (pd.k > 0) {
+          LevelData& pdl = s->data[g][pd.k - 1];
+          pdl.csr = pd.csr;
+          pdl.csr_offset = lo[g];
+          pdl.csr_n = pd.n_parents;
+        }
+        if (s->opts.flags & ATF_FLAG_TIMING) {
+          cudaEventElapsedTime(&d.ms, s->events[g][pd.k].first, s->events[g][pd.k].second);
+          cudaEventElapsedTime(&d.expand_ms, s->events[g][pd.k].first, s->events[g][pd.k].mid);
+          d.pairs = d.seg_skip ? h_pairs[g] : d.evals;
+        }
+        mine[g].nd = 1;
+        mine[g].cnt[0] = total;
+      }
+      if (!redo) break;
+    }
+    if (!any_open) break;
+    // exchange: one record per group and rank
+    for (size_t g = 0; g < G; g++) {
+      if (mine[g].nd != 1) continue;
+      atf_status e = dist_desc(s, (int)g, s->data[g][k[g]].rec, mine[g].desc);
+      if (e) return e;
+    }
+    if (ag(mine.data(), all.data(), sizeof(DistGroup) * G, ctx) != 0)
+      return fail(s, ATF_ERR_CUDA, "all-gather callback failed in round %d", round);
+    for (size_t g = 0; g < G; g++) {
+      const uint32_t nd = mine[g].nd;
+      if (!nd) continue;
+      for (int r = 0; r < world; r++)
+        if (all[(size_t)r * G + g].nd != nd) return fail(s, ATF_ERR_STATE, "ranks out of step (group %zu)", g);
+      // global offsets of this rank's part of every completed level; CSR entries -> global
+      for (uint32_t d = 0; d < nd; d++) {
+        uint64_t before = 0, tot = 0;
+        for (int r = 0; r < world; r++) {
+          const uint64_t c = all[(size_t)r * G + g].cnt[d];
+          if (r < rank) before += c;
+          tot += c;
+        }
+        LevelData& ld = s->data[g][k[g] + d];
+        ld.offset = before;
+        if (d + 1 < nd) {  // a tail's inner level: its CSR (this rank's nodes) came with it
+          ld.csr_offset = before;
+          ld.csr_n = ld.n;
+        }
+        // the CSR of the level above points into this rank's local child array
+        LevelData* pl = k[g] + (int)d > 0 ? &s->data[g][k[g] + d - 1] : nullptr;
+        if (pl && pl->csr && before) {
+          int ce = launch_add_offset(pl->csr, pl->csr_n + 1, before, st);
+          if (ce) return fail(s, ATF_ERR_CUDA, "csr fix-up");
+        }
+        F[g] = tot;
+      }
+      k[g] += (int)nd;
+      const int L = (int)s->groups[g].levels.size();
+      if (k[g] >= L) continue;
+      // the next parent slice, copied from the ranks holding it
+      const uint64_t Fg = F[g];
+      lo[g] = (uint64_t)((unsigned __int128)Fg * rank / world);
+      hi[g] = (uint64_t)((unsigned __int128)Fg * (rank + 1) / world);
+      const uint64_t np = hi[g] - lo[g];
+      if (np == 0) continue;
+      const int W = s->groups[g].words;
+      auto& gbf = s->gb[g];
+      atf_status e = ensure_buf(s, &gbf.pbuf, &gbf.pbuf_cap, np * W * 4, "parent slice");
+      if (e) return e;
+      uint64_t pos = 0;  // global index of records[0] of rank q
+      for (int q = 0; q < world; q++) {
+        const DistGroup& dg = all[(size_t)q * G + g];
+        const uint64_t n = dg.cnt[0], a0 = std::max(pos, lo[g]), a1 = std::min(pos + n, hi[g]);
+        if (a1 > a0) {
+          const char* src = nullptr;
+          if ((e = dist_peer_ptr(s, q, dg.desc, &src))) return e;
+          CUDA_TRY(s, cudaMemcpyAsync(gbf.pbuf + (a0 - lo[g]) * W * 4, src + (a0 - pos) * W * 4, (a1 - a0) * W * 4,
+                                      cudaMemcpyDeviceToDevice, st));
+        }
+        pos += n;
+      }
+      frontier[g] = (const uint32_t*)gbf.pbuf;
+    }
+  }
+  s->gsize.assign(G, 0);
+  for (size_t g = 0; g < G; g++) s->gsize[g] = s->groups[g].levels.empty() ? 0 : (k[g] >= (int)s->groups[g].levels.size() ? F[g] : 0);
+  s->shard_rank = rank;
+  s->shard_world = world;
+  s->state = FINAL_SHARD;
+  return ATF_OK;
+}
+
 static atf_status generate_impl(atf_space* s) {
   NvtxRange nvtx("atf_space_generate");
   atf_status e = plan(s);
@@ -1988,6 +2275,8 @@ atf_status atf_space_plan_json(const atf_space* s, char* buf, size_t cap, size_t
 atf_status atf_space_generate(atf_space* s) {
   if (!s) return ATF_ERR_INVALID_ARG;
   if (s->state == SHARDED) return fail(s, ATF_ERR_STATE, "space holds an unfinalized shard");
+  if (s->dev_ready && s->ipc_alloc) release_device(s);  // back to the configured allocator
+  s->ipc_alloc = false;
   if (s->state == BUILDING) {
     atf_status e = atf_space_plan(s);
     if (e) return e;
@@ -2049,6 +2338,10 @@ atf_status atf_space_level_view(const atf_space* s, int32_t g, int32_t k, atf_le
   out->field_word = lp.field_word;
   out->field_shift = lp.field_shift;
   out->field_bits = lp.field_bits;
+  // the CSR covers this rank's nodes of level k (single GPU / generate_shard) or the parent slice
+  // it expanded (generate_dist)
+  out->csr_offset = d.csr_n != UINT64_MAX ? d.csr_offset : d.offset;
+  out->csr_nodes = d.csr_n != UINT64_MAX ? d.csr_n : d.n;
   return ATF_OK;
 }
 
@@ -2320,6 +2613,8 @@ atf_status atf_space_generate_shard(atf_space* s, int32_t rank, int32_t world, i
     atf_status e = atf_space_plan(s);
     if (e) return e;
   }
+  if (s->dev_ready && s->ipc_alloc) release_device(s);
+  s->ipc_alloc = false;
   atf_status e = ensure_device(s);
   if (e) return e;
   size_t G = s->groups.size();
@@ -2482,6 +2777,37 @@ atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, si
     buf[n] = 0;
   }
   return ATF_OK;
+}
+
+atf_status atf_space_generate_dist(atf_space* s, int32_t rank, int32_t world, atf_allgather_fn allgather, void* ctx) {
+  if (!s || !allgather || world < 1 || rank < 0 || rank >= world) return fail(s, ATF_ERR_INVALID_ARG, "bad rank/world");
+  if (s->state == BUILDING) {
+    atf_status e = atf_space_plan(s);
+    if (e) return e;
+  }
+  if (s->dev_ready && !s->ipc_alloc) release_device(s);  // arenas must be exportable (cudaMalloc)
+  s->ipc_alloc = true;
+  atf_status e = ensure_device(s);
+  if (e) return e;
+  const size_t G = s->groups.size();
+  s->data.assign(G, {});
+  s->tails.assign(G, {});
+  for (size_t g = 0; g < G; g++) {
+    s->data[g].assign(s->groups[g].levels.size(), LevelData{});
+    for (auto& c : s->arena[g]) c.used = 0;
+  }
+  if ((s->opts.flags & ATF_FLAG_TIMING) && s->events.size() != G) {
+    s->events.assign(G, {});
+    for (size_t g = 0; g < G; g++) {
+      s->events[g].resize(s->groups[g].levels.size());
+      for (auto& ev : s->events[g]) {
+        CUDA_TRY(s, cudaEventCreate(&ev.first));
+        CUDA_TRY(s, cudaEventCreate(&ev.mid));
+        CUDA_TRY(s, cudaEventCreate(&ev.second));
+      }
+    }
+  }
+  return generate_dist_impl(s, rank, world, allgather, ctx);
 }
 
 atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, size_t* len_out, int32_t* k0_out) {

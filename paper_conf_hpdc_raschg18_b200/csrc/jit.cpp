@@ -478,90 +478,73 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
     s += "      if (lane == 0) a.tile_total[(u64)" + ds + " * a.n_tiles + tile] = v; }\n";
   }
   s += "  }\n}\n";
-  // ---- emit: chunk walk.  emit_d takes a chunk of <= CS_d nodes of level d - 1 (lane = node),
-  // evaluates their level-d masks, writes their CSR entries and appends their children (records +
-  // the frontier lane they descend from) to level d's shared-memory buffer, then walks those
-  // children in chunks of CS_{d+1}.  Chunks go in node order at every depth, so each level's
-  // output is its canonical order; a level's buffer is flushed to global memory as coalesced
-  // vectors only when the next chunk's children would not fit (and at the end of the tile).
-  // CS_d * r_d <= 256 keeps every buffer <= 256 records whatever r.  Per-warp shared memory:
-  // node constants [32][NC], then per level d: records [BC_d][W], frontier lanes [BC_d].
-  std::vector<int> CS(nl), BC(nl), off(nl + 1, 0), ooff(nl, 0);
-  for (int d = 0; d < nl; d++) {
-    CS[d] = std::max(1, std::min(32, 256 / t.lv[d].r));
-    BC[d] = std::max(256, CS[d] * t.lv[d].r);
-  }
-  off[0] = (4 * 32 * NC + 15) & ~15;
-  for (int d = 0; d < nl; d++) {
-    ooff[d] = off[d] + BC[d] * W * 4;
-    off[d + 1] = (ooff[d] + BC[d] + 15) & ~15;
-  }
-  const std::string WB = std::to_string(off[nl]), NCs = std::to_string(NC);
-  if (warp_bytes) *warp_bytes = off[nl];
-  const std::string V = W == 1 ? "u32" : (W == 2 ? "uint2" : "uint4"), VPR = std::to_string(W <= 4 ? 1 : 2);
-  for (int d = 0; d < nl; d++) {  // flush of level d
-    const std::string ds = std::to_string(d);
-    s += "__device__ __forceinline__ void flush" + ds + "(const TailJitArgs& a, u64* cur, u32* fill, unsigned char* wbuf, int lane) {\n";
-    s += "  const u32 n = fill[" + ds + "] * " + VPR + ";\n";
-    s += "  const " + V + "* src = reinterpret_cast<const " + V + "*>(wbuf + " + std::to_string(off[d]) + ");\n";
-    s += "  " + V + "* dst = reinterpret_cast<" + V + "*>(a.rec[" + ds + "] + cur[" + ds + "] * " + Ws + ");\n";
-    s += "#pragma unroll 4\n  for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
-    s += "  cur[" + ds + "] += fill[" + ds + "];\n  fill[" + ds + "] = 0;\n  __syncwarp();\n}\n";
-  }
+  // ---- emit: lane = frontier node, depth-first (like the count), output staged per warp.
+  // Each lane recounts its subtree (cnt_d), a warp scan per level gives its nodes' tile-local
+  // positions; the lane then writes its subtree depth-first — a node's level-d descendants come
+  // out in canonical order — records and CSR entries (first child = the child level's running
+  // position) into the warp's shared-memory staging area, which the warp then copies out as
+  // coalesced vectors (one contiguous run per level and per CSR array).  A tile whose output
+  // exceeds the staging area (the sizes are known before writing) writes straight to global.
+  constexpr int kStage = 12288;  // staging bytes per warp
+  if (warp_bytes) *warp_bytes = kStage;
+  const std::string NLs = std::to_string(nl), NCs = std::to_string(NC);
   for (int d = nl - 1; d >= 0; d--) {
     const std::string ds = std::to_string(d);
-    s += "__device__ __forceinline__ void emit" + ds + "(const TailJitArgs& a, const u32* w, u32 org, bool valid, u64 gidx, "
-         "u64* cur, u32* fill, unsigned char* wbuf, int lane) {\n";
-    s += "  const u32* s_nc = reinterpret_cast<const u32*>(wbuf);\n";
-    s += "  u32 m = valid ? tmask" + ds + "(a, w, s_nc + org * " + NCs + ") : 0u;\n";
-    s += "  const u32 c = __popc(m);\n  u32 incl = c;\n";
-    s += "#pragma unroll\n  for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
-         "if (lane >= o) incl += y; }\n";
-    s += "  const u32 T = __shfl_sync(0xffffffffu, incl, 31);\n";
-    s += "  if (fill[" + ds + "] + T > " + std::to_string(BC[d]) + "u) flush" + ds + "(a, cur, fill, wbuf, lane);\n";
-    s += "  const u32 base = fill[" + ds + "];\n  u32 k = base + incl - c;\n";
-    s += "  if (valid) a.csr[" + ds + "][gidx] = cur[" + ds + "] + k;\n";
-    s += "  u32* buf = reinterpret_cast<u32*>(wbuf + " + std::to_string(off[d]) + ");\n";
-    s += "  unsigned char* obuf = wbuf + " + std::to_string(ooff[d]) + ";\n";
-    s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n";
-    s += child(d, "w", "(buf + k * " + Ws + ")", "    ");
-    s += "    obuf[k] = (unsigned char)org;\n    k++;\n  }\n  __syncwarp();\n";
-    s += "  fill[" + ds + "] = base + T;\n";
+    s += "__device__ __forceinline__ void dfs" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cur, "
+         "const u64* base, unsigned char* sm, bool staged, const u32* roff, const u32* coff) {\n";
+    s += "  u32 m = tmask" + ds + "(a, w, nc);\n";
+    s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
+    s += child(d, "w", "cw", "    ");
+    s += "    const u32 slot = cur[" + ds + "]++;\n";
+    s += "    if (staged) {\n      u32* dst = reinterpret_cast<u32*>(sm + roff[" + ds + "]) + slot * " + Ws + ";\n";
+    for (int w = 0; w < W; w++) s += "      dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
+    s += "    } else {\n      u32* dst = a.rec[" + ds + "] + (base[" + ds + "] + slot) * " + Ws + ";\n";
+    for (int w = 0; w < W; w++) s += "      dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
+    s += "    }\n";
     if (d + 1 < nl) {
-      const std::string cs = std::to_string(CS[d + 1]);
-      s += "  const u64 g0 = cur[" + ds + "] + base;\n";
-      s += "  for (u32 s0 = 0; s0 < T; s0 += " + cs + ") {\n    const bool v = lane < " + cs + " && s0 + lane < T;\n";
-      s += "    const u32 ix = base + s0 + (v ? lane : 0);\n    u32 cw[" + Ws + "];\n";
-      for (int w = 0; w < W; w++) s += "    cw[" + std::to_string(w) + "] = buf[ix * " + Ws + " + " + std::to_string(w) + "];\n";
-      s += "    emit" + std::to_string(d + 1) + "(a, cw, obuf[ix], v, g0 + s0 + lane, cur, fill, wbuf, lane);\n  }\n";
+      const std::string d1 = std::to_string(d + 1);
+      s += "    const u64 fc = base[" + d1 + "] + cur[" + d1 + "];\n";
+      s += "    if (staged) *reinterpret_cast<u64*>(sm + coff[" + ds + "] + slot * 8u) = fc;\n";
+      s += "    else a.csr[" + d1 + "][base[" + ds + "] + slot] = fc;\n";
+      s += "    dfs" + d1 + "(a, cw, nc, cur, base, sm, staged, roff, coff);\n";
     }
-    s += "}\n";
+    s += "  }\n}\n";
   }
   s += "extern \"C\" __global__ void __launch_bounds__(128) atf_tail_emit(const __grid_constant__ TailJitArgs a) {\n";
   s += "  extern __shared__ __align__(16) unsigned char smem[];\n";
-  s += "  const int lane = threadIdx.x & 31;\n  unsigned char* wbuf = smem + (threadIdx.x >> 5) * " + WB + ";\n";
-  s += "  u32* s_nc = reinterpret_cast<u32*>(wbuf);\n";
+  s += "  const int lane = threadIdx.x & 31;\n  unsigned char* sm = smem + (threadIdx.x >> 5) * " + std::to_string(kStage) + ";\n";
   s += "  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n  const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n";
-  s += "  if (gw == 0 && lane < " + std::to_string(nl) + ") {\n";
+  s += "  if (gw == 0 && lane < " + NLs + ") {\n";
   s += "    const u64 above = lane == 0 ? a.n_parents : a.tile_base[(u64)(lane - 1) * (a.n_tiles + 1) + a.n_tiles];\n";
   s += "    a.csr[lane][above] = a.tile_base[(u64)lane * (a.n_tiles + 1) + a.n_tiles];\n  }\n";
-  s += "  for (u64 tile = gw; tile < a.n_tiles; tile += nw) {\n    u64 cur[" + std::to_string(nl) + "];\n    u32 fill[" +
-       std::to_string(nl) + "];\n";
-  for (int d = 0; d < nl; d++)
-    s += "    cur[" + std::to_string(d) + "] = a.tile_base[(u64)" + std::to_string(d) + " * (a.n_tiles + 1) + tile]; fill[" +
-         std::to_string(d) + "] = 0;\n";
-  s += "    const u64 nd0 = tile * 32;\n    const bool vl = nd0 + lane < a.n_parents;\n    u32 w[" + Ws + "];\n";
-  s += "    for (int i = 0; i < " + Ws + "; i++) w[i] = vl ? __ldg(a.parent_rec + (nd0 + lane) * " + Ws + " + i) : 0u;\n";
-  s += "    { u32 nc[" + NCs + "];\n      tnc(a, w, nc);\n      for (int i = 0; i < " + NCs + "; i++) s_nc[lane * " + NCs +
-       " + i] = nc[i]; }\n    __syncwarp();\n";
-  const std::string cs0 = std::to_string(CS[0]);
-  s += "    for (u32 s0 = 0; s0 < 32; s0 += " + cs0 + ") {\n";
-  s += "      const u32 src = s0 + (lane < " + cs0 + " ? lane : 0);\n      u32 cw[" + Ws + "];\n";
-  for (int w = 0; w < W; w++) s += "      cw[" + std::to_string(w) + "] = __shfl_sync(0xffffffffu, w[" + std::to_string(w) + "], src & 31);\n";
-  s += "      const bool v = lane < " + cs0 + " && s0 + lane < 32 && nd0 + s0 + lane < a.n_parents;\n";
-  s += "      emit0(a, cw, src & 31, v, nd0 + s0 + lane, cur, fill, wbuf, lane);\n    }\n";
-  for (int d = 0; d < nl; d++) s += "    flush" + std::to_string(d) + "(a, cur, fill, wbuf, lane);\n";
-  s += "  }\n}\n";
+  s += "  for (u64 tile = gw; tile < a.n_tiles; tile += nw) {\n";
+  s += "    const u64 nd = tile * 32 + lane;\n    const bool valid = nd < a.n_parents;\n    u32 w[" + Ws + "];\n";
+  s += "    for (int i = 0; i < " + Ws + "; i++) w[i] = valid ? __ldg(a.parent_rec + nd * " + Ws + " + i) : 0u;\n";
+  s += "    u32 nc[" + NCs + "];\n    u32 cnt[" + NLs + "] = {};\n";
+  s += "    if (valid) { tnc(a, w, nc); cnt0(a, w, nc, cnt); }\n";
+  s += "    u32 cur[" + NLs + "], T[" + NLs + "];\n    u64 base[" + NLs + "];\n    u32 need = 0;\n";
+  s += "#pragma unroll\n    for (int d = 0; d < " + NLs + "; d++) {\n";
+  s += "      u32 incl = cnt[d];\n#pragma unroll\n      for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
+       "if (lane >= o) incl += y; }\n";
+  s += "      T[d] = __shfl_sync(0xffffffffu, incl, 31);\n      cur[d] = incl - cnt[d];\n";
+  s += "      base[d] = a.tile_base[(u64)d * (a.n_tiles + 1) + tile];\n";
+  s += "      need += T[d] * " + std::to_string(W * 4) + "u + (d + 1 < " + NLs + " ? T[d] * 8u : 0u);\n    }\n";
+  // frontier CSR
+  s += "    if (valid) a.csr[0][nd] = base[0] + cur[0];\n";
+  // staging layout: CSR regions first (8-byte aligned), then records
+  s += "    const bool staged = need <= " + std::to_string(kStage) + "u;\n    u32 roff[" + NLs + "], coff[" + NLs + "];\n";
+  s += "    { u32 o = 0;\n      for (int d = 0; d + 1 < " + NLs + "; d++) { coff[d] = o; o += T[d] * 8u; }\n";
+  s += "      coff[" + std::to_string(nl - 1) + "] = o;\n      for (int d = 0; d < " + NLs + "; d++) { roff[d] = o; o += T[d] * " +
+       std::to_string(W * 4) + "u; } }\n";
+  s += "    if (valid) dfs0(a, w, nc, cur, base, sm, staged, roff, coff);\n";
+  s += "    if (staged) {\n      __syncwarp();\n";
+  // copy records (u32 granularity keeps any alignment of roff) and CSR (u64)
+  s += "      for (int d = 0; d < " + NLs + "; d++) {\n";
+  s += "        const u32* src = reinterpret_cast<const u32*>(sm + roff[d]);\n        u32* dst = a.rec[d] + base[d] * " + Ws + ";\n";
+  s += "        const u32 n = T[d] * " + Ws + "u;\n#pragma unroll 4\n        for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
+  s += "        if (d + 1 < " + NLs + ") {\n          const u64* cs = reinterpret_cast<const u64*>(sm + coff[d]);\n";
+  s += "          u64* cd = a.csr[d + 1] + base[d];\n#pragma unroll 4\n          for (u32 v = lane; v < T[d]; v += 32) cd[v] = cs[v];\n        }\n";
+  s += "      }\n      __syncwarp();\n    }\n  }\n}\n";
   return s;
 }
 

@@ -131,6 +131,27 @@ class Space:
         L.check(L.atf_space_generate_shard(self._h, rank, world, buf, cap, C.byref(n)), self._h)
         return list(buf[: n.value])
 
+    def generate_dist(self, rank: int, world: int, allgather) -> None:
+        """Balanced multi-GPU generation (atf_space_generate_dist): `allgather(data: bytes) ->
+        bytes` must return the concatenation of every rank's `data` in rank order."""
+        err = []
+
+        def _cb(send, recv, nbytes, _ctx):
+            try:
+                out = allgather(C.string_at(send, nbytes))
+                assert len(out) == nbytes * world
+                C.memmove(recv, out, len(out))
+                return 0
+            except Exception as ex:  # noqa: BLE001 -- reported through the status code
+                err.append(ex)
+                return 1
+
+        cb = L.ALLGATHER_FN(_cb)
+        st = L.atf_space_generate_dist(self._h, rank, world, cb, None)
+        if err:
+            raise err[0]
+        L.check(st, self._h)
+
     def finalize_shard(self, all_counts: List[List[int]]) -> None:
         world = len(all_counts)
         n = len(all_counts[0])
@@ -183,7 +204,8 @@ class Space:
         n, W = v["n_nodes"], v["words"]
         rec = (torch.as_tensor(_CAI(v["records"], (n, W), "<i4"), device=dev) if n and v["records"]
                else torch.zeros((0, W), dtype=torch.int32, device=dev))
-        csr = torch.as_tensor(_CAI(v["csr"], (n + 1,), "<i8"), device=dev) if v["csr"] else None
+        nc = v["csr_nodes"]
+        csr = torch.as_tensor(_CAI(v["csr"], (nc + 1,), "<i8"), device=dev) if v["csr"] else None
         return rec, csr
 
     def stats(self) -> List[dict]:

@@ -762,3 +762,119 @@ def test_allocator_failure_is_reported_and_space_destroys_cleanly(Space):
         st, S, _ = run(k)
         assert st == -2, (k, st)          # ATF_ERR_OOM
     assert run(-1)[:2] == (0, ref)
+
+
+# ---------------------------------------------------------------- balanced multi-GPU generation
+def _dist_check(Space, spec, world, flags=0):
+    """generate_dist on `world` virtual ranks (spaces of this process): global sizes = the oracle's,
+    every level's rank slices (records, by offset) concatenate to the single-GPU level, and the
+    ranks' CSR slices (by csr_offset) concatenate to the single-GPU CSR; every rank expanded
+    ~1/world of every level's parents (the balance rule)."""
+    from paper_conf_hpdc_raschg18_b200.shard import virtual_ranks
+    ref = orc.info(spec, threads=8)
+    with Space(spec, flags=flags) as one:
+        one.generate()
+        G = one.num_groups()
+        want = {(g, k): tuple(t.clone() if t is not None else None for t in one.level_tensors(g, k))
+                for g in range(G) for k in range(one.num_levels(g))}
+        sizes = one.group_sizes()
+    spaces = [Space(spec, flags=flags) for _ in range(world)]
+    try:
+        virtual_ranks(spaces)
+        assert sizes == [g["size"] for g in ref["groups"]]
+        for sp in spaces:
+            assert sp.group_sizes() == sizes
+            assert sp.size() == int(ref["S"])
+        for (g, k), (wrec, wcsr) in want.items():
+            parts, cparts = [], []
+            for sp in spaces:
+                v = sp.level_view(g, k)
+                rec, csr = sp.level_tensors(g, k)
+                parts.append((v["offset"], rec))
+                if csr is not None:
+                    cparts.append((v["csr_offset"], csr))
+            parts.sort(key=lambda t: t[0])
+            pos = 0
+            for off, rec in parts:
+                assert off == pos, (g, k)
+                pos += rec.shape[0]
+            assert torch.equal(torch.cat([r for _, r in parts]), wrec), (g, k)
+            if wcsr is not None:
+                cparts.sort(key=lambda t: t[0])
+                got = torch.cat([c[:-1] for _, c in cparts] + [cparts[-1][1][-1:]])
+                assert torch.equal(got, wcsr), ("csr", g, k)
+                # balance: every rank's parent slice is floor/ceil of f_k / world
+                n = wrec.shape[0]
+                for _, c in cparts:
+                    assert abs((c.shape[0] - 1) - n / world) <= 1, (g, k)
+    finally:
+        for sp in spaces:
+            sp.close()
+
+
+@pytest.mark.parametrize("world", [2, 3, 8])
+@pytest.mark.parametrize("name", ["C5-300x4", "C3-IS1", "C2-256", "C5-4096x3", "fig1", "C1"])
+def test_dist_virtual_ranks_match_single_gpu(Space, world, name):
+    _dist_check(Space, SMALL[name](), world)
+
+
+@pytest.mark.parametrize("seed", range(0, 40, 4))
+def test_dist_virtual_ranks_fuzz(Space, seed):
+    _dist_check(Space, A.random_spec(seed), 3)
+    _dist_check(Space, A.random_wide_spec(seed), 2)
+
+
+def test_dist_virtual_ranks_headline_flags(Space):
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    _dist_check(Space, A.c5_chains(4096, 4), 4, flags=L.ATF_FLAG_NO_SEG_BOUNDS)
+    _dist_check(Space, A.c3_xgemm((20, 96, 8)), 4, flags=L.ATF_FLAG_NO_JIT)
+
+
+def test_dist_two_processes_cuda_ipc(Space, tmp_path):
+    """Two processes on the one GPU, gloo all-gather: the parent slices cross processes through
+    CUDA IPC (cudaIpcGetMemHandle / OpenMemHandle), the path every rank of an 8-GPU node uses."""
+    import subprocess
+    import sys
+    script = tmp_path / "ipc_ranks.py"
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    script.write_text(f"""
+import os, sys, torch, numpy as np
+sys.path.insert(0, {root!r})
+import torch.distributed as dist
+import atfspec as A
+from paper_conf_hpdc_raschg18_b200 import Space
+from paper_conf_hpdc_raschg18_b200.shard import generate_balanced
+dist.init_process_group("gloo")
+r = dist.get_rank()
+torch.cuda.set_device(0)
+with Space(A.c5_chains(300, 4)) as sp:
+    generate_balanced(sp)
+    out = {{"sizes": sp.group_sizes()}}
+    for g in range(sp.num_groups()):
+        for k in range(sp.num_levels(g)):
+            v = sp.level_view(g, k)
+            rec, csr = sp.level_tensors(g, k)
+            out[f"r{{g}}_{{k}}"] = (v["offset"], rec.cpu().numpy())
+            if csr is not None:
+                out[f"c{{g}}_{{k}}"] = (v["csr_offset"], csr.cpu().numpy())
+    np.save({str(tmp_path)!r} + f"/rank{{r}}.npy", out, allow_pickle=True)
+dist.destroy_process_group()
+""")
+    env = dict(os.environ, MASTER_ADDR="127.0.0.1")
+    p = subprocess.run([sys.executable, "-m", "torch.distributed.run", "--nnodes=1", "--nproc-per-node=2",
+                        "--master-addr", "127.0.0.1", "--master-port", "29531", str(script)],
+                       capture_output=True, text=True, timeout=600, env=env)
+    assert p.returncode == 0, p.stdout[-3000:] + p.stderr[-3000:]
+    res = [np.load(tmp_path / f"rank{r}.npy", allow_pickle=True).item() for r in range(2)]
+    spec = A.c5_chains(300, 4)
+    with Space(spec) as one:
+        one.generate()
+        assert res[0]["sizes"] == res[1]["sizes"] == one.group_sizes()
+        for g in range(one.num_groups()):
+            for k in range(one.num_levels(g)):
+                rec, csr = one.level_tensors(g, k)
+                parts = sorted([res[r][f"r{g}_{k}"] for r in range(2)], key=lambda t: t[0])
+                assert np.array_equal(np.concatenate([p for _, p in parts]), rec.cpu().numpy())
+                if csr is not None:
+                    cp = sorted([res[r][f"c{g}_{k}"] for r in range(2)], key=lambda t: t[0])
+                    assert np.array_equal(np.concatenate([cp[0][1][:-1], cp[1][1]]), csr.cpu().numpy())

@@ -173,3 +173,80 @@ def test_gloo_world2_shard_protocol(oracle_bin):
         for i, f in enumerate(first):
             if f is not None and counts[i]:
                 assert before[i] == f                            # global offset of this rank's run
+
+
+# ---------------------------------------------------------------- balanced per-level protocol, gloo world 2
+def _balanced_rank_main(rank, world, port, q):
+    """atf_space_generate_dist's protocol restated on the CPU (plain loops over the chain tree):
+    level k is expanded from the parent slice [r F / N, (r+1) F / N) of level k - 1, the ranks
+    all-gather one byte record per level through shard._allgather_bytes (gloo), and the next
+    parent slice is taken from the concatenation of the ranks' children."""
+    import struct
+    os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_hpdc_raschg18_b200.shard import _allgather_bytes
+        spec = A.c5_chains(R, LEN)
+        out = []
+        for g in range(3):
+            params = spec.params[g * LEN:(g + 1) * LEN]
+            vals = [list(range(p.range["begin"], p.range["end"] + 1, p.range.get("step", 1))) for p in params]
+            frontier = [()]
+            F = 1
+            per_level = []
+            for k in range(LEN):
+                lo, hi = F * rank // world, F * (rank + 1) // world
+                kids = []
+                for path in frontier[lo:hi]:
+                    for j, x in enumerate(vals[k]):
+                        if k == 0:
+                            ok = True
+                        else:
+                            pv = vals[k - 1][path[-1]]
+                            ok = (pv % x == 0) if g != 1 else (x % pv == 0)
+                        if ok:
+                            kids.append(path + (j,))
+                rec = struct.pack("<q", len(kids))
+                allb = _allgather_bytes(rec)
+                counts = [struct.unpack_from("<q", allb, 8 * r)[0] for r in range(world)]
+                # the real library copies the parent slice from the ranks' arenas; here every rank
+                # rebuilds the level from the gathered children (small spec)
+                gathered = _allgather_bytes(repr(kids).encode().ljust(1 << 20))
+                full = []
+                for r in range(world):
+                    full += eval(gathered[r << 20:(r + 1) << 20].rstrip())
+                assert len(full) == sum(counts)
+                per_level.append((hi - lo, sum(counts), sum(counts[:rank]), kids[:1]))
+                frontier, F = full, len(full)
+            out.append(per_level)
+        q.put((rank, out))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_gloo_world2_balanced_protocol(oracle_bin):
+    from oracle import run as orc
+    spec = A.c5_chains(R, LEN)
+    ref = orc.info(spec)
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_balanced_rank_main, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    for _ in range(world):
+        rank, out = q.get(timeout=240)
+        res[rank] = out
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for g in range(3):
+        f = [lv["f"] for lv in ref["groups"][g]["levels"]]
+        for k in range(LEN):
+            parents = [res[r][g][k][0] for r in range(world)]
+            F = 1 if k == 0 else f[k - 1]
+            assert sum(parents) == F and max(parents) - min(parents) <= 1   # balanced parent slices
+            assert res[0][g][k][1] == res[1][g][k][1] == f[k]               # global level size = oracle f_k
+            assert res[0][g][k][2] == 0                                     # rank offsets: exclusive scan
