@@ -183,6 +183,30 @@ def enum_code(rng: dict, name: str) -> int:
     return rng["names"].index(name)
 
 
+def floats(*values: float) -> dict:
+    """A float-valued parameter by position index (S§8(f) NEXT-3; P:57 ranges of "arbitrary
+    fundamental type T (e.g., bool, integer, or float)"): a SET of the positions 0..n-1 in the
+    listed order, the float values kept as the display names (Space.to_named maps positions back).
+    Constraints see the position; for an ascending list (float_interval) order comparisons on
+    positions equal order comparisons on values (``X <= float_code(rng, 0.5)``)."""
+    vals = [float(v) for v in values]
+    if len(set(vals)) != len(vals):
+        raise ValueError("duplicate float value")  # reading #5
+    return {"kind": "set", "values": list(range(len(vals))), "names": vals}
+
+
+def float_interval(begin: float, end: float, step: float) -> dict:
+    """``atf::interval<float>(begin, end, step)``: begin + i * step for i = 0, 1, ... while <= end
+    (inclusive, reading #1; a tolerance of 1e-9 * step absorbs the float rounding of the bound)."""
+    n = int((end - begin) / step + 1e-9) + 1
+    return floats(*[begin + i * step for i in range(max(0, n))])
+
+
+def float_code(rng: dict, value: float) -> int:
+    """Position of `value` in a float parameter's range (exact match)."""
+    return rng["names"].index(float(value))
+
+
 @dataclass
 class Param:
     name: str

@@ -372,8 +372,10 @@ def predicted_scaling(spec, worlds=(2, 4, 8), reps=3, ag_us=25.0):
                 rounds = len(vag.round_s[0])
                 t = sum(max(vag.round_s[r][i] for r in range(N)) for i in range(rounds)) + (rounds - 1) * ag_us * 1e-6
                 if best is None or t < best[0]:
-                    best = (t, rounds, [sum(x) for x in vag.round_s])
-            out[N] = {"T_ms": best[0] * 1e3, "rounds": best[1], "rank_busy_ms": [round(x * 1e3, 3) for x in best[2]]}
+                    best = (t, rounds, [sum(x) for x in vag.round_s],
+                            [round(max(vag.round_s[r][i] for r in range(N)) * 1e3, 3) for i in range(rounds)])
+            out[N] = {"T_ms": best[0] * 1e3, "rounds": best[1], "rank_busy_ms": [round(x * 1e3, 3) for x in best[2]],
+                      "round_max_ms": best[3]}
         finally:
             for sp in spaces:
                 sp.close()

@@ -287,10 +287,13 @@ atf_status atf_space_encode_indices(const atf_space* s, const int32_t* d_values,
 
 /* CLTune-style baseline ("CLTune generates the search space
  * by filtering the full cartesian product"): every tuple of R_1 x ... x R_P is
- * enumerated on the GPU and every constraint interpreted (no groups, no pruning of
- * subtrees); *h_count = the number of valid tuples (= S), *h_tuples (optional) = the
- * product size.  Synchronous.  Needs only a planned space (callable before generate);
- * ATF_ERR_OVERFLOW if the product is >= 2^64. */
+ * enumerated on the GPU (no groups, no pruning of subtrees) and tested against the
+ * constraints with the generic bytecode interpreter, parameter by parameter in declaration
+ * order; a tuple is rejected at its first failing constraint, as a C++ conjunction of CLTune's
+ * per-parameter std::function predicates would (the accepted set is the same).  *h_count =
+ * the number of valid tuples (= S), *h_tuples (optional) = the product size.  Synchronous.
+ * Needs only a planned space (callable before generate); ATF_ERR_OVERFLOW if the product is
+ * >= 2^64. */
 atf_status atf_space_filter_product(atf_space* s, uint64_t* h_count, uint64_t* h_tuples);
 
 /* Random neighbours for simulated annealing ("a random neighbor c' of the

@@ -61,6 +61,7 @@ using u128 = unsigned __int128;
 struct Json {
   enum Kind { NUL, NUM, STR, ARR, OBJ, BOOL } kind = NUL;
   i64 num = 0;
+  bool integral = true;  // NUM without fraction / exponent
   bool b = false;
   std::string str;
   std::vector<Json> arr;
@@ -127,6 +128,14 @@ struct JsonParser {
       if (s[i] == '-') i++;
       while (i < s.size() && isdigit((unsigned char)s[i])) i++;
       j.num = std::stoll(s.substr(st, i - st));
+      // a fraction / exponent (display metadata such as the float values of atfspec.floats):
+      // consumed and marked; a spec field read as an integer rejects it
+      if (i < s.size() && (s[i] == '.' || s[i] == 'e' || s[i] == 'E')) {
+        j.integral = false;
+        while (i < s.size() && (isdigit((unsigned char)s[i]) || s[i] == '.' || s[i] == 'e' || s[i] == 'E' ||
+                                s[i] == '+' || s[i] == '-'))
+          i++;
+      }
     }
     return j;
   }
@@ -191,6 +200,7 @@ static std::vector<i64> materialise(const Json& r) {
     }
   } else if (kind == "set") {
     for (auto& x : r.at("values").arr) {
+      if (x.kind != Json::NUM || !x.integral) throw std::runtime_error("range: set values must be integers");
       for (i64 y : v)
         if (y == x.num) throw std::runtime_error("range: duplicate set value");  // reading #5
       if (x.num < INT32_MIN || x.num > INT32_MAX) throw std::runtime_error("range: value outside int32");
@@ -533,8 +543,11 @@ static int cmd_info(const Spec& s, int threads, bool want_hash) {
     if (r && U > (~(u128)0) / r) Uover = true; else U *= r;
   }
   std::printf("],\"groups\":[");
+  double gen_s = 0;  // O2 generation time (steady clock; spec parsing and printing excluded)
   for (size_t g = 0; g < groups.size(); g++) {
+    const auto tg = std::chrono::steady_clock::now();
     auto res = run_group_parallel(s, groups[g], threads, want_hash);
+    gen_s += std::chrono::duration<double>(std::chrono::steady_clock::now() - tg).count();
     size_t L = groups[g].size();
     std::vector<LevelStats> lv(L);
     u64 n = 0, H = 0;
@@ -558,6 +571,7 @@ static int cmd_info(const Spec& s, int threads, bool want_hash) {
   std::printf("],\"S\":\"%s\",\"unconstrained\":\"%s\"", Sover ? "overflow" : u128_str(S).c_str(),
               Uover ? "overflow" : u128_str(U).c_str());
   if (g_native_check) std::printf(",\"native_mismatch\":%" PRIu64, (u64)g_native_mismatch.load());
+  std::printf(",\"gen_seconds\":%.6f,\"threads\":%d", gen_s, threads);
   std::printf(",\"overflow\":%s}\n", g_overflow ? "true" : "false");
   return 0;
 }
@@ -573,6 +587,7 @@ static int cmd_o1(const Spec& s, const char* out) {
   struct Row { std::vector<u64> key; std::vector<i64> vals; };
   std::vector<Row> rows;
   u64 evaluated = 0;
+  const auto t0 = std::chrono::steady_clock::now();
   if (P == s.params.size() && P > 0) {
     for (;;) {
       for (size_t p = 0; p < P; p++) vals[p] = s.params[p].values[pos[p]];
@@ -596,14 +611,15 @@ static int cmd_o1(const Spec& s, const char* out) {
     }
   }
   std::stable_sort(rows.begin(), rows.end(), [](const Row& a, const Row& b) { return a.key < b.key; });
+  const double o1_s = std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count();
   if (out) {
     FILE* f = std::fopen(out, "wb");
     for (auto& r : rows)
       for (i64 v : r.vals) { int32_t w = (int32_t)v; std::fwrite(&w, 4, 1, f); }
     std::fclose(f);
   }
-  std::printf("{\"S\":%zu,\"evaluated\":%" PRIu64 ",\"overflow\":%s}\n", rows.size(), evaluated,
-              g_overflow ? "true" : "false");
+  std::printf("{\"S\":%zu,\"evaluated\":%" PRIu64 ",\"seconds\":%.6f,\"overflow\":%s}\n", rows.size(), evaluated,
+              o1_s, g_overflow ? "true" : "false");
   return 0;
 }
 

@@ -320,6 +320,11 @@ void* jit_wide_kernel(const LevelArgs& a, int words, const std::vector<int32_t>&
                       const std::vector<uint32_t>& cand_magics);
 int jit_wide_smem(int r, int words);
 int jit_wide_launch(void* kernel, const LevelArgs& a, int words, void* stream);
+// jit.cpp: batched decode of one generated space (A9), specialised (nullptr if NVRTC fails)
+std::string jit_decode_source(const DecodeArgs& a);
+void* jit_decode_kernel(const DecodeArgs& a);
+int jit_decode_launch(void* kernel, const DecodeArgs& a, const uint64_t* idx, const uint64_t* digits, int64_t n,
+                      int32_t* out, int64_t ld, unsigned int* bad, void* stream);
 int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out,
                           int64_t ld, unsigned int* bad_flag, void* stream);
 int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,

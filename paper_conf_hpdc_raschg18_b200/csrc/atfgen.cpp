@@ -171,6 +171,8 @@ struct atf_space {
     uint64_t tot[kMaxTail] = {};  // node count of every tail level
   };
   std::vector<Tail> tails;
+  void* decode_jit = nullptr;   // specialised decoder of the current generation (jit.cpp)
+  bool decode_jit_tried = false;
   // shards
   bool ipc_alloc = false;      // arena chunks from cudaMalloc (exported by CUDA IPC to peer ranks)
   struct PeerMap { int rank; char handle[64]; char* base; };
@@ -1682,7 +1684,7 @@ struct DistDesc {       // where a rank's slice of a level lives
   char handle[64];      // cudaIpcMemHandle_t of the allocation
 };
 struct DistGroup {      // per group, per round
-  uint32_t nd, pad;     // levels completed this round (0, 1 or a tail's nl)
+  uint32_t nd, repl;    // levels completed this round (0, 1 or a tail's nl); replicated level
   uint64_t cnt[kMaxTail];
   DistDesc desc;        // records of the last completed level
 };
@@ -1736,9 +1738,14 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
   std::vector<uint64_t> lo(G, 0), hi(G, 0);      // this rank's parent slice of the frontier
   std::vector<const uint32_t*> frontier(G, s->d_root);
   std::vector<DistGroup> mine(G), all((size_t)world * G);
-  for (size_t g = 0; g < G; g++) {  // level 0: the root (one parent), expanded by rank 0
+  // Small levels are replicated: every rank expands the whole frontier while it costs less than
+  // kReplEvals candidate pairs (no exchange, no copy; the first distributed level takes its
+  // parent slice straight from the local copy).  C5: levels 1-3 replicated, 4-8 distributed.
+  constexpr uint64_t kReplEvals = 1ull << 28;
+  std::vector<char> repl(G, 1);
+  for (size_t g = 0; g < G; g++) {  // level 0: the root (one parent)
     lo[g] = 0;
-    hi[g] = rank == 0 ? 1 : 0;
+    hi[g] = 1;
   }
   for (int round = 0;; round++) {
     char rname[48];
@@ -1861,19 +1868,50 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
       if (!redo) break;
     }
     if (!any_open) break;
-    // exchange: one record per group and rank
+    // exchange: one record per group and rank (skipped when every completed level is replicated:
+    // all ranks take that decision from the same global sizes)
+    bool need_ag = false;
     for (size_t g = 0; g < G; g++) {
-      if (mine[g].nd != 1) continue;
+      mine[g].repl = repl[g];
+      if (mine[g].nd && !repl[g]) need_ag = true;
+      if (mine[g].nd != 1 || repl[g]) continue;
       atf_status e = dist_desc(s, (int)g, s->data[g][k[g]].rec, mine[g].desc);
       if (e) return e;
     }
-    if (ag(mine.data(), all.data(), sizeof(DistGroup) * G, ctx) != 0)
-      return fail(s, ATF_ERR_CUDA, "all-gather callback failed in round %d", round);
+    if (need_ag) {
+      if (ag(mine.data(), all.data(), sizeof(DistGroup) * G, ctx) != 0)
+        return fail(s, ATF_ERR_CUDA, "all-gather callback failed in round %d", round);
+    } else {
+      for (int r = 0; r < world; r++)
+        for (size_t g = 0; g < G; g++) all[(size_t)r * G + g] = mine[g];
+    }
     for (size_t g = 0; g < G; g++) {
       const uint32_t nd = mine[g].nd;
       if (!nd) continue;
       for (int r = 0; r < world; r++)
         if (all[(size_t)r * G + g].nd != nd) return fail(s, ATF_ERR_STATE, "ranks out of step (group %zu)", g);
+      if (repl[g]) {  // every rank holds the whole level(s)
+        for (uint32_t d = 0; d < nd; d++) {
+          LevelData& ld = s->data[g][k[g] + d];
+          ld.offset = 0;
+          if (d + 1 < nd) { ld.csr_offset = 0; ld.csr_n = ld.n; }
+          F[g] = mine[g].cnt[d];
+        }
+        k[g] += (int)nd;
+        if (k[g] >= (int)s->groups[g].levels.size()) continue;
+        const uint64_t Fg = F[g];
+        const LevelData& ld = s->data[g][k[g] - 1];
+        if (Fg * (uint64_t)s->groups[g].levels[k[g]].r >= kReplEvals) {
+          repl[g] = 0;  // distribute from here on: this rank's slice of the local copy
+          lo[g] = (uint64_t)((unsigned __int128)Fg * rank / world);
+          hi[g] = (uint64_t)((unsigned __int128)Fg * (rank + 1) / world);
+        } else {
+          lo[g] = 0;
+          hi[g] = Fg;
+        }
+        frontier[g] = ld.rec ? ld.rec + lo[g] * s->groups[g].words : s->d_root;
+        continue;
+      }
       // global offsets of this rank's part of every completed level; CSR entries -> global
       for (uint32_t d = 0; d < nd; d++) {
         uint64_t before = 0, tot = 0;
@@ -1934,6 +1972,8 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
 
 static atf_status generate_impl(atf_space* s) {
   NvtxRange nvtx("atf_space_generate");
+  s->decode_jit = nullptr;  // the decoder's immediates (group sizes) belong to one generation
+  s->decode_jit_tried = false;
   atf_status e = plan(s);
   if (e) return e;
   if ((e = ensure_device(s))) return e;
@@ -2361,8 +2401,15 @@ static atf_status decode_common(const atf_space* cs, const uint64_t* idx, const 
   DecodeArgs a;
   make_decode_args(s, a);
   CUDA_TRY(s, cudaMemsetAsync(s->d_bad, 0, 4, st));
-  int ce = idx ? launch_decode_indices(a, idx, n, out, ld, s->d_bad, st)
-               : launch_decode_digits(a, digits, n, out, ld, s->d_bad, st);
+  // large batches: the decoder specialised for this space (NVRTC, compiled once per space)
+  if (n >= (1 << 18) && !(s->opts.flags & ATF_FLAG_NO_JIT) && !s->decode_jit_tried) {
+    s->decode_jit = jit_decode_kernel(a);
+    s->decode_jit_tried = true;
+  }
+  int ce = (n >= (1 << 18) && s->decode_jit && !(s->opts.flags & ATF_FLAG_NO_JIT))
+               ? jit_decode_launch(s->decode_jit, a, idx, digits, n, out, ld, s->d_bad, st)
+               : (idx ? launch_decode_indices(a, idx, n, out, ld, s->d_bad, st)
+                      : launch_decode_digits(a, digits, n, out, ld, s->d_bad, st));
   if (ce) return fail(s, ATF_ERR_CUDA, "decode launch: %s", cudaGetErrorString((cudaError_t)ce));
   // the bad-index flag is read back only when someone could be out of range: always
   // check (one 4-byte copy) — it costs a sync, so the flag copy is async and we

@@ -479,34 +479,34 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   }
   s += "  }\n}\n";
   // ---- emit: lane = frontier node, depth-first (like the count), output staged per warp.
-  // Each lane recounts its subtree (cnt_d), a warp scan per level gives its nodes' tile-local
-  // positions; the lane then writes its subtree depth-first — a node's level-d descendants come
-  // out in canonical order — records and CSR entries (first child = the child level's running
-  // position) into the warp's shared-memory staging area, which the warp then copies out as
-  // coalesced vectors (one contiguous run per level and per CSR array).  A tile whose output
-  // exceeds the staging area (the sizes are known before writing) writes straight to global.
-  constexpr int kStage = 12288;  // staging bytes per warp
+  // Each lane recounts its subtree (cnt_d); warp scans give its nodes' tile-local positions per
+  // level (a node's level-d descendants come out of a depth-first walk in canonical order).  The
+  // warp then writes the tile in "parts": runs of consecutive lanes whose output (records, and
+  // CSR entries as u32 offsets from the child level's tile base) fits the warp's staging area;
+  // the lanes of a part write their subtrees into shared memory, the warp copies every level's
+  // run out as coalesced words.  A single lane whose subtree alone exceeds the area writes
+  // straight to global memory.
+  constexpr int kStage = 8192;  // staging bytes per warp
   if (warp_bytes) *warp_bytes = kStage;
-  const std::string NLs = std::to_string(nl), NCs = std::to_string(NC);
+  const std::string NLs = std::to_string(nl), NCs = std::to_string(NC), RB = std::to_string(W * 4);
   for (int d = nl - 1; d >= 0; d--) {
     const std::string ds = std::to_string(d);
     s += "__device__ __forceinline__ void dfs" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cur, "
-         "const u64* base, unsigned char* sm, bool staged, const u32* roff, const u32* coff) {\n";
+         "const u64* base, const u32* pb, unsigned char* sm, bool staged, const u32* roff, const u32* coff) {\n";
     s += "  u32 m = tmask" + ds + "(a, w, nc);\n";
     s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
     s += child(d, "w", "cw", "    ");
     s += "    const u32 slot = cur[" + ds + "]++;\n";
-    s += "    if (staged) {\n      u32* dst = reinterpret_cast<u32*>(sm + roff[" + ds + "]) + slot * " + Ws + ";\n";
+    s += "    if (staged) {\n      u32* dst = reinterpret_cast<u32*>(sm + roff[" + ds + "]) + (slot - pb[" + ds + "]) * " + Ws + ";\n";
     for (int w = 0; w < W; w++) s += "      dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
     s += "    } else {\n      u32* dst = a.rec[" + ds + "] + (base[" + ds + "] + slot) * " + Ws + ";\n";
     for (int w = 0; w < W; w++) s += "      dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
     s += "    }\n";
     if (d + 1 < nl) {
       const std::string d1 = std::to_string(d + 1);
-      s += "    const u64 fc = base[" + d1 + "] + cur[" + d1 + "];\n";
-      s += "    if (staged) *reinterpret_cast<u64*>(sm + coff[" + ds + "] + slot * 8u) = fc;\n";
-      s += "    else a.csr[" + d1 + "][base[" + ds + "] + slot] = fc;\n";
-      s += "    dfs" + d1 + "(a, cw, nc, cur, base, sm, staged, roff, coff);\n";
+      s += "    if (staged) reinterpret_cast<u32*>(sm + coff[" + ds + "])[slot - pb[" + ds + "]] = cur[" + d1 + "];\n";
+      s += "    else a.csr[" + d1 + "][base[" + ds + "] + slot] = base[" + d1 + "] + cur[" + d1 + "];\n";
+      s += "    dfs" + d1 + "(a, cw, nc, cur, base, pb, sm, staged, roff, coff);\n";
     }
     s += "  }\n}\n";
   }
@@ -522,29 +522,41 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "    for (int i = 0; i < " + Ws + "; i++) w[i] = valid ? __ldg(a.parent_rec + nd * " + Ws + " + i) : 0u;\n";
   s += "    u32 nc[" + NCs + "];\n    u32 cnt[" + NLs + "] = {};\n";
   s += "    if (valid) { tnc(a, w, nc); cnt0(a, w, nc, cnt); }\n";
-  s += "    u32 cur[" + NLs + "], T[" + NLs + "];\n    u64 base[" + NLs + "];\n    u32 need = 0;\n";
+  s += "    u32 off[" + NLs + "];\n    u64 base[" + NLs + "];\n    u32 bytes = 0;\n";
   s += "#pragma unroll\n    for (int d = 0; d < " + NLs + "; d++) {\n";
   s += "      u32 incl = cnt[d];\n#pragma unroll\n      for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
        "if (lane >= o) incl += y; }\n";
-  s += "      T[d] = __shfl_sync(0xffffffffu, incl, 31);\n      cur[d] = incl - cnt[d];\n";
-  s += "      base[d] = a.tile_base[(u64)d * (a.n_tiles + 1) + tile];\n";
-  s += "      need += T[d] * " + std::to_string(W * 4) + "u + (d + 1 < " + NLs + " ? T[d] * 8u : 0u);\n    }\n";
-  // frontier CSR
-  s += "    if (valid) a.csr[0][nd] = base[0] + cur[0];\n";
-  // staging layout: CSR regions first (8-byte aligned), then records
-  s += "    const bool staged = need <= " + std::to_string(kStage) + "u;\n    u32 roff[" + NLs + "], coff[" + NLs + "];\n";
-  s += "    { u32 o = 0;\n      for (int d = 0; d + 1 < " + NLs + "; d++) { coff[d] = o; o += T[d] * 8u; }\n";
-  s += "      coff[" + std::to_string(nl - 1) + "] = o;\n      for (int d = 0; d < " + NLs + "; d++) { roff[d] = o; o += T[d] * " +
-       std::to_string(W * 4) + "u; } }\n";
-  s += "    if (valid) dfs0(a, w, nc, cur, base, sm, staged, roff, coff);\n";
-  s += "    if (staged) {\n      __syncwarp();\n";
-  // copy records (u32 granularity keeps any alignment of roff) and CSR (u64)
-  s += "      for (int d = 0; d < " + NLs + "; d++) {\n";
-  s += "        const u32* src = reinterpret_cast<const u32*>(sm + roff[d]);\n        u32* dst = a.rec[d] + base[d] * " + Ws + ";\n";
-  s += "        const u32 n = T[d] * " + Ws + "u;\n#pragma unroll 4\n        for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
-  s += "        if (d + 1 < " + NLs + ") {\n          const u64* cs = reinterpret_cast<const u64*>(sm + coff[d]);\n";
-  s += "          u64* cd = a.csr[d + 1] + base[d];\n#pragma unroll 4\n          for (u32 v = lane; v < T[d]; v += 32) cd[v] = cs[v];\n        }\n";
-  s += "      }\n      __syncwarp();\n    }\n  }\n}\n";
+  s += "      off[d] = incl - cnt[d];\n      base[d] = a.tile_base[(u64)d * (a.n_tiles + 1) + tile];\n";
+  s += "      bytes += cnt[d] * (" + RB + "u + (d + 1 < " + NLs + " ? 4u : 0u));\n    }\n";
+  s += "    if (valid) a.csr[0][nd] = base[0] + off[0];\n";
+  // inclusive byte prefix per lane
+  s += "    u32 bincl = bytes;\n#pragma unroll\n    for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, bincl, o); "
+       "if (lane >= o) bincl += y; }\n";
+  s += "    for (int p0 = 0; p0 < 32;) {\n";
+  s += "      const u32 b0 = p0 ? __shfl_sync(0xffffffffu, bincl, p0 - 1) : 0u;\n";
+  s += "      const unsigned fit = __ballot_sync(0xffffffffu, lane >= p0 && bincl - b0 <= " + std::to_string(kStage) + "u);\n";
+  s += "      const int p1 = fit ? 32 - __clz(fit) : p0 + 1;  // lanes [p0, p1)\n";
+  s += "      const bool staged = fit != 0u;\n";
+  s += "      u32 pb[" + NLs + "], pe[" + NLs + "], roff[" + NLs + "], coff[" + NLs + "];\n";
+  s += "      u32 o = 0;\n";
+  s += "#pragma unroll\n      for (int d = 0; d < " + NLs + "; d++) {\n";
+  s += "        pb[d] = __shfl_sync(0xffffffffu, off[d], p0);\n";
+  s += "        const u32 last = __shfl_sync(0xffffffffu, off[d] + cnt[d], p1 - 1);\n        pe[d] = last;\n";
+  s += "        if (d + 1 < " + NLs + ") { coff[d] = o; o += (last - pb[d]) * 4u; }\n      }\n";
+  s += "      o = (o + 15u) & ~15u;\n";
+  s += "#pragma unroll\n      for (int d = 0; d < " + NLs + "; d++) { roff[d] = o; o += (pe[d] - pb[d]) * " + RB + "u; }\n";
+  s += "      if (lane >= p0 && lane < p1 && valid) {\n        u32 cur[" + NLs + "];\n";
+  s += "#pragma unroll\n        for (int d = 0; d < " + NLs + "; d++) cur[d] = off[d];\n";
+  s += "        dfs0(a, w, nc, cur, base, pb, sm, staged, roff, coff);\n      }\n";
+  s += "      if (staged) {\n        __syncwarp();\n";
+  s += "#pragma unroll\n        for (int d = 0; d < " + NLs + "; d++) {\n";
+  s += "          const u32 n = (pe[d] - pb[d]) * " + Ws + "u;\n";
+  s += "          const u32* src = reinterpret_cast<const u32*>(sm + roff[d]);\n          u32* dst = a.rec[d] + (base[d] + pb[d]) * " + Ws + ";\n";
+  s += "#pragma unroll 4\n          for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
+  s += "          if (d + 1 < " + NLs + ") {\n            const u32* cs = reinterpret_cast<const u32*>(sm + coff[d]);\n";
+  s += "            u64* cd = a.csr[d + 1] + base[d] + pb[d];\n            const u64 cb = base[d + 1 < " + NLs + " ? d + 1 : d];\n";
+  s += "#pragma unroll 4\n            for (u32 v = lane; v < pe[d] - pb[d]; v += 32) cd[v] = cb + cs[v];\n          }\n";
+  s += "        }\n        __syncwarp();\n      }\n      p0 = p1;\n    }\n  }\n}\n";
   return s;
 }
 
@@ -749,6 +761,92 @@ std::string gen_wide_source(const LevelArgs& a, int W, const std::vector<int32_t
   s += "    if (staged && sgb + total <= a.stash_cap) {\n      __syncwarp();\n";
   s += "      for (u32 v = lane; v < total * " + Ws + "u; v += 32) a.stash[sgb * " + Ws + " + v] = s_st[v];\n    }\n";
   s += "    __syncwarp();\n  }\n}\n";
+  return s;
+}
+
+// ---------------------------------------------------------------- batched decode
+// The decoder of one generated space (A9): group sizes and their multiply-high
+// magics, record widths, field positions and output columns as immediates, so an index costs
+// its mixed-radix digits (multiply-high + at most two corrections per group), one leaf gather
+// per group (ld.global.cg: 32-byte sectors from L2, no 128-byte L1 line fills for a random
+// 8-byte read) and one table load + store per parameter.
+struct DecodeJitArgs {
+  const uint64_t* idx;
+  const uint64_t* digits;
+  int64_t n;
+  int32_t* out;
+  int64_t ld;
+  unsigned int* bad;
+  const uint32_t* leaves[kMaxGroups];
+  const int32_t* range[kMaxLevels];
+};
+
+std::string gen_decode_source(const DecodeArgs& a) {
+  std::string s = kPrelude;
+  s += "struct DecodeJitArgs { const u64* idx; const u64* digits; i64 n; i32* out; i64 ld; u32* bad; "
+       "const u32* leaves[" + std::to_string(kMaxGroups) + "]; const i32* range[" + std::to_string(kMaxLevels) + "]; };\n";
+  s += "__device__ __forceinline__ uint2 ldcg2(const u32* p) { uint2 v; asm volatile(\"ld.global.cg.v2.u32 {%0,%1}, [%2];\" "
+       ": \"=r\"(v.x), \"=r\"(v.y) : \"l\"(p)); return v; }\n";
+  s += "__device__ __forceinline__ uint4 ldcg4(const u32* p) { uint4 v; asm volatile(\"ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];\" "
+       ": \"=r\"(v.x), \"=r\"(v.y), \"=r\"(v.z), \"=r\"(v.w) : \"l\"(p)); return v; }\n";
+  s += "__device__ __forceinline__ u32 ldcg1(const u32* p) { u32 v; asm volatile(\"ld.global.cg.u32 %0, [%1];\" : \"=r\"(v) : \"l\"(p)); return v; }\n";
+  unsigned __int128 S = 1;
+  bool fits = true;
+  for (int g = 0; g < a.n_groups; g++) {
+    S *= a.gsize[g];
+    if (S >> 64) fits = false;
+  }
+  char buf[64];
+  s += "extern \"C\" __global__ void __launch_bounds__(256) atf_decode_jit(const __grid_constant__ DecodeJitArgs a) {\n";
+  s += "  for (i64 i = (i64)blockIdx.x * blockDim.x + threadIdx.x; i < a.n; i += (i64)gridDim.x * blockDim.x) {\n";
+  s += "    bool valid = true;\n";
+  for (int g = 0; g < a.n_groups; g++) s += "    u64 d" + std::to_string(g) + ";\n";
+  s += "    if (a.idx) {\n      u64 rem = __ldcs(a.idx + i);\n";
+  snprintf(buf, sizeof buf, "0x%llxull", (unsigned long long)(uint64_t)S);
+  s += fits ? "      valid = rem < " + std::string(buf) + ";\n" : "      valid = false;\n";
+  for (int g = a.n_groups - 1; g >= 0; g--) {
+    const std::string gs = std::to_string(g);
+    char sz[32], mg[32];
+    snprintf(sz, sizeof sz, "0x%llxull", (unsigned long long)a.gsize[g]);
+    snprintf(mg, sizeof mg, "0x%llxull", (unsigned long long)a.gmagic[g]);
+    if (a.gsize[g] == 1) { s += "      d" + gs + " = 0;\n"; continue; }
+    if (a.gsize[g] == 0) { s += "      d" + gs + " = 0;\n"; continue; }
+    s += "      { u64 q = __umul64hi(rem, " + std::string(mg) + "); u64 r = rem - q * " + sz + ";\n";
+    s += "        if (r >= " + std::string(sz) + ") { q++; r -= " + sz + "; }\n";
+    s += "        if (r >= " + std::string(sz) + ") { q++; r -= " + sz + "; }\n";
+    s += "        d" + gs + " = r; rem = q; }\n";
+  }
+  s += "    } else {\n";
+  for (int g = 0; g < a.n_groups; g++) {
+    const std::string gs = std::to_string(g);
+    char sz[32];
+    snprintf(sz, sizeof sz, "0x%llxull", (unsigned long long)a.gsize[g]);
+    s += "      d" + gs + " = __ldcs(a.digits + (i64)" + gs + " * a.n + i); valid = valid && d" + gs + " < " + sz + ";\n";
+  }
+  s += "    }\n";
+  s += "    if (!valid) {\n      for (int p = 0; p < " + std::to_string(a.n_params) +
+       "; p++) a.out[(i64)p * a.ld + i] = (i32)0x80000000;\n      atomicOr(a.bad, 1u);\n      continue;\n    }\n";
+  for (int g = 0; g < a.n_groups; g++) {
+    const std::string gs = std::to_string(g);
+    const int W = a.words[g];
+    s += "    {\n      const u32* rp = a.leaves[" + gs + "] + d" + gs + " * " + std::to_string(W) + "ull;\n";
+    if (W == 1) s += "      const u32 w0 = ldcg1(rp);\n";
+    else if (W == 2) s += "      const uint2 v = ldcg2(rp); const u32 w0 = v.x, w1 = v.y;\n";
+    else {
+      s += "      const uint4 v = ldcg4(rp); const u32 w0 = v.x, w1 = v.y, w2 = v.z, w3 = v.w;\n";
+      if (W == 8) s += "      const uint4 u = ldcg4(rp + 4); const u32 w4 = u.x, w5 = u.y, w6 = u.z, w7 = u.w;\n";
+    }
+    for (int l = a.lvl_begin[g]; l < a.lvl_begin[g + 1]; l++) {
+      const uint32_t bits = (uint32_t)a.lvl_bits[l];
+      std::string pos = bits ? "((w" + std::to_string(a.lvl_word[l]) + " >> " + std::to_string(a.lvl_shift[l]) + ") & " +
+                                   hex(bits >= 32 ? 0xffffffffu : ((1u << bits) - 1u)) + ")"
+                             : std::string("0u");
+      s += "      a.out[(i64)" + std::to_string(a.lvl_param[l]) + " * a.ld + i] = __ldg(a.range[" + std::to_string(l) + "] + " +
+           pos + ");\n";
+    }
+    s += "    }\n";
+  }
+  s += "  }\n}\n";
   return s;
 }
 
@@ -993,6 +1091,41 @@ int jit_wide_launch(void* kernel, const LevelArgs& a, int words, void* stream) {
   void* args[] = {&j};
   return (int)cudaLaunchKernel((const void*)kernel, dim3((unsigned)grid), dim3(256), args, (size_t)smem,
                                (cudaStream_t)stream);
+}
+
+
+// ---- batched decode: specialised kernel of a generated space (nullptr: generic kernel)
+std::string jit_decode_source(const DecodeArgs& a) { return gen_decode_source(a); }
+
+void* jit_decode_kernel(const DecodeArgs& a) {
+  const std::string src = gen_decode_source(a);
+  cudaKernel_t k = compile(src, "atf_decode_jit");
+  return (void*)k;
+}
+
+int jit_decode_launch(void* kernel, const DecodeArgs& a, const uint64_t* idx, const uint64_t* digits, int64_t n,
+                      int32_t* out, int64_t ld, unsigned int* bad, void* stream) {
+  DecodeJitArgs j;
+  std::memset(&j, 0, sizeof j);
+  j.idx = idx;
+  j.digits = digits;
+  j.n = n;
+  j.out = out;
+  j.ld = ld;
+  j.bad = bad;
+  for (int g = 0; g < a.n_groups; g++) j.leaves[g] = a.leaves[g];
+  for (int l = 0; l < a.lvl_begin[a.n_groups]; l++) j.range[l] = a.lvl_range[l];
+  static int sms = 0;
+  if (!sms) {
+    int dev = 0;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  }
+  int64_t blocks = (n + 255) / 256;
+  if (blocks > (int64_t)sms * 8) blocks = (int64_t)sms * 8;
+  if (blocks < 1) blocks = 1;
+  void* args[] = {&j};
+  return (int)cudaLaunchKernel((const void*)kernel, dim3((unsigned)blocks), dim3(256), args, 0, (cudaStream_t)stream);
 }
 
 }  // namespace atf

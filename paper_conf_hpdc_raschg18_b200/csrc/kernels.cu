@@ -224,16 +224,17 @@ __global__ void decode_kernel(const __grid_constant__ DecodeArgs a, const uint64
       const uint32_t* rp = a.leaves[g] + d * (uint64_t)W;
       // record words in registers (static indices only: no local-memory array)
       uint32_t rec[8] = {0, 0, 0, 0, 0, 0, 0, 0};
+      // random gather: L2 only (32-byte sectors), no 128-byte L1 line fill
       if (W == 1) {
-        rec[0] = __ldg(rp);
+        rec[0] = __ldcg(rp);
       } else if (W == 2) {
-        const uint2 v = __ldg(reinterpret_cast<const uint2*>(rp));
+        const uint2 v = __ldcg(reinterpret_cast<const uint2*>(rp));
         rec[0] = v.x; rec[1] = v.y;
       } else {
-        const uint4 v = __ldg(reinterpret_cast<const uint4*>(rp));
+        const uint4 v = __ldcg(reinterpret_cast<const uint4*>(rp));
         rec[0] = v.x; rec[1] = v.y; rec[2] = v.z; rec[3] = v.w;
         if (W == 8) {
-          const uint4 u = __ldg(reinterpret_cast<const uint4*>(rp) + 1);
+          const uint4 u = __ldcg(reinterpret_cast<const uint4*>(rp) + 1);
           rec[4] = u.x; rec[5] = u.y; rec[6] = u.z; rec[7] = u.w;
         }
       }

@@ -304,3 +304,20 @@ def test_new_entry_points_validate_without_a_gpu(L):
         assert LL.atf_space_filter_product(sp, C.byref(cnt), C.byref(tot)) == -7  # OVERFLOW
     finally:
         LL.atf_space_destroy(sp)
+
+
+def test_float_parameters_are_monotone_positions():
+    """NEXT-3 floats by position (atfspec.floats / float_interval): positions 0..n-1 in the listed
+    order; for an interval, position order = value order, so X <= float_code(v) selects the
+    values <= v; the oracle enumerates the positions like any SET."""
+    from oracle import run as orc
+    r = A.float_interval(0.1, 1.0, 0.1)
+    assert len(r["values"]) == 10 and r["values"] == list(range(10))
+    vals = r["names"]
+    assert all(a < b for a, b in zip(vals, vals[1:]))
+    s = A.Spec("f")
+    s.add("t", r, A.X <= A.float_code(r, vals[4]))
+    d, rows = orc.o1(s)
+    assert [vals[int(x)] for x in rows[:, 0]] == [v for v in vals if v <= vals[4]]
+    with pytest.raises(ValueError):
+        A.floats(0.5, 0.5)

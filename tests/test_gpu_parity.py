@@ -792,8 +792,20 @@ def _dist_check(Space, spec, world, flags=0):
                 rec, csr = sp.level_tensors(g, k)
                 parts.append((v["offset"], rec))
                 if csr is not None:
-                    cparts.append((v["csr_offset"], csr))
+                    cparts.append((v["csr_offset"], csr, v["offset"], rec.shape[0]))
+            if all(off == 0 and r.shape[0] == wrec.shape[0] for off, r in parts) and world > 1 and wrec.shape[0]:
+                # a replicated (small) level: every rank holds all of it
+                for _, r in parts:
+                    assert torch.equal(r, wrec), (g, k)
+                for c in cparts:
+                    if c[0] == 0 and c[1].shape[0] == wrec.shape[0] + 1:
+                        assert torch.equal(c[1], wcsr), ("csr", g, k)
+                if all(c[0] == 0 and c[1].shape[0] == wrec.shape[0] + 1 for c in cparts):
+                    continue
+                # the first distributed level's parents: slices of the replicated level
             parts.sort(key=lambda t: t[0])
+            if all(off == 0 and r.shape[0] == wrec.shape[0] for off, r in parts) and world > 1:
+                parts = parts[:1]
             pos = 0
             for off, rec in parts:
                 assert off == pos, (g, k)
@@ -801,12 +813,14 @@ def _dist_check(Space, spec, world, flags=0):
             assert torch.equal(torch.cat([r for _, r in parts]), wrec), (g, k)
             if wcsr is not None:
                 cparts.sort(key=lambda t: t[0])
-                got = torch.cat([c[:-1] for _, c in cparts] + [cparts[-1][1][-1:]])
+                got = torch.cat([c[1][:-1] for c in cparts] + [cparts[-1][1][-1:]])
                 assert torch.equal(got, wcsr), ("csr", g, k)
-                # balance: every rank's parent slice is floor/ceil of f_k / world
+                # balance: a rank's parent slice (CSR not covering exactly its own nodes, i.e. not
+                # inside a fused tail) is floor/ceil of f_k / world
                 n = wrec.shape[0]
-                for _, c in cparts:
-                    assert abs((c.shape[0] - 1) - n / world) <= 1, (g, k)
+                for c in cparts:
+                    if (c[0], c[1].shape[0] - 1) != (c[2], c[3]):
+                        assert abs((c[1].shape[0] - 1) - n / world) <= 1, (g, k)
     finally:
         for sp in spaces:
             sp.close()
@@ -873,8 +887,35 @@ dist.destroy_process_group()
         for g in range(one.num_groups()):
             for k in range(one.num_levels(g)):
                 rec, csr = one.level_tensors(g, k)
+                rec = rec.cpu().numpy()
                 parts = sorted([res[r][f"r{g}_{k}"] for r in range(2)], key=lambda t: t[0])
-                assert np.array_equal(np.concatenate([p for _, p in parts]), rec.cpu().numpy())
+                if all(off == 0 and p.shape[0] == rec.shape[0] for off, p in parts):   # replicated level
+                    assert all(np.array_equal(p, rec) for _, p in parts)
+                else:
+                    assert np.array_equal(np.concatenate([p for _, p in parts]), rec)
                 if csr is not None:
+                    csr = csr.cpu().numpy()
                     cp = sorted([res[r][f"c{g}_{k}"] for r in range(2)], key=lambda t: t[0])
-                    assert np.array_equal(np.concatenate([cp[0][1][:-1], cp[1][1]]), csr.cpu().numpy())
+                    if all(off == 0 and c.shape[0] == csr.shape[0] for off, c in cp):
+                        assert all(np.array_equal(c, csr) for _, c in cp)
+                    else:
+                        assert np.array_equal(np.concatenate([cp[0][1][:-1], cp[1][1]]), csr)
+
+
+def test_float_parameters_by_position(Space):
+    """Float-valued parameters (NEXT-3, "float") by position index: a tolerance in
+    float_interval(0.25, 2.0, 0.25) constrained through its (monotone) positions together with
+    integer parameters; the space equals the oracle's (which sees the same positions), and
+    to_named gives the float values."""
+    s = A.Spec("float_space")
+    tol = A.float_interval(0.25, 2.0, 0.25)
+    s.add("TS", A.interval(1, 64), A.divides(64))
+    s.add("TOL", tol, (A.X <= A.float_code(tol, 1.0)) | (s.P("TS") >= 16))
+    s.add("UNROLL", A.interval(1, 8), A.divides(s.P("TS")) & (A.X * (s.P("TOL") + 1) <= 16))
+    _check_against_oracle(Space, s)
+    with Space(s) as sp:
+        sp.generate()
+        named = sp.to_named(sp.decode(torch.arange(sp.size(), dtype=torch.int64, device="cuda")))
+        assert all(isinstance(r["TOL"], float) for r in named)
+        assert all(r["TOL"] <= 1.0 or r["TS"] >= 16 for r in named)
+        assert {r["TOL"] for r in named} == {0.25 * i for i in range(1, 9)}
