@@ -117,6 +117,10 @@ typedef struct {
                                      divisibility filter by their |x| bounds (x | n needs
                                      |x| <= |n|) without evaluating their pairs; the result is
                                      identical, the evaluated-pair count is not */
+#define ATF_FLAG_NO_REPLAY 256u  /* every generation sizes its levels one round at a time (a host
+                                     synchronisation per level round) instead of replaying the
+                                     previous generation's level sizes (one synchronisation,
+                                     totals verified; DESIGN.md §5 "Steady state")              */
 #define ATF_FLAG_NO_TAIL 128u     /* expand a group's trailing narrow levels one at a time instead
                                      of the fused narrow tail (two launches for up to 4 levels,
                                      DESIGN.md §5); kept for parity coverage and A/B timing    */

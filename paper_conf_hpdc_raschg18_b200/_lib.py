@@ -27,6 +27,7 @@ ATF_RANGE_INTERVAL, ATF_RANGE_POW2, ATF_RANGE_SET, ATF_RANGE_GEN = 0, 1, 2, 3
 ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT, ATF_FLAG_SERIAL_GROUPS = 1, 2, 8, 16, 32
 ATF_FLAG_NO_SEG_BOUNDS = 64
 ATF_FLAG_NO_TAIL = 128
+ATF_FLAG_NO_REPLAY = 256
 
 
 class atf_range(C.Structure):

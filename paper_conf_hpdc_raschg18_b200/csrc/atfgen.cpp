@@ -95,6 +95,8 @@ struct GroupPlan {
 struct Chunk {
   char* p = nullptr;
   size_t size = 0, used = 0;
+  bool has_ipc = false;  // ipc handle exported (generate_dist)
+  char ipc[64];
 };
 
 struct LevelData {
@@ -171,6 +173,13 @@ struct atf_space {
     uint64_t tot[kMaxTail] = {};  // node count of every tail level
   };
   std::vector<Tail> tails;
+  // replay (DESIGN.md §5 "Steady state"): the level sizes of the last complete single-GPU
+  // generation; the next generation of the space sizes every allocation and launch from them
+  // and synchronises once, then verifies every level's total against them
+  std::vector<std::vector<uint64_t>> replay_f;
+  bool replay_ok = false;
+  unsigned long long* d_replay = nullptr;  // per round: [totals u64 | ovf u32] of every group
+  size_t replay_cap = 0;                   // rounds
   void* decode_jit = nullptr;   // specialised decoder of the current generation (jit.cpp)
   bool decode_jit_tried = false;
   // shards
@@ -1073,6 +1082,10 @@ static void release_device(atf_space* s) {
   s->d_range.clear();
   s->d_sorted.clear();
   dfree(s, s->d_status, s->status_cap * 8);
+  dfree(s, (char*)s->d_replay, s->replay_cap * 12 * kMaxGroups);
+  s->d_replay = nullptr;
+  s->replay_cap = 0;
+  s->replay_ok = false;
   for (auto& b : s->gb) {
     dfree(s, b.scratch, b.scratch_cap);
     dfree(s, (char*)b.stash, b.stash_cap);
@@ -1140,7 +1153,7 @@ static void fill_level_ptrs(atf_space* s, const LevelPlan& lp, LevelArgs& a) {
 }
 
 static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parents, uint64_t n_parents, Pending& pd,
-                              bool own_stream) {
+                              bool own_stream, uint64_t known = UINT64_MAX) {
   GroupPlan& gp = s->groups[g];
   LevelPlan& lp = gp.levels[k];
   cudaStream_t st = (cudaStream_t)s->opts.stream;  // allocations, memsets
@@ -1233,6 +1246,7 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     est = std::min<uint64_t>(exact, 16 * n_parents + 1024);
   }
   est = std::min<uint64_t>(est, (4ull << 30) / (gp.words * 4));  // at most 4 GB up front
+  if (known != UINT64_MAX) est = known;  // replay: the exact size from the previous generation
   int which = -1;
   size_t tail = arena_tail(s, g, &which);
   const size_t want = std::max<size_t>((size_t)est * gp.words * 4, (size_t)gp.words * 4 * 64);
@@ -1244,6 +1258,10 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   size_t off = (c.used + 255) & ~(size_t)255;
   uint32_t* child = (uint32_t*)(c.p + off);
   uint64_t cap = (c.size - off) / (gp.words * 4);
+  if (known != UINT64_MAX) {  // replay: reserve now (no sync before the next level is queued)
+    cap = known;
+    c.used = off + ((known * gp.words * 4 + 255) & ~(uint64_t)255);
+  }
   a.child_rec = child;
   a.child_cap = cap;
   a.csr = (uint64_t*)csr;
@@ -1667,6 +1685,119 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
   return ATF_OK;
 }
 
+// ---------------------------------------------------------------- replay
+// Steady-state generation of a space generated before (the bench's timed steps, a service
+// regenerating the same spec): every level's size is the previous generation's, so allocations
+// and launch geometry are exact up front and all level rounds are queued without a host sync
+// (the per-round totals are copied into a device log); one synchronisation at the end, then
+// every level's total and overflow flag is checked against the expected values.  The device
+// still evaluates every pair and writes every record.  Returns ATF_ERR_STATE on any mismatch
+// (the caller then regenerates level by level).
+static atf_status run_levels_replay(atf_space* s) {
+  NvtxRange nvtx("atf replay");
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  const size_t G = s->groups.size();
+  int max_rounds = 0;
+  for (size_t g = 0; g < G; g++) max_rounds = std::max(max_rounds, (int)s->groups[g].levels.size() + 1);
+  if ((size_t)max_rounds > s->replay_cap) {
+    dfree(s, (char*)s->d_replay, s->replay_cap * 12 * kMaxGroups);
+    s->replay_cap = (size_t)max_rounds;
+    s->d_replay = (unsigned long long*)dalloc(s, s->replay_cap * 12 * kMaxGroups);
+    if (!s->d_replay) { s->replay_cap = 0; return fail(s, ATF_ERR_OOM, "replay log"); }
+  }
+  std::vector<int> k(G, 0);
+  std::vector<const uint32_t*> frontier(G, s->d_root);
+  std::vector<uint64_t> fsize(G, 1);
+  struct Expect { int round, g; uint64_t total; };
+  std::vector<Expect> expect;
+  std::vector<std::pair<int, int>> timed;  // (g, k) single levels with timing events
+  std::vector<int> tails_done;
+  int round = 0;
+  for (;; round++) {
+    int active = 0;
+    for (size_t g = 0; g < G; g++)
+      if (k[g] < (int)s->groups[g].levels.size() && fsize[g] > 0 && s->groups[g].levels[k[g]].r > 0) active++;
+    bool any = false;
+    std::vector<Pending> pend;
+    if (active) CUDA_TRY(s, cudaMemsetAsync(s->d_totals, 0, 16 * kMaxGroups, st));
+    if (active && (s->opts.flags & ATF_FLAG_TIMING)) CUDA_TRY(s, cudaMemsetAsync(s->d_pairs, 0, 8 * kMaxGroups, st));
+    for (size_t g = 0; g < G; g++) {
+      const int L = (int)s->groups[g].levels.size();
+      if (k[g] >= L) continue;
+      any = true;
+      if (fsize[g] == 0 || s->groups[g].levels[k[g]].r == 0) {  // as run_levels: all deeper levels empty
+        for (int kk = k[g]; kk < L; kk++) {
+          LevelData& d = s->data[g][kk];
+          d.rec = nullptr;
+          d.n = 0;
+          d.evals = (kk == k[g]) ? fsize[g] * (uint64_t)s->groups[g].levels[kk].r : 0;
+          d.pairs = d.evals;
+          if (kk > 0 && kk == k[g] && fsize[g] > 0) {
+            atf_status e = ATF_OK;
+            char* csr = arena_take(s, (int)g, (fsize[g] + 1) * 8, &e);
+            if (!csr) return e ? e : fail(s, ATF_ERR_OOM, "csr");
+            CUDA_TRY(s, cudaMemsetAsync(csr, 0, (fsize[g] + 1) * 8, st));
+            s->data[g][kk - 1].csr = (uint64_t*)csr;
+          }
+        }
+        k[g] = L;
+        continue;
+      }
+      Pending pd;
+      atf_status e;
+      auto& T = s->tails[g];
+      if (T.phase == 1) {
+        if ((e = queue_tail_emit(s, (int)g, pd, active > 1))) return e;
+        tails_done.push_back((int)g);
+        k[g] = L;
+      } else if (k[g] == tail_start(s, (int)g)) {
+        if ((e = queue_tail_count(s, (int)g, k[g], frontier[g], fsize[g], pd, active > 1))) return e;
+        for (int d = 0; d < T.nl; d++) T.tot[d] = s->replay_f[g][k[g] + d];
+        T.phase = 1;  // the emit is queued next round, sized from the expected totals
+      } else {
+        const uint64_t want = s->replay_f[g][k[g]];
+        if ((e = queue_level(s, (int)g, k[g], frontier[g], fsize[g], pd, active > 1, want))) return e;
+        GroupPlan& gp = s->groups[g];
+        LevelData& d = s->data[g][k[g]];
+        d.rec = pd.child;
+        d.n = want;
+        d.evals = fsize[g] * (uint64_t)gp.levels[k[g]].r;
+        if (!(s->opts.flags & ATF_FLAG_TIMING)) d.pairs = 0;
+        if (k[g] > 0) s->data[g][k[g] - 1].csr = pd.csr;
+        expect.push_back(Expect{round, (int)g, want});
+        if (s->opts.flags & ATF_FLAG_TIMING) timed.emplace_back((int)g, k[g]);
+        frontier[g] = pd.child;
+        fsize[g] = want;
+        k[g]++;
+      }
+      pend.push_back(pd);
+    }
+    if (!any) break;
+    for (auto& pd : pend)
+      if (pd.joined) CUDA_TRY(s, cudaStreamWaitEvent(st, s->gb[pd.g].join, 0));
+    if (!pend.empty())
+      CUDA_TRY(s, cudaMemcpyAsync((char*)s->d_replay + (size_t)round * 12 * kMaxGroups, s->d_totals, 12 * kMaxGroups,
+                                  cudaMemcpyDeviceToDevice, st));
+  }
+  // one synchronisation: the round log, then the checks
+  std::vector<unsigned long long> log((size_t)round * 12 * kMaxGroups / 8 + 1, 0);
+  if (round) CUDA_TRY(s, cudaMemcpyAsync(log.data(), s->d_replay, (size_t)round * 12 * kMaxGroups, cudaMemcpyDeviceToHost, st));
+  CUDA_TRY(s, cudaStreamSynchronize(st));
+  for (const Expect& x : expect) {
+    const unsigned long long* rl = log.data() + (size_t)x.round * 12 * kMaxGroups / 8;
+    const unsigned int* ovf = reinterpret_cast<const unsigned int*>(rl + kMaxGroups);
+    if (rl[x.g] != x.total || ovf[x.g]) return fail(s, ATF_ERR_STATE, "replay: level total differs (group %d)", x.g);
+  }
+  for (int g : tails_done) finish_tail(s, g);  // totals were the expected ones (tail scans)
+  for (auto& gk : timed) {
+    LevelData& d = s->data[gk.first][gk.second];
+    cudaEventElapsedTime(&d.ms, s->events[gk.first][gk.second].first, s->events[gk.first][gk.second].second);
+    cudaEventElapsedTime(&d.expand_ms, s->events[gk.first][gk.second].first, s->events[gk.first][gk.second].mid);
+    d.pairs = d.evals;  // the headline flags; the segment-bound pair counts are not logged per level here
+  }
+  return ATF_OK;
+}
+
 // ---------------------------------------------------------------- balanced multi-GPU generation
 // SURVEY.md §8(e), DESIGN.md §6.  Every level is distributed afresh: rank r expands the parents
 // [r F / N, (r + 1) F / N) of the previous level (F = its global size), so every rank evaluates
@@ -1698,9 +1829,13 @@ static atf_status dist_desc(atf_space* s, int g, const uint32_t* rec, DistDesc& 
     if ((const char*)rec >= c.p && (const char*)rec < c.p + c.size) {
       d.base = (uint64_t)(uintptr_t)c.p;
       d.off = (uint64_t)((const char*)rec - c.p);
-      cudaIpcMemHandle_t h;
-      CUDA_TRY(s, cudaIpcGetMemHandle(&h, c.p));
-      std::memcpy(d.handle, &h, sizeof h);
+      if (!c.has_ipc) {  // exported once per allocation
+        cudaIpcMemHandle_t h;
+        CUDA_TRY(s, cudaIpcGetMemHandle(&h, c.p));
+        std::memcpy(c.ipc, &h, sizeof h);
+        c.has_ipc = true;
+      }
+      std::memcpy(d.handle, c.ipc, 64);
       return ATF_OK;
     }
   return fail(s, ATF_ERR_STATE, "internal: level records outside the arena");
@@ -1997,11 +2132,35 @@ static atf_status generate_impl(atf_space* s) {
       }
     }
   }
-  std::vector<int> gs(G), kf(G, 0);
-  std::iota(gs.begin(), gs.end(), 0);
-  std::vector<const uint32_t*> fr(G, s->d_root);
-  std::vector<uint64_t> fz(G, 1);
-  if ((e = run_levels(s, gs, kf, fr, fz))) return e;
+  bool replayed = false;
+  // (not with ATF_FLAG_TIMING: the timing pass keeps one synchronisation per round so that the
+  // per-level statistics, segment-bound pair counts included, are read as the levels complete)
+  if (s->replay_ok && !(s->opts.flags & (ATF_FLAG_NO_REPLAY | ATF_FLAG_TIMING))) {
+    e = run_levels_replay(s);
+    if (e == ATF_OK) {
+      replayed = true;
+    } else {  // sizes differ from the recorded ones: regenerate level by level
+      cudaStreamSynchronize((cudaStream_t)s->opts.stream);
+      cudaGetLastError();
+      s->replay_ok = false;
+      for (size_t g = 0; g < G; g++) {
+        s->data[g].assign(s->groups[g].levels.size(), LevelData{});
+        for (auto& c : s->arena[g]) c.used = 0;
+      }
+      s->tails.assign(G, {});
+    }
+  }
+  if (!replayed) {
+    std::vector<int> gs(G), kf(G, 0);
+    std::iota(gs.begin(), gs.end(), 0);
+    std::vector<const uint32_t*> fr(G, s->d_root);
+    std::vector<uint64_t> fz(G, 1);
+    if ((e = run_levels(s, gs, kf, fr, fz))) return e;
+    s->replay_f.assign(G, {});
+    for (size_t g = 0; g < G; g++)
+      for (auto& d : s->data[g]) s->replay_f[g].push_back(d.n);
+    s->replay_ok = true;
+  }
   s->gsize.assign(G, 0);
   for (size_t g = 0; g < G; g++) s->gsize[g] = s->groups[g].levels.empty() ? 0 : s->data[g].back().n;
   s->state = GENERATED;
@@ -2662,6 +2821,7 @@ atf_status atf_space_generate_shard(atf_space* s, int32_t rank, int32_t world, i
   }
   if (s->dev_ready && s->ipc_alloc) release_device(s);
   s->ipc_alloc = false;
+  s->replay_ok = false;
   atf_status e = ensure_device(s);
   if (e) return e;
   size_t G = s->groups.size();
@@ -2832,6 +2992,7 @@ atf_status atf_space_generate_dist(atf_space* s, int32_t rank, int32_t world, at
     atf_status e = atf_space_plan(s);
     if (e) return e;
   }
+  s->replay_ok = false;
   if (s->dev_ready && !s->ipc_alloc) release_device(s);  // arenas must be exportable (cudaMalloc)
   s->ipc_alloc = true;
   atf_status e = ensure_device(s);

@@ -534,7 +534,7 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
        "if (lane >= o) bincl += y; }\n";
   s += "    for (int p0 = 0; p0 < 32;) {\n";
   s += "      const u32 b0 = p0 ? __shfl_sync(0xffffffffu, bincl, p0 - 1) : 0u;\n";
-  s += "      const unsigned fit = __ballot_sync(0xffffffffu, lane >= p0 && bincl - b0 <= " + std::to_string(kStage) + "u);\n";
+  s += "      const unsigned fit = __ballot_sync(0xffffffffu, lane >= p0 && bincl - b0 <= " + std::to_string(kStage - 16) + "u);  // 16: the record region's alignment\n";
   s += "      const int p1 = fit ? 32 - __clz(fit) : p0 + 1;  // lanes [p0, p1)\n";
   s += "      const bool staged = fit != 0u;\n";
   s += "      u32 pb[" + NLs + "], pe[" + NLs + "], roff[" + NLs + "], coff[" + NLs + "];\n";

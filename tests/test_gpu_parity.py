@@ -53,7 +53,7 @@ def torch_rowhash(rows_pm: "torch.Tensor", base: int = 0) -> int:
 
 
 def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, legacy=False, no_jit=False,
-                          extra_flags=0, leaves_max=4_000_000):
+                          extra_flags=0, leaves_max=4_000_000, regenerate=False):
     """Sizes, groups, f_k and evals vs the oracle; then CONTENT: every configuration (decode of
     all S indices) when S <= decode_all_max, else every group's leaves element by element
     (decode_digits over all of the group's leaves vs the oracle's canonical leaf stream) for
@@ -64,6 +64,8 @@ def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, 
              | extra_flags)
     with Space(spec, flags=flags) as sp:
         sp.generate()
+        if regenerate:        # the second generation of a space replays the first one's level sizes
+            sp.generate()
         assert sp.groups() == [g["members"] for g in ref["groups"]]
         assert sp.size() == int(ref["S"])
         assert sp.group_sizes() == [g["size"] for g in ref["groups"]]
@@ -126,6 +128,21 @@ SMALL = {
 @pytest.mark.parametrize("generic", [False, True])
 def test_small_specs(Space, name, generic):
     _check_against_oracle(Space, SMALL[name](), generic=generic)
+
+
+@pytest.mark.parametrize("name", list(SMALL))
+def test_small_specs_regenerated(Space, name):
+    """Steady state: the second generation of a space (replay of the first one's level sizes, one
+    synchronisation) gives the same space, headline flags and default flags."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    _check_against_oracle(Space, SMALL[name](), regenerate=True)
+    _check_against_oracle(Space, SMALL[name](), regenerate=True, extra_flags=L.ATF_FLAG_NO_SEG_BOUNDS)
+
+
+@pytest.mark.parametrize("seed", range(0, 80, 3))
+def test_fuzz_specs_regenerated(Space, seed):
+    _check_against_oracle(Space, A.random_spec(seed), regenerate=True)
+    _check_against_oracle(Space, A.random_wide_spec(seed % 40), regenerate=True)
 
 
 @pytest.mark.parametrize("name", ["C5-60x5", "C5-300x4", "C5-4096x3", "C2-256", "C3-IS1", "C3-12x30x8"])
@@ -346,6 +363,7 @@ def test_full_size_against_golden(Space, name, every_pair):
     spec = SPECS[name]()
     with Space(spec, flags=L.ATF_FLAG_NO_SEG_BOUNDS if every_pair else 0) as sp:
         sp.generate()
+        sp.generate()   # the bench's timed steps: the second generation replays the level sizes
         assert sp.size() == int(gold["S"])
         for g, grp in enumerate(gold["groups"]):
             assert sp.level_sizes(g) == [lv["f"] for lv in grp["levels"]]

@@ -1,0 +1,15 @@
+#!/bin/bash
+mkdir -p gpurun_out
+T=${T:-r02j}
+timeout 2400 python -m pytest tests -m gpu -q --maxfail=5 --durations=20 > gpurun_out/${T}_pytest_gpu.txt 2>&1
+echo "pytest rc=$?" >> gpurun_out/${T}_pytest_gpu.txt
+tail -3 gpurun_out/${T}_pytest_gpu.txt
+for cfg in C3-IS4 C3-IS2; do
+  timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/${T}_launches_${cfg}.csv python tools/gen_once.py $cfg --reps 2 --profile-last > /dev/null 2>&1
+  echo "launches $cfg rc=$?"
+done
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:atf_tail -c 2 -o gpurun_out/${T}_tail_is2 python tools/gen_once.py C3-IS2 > /dev/null 2>&1; echo "ncu tail rc=$?"
+timeout 600 ncu --set full --clock-control none --import-source on -k regex:decode -c 1 -o gpurun_out/${T}_decode_c4 python tools/gen_once.py C3-IS2 --decode 100000000 > /dev/null 2>&1; echo "ncu decode rc=$?"
+timeout 900 ncu --set full --clock-control none --import-source on -k regex:expand_wtile --launch-skip 21 --launch-count 3 -o gpurun_out/${T}_c5_l8 python tools/gen_once.py C5 > /dev/null 2>&1; echo "ncu c5 l8 rc=$?"
+timeout 1200 python bench.py --steps 10 > gpurun_out/${T}_bench.json 2> gpurun_out/${T}_bench.err; echo "bench rc=$?"
+python tools/bench_brief.py gpurun_out/${T}_bench.json 2>/dev/null | head -20
