@@ -114,6 +114,7 @@ struct LevelArgs {
   int32_t rw, sw;           // wide: bitmap words per node (chunk/32), summary words (ceil(rw/32))
   int32_t qcap;             // wide: slow-path queue entries per tile
   int32_t nseg;             // warp-tile: candidate segments of 32*cpt per node (<= kMaxSeg)
+  int32_t seg_on;           // warp-tile: the per-segment |x| bounds below are applied
   // warp-tile hot filter, per segment: min / max |x| over its candidates (0 / 0xffffffff
   // when a candidate is 0).  x | n with n != 0 needs |x| <= |n|, d | x with x != 0 needs
   // |x| >= |d|: a node quad outside a segment's bounds has no item there
@@ -141,6 +142,7 @@ struct TailArgs {
   uint64_t n_tiles;            // ceil(n_parents / 32)
   uint32_t* tile_total;        // [nl][n_tiles] (tail_count)
   const uint64_t* tile_base;   // [nl][n_tiles + 1] exclusive scans of tile_total per level
+  uint32_t* node_cnt;          // [nl][n_parents] per frontier node subtree counts (NVRTC kernels)
   uint64_t* csr[kMaxTail];     // csr[0]: CSR of the frontier level [n_parents + 1];
                                // csr[d] (d >= 1): CSR of tail level d - 1
   uint32_t* rec[kMaxTail];     // records of tail level d (tail_emit)

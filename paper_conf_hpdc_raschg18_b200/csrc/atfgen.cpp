@@ -1164,6 +1164,7 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   fill_level_ptrs(s, lp, a);
   const bool seg_bounds = (s->opts.flags & ATF_FLAG_NO_SEG_BOUNDS) == 0;
   choose_geometry(a, gp.words, (s->opts.flags & ATF_FLAG_LEGACY_WIDE) != 0, seg_bounds);
+  a.seg_on = (a.kind == K_WTILE && a.hot != HOT_NONE && seg_bounds) ? 1 : 0;
   if (a.kind == K_WTILE && a.hot != HOT_NONE && !seg_bounds) {
     // every pair is evaluated: bounds that no node quad can fall outside of
     for (int sg = 0; sg < kMaxSeg; sg++) { a.seg_lo[sg] = 0u; a.seg_hi[sg] = 0xffffffffu; }
@@ -1437,12 +1438,14 @@ static atf_status queue_tail_count(atf_space* s, int g, int k0, const uint32_t* 
   // scratch: tile_total u32[nl][n] | tile_base u64[nl][n+1] | scan status u64[nl][ns] | counters u32[nl]
   const size_t n = t.n_tiles, ns = (n + 1023) / 1024 + 1;
   const size_t o_tot = 0, o_base = (o_tot + 4 * nl * n + 15) & ~(size_t)15, o_stat = o_base + 8 * nl * (n + 1);
-  const size_t o_cnt = o_stat + 8 * nl * ns, bytes = o_cnt + 4 * nl + 16;
+  const size_t o_cnt = o_stat + 8 * nl * ns, o_nc = (o_cnt + 4 * nl + 16 + 15) & ~(size_t)15;
+  const size_t bytes = o_nc + 4 * (size_t)nl * n_parents + 16;
   atf_status e = ensure_buf(s, &gbf.scratch, &gbf.scratch_cap, bytes, "tail scratch");
   if (e) return e;
   t.tile_total = (uint32_t*)(gbf.scratch + o_tot);
   t.tile_base = (const uint64_t*)(gbf.scratch + o_base);
-  CUDA_TRY(s, cudaMemsetAsync(gbf.scratch + o_stat, 0, bytes - o_stat, st));
+  t.node_cnt = (uint32_t*)(gbf.scratch + o_nc);
+  CUDA_TRY(s, cudaMemsetAsync(gbf.scratch + o_stat, 0, o_nc - o_stat, st));
   const bool serial = !own_stream || (s->opts.flags & ATF_FLAG_SERIAL_GROUPS) != 0;
   cudaStream_t ls = serial ? st : gbf.stream;
   if (!serial) {
@@ -2565,10 +2568,19 @@ static atf_status decode_common(const atf_space* cs, const uint64_t* idx, const 
     s->decode_jit = jit_decode_kernel(a);
     s->decode_jit_tried = true;
   }
-  int ce = (n >= (1 << 18) && s->decode_jit && !(s->opts.flags & ATF_FLAG_NO_JIT))
+  // random leaf gathers: ask for 32-byte L2 fetches for this launch (the default granularity
+  // fetches a whole line per 8-byte record)
+  size_t gran = 0;
+  const bool big = n >= (1 << 18);
+  if (big && cudaDeviceGetLimit(&gran, cudaLimitMaxL2FetchGranularity) == cudaSuccess && gran != 32)
+    cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, 32);
+  cudaGetLastError();
+  int ce = (big && s->decode_jit && !(s->opts.flags & ATF_FLAG_NO_JIT))
                ? jit_decode_launch(s->decode_jit, a, idx, digits, n, out, ld, s->d_bad, st)
                : (idx ? launch_decode_indices(a, idx, n, out, ld, s->d_bad, st)
                       : launch_decode_digits(a, digits, n, out, ld, s->d_bad, st));
+  if (big && gran && gran != 32) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, gran);
+  cudaGetLastError();
   if (ce) return fail(s, ATF_ERR_CUDA, "decode launch: %s", cudaGetErrorString((cudaError_t)ce));
   // the bad-index flag is read back only when someone could be out of range: always
   // check (one 4-byte copy) — it costs a sync, so the flag copy is async and we

@@ -934,22 +934,29 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
     // ---- hot loop (A4): item words = per-node ballots of the superset filter
     const int nq = (tn + 3) >> 2;
     if (HOT != HOT_NONE) {
+      const bool seg_on = a.seg_on != 0;  // segment bounds in force (not the headline flags)
+      pairs += (uint64_t)tn * (uint64_t)r;  // less the pairs of skipped quad segments below
       for (int sg = 0; sg < nseg; sg++) {
         uint32_t hm[CPT];
         const uint32_t* tp = s_tab + sg * SEG + lane;
 #pragma unroll
         for (int c = 0; c < CPT; c++) hm[c] = tp[c * 32];
-        uint32_t sb = HOT == HOT_DIVX ? a.seg_lo[0] : a.seg_hi[0];  // no dynamic param indexing
+        uint32_t sb = 0;
+        if (seg_on) {
+          sb = HOT == HOT_DIVX ? a.seg_lo[0] : a.seg_hi[0];  // no dynamic param indexing
 #pragma unroll
-        for (int i = 1; i < kMaxSeg; i++)
-          if (sg == i) sb = HOT == HOT_DIVX ? a.seg_lo[i] : a.seg_hi[i];
+          for (int i = 1; i < kMaxSeg; i++)
+            if (sg == i) sb = HOT == HOT_DIVX ? a.seg_lo[i] : a.seg_hi[i];
+        }
         for (int q = 0; q < nq; q++) {
-          const uint32_t qv = __shfl_sync(FULL, qb, 4 * q);
-          if (HOT == HOT_DIVX ? qv < sb : qv > sb) {
-            if (lane == 0) *reinterpret_cast<uint4*>(s_items + sg * kWT + 4 * q) = make_uint4(0u, 0u, 0u, 0u);
-            continue;
+          if (seg_on) {
+            const uint32_t qv = __shfl_sync(FULL, qb, 4 * q);
+            if (HOT == HOT_DIVX ? qv < sb : qv > sb) {
+              if (lane == 0) *reinterpret_cast<uint4*>(s_items + sg * kWT + 4 * q) = make_uint4(0u, 0u, 0u, 0u);
+              pairs -= (uint64_t)min(4, tn - 4 * q) * (uint64_t)min(SEG, r - sg * SEG);
+              continue;
+            }
           }
-          pairs += (uint64_t)min(4, tn - 4 * q) * (uint64_t)min(SEG, r - sg * SEG);
           const uint4 n4 = *reinterpret_cast<const uint4*>(s_hot + 4 * q);
           uint32_t m0 = 0xffffffffu, m1 = 0xffffffffu, m2 = 0xffffffffu, m3 = 0xffffffffu;
 #pragma unroll

@@ -353,6 +353,7 @@ struct TailJitArgs {
   uint64_t n_parents, n_tiles;
   uint32_t* tile_total;
   const uint64_t* tile_base;
+  uint32_t* node_cnt;  // [nl][n_parents] subtree counts per frontier node (count -> emit)
   uint64_t* csr[kMaxTail];
   uint32_t* rec[kMaxTail];
   const int32_t* l0_range[kMaxSlots];
@@ -367,7 +368,7 @@ struct TailJitArgs {
 
 const char* kTailPrelude = R"(
 struct TailJitArgs { const u32* parent_rec; u64 n_parents, n_tiles; u32* tile_total; const u64* tile_base;
-                     u64* csr[4]; u32* rec[4];
+                     u32* node_cnt; u64* csr[4]; u32* rec[4];
                      const i32* l0_range[24]; const u32* l0_magic[24]; const i32* l1_range[24]; const u32* l1_magic[24];
                      const i32* l2_range[24]; const u32* l2_magic[24]; const i32* l3_range[24]; const u32* l3_magic[24]; };
 )";
@@ -471,7 +472,10 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "    const u64 nd = tile * 32 + lane;\n    u32 cnt[" + std::to_string(nl) + "] = {};\n";
   s += "    if (nd < a.n_parents) {\n      u32 w[" + Ws + "];\n";
   s += "      for (int i = 0; i < " + Ws + "; i++) w[i] = __ldg(a.parent_rec + nd * " + Ws + " + i);\n";
-  s += "      u32 nc[" + std::to_string(NC) + "];\n      tnc(a, w, nc);\n      cnt0(a, w, nc, cnt);\n    }\n";
+  s += "      u32 nc[" + std::to_string(NC) + "];\n      tnc(a, w, nc);\n      cnt0(a, w, nc, cnt);\n";
+  for (int d = 0; d < nl; d++)
+    s += "      a.node_cnt[(u64)" + std::to_string(d) + " * a.n_parents + nd] = cnt[" + std::to_string(d) + "];\n";
+  s += "    }\n";
   for (int d = 0; d < nl; d++) {
     const std::string ds = std::to_string(d);
     s += "    { u32 v = cnt[" + ds + "];\n#pragma unroll\n      for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);\n";
@@ -521,7 +525,10 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "    const u64 nd = tile * 32 + lane;\n    const bool valid = nd < a.n_parents;\n    u32 w[" + Ws + "];\n";
   s += "    for (int i = 0; i < " + Ws + "; i++) w[i] = valid ? __ldg(a.parent_rec + nd * " + Ws + " + i) : 0u;\n";
   s += "    u32 nc[" + NCs + "];\n    u32 cnt[" + NLs + "] = {};\n";
-  s += "    if (valid) { tnc(a, w, nc); cnt0(a, w, nc, cnt); }\n";
+  s += "    if (valid) {\n      tnc(a, w, nc);\n";   // the subtree counts come from the count pass
+  for (int d = 0; d < nl; d++)
+    s += "      cnt[" + std::to_string(d) + "] = __ldcs(a.node_cnt + (u64)" + std::to_string(d) + " * a.n_parents + nd);\n";
+  s += "    }\n";
   s += "    u32 off[" + NLs + "];\n    u64 base[" + NLs + "];\n    u32 bytes = 0;\n";
   s += "#pragma unroll\n    for (int d = 0; d < " + NLs + "; d++) {\n";
   s += "      u32 incl = cnt[d];\n#pragma unroll\n      for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
@@ -678,7 +685,7 @@ std::string gen_wide_source(const LevelArgs& a, int W, const std::vector<int32_t
   }
   static const char* rel[] = {"==", "!=", "<", "<=", ">", ">="};
   if (a.n_terms > 0 && a.terms[0].kind == T_QDIV) return "";  // a quotient test is never the cheapest conjunct
-  s += "    u32 cnt = 0;\n";
+  s += "    u32 cnt = 0, nzw = 0;  // nzw bit j: candidate word j has survivors\n";
   // first conjunct: divisibility tests (x | n, d | x) in groups of 4 candidates, a superset
   // test per group (min of the 4 magic products, VIMNMX3) whose survivors are re-tested exactly
   // below; comparisons exactly per candidate
@@ -735,7 +742,8 @@ std::string gen_wide_source(const LevelArgs& a, int W, const std::vector<int32_t
       }
       s += "        if (!ok) mw &= ~(1u << c);\n      }\n";
     }
-    s += "      if (!alive) mw = 0u;\n      s_m[" + std::to_string(32 * j) + " + lane] = mw;\n      cnt += __popc(mw);\n    }\n";
+    s += "      if (!alive) mw = 0u;\n      s_m[" + std::to_string(32 * j) + " + lane] = mw;\n      cnt += __popc(mw);\n";
+    s += "      nzw |= (u32)(mw != 0u) << " + std::to_string(j) + ";\n    }\n";
   }
   // tile scan, stash segment, CSR
   s += "    u32 incl = cnt;\n#pragma unroll\n    for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); if (lane >= o) incl += y; }\n";
@@ -747,7 +755,8 @@ std::string gen_wide_source(const LevelArgs& a, int W, const std::vector<int32_t
   s += "    const bool staged = total <= " + std::to_string(stage) + "u;\n";
   s += "    __syncwarp();\n";
   const int fw = a.field_word, fs = a.field_shift;
-  s += "    for (int j = 0; j < " + std::to_string(NWD) + "; j++) {\n      u32 mw = s_m[j * 32 + lane];\n";
+  s += "    while (nzw) {  // the node's nonzero words only\n      const int j = __ffs(nzw) - 1;\n      nzw &= nzw - 1;\n"
+       "      u32 mw = s_m[j * 32 + lane];\n";
   s += "      while (mw) {\n        const u32 c = __ffs(mw) - 1;\n        mw &= mw - 1;\n        const u32 pos = (u32)j * 32u + c;\n";
   s += "        if (staged) {\n";
   for (int wd = 0; wd < W; wd++)
@@ -1000,6 +1009,7 @@ int jit_tail_launch(void* handle, const TailArgs& t, bool emit, void* stream) {
   j.n_tiles = t.n_tiles;
   j.tile_total = t.tile_total;
   j.tile_base = t.tile_base;
+  j.node_cnt = t.node_cnt;
   for (int d = 0; d < kMaxTail; d++) {
     j.csr[d] = t.csr[d];
     j.rec[d] = t.rec[d];
