@@ -1,5 +1,5 @@
 """Per-CUDA-line warp-stall samples and executed instructions from an ncu report
-(--page source --print-source cuda,sass): python tools/ncu_source.py rep [top]"""
+(--page source --print-source cuda,sass): python tools/ncu_source.py rep [top] [kernel-name]"""
 import csv
 import io
 import subprocess
@@ -7,7 +7,8 @@ import sys
 
 rep = sys.argv[1]
 top = int(sys.argv[2]) if len(sys.argv) > 2 else 25
-out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+kfilter = ["-k", sys.argv[3]] if len(sys.argv) > 3 else []
+out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"] + kfilter,
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(out)))
 agg, src, fname = {}, {}, None
@@ -31,5 +32,6 @@ for r in rows:
 tot_s = sum(v[0] for v in agg.values()) or 1
 tot_i = sum(v[1] for v in agg.values()) or 1
 print(f"total stall samples {tot_s:.0f}, warp instructions {tot_i:.3g}")
-for k, v in sorted(agg.items(), key=lambda kv: -kv[1][0])[:top]:
+order = 1 if "--by-inst" in sys.argv else 0
+for k, v in sorted(agg.items(), key=lambda kv: -kv[1][order])[:top]:
     print(f"{k[0]:>16}:{k[1]:<5d} stall {100*v[0]/tot_s:5.1f}%  inst {100*v[1]/tot_i:5.1f}%  {src[k].strip()[:80]}")
