@@ -493,10 +493,15 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   constexpr int kStage = 8192;  // staging bytes per warp
   if (warp_bytes) *warp_bytes = kStage;
   const std::string NLs = std::to_string(nl), NCs = std::to_string(NC), RB = std::to_string(W * 4);
+  // The leaf level is not written by the depth-first walk when staged: a level-(nl-2) node stores
+  // its leaf mask instead (and advances the leaf cursor by its popcount), and a balanced pass over
+  // the part's level-(nl-2) nodes (lane-strided) writes the leaves afterwards, so the walk's
+  // divergence does not reach the largest level.
+  const int LP = nl - 2;  // parents of the leaves
   for (int d = nl - 1; d >= 0; d--) {
     const std::string ds = std::to_string(d);
     s += "__device__ __forceinline__ void dfs" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cur, "
-         "const u64* base, const u32* pb, unsigned char* sm, bool staged, const u32* roff, const u32* coff) {\n";
+         "const u64* base, const u32* pb, unsigned char* sm, bool staged, const u32* roff, const u32* coff, u32 lmo) {\n";
     s += "  u32 m = tmask" + ds + "(a, w, nc);\n";
     s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
     s += child(d, "w", "cw", "    ");
@@ -510,7 +515,13 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
       const std::string d1 = std::to_string(d + 1);
       s += "    if (staged) reinterpret_cast<u32*>(sm + coff[" + ds + "])[slot - pb[" + ds + "]] = cur[" + d1 + "];\n";
       s += "    else a.csr[" + d1 + "][base[" + ds + "] + slot] = base[" + d1 + "] + cur[" + d1 + "];\n";
-      s += "    dfs" + d1 + "(a, cw, nc, cur, base, pb, sm, staged, roff, coff);\n";
+      if (d == LP) {
+        s += "    if (staged) {\n      const u32 lm = tmask" + d1 + "(a, cw, nc);\n";
+        s += "      reinterpret_cast<u32*>(sm + lmo)[slot - pb[" + ds + "]] = lm;\n      cur[" + d1 + "] += __popc(lm);\n";
+        s += "    } else {\n      dfs" + d1 + "(a, cw, nc, cur, base, pb, sm, staged, roff, coff, lmo);\n    }\n";
+      } else {
+        s += "    dfs" + d1 + "(a, cw, nc, cur, base, pb, sm, staged, roff, coff, lmo);\n";
+      }
     }
     s += "  }\n}\n";
   }
@@ -534,7 +545,7 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "      u32 incl = cnt[d];\n#pragma unroll\n      for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
        "if (lane >= o) incl += y; }\n";
   s += "      off[d] = incl - cnt[d];\n      base[d] = a.tile_base[(u64)d * (a.n_tiles + 1) + tile];\n";
-  s += "      bytes += cnt[d] * (" + RB + "u + (d + 1 < " + NLs + " ? 4u : 0u));\n    }\n";
+  s += "      bytes += cnt[d] * (" + RB + "u + (d + 1 < " + NLs + " ? 4u : 0u) + (d == " + std::to_string(nl - 2) + " ? 4u : 0u));\n    }\n";
   s += "    if (valid) a.csr[0][nd] = base[0] + off[0];\n";
   // inclusive byte prefix per lane
   s += "    u32 bincl = bytes;\n#pragma unroll\n    for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, bincl, o); "
@@ -550,16 +561,41 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "        pb[d] = __shfl_sync(0xffffffffu, off[d], p0);\n";
   s += "        const u32 last = __shfl_sync(0xffffffffu, off[d] + cnt[d], p1 - 1);\n        pe[d] = last;\n";
   s += "        if (d + 1 < " + NLs + ") { coff[d] = o; o += (last - pb[d]) * 4u; }\n      }\n";
+  s += "      const u32 lmo = o;  // leaf masks of the part's level-" + std::to_string(nl - 2) + " nodes\n";
+  s += "      o += (pe[" + std::to_string(nl - 2) + "] - pb[" + std::to_string(nl - 2) + "]) * 4u;\n";
   s += "      o = (o + 15u) & ~15u;\n";
   s += "#pragma unroll\n      for (int d = 0; d < " + NLs + "; d++) { roff[d] = o; o += (pe[d] - pb[d]) * " + RB + "u; }\n";
   s += "      if (lane >= p0 && lane < p1 && valid) {\n        u32 cur[" + NLs + "];\n";
   s += "#pragma unroll\n        for (int d = 0; d < " + NLs + "; d++) cur[d] = off[d];\n";
-  s += "        dfs0(a, w, nc, cur, base, pb, sm, staged, roff, coff);\n      }\n";
+  s += "        dfs0(a, w, nc, cur, base, pb, sm, staged, roff, coff, lmo);\n      }\n";
   s += "      if (staged) {\n        __syncwarp();\n";
+  {  // balanced leaf pass
+    const std::string lp = std::to_string(nl - 2), ll = std::to_string(nl - 1);
+    const int fw = t.lv[nl - 1].field_word, fs = t.lv[nl - 1].field_shift;
+    s += "        {  // leaves of the part's level-" + lp + " nodes, lane-strided\n";
+    s += "          const u32 nn = pe[" + lp + "] - pb[" + lp + "];\n";
+    s += "          const u32* lms = reinterpret_cast<const u32*>(sm + lmo);\n";
+    s += "          const u32* cst = reinterpret_cast<const u32*>(sm + coff[" + lp + "]);\n";
+    s += "          for (u32 i = lane; i < nn; i += 32) {\n            u32 lm = lms[i];\n            if (!lm) continue;\n";
+    s += "            u32 k = cst[i] - pb[" + ll + "];\n";
+    s += "            const u32* pr = reinterpret_cast<const u32*>(sm + roff[" + lp + "]) + i * " + Ws + ";\n";
+    s += "            u32 pw[" + Ws + "];\n";
+    for (int w = 0; w < W; w++) s += "            pw[" + std::to_string(w) + "] = pr[" + std::to_string(w) + "];\n";
+    s += "            while (lm) {\n              const u32 cc = __ffs(lm) - 1;\n              lm &= lm - 1;\n";
+    s += "              u32* dst = reinterpret_cast<u32*>(sm + roff[" + ll + "]) + k * " + Ws + ";\n";
+    for (int w = 0; w < W; w++)
+      s += "              dst[" + std::to_string(w) + "] = pw[" + std::to_string(w) + "]" +
+           (w == fw && t.lv[nl - 1].r > 1 ? " | (cc << " + std::to_string(fs) + ")" : "") + ";\n";
+    s += "              k++;\n            }\n          }\n          __syncwarp();\n        }\n";
+  }
   s += "#pragma unroll\n        for (int d = 0; d < " + NLs + "; d++) {\n";
   s += "          const u32 n = (pe[d] - pb[d]) * " + Ws + "u;\n";
   s += "          const u32* src = reinterpret_cast<const u32*>(sm + roff[d]);\n          u32* dst = a.rec[d] + (base[d] + pb[d]) * " + Ws + ";\n";
-  s += "#pragma unroll 4\n          for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
+  if (W % 2 == 0)  // 8-byte aligned on both sides (records of even W, 8-byte CSR regions before them)
+    s += "          { const uint2* s2 = reinterpret_cast<const uint2*>(src); uint2* d2 = reinterpret_cast<uint2*>(dst);\n"
+         "#pragma unroll 4\n            for (u32 v = lane; v < n / 2; v += 32) d2[v] = s2[v]; }\n";
+  else
+    s += "#pragma unroll 4\n          for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
   s += "          if (d + 1 < " + NLs + ") {\n            const u32* cs = reinterpret_cast<const u32*>(sm + coff[d]);\n";
   s += "            u64* cd = a.csr[d + 1] + base[d] + pb[d];\n            const u64 cb = base[d + 1 < " + NLs + " ? d + 1 : d];\n";
   s += "#pragma unroll 4\n            for (u32 v = lane; v < pe[d] - pb[d]; v += 32) cd[v] = cb + cs[v];\n          }\n";
