@@ -532,19 +532,33 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "  if (gw == 0 && lane < " + NLs + ") {\n";
   s += "    const u64 above = lane == 0 ? a.n_parents : a.tile_base[(u64)(lane - 1) * (a.n_tiles + 1) + a.n_tiles];\n";
   s += "    a.csr[lane][above] = a.tile_base[(u64)lane * (a.n_tiles + 1) + a.n_tiles];\n  }\n";
+  // the next tile's parent records, subtree counts and tile bases are loaded while this tile is
+  // emitted (software pipelining over the persistent grid-stride loop)
+  auto load_next = [&](const std::string& t, const std::string& ind) {
+    std::string c;
+    c += ind + "{ const u64 xn = " + t + " * 32 + lane; const bool xv = xn < a.n_parents;\n";
+    c += ind + "  for (int i = 0; i < " + Ws + "; i++) pw_[i] = xv ? __ldg(a.parent_rec + xn * " + Ws + " + i) : 0u;\n";
+    for (int d = 0; d < nl; d++)
+      c += ind + "  pc_[" + std::to_string(d) + "] = xv ? __ldcs(a.node_cnt + (u64)" + std::to_string(d) + " * a.n_parents + xn) : 0u;\n";
+    for (int d = 0; d < nl; d++)
+      c += ind + "  pb_[" + std::to_string(d) + "] = a.tile_base[(u64)" + std::to_string(d) + " * (a.n_tiles + 1) + " + t + "];\n";
+    c += ind + "}\n";
+    return c;
+  };
+  s += "  u32 pw_[" + Ws + "], pc_[" + NLs + "];\n  u64 pb_[" + NLs + "];\n";
+  s += "  if (gw < a.n_tiles) {\n" + load_next("gw", "    ") + "  }\n";
   s += "  for (u64 tile = gw; tile < a.n_tiles; tile += nw) {\n";
-  s += "    const u64 nd = tile * 32 + lane;\n    const bool valid = nd < a.n_parents;\n    u32 w[" + Ws + "];\n";
-  s += "    for (int i = 0; i < " + Ws + "; i++) w[i] = valid ? __ldg(a.parent_rec + nd * " + Ws + " + i) : 0u;\n";
-  s += "    u32 nc[" + NCs + "];\n    u32 cnt[" + NLs + "] = {};\n";
-  s += "    if (valid) {\n      tnc(a, w, nc);\n";   // the subtree counts come from the count pass
-  for (int d = 0; d < nl; d++)
-    s += "      cnt[" + std::to_string(d) + "] = __ldcs(a.node_cnt + (u64)" + std::to_string(d) + " * a.n_parents + nd);\n";
-  s += "    }\n";
-  s += "    u32 off[" + NLs + "];\n    u64 base[" + NLs + "];\n    u32 bytes = 0;\n";
+  s += "    const u64 nd = tile * 32 + lane;\n    const bool valid = nd < a.n_parents;\n    u32 w[" + Ws + "], cnt[" + NLs + "];\n    u64 base[" + NLs + "];\n";
+  s += "#pragma unroll\n    for (int i = 0; i < " + Ws + "; i++) w[i] = pw_[i];\n";
+  s += "#pragma unroll\n    for (int d = 0; d < " + NLs + "; d++) { cnt[d] = pc_[d]; base[d] = pb_[d]; }\n";
+  s += "    if (tile + nw < a.n_tiles) {\n" + load_next("(tile + nw)", "      ") + "    }\n";
+  s += "    u32 nc[" + NCs + "];\n";
+  s += "    if (valid) tnc(a, w, nc);\n";
+  s += "    u32 off[" + NLs + "];\n    u32 bytes = 0;\n";
   s += "#pragma unroll\n    for (int d = 0; d < " + NLs + "; d++) {\n";
   s += "      u32 incl = cnt[d];\n#pragma unroll\n      for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
        "if (lane >= o) incl += y; }\n";
-  s += "      off[d] = incl - cnt[d];\n      base[d] = a.tile_base[(u64)d * (a.n_tiles + 1) + tile];\n";
+  s += "      off[d] = incl - cnt[d];\n";
   s += "      bytes += cnt[d] * (" + RB + "u + (d + 1 < " + NLs + " ? 4u : 0u) + (d == " + std::to_string(nl - 2) + " ? 4u : 0u));\n    }\n";
   s += "    if (valid) a.csr[0][nd] = base[0] + off[0];\n";
   // inclusive byte prefix per lane

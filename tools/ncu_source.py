@@ -1,13 +1,20 @@
 """Per-CUDA-line warp-stall samples and executed instructions from an ncu report
-(--page source --print-source cuda,sass): python tools/ncu_source.py rep [top] [kernel-name]"""
+(--page source --print-source cuda,sass): python tools/ncu_source.py rep [top] [kernel-name]
+[--skip=N] (the N-th launch of that kernel only) [--src=file] (source text for the line numbers,
+e.g. an NVRTC source written by tools/dump_jit.py) [--by-inst]"""
 import csv
 import io
 import subprocess
 import sys
 
-rep = sys.argv[1]
-top = int(sys.argv[2]) if len(sys.argv) > 2 else 25
-kfilter = ["-k", sys.argv[3]] if len(sys.argv) > 3 else []
+pos = [a for a in sys.argv[1:] if not a.startswith("--")]
+opt = dict(a[2:].split("=", 1) for a in sys.argv[1:] if a.startswith("--") and "=" in a)
+rep = pos[0]
+top = int(pos[1]) if len(pos) > 1 else 25
+kfilter = ["-k", pos[2]] if len(pos) > 2 else []
+if "skip" in opt:
+    kfilter += ["--launch-skip", opt["skip"], "--launch-count", "1"]
+local = open(opt["src"]).read().split("\n") if "src" in opt else None
 out = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"] + kfilter,
                      capture_output=True, text=True).stdout
 rows = list(csv.reader(io.StringIO(out)))
@@ -23,7 +30,7 @@ for r in rows:
     if hdr is None or len(r) != len(hdr) or not r[0].strip():
         continue
     key = (fname, int(r[0]))
-    src[key] = r[1]
+    src[key] = local[int(r[0]) - 1] if local and 0 < int(r[0]) <= len(local) else r[1]
     s = float(r[4] or 0)
     ins = float(r[7] or 0)
     a = agg.setdefault(key, [0.0, 0.0])
