@@ -90,6 +90,8 @@ struct GroupPlan {
   std::vector<LevelPlan> levels;
   void* tail_jit = nullptr;   // NVRTC-specialised tail kernels (jit.cpp), if any
   int tail_jit_k0 = -1;       // tail start they were built for (-1: not tried)
+  int tail_ext_k0 = -1;       // extended tail start tried (NVRTC only), and whether it compiled
+  bool tail_ext_ok = false;
 };
 
 struct Chunk {
@@ -1375,25 +1377,6 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
 }
 
 // ---------------------------------------------------------------- fused narrow tail
-// First level of group g's fused narrow tail (DESIGN.md §5): the longest run of trailing
-// levels (2..kMaxTail) that are all narrow fast levels with 1 <= r <= 32 and whose per-warp
-// emit buffers (32 * r * words * 4 bytes per level) fit 16 KB; -1 if none.
-static int tail_start(const atf_space* s, int g) {
-  if (s->opts.flags & (ATF_FLAG_NO_TAIL | ATF_FLAG_LEGACY_WIDE | ATF_FLAG_GENERIC_ONLY)) return -1;
-  const GroupPlan& gp = s->groups[g];
-  const int L = (int)gp.levels.size();
-  int k0 = L, bytes = 0;
-  while (k0 > 0 && L - k0 < kMaxTail) {
-    const LevelPlan& lp = gp.levels[k0 - 1];
-    if (!lp.proto.nf_ok || lp.generic || lp.r < 1 || lp.r > 32) break;
-    const int b = 32 * lp.r * gp.words * 4;
-    if (bytes + b > 16 * 1024) break;
-    bytes += b;
-    k0--;
-  }
-  return L - k0 >= 2 ? k0 : -1;
-}
-
 // Candidate tables and ancestor levels of a tail's levels (the NVRTC generator's inputs).
 static void tail_jit_inputs(const atf_space* s, const GroupPlan& gp, int k0, int nl,
                             std::vector<std::vector<int32_t>>& cx, std::vector<std::vector<uint32_t>>& cm,
@@ -1411,6 +1394,65 @@ static void tail_jit_inputs(const atf_space* s, const GroupPlan& gp, int k0, int
     for (int q : lp.pv_param)
       pv_level[d].push_back((int)(std::find(gp.members.begin(), gp.members.end(), q) - gp.members.begin()));
   }
+}
+
+// The generator's view of a tail starting at k0 (level prototypes; no device pointers).
+static TailArgs tail_protos(const GroupPlan& gp, int k0) {
+  TailArgs t;
+  std::memset(&t, 0, sizeof t);
+  t.nl = (int)gp.levels.size() - k0;
+  for (int d = 0; d < t.nl; d++) {
+    t.lv[d] = gp.levels[k0 + d].proto;
+    t.lv[d].r = gp.levels[k0 + d].r;
+  }
+  return t;
+}
+
+// First level of group g's fused narrow tail (DESIGN.md §5): the longest run of trailing
+// levels (2..kMaxTail) that are all narrow fast levels with 1 <= r <= 32 and whose per-warp
+// emit buffers (32 * r * words * 4 bytes per level) fit 16 KB; -1 if none.  These rules are the
+// generic tail kernels' (expand.cuh).  The NVRTC tail has neither limit for its inner levels: it
+// takes r <= 64 (u64 masks) above the leaf level and stages any subtree size in parts, so when
+// the longer run it allows compiles (tried once per group, here, before the tail is chosen),
+// that run is the tail.  `assume_jit`: the extended choice without compiling (source tests).
+static int tail_start(atf_space* s, int g, bool assume_jit = false) {
+  if (s->opts.flags & (ATF_FLAG_NO_TAIL | ATF_FLAG_LEGACY_WIDE | ATF_FLAG_GENERIC_ONLY)) return -1;
+  GroupPlan& gp = s->groups[g];
+  const int L = (int)gp.levels.size();
+  int k0 = L, bytes = 0;
+  while (k0 > 0 && L - k0 < kMaxTail) {
+    const LevelPlan& lp = gp.levels[k0 - 1];
+    if (!lp.proto.nf_ok || lp.generic || lp.r < 1 || lp.r > 32) break;
+    const int b = 32 * lp.r * gp.words * 4;
+    if (bytes + b > 16 * 1024) break;
+    bytes += b;
+    k0--;
+  }
+  const int k0c = L - k0 >= 2 ? k0 : -1;
+  if (s->opts.flags & ATF_FLAG_NO_JIT) return k0c;
+  int ke = L;
+  while (ke > 0 && L - ke < kMaxTail) {
+    const LevelPlan& lp = gp.levels[ke - 1];
+    if (!lp.proto.nf_ok || lp.generic || lp.r < 1 || lp.r > (ke == L ? 32 : 64)) break;
+    ke--;
+  }
+  if (L - ke < 2 || (k0c >= 0 && ke >= k0c)) return k0c;
+  if (assume_jit) return ke;
+  if (gp.tail_ext_k0 != ke) {
+    gp.tail_ext_k0 = ke;
+    std::vector<std::vector<int32_t>> cx;
+    std::vector<std::vector<uint32_t>> cm;
+    std::vector<std::vector<int>> pvl;
+    tail_jit_inputs(s, gp, ke, L - ke, cx, cm, pvl);
+    const TailArgs t = tail_protos(gp, ke);
+    void* kern = jit_tail_kernels(t, gp.words, cx, cm, ke, pvl);
+    gp.tail_ext_ok = kern != nullptr;
+    if (kern) {
+      gp.tail_jit = kern;
+      gp.tail_jit_k0 = ke;
+    }
+  }
+  return gp.tail_ext_ok ? ke : k0c;
 }
 
 // Count round of the tail of group g from frontier `parents` (level k0 - 1, n_parents nodes):
@@ -3036,17 +3078,11 @@ atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, 
   if (e) return e;
   if (g < 0 || g >= (int)s->groups.size()) return ATF_ERR_INVALID_ARG;
   const GroupPlan& gp = s->groups[g];
-  const int k0 = tail_start(s, g);
+  const int k0 = tail_start(s, g, /*assume_jit=*/true);
   if (k0_out) *k0_out = k0;
   std::string src;
   if (k0 >= 0) {
-    TailArgs t;
-    std::memset(&t, 0, sizeof t);
-    t.nl = (int)gp.levels.size() - k0;
-    for (int d = 0; d < t.nl; d++) {
-      t.lv[d] = gp.levels[k0 + d].proto;
-      t.lv[d].r = gp.levels[k0 + d].r;
-    }
+    const TailArgs t = tail_protos(gp, k0);
     std::vector<std::vector<int32_t>> cx;
     std::vector<std::vector<uint32_t>> cm;
     std::vector<std::vector<int>> pvl;

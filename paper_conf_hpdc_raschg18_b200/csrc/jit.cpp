@@ -307,24 +307,26 @@ std::string nc_code(const LevelArgs& a, int t, const OpGen& g, const std::string
   return s + ind + "}\n";
 }
 
-// Mask code of term t from its node constants `nc` (base index i0) over r <= 32 candidates.
+// Mask code of term t from its node constants `nc` (base index i0) over r <= 64 candidates
+// (mask type u32 for r <= 32, else u64).
 std::string term_mask_code(const LevelArgs& a, int t, const std::vector<int32_t>& cx, const std::vector<uint32_t>& cm,
                            const std::string& nc) {
   const Term& T = a.terms[t];
   const int r = a.r;
-  std::string s = "  if (m) {  // term " + std::to_string(t) + "\n    u32 mm = 0u;\n";
+  const std::string MT = r > 32 ? "u64" : "u32";
+  std::string s = "  if (m) {  // term " + std::to_string(t) + "\n    " + MT + " mm = 0u;\n";
   switch (T.kind) {
     case T_DIVX: case T_DIVPROD:
       s += "    const u32 n = " + nc + "[0];\n";
       if (T.kind == T_DIVPROD) s += "    if (n == 0xffffffffu) m = 0u;\n";
       for (int c = 0; c < r; c++)
-        if (cx[c] != 0) s += "    mm |= (u32)(n * " + hex(cm[c]) + " < 0x10000u) << " + std::to_string(c) + ";\n";
+        if (cx[c] != 0) s += "    mm |= (" + MT + ")(n * " + hex(cm[c]) + " < 0x10000u) << " + std::to_string(c) + ";\n";
       break;
     case T_MULX:
       s += "    const u32 md = " + nc + "[0], mq = " + nc + "[1];\n    if (" + nc + "[2]) m = 0u;\n";
       for (int c = 0; c < r; c++) {
         const uint32_t ax = cx[c] < 0 ? 0u - (uint32_t)cx[c] : (uint32_t)cx[c];
-        s += "    mm |= (u32)(" + hex(ax) + " * md <= mq) << " + std::to_string(c) + ";\n";
+        s += "    mm |= (" + MT + ")(" + hex(ax) + " * md <= mq) << " + std::to_string(c) + ";\n";
       }
       break;
     case T_QDIV:
@@ -334,14 +336,14 @@ std::string term_mask_code(const LevelArgs& a, int t, const std::vector<int32_t>
         if (ax == 0) continue;  // x == 0 rejects
         const std::string q = ax == 1 ? std::string("num") : "__umulhi(num, " + hex(cm[c]) + ")";
         s += "    if ((m >> " + std::to_string(c) + ") & 1u) { const u32 q = " + q +
-             "; if (q != 0u && divisible16(nb, q)) mm |= 1u << " + std::to_string(c) + "; }\n";
+             "; if (q != 0u && divisible16(nb, q)) mm |= (" + MT + ")1u << " + std::to_string(c) + "; }\n";
       }
       break;
     default: {
       static const char* rel[] = {"==", "!=", "<", "<=", ">", ">="};
       s += "    const i32 A = (i32)" + nc + "[0], B = (i32)" + nc + "[1];\n";
       for (int c = 0; c < r; c++)
-        s += "    mm |= (u32)(A * " + std::to_string(cx[c]) + " " + rel[T.rel - R_EQ] + " B) << " + std::to_string(c) + ";\n";
+        s += "    mm |= (" + MT + ")(A * " + std::to_string(cx[c]) + " " + rel[T.rel - R_EQ] + " B) << " + std::to_string(c) + ";\n";
     }
   }
   return s + "    m &= mm;\n  }\n";
@@ -396,7 +398,8 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   int NNC = 0;
   for (int d = 0; d < nl; d++) {
     const LevelArgs& a = t.lv[d];
-    if (a.n_terms == 0 || a.r > 32 || a.r < 1 || (int)cx[d].size() != a.r) return "";
+    // masks: u32, or u64 for 32 < r <= 64 on a non-leaf level (the leaf masks are staged as u32)
+    if (a.n_terms == 0 || a.r > (d + 1 < nl ? 64 : 32) || a.r < 1 || (int)cx[d].size() != a.r) return "";
     auto above = [&](const NfOp& o) {
       if (o.kind == NF_CONST) return true;
       if (o.kind == NF_PV) return pv_level[d][o.s1] < k0;
@@ -433,9 +436,13 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
     OpGen g(a, "l" + std::to_string(d), "");
     for (int tt = 0; tt < a.n_terms; tt++)
       if (ncoff[d][tt] < 0) g.mark_term(tt);
-    s += "__device__ __forceinline__ u32 tmask" + std::to_string(d) + "(const TailJitArgs& a, const u32* w, const u32* nc) {\n";
+    const std::string MT = a.r > 32 ? "u64" : "u32";
+    s += "__device__ __forceinline__ " + MT + " tmask" + std::to_string(d) + "(const TailJitArgs& a, const u32* w, const u32* nc) {\n";
     s += g.loads("  ");
-    s += "  u32 m = " + hex(a.r >= 32 ? 0xffffffffu : ((1u << a.r) - 1u)) + ";\n";
+    if (a.r > 32)
+      s += "  u64 m = " + (a.r == 64 ? std::string("0xffffffffffffffffull") : "((1ull << " + std::to_string(a.r) + ") - 1ull)") + ";\n";
+    else
+      s += "  u32 m = " + hex(a.r >= 32 ? 0xffffffffu : ((1u << a.r) - 1u)) + ";\n";
     for (int tt = 0; tt < a.n_terms; tt++) {
       if (ncoff[d][tt] >= 0) {
         s += term_mask_code(a, tt, cx[d], cm[d], "(nc + " + std::to_string(ncoff[d][tt]) + ")");
@@ -458,9 +465,9 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   for (int d = nl - 1; d >= 0; d--) {
     const std::string ds = std::to_string(d);
     s += "__device__ __forceinline__ void cnt" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cnt) {\n";
-    s += "  u32 m = tmask" + ds + "(a, w, nc);\n  cnt[" + ds + "] += __popc(m);\n";
+    s += "  auto m = tmask" + ds + "(a, w, nc);\n  cnt[" + ds + "] += __popcll((u64)m);\n";
     if (d + 1 < nl) {
-      s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
+      s += "  while (m) {\n    const u32 cc = __ffsll((long long)m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
       s += child(d, "w", "cw", "    ");
       s += "    cnt" + std::to_string(d + 1) + "(a, cw, nc, cnt);\n  }\n";
     }
@@ -502,8 +509,8 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
     const std::string ds = std::to_string(d);
     s += "__device__ __forceinline__ void dfs" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cur, "
          "const u64* base, const u32* pb, unsigned char* sm, bool staged, const u32* roff, const u32* coff, u32 lmo) {\n";
-    s += "  u32 m = tmask" + ds + "(a, w, nc);\n";
-    s += "  while (m) {\n    const u32 cc = __ffs(m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
+    s += "  auto m = tmask" + ds + "(a, w, nc);\n";
+    s += "  while (m) {\n    const u32 cc = __ffsll((long long)m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
     s += child(d, "w", "cw", "    ");
     s += "    const u32 slot = cur[" + ds + "]++;\n";
     s += "    if (staged) {\n      u32* dst = reinterpret_cast<u32*>(sm + roff[" + ds + "]) + (slot - pb[" + ds + "]) * " + Ws + ";\n";
