@@ -1408,16 +1408,13 @@ static TailArgs tail_protos(const GroupPlan& gp, int k0) {
   return t;
 }
 
-// First level of group g's fused narrow tail: the longest run of trailing
-// levels (2..kMaxTail) that are all narrow fast levels with 1 <= r <= 32 and whose per-warp
-// emit buffers (32 * r * words * 4 bytes per level) fit 16 KB; -1 if none.  These rules are the
-// generic tail kernels' (expand.cuh).  The NVRTC tail has neither limit for its inner levels: it
-// takes r <= 64 (u64 masks) above the leaf level and stages any subtree size in parts, so when
-// the longer run it allows compiles (tried once per group, here, before the tail is chosen),
-// that run is the tail.  `assume_jit`: the extended choice without compiling (source tests).
-static int tail_start(atf_space* s, int g, bool assume_jit = false) {
+// First level of group g's fused narrow tail for the generic tail kernels (expand.cuh): the
+// longest run of trailing levels (2..kMaxTail) that are all narrow fast levels with
+// 1 <= r <= 32 and whose per-warp emit buffers (32 * r * words * 4 bytes per level) fit 16 KB;
+// -1 if none.
+static int tail_start_generic(const atf_space* s, int g) {
   if (s->opts.flags & (ATF_FLAG_NO_TAIL | ATF_FLAG_LEGACY_WIDE | ATF_FLAG_GENERIC_ONLY)) return -1;
-  GroupPlan& gp = s->groups[g];
+  const GroupPlan& gp = s->groups[g];
   const int L = (int)gp.levels.size();
   int k0 = L, bytes = 0;
   while (k0 > 0 && L - k0 < kMaxTail) {
@@ -1428,22 +1425,35 @@ static int tail_start(atf_space* s, int g, bool assume_jit = false) {
     bytes += b;
     k0--;
   }
-  const int k0c = L - k0 >= 2 ? k0 : -1;
-  if (s->opts.flags & ATF_FLAG_NO_JIT) return k0c;
+  return L - k0 >= 2 ? k0 : -1;
+}
+
+// The NVRTC tail has neither limit for its inner levels: it takes r <= 64 (u64 masks) above
+// the leaf level and stages any subtree size in parts.  Its longer run (-1 if it is not longer
+// than the generic one, or NVRTC is off).
+static int tail_start_ext(const atf_space* s, int g) {
+  if (s->opts.flags & (ATF_FLAG_NO_TAIL | ATF_FLAG_LEGACY_WIDE | ATF_FLAG_GENERIC_ONLY | ATF_FLAG_NO_JIT)) return -1;
+  const GroupPlan& gp = s->groups[g];
+  const int L = (int)gp.levels.size();
   int ke = L;
   while (ke > 0 && L - ke < kMaxTail) {
     const LevelPlan& lp = gp.levels[ke - 1];
     if (!lp.proto.nf_ok || lp.generic || lp.r < 1 || lp.r > (ke == L ? 32 : 64)) break;
     ke--;
   }
-  if (L - ke < 2 || (k0c >= 0 && ke >= k0c)) return k0c;
-  if (assume_jit) return ke;
+  const int kc = tail_start_generic(s, g);
+  return (L - ke >= 2 && (kc < 0 || ke < kc)) ? ke : -1;
+}
+
+// The tail's kernels for a start it was not built for yet (once per group and start).
+static bool tail_ext_compiled(atf_space* s, int g, int ke) {
+  GroupPlan& gp = s->groups[g];
   if (gp.tail_ext_k0 != ke) {
     gp.tail_ext_k0 = ke;
     std::vector<std::vector<int32_t>> cx;
     std::vector<std::vector<uint32_t>> cm;
     std::vector<std::vector<int>> pvl;
-    tail_jit_inputs(s, gp, ke, L - ke, cx, cm, pvl);
+    tail_jit_inputs(s, gp, ke, (int)gp.levels.size() - ke, cx, cm, pvl);
     const TailArgs t = tail_protos(gp, ke);
     void* kern = jit_tail_kernels(t, gp.words, cx, cm, ke, pvl);
     gp.tail_ext_ok = kern != nullptr;
@@ -1452,7 +1462,25 @@ static int tail_start(atf_space* s, int g, bool assume_jit = false) {
       gp.tail_jit_k0 = ke;
     }
   }
-  return gp.tail_ext_ok ? ke : k0c;
+  return gp.tail_ext_ok;
+}
+
+// Does group g's fused tail start at level k (frontier = the level above, `frontier` nodes in
+// the whole space)?  The longer NVRTC run when it compiles and its frontier holds at least
+// kTailExtMinFrontier nodes (a deeper tail over a small frontier leaves most SMs idle; the
+// frontier size is known when level k is reached, so the choice is made then, the same way in
+// every generation and on every rank), else the generic run.
+constexpr uint64_t kTailExtMinFrontier = 65536;
+static bool tail_here(atf_space* s, int g, int k, uint64_t frontier) {
+  const int ke = tail_start_ext(s, g);
+  if (ke >= 0 && k == ke && frontier >= kTailExtMinFrontier && tail_ext_compiled(s, g, ke)) return true;
+  return k == tail_start_generic(s, g);
+}
+
+// The longest tail (source tests): the NVRTC run when there is one.
+static int tail_start(const atf_space* s, int g) {
+  const int ke = tail_start_ext(s, g);
+  return ke >= 0 ? ke : tail_start_generic(s, g);
 }
 
 // Count round of the tail of group g from frontier `parents` (level k0 - 1, n_parents nodes):
@@ -1665,7 +1693,7 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       atf_status e;
       if (s->tails[g].phase == 1) {
         e = queue_tail_emit(s, g, pd, active > 1);
-      } else if (k[i] == tail_start(s, g)) {
+      } else if (tail_here(s, g, k[i], fsize[i])) {
         e = queue_tail_count(s, g, k[i], frontier[i], fsize[i], pd, active > 1);
       } else {
         e = queue_level(s, g, k[i], frontier[i], fsize[i], pd, active > 1);
@@ -1795,7 +1823,7 @@ static atf_status run_levels_replay(atf_space* s) {
         if ((e = queue_tail_emit(s, (int)g, pd, active > 1))) return e;
         tails_done.push_back((int)g);
         k[g] = L;
-      } else if (k[g] == tail_start(s, (int)g)) {
+      } else if (tail_here(s, (int)g, k[g], fsize[g])) {
         if ((e = queue_tail_count(s, (int)g, k[g], frontier[g], fsize[g], pd, active > 1))) return e;
         for (int d = 0; d < T.nl; d++) T.tot[d] = s->replay_f[g][k[g] + d];
         T.phase = 1;  // the emit is queued next round, sized from the expected totals
@@ -1976,7 +2004,7 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
         atf_status e;
         if (s->tails[g].phase == 1) {
           e = queue_tail_emit(s, (int)g, pd, active > 1);
-        } else if (k[g] == tail_start(s, (int)g)) {
+        } else if (tail_here(s, (int)g, k[g], F[g])) {
           e = queue_tail_count(s, (int)g, k[g], frontier[g], np, pd, active > 1);
         } else {
           e = queue_level(s, (int)g, k[g], frontier[g], np, pd, active > 1);
@@ -3078,7 +3106,7 @@ atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, 
   if (e) return e;
   if (g < 0 || g >= (int)s->groups.size()) return ATF_ERR_INVALID_ARG;
   const GroupPlan& gp = s->groups[g];
-  const int k0 = tail_start(s, g, /*assume_jit=*/true);
+  const int k0 = tail_start(s, g);
   if (k0_out) *k0_out = k0;
   std::string src;
   if (k0 >= 0) {

@@ -489,44 +489,52 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
     s += "      if (lane == 0) a.tile_total[(u64)" + ds + " * a.n_tiles + tile] = v; }\n";
   }
   s += "  }\n}\n";
-  // ---- emit: level-synchronous passes over a warp tile of 32 frontier nodes, staged per warp.
-  // The count pass's subtree counts + warp scans give every lane's tile-local positions per level
-  // and a per-lane byte size.  The warp writes the tile in "parts": runs of consecutive lanes
-  // whose output (records, CSR entries as u32 tile-local child offsets, a u8 frontier-lane tag
-  // per inner node) fits the warp's staging area.  Per part, pass 0: each frontier lane writes
-  // its children (its node constants in registers); pass d >= 1: the lanes stride over the part's
-  // level-(d-1) nodes in canonical order, 32 at a time, each computing one node's child mask
-  // (node constants of the node's frontier lane from a shared-memory table), a warp scan places
-  // the children, so the mask work is balanced across lanes whatever the subtree shapes.  The
-  // warp then copies every level's run out as coalesced vectors.  A single lane whose subtree
-  // alone exceeds the area writes it depth-first straight to global memory.
+  // ---- emit: lane = frontier node, depth-first (like the count), output staged per warp.
+  // Each lane recounts its subtree (cnt_d); warp scans give its nodes' tile-local positions per
+  // level (a node's level-d descendants come out of a depth-first walk in canonical order).  The
+  // warp then writes the tile in "parts": runs of consecutive lanes whose output (records, and
+  // CSR entries as u32 offsets from the child level's tile base) fits the warp's staging area;
+  // the lanes of a part write their subtrees into shared memory, the warp copies every level's
+  // run out as coalesced words.  A single lane whose subtree alone exceeds the area writes
+  // straight to global memory.
   constexpr int kStage = 8192;  // staging bytes per warp
   if (warp_bytes) *warp_bytes = kStage;
   const std::string NLs = std::to_string(nl), NCs = std::to_string(NC), RB = std::to_string(W * 4);
-  const int NCB = (NC * 32 * 4 + 15) & ~15;  // node-constant table at the start of the area
-  const std::string NCBs = std::to_string(NCB);
-  // depth-first direct path (one oversized lane)
+  // The leaf level is not written by the depth-first walk when staged: a level-(nl-2) node stores
+  // its leaf mask instead (and advances the leaf cursor by its popcount), and a balanced pass over
+  // the part's level-(nl-2) nodes (lane-strided) writes the leaves afterwards, so the walk's
+  // divergence does not reach the largest level.
+  const int LP = nl - 2;  // parents of the leaves
   for (int d = nl - 1; d >= 0; d--) {
     const std::string ds = std::to_string(d);
     s += "__device__ __forceinline__ void dfs" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cur, "
-         "const u64* base) {\n";
+         "const u64* base, const u32* pb, unsigned char* sm, bool staged, const u32* roff, const u32* coff, u32 lmo) {\n";
     s += "  auto m = tmask" + ds + "(a, w, nc);\n";
     s += "  while (m) {\n    const u32 cc = __ffsll((long long)m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
     s += child(d, "w", "cw", "    ");
     s += "    const u32 slot = cur[" + ds + "]++;\n";
-    s += "    u32* dst = a.rec[" + ds + "] + (base[" + ds + "] + slot) * " + Ws + ";\n";
-    for (int w = 0; w < W; w++) s += "    dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
+    s += "    if (staged) {\n      u32* dst = reinterpret_cast<u32*>(sm + roff[" + ds + "]) + (slot - pb[" + ds + "]) * " + Ws + ";\n";
+    for (int w = 0; w < W; w++) s += "      dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
+    s += "    } else {\n      u32* dst = a.rec[" + ds + "] + (base[" + ds + "] + slot) * " + Ws + ";\n";
+    for (int w = 0; w < W; w++) s += "      dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
+    s += "    }\n";
     if (d + 1 < nl) {
       const std::string d1 = std::to_string(d + 1);
-      s += "    a.csr[" + d1 + "][base[" + ds + "] + slot] = base[" + d1 + "] + cur[" + d1 + "];\n";
-      s += "    dfs" + d1 + "(a, cw, nc, cur, base);\n";
+      s += "    if (staged) reinterpret_cast<u32*>(sm + coff[" + ds + "])[slot - pb[" + ds + "]] = cur[" + d1 + "];\n";
+      s += "    else a.csr[" + d1 + "][base[" + ds + "] + slot] = base[" + d1 + "] + cur[" + d1 + "];\n";
+      if (d == LP) {
+        s += "    if (staged) {\n      const u32 lm = tmask" + d1 + "(a, cw, nc);\n";
+        s += "      reinterpret_cast<u32*>(sm + lmo)[slot - pb[" + ds + "]] = lm;\n      cur[" + d1 + "] += __popc(lm);\n";
+        s += "    } else {\n      dfs" + d1 + "(a, cw, nc, cur, base, pb, sm, staged, roff, coff, lmo);\n    }\n";
+      } else {
+        s += "    dfs" + d1 + "(a, cw, nc, cur, base, pb, sm, staged, roff, coff, lmo);\n";
+      }
     }
     s += "  }\n}\n";
   }
   s += "extern \"C\" __global__ void __launch_bounds__(128) atf_tail_emit(const __grid_constant__ TailJitArgs a) {\n";
   s += "  extern __shared__ __align__(16) unsigned char smem[];\n";
   s += "  const int lane = threadIdx.x & 31;\n  unsigned char* sm = smem + (threadIdx.x >> 5) * " + std::to_string(kStage) + ";\n";
-  s += "  u32* ncs = reinterpret_cast<u32*>(sm);  // [NC][32] node constants of the tile's frontier lanes\n";
   s += "  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n  const u64 gw = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5;\n";
   s += "  if (gw == 0 && lane < " + NLs + ") {\n";
   s += "    const u64 above = lane == 0 ? a.n_parents : a.tile_base[(u64)(lane - 1) * (a.n_tiles + 1) + a.n_tiles];\n";
@@ -551,88 +559,68 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "#pragma unroll\n    for (int i = 0; i < " + Ws + "; i++) w[i] = pw_[i];\n";
   s += "#pragma unroll\n    for (int d = 0; d < " + NLs + "; d++) { cnt[d] = pc_[d]; base[d] = pb_[d]; }\n";
   s += "    if (tile + nw < a.n_tiles) {\n" + load_next("(tile + nw)", "      ") + "    }\n";
-  s += "    u32 nc[" + NCs + "] = {};\n";
+  s += "    u32 nc[" + NCs + "];\n";
   s += "    if (valid) tnc(a, w, nc);\n";
-  s += "    __syncwarp();  // the previous tile's last reads of the table\n";
-  s += "#pragma unroll\n    for (int k = 0; k < " + NCs + "; k++) ncs[k * 32 + lane] = nc[k];\n";
   s += "    u32 off[" + NLs + "];\n    u32 bytes = 0;\n";
   s += "#pragma unroll\n    for (int d = 0; d < " + NLs + "; d++) {\n";
   s += "      u32 incl = cnt[d];\n#pragma unroll\n      for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
        "if (lane >= o) incl += y; }\n";
   s += "      off[d] = incl - cnt[d];\n";
-  s += "      bytes += cnt[d] * (" + RB + "u + (d + 1 < " + NLs + " ? 5u : 0u));\n    }\n";
+  s += "      bytes += cnt[d] * (" + RB + "u + (d + 1 < " + NLs + " ? 4u : 0u) + (d == " + std::to_string(nl - 2) + " ? 4u : 0u));\n    }\n";
   s += "    if (valid) a.csr[0][nd] = base[0] + off[0];\n";
   // inclusive byte prefix per lane
   s += "    u32 bincl = bytes;\n#pragma unroll\n    for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, bincl, o); "
        "if (lane >= o) bincl += y; }\n";
-  s += "    __syncwarp();\n";
   s += "    for (int p0 = 0; p0 < 32;) {\n";
   s += "      const u32 b0 = p0 ? __shfl_sync(0xffffffffu, bincl, p0 - 1) : 0u;\n";
-  s += "      const unsigned fit = __ballot_sync(0xffffffffu, lane >= p0 && bincl - b0 <= " + std::to_string(kStage - NCB - 16) +
-       "u);  // 16: the record region's alignment\n";
+  s += "      const unsigned fit = __ballot_sync(0xffffffffu, lane >= p0 && bincl - b0 <= " + std::to_string(kStage - 16) + "u);  // 16: the record region's alignment\n";
   s += "      const int p1 = fit ? 32 - __clz(fit) : p0 + 1;  // lanes [p0, p1)\n";
-  s += "      if (!fit) {  // lane p0's subtree alone exceeds the area: depth-first, straight to global memory\n";
-  s += "        if (lane == p0 && valid) {\n          u32 cur[" + NLs + "];\n";
-  s += "#pragma unroll\n          for (int d = 0; d < " + NLs + "; d++) cur[d] = off[d];\n";
-  s += "          dfs0(a, w, nc, cur, base);\n        }\n        __syncwarp();\n        p0 = p1;\n        continue;\n      }\n";
-  s += "      u32 pb[" + NLs + "], pe[" + NLs + "], roff[" + NLs + "], coff[" + NLs + "], toff[" + NLs + "];\n";
-  s += "      u32 o = " + NCBs + "u;\n";
+  s += "      const bool staged = fit != 0u;\n";
+  s += "      u32 pb[" + NLs + "], pe[" + NLs + "], roff[" + NLs + "], coff[" + NLs + "];\n";
+  s += "      u32 o = 0;\n";
   s += "#pragma unroll\n      for (int d = 0; d < " + NLs + "; d++) {\n";
   s += "        pb[d] = __shfl_sync(0xffffffffu, off[d], p0);\n";
-  s += "        pe[d] = __shfl_sync(0xffffffffu, off[d] + cnt[d], p1 - 1);\n";
-  s += "        if (d + 1 < " + NLs + ") { coff[d] = o; o += (pe[d] - pb[d]) * 4u; }\n      }\n";
-  s += "#pragma unroll\n      for (int d = 0; d + 1 < " + NLs + "; d++) { toff[d] = o; o += pe[d] - pb[d]; }\n";
+  s += "        const u32 last = __shfl_sync(0xffffffffu, off[d] + cnt[d], p1 - 1);\n        pe[d] = last;\n";
+  s += "        if (d + 1 < " + NLs + ") { coff[d] = o; o += (last - pb[d]) * 4u; }\n      }\n";
+  s += "      const u32 lmo = o;  // leaf masks of the part's level-" + std::to_string(nl - 2) + " nodes\n";
+  s += "      o += (pe[" + std::to_string(nl - 2) + "] - pb[" + std::to_string(nl - 2) + "]) * 4u;\n";
   s += "      o = (o + 15u) & ~15u;\n";
   s += "#pragma unroll\n      for (int d = 0; d < " + NLs + "; d++) { roff[d] = o; o += (pe[d] - pb[d]) * " + RB + "u; }\n";
-  // pass 0: the frontier lanes' children
-  {
-    s += "      if (lane >= p0 && lane < p1 && valid) {  // pass 0: the part's frontier lanes\n";
-    s += "        auto m = tmask0(a, w, nc);\n        u32 slot = off[0] - pb[0];\n";
-    s += "        while (m) {\n          const u32 cc = __ffsll((long long)m) - 1;\n          m &= m - 1;\n";
-    s += "          u32 cw[" + Ws + "];\n" + child(0, "w", "cw", "          ");
-    s += "          u32* dst = reinterpret_cast<u32*>(sm + roff[0]) + slot * " + Ws + ";\n";
-    for (int w = 0; w < W; w++) s += "          dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
-    if (nl > 1) s += "          sm[toff[0] + slot] = (unsigned char)lane;\n";
-    s += "          slot++;\n        }\n      }\n      __syncwarp();\n";
-  }
-  // passes 1..nl-1: balanced over the part's level-(d-1) nodes
-  for (int d = 1; d < nl; d++) {
-    const std::string ds = std::to_string(d), dp = std::to_string(d - 1);
-    s += "      {  // pass " + ds + ": children of the part's level-" + dp + " nodes, 32 nodes at a time\n";
-    s += "        const u32 n = pe[" + dp + "] - pb[" + dp + "];\n        u32 run = 0;\n";
-    s += "        for (u32 c0 = 0; c0 < n; c0 += 32) {\n";
-    s += "          const u32 i = c0 + lane;\n          const bool act = i < n;\n";
-    s += "          u32 pw[" + Ws + "], ncl[" + NCs + "];\n          u32 tg = 0;\n";
-    s += "          if (act) {\n            const u32* pr = reinterpret_cast<const u32*>(sm + roff[" + dp + "]) + i * " + Ws + ";\n";
+  s += "      if (lane >= p0 && lane < p1 && valid) {\n        u32 cur[" + NLs + "];\n";
+  s += "#pragma unroll\n        for (int d = 0; d < " + NLs + "; d++) cur[d] = off[d];\n";
+  s += "        dfs0(a, w, nc, cur, base, pb, sm, staged, roff, coff, lmo);\n      }\n";
+  s += "      if (staged) {\n        __syncwarp();\n";
+  {  // balanced leaf pass
+    const std::string lp = std::to_string(nl - 2), ll = std::to_string(nl - 1);
+    const int fw = t.lv[nl - 1].field_word, fs = t.lv[nl - 1].field_shift;
+    s += "        {  // leaves of the part's level-" + lp + " nodes, lane-strided\n";
+    s += "          const u32 nn = pe[" + lp + "] - pb[" + lp + "];\n";
+    s += "          const u32* lms = reinterpret_cast<const u32*>(sm + lmo);\n";
+    s += "          const u32* cst = reinterpret_cast<const u32*>(sm + coff[" + lp + "]);\n";
+    s += "          for (u32 i = lane; i < nn; i += 32) {\n            u32 lm = lms[i];\n            if (!lm) continue;\n";
+    s += "            u32 k = cst[i] - pb[" + ll + "];\n";
+    s += "            const u32* pr = reinterpret_cast<const u32*>(sm + roff[" + lp + "]) + i * " + Ws + ";\n";
+    s += "            u32 pw[" + Ws + "];\n";
     for (int w = 0; w < W; w++) s += "            pw[" + std::to_string(w) + "] = pr[" + std::to_string(w) + "];\n";
-    s += "            tg = sm[toff[" + dp + "] + i];\n";
-    s += "#pragma unroll\n            for (int k = 0; k < " + NCs + "; k++) ncl[k] = ncs[k * 32 + tg];\n";
-    s += "          }\n";
-    s += "          auto m = tmask" + ds + "(a, pw, ncl);\n          if (!act) m = 0;\n";
-    s += "          const u32 c = __popcll((u64)m);\n          u32 incl = c;\n";
-    s += "#pragma unroll\n          for (int o2 = 1; o2 < 32; o2 <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o2); if (lane >= o2) incl += y; }\n";
-    s += "          u32 slot = run + incl - c;\n          run += __shfl_sync(0xffffffffu, incl, 31);\n";
-    s += "          if (act) reinterpret_cast<u32*>(sm + coff[" + dp + "])[i] = pb[" + ds + "] + slot;\n";
-    s += "          while (m) {\n            const u32 cc = __ffsll((long long)m) - 1;\n            m &= m - 1;\n";
-    s += "            u32 cw[" + Ws + "];\n" + child(d, "pw", "cw", "            ");
-    s += "            u32* dst = reinterpret_cast<u32*>(sm + roff[" + ds + "]) + slot * " + Ws + ";\n";
-    for (int w = 0; w < W; w++) s += "            dst[" + std::to_string(w) + "] = cw[" + std::to_string(w) + "];\n";
-    if (d + 1 < nl) s += "            sm[toff[" + ds + "] + slot] = (unsigned char)tg;\n";
-    s += "            slot++;\n          }\n        }\n        __syncwarp();\n      }\n";
+    s += "            while (lm) {\n              const u32 cc = __ffs(lm) - 1;\n              lm &= lm - 1;\n";
+    s += "              u32* dst = reinterpret_cast<u32*>(sm + roff[" + ll + "]) + k * " + Ws + ";\n";
+    for (int w = 0; w < W; w++)
+      s += "              dst[" + std::to_string(w) + "] = pw[" + std::to_string(w) + "]" +
+           (w == fw && t.lv[nl - 1].r > 1 ? " | (cc << " + std::to_string(fs) + ")" : "") + ";\n";
+    s += "              k++;\n            }\n          }\n          __syncwarp();\n        }\n";
   }
-  // copy-out
-  s += "#pragma unroll\n      for (int d = 0; d < " + NLs + "; d++) {\n";
-  s += "        const u32 n = (pe[d] - pb[d]) * " + Ws + "u;\n";
-  s += "        const u32* src = reinterpret_cast<const u32*>(sm + roff[d]);\n        u32* dst = a.rec[d] + (base[d] + pb[d]) * " + Ws + ";\n";
-  if (W % 2 == 0)  // 8-byte aligned on both sides (records of even W, 16-byte aligned regions)
-    s += "        { const uint2* s2 = reinterpret_cast<const uint2*>(src); uint2* d2 = reinterpret_cast<uint2*>(dst);\n"
-         "#pragma unroll 4\n          for (u32 v = lane; v < n / 2; v += 32) d2[v] = s2[v]; }\n";
+  s += "#pragma unroll\n        for (int d = 0; d < " + NLs + "; d++) {\n";
+  s += "          const u32 n = (pe[d] - pb[d]) * " + Ws + "u;\n";
+  s += "          const u32* src = reinterpret_cast<const u32*>(sm + roff[d]);\n          u32* dst = a.rec[d] + (base[d] + pb[d]) * " + Ws + ";\n";
+  if (W % 2 == 0)  // 8-byte aligned on both sides (records of even W, 8-byte CSR regions before them)
+    s += "          { const uint2* s2 = reinterpret_cast<const uint2*>(src); uint2* d2 = reinterpret_cast<uint2*>(dst);\n"
+         "#pragma unroll 4\n            for (u32 v = lane; v < n / 2; v += 32) d2[v] = s2[v]; }\n";
   else
-    s += "#pragma unroll 4\n        for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
-  s += "        if (d + 1 < " + NLs + ") {\n          const u32* cs = reinterpret_cast<const u32*>(sm + coff[d]);\n";
-  s += "          u64* cd = a.csr[d + 1] + base[d] + pb[d];\n          const u64 cb = base[d + 1 < " + NLs + " ? d + 1 : d];\n";
-  s += "#pragma unroll 4\n          for (u32 v = lane; v < pe[d] - pb[d]; v += 32) cd[v] = cb + cs[v];\n        }\n";
-  s += "      }\n      __syncwarp();\n      p0 = p1;\n    }\n  }\n}\n";
+    s += "#pragma unroll 4\n          for (u32 v = lane; v < n; v += 32) dst[v] = src[v];\n";
+  s += "          if (d + 1 < " + NLs + ") {\n            const u32* cs = reinterpret_cast<const u32*>(sm + coff[d]);\n";
+  s += "            u64* cd = a.csr[d + 1] + base[d] + pb[d];\n            const u64 cb = base[d + 1 < " + NLs + " ? d + 1 : d];\n";
+  s += "#pragma unroll 4\n            for (u32 v = lane; v < pe[d] - pb[d]; v += 32) cd[v] = cb + cs[v];\n          }\n";
+  s += "        }\n        __syncwarp();\n      }\n      p0 = p1;\n    }\n  }\n}\n";
   return s;
 }
 

@@ -223,6 +223,20 @@ def test_tail_kernel_runs(Space):
             assert [x["level"] for x in sp.stats() if x["group"] == 0 and x["kernel"] == 5] == want
 
 
+def test_extended_tail_runs(Space):
+    """C3-IS4: the NVRTC tail also takes KWI (r = 64 > 32, u64 masks) since its frontier (NDIMB's
+    level, 6.8e6 nodes) is large; the generic tail kernels keep the r <= 32 run VWM, VWN.  Both
+    generate the golden space (test_full_size_against_golden covers the content)."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    spec = A.c3_xgemm("IS4")
+    for flags, kern, want in ((0, 6, [7, 8, 9]), (L.ATF_FLAG_NO_JIT, 5, [8, 9])):
+        with Space(spec, flags=L.ATF_FLAG_TIMING | flags) as sp:
+            sp.generate()
+            st = [x for x in sp.stats() if x["group"] == 0]
+            assert [x["level"] for x in st if x["kernel"] == kern] == want
+            assert sp.size() == 1613777840
+
+
 def test_jit_kernels_run(Space):
     """The narrow levels of C3 run the NVRTC-specialised kernel (kernel id 4) on the GPU box."""
     from paper_conf_hpdc_raschg18_b200 import _lib as L
