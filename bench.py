@@ -348,42 +348,80 @@ def secondary_n1(steps, warmup, sm_mhz):
     return out
 
 
-def predicted_scaling(spec, worlds=(2, 4, 8), reps=3, ag_us=25.0):
+def predicted_scaling(spec, worlds=(2, 4, 8), reps=3, ag_us=25.0, flag_us=10.0):
     """One-GPU prediction of the balanced multi-GPU generation (atf_space_generate_dist,
     DESIGN.md §6): N virtual ranks (N spaces of this process) run the real per-level protocol
     (same kernels, same partition, parent slices copied between ranks' arenas), one rank at a
-    time per level round; each rank's round is timed on the host (launches + device work +
-    sync).  T_N = sum over rounds of the slowest rank's round + rounds x an all-gather latency
-    (ag_us, an assumption: an NCCL all-gather of < 2 KB over NVLink; not measurable on one GPU);
-    efficiency = T_1 / (N T_N), T_1 from the same procedure with one rank.  A prediction, not a
-    scaling measurement (no NVLink transfers, no contention between real GPUs)."""
+    time per level round, so each rank's round runs alone on the GPU.
+
+    "sync": the synchronous protocol (first generations): each rank's round timed on the host
+    (launches + device work + sync); T_N = sum over rounds of the slowest rank's round + rounds x
+    an all-gather latency (ag_us, an assumption: a < 2 KB NCCL all-gather over NVLink).
+    "replay": the steady state (every later generation; no host synchronisation per round, device
+    flags between ranks): each rank's round timed on the DEVICE (CUDA events around its kernels,
+    CSR fix-ups and peer copies, ATF_FLAG_TIMING); T_N = sum over rounds of the slowest rank's
+    device round + exchanged rounds x flag_us (a flag-set + flag-wait over NVLink, assumed) + one
+    verdict all-gather (ag_us).  Validated at N = 1: the measured replay time of one rank
+    ("replay_measured_1_ms", CUDA events around generate_dist, world 1, steady state).
+    efficiency = T_1 / (N T_N) with T_1 from the same procedure.  A prediction, not a scaling
+    measurement (no NVLink transfers, no contention between real GPUs)."""
     import torch
-    from paper_conf_hpdc_raschg18_b200 import Space
+    from paper_conf_hpdc_raschg18_b200 import Space, _lib as L
     from paper_conf_hpdc_raschg18_b200.shard import virtual_ranks
     out = {}
     for N in (1,) + tuple(worlds):
-        spaces = [Space(spec, flags=headline_flags()) for _ in range(N)]
-        try:
-            virtual_ranks(spaces)  # warm-up: arenas, JIT, IPC mappings
-            best = None
-            for _ in range(reps):
+        rec = {}
+        for mode, extra in (("sync", L.ATF_FLAG_NO_REPLAY), ("replay", L.ATF_FLAG_TIMING)):
+            spaces = [Space(spec, flags=headline_flags() | extra) for _ in range(N)]
+            try:
+                virtual_ranks(spaces)  # warm-up: arenas, JIT, IPC mappings
+                best = None
+                for _ in range(reps):
+                    torch.cuda.synchronize()
+                    vag = virtual_ranks(spaces, serialize=True)
+                    if mode == "sync":
+                        per = [vag.round_s[r] for r in range(N)]
+                        rounds = len(per[0])
+                        t = sum(max(per[r][i] for r in range(N)) for i in range(rounds)) + (rounds - 1) * ag_us * 1e-6
+                    else:
+                        per = [[x * 1e-3 for x in sp.dist_round_ms()] for sp in spaces]
+                        rounds = len(per[0])
+                        ex = vag.calls[0]  # exchanged rounds (one all-gather each)
+                        t = sum(max(per[r][i] for r in range(N)) for i in range(rounds)) + \
+                            (ex * flag_us + ag_us) * 1e-6
+                    if best is None or t < best[0]:
+                        best = (t, rounds, [sum(x) for x in per],
+                                [round(max(per[r][i] for r in range(N)) * 1e3, 3) for i in range(rounds)])
+                rec[mode] = {"T_ms": best[0] * 1e3, "rounds": best[1], "rank_busy_ms": [round(x * 1e3, 3) for x in best[2]],
+                             "round_max_ms": best[3]}
+            finally:
+                for sp in spaces:
+                    sp.close()
+        out[N] = rec
+    # N = 1 steady-state replay, measured (validates the device-time model)
+    sp = Space(spec, flags=headline_flags(), stream=torch.cuda.Stream())
+    try:
+        with torch.cuda.stream(sp._stream_obj):
+            for _ in range(3):
+                sp.generate_dist(0, 1, lambda b: b)
+            ts = []
+            for _ in range(reps + 2):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record()
+                sp.generate_dist(0, 1, lambda b: b)
+                e1.record()
                 torch.cuda.synchronize()
-                vag = virtual_ranks(spaces, serialize=True)
-                rounds = len(vag.round_s[0])
-                t = sum(max(vag.round_s[r][i] for r in range(N)) for i in range(rounds)) + (rounds - 1) * ag_us * 1e-6
-                if best is None or t < best[0]:
-                    best = (t, rounds, [sum(x) for x in vag.round_s],
-                            [round(max(vag.round_s[r][i] for r in range(N)) * 1e3, 3) for i in range(rounds)])
-            out[N] = {"T_ms": best[0] * 1e3, "rounds": best[1], "rank_busy_ms": [round(x * 1e3, 3) for x in best[2]],
-                      "round_max_ms": best[3]}
-        finally:
-            for sp in spaces:
-                sp.close()
-    t1 = out[1]["T_ms"]
-    for N in worlds:
-        out[N]["efficiency"] = t1 / (N * out[N]["T_ms"])
-    return {"method": predicted_scaling.__doc__.split("\n\n")[0].replace("\n", " "), "allgather_us_assumed": ag_us,
-            "per_world": {str(k): v for k, v in out.items()}}
+                ts.append(e0.elapsed_time(e1))
+        measured1 = min(ts)
+    finally:
+        sp.close()
+    res = {"method": predicted_scaling.__doc__.split("\n\n")[0].replace("\n", " "),
+           "allgather_us_assumed": ag_us, "flag_us_assumed": flag_us, "replay_measured_1_ms": measured1}
+    for mode in ("sync", "replay"):
+        t1 = out[1][mode]["T_ms"]
+        res[mode] = {str(N): dict(out[N][mode], **({"efficiency": t1 / (N * out[N][mode]["T_ms"])} if N > 1 else {}))
+                     for N in out}
+    return res
 
 
 def cpu_baseline(spec, budget_s=15.0):

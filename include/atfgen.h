@@ -220,6 +220,22 @@ atf_status atf_space_finalize_shard(atf_space* s, const int64_t* h_all_counts, i
  * with the same spec; errors are local (a failing rank makes the others fail in the callback). */
 typedef int (*atf_allgather_fn)(const void* send, void* recv, size_t bytes, void* ctx);
 atf_status atf_space_generate_dist(atf_space* s, int32_t rank, int32_t world, atf_allgather_fn allgather, void* ctx);
+/* Steady state of atf_space_generate_dist (like the single-GPU replay): the
+ * space logs every round's all-gathered records.  The next call with the same rank, world and
+ * flags sizes every level from the log (its allocations -- hence the addresses peers read --
+ * are then those the replay reproduces); if every count matched, later calls queue all rounds
+ * with no host synchronisation and no all-gather per round: each rank marks a finished round in
+ * a device flag array (exported by CUDA IPC) and its stream waits on the owners' flags before a
+ * peer copy.  One synchronisation and ONE all-gather of 4-byte verdicts per call then check
+ * every level total, overflow flag, wait time-out and address against the log on every rank; a
+ * failed check regenerates with the synchronous protocol in the same call.  Not used with
+ * ATF_FLAG_NO_REPLAY or ATF_FLAG_TIMING.  Ranks sharing one device must use different streams
+ * (a wait on the legacy default stream would block the owner's work until its 2 s time-out).
+ *
+ * atf_space_dist_round_ms: with ATF_FLAG_TIMING, the device time of each round of this rank's
+ * last atf_space_generate_dist (CUDA events on the space's stream around the round's kernels,
+ * CSR fix-ups and peer copies), out[0..n) (host), *n_out = rounds; ATF_ERR_STATE without them. */
+atf_status atf_space_dist_round_ms(const atf_space* s, float* out, int32_t cap, int32_t* n_out);
 
 /* ---- results (state GENERATED) ---------------------------------------------------- */
 

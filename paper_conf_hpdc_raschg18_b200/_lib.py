@@ -91,6 +91,7 @@ _SIGS = {
                                   C.c_void_p, C.c_void_p]),
     "atf_space_stats": (_st, [SP, C.POINTER(atf_level_stats), C.c_int32, C.POINTER(C.c_int32)]),
     "atf_space_generate_dist": (_st, [SP, C.c_int32, C.c_int32, ALLGATHER_FN, C.c_void_p]),
+    "atf_space_dist_round_ms": (_st, [SP, C.POINTER(C.c_float), C.c_int32, C.POINTER(C.c_int32)]),
     "atf_space_destroy": (None, [SP]),
     "atf_status_str": (C.c_char_p, [_st]),
     "atf_space_last_error": (C.c_char_p, [SP]),

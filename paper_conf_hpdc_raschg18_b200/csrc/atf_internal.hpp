@@ -338,6 +338,8 @@ int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long 
                     unsigned int* counter, void* stream, uint32_t* piece_tile = nullptr,
                     uint64_t piece_cap = 0);
 int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
+int launch_dist_flag_set(unsigned long long* f, unsigned long long v, void* stream);
+int launch_dist_flag_wait(const unsigned long long* f, unsigned long long v, unsigned long long* err, void* stream);
 int launch_divisible16_check(unsigned long long* mismatches, void* stream);
 int launch_encode(const EncodeArgs& a, const int32_t* vals, int64_t ld, int64_t n, uint64_t* digits, uint64_t* idx,
                   void* stream);

@@ -121,6 +121,19 @@ struct LevelData {
 
 }  // namespace
 
+// ---- balanced multi-GPU generation records (generate_dist)
+struct DistDesc {       // where a rank's slice of a level (or its round-flag array) lives
+  int64_t pid;          // owning process
+  uint64_t base, off;   // allocation base (device pointer in the owner) and byte offset
+  char handle[64];      // cudaIpcMemHandle_t of the allocation
+};
+struct DistGroup {      // per group, per round
+  uint32_t nd, repl;    // levels completed this round (0, 1 or a tail's nl); replicated level
+  uint64_t cnt[kMaxTail];
+  DistDesc desc;        // records of the last completed level
+};
+constexpr int kDistMaxRounds = 256;
+
 struct atf_space {
   atf_space_opts opts{};
   int state = BUILDING;
@@ -189,6 +202,25 @@ struct atf_space {
   struct PeerMap { int rank; char handle[64]; char* base; };
   std::vector<PeerMap> peers;  // opened IPC allocations of other ranks (generate_dist)
   int shard_rank = 0, shard_world = 1;
+  // replayed balanced generation (DESIGN.md §6 "Steady state"): the last synchronous
+  // generation's per-round all-gathers; once a generation with known sizes reproduced every
+  // count, later ones queue all rounds without host synchronisation (device flags order the
+  // cross-rank copies) and check everything once at the end
+  struct DistLog {
+    int world = 0, rank = -1;
+    size_t G = 0;
+    uint32_t flags = 0;
+    std::vector<std::vector<DistGroup>> all;  // [round][world * G]
+    std::vector<char> exchanged;               // [round]: an all-gather took place
+    std::vector<DistDesc> flag_desc;           // [world]
+    bool pure_ok = false;
+  } dlog;
+  unsigned long long* d_dflags = nullptr;  // [kDistMaxRounds] round flags | [1] wait timeout
+  char dflags_ipc[64] = {};
+  bool dflags_has_ipc = false;
+  unsigned long long dist_epoch = 0;
+  std::vector<cudaEvent_t> dist_ev;        // per round: [start, end] (ATF_FLAG_TIMING)
+  std::vector<float> dist_round_ms;        // device time of this rank's rounds, last generation
   std::vector<int> shard_cut;  // per group: first level expanded on a slice (L = none)
 };
 
@@ -1075,6 +1107,12 @@ static size_t arena_tail(atf_space* s, int g, int* which) {
 }
 
 static void release_device(atf_space* s) {
+  dfree(s, (char*)s->d_dflags, 8 * (kDistMaxRounds + 2));
+  s->d_dflags = nullptr;
+  s->dflags_has_ipc = false;
+  s->dlog = atf_space::DistLog{};
+  for (auto ev : s->dist_ev) cudaEventDestroy(ev);
+  s->dist_ev.clear();
   for (size_t g = 0; g < s->arena.size(); g++)
     for (auto& c : s->arena[g]) dfree(s, c.p, c.size);
   s->arena.clear();
@@ -1881,19 +1919,6 @@ static atf_status run_levels_replay(atf_space* s) {
 // global child indices, and copy their next parent slice from the owning ranks: CUDA IPC
 // pointers (one process per GPU: peer memory over NVLink / NVSwitch) or plain pointers (ranks
 // in one process).
-namespace {
-struct DistDesc {       // where a rank's slice of a level lives
-  int64_t pid;          // owning process
-  uint64_t base, off;   // allocation base (device pointer in the owner) and byte offset
-  char handle[64];      // cudaIpcMemHandle_t of the allocation
-};
-struct DistGroup {      // per group, per round
-  uint32_t nd, repl;    // levels completed this round (0, 1 or a tail's nl); replicated level
-  uint64_t cnt[kMaxTail];
-  DistDesc desc;        // records of the last completed level
-};
-}  // namespace
-
 static atf_status dist_desc(atf_space* s, int g, const uint32_t* rec, DistDesc& d) {
   std::memset(&d, 0, sizeof d);
   d.pid = (int64_t)getpid();
@@ -1937,15 +1962,75 @@ static atf_status dist_peer_ptr(atf_space* s, int q, const DistDesc& d, const ch
   return ATF_OK;
 }
 
-static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allgather_fn ag, void* ctx) {
-  NvtxRange nvtx("atf_space_generate_dist");
+// This rank's round-flag array (allocated and exported once per space).
+static atf_status dist_flags_desc(atf_space* s, DistDesc& d) {
+  std::memset(&d, 0, sizeof d);
+  d.pid = (int64_t)getpid();
+  if (!s->d_dflags) {
+    s->d_dflags = (unsigned long long*)dalloc(s, 8 * (kDistMaxRounds + 2));
+    if (!s->d_dflags) return fail(s, ATF_ERR_OOM, "round flags");
+    CUDA_TRY(s, cudaMemset(s->d_dflags, 0, 8 * (kDistMaxRounds + 2)));
+    s->dist_epoch = 0;
+    s->dflags_has_ipc = false;
+  }
+  if (!s->dflags_has_ipc) {
+    cudaIpcMemHandle_t h;
+    CUDA_TRY(s, cudaIpcGetMemHandle(&h, s->d_dflags));
+    std::memcpy(s->dflags_ipc, &h, sizeof h);
+    s->dflags_has_ipc = true;
+  }
+  d.base = (uint64_t)(uintptr_t)s->d_dflags;
+  std::memcpy(d.handle, s->dflags_ipc, 64);
+  return ATF_OK;
+}
+
+// One balanced generation.  mode 0: synchronous rounds (sizes found on the device, one
+// all-gather per round), recorded in s->dlog.  mode 1: the same with every level sized from the
+// log (the allocation sequence -- hence every address a peer reads -- is the one mode 2 will
+// reproduce); if every count matches, mode 2 is allowed next.  mode 2: no host synchronisation
+// and no all-gather per round: counts, offsets and peer addresses come from the log, a rank
+// publishes each round in its flag array and waits on the owners' flags before its peer copies;
+// at the end every rank checks its level totals, overflow flags, wait time-outs and its own
+// addresses against the log, and one all-gather of the verdicts decides for all ranks
+// (ATF_ERR_STATE: regenerate with mode 0).
+static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allgather_fn ag, void* ctx, int mode,
+                                     bool* verdict_done) {
+  *verdict_done = false;
+  NvtxRange nvtx(mode == 2 ? "atf_space_generate_dist (replay)" : "atf_space_generate_dist");
   cudaStream_t st = (cudaStream_t)s->opts.stream;
   const size_t G = s->groups.size();
+  auto& X = s->dlog;
   std::vector<int> k(G, 0);
   std::vector<uint64_t> F(G, 1);                 // global size of the frontier (level k - 1)
   std::vector<uint64_t> lo(G, 0), hi(G, 0);      // this rank's parent slice of the frontier
   std::vector<const uint32_t*> frontier(G, s->d_root);
   std::vector<DistGroup> mine(G), all((size_t)world * G);
+  const size_t pay = sizeof(DistGroup) * G + sizeof(DistDesc);
+  std::vector<char> sendb(pay), recvb(pay * world);
+  DistDesc my_flags;
+  atf_status e0 = dist_flags_desc(s, my_flags);
+  if (e0) return e0;
+  const bool timing = (s->opts.flags & ATF_FLAG_TIMING) != 0;
+  std::vector<std::vector<DistGroup>> rec_all;   // this generation's per-round records (modes 0, 1)
+  std::vector<char> rec_ex;
+  std::vector<DistDesc> rec_fd;
+  bool counts_match = mode == 1;
+  bool bad = false;                              // mode 2: own address differs from the log
+  struct Expect { int round, g; uint64_t total; };
+  std::vector<Expect> expect;
+  const unsigned long long epoch = mode == 2 ? ++s->dist_epoch : 0;
+  if (timing && s->dist_ev.size() < 2 * (size_t)kDistMaxRounds) {
+    for (auto ev : s->dist_ev) cudaEventDestroy(ev);
+    s->dist_ev.assign(2 * kDistMaxRounds, nullptr);
+    for (auto& ev : s->dist_ev) CUDA_TRY(s, cudaEventCreate(&ev));
+  }
+  s->dist_round_ms.clear();
+  if (mode == 2 && (size_t)kDistMaxRounds > s->replay_cap) {
+    dfree(s, (char*)s->d_replay, s->replay_cap * 12 * kMaxGroups);
+    s->replay_cap = kDistMaxRounds;
+    s->d_replay = (unsigned long long*)dalloc(s, s->replay_cap * 12 * kMaxGroups);
+    if (!s->d_replay) { s->replay_cap = 0; return fail(s, ATF_ERR_OOM, "replay log"); }
+  }
   // Small levels are replicated: every rank expands the whole frontier while it costs less than
   // kReplEvals candidate pairs (no exchange, no copy; the first distributed level takes its
   // parent slice straight from the local copy).  C5: levels 1-3 replicated, 4-8 distributed.
@@ -1955,10 +2040,15 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
     lo[g] = 0;
     hi[g] = 1;
   }
-  for (int round = 0;; round++) {
+  int round = 0;
+  for (;; round++) {
+    if (round >= kDistMaxRounds) return fail(s, ATF_ERR_STATE, "generate_dist: too many rounds");
+    if (mode == 2 && round >= (int)X.all.size()) return fail(s, ATF_ERR_STATE, "generate_dist replay: log too short");
+    const DistGroup* logged = mode >= 1 && round < (int)X.all.size() ? X.all[round].data() + (size_t)rank * G : nullptr;
     char rname[48];
     snprintf(rname, sizeof rname, "atf dist round %d", round);
     NvtxRange nvtx_round(rname);
+    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[2 * round], st));
     std::vector<Pending> pend;
     int active = 0;
     for (size_t g = 0; g < G; g++)
@@ -1968,7 +2058,7 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
     for (int attempt = 0;; attempt++) {
       pend.clear();
       CUDA_TRY(s, cudaMemsetAsync(s->d_totals, 0, 16 * kMaxGroups, st));
-      if (s->opts.flags & ATF_FLAG_TIMING) CUDA_TRY(s, cudaMemsetAsync(s->d_pairs, 0, 8 * kMaxGroups, st));
+      if (timing) CUDA_TRY(s, cudaMemsetAsync(s->d_pairs, 0, 8 * kMaxGroups, st));
       for (size_t g = 0; g < G; g++) {
         const int L = (int)s->groups[g].levels.size();
         if (k[g] >= L || mine[g].nd) continue;
@@ -1984,12 +2074,9 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
           d.evals = np * (uint64_t)s->groups[g].levels[k[g]].r;
           d.pairs = d.evals;
           if (k[g] > 0) {
-            char* csr = arena_alloc(s, (int)g, (np + 1) * 8);
-            if (!csr) {
-              atf_status e = arena_grow(s, (int)g, (np + 1) * 8);
-              if (e) return e;
-              csr = arena_alloc(s, (int)g, (np + 1) * 8);
-            }
+            atf_status e = ATF_OK;
+            char* csr = arena_take(s, (int)g, (np + 1) * 8, &e);
+            if (!csr) return e ? e : fail(s, ATF_ERR_OOM, "csr");
             CUDA_TRY(s, cudaMemsetAsync(csr, 0, (np + 1) * 8, st));
             LevelData& pdl = s->data[g][k[g] - 1];
             pdl.csr = (uint64_t*)csr;
@@ -2002,12 +2089,46 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
         }
         Pending pd;
         atf_status e;
-        if (s->tails[g].phase == 1) {
+        auto& T = s->tails[g];
+        if (T.phase == 1) {
           e = queue_tail_emit(s, (int)g, pd, active > 1);
         } else if (tail_here(s, (int)g, k[g], F[g])) {
           e = queue_tail_count(s, (int)g, k[g], frontier[g], np, pd, active > 1);
+          if (!e && mode == 2) {  // sizes from the log: the emit follows in the same queue
+            if (!logged || logged[g].nd != (uint32_t)T.nl) return fail(s, ATF_ERR_STATE, "replay: tail log");
+            for (int d = 0; d < T.nl; d++) T.tot[d] = logged[g].cnt[d];
+            T.phase = 1;
+            pend.push_back(pd);
+            e = queue_tail_emit(s, (int)g, pd, active > 1);
+          }
         } else {
-          e = queue_level(s, (int)g, k[g], frontier[g], np, pd, active > 1);
+          uint64_t want = UINT64_MAX;
+          if (logged) {
+            if (logged[g].nd != 1) {
+              if (mode == 2) return fail(s, ATF_ERR_STATE, "replay: level log");
+              counts_match = false;
+            } else {
+              want = logged[g].cnt[0];
+            }
+          }
+          e = queue_level(s, (int)g, k[g], frontier[g], np, pd, active > 1, mode >= 1 ? want : UINT64_MAX);
+          if (!e && mode == 2) {
+            GroupPlan& gp = s->groups[g];
+            LevelData& d = s->data[g][k[g]];
+            d.rec = pd.child;
+            d.n = want;
+            d.evals = np * (uint64_t)gp.levels[k[g]].r;
+            d.pairs = d.evals;
+            if (k[g] > 0) {
+              LevelData& pdl = s->data[g][k[g] - 1];
+              pdl.csr = pd.csr;
+              pdl.csr_offset = lo[g];
+              pdl.csr_n = np;
+            }
+            expect.push_back(Expect{round, (int)g, want});
+            mine[g].nd = 1;
+            mine[g].cnt[0] = want;
+          }
         }
         if (e) return e;
         pend.push_back(pd);
@@ -2015,6 +2136,21 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
       if (pend.empty()) break;
       for (auto& pd : pend)
         if (pd.joined) CUDA_TRY(s, cudaStreamWaitEvent(st, s->gb[pd.g].join, 0));
+      if (mode == 2) {  // no synchronisation: the round's totals go to the device log
+        CUDA_TRY(s, cudaMemcpyAsync((char*)s->d_replay + (size_t)round * 12 * kMaxGroups, s->d_totals,
+                                    12 * kMaxGroups, cudaMemcpyDeviceToDevice, st));
+        for (auto& pd : pend)
+          if (pd.kind == 2) {
+            const int g = pd.g;
+            finish_tail(s, g);
+            auto& T = s->tails[g];
+            s->data[g][T.k0 > 0 ? T.k0 - 1 : 0].csr_offset = lo[g];
+            if (T.k0 > 0) s->data[g][T.k0 - 1].csr_n = hi[g] - lo[g];
+            mine[g].nd = (uint32_t)T.nl;
+            for (int d = 0; d < T.nl; d++) mine[g].cnt[d] = T.tot[d];
+          }
+        break;
+      }
       CUDA_TRY(s, cudaMemcpyAsync(s->h_ctl.data(), s->d_totals, 12 * kMaxGroups, cudaMemcpyDeviceToHost, st));
       for (auto& pd : pend)
         if (pd.kind == 1) {
@@ -2025,8 +2161,7 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
         }
       CUDA_TRY(s, cudaStreamSynchronize(st));
       unsigned long long h_pairs[kMaxGroups] = {};
-      if (s->opts.flags & ATF_FLAG_TIMING)
-        CUDA_TRY(s, cudaMemcpy(h_pairs, s->d_pairs, sizeof(h_pairs), cudaMemcpyDeviceToHost));
+      if (timing) CUDA_TRY(s, cudaMemcpy(h_pairs, s->d_pairs, sizeof(h_pairs), cudaMemcpyDeviceToHost));
       bool redo = false;
       for (auto& pd : pend) {
         const int g = pd.g;
@@ -2047,6 +2182,7 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
         const uint64_t total = s->h_totals[g];
         GroupPlan& gp = s->groups[g];
         if (s->h_flags[g] || total > pd.cap) {  // overflow: grow and redo within this round
+          counts_match = false;
           s->stash_hint = std::max<uint64_t>(s->stash_hint, total);
           atf_status e = arena_grow(s, g, total * gp.words * 4 + (pd.n_parents + 1) * 8);
           if (e) return e;
@@ -2065,7 +2201,7 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
           pdl.csr_offset = lo[g];
           pdl.csr_n = pd.n_parents;
         }
-        if (s->opts.flags & ATF_FLAG_TIMING) {
+        if (timing) {
           cudaEventElapsedTime(&d.ms, s->events[g][pd.k].first, s->events[g][pd.k].second);
           cudaEventElapsedTime(&d.expand_ms, s->events[g][pd.k].first, s->events[g][pd.k].mid);
           d.pairs = d.seg_skip ? h_pairs[g] : d.evals;
@@ -2086,13 +2222,50 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
       atf_status e = dist_desc(s, (int)g, s->data[g][k[g]].rec, mine[g].desc);
       if (e) return e;
     }
-    if (need_ag) {
-      if (ag(mine.data(), all.data(), sizeof(DistGroup) * G, ctx) != 0)
+    if (mode == 2) {
+      if ((bool)X.exchanged[round] != need_ag) return fail(s, ATF_ERR_STATE, "replay: round structure");
+      all = X.all[round];
+      for (size_t g = 0; g < G; g++) {  // peers read what the log says this rank wrote
+        const DistGroup& lg = all[(size_t)rank * G + g];
+        if (lg.nd != mine[g].nd || (mine[g].nd == 1 && !repl[g] &&
+                                    (lg.desc.base != mine[g].desc.base || lg.desc.off != mine[g].desc.off)))
+          bad = true;
+      }
+    } else if (need_ag) {
+      std::memcpy(sendb.data(), mine.data(), sizeof(DistGroup) * G);
+      std::memcpy(sendb.data() + sizeof(DistGroup) * G, &my_flags, sizeof(DistDesc));
+      if (ag(sendb.data(), recvb.data(), pay, ctx) != 0)
         return fail(s, ATF_ERR_CUDA, "all-gather callback failed in round %d", round);
+      for (int r = 0; r < world; r++) {
+        std::memcpy(all.data() + (size_t)r * G, recvb.data() + pay * r, sizeof(DistGroup) * G);
+        if (rec_fd.empty() || (int)rec_fd.size() < world) {
+          DistDesc fd;
+          std::memcpy(&fd, recvb.data() + pay * r + sizeof(DistGroup) * G, sizeof fd);
+          if ((int)rec_fd.size() == r) rec_fd.push_back(fd);
+        }
+      }
     } else {
       for (int r = 0; r < world; r++)
         for (size_t g = 0; g < G; g++) all[(size_t)r * G + g] = mine[g];
     }
+    if (mode != 2) {
+      if (mode == 1) {  // same counts as the log on every rank?
+        if (round >= (int)X.all.size() || (bool)X.exchanged[round] != need_ag) {
+          counts_match = false;
+        } else {
+          for (size_t i = 0; i < all.size() && counts_match; i++) {
+            const DistGroup &x = all[i], &y = X.all[round][i];
+            if (x.nd != y.nd || std::memcmp(x.cnt, y.cnt, sizeof x.cnt) != 0) counts_match = false;
+          }
+        }
+      }
+      rec_all.push_back(all);
+      rec_ex.push_back(need_ag ? 1 : 0);
+    }
+    // bookkeeping and CSR fix-ups of every group, then (replay) this rank's round flag, then the
+    // peer copies: a rank publishes its round before it waits on anyone's
+    struct Copy { int g; };
+    std::vector<int> copy_groups;
     for (size_t g = 0; g < G; g++) {
       const uint32_t nd = mine[g].nd;
       if (!nd) continue;
@@ -2145,12 +2318,19 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
       k[g] += (int)nd;
       const int L = (int)s->groups[g].levels.size();
       if (k[g] >= L) continue;
-      // the next parent slice, copied from the ranks holding it
       const uint64_t Fg = F[g];
       lo[g] = (uint64_t)((unsigned __int128)Fg * rank / world);
       hi[g] = (uint64_t)((unsigned __int128)Fg * (rank + 1) / world);
+      if (hi[g] > lo[g]) copy_groups.push_back((int)g);
+    }
+    if (mode == 2 && need_ag && world > 1) {
+      int ce = launch_dist_flag_set(s->d_dflags + round, epoch, st);
+      if (ce) return fail(s, ATF_ERR_CUDA, "round flag");
+    }
+    std::vector<char> waited(world, 0);
+    for (int g : copy_groups) {
+      // the next parent slice, copied from the ranks holding it
       const uint64_t np = hi[g] - lo[g];
-      if (np == 0) continue;
       const int W = s->groups[g].words;
       auto& gbf = s->gb[g];
       atf_status e = ensure_buf(s, &gbf.pbuf, &gbf.pbuf_cap, np * W * 4, "parent slice");
@@ -2162,6 +2342,14 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
         if (a1 > a0) {
           const char* src = nullptr;
           if ((e = dist_peer_ptr(s, q, dg.desc, &src))) return e;
+          if (mode == 2 && q != rank && !waited[q]) {  // the owner's round is complete
+            const char* fp = nullptr;
+            if ((e = dist_peer_ptr(s, q, X.flag_desc[q], &fp))) return e;
+            int ce = launch_dist_flag_wait((const unsigned long long*)fp + round, epoch,
+                                           s->d_dflags + kDistMaxRounds, st);
+            if (ce) return fail(s, ATF_ERR_CUDA, "round flag wait");
+            waited[q] = 1;
+          }
           CUDA_TRY(s, cudaMemcpyAsync(gbf.pbuf + (a0 - lo[g]) * W * 4, src + (a0 - pos) * W * 4, (a1 - a0) * W * 4,
                                       cudaMemcpyDeviceToDevice, st));
         }
@@ -2169,17 +2357,95 @@ static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allg
       }
       frontier[g] = (const uint32_t*)gbf.pbuf;
     }
+    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[2 * round + 1], st));
   }
   s->gsize.assign(G, 0);
   for (size_t g = 0; g < G; g++) s->gsize[g] = s->groups[g].levels.empty() ? 0 : (k[g] >= (int)s->groups[g].levels.size() ? F[g] : 0);
   s->shard_rank = rank;
   s->shard_world = world;
+  if (mode == 2) {
+    // one synchronisation, then the checks, then one all-gather of the verdicts
+    std::vector<unsigned long long> log((size_t)round * 12 * kMaxGroups / 8 + 1, 0);
+    unsigned long long werr = 0;
+    if (round) CUDA_TRY(s, cudaMemcpyAsync(log.data(), s->d_replay, (size_t)round * 12 * kMaxGroups, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(s, cudaMemcpyAsync(&werr, s->d_dflags + kDistMaxRounds, 8, cudaMemcpyDeviceToHost, st));
+    CUDA_TRY(s, cudaStreamSynchronize(st));
+    bool ok = !bad && werr == 0 && round == (int)X.all.size();
+    for (const Expect& x : expect) {
+      const unsigned long long* rl = log.data() + (size_t)x.round * 12 * kMaxGroups / 8;
+      const unsigned int* ovf = reinterpret_cast<const unsigned int*>(rl + kMaxGroups);
+      if (rl[x.g] != x.total || ovf[x.g]) ok = false;
+    }
+    if (werr) CUDA_TRY(s, cudaMemset(s->d_dflags + kDistMaxRounds, 0, 8));
+    int32_t mine_ok = ok ? 1 : 0;
+    std::vector<int32_t> oks(world, 0);
+    *verdict_done = true;
+    if (ag(&mine_ok, oks.data(), sizeof(int32_t), ctx) != 0) return fail(s, ATF_ERR_CUDA, "all-gather callback failed (replay check)");
+    for (int r = 0; r < world; r++)
+      if (!oks[r]) return fail(s, ATF_ERR_STATE, "generate_dist replay: rank %d's checks failed", r);
+  } else {
+    if ((int)rec_fd.size() < world) {  // no exchange took place (world 1 or all levels replicated)
+      rec_fd.assign(world, my_flags);
+    }
+    X.world = world;
+    X.rank = rank;
+    X.G = G;
+    X.flags = s->opts.flags;
+    X.all = std::move(rec_all);
+    X.exchanged = std::move(rec_ex);
+    X.flag_desc = std::move(rec_fd);
+    X.pure_ok = mode == 1 && counts_match;
+  }
+  if (timing) {
+    for (int r = 0; r < round; r++) {
+      float ms = 0.f;
+      cudaEventElapsedTime(&ms, s->dist_ev[2 * r], s->dist_ev[2 * r + 1]);
+      s->dist_round_ms.push_back(ms);
+    }
+  }
   s->state = FINAL_SHARD;
   return ATF_OK;
 }
 
+static void dist_reset(atf_space* s) {
+  const size_t G = s->groups.size();
+  s->data.assign(G, {});
+  s->tails.assign(G, {});
+  for (size_t g = 0; g < G; g++) {
+    s->data[g].assign(s->groups[g].levels.size(), LevelData{});
+    for (auto& c : s->arena[g]) c.used = 0;
+  }
+}
+
+// Mode choice (generate_dist_pass): replay once a synchronous generation with the same ranks,
+// flags and log-sized levels reproduced every count; a failed replay (all ranks learn it from
+// the verdict all-gather) is regenerated synchronously at once.
+static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allgather_fn ag, void* ctx) {
+  auto& X = s->dlog;
+  const bool same = X.world == world && X.rank == rank && X.G == s->groups.size() && X.flags == s->opts.flags &&
+                    !X.all.empty();
+  const bool replay_allowed = !(s->opts.flags & (ATF_FLAG_NO_REPLAY | ATF_FLAG_TIMING));
+  const int mode = (same && replay_allowed) ? (X.pure_ok ? 2 : 1) : 0;
+  bool verdict = false;
+  atf_status e = generate_dist_pass(s, rank, world, ag, ctx, mode, &verdict);
+  if (mode != 2 || e == ATF_OK) return e;
+  if (!verdict) {  // failed before the checks: drain, then tell the other ranks
+    cudaStreamSynchronize((cudaStream_t)s->opts.stream);
+    cudaGetLastError();
+    int32_t zero = 0;
+    std::vector<int32_t> oks(world, 0);
+    if (ag(&zero, oks.data(), sizeof(int32_t), ctx) != 0) return fail(s, ATF_ERR_CUDA, "all-gather callback failed (replay check)");
+  }
+  X.pure_ok = false;
+  X.all.clear();
+  dist_reset(s);
+  return generate_dist_pass(s, rank, world, ag, ctx, 0, &verdict);
+}
+
 static atf_status generate_impl(atf_space* s) {
   NvtxRange nvtx("atf_space_generate");
+  s->dlog.all.clear();  // a balanced generation's log describes arena contents this one replaces
+  s->dlog.pure_ok = false;
   s->decode_jit = nullptr;  // the decoder's immediates (group sizes) belong to one generation
   s->decode_jit_tried = false;
   atf_status e = plan(s);
@@ -3080,12 +3346,7 @@ atf_status atf_space_generate_dist(atf_space* s, int32_t rank, int32_t world, at
   atf_status e = ensure_device(s);
   if (e) return e;
   const size_t G = s->groups.size();
-  s->data.assign(G, {});
-  s->tails.assign(G, {});
-  for (size_t g = 0; g < G; g++) {
-    s->data[g].assign(s->groups[g].levels.size(), LevelData{});
-    for (auto& c : s->arena[g]) c.used = 0;
-  }
+  dist_reset(s);
   if ((s->opts.flags & ATF_FLAG_TIMING) && s->events.size() != G) {
     s->events.assign(G, {});
     for (size_t g = 0; g < G; g++) {
@@ -3098,6 +3359,15 @@ atf_status atf_space_generate_dist(atf_space* s, int32_t rank, int32_t world, at
     }
   }
   return generate_dist_impl(s, rank, world, allgather, ctx);
+}
+
+atf_status atf_space_dist_round_ms(const atf_space* s, float* out, int32_t cap, int32_t* n_out) {
+  if (!s || !n_out || cap < 0) return ATF_ERR_INVALID_ARG;
+  if (s->dist_round_ms.empty()) return ATF_ERR_STATE;
+  *n_out = (int32_t)s->dist_round_ms.size();
+  if (out)
+    for (int32_t i = 0; i < cap && i < *n_out; i++) out[i] = s->dist_round_ms[i];
+  return ATF_OK;
 }
 
 atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, size_t* len_out, int32_t* k0_out) {

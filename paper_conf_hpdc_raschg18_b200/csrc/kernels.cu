@@ -596,4 +596,37 @@ int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream) {
   return (int)cudaGetLastError();
 }
 
+// ---- cross-rank round flags of the replayed balanced multi-GPU generation:
+// the owner publishes "round r of generation `epoch` is complete" after the round's kernels
+// (stream order) with a system-scope release; a consumer's stream spins on the owner's flag
+// (peer memory) with an acquire before copying the owner's records.  A wait that does not see
+// the flag within ~2 s gives up and raises `err` (the generation then fails its checks and is
+// regenerated with the synchronous protocol) instead of hanging the device.
+__global__ void dist_flag_set_kernel(unsigned long long* f, unsigned long long v) {
+  __threadfence_system();
+  asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(f), "l"(v) : "memory");
+}
+__global__ void dist_flag_wait_kernel(const unsigned long long* f, unsigned long long v, unsigned long long* err) {
+  unsigned long long t0, t, x;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  for (;;) {
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(x) : "l"(f) : "memory");
+    if (x >= v) return;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > 2000000000ull) {
+      atomicExch(err, 1ull);
+      return;
+    }
+    __nanosleep(200);
+  }
+}
+int launch_dist_flag_set(unsigned long long* f, unsigned long long v, void* stream) {
+  dist_flag_set_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(f, v);
+  return (int)cudaGetLastError();
+}
+int launch_dist_flag_wait(const unsigned long long* f, unsigned long long v, unsigned long long* err, void* stream) {
+  dist_flag_wait_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(f, v, err);
+  return (int)cudaGetLastError();
+}
+
 }  // namespace atf

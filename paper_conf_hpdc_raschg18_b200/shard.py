@@ -70,6 +70,7 @@ class VirtualAllGather:
         self.serialize = serialize
         self.lock = threading.Lock()
         self.round_s = [[] for _ in range(world)]
+        self.calls = [0] * world
         self._t0 = [0.0] * world
 
     def start(self, rank: int):
@@ -78,6 +79,7 @@ class VirtualAllGather:
             self._t0[rank] = time.perf_counter()
 
     def __call__(self, rank: int, data: bytes) -> bytes:
+        self.calls[rank] += 1
         if self.serialize:
             self.round_s[rank].append(time.perf_counter() - self._t0[rank])
             self.lock.release()

@@ -152,6 +152,14 @@ class Space:
             raise err[0]
         L.check(st, self._h)
 
+    def dist_round_ms(self) -> List[float]:
+        """Device time of each round of the last generate_dist (ATF_FLAG_TIMING)."""
+        n = C.c_int32()
+        L.check(L.atf_space_dist_round_ms(self._h, None, 0, C.byref(n)), self._h)
+        buf = (C.c_float * max(1, n.value))()
+        L.check(L.atf_space_dist_round_ms(self._h, buf, n.value, C.byref(n)), self._h)
+        return list(buf[: n.value])
+
     def finalize_shard(self, all_counts: List[List[int]]) -> None:
         world = len(all_counts)
         n = len(all_counts[0])

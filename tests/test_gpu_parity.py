@@ -797,11 +797,14 @@ def test_allocator_failure_is_reported_and_space_destroys_cleanly(Space):
 
 
 # ---------------------------------------------------------------- balanced multi-GPU generation
-def _dist_check(Space, spec, world, flags=0):
+def _dist_check(Space, spec, world, flags=0, gens=1, streams=False):
     """generate_dist on `world` virtual ranks (spaces of this process): global sizes = the oracle's,
     every level's rank slices (records, by offset) concatenate to the single-GPU level, and the
     ranks' CSR slices (by csr_offset) concatenate to the single-GPU CSR; every rank expanded
-    ~1/world of every level's parents (the balance rule)."""
+    ~1/world of every level's parents (the balance rule).  `gens` generations of the same spaces
+    (the third and later replay: one all-gather each, device flags between the ranks' streams;
+    `streams`: one CUDA stream per rank, concurrent ranks).  Returns the all-gather calls per
+    generation."""
     from paper_conf_hpdc_raschg18_b200.shard import virtual_ranks
     ref = orc.info(spec, threads=8)
     with Space(spec, flags=flags) as one:
@@ -810,9 +813,21 @@ def _dist_check(Space, spec, world, flags=0):
         want = {(g, k): tuple(t.clone() if t is not None else None for t in one.level_tensors(g, k))
                 for g in range(G) for k in range(one.num_levels(g))}
         sizes = one.group_sizes()
-    spaces = [Space(spec, flags=flags) for _ in range(world)]
+    spaces = [Space(spec, flags=flags, stream=torch.cuda.Stream() if streams else None) for _ in range(world)]
+    calls = []
     try:
-        virtual_ranks(spaces)
+        for _ in range(gens):
+            vag = virtual_ranks(spaces)
+            calls.append(vag.calls[0])
+            _dist_compare(spaces, want, sizes, ref, world)
+    finally:
+        for sp in spaces:
+            sp.close()
+    return calls
+
+
+def _dist_compare(spaces, want, sizes, ref, world):
+    if True:
         assert sizes == [g["size"] for g in ref["groups"]]
         for sp in spaces:
             assert sp.group_sizes() == sizes
@@ -853,9 +868,6 @@ def _dist_check(Space, spec, world, flags=0):
                 for c in cparts:
                     if (c[0], c[1].shape[0] - 1) != (c[2], c[3]):
                         assert abs((c[1].shape[0] - 1) - n / world) <= 1, (g, k)
-    finally:
-        for sp in spaces:
-            sp.close()
 
 
 @pytest.mark.parametrize("world", [2, 3, 8])
@@ -876,6 +888,31 @@ def test_dist_virtual_ranks_headline_flags(Space):
     _dist_check(Space, A.c3_xgemm((20, 96, 8)), 4, flags=L.ATF_FLAG_NO_JIT)
 
 
+@pytest.mark.parametrize("world", [1, 2, 3])
+@pytest.mark.parametrize("name", ["C5-300x4", "C3-IS1", "C2-256", "C5-4096x3", "fig1"])
+def test_dist_replay_virtual_ranks(Space, world, name):
+    """Steady state of generate_dist: the first generation synchronises per round, the second
+    sizes every level from the log, the third and later replay with device flags (one all-gather
+    per generation, the verdicts) -- every generation identical to the single-GPU space."""
+    calls = _dist_check(Space, SMALL[name](), world, gens=4, streams=True)
+    assert calls[2] == calls[3] == 1, calls
+    assert calls[0] == calls[1] >= 1, calls
+
+
+@pytest.mark.parametrize("seed", range(0, 24, 5))
+def test_dist_replay_fuzz(Space, seed):
+    calls = _dist_check(Space, A.random_spec(seed), 3, gens=3, streams=True)
+    assert calls[2] == 1, calls
+
+
+def test_dist_replay_headline_flags(Space):
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    calls = _dist_check(Space, A.c5_chains(4096, 4), 4, flags=L.ATF_FLAG_NO_SEG_BOUNDS, gens=3, streams=True)
+    assert calls[2] == 1, calls
+    calls = _dist_check(Space, A.c5_chains(4096, 4), 2, flags=L.ATF_FLAG_NO_REPLAY, gens=3, streams=True)
+    assert calls[2] == calls[0] > 1, calls   # replay off: one all-gather per round every time
+
+
 def test_dist_two_processes_cuda_ipc(Space, tmp_path):
     """Two processes on the one GPU, gloo all-gather: the parent slices cross processes through
     CUDA IPC (cudaIpcGetMemHandle / OpenMemHandle), the path every rank of an 8-GPU node uses."""
@@ -893,9 +930,21 @@ from paper_conf_hpdc_raschg18_b200.shard import generate_balanced
 dist.init_process_group("gloo")
 r = dist.get_rank()
 torch.cuda.set_device(0)
-with Space(A.c5_chains(300, 4)) as sp:
-    generate_balanced(sp)
-    out = {{"sizes": sp.group_sizes()}}
+calls = []
+def ag(b):
+    calls.append(len(b))
+    t = torch.frombuffer(bytearray(b), dtype=torch.uint8)
+    o = torch.empty(2 * t.numel(), dtype=torch.uint8)
+    dist.all_gather_into_tensor(o, t)
+    return o.numpy().tobytes()
+with Space(A.c5_chains(300, 4), stream=torch.cuda.Stream()) as sp:
+    ncalls = []
+    for _ in range(4):   # synchronous, log-sized, then two replays (device flags across processes)
+        n0 = len(calls)
+        sp.generate_dist(r, 2, ag)
+        ncalls.append(len(calls) - n0)
+    torch.cuda.synchronize()
+    out = {{"sizes": sp.group_sizes(), "calls": ncalls}}
     for g in range(sp.num_groups()):
         for k in range(sp.num_levels(g)):
             v = sp.level_view(g, k)
@@ -913,6 +962,8 @@ dist.destroy_process_group()
     assert p.returncode == 0, p.stdout[-3000:] + p.stderr[-3000:]
     res = [np.load(tmp_path / f"rank{r}.npy", allow_pickle=True).item() for r in range(2)]
     spec = A.c5_chains(300, 4)
+    for r in range(2):
+        assert res[r]["calls"][2] == res[r]["calls"][3] == 1, res[r]["calls"]
     with Space(spec) as one:
         one.generate()
         assert res[0]["sizes"] == res[1]["sizes"] == one.group_sizes()
