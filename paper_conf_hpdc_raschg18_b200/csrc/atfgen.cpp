@@ -2019,9 +2019,9 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
   struct Expect { int round, g; uint64_t total; };
   std::vector<Expect> expect;
   const unsigned long long epoch = mode == 2 ? ++s->dist_epoch : 0;
-  if (timing && s->dist_ev.size() < 2 * (size_t)kDistMaxRounds) {
+  if (timing && s->dist_ev.size() < 4 * (size_t)kDistMaxRounds) {
     for (auto ev : s->dist_ev) cudaEventDestroy(ev);
-    s->dist_ev.assign(2 * kDistMaxRounds, nullptr);
+    s->dist_ev.assign(4 * kDistMaxRounds, nullptr);
     for (auto& ev : s->dist_ev) CUDA_TRY(s, cudaEventCreate(&ev));
   }
   s->dist_round_ms.clear();
@@ -2043,12 +2043,12 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
   int round = 0;
   for (;; round++) {
     if (round >= kDistMaxRounds) return fail(s, ATF_ERR_STATE, "generate_dist: too many rounds");
-    if (mode == 2 && round >= (int)X.all.size()) return fail(s, ATF_ERR_STATE, "generate_dist replay: log too short");
+    if (mode == 2 && round >= (int)X.all.size()) break;  // every logged round replayed (checked below)
     const DistGroup* logged = mode >= 1 && round < (int)X.all.size() ? X.all[round].data() + (size_t)rank * G : nullptr;
     char rname[48];
     snprintf(rname, sizeof rname, "atf dist round %d", round);
     NvtxRange nvtx_round(rname);
-    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[2 * round], st));
+    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round], st));
     std::vector<Pending> pend;
     int active = 0;
     for (size_t g = 0; g < G; g++)
@@ -2212,6 +2212,7 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
       if (!redo) break;
     }
     if (!any_open) break;
+    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round + 1], st));  // (synchronised above)
     // exchange: one record per group and rank (skipped when every completed level is replicated:
     // all ranks take that decision from the same global sizes)
     bool need_ag = false;
@@ -2264,6 +2265,7 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
     }
     // bookkeeping and CSR fix-ups of every group, then (replay) this rank's round flag, then the
     // peer copies: a rank publishes its round before it waits on anyone's
+    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round + 2], st));
     struct Copy { int g; };
     std::vector<int> copy_groups;
     for (size_t g = 0; g < G; g++) {
@@ -2357,7 +2359,7 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
       }
       frontier[g] = (const uint32_t*)gbf.pbuf;
     }
-    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[2 * round + 1], st));
+    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round + 3], st));
   }
   s->gsize.assign(G, 0);
   for (size_t g = 0; g < G; g++) s->gsize[g] = s->groups[g].levels.empty() ? 0 : (k[g] >= (int)s->groups[g].levels.size() ? F[g] : 0);
@@ -2397,10 +2399,12 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
     X.pure_ok = mode == 1 && counts_match;
   }
   if (timing) {
-    for (int r = 0; r < round; r++) {
-      float ms = 0.f;
-      cudaEventElapsedTime(&ms, s->dist_ev[2 * r], s->dist_ev[2 * r + 1]);
-      s->dist_round_ms.push_back(ms);
+    CUDA_TRY(s, cudaStreamSynchronize(st));
+    for (int r = 0; r < round; r++) {  // the round's kernels + its fix-ups and peer copies (not the
+      float a = 0.f, b = 0.f;         // host wait for the all-gather in between)
+      cudaEventElapsedTime(&a, s->dist_ev[4 * r], s->dist_ev[4 * r + 1]);
+      cudaEventElapsedTime(&b, s->dist_ev[4 * r + 2], s->dist_ev[4 * r + 3]);
+      s->dist_round_ms.push_back(a + b);
     }
   }
   s->state = FINAL_SHARD;
@@ -3367,6 +3371,12 @@ atf_status atf_space_dist_round_ms(const atf_space* s, float* out, int32_t cap, 
   *n_out = (int32_t)s->dist_round_ms.size();
   if (out)
     for (int32_t i = 0; i < cap && i < *n_out; i++) out[i] = s->dist_round_ms[i];
+  return ATF_OK;
+}
+
+atf_status atf_test_set_tail_stage(int32_t bytes) {
+  if (bytes != 0 && (bytes < 2048 || bytes > 49152 || bytes % 16)) return ATF_ERR_INVALID_ARG;
+  jit_set_tail_stage(bytes);
   return ATF_OK;
 }
 

@@ -1,3 +1,4 @@
+#include <atomic>
 // jit.cpp — level-specialised narrow kernels compiled at plan time with NVRTC for sm_100a.
 //
 // A narrow fast level (expand_nfast, r <= 32) evaluates the same few conjuncts for every
@@ -385,6 +386,8 @@ struct TailJitArgs { const u32* parent_rec; u64 n_parents, n_tiles; u32* tile_to
 //                   canonical order; children staged in per-warp shared-memory buffers (with the
 //                   frontier lane they descend from, whose node constants sit in shared memory),
 //                   written out as coalesced vectors, CSR entries of every chunk.
+std::atomic<int> g_tail_stage{8192};  // tail emit staging bytes per warp (atf_test_set_tail_stage)
+
 std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vector<int32_t>>& cx,
                             const std::vector<std::vector<uint32_t>>& cm, int k0,
                             const std::vector<std::vector<int>>& pv_level, int* warp_bytes) {
@@ -497,7 +500,7 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   // the lanes of a part write their subtrees into shared memory, the warp copies every level's
   // run out as coalesced words.  A single lane whose subtree alone exceeds the area writes
   // straight to global memory.
-  constexpr int kStage = 8192;  // staging bytes per warp
+  const int kStage = g_tail_stage.load();  // staging bytes per warp (8192; test hook)
   if (warp_bytes) *warp_bytes = kStage;
   const std::string NLs = std::to_string(nl), NCs = std::to_string(NC), RB = std::to_string(W * 4);
   // The leaf level is not written by the depth-first walk when staged: a level-(nl-2) node stores
@@ -1195,4 +1198,8 @@ int jit_decode_launch(void* kernel, const DecodeArgs& a, const uint64_t* idx, co
   return (int)cudaLaunchKernel((const void*)kernel, dim3((unsigned)blocks), dim3(256), args, 0, (cudaStream_t)stream);
 }
 
+}  // namespace atf
+
+namespace atf {
+void jit_set_tail_stage(int bytes) { g_tail_stage.store(bytes > 0 ? bytes : 8192); }
 }  // namespace atf
