@@ -339,6 +339,7 @@ int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long 
                     uint64_t piece_cap = 0);
 int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
 void jit_set_tail_stage(int bytes);  // test hook: tail emit staging bytes per warp (0: default)
+int launch_host_gate(const unsigned int* flag, unsigned int v, void* stream);
 int launch_dist_flag_set(unsigned long long* f, unsigned long long v, void* stream);
 int launch_dist_flag_wait(const unsigned long long* f, unsigned long long v, unsigned long long* err, void* stream);
 int launch_divisible16_check(unsigned long long* mismatches, void* stream);

@@ -12,6 +12,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <atomic>
 #include <cstdarg>
 #include <cstdio>
 #include <cstring>
@@ -221,6 +222,9 @@ struct atf_space {
   unsigned long long dist_epoch = 0;
   std::vector<cudaEvent_t> dist_ev;        // per round: [start, end] (ATF_FLAG_TIMING)
   std::vector<float> dist_round_ms;        // device time of this rank's rounds, last generation
+  unsigned int* h_gate = nullptr;          // mapped host word releasing the timing gates
+  unsigned int* d_gate = nullptr;
+  unsigned int gate_v = 0;
   std::vector<int> shard_cut;  // per group: first level expanded on a slice (L = none)
 };
 
@@ -1113,6 +1117,8 @@ static void release_device(atf_space* s) {
   s->dlog = atf_space::DistLog{};
   for (auto ev : s->dist_ev) cudaEventDestroy(ev);
   s->dist_ev.clear();
+  if (s->h_gate) cudaFreeHost(s->h_gate);
+  s->h_gate = s->d_gate = nullptr;
   for (size_t g = 0; g < s->arena.size(); g++)
     for (auto& c : s->arena[g]) dfree(s, c.p, c.size);
   s->arena.clear();
@@ -1984,6 +1990,25 @@ static atf_status dist_flags_desc(atf_space* s, DistDesc& d) {
   return ATF_OK;
 }
 
+// Timing gate (ATF_FLAG_TIMING): hold the stream, queue, release (see host_gate_kernel).
+static atf_status gate_hold(atf_space* s, cudaStream_t st) {
+  if (!s->h_gate) {
+    CUDA_TRY(s, cudaHostAlloc((void**)&s->h_gate, 64, cudaHostAllocMapped));
+    CUDA_TRY(s, cudaHostGetDevicePointer((void**)&s->d_gate, s->h_gate, 0));
+    *(volatile unsigned int*)s->h_gate = 0;
+    s->gate_v = 0;
+  }
+  int ce = launch_host_gate(s->d_gate, ++s->gate_v, st);
+  if (ce) return fail(s, ATF_ERR_CUDA, "timing gate");
+  return ATF_OK;
+}
+static void gate_release(atf_space* s) {
+  if (s->h_gate) {
+    std::atomic_thread_fence(std::memory_order_seq_cst);
+    *(volatile unsigned int*)s->h_gate = s->gate_v;
+  }
+}
+
 // One balanced generation.  mode 0: synchronous rounds (sizes found on the device, one
 // all-gather per round), recorded in s->dlog.  mode 1: the same with every level sized from the
 // log (the allocation sequence -- hence every address a peer reads -- is the one mode 2 will
@@ -2048,7 +2073,11 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
     char rname[48];
     snprintf(rname, sizeof rname, "atf dist round %d", round);
     NvtxRange nvtx_round(rname);
-    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round], st));
+    if (timing) {
+      atf_status e = gate_hold(s, st);
+      if (e) return e;
+      CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round], st));
+    }
     std::vector<Pending> pend;
     int active = 0;
     for (size_t g = 0; g < G; g++)
@@ -2159,6 +2188,7 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
             CUDA_TRY(s, cudaMemcpyAsync(&T.tot[d], T.t.tile_base + d * (T.t.n_tiles + 1) + T.t.n_tiles, 8,
                                         cudaMemcpyDeviceToHost, st));
         }
+      if (timing) gate_release(s);
       CUDA_TRY(s, cudaStreamSynchronize(st));
       unsigned long long h_pairs[kMaxGroups] = {};
       if (timing) CUDA_TRY(s, cudaMemcpy(h_pairs, s->d_pairs, sizeof(h_pairs), cudaMemcpyDeviceToHost));
@@ -2265,7 +2295,11 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
     }
     // bookkeeping and CSR fix-ups of every group, then (replay) this rank's round flag, then the
     // peer copies: a rank publishes its round before it waits on anyone's
-    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round + 2], st));
+    if (timing) {
+      atf_status e = gate_hold(s, st);
+      if (e) return e;
+      CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round + 2], st));
+    }
     struct Copy { int g; };
     std::vector<int> copy_groups;
     for (size_t g = 0; g < G; g++) {
@@ -2359,7 +2393,10 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
       }
       frontier[g] = (const uint32_t*)gbf.pbuf;
     }
-    if (timing) CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round + 3], st));
+    if (timing) {
+      CUDA_TRY(s, cudaEventRecord(s->dist_ev[4 * round + 3], st));
+      gate_release(s);
+    }
   }
   s->gsize.assign(G, 0);
   for (size_t g = 0; g < G; g++) s->gsize[g] = s->groups[g].levels.empty() ? 0 : (k[g] >= (int)s->groups[g].levels.size() ? F[g] : 0);

@@ -620,6 +620,23 @@ __global__ void dist_flag_wait_kernel(const unsigned long long* f, unsigned long
     __nanosleep(200);
   }
 }
+// Host-released gate (the balanced generation's round timing, ATF_FLAG_TIMING): the stream
+// holds until the host writes `v` to the mapped word, so a round's launches are all queued
+// before the device starts it and its CUDA events measure device work only (as in the replay,
+// where the host runs ahead).  100 ms time-out.
+__global__ void host_gate_kernel(const volatile unsigned int* flag, unsigned int v) {
+  unsigned long long t0, t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t0));
+  while (*flag < v) {
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    if (t - t0 > 100000000ull) return;  // 100 ms: a host call that synchronises while the gate is held
+    __nanosleep(100);
+  }
+}
+int launch_host_gate(const unsigned int* flag, unsigned int v, void* stream) {
+  host_gate_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(flag, v);
+  return (int)cudaGetLastError();
+}
 int launch_dist_flag_set(unsigned long long* f, unsigned long long v, void* stream) {
   dist_flag_set_kernel<<<1, 1, 0, (cudaStream_t)stream>>>(f, v);
   return (int)cudaGetLastError();

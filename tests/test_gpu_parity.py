@@ -896,7 +896,7 @@ def test_dist_replay_virtual_ranks(Space, world, name):
     per generation, the verdicts) -- every generation identical to the single-GPU space."""
     calls = _dist_check(Space, SMALL[name](), world, gens=4, streams=True)
     assert calls[2] == calls[3] == 1, calls
-    assert calls[0] == calls[1] >= 1, calls
+    assert calls[0] == calls[1], calls   # (0 when every level is replicated)
 
 
 @pytest.mark.parametrize("seed", range(0, 24, 5))
