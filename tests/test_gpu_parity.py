@@ -909,8 +909,10 @@ def test_dist_replay_headline_flags(Space):
     from paper_conf_hpdc_raschg18_b200 import _lib as L
     calls = _dist_check(Space, A.c5_chains(4096, 4), 4, flags=L.ATF_FLAG_NO_SEG_BOUNDS, gens=3, streams=True)
     assert calls[2] == 1, calls
-    calls = _dist_check(Space, A.c5_chains(4096, 4), 2, flags=L.ATF_FLAG_NO_REPLAY, gens=3, streams=True)
-    assert calls[2] == calls[0] > 1, calls   # replay off: one all-gather per round every time
+    calls = _dist_check(Space, A.c5_chains(4096, 5), 2, flags=L.ATF_FLAG_NO_SEG_BOUNDS, gens=3, streams=True)
+    assert calls[0] == calls[1] == 2 and calls[2] == 1, calls   # levels 4, 5 distributed
+    calls = _dist_check(Space, A.c5_chains(4096, 5), 2, flags=L.ATF_FLAG_NO_REPLAY, gens=3, streams=True)
+    assert calls == [2, 2, 2], calls   # replay off: one all-gather per distributed round every time
 
 
 def test_dist_two_processes_cuda_ipc(Space, tmp_path):
