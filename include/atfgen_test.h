@@ -41,6 +41,10 @@ atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, 
 /* Staging bytes per warp of the fused tail's emit kernel for spaces planned afterwards (tuning
  * experiments; 0 restores the default 8192, a multiple of 16 in [2048, 49152] otherwise). */
 atf_status atf_test_set_tail_stage(int32_t bytes);
+/* Geometry knobs for spaces planned / generated afterwards (tuning experiments; 0 = default):
+ * warp tiles per SM below which the warp-tile kernel halves its nodes per tile (256), and
+ * log2 of the candidate-pair count below which generate_dist replicates a level (28). */
+atf_status atf_test_set_geometry(int32_t tiles_per_sm, int32_t repl_log2);
 #ifdef __cplusplus
 }
 #endif

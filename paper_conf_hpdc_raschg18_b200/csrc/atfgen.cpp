@@ -862,6 +862,12 @@ static atf_status plan(atf_space* s) {
 // r <= 64 -> narrow kernel (thread per node); otherwise the wide
 // kernel with cpt candidates per thread, a hot filter when a conjunct allows one, and
 // ~2^18 (node, candidate) pairs per tile.
+// Tuning knobs with test hooks (atf_test_set_geometry): warp tiles per SM below which the
+// warp-tile kernel halves its nodes per tile, and the pair count below which generate_dist
+// replicates a level instead of distributing it.
+static std::atomic<int> g_tiles_per_sm{256};
+static std::atomic<int> g_repl_log2{28};
+
 static void choose_geometry(LevelArgs& a, int words, bool legacy_wide, bool seg_bounds = true) {
   const int r = a.r;
   a.hot = HOT_NONE;
@@ -909,7 +915,8 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide, bool seg_
       // node quad of the hot loop) until ~256 tiles per SM exist: more tiles shorten the tail
       // of heavy tiles (nodes with thousands of children); measured sweet spot on C5
       int tnodes = kWT;
-      while (tnodes > 4 && (a.n_parents + tnodes - 1) / tnodes < 148ull * 256) tnodes >>= 1;
+      const uint64_t want_tiles = 148ull * (uint64_t)g_tiles_per_sm.load();
+      while (tnodes > 4 && (a.n_parents + tnodes - 1) / tnodes < want_tiles) tnodes >>= 1;
       a.tile_nodes = tnodes;
       // 8 warps per CTA unless the level has too few tiles to give every SM a full CTA
       const uint64_t tiles = (a.n_parents + tnodes - 1) / tnodes;
@@ -2059,7 +2066,7 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
   // Small levels are replicated: every rank expands the whole frontier while it costs less than
   // kReplEvals candidate pairs (no exchange, no copy; the first distributed level takes its
   // parent slice straight from the local copy).  C5: levels 1-3 replicated, 4-8 distributed.
-  constexpr uint64_t kReplEvals = 1ull << 28;
+  const uint64_t kReplEvals = 1ull << g_repl_log2.load();
   std::vector<char> repl(G, 1);
   for (size_t g = 0; g < G; g++) {  // level 0: the root (one parent)
     lo[g] = 0;
@@ -3408,6 +3415,13 @@ atf_status atf_space_dist_round_ms(const atf_space* s, float* out, int32_t cap, 
   *n_out = (int32_t)s->dist_round_ms.size();
   if (out)
     for (int32_t i = 0; i < cap && i < *n_out; i++) out[i] = s->dist_round_ms[i];
+  return ATF_OK;
+}
+
+atf_status atf_test_set_geometry(int32_t tiles_per_sm, int32_t repl_log2) {
+  if (tiles_per_sm < 0 || tiles_per_sm > 4096 || repl_log2 < 0 || repl_log2 > 62) return ATF_ERR_INVALID_ARG;
+  g_tiles_per_sm.store(tiles_per_sm ? tiles_per_sm : 256);
+  g_repl_log2.store(repl_log2 ? repl_log2 : 28);
   return ATF_OK;
 }
 

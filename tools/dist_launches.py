@@ -1,6 +1,6 @@
-"""Kernel launches of one virtual rank's balanced generation (for an ncu launch list):
-N spaces, serialized virtual ranks; the last generation of rank `r` is bracketed by
-cudaProfilerStart/Stop.   ncu --profile-from-start off ... python tools/dist_launches.py N r"""
+"""Kernel launches of a balanced generation over N virtual ranks (for an ncu launch list):
+serialized virtual ranks (one rank's round at a time on the GPU); the third generation is
+bracketed by cudaProfilerStart/Stop.   ncu --profile-from-start off ... python tools/dist_launches.py N"""
 import os
 import sys
 
@@ -27,13 +27,8 @@ def gen(profile):
         try:
             torch.cuda.set_device(0)
             vag.start(r)
-            if profile and r == R:
-                torch.cuda.synchronize()
-                torch.cuda.cudart().cudaProfilerStart()
             spaces[r].generate_dist(r, N, lambda b: vag(r, b))
             torch.cuda.synchronize()
-            if profile and r == R:
-                torch.cuda.cudart().cudaProfilerStop()
             vag.finish(r)
         except Exception as ex:  # noqa: BLE001
             errs.append(ex)
@@ -49,5 +44,9 @@ def gen(profile):
 
 gen(False)
 gen(False)
+torch.cuda.synchronize()
+torch.cuda.cudart().cudaProfilerStart()
 gen(True)
+torch.cuda.synchronize()
+torch.cuda.cudart().cudaProfilerStop()
 print("ok")

@@ -16,7 +16,8 @@ import torch  # noqa: E402
 import atfspec as A  # noqa: E402
 from paper_conf_hpdc_raschg18_b200 import Space, _lib as L  # noqa: E402
 
-SPECS = [A.c2_xgemm_direct(256), A.c3_xgemm("IS1"), A.c5_chains(300, 4), A.c5_chains(4096, 2), A.saxpy(360)]
+SPECS = [A.c2_xgemm_direct(256), A.c3_xgemm("IS1"), A.c3_xgemm((20, 96, 8)), A.c5_chains(300, 4), A.c5_chains(4096, 2),
+         A.saxpy(360)]
 FLAGS = [0, L.ATF_FLAG_NO_SEG_BOUNDS, L.ATF_FLAG_NO_TAIL | L.ATF_FLAG_NO_JIT]
 
 for spec in SPECS:
@@ -31,5 +32,16 @@ for spec in SPECS:
             back = sp.encode_digits(rows)
             assert torch.equal(back, dig), spec.name
             print(spec.name, fl, sp.size(), flush=True)
+torch.cuda.synchronize()
+# balanced multi-GPU generation: two virtual ranks on their own streams, three generations
+# (synchronous, log-sized, replay with device round flags)
+from paper_conf_hpdc_raschg18_b200.shard import virtual_ranks  # noqa: E402
+for spec in (A.c5_chains(4096, 4), A.c3_xgemm((20, 96, 8))):
+    spaces = [Space(spec, flags=L.ATF_FLAG_NO_SEG_BOUNDS, stream=torch.cuda.Stream()) for _ in range(2)]
+    for _ in range(3):
+        virtual_ranks(spaces)
+        print("dist", spec.name, [sp.group_sizes() for sp in spaces], flush=True)
+    for sp in spaces:
+        sp.close()
 torch.cuda.synchronize()
 print("sanitize run ok")
