@@ -214,8 +214,10 @@ struct atf_space {
     std::vector<std::vector<DistGroup>> all;  // [round][world * G]
     std::vector<char> exchanged;               // [round]: an all-gather took place
     std::vector<DistDesc> flag_desc;           // [world]
+    std::vector<uint64_t> cap_lo, cap_n;       // the group-to-rank assignment it was made with
     bool pure_ok = false;
   } dlog;
+  std::vector<double> group_work;  // candidate pairs per group of the last generation (all ranks)
   unsigned long long* d_dflags = nullptr;  // [kDistMaxRounds] round flags | [1] wait timeout
   char dflags_ipc[64] = {};
   bool dflags_has_ipc = false;
@@ -2016,6 +2018,42 @@ static void gate_release(atf_space* s) {
   }
 }
 
+// Group-to-rank assignment of the balanced generation.  Ranks are laid on a line
+// of world * kCapU capacity units; group g owns the units [cap_lo, cap_lo + cap_n) and rank q
+// expands the share of every level of g that its units [q kCapU, (q+1) kCapU) overlap.  With
+// the previous generation's candidate pairs per group (identical on every rank), cap_n is
+// proportional to them: every rank gets 1/world of the total work, and a rank works on one or
+// two groups with slices of 1/(world * share) instead of every group at 1/world (fewer, larger
+// kernels per round).  Without that information (first generation, one group, one rank)
+// every group spans all ranks: cap_lo = 0, cap_n = world * kCapU (slices [rF/N, (r+1)F/N)).
+constexpr uint64_t kCapU = 1ull << 20;
+static void dist_assignment(const atf_space* s, int world, std::vector<uint64_t>& c, std::vector<uint64_t>& u) {
+  const size_t G = s->groups.size();
+  const uint64_t units = (uint64_t)world * kCapU;
+  c.assign(G, 0);
+  u.assign(G, units);
+  double W = 0;
+  for (double w : s->group_work) W += w;
+  if (world == 1 || G < 2 || s->group_work.size() != G || !(W > 0)) return;
+  uint64_t used = 0;
+  size_t big = 0;
+  for (size_t g = 0; g < G; g++) {
+    u[g] = std::max<uint64_t>(1, (uint64_t)(s->group_work[g] / W * (double)units));
+    used += u[g];
+    if (s->group_work[g] > s->group_work[big]) big = g;
+  }
+  if (used > units) {  // (only through the 1-unit minimum) shave the largest group
+    u[big] -= std::min(u[big] - 1, used - units);
+  } else {
+    u[big] += units - used;
+  }
+  uint64_t at = 0;
+  for (size_t g = 0; g < G; g++) {
+    c[g] = at;
+    at += u[g];
+  }
+}
+
 // One balanced generation.  mode 0: synchronous rounds (sizes found on the device, one
 // all-gather per round), recorded in s->dlog.  mode 1: the same with every level sized from the
 // log (the allocation sequence -- hence every address a peer reads -- is the one mode 2 will
@@ -2068,9 +2106,30 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
   // parent slice straight from the local copy).  C5: levels 1-3 replicated, 4-8 distributed.
   const uint64_t kReplEvals = 1ull << g_repl_log2.load();
   std::vector<char> repl(G, 1);
-  for (size_t g = 0; g < G; g++) {  // level 0: the root (one parent)
+  std::vector<uint64_t> cap_lo, cap_n;
+  dist_assignment(s, world, cap_lo, cap_n);
+  if (mode >= 1 && (cap_lo != X.cap_lo || cap_n != X.cap_n)) return fail(s, ATF_ERR_STATE, "internal: assignment changed");
+  bool subsets = false;  // some group does not span every rank
+  for (size_t g = 0; g < G; g++) subsets |= cap_lo[g] != 0 || cap_n[g] != (uint64_t)world * kCapU;
+  // this rank's share [l, h) of a level of group g with Fg nodes (empty: not a member of g)
+  auto share = [&](size_t g, uint64_t Fg, uint64_t& l, uint64_t& h) {
+    const uint64_t c = cap_lo[g], u = cap_n[g], q0 = (uint64_t)rank * kCapU, q1 = q0 + kCapU;
+    const uint64_t a = std::max(c, q0), b = std::min(c + u, q1);
+    if (b <= a) {
+      l = h = 0;
+      return false;
+    }
+    l = (uint64_t)((unsigned __int128)Fg * (a - c) / u);
+    h = (uint64_t)((unsigned __int128)Fg * (b - c) / u);
+    return true;
+  };
+  std::vector<char> member(G, 0);
+  std::vector<double> work(G, 0.0);
+  for (size_t g = 0; g < G; g++) {  // level 0: the root (one parent), expanded by the group's ranks
+    uint64_t l, h;
+    member[g] = share(g, 1, l, h) ? 1 : 0;
     lo[g] = 0;
-    hi[g] = 1;
+    hi[g] = member[g] ? 1 : 0;
   }
   int round = 0;
   for (;; round++) {
@@ -2102,13 +2161,18 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
         const uint64_t np = hi[g] - lo[g];
         const bool empty_range = s->groups[g].levels[k[g]].r == 0;
         if (np == 0 || empty_range) {
-          // no local parents (or an empty range): this rank's part of the level is empty; the
-          // parents' CSR entries are all zero
-          LevelData& d = s->data[g][k[g]];
-          d.rec = nullptr;
-          d.n = 0;
-          d.evals = np * (uint64_t)s->groups[g].levels[k[g]].r;
-          d.pairs = d.evals;
+          // no local parents (or an empty range): this rank's part of the level is empty (and,
+          // at the start of the group's fused tail, of every tail level: the ranks that have
+          // parents complete the tail's levels in this round); the parents' CSR entries are 0
+          const int nd = (!empty_range && s->tails[g].phase == 0 && tail_here(s, (int)g, k[g], F[g])) ? L - k[g] : 1;
+          for (int d = 0; d < nd; d++) {
+            LevelData& ld = s->data[g][k[g] + d];
+            ld.rec = nullptr;
+            ld.n = 0;
+            ld.csr = nullptr;
+            ld.evals = d == 0 ? np * (uint64_t)s->groups[g].levels[k[g]].r : 0;
+            ld.pairs = ld.evals;
+          }
           if (k[g] > 0) {
             atf_status e = ATF_OK;
             char* csr = arena_take(s, (int)g, (np + 1) * 8, &e);
@@ -2119,8 +2183,8 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
             pdl.csr_offset = lo[g];
             pdl.csr_n = np;
           }
-          mine[g].nd = 1;
-          mine[g].cnt[0] = 0;
+          mine[g].nd = (uint32_t)nd;
+          for (int d = 0; d < nd; d++) mine[g].cnt[d] = 0;
           continue;
         }
         Pending pd;
@@ -2255,7 +2319,8 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
     bool need_ag = false;
     for (size_t g = 0; g < G; g++) {
       mine[g].repl = repl[g];
-      if (mine[g].nd && !repl[g]) need_ag = true;
+      // (with subsets, the non-members of a group learn its replicated levels' sizes here too)
+      if (mine[g].nd && (!repl[g] || subsets)) need_ag = true;
       if (mine[g].nd != 1 || repl[g]) continue;
       atf_status e = dist_desc(s, (int)g, s->data[g][k[g]].rec, mine[g].desc);
       if (e) return e;
@@ -2314,12 +2379,15 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
       if (!nd) continue;
       for (int r = 0; r < world; r++)
         if (all[(size_t)r * G + g].nd != nd) return fail(s, ATF_ERR_STATE, "ranks out of step (group %zu)", g);
-      if (repl[g]) {  // every rank holds the whole level(s)
+      if (repl[g]) {  // every rank of the group holds the whole level(s)
         for (uint32_t d = 0; d < nd; d++) {
           LevelData& ld = s->data[g][k[g] + d];
           ld.offset = 0;
           if (d + 1 < nd) { ld.csr_offset = 0; ld.csr_n = ld.n; }
-          F[g] = mine[g].cnt[d];
+          uint64_t fg = 0;  // the members' count (non-members hold none)
+          for (int r = 0; r < world; r++) fg = std::max<uint64_t>(fg, all[(size_t)r * G + g].cnt[d]);
+          work[g] += (double)F[g] * (double)s->groups[g].levels[k[g] + d].r;
+          F[g] = fg;
         }
         k[g] += (int)nd;
         if (k[g] >= (int)s->groups[g].levels.size()) continue;
@@ -2327,13 +2395,12 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
         const LevelData& ld = s->data[g][k[g] - 1];
         if (Fg * (uint64_t)s->groups[g].levels[k[g]].r >= kReplEvals) {
           repl[g] = 0;  // distribute from here on: this rank's slice of the local copy
-          lo[g] = (uint64_t)((unsigned __int128)Fg * rank / world);
-          hi[g] = (uint64_t)((unsigned __int128)Fg * (rank + 1) / world);
+          share(g, Fg, lo[g], hi[g]);
         } else {
           lo[g] = 0;
-          hi[g] = Fg;
+          hi[g] = member[g] ? Fg : 0;
         }
-        frontier[g] = ld.rec ? ld.rec + lo[g] * s->groups[g].words : s->d_root;
+        frontier[g] = (ld.rec && hi[g] > lo[g]) ? ld.rec + lo[g] * s->groups[g].words : s->d_root;
         continue;
       }
       // global offsets of this rank's part of every completed level; CSR entries -> global
@@ -2356,14 +2423,13 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
           int ce = launch_add_offset(pl->csr, pl->csr_n + 1, before, st);
           if (ce) return fail(s, ATF_ERR_CUDA, "csr fix-up");
         }
+        work[g] += (double)F[g] * (double)s->groups[g].levels[k[g] + d].r;
         F[g] = tot;
       }
       k[g] += (int)nd;
       const int L = (int)s->groups[g].levels.size();
       if (k[g] >= L) continue;
-      const uint64_t Fg = F[g];
-      lo[g] = (uint64_t)((unsigned __int128)Fg * rank / world);
-      hi[g] = (uint64_t)((unsigned __int128)Fg * (rank + 1) / world);
+      share(g, F[g], lo[g], hi[g]);
       if (hi[g] > lo[g]) copy_groups.push_back((int)g);
     }
     if (mode == 2 && need_ag && world > 1) {
@@ -2409,6 +2475,7 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
   for (size_t g = 0; g < G; g++) s->gsize[g] = s->groups[g].levels.empty() ? 0 : (k[g] >= (int)s->groups[g].levels.size() ? F[g] : 0);
   s->shard_rank = rank;
   s->shard_world = world;
+  s->group_work = work;
   if (mode == 2) {
     // one synchronisation, then the checks, then one all-gather of the verdicts
     std::vector<unsigned long long> log((size_t)round * 12 * kMaxGroups / 8 + 1, 0);
@@ -2440,6 +2507,8 @@ static atf_status generate_dist_pass(atf_space* s, int rank, int world, atf_allg
     X.all = std::move(rec_all);
     X.exchanged = std::move(rec_ex);
     X.flag_desc = std::move(rec_fd);
+    X.cap_lo = cap_lo;
+    X.cap_n = cap_n;
     X.pure_ok = mode == 1 && counts_match;
   }
   if (timing) {
@@ -2470,8 +2539,10 @@ static void dist_reset(atf_space* s) {
 // the verdict all-gather) is regenerated synchronously at once.
 static atf_status generate_dist_impl(atf_space* s, int rank, int world, atf_allgather_fn ag, void* ctx) {
   auto& X = s->dlog;
+  std::vector<uint64_t> cl, cn;
+  dist_assignment(s, world, cl, cn);
   const bool same = X.world == world && X.rank == rank && X.G == s->groups.size() && X.flags == s->opts.flags &&
-                    !X.all.empty();
+                    !X.all.empty() && cl == X.cap_lo && cn == X.cap_n;
   const bool replay_allowed = !(s->opts.flags & (ATF_FLAG_NO_REPLAY | ATF_FLAG_TIMING));
   const int mode = (same && replay_allowed) ? (X.pure_ok ? 2 : 1) : 0;
   bool verdict = false;
@@ -2550,6 +2621,14 @@ static atf_status generate_impl(atf_space* s) {
   }
   s->gsize.assign(G, 0);
   for (size_t g = 0; g < G; g++) s->gsize[g] = s->groups[g].levels.empty() ? 0 : s->data[g].back().n;
+  s->group_work.assign(G, 0.0);  // candidate pairs per group (generate_dist's assignment)
+  for (size_t g = 0; g < G; g++) {
+    uint64_t f = 1;
+    for (size_t k = 0; k < s->data[g].size(); k++) {
+      s->group_work[g] += (double)f * (double)s->groups[g].levels[k].r;
+      f = s->data[g][k].n;
+    }
+  }
   s->state = GENERATED;
   return ATF_OK;
 }
