@@ -28,6 +28,7 @@ ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT, A
 ATF_FLAG_NO_SEG_BOUNDS = 64
 ATF_FLAG_NO_TAIL = 128
 ATF_FLAG_NO_REPLAY = 256
+ATF_FLAG_DIST_SUBSETS = 512
 
 
 class atf_range(C.Structure):
