@@ -12,6 +12,7 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <array>
 #include <atomic>
 #include <cstdarg>
 #include <cstdio>
@@ -101,6 +102,8 @@ struct Chunk {
   bool has_ipc = false;  // ipc handle exported (generate_dist)
   char ipc[64];
 };
+
+struct ReplayExpect { int round, g; uint64_t total; };  // a replayed level's expected total
 
 struct LevelData {
   uint32_t* rec = nullptr;
@@ -196,6 +199,22 @@ struct atf_space {
   bool replay_ok = false;
   unsigned long long* d_replay = nullptr;  // per round: [totals u64 | ovf u32] of every group
   size_t replay_cap = 0;                   // rounds
+  int replays = 0;                         // replays since the last level-by-level generation
+  // the replay's launches captured once as a CUDA graph (DESIGN.md §5 "Steady state"): later
+  // generations launch it whole; valid while no buffer it references moved (buf_epoch)
+  cudaGraphExec_t graph_exec = nullptr;
+  uint64_t graph_epoch = 0, buf_epoch = 0;
+  bool capturing = false;
+  cudaStream_t cap_stream = nullptr;
+  cudaEvent_t cap_ev = nullptr;
+  struct GraphSnap {  // host-side state of the captured generation
+    std::vector<std::vector<LevelData>> data;
+    std::vector<std::vector<size_t>> used;
+    std::vector<Tail> tails;
+    int rounds = 0;
+    std::vector<ReplayExpect> expect;
+    std::vector<int> tails_done;
+  } gsnap;
   void* decode_jit = nullptr;   // specialised decoder of the current generation (jit.cpp)
   bool decode_jit_tried = false;
   // shards
@@ -252,6 +271,8 @@ static atf_status fail(atf_space* s, atf_status st, const char* fmt, ...) {
 static void* dalloc(atf_space* s, size_t bytes) {
   if (bytes == 0) bytes = 16;
   void* p = nullptr;
+  if (s->capturing) return nullptr;  // graph capture: no allocation (the capture is abandoned)
+  s->buf_epoch++;
   if (s->ipc_alloc) {  // generate_dist: peers map the arena through CUDA IPC
     if (cudaMalloc(&p, bytes) != cudaSuccess) {
       cudaGetLastError();
@@ -269,6 +290,7 @@ static void* dalloc(atf_space* s, size_t bytes) {
 }
 static void dfree(atf_space* s, void* p, size_t bytes) {
   if (!p) return;
+  s->buf_epoch++;
   if (s->ipc_alloc) {
     cudaStreamSynchronize((cudaStream_t)s->opts.stream);
     cudaFree(p);
@@ -1078,6 +1100,7 @@ static atf_status ensure_device(atf_space* s) {
 
 static atf_status ensure_buf(atf_space* s, char** p, size_t* cap, size_t bytes, const char* what) {
   if (bytes <= *cap) return ATF_OK;
+  if (s->capturing) return fail(s, ATF_ERR_OOM, "%s: growth during graph capture", what);
   dfree(s, *p, *cap);
   size_t c = std::max<size_t>(bytes, *cap * 2);
   *p = (char*)dalloc(s, c);
@@ -1119,7 +1142,18 @@ static size_t arena_tail(atf_space* s, int g, int* which) {
   return best;
 }
 
+static void drop_graph(atf_space* s) {
+  if (s->graph_exec) cudaGraphExecDestroy(s->graph_exec);
+  s->graph_exec = nullptr;
+  s->replays = 0;
+}
+
 static void release_device(atf_space* s) {
+  drop_graph(s);
+  if (s->cap_stream) cudaStreamDestroy(s->cap_stream);
+  if (s->cap_ev) cudaEventDestroy(s->cap_ev);
+  s->cap_stream = nullptr;
+  s->cap_ev = nullptr;
   dfree(s, (char*)s->d_dflags, 8 * (kDistMaxRounds + 2));
   s->d_dflags = nullptr;
   s->dflags_has_ipc = false;
@@ -1141,6 +1175,7 @@ static void release_device(atf_space* s) {
   s->d_replay = nullptr;
   s->replay_cap = 0;
   s->replay_ok = false;
+  drop_graph(s);
   for (auto& b : s->gb) {
     dfree(s, b.scratch, b.scratch_cap);
     dfree(s, (char*)b.stash, b.stash_cap);
@@ -1819,25 +1854,15 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
 // every level's total and overflow flag is checked against the expected values.  The device
 // still evaluates every pair and writes every record.  Returns ATF_ERR_STATE on any mismatch
 // (the caller then regenerates level by level).
-static atf_status run_levels_replay(atf_space* s) {
-  NvtxRange nvtx("atf replay");
+// Queue every round of a replay (no synchronisation); host-side level data as the kernels will
+// leave it.  `rounds`, `expect`, `tails_done` describe the checks.
+static atf_status replay_queue(atf_space* s, int& rounds_out, std::vector<ReplayExpect>& expect,
+                               std::vector<std::pair<int, int>>& timed, std::vector<int>& tails_done) {
   cudaStream_t st = (cudaStream_t)s->opts.stream;
   const size_t G = s->groups.size();
-  int max_rounds = 0;
-  for (size_t g = 0; g < G; g++) max_rounds = std::max(max_rounds, (int)s->groups[g].levels.size() + 1);
-  if ((size_t)max_rounds > s->replay_cap) {
-    dfree(s, (char*)s->d_replay, s->replay_cap * 12 * kMaxGroups);
-    s->replay_cap = (size_t)max_rounds;
-    s->d_replay = (unsigned long long*)dalloc(s, s->replay_cap * 12 * kMaxGroups);
-    if (!s->d_replay) { s->replay_cap = 0; return fail(s, ATF_ERR_OOM, "replay log"); }
-  }
   std::vector<int> k(G, 0);
   std::vector<const uint32_t*> frontier(G, s->d_root);
   std::vector<uint64_t> fsize(G, 1);
-  struct Expect { int round, g; uint64_t total; };
-  std::vector<Expect> expect;
-  std::vector<std::pair<int, int>> timed;  // (g, k) single levels with timing events
-  std::vector<int> tails_done;
   int round = 0;
   for (;; round++) {
     int active = 0;
@@ -1890,7 +1915,7 @@ static atf_status run_levels_replay(atf_space* s) {
         d.evals = fsize[g] * (uint64_t)gp.levels[k[g]].r;
         if (!(s->opts.flags & ATF_FLAG_TIMING)) d.pairs = 0;
         if (k[g] > 0) s->data[g][k[g] - 1].csr = pd.csr;
-        expect.push_back(Expect{round, (int)g, want});
+        expect.push_back(ReplayExpect{round, (int)g, want});
         if (s->opts.flags & ATF_FLAG_TIMING) timed.emplace_back((int)g, k[g]);
         frontier[g] = pd.child;
         fsize[g] = want;
@@ -1905,11 +1930,19 @@ static atf_status run_levels_replay(atf_space* s) {
       CUDA_TRY(s, cudaMemcpyAsync((char*)s->d_replay + (size_t)round * 12 * kMaxGroups, s->d_totals, 12 * kMaxGroups,
                                   cudaMemcpyDeviceToDevice, st));
   }
+  rounds_out = round;
+  return ATF_OK;
+}
+
+// One synchronisation, then every level total and overflow flag against the expected ones.
+static atf_status replay_check(atf_space* s, int round, const std::vector<ReplayExpect>& expect,
+                               const std::vector<std::pair<int, int>>& timed, const std::vector<int>& tails_done) {
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
   // one synchronisation: the round log, then the checks
   std::vector<unsigned long long> log((size_t)round * 12 * kMaxGroups / 8 + 1, 0);
   if (round) CUDA_TRY(s, cudaMemcpyAsync(log.data(), s->d_replay, (size_t)round * 12 * kMaxGroups, cudaMemcpyDeviceToHost, st));
   CUDA_TRY(s, cudaStreamSynchronize(st));
-  for (const Expect& x : expect) {
+  for (const ReplayExpect& x : expect) {
     const unsigned long long* rl = log.data() + (size_t)x.round * 12 * kMaxGroups / 8;
     const unsigned int* ovf = reinterpret_cast<const unsigned int*>(rl + kMaxGroups);
     if (rl[x.g] != x.total || ovf[x.g]) return fail(s, ATF_ERR_STATE, "replay: level total differs (group %d)", x.g);
@@ -1922,6 +1955,100 @@ static atf_status run_levels_replay(atf_space* s) {
     d.pairs = d.evals;  // the headline flags; the segment-bound pair counts are not logged per level here
   }
   return ATF_OK;
+}
+
+
+static void replay_reset(atf_space* s) {
+  const size_t G = s->groups.size();
+  for (size_t g = 0; g < G; g++) {
+    s->data[g].assign(s->groups[g].levels.size(), LevelData{});
+    for (auto& c : s->arena[g]) c.used = 0;
+  }
+  s->tails.assign(G, {});
+}
+
+static atf_status run_levels_replay(atf_space* s) {
+  NvtxRange nvtx("atf replay");
+  cudaStream_t user_st = (cudaStream_t)s->opts.stream;
+  const size_t G = s->groups.size();
+  int max_rounds = 0;
+  for (size_t g = 0; g < G; g++) max_rounds = std::max(max_rounds, (int)s->groups[g].levels.size() + 1);
+  if ((size_t)max_rounds > s->replay_cap) {
+    dfree(s, (char*)s->d_replay, s->replay_cap * 12 * kMaxGroups);
+    s->replay_cap = (size_t)max_rounds;
+    s->d_replay = (unsigned long long*)dalloc(s, s->replay_cap * 12 * kMaxGroups);
+    if (!s->d_replay) { s->replay_cap = 0; return fail(s, ATF_ERR_OOM, "replay log"); }
+  }
+  auto& S = s->gsnap;
+  if (s->graph_exec && s->graph_epoch == s->buf_epoch) {
+    // the captured generation: its host-side state, then one graph launch
+    NvtxRange nvtx_g("atf replay (graph)");
+    s->data = S.data;
+    for (size_t g = 0; g < G; g++)
+      for (size_t i = 0; i < s->arena[g].size() && i < S.used[g].size(); i++) s->arena[g][i].used = S.used[g][i];
+    s->tails = S.tails;
+    CUDA_TRY(s, cudaGraphLaunch(s->graph_exec, user_st));
+    s->replays++;
+    return replay_check(s, S.rounds, S.expect, {}, S.tails_done);
+  }
+  if (s->graph_exec) {  // stale: a buffer it references moved
+    cudaGraphExecDestroy(s->graph_exec);
+    s->graph_exec = nullptr;
+  }
+  // the second replay in a row (every buffer sized by the first) is captured as a graph
+  const bool capture = s->replays >= 1 && !(s->opts.flags & ATF_FLAG_TIMING);
+  int rounds = 0;
+  std::vector<ReplayExpect> expect;
+  std::vector<std::pair<int, int>> timed;
+  std::vector<int> tails_done;
+  atf_status e = ATF_OK;
+  bool captured = false;
+  if (capture) {
+    if (!s->cap_stream) CUDA_TRY(s, cudaStreamCreateWithFlags(&s->cap_stream, cudaStreamNonBlocking));
+    if (!s->cap_ev) CUDA_TRY(s, cudaEventCreateWithFlags(&s->cap_ev, cudaEventDisableTiming));
+    cudaGraph_t graph = nullptr;
+    if (cudaStreamBeginCapture(s->cap_stream, cudaStreamCaptureModeThreadLocal) == cudaSuccess) {
+      s->opts.stream = s->cap_stream;
+      s->capturing = true;
+      e = replay_queue(s, rounds, expect, timed, tails_done);
+      const cudaError_t ce = cudaStreamEndCapture(s->cap_stream, &graph);
+      s->capturing = false;
+      s->opts.stream = user_st;
+      if (e == ATF_OK && ce == cudaSuccess && graph &&
+          cudaGraphInstantiate(&s->graph_exec, graph, 0) == cudaSuccess) {
+        captured = true;
+      } else {
+        s->graph_exec = nullptr;
+      }
+      if (graph) cudaGraphDestroy(graph);
+    }
+    cudaGetLastError();
+    if (captured) {
+      S.data = s->data;
+      S.used.assign(G, {});
+      for (size_t g = 0; g < G; g++)
+        for (auto& c : s->arena[g]) S.used[g].push_back(c.used);
+      S.tails = s->tails;
+      S.rounds = rounds;
+      S.expect = expect;
+      S.tails_done = tails_done;
+      s->graph_epoch = s->buf_epoch;
+      CUDA_TRY(s, cudaGraphLaunch(s->graph_exec, user_st));
+    } else {  // not capturable (e.g. a buffer had to grow): the plain replay
+      s->err.clear();
+      replay_reset(s);
+      rounds = 0;
+      expect.clear();
+      timed.clear();
+      tails_done.clear();
+    }
+  }
+  if (!captured) {
+    e = replay_queue(s, rounds, expect, timed, tails_done);
+    if (e) return e;
+  }
+  s->replays++;
+  return replay_check(s, rounds, expect, timed, tails_done);
 }
 
 // ---------------------------------------------------------------- balanced multi-GPU generation
@@ -2601,6 +2728,7 @@ static atf_status generate_impl(atf_space* s) {
       cudaStreamSynchronize((cudaStream_t)s->opts.stream);
       cudaGetLastError();
       s->replay_ok = false;
+      drop_graph(s);
       for (size_t g = 0; g < G; g++) {
         s->data[g].assign(s->groups[g].levels.size(), LevelData{});
         for (auto& c : s->arena[g]) c.used = 0;
@@ -3297,6 +3425,7 @@ atf_status atf_space_generate_shard(atf_space* s, int32_t rank, int32_t world, i
   if (s->dev_ready && s->ipc_alloc) release_device(s);
   s->ipc_alloc = false;
   s->replay_ok = false;
+  drop_graph(s);
   atf_status e = ensure_device(s);
   if (e) return e;
   size_t G = s->groups.size();
@@ -3468,6 +3597,7 @@ atf_status atf_space_generate_dist(atf_space* s, int32_t rank, int32_t world, at
     if (e) return e;
   }
   s->replay_ok = false;
+  drop_graph(s);
   if (s->dev_ready && !s->ipc_alloc) release_device(s);  // arenas must be exportable (cudaMalloc)
   s->ipc_alloc = true;
   atf_status e = ensure_device(s);

@@ -64,8 +64,9 @@ def _check_against_oracle(Space, spec, generic=False, decode_all_max=3_000_000, 
              | extra_flags)
     with Space(spec, flags=flags) as sp:
         sp.generate()
-        if regenerate:        # the second generation of a space replays the first one's level sizes
-            sp.generate()
+        if regenerate:        # the second generation of a space replays the first one's level sizes;
+            for _ in range(3):  # the third is captured as a CUDA graph, the fourth launches it
+                sp.generate()
         assert sp.groups() == [g["members"] for g in ref["groups"]]
         assert sp.size() == int(ref["S"])
         assert sp.group_sizes() == [g["size"] for g in ref["groups"]]
@@ -132,11 +133,37 @@ def test_small_specs(Space, name, generic):
 
 @pytest.mark.parametrize("name", list(SMALL))
 def test_small_specs_regenerated(Space, name):
-    """Steady state: the second generation of a space (replay of the first one's level sizes, one
-    synchronisation) gives the same space, headline flags and default flags."""
+    """Steady state: later generations of a space (replay of the first one's level sizes, one
+    synchronisation; from the third on one CUDA graph launch) give the same space, headline flags
+    and default flags."""
     from paper_conf_hpdc_raschg18_b200 import _lib as L
     _check_against_oracle(Space, SMALL[name](), regenerate=True)
     _check_against_oracle(Space, SMALL[name](), regenerate=True, extra_flags=L.ATF_FLAG_NO_SEG_BOUNDS)
+
+
+def test_graph_replay_follows_buffer_moves(Space):
+    """The captured replay graph references the space's buffers: an operation that reallocates
+    one between generations (here: decodes of growing size) makes the next generation capture a
+    new graph; every generation's levels equal the first one's."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    spec = A.c3_xgemm((20, 96, 8))
+    with Space(spec, flags=L.ATF_FLAG_NO_SEG_BOUNDS) as sp:
+        sp.generate()
+        G = sp.num_groups()
+        want = [[tuple(t.clone() if t is not None else None for t in sp.level_tensors(g, k))
+                 for k in range(sp.num_levels(g))] for g in range(G)]
+        S = sp.size()
+        for i in range(6):
+            if i in (3, 4):
+                n = min(S, 1000 * (10 ** i))
+                sp.decode(torch.arange(n, dtype=torch.int64, device="cuda") % S)
+            sp.generate()
+            for g in range(G):
+                for k in range(sp.num_levels(g)):
+                    rec, csr = sp.level_tensors(g, k)
+                    assert torch.equal(rec, want[g][k][0]), (i, g, k)
+                    if csr is not None:
+                        assert torch.equal(csr, want[g][k][1]), (i, g, k)
 
 
 @pytest.mark.parametrize("seed", range(0, 80, 3))
