@@ -103,7 +103,8 @@ struct LevelArgs {
   uint32_t* tile_total;     // [n_tiles] children per tile
   unsigned long long* tile_seg;  // [n_tiles] stash segment (records)
   const uint64_t* tile_base;     // [n_tiles + 1] exclusive scan of tile_total
-  const uint32_t* piece_tile;    // [total / kPiece + 1] tile holding output record p * kPiece
+  const uint32_t* piece_tile;    // [total >> piece_shift + 1] tile holding output record p << piece_shift
+  int32_t piece_shift;           // level_emit_kernel's piece size (2^7 for small levels, else 2^kPieceShift)
   // geometry (host choose_geometry)
   int32_t kind;             // K_NARROW: one thread per frontier node, r <= 64 candidates each
                             // K_WIDE:   each thread owns cpt consecutive candidates of a chunk
@@ -154,6 +155,7 @@ constexpr int kNfNPL = 4;  // narrow fast kernel: frontier nodes per lane (warp 
 constexpr int kWT = 32;        // warp-tile kernel: frontier nodes per warp tile (one per lane)
 constexpr int kItemCap = 512;  // warp-tile kernel: items whose exact masks pass 1 keeps for the emit pass
 constexpr int kPieceShift = 10;  // level_emit_kernel copies the level in pieces of 2^10 records
+                                 // (2^7 for levels below 2^20 records: more warps on a small level)
 // Hot-loop filter of the wide kernel: a superset test of one conjunct, 2 instructions per
 // (node, candidate) pair (IMAD + ISETP.OR into a per-node predicate).
 enum HotKind : int32_t {
@@ -336,7 +338,7 @@ int launch_decode128(const DecodeArgs& a, const uint64_t* idx_lo, const uint64_t
                      uint64_t S_hi, void* stream);
 int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long long* status,
                     unsigned int* counter, void* stream, uint32_t* piece_tile = nullptr,
-                    uint64_t piece_cap = 0);
+                    uint64_t piece_cap = 0, int piece_shift = kPieceShift);
 int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
 void jit_set_tail_stage(int bytes);  // test hook: tail emit staging bytes per warp (0: default)
 int launch_host_gate(const unsigned int* flag, unsigned int v, void* stream);

@@ -1383,7 +1383,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     const size_t o_seg = 0, o_base = o_seg + 8 * n, o_tot = o_base + 8 * (n + 1);
     const size_t o_scan = (o_tot + 4 * n + 15) & ~(size_t)15, o_cnt = o_scan + 8 * nscan, o_top = o_cnt + 16;
     const size_t o_piece = o_top + 16;
-    piece_cap = (a.stash_cap >> kPieceShift) + 2;
+    a.piece_shift = est < (1ull << 20) ? 7 : kPieceShift;
+    piece_cap = (a.stash_cap >> a.piece_shift) + 2;
     if ((e = ensure_buf(s, &gbf.scratch, &gbf.scratch_cap, o_piece + 4 * piece_cap, "tile scratch"))) return e;
     char* const d_scratch = gbf.scratch;
     a.tile_seg = (unsigned long long*)(d_scratch + o_seg);
@@ -1453,7 +1454,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     if (!ce) ce = launch_nfast_emit(a, gp.words, ls);
     if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   } else {
-    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, ls, piece_tile, piece_cap);
+    ce = launch_scan_u32(a.tile_total, scan_out, (int64_t)a.n_tiles, scan_status, scan_counter, ls, piece_tile, piece_cap,
+                         a.piece_shift);
     if (!ce) ce = launch_level_emit(a, gp.words, ls);
     if (ce) return fail(s, ATF_ERR_CUDA, "level scan/emit (group %d level %d): %s", g, k, cudaGetErrorString((cudaError_t)ce));
   }

@@ -87,7 +87,8 @@ template <int W>
 __global__ void __launch_bounds__(256) level_emit_kernel(const __grid_constant__ LevelArgs a) {
   using V = typename RecVec<W>::T;
   constexpr int VPR = W == 8 ? 2 : 1;  // vectors per record
-  constexpr uint64_t P = 1ull << kPieceShift;
+  const int psh = a.piece_shift;
+  const uint64_t P = 1ull << psh;
   const int lane = threadIdx.x & 31;
   const uint64_t gt = (uint64_t)blockIdx.x * blockDim.x + threadIdx.x;
   const uint64_t nt = (uint64_t)gridDim.x * blockDim.x;
@@ -115,9 +116,9 @@ __global__ void __launch_bounds__(256) level_emit_kernel(const __grid_constant__
   // and stash segment); each output record finds its tile by a 5-step shuffle search of
   // the window; 4 records per lane in flight.
   const uint64_t gw = gt >> 5, nw = nt >> 5;
-  const uint64_t n_pieces = (total + P - 1) >> kPieceShift;
+  const uint64_t n_pieces = (total + P - 1) >> psh;
   for (uint64_t p = gw; p < n_pieces; p += nw) {
-    uint64_t o = p << kPieceShift;
+    uint64_t o = p << psh;
     const uint64_t o_end = min(o + P, total);
     uint64_t t0 = a.piece_tile[p];
     while (o < o_end) {
@@ -169,7 +170,7 @@ int launch_level_emit(const LevelArgs& a, int words, void* stream) {
   const int sms = cached_sm_count();
   // enough warps for the larger of the parents (CSR) and the records (pieces); the
   // record count is only known on the device, so the grid covers the stash capacity
-  const uint64_t pieces = (a.stash_cap >> kPieceShift) + 1;
+  const uint64_t pieces = (a.stash_cap >> a.piece_shift) + 1;
   uint64_t blocks = std::max<uint64_t>((a.n_parents + 255) / 256, (pieces + 7) / 8);
   const uint64_t cap = (uint64_t)sms * 8;
   if (blocks > cap) blocks = cap;
@@ -517,7 +518,7 @@ int launch_divisible16_check(unsigned long long* mismatches, void* stream) {
 // Exclusive scan u32 -> u64 with the same look-back as expand_kernel; out[n] = total.
 __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restrict__ out, int64_t n,
                             unsigned long long* status, unsigned int* counter, uint64_t n_tiles,
-                            uint32_t* __restrict__ piece_tile, uint64_t piece_cap) {
+                            uint32_t* __restrict__ piece_tile, uint64_t piece_cap, int psh) {
   __shared__ uint32_t s_tile;
   __shared__ unsigned long long s_wt[33];
   __shared__ unsigned long long s_base;
@@ -562,8 +563,8 @@ __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restric
       if (i0 + q < n) {
         out[i0 + q] = run;
         if (piece_tile && v[q]) {  // pieces whose first record lies in element i0 + q
-          constexpr uint64_t P = 1ull << kPieceShift;
-          for (uint64_t p = (run + P - 1) >> kPieceShift; (p << kPieceShift) < run + v[q] && p < piece_cap; p++)
+          const uint64_t P = 1ull << psh;
+          for (uint64_t p = (run + P - 1) >> psh; (p << psh) < run + v[q] && p < piece_cap; p++)
             piece_tile[p] = (uint32_t)(i0 + q);
         }
       }
@@ -574,13 +575,14 @@ __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restric
 }
 
 int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long long* status, unsigned int* counter,
-                    void* stream, uint32_t* piece_tile, uint64_t piece_cap) {
+                    void* stream, uint32_t* piece_tile, uint64_t piece_cap, int piece_shift) {
   const int B = 256;
   const uint64_t n_tiles = n > 0 ? (uint64_t)((n + B * 4 - 1) / (B * 4)) : 1;
   const int sms = cached_sm_count();
   uint64_t grid = (uint64_t)sms * 4;
   if (grid > n_tiles) grid = n_tiles;
-  scan_kernel<<<(unsigned)grid, B, 0, (cudaStream_t)stream>>>(in, out, n, status, counter, n_tiles, piece_tile, piece_cap);
+  scan_kernel<<<(unsigned)grid, B, 0, (cudaStream_t)stream>>>(in, out, n, status, counter, n_tiles, piece_tile, piece_cap,
+                                                                 piece_shift);
   return (int)cudaGetLastError();
 }
 
