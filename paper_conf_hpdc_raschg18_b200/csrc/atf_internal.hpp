@@ -339,6 +339,9 @@ int launch_decode128(const DecodeArgs& a, const uint64_t* idx_lo, const uint64_t
 int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long long* status,
                     unsigned int* counter, void* stream, uint32_t* piece_tile = nullptr,
                     uint64_t piece_cap = 0, int piece_shift = kPieceShift);
+// `batch` independent scans of n elements in one launch (see scan_kernel)
+int launch_scan_u32_batch(const uint32_t* in, uint64_t* out, int64_t n, int batch, unsigned long long* status,
+                          uint64_t status_stride, unsigned int* counter, void* stream);
 int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
 void jit_set_tail_stage(int bytes);  // test hook: tail emit staging bytes per warp (0: default)
 int launch_host_gate(const unsigned int* flag, unsigned int v, void* stream);

@@ -1626,14 +1626,13 @@ static atf_status queue_tail_count(atf_space* s, int g, int k0, const uint32_t* 
   int ce = tj ? jit_tail_launch(tj, t, false, ls) : launch_tail_count(t, gp.words, ls);
   if (ce) return fail(s, ATF_ERR_CUDA, "tail count launch (group %d): %s", g, cudaGetErrorString((cudaError_t)ce));
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0].mid, ls));
-  for (int d = 0; d < nl && !ce; d++)
-    ce = launch_scan_u32(t.tile_total + d * n, (uint64_t*)t.tile_base + d * (n + 1), (int64_t)n,
-                         (unsigned long long*)(gbf.scratch + o_stat) + d * ns, (unsigned int*)(gbf.scratch + o_cnt) + d,
-                         ls);
+  if (!ce)  // one launch scans every tail level's tile counts
+    ce = launch_scan_u32_batch(t.tile_total, (uint64_t*)t.tile_base, (int64_t)n, nl,
+                               (unsigned long long*)(gbf.scratch + o_stat), ns, (unsigned int*)(gbf.scratch + o_cnt), ls);
   if (ce) return fail(s, ATF_ERR_CUDA, "tail scan (group %d): %s", g, cudaGetErrorString((cudaError_t)ce));
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k0].second, ls));
   if (!serial) CUDA_TRY(s, cudaEventRecord(gbf.join, ls));
-  s->data[g][k0].launches += 1 + nl;
+  s->data[g][k0].launches += 2;
   pd = Pending{};
   pd.g = g;
   pd.k = k0;

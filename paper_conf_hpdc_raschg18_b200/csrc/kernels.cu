@@ -516,9 +516,15 @@ int launch_divisible16_check(unsigned long long* mismatches, void* stream) {
 
 // ---------------------------------------------------------------- standalone scan (tests)
 // Exclusive scan u32 -> u64 with the same look-back as expand_kernel; out[n] = total.
+// blockIdx.y selects one of several independent scans of equal length (the fused tail's levels):
+// arrays at in + y * n, out + y * (n + 1), status + y * st_stride, counter + y.
 __global__ void scan_kernel(const uint32_t* __restrict__ in, uint64_t* __restrict__ out, int64_t n,
                             unsigned long long* status, unsigned int* counter, uint64_t n_tiles,
-                            uint32_t* __restrict__ piece_tile, uint64_t piece_cap, int psh) {
+                            uint32_t* __restrict__ piece_tile, uint64_t piece_cap, int psh, uint64_t st_stride) {
+  in += (uint64_t)blockIdx.y * (uint64_t)n;
+  out += (uint64_t)blockIdx.y * (uint64_t)(n + 1);
+  status += (uint64_t)blockIdx.y * st_stride;
+  counter += blockIdx.y;
   __shared__ uint32_t s_tile;
   __shared__ unsigned long long s_wt[33];
   __shared__ unsigned long long s_base;
@@ -582,7 +588,18 @@ int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long 
   uint64_t grid = (uint64_t)sms * 4;
   if (grid > n_tiles) grid = n_tiles;
   scan_kernel<<<(unsigned)grid, B, 0, (cudaStream_t)stream>>>(in, out, n, status, counter, n_tiles, piece_tile, piece_cap,
-                                                                 piece_shift);
+                                                                 piece_shift, 0);
+  return (int)cudaGetLastError();
+}
+int launch_scan_u32_batch(const uint32_t* in, uint64_t* out, int64_t n, int batch, unsigned long long* status,
+                          uint64_t status_stride, unsigned int* counter, void* stream) {
+  const int B = 256;
+  const uint64_t n_tiles = n > 0 ? (uint64_t)((n + B * 4 - 1) / (B * 4)) : 1;
+  const int sms = cached_sm_count();
+  uint64_t grid = (uint64_t)sms * 4;
+  if (grid > n_tiles) grid = n_tiles;
+  scan_kernel<<<dim3((unsigned)grid, (unsigned)batch), B, 0, (cudaStream_t)stream>>>(
+      in, out, n, status, counter, n_tiles, nullptr, 0, kPieceShift, status_stride);
   return (int)cudaGetLastError();
 }
 
