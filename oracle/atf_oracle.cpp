@@ -166,19 +166,20 @@ static i64 run_value(const std::vector<int32_t>& code, i64 x, const i64* vals, b
 // ... from begin to end using the optional step_size"; "the interval comprises the
 // elements generator(i) for each i from begin to end"; "atf::set(val_1,...,val_n)".
 static std::vector<i64> materialise(const Json& r) {
+  // values are int64 ("arbitrary fundamental type T"; reading #22): an index
+  // or value outside int64 is an error
   std::string kind = r.at("kind").str;
   std::vector<i64> v;
   if (kind == "interval" || kind == "pow2") {
     i64 b = r.at("begin").num, e = r.at("end").num, st = r.at("step").num;
     if (st <= 0) throw std::runtime_error("range: step must be positive");
-    for (i64 i = b; i <= e; i += st) {          // inclusive both ends (reading #1)
+    for (__int128 i = b; i <= e; i += st) {     // inclusive both ends (reading #1)
       if (kind == "interval") {
-        if (i < INT32_MIN || i > INT32_MAX) throw std::runtime_error("range: value outside int32");
-        v.push_back(i);
+        v.push_back((i64)i);
       } else {
-        if (i < 0 || i > 30) throw std::runtime_error("range: pow2 exponent outside [0,30]");
+        if (i < 0 || i > 62) throw std::runtime_error("range: pow2 exponent outside [0,62]");
         i64 p = 1;
-        for (i64 k = 0; k < i; k++) p *= 2;      // exact 2^i (reading #3)
+        for (i64 k = 0; k < (i64)i; k++) p *= 2;  // exact 2^i (reading #3)
         v.push_back(p);
       }
     }
@@ -189,11 +190,10 @@ static std::vector<i64> materialise(const Json& r) {
     for (auto& w : r.at("code").arr) code.push_back((int32_t)w.num);
     for (size_t k = 0; k < code.size(); k += (code[k] == CONST ? 3 : 1))
       if (code[k] == PARAM) throw std::runtime_error("range: generator references a parameter");
-    for (i64 i = b; i <= e; i += st) {
+    for (__int128 i = b; i <= e; i += st) {
       bool poison = false;
-      i64 y = run_value(code, i, nullptr, poison);
+      i64 y = run_value(code, (i64)i, nullptr, poison);
       if (poison) throw std::runtime_error("range: generator poison");
-      if (y < INT32_MIN || y > INT32_MAX) throw std::runtime_error("range: value outside int32");
       for (i64 z : v)
         if (z == y) throw std::runtime_error("range: duplicate generator value");  // reading #5
       v.push_back(y);
@@ -203,13 +203,24 @@ static std::vector<i64> materialise(const Json& r) {
       if (x.kind != Json::NUM || !x.integral) throw std::runtime_error("range: set values must be integers");
       for (i64 y : v)
         if (y == x.num) throw std::runtime_error("range: duplicate set value");  // reading #5
-      if (x.num < INT32_MIN || x.num > INT32_MAX) throw std::runtime_error("range: value outside int32");
       v.push_back(x.num);
     }
   } else {
     throw std::runtime_error("range: unknown kind " + kind);
   }
   return v;
+}
+
+// Value width of the files this oracle reads and writes (o1 / leaves / decode rows, check
+// input): int32 while every value of the spec fits int32, else int64 (reading #22).
+static bool g_w64 = false;
+static void put_val(FILE* f, i64 v) {
+  if (g_w64) {
+    std::fwrite(&v, 8, 1, f);
+  } else {
+    int32_t w = (int32_t)v;
+    std::fwrite(&w, 4, 1, f);
+  }
 }
 
 static Spec load_spec(const std::string& path) {
@@ -249,6 +260,8 @@ static Spec load_spec(const std::string& path) {
           i += 1;
         }
       }
+    for (i64 v : p.values)
+      if (v < INT32_MIN || v > INT32_MAX) g_w64 = true;
     s.params.push_back(p);
   }
   return s;
@@ -476,7 +489,7 @@ struct GroupRun {
 static inline u64 rowhash(const i64* v, size_t n) {
   u64 z = 0x243F6A8885A308D3ull;
   for (size_t k = 0; k < n; k++) {
-    z ^= (u64)(uint32_t)(int32_t)v[k];
+    z ^= g_w64 ? (u64)v[k] : (u64)(uint32_t)(int32_t)v[k];
     z *= 0x9E3779B97F4A7C15ull;
     z ^= z >> 32;
   }
@@ -615,7 +628,7 @@ static int cmd_o1(const Spec& s, const char* out) {
   if (out) {
     FILE* f = std::fopen(out, "wb");
     for (auto& r : rows)
-      for (i64 v : r.vals) { int32_t w = (int32_t)v; std::fwrite(&w, 4, 1, f); }
+      for (i64 v : r.vals) put_val(f, v);
     std::fclose(f);
   }
   std::printf("{\"S\":%zu,\"evaluated\":%" PRIu64 ",\"seconds\":%.6f,\"overflow\":%s}\n", rows.size(), evaluated,
@@ -632,7 +645,7 @@ static int cmd_leaves(const Spec& s, int g, const char* out) {
   FILE* f = std::fopen(out, "wb");
   u64 n = 0;
   gr.sink = [&](const i64* gv) {
-    for (size_t k = 0; k < gr.members.size(); k++) { int32_t w = (int32_t)gv[k]; std::fwrite(&w, 4, 1, f); }
+    for (size_t k = 0; k < gr.members.size(); k++) put_val(f, gv[k]);
     n++;
   };
   gr.run(0, SIZE_MAX);
@@ -641,7 +654,8 @@ static int cmd_leaves(const Spec& s, int g, const char* out) {
   return 0;
 }
 
-// decode: indices (u64 little-endian file) -> values, int32 SoA [P][n].  Streams each
+// decode: indices (u64 little-endian file) -> values, int32 SoA [P][n] (int64 if g_w64; invalid
+// rows INT32_MIN / INT64_MIN).  Streams each
 // group in canonical order and picks the requested digits (no materialisation).
 static int cmd_decode(const Spec& s, const char* idxfile, const char* out, int threads) {
   auto groups = groups_of(s);
@@ -663,7 +677,7 @@ static int cmd_decode(const Spec& s, const char* idxfile, const char* out, int t
     std::fclose(f);
   }
   size_t n = idx.size();
-  std::vector<int32_t> res(P * n, INT32_MIN);
+  std::vector<i64> res(P * n, g_w64 ? INT64_MIN : (i64)INT32_MIN);
   u64 bad = 0;
   // digits: group G-1 least significant
   std::vector<std::vector<u64>> digit(G, std::vector<u64>(n));
@@ -684,7 +698,7 @@ static int cmd_decode(const Spec& s, const char* idxfile, const char* out, int t
     gr.members = groups[g];
     gr.sink = [&](const i64* gv) {
       while (cur < order.size() && digit[g][order[cur]] == leaf) {
-        for (size_t k = 0; k < gr.members.size(); k++) res[(size_t)gr.members[k] * n + order[cur]] = (int32_t)gv[k];
+        for (size_t k = 0; k < gr.members.size(); k++) res[(size_t)gr.members[k] * n + order[cur]] = gv[k];
         cur++;
       }
       leaf++;
@@ -700,7 +714,7 @@ static int cmd_decode(const Spec& s, const char* idxfile, const char* out, int t
   }
   if (std::strcmp(out, "-") != 0) {
     FILE* f = std::fopen(out, "wb");
-    std::fwrite(res.data(), 4, res.size(), f);
+    for (i64 v : res) put_val(f, v);
     std::fclose(f);
   }
   std::printf("{\"n\":%zu,\"invalid\":%" PRIu64 ",\"S\":\"%s\",\"hash\":\"%" PRIu64 "\"}\n", n, bad,
@@ -708,21 +722,23 @@ static int cmd_decode(const Spec& s, const char* idxfile, const char* out, int t
   return 0;
 }
 
-// check: rows of values (int32 [n][P]) -> how many satisfy every constraint
+// check: rows of values (int32 [n][P], int64 if g_w64) -> how many satisfy every constraint
 static int cmd_check(const Spec& s, const char* rowfile, const char* flagfile) {
   size_t P = s.params.size();
   FILE* f = std::fopen(rowfile, "rb");
   FILE* ff = flagfile ? std::fopen(flagfile, "wb") : nullptr;  // optional: one byte per row
   std::vector<int32_t> row(P);
+  std::vector<i64> row64(P);
   std::vector<i64> vals(P);
   u64 n = 0, ok = 0, in_range = 0;
-  while (std::fread(row.data(), 4, P, f) == P) {
+  for (;;) {
+    if (g_w64 ? std::fread(row64.data(), 8, P, f) != P : std::fread(row.data(), 4, P, f) != P) break;
     n++;
     bool good = true, inr = true;
     for (size_t p = 0; p < P; p++) {
-      vals[p] = row[p];
+      vals[p] = g_w64 ? row64[p] : (i64)row[p];
       auto& R = s.params[p].values;
-      if (std::find(R.begin(), R.end(), (i64)row[p]) == R.end()) inr = false;
+      if (std::find(R.begin(), R.end(), vals[p]) == R.end()) inr = false;
     }
     for (size_t p = 0; p < P; p++) good = constraint_holds(s, (int)p, vals[p], vals.data()) && good;
     ok += (good && inr);
@@ -793,7 +809,7 @@ static int cmd_time(const Spec& s, int threads, double budget_s) {
 int main(int argc, char** argv) {
   if (argc < 3) {
     std::fprintf(stderr,
-                 "usage: atf_oracle info|o1|leaves|decode|check|time SPEC.json [args] [--threads T] "
+                 "usage: atf_oracle info|o1|leaves|decode|check|time|width SPEC.json [args] [--threads T] "
                  "[--native c1|c2:N|c3:M,N,K|saxpy:N] [--native-check] [--hash] [--budget S]\n");
     return 2;
   }
@@ -815,6 +831,7 @@ int main(int argc, char** argv) {
   try {
     Spec s = load_spec(pos.at(0));
     if (cmd == "info") return cmd_info(s, threads, want_hash);
+    if (cmd == "width") return std::printf("{\"w64\":%s}\n", g_w64 ? "true" : "false"), 0;
     if (cmd == "o1") return cmd_o1(s, pos.size() > 1 ? pos[1].c_str() : nullptr);
     if (cmd == "leaves") return cmd_leaves(s, std::atoi(pos.at(1).c_str()), pos.at(2).c_str());
     if (cmd == "decode") return cmd_decode(s, pos.at(1).c_str(), pos.at(2).c_str(), threads);

@@ -54,25 +54,41 @@ def info(spec, threads: int = 1, hash: bool = False, native: Optional[str] = Non
         return _run(args, timeout)
 
 
+def width(spec) -> bool:
+    """True when some value of the spec lies outside int32: the oracle's row files (o1 / leaves /
+    decode output, check input) are then int64 instead of int32 (reading #22)."""
+    with tempfile.TemporaryDirectory() as td:
+        return bool(_run(["width", _spec_path(spec, td)])["w64"])
+
+
+def vdtype(spec):
+    return np.int64 if width(spec) else np.int32
+
+
 def o1(spec, timeout=None):
-    """Literal brute force over the full product; rows (int32 [S][P]) in canonical order."""
+    """Literal brute force over the full product; rows (int32 [S][P], int64 for specs with values
+    outside int32) in canonical order."""
+    dt = vdtype(spec)
     with tempfile.TemporaryDirectory() as td:
         out = os.path.join(td, "rows.bin")
         d = _run(["o1", _spec_path(spec, td), out], timeout)
-        rows = np.fromfile(out, dtype=np.int32) if os.path.exists(out) else np.zeros(0, np.int32)
+        rows = np.fromfile(out, dtype=dt) if os.path.exists(out) else np.zeros(0, dt)
         P = len(spec.params) if not isinstance(spec, str) else None
         return d, (rows.reshape(-1, P) if P else rows)
 
 
 def leaves(spec, group: int, n_members: int, timeout=None) -> np.ndarray:
+    dt = vdtype(spec)
     with tempfile.TemporaryDirectory() as td:
         out = os.path.join(td, "leaves.bin")
         _run(["leaves", _spec_path(spec, td), group, out], timeout)
-        return np.fromfile(out, dtype=np.int32).reshape(-1, n_members)
+        return np.fromfile(out, dtype=dt).reshape(-1, n_members)
 
 
 def decode(spec, indices: np.ndarray, threads: int = 1, want_rows: bool = True, timeout=None):
-    """indices (uint64) -> (info, int32 SoA [P][n] or None).  info has 'hash' and 'invalid'."""
+    """indices (uint64) -> (info, int32 SoA [P][n] or None; int64 for specs with values outside
+    int32).  info has 'hash' and 'invalid'."""
+    dt = vdtype(spec) if want_rows else None
     with tempfile.TemporaryDirectory() as td:
         idx = os.path.join(td, "idx.bin")
         np.ascontiguousarray(indices, dtype=np.uint64).tofile(idx)
@@ -81,16 +97,17 @@ def decode(spec, indices: np.ndarray, threads: int = 1, want_rows: bool = True, 
         if not want_rows:
             return d, None
         P = len(spec.params)
-        return d, np.fromfile(out, dtype=np.int32).reshape(P, -1)
+        return d, np.fromfile(out, dtype=dt).reshape(P, -1)
 
 
 def check(spec, rows: np.ndarray, timeout=None, per_row: bool = False) -> dict:
     """Constraint check of configurations rows[n][P] (valid iff every parameter's
     value is in its range and every constraint holds).  per_row: also return "flags", a
     uint8 array with 1 for each valid row."""
+    dt = vdtype(spec)
     with tempfile.TemporaryDirectory() as td:
         f = os.path.join(td, "rows.bin")
-        np.ascontiguousarray(rows, dtype=np.int32).tofile(f)
+        np.ascontiguousarray(rows, dtype=dt).tofile(f)
         args = ["check", _spec_path(spec, td), f]
         if per_row:
             args.append(os.path.join(td, "flags.bin"))
@@ -105,15 +122,17 @@ def time_sample(spec, threads: int, budget_s: float, timeout=None) -> dict:
         return _run(["time", _spec_path(spec, td), "--threads", threads, "--budget", budget_s], timeout)
 
 
-def rowhash_rows(rows: np.ndarray) -> int:
+def rowhash_rows(rows: np.ndarray, w64: bool = False) -> int:
     """Order-dependent hash H = sum_i rowhash(row_i) * (2i+1) mod 2^64 (same definition as the
-    C++ oracle's; used to compare large row sequences without storing them)."""
+    C++ oracle's; used to compare large row sequences without storing them).  w64: the spec has
+    values outside int32 and its rows hash their full 64-bit values."""
     rows = np.ascontiguousarray(rows)
     n = rows.shape[0]
     with np.errstate(over="ignore"):
         z = np.full(n, 0x243F6A8885A308D3, dtype=np.uint64)
         for k in range(rows.shape[1]):
-            z ^= rows[:, k].astype(np.int64).astype(np.uint64) & np.uint64(0xFFFFFFFF)
+            col = rows[:, k].astype(np.int64).astype(np.uint64)
+            z ^= col if w64 else col & np.uint64(0xFFFFFFFF)
             z *= np.uint64(0x9E3779B97F4A7C15)
             z ^= z >> np.uint64(32)
         w = np.arange(n, dtype=np.uint64) * np.uint64(2) + np.uint64(1)
