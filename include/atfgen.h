@@ -61,25 +61,36 @@ typedef enum {
   ATF_ERR_LIMIT = -10       /* a documented v1 limit is exceeded                       */
 } atf_status;
 
-/* Range kinds.
- *   INTERVAL: values begin, begin+step, ..., <= end (inclusive, reading #1); int32.
- *   POW2:     values 2^i for i = begin, begin+step, ..., <= end; 0 <= i <= 30
+/* Range kinds ("a range of values of an arbitrary fundamental type T (e.g., bool,
+ * integer, or float)").  Values are int64 (reading #22); a space whose values all fit int32
+ * is an "int32 space" (decoded by the int32 entry points), otherwise an "int64 space"
+ * (atf_space_value_bits() == 64; decoded by the *_i64 entry points).
+ *   INTERVAL: values begin, begin+step, ..., <= end (inclusive, reading #1), any int64.
+ *   POW2:     values 2^i for i = begin, begin+step, ..., <= end; 0 <= i <= 62
  *             ("atf::interval<size_t>(1,10,[](i){return pow(2,i);})" = first ten powers of 2).
- *   SET:      values[0..n_values) in the listed order; duplicates -> ATF_ERR_DUPLICATE.
+ *   SET:      values[0..n_values) (int32) in the listed order; duplicates -> ATF_ERR_DUPLICATE.
  *             bool and enum parameters are SETs of ints ({0,1} for bools).
  *   GEN:      the general generator of P:57 ("the elements generator(i) for each i from
  *             begin to end"): values gen(i) for i = begin, begin+step, ..., <= end, where
  *             gen is a bytecode program (`values` = its int32 words, `n_values` = their
  *             number) in which X is i (PARAM is not allowed).  Evaluated exactly in int64
- *             on the host when the parameter is added; a poisoned or non-int32 value ->
- *             ATF_ERR_BYTECODE, a repeated value -> ATF_ERR_DUPLICATE (reading #5). */
-typedef enum { ATF_RANGE_INTERVAL = 0, ATF_RANGE_POW2 = 1, ATF_RANGE_SET = 2, ATF_RANGE_GEN = 3 } atf_range_kind;
+ *             on the host when the parameter is added; a poisoned value or int64 overflow ->
+ *             ATF_ERR_BYTECODE / ATF_ERR_OVERFLOW, a repeated value -> ATF_ERR_DUPLICATE
+ *             (reading #5).
+ *   SET64:    values64[0..n_values) (int64) in the listed order; duplicates -> ATF_ERR_DUPLICATE.
+ * A parameter whose values do not all fit int32 is expanded by the generic kernels (every
+ * conjunct of its own level interpreted in int64; the levels that reference it read its int64
+ * value table); int32 parameters keep every fast path. */
+typedef enum {
+  ATF_RANGE_INTERVAL = 0, ATF_RANGE_POW2 = 1, ATF_RANGE_SET = 2, ATF_RANGE_GEN = 3, ATF_RANGE_SET64 = 4
+} atf_range_kind;
 
 typedef struct {
-  int32_t kind;           /* atf_range_kind */
+  int32_t kind;             /* atf_range_kind */
   int64_t begin, end, step;
-  const int32_t* values;  /* SET only: host pointer, copied */
-  int64_t n_values;
+  const int32_t* values;    /* SET / GEN: host pointer, copied */
+  int64_t n_values;         /* SET / GEN / SET64: number of entries */
+  const int64_t* values64;  /* SET64 only: host pointer, copied */
 } atf_range;
 
 /* Device allocator hooks (e.g. PyTorch's caching allocator).  If alloc is NULL
@@ -275,7 +286,9 @@ atf_status atf_space_level_view(const atf_space* s, int32_t g, int32_t k, atf_le
  * ATF_ERR_OVERFLOW) into configurations: d_out is int32 SoA, column p (the
  * value of parameter p) at d_out + p*ld, ld >= n.  Rows whose index >= S are
  * filled with INT32_MIN and the call returns ATF_ERR_INDEX (after a stream sync).
- * Otherwise asynchronous on `stream` (NULL = the space's stream). */
+ * Otherwise asynchronous on `stream` (NULL = the space's stream).  The int32 decoders
+ * (decode_indices / decode_digits / decode_indices128 / decode_range) return
+ * ATF_ERR_OVERFLOW on an int64 space (reading #22): use the *_i64 decoders below. */
 atf_status atf_space_decode_indices(const atf_space* s, const uint64_t* d_idx, int64_t n,
                                     int32_t* d_out, int64_t ld, void* stream);
 /* Like decode_indices but with per-group digits: d_digits is [G][n] uint64
@@ -294,6 +307,20 @@ atf_status atf_space_decode_indices128(const atf_space* s, const uint64_t* d_idx
 atf_status atf_space_decode_range(const atf_space* s, uint64_t first_lo, uint64_t first_hi, int64_t n, int32_t* d_out,
                                   int64_t ld, void* stream);
 
+/* int64 configurations (P:57 values of any integer type; reading #22): the same decoders with
+ * int64 SoA output (column p at d_out + p*ld), valid on every generated space (an int32
+ * space's values are sign-extended).  Rows out of range are filled with INT64_MIN and the call
+ * returns ATF_ERR_INDEX (after a stream sync); otherwise asynchronous on `stream`. */
+atf_status atf_space_decode_indices_i64(const atf_space* s, const uint64_t* d_idx, int64_t n, int64_t* d_out,
+                                        int64_t ld, void* stream);
+atf_status atf_space_decode_digits_i64(const atf_space* s, const uint64_t* d_digits, int64_t n, int64_t* d_out,
+                                       int64_t ld, void* stream);
+atf_status atf_space_decode_range_i64(const atf_space* s, uint64_t first_lo, uint64_t first_hi, int64_t n,
+                                      int64_t* d_out, int64_t ld, void* stream);
+/* 32 if every parameter value fits int32 (the int32 decoders, encode, neighbours and the
+ * full-product filter apply), else 64.  Callable from BUILDING on. */
+atf_status atf_space_value_bits(const atf_space* s, int32_t* bits);
+
 /* Encode = inverse of decode (the index access of P:229-231 read
  * backwards, which also answers membership): d_values is a batch of n configurations,
  * int32 SoA (value of parameter p at d_values + p*ld, ld >= n).  Each row is located by a
@@ -303,7 +330,7 @@ atf_status atf_space_decode_range(const atf_space* s, uint64_t first_lo, uint64_
  * mixed-radix index d_idx[n] (group 0 most significant; UINT64_MAX for rows not in the
  * space) and needs S < 2^64 (else ATF_ERR_OVERFLOW).  Asynchronous on `stream`
  * (NULL = the space's stream); device buffers are borrowed until the work completes.
- * ATF_ERR_STATE before generate and on shard spaces. */
+ * ATF_ERR_STATE before generate and on shard spaces; ATF_ERR_LIMIT on an int64 space. */
 atf_status atf_space_encode_digits(const atf_space* s, const int32_t* d_values, int64_t n, int64_t ld,
                                    uint64_t* d_digits, void* stream);
 atf_status atf_space_encode_indices(const atf_space* s, const int32_t* d_values, int64_t n, int64_t ld,
@@ -317,7 +344,7 @@ atf_status atf_space_encode_indices(const atf_space* s, const int32_t* d_values,
  * per-parameter std::function predicates would (the accepted set is the same).  *h_count =
  * the number of valid tuples (= S), *h_tuples (optional) = the product size.  Synchronous.
  * Needs only a planned space (callable before generate); ATF_ERR_OVERFLOW if the product is
- * >= 2^64. */
+ * >= 2^64; ATF_ERR_LIMIT on an int64 space. */
 atf_status atf_space_filter_product(atf_space* s, uint64_t* h_count, uint64_t* h_tuples);
 
 /* Random neighbours for simulated annealing ("a random neighbor c' of the
@@ -328,7 +355,7 @@ atf_status atf_space_filter_product(atf_space* s, uint64_t* h_count, uint64_t* h
  * the first draw whose row is in the space (tree walk of the changed parameter's group)
  * is kept.  d_moved[i] = the changed parameter id, or -1 (row copied unchanged).  Rows of
  * d_in must be valid configurations.  Asynchronous on `stream`.  ATF_ERR_STATE before
- * generate and on shard spaces. */
+ * generate and on shard spaces; ATF_ERR_LIMIT on an int64 space. */
 atf_status atf_space_neighbors(const atf_space* s, const int32_t* d_in, int64_t ld_in, int64_t n, uint64_t seed,
                                int32_t max_tries, int32_t* d_out, int64_t ld_out, int32_t* d_moved, void* stream);
 

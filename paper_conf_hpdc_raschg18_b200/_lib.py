@@ -23,7 +23,7 @@ ATF_OK = 0
 STATUS = {0: "ATF_OK", -1: "ATF_ERR_INVALID_ARG", -2: "ATF_ERR_OOM", -3: "ATF_ERR_CUDA", -4: "ATF_ERR_STATE",
           -5: "ATF_ERR_BYTECODE", -6: "ATF_ERR_FORWARD_REF", -7: "ATF_ERR_OVERFLOW", -8: "ATF_ERR_INDEX",
           -9: "ATF_ERR_DUPLICATE", -10: "ATF_ERR_LIMIT"}
-ATF_RANGE_INTERVAL, ATF_RANGE_POW2, ATF_RANGE_SET, ATF_RANGE_GEN = 0, 1, 2, 3
+ATF_RANGE_INTERVAL, ATF_RANGE_POW2, ATF_RANGE_SET, ATF_RANGE_GEN, ATF_RANGE_SET64 = 0, 1, 2, 3, 4
 ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT, ATF_FLAG_SERIAL_GROUPS = 1, 2, 8, 16, 32
 ATF_FLAG_NO_SEG_BOUNDS = 64
 ATF_FLAG_NO_TAIL = 128
@@ -33,7 +33,7 @@ ATF_FLAG_DIST_SUBSETS = 512
 
 class atf_range(C.Structure):
     _fields_ = [("kind", C.c_int32), ("begin", C.c_int64), ("end", C.c_int64), ("step", C.c_int64),
-                ("values", C.POINTER(C.c_int32)), ("n_values", C.c_int64)]
+                ("values", C.POINTER(C.c_int32)), ("n_values", C.c_int64), ("values64", C.POINTER(C.c_int64))]
 
 
 ALLOC_FN = C.CFUNCTYPE(C.c_void_p, C.c_size_t, C.c_void_p, C.c_void_p)
@@ -85,6 +85,10 @@ _SIGS = {
     "atf_space_decode_indices128": (_st, [SP, C.c_void_p, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_space_decode_range": (_st, [SP, C.c_uint64, C.c_uint64, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_space_decode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
+    "atf_space_decode_indices_i64": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
+    "atf_space_decode_digits_i64": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
+    "atf_space_decode_range_i64": (_st, [SP, C.c_uint64, C.c_uint64, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
+    "atf_space_value_bits": (_st, [SP, C.POINTER(C.c_int32)]),
     "atf_space_encode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p]),
     "atf_space_encode_indices": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p, C.c_void_p]),
     "atf_space_filter_product": (_st, [SP, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),

@@ -60,7 +60,8 @@ struct LevelArgs {
   const uint32_t* parent_rec;
   uint64_t n_parents;
   // candidates = materialised range of the level's parameter
-  const int32_t* cand;
+  const int32_t* cand;         // int64 parameter (reading #22): the positions 0..r-1
+  const int64_t* cand64;       // int64 parameter: its values (else null); generic terms only
   const uint32_t* cand_magic;  // ceil(2^32/|x|) mod 2^32 per candidate (2^16 for x == 0), host-computed
   const uint32_t* cand_abs;    // |x| per candidate; both padded to a multiple of 128
   int32_t r;
@@ -70,6 +71,7 @@ struct LevelArgs {
   int32_t n_pv;
   int32_t pv_word[kMaxSlots], pv_shift[kMaxSlots], pv_bits[kMaxSlots];
   const int32_t* pv_range[kMaxSlots];
+  const int64_t* pv_range64[kMaxSlots];  // int64 ancestors: their value tables (else null)
   // slots [n_pv, n_slots): hoisted node-invariant expressions (code[inv_off..+inv_len))
   int32_t n_slots;
   int16_t inv_off[kMaxSlots], inv_len[kMaxSlots];
@@ -178,6 +180,7 @@ struct DecodeArgs {
   int16_t lvl_param[kMaxLevels];
   int16_t lvl_word[kMaxLevels], lvl_shift[kMaxLevels], lvl_bits[kMaxLevels];
   const int32_t* lvl_range[kMaxLevels];
+  const int64_t* lvl_range64[kMaxLevels];  // int64 parameters' value tables (else null), reading #22
 };
 
 // Encode (inverse decode): configuration -> per-group leaf index by
@@ -329,12 +332,13 @@ std::string jit_decode_source(const DecodeArgs& a);
 void* jit_decode_kernel(const DecodeArgs& a);
 int jit_decode_launch(void* kernel, const DecodeArgs& a, const uint64_t* idx, const uint64_t* digits, int64_t n,
                       int32_t* out, int64_t ld, unsigned int* bad, void* stream);
-int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out,
+// out: int32 SoA, or int64 SoA when w64 (reading #22)
+int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, void* out, int w64,
                           int64_t ld, unsigned int* bad_flag, void* stream);
-int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out,
+int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, void* out, int w64,
                          int64_t ld, unsigned int* bad_flag, void* stream);
 int launch_decode128(const DecodeArgs& a, const uint64_t* idx_lo, const uint64_t* idx_hi, uint64_t first_lo,
-                     uint64_t first_hi, int64_t n, int32_t* out, int64_t ld, unsigned int* bad, uint64_t S_lo,
+                     uint64_t first_hi, int64_t n, void* out, int w64, int64_t ld, unsigned int* bad, uint64_t S_lo,
                      uint64_t S_hi, void* stream);
 int launch_scan_u32(const uint32_t* in, uint64_t* out, int64_t n, unsigned long long* status,
                     unsigned int* counter, void* stream, uint32_t* piece_tile = nullptr,

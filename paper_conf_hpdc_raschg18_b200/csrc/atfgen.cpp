@@ -45,7 +45,12 @@ enum State { BUILDING = 0, PLANNED = 1, GENERATED = 2, SHARDED = 3, FINAL_SHARD 
 
 struct ParamDef {
   std::string name;
-  std::vector<int32_t> values;                 // materialised range
+  // materialised range.  int32 parameter: the values.  int64 parameter (some value
+  // outside int32, reading #22): the range positions 0..r-1, the values in values64; the
+  // kernels map a position to its value through the int64 table (generic paths only).
+  std::vector<int32_t> values;
+  std::vector<int64_t> values64;
+  bool v64 = false;
   std::vector<std::vector<int32_t>> programs;  // ANDed constraints
   int64_t vmin = 0, vmax = 0;
 };
@@ -148,6 +153,7 @@ struct atf_space {
   // device state
   bool dev_ready = false;
   std::vector<int32_t*> d_range;
+  std::vector<const int64_t*> d_range64;  // int64 parameters' value tables (else null)
   std::vector<int32_t*> d_sorted;  // per parameter: [values sorted ascending][their positions] (encode)
   std::vector<std::vector<Chunk>> arena;  // per group
   std::vector<std::vector<LevelData>> data;
@@ -785,6 +791,8 @@ static atf_status compile_level(const std::vector<ParamDef>& P, int p, const std
       return false;
     };
     bool ok = a.n_gates == 0 && !lp.generic;
+    for (int r : lp.pv_param)
+      if (P[r].v64) ok = false;  // the fast paths read int32 value tables only
     for (int t = 0; ok && t < a.n_terms; t++) {
       const Term& T = a.terms[t];
       switch (T.kind) {
@@ -869,8 +877,9 @@ static atf_status plan(atf_space* s) {
       lp.field_shift = fs[l];
       lp.field_bits = fb[l];
       std::string why;
+      // an int64 parameter's own level is interpreted in int64 (reading #22)
       atf_status st = compile_level(s->params, p, g.members, (int)l, fw, fs, fb,
-                                    (s->opts.flags & ATF_FLAG_GENERIC_ONLY) != 0, lp, &why);
+                                    (s->opts.flags & ATF_FLAG_GENERIC_ONLY) != 0 || s->params[p].v64, lp, &why);
       if (st != ATF_OK) return fail(s, st, "parameter %s: %s", s->params[p].name.c_str(), why.c_str());
       lp.proto.level = (int)l;
       lp.proto.field_word = fw[l];
@@ -1037,6 +1046,15 @@ static atf_status ensure_device(atf_space* s) {
     off_sorted[p] = words;
     words += (2 * r + 3) / 4 * 4;
   }
+  // int64 parameters: their int64 value tables (8-byte aligned), reading #22
+  std::vector<size_t> off_range64(np, 0);
+  for (size_t p = 0; p < np; p++)
+    if (s->params[p].v64) {
+      words = (words + 3) / 4 * 4;
+      off_range64[p] = words;
+      words += 2 * s->params[p].values64.size();
+    }
+  words = (words + 3) / 4 * 4;
   // totals u64[kMaxGroups] | ovf[kMaxGroups] | tile counters[kMaxGroups] | bad[4] | root[16]:
   // one memset per level round resets [totals, ovf, counters], one copy reads [totals, ovf]
   const size_t off_scr = words;
@@ -1062,6 +1080,9 @@ static atf_status ensure_device(atf_space* s) {
       sb[r + j] = idx[j];
     }
   }
+  for (size_t p = 0; p < np; p++)
+    if (s->params[p].v64)
+      std::memcpy(host.data() + off_range64[p], s->params[p].values64.data(), 8 * s->params[p].values64.size());
   s->table_bytes = words * 4;
   s->d_table = (int32_t*)dalloc(s, s->table_bytes);
   if (!s->d_table) return fail(s, ATF_ERR_OOM, "parameter tables (%zu bytes)", s->table_bytes);
@@ -1070,9 +1091,11 @@ static atf_status ensure_device(atf_space* s) {
                               (cudaStream_t)s->opts.stream));
   s->d_range.assign(np, nullptr);
   s->d_sorted.assign(np, nullptr);
+  s->d_range64.assign(np, nullptr);
   for (size_t p = 0; p < np; p++) {
     s->d_range[p] = s->d_table + off_range[p];
     s->d_sorted[p] = s->d_table + off_sorted[p];
+    if (s->params[p].v64) s->d_range64[p] = reinterpret_cast<const int64_t*>(s->d_table + off_range64[p]);
   }
   int32_t* scr = s->d_table + off_scr;
   s->d_totals = (unsigned long long*)scr;
@@ -1169,6 +1192,7 @@ static void release_device(atf_space* s) {
   s->d_table = nullptr;
   s->table_bytes = 0;
   s->d_range.clear();
+  s->d_range64.clear();
   s->d_sorted.clear();
   dfree(s, s->d_status, s->status_cap * 8);
   dfree(s, (char*)s->d_replay, s->replay_cap * 12 * kMaxGroups);
@@ -1231,12 +1255,14 @@ struct Pending {
 // ancestor's value and magic table (see ensure_device: [values rp][magic rp][abs rp])
 static void fill_level_ptrs(atf_space* s, const LevelPlan& lp, LevelArgs& a) {
   a.cand = s->d_range[lp.param];
+  a.cand64 = s->d_range64[lp.param];  // int64 parameter: cand holds positions (reading #22)
   const size_t rp = ((size_t)lp.r + 127) / 128 * 128;
   a.cand_magic = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + rp;
   a.cand_abs = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + 2 * rp;
   a.r = lp.r;
   for (int i = 0; i < a.n_pv; i++) {
     a.pv_range[i] = s->d_range[lp.pv_param[i]];
+    a.pv_range64[i] = s->d_range64[lp.pv_param[i]];
     const size_t rpi = (s->params[lp.pv_param[i]].values.size() + 127) / 128 * 128;
     a.pv_magic[i] = reinterpret_cast<const uint32_t*>(s->d_range[lp.pv_param[i]]) + rpi;
   }
@@ -2781,6 +2807,7 @@ static atf_status make_decode_args(const atf_space* s, DecodeArgs& a) {
       a.lvl_shift[l] = (int16_t)lp.field_shift;
       a.lvl_bits[l] = (int16_t)lp.field_bits;
       a.lvl_range[l] = s->d_range[lp.param];
+      a.lvl_range64[l] = s->d_range64[lp.param];
       l++;
     }
   }
@@ -2860,7 +2887,8 @@ atf_status atf_space_add_param(atf_space* s, const char* name, const atf_range* 
     if (p.name == name) return fail(s, ATF_ERR_DUPLICATE, "duplicate parameter name %s (P:53: unique)", name);
   ParamDef pd;
   pd.name = name;
-  // P:57 ranges; readings #1-#3, #5
+  // P:57 ranges; readings #1-#3, #5, #22 (values materialised in int64)
+  std::vector<int64_t> vals;
   if (range->kind == ATF_RANGE_INTERVAL || range->kind == ATF_RANGE_POW2) {
     if (range->step <= 0) return fail(s, ATF_ERR_INVALID_ARG, "step must be positive");
     if (range->end >= range->begin) {
@@ -2869,11 +2897,10 @@ atf_status atf_space_add_param(atf_space* s, const char* name, const atf_range* 
     }
     for (i128 i = range->begin; i <= range->end; i += range->step) {
       if (range->kind == ATF_RANGE_INTERVAL) {
-        if (i < INT32_MIN || i > INT32_MAX) return fail(s, ATF_ERR_INVALID_ARG, "interval value outside int32");
-        pd.values.push_back((int32_t)i);
+        vals.push_back((int64_t)i);
       } else {
-        if (i < 0 || i > 30) return fail(s, ATF_ERR_INVALID_ARG, "pow2 exponent outside [0,30]");
-        pd.values.push_back((int32_t)(1u << (int)i));
+        if (i < 0 || i > 62) return fail(s, ATF_ERR_INVALID_ARG, "pow2 exponent outside [0,62]");
+        vals.push_back((int64_t)1 << (int)i);
       }
     }
   } else if (range->kind == ATF_RANGE_GEN) {
@@ -2944,29 +2971,38 @@ atf_status atf_space_add_param(atf_space* s, const char* name, const atf_range* 
       }
       if (bad || sp != 1) return fail(s, ATF_ERR_BYTECODE, "generator of %s: malformed program", name);
       if (poison) return fail(s, ATF_ERR_BYTECODE, "generator of %s: zero divisor at i = %lld", name, (long long)i);
-      if (st[0] < INT32_MIN || st[0] > INT32_MAX)
-        return fail(s, ATF_ERR_BYTECODE, "generator of %s: value outside int32 at i = %lld", name, (long long)i);
-      pd.values.push_back((int32_t)st[0]);
+      vals.push_back(st[0]);
     }
-    std::vector<int32_t> sorted(pd.values);
+    std::vector<int64_t> sorted(vals);
     std::sort(sorted.begin(), sorted.end());
     if (std::adjacent_find(sorted.begin(), sorted.end()) != sorted.end())
       return fail(s, ATF_ERR_DUPLICATE, "generator of %s repeats a value", name);
-  } else if (range->kind == ATF_RANGE_SET) {
-    if (range->n_values < 0 || (range->n_values > 0 && !range->values))
+  } else if (range->kind == ATF_RANGE_SET || range->kind == ATF_RANGE_SET64) {
+    const bool w = range->kind == ATF_RANGE_SET64;
+    if (range->n_values < 0 || (range->n_values > 0 && !(w ? (const void*)range->values64 : (const void*)range->values)))
       return fail(s, ATF_ERR_INVALID_ARG, "bad set");
     if (range->n_values > ATF_MAX_RANGE) return fail(s, ATF_ERR_LIMIT, "set larger than 2^24");
-    std::vector<int32_t> sorted(range->values, range->values + range->n_values);
+    for (int64_t j = 0; j < range->n_values; j++) vals.push_back(w ? range->values64[j] : (int64_t)range->values[j]);
+    std::vector<int64_t> sorted(vals);
     std::sort(sorted.begin(), sorted.end());
     if (std::adjacent_find(sorted.begin(), sorted.end()) != sorted.end())
       return fail(s, ATF_ERR_DUPLICATE, "duplicate value in set of %s", name);
-    pd.values.assign(range->values, range->values + range->n_values);
   } else {
     return fail(s, ATF_ERR_INVALID_ARG, "unknown range kind %d", range->kind);
   }
-  if (!pd.values.empty()) {
-    pd.vmin = *std::min_element(pd.values.begin(), pd.values.end());
-    pd.vmax = *std::max_element(pd.values.begin(), pd.values.end());
+  // int32 parameter: the values; int64 parameter: positions + the int64 table (reading #22)
+  for (int64_t v : vals)
+    if (v < INT32_MIN || v > INT32_MAX) pd.v64 = true;
+  if (pd.v64) {
+    pd.values64 = vals;
+    pd.values.resize(vals.size());
+    std::iota(pd.values.begin(), pd.values.end(), 0);
+  } else {
+    pd.values.assign(vals.begin(), vals.end());
+  }
+  if (!vals.empty()) {
+    pd.vmin = *std::min_element(vals.begin(), vals.end());
+    pd.vmax = *std::max_element(vals.begin(), vals.end());
   }
   s->params.push_back(std::move(pd));
   if (out_id) *out_id = (int32_t)s->params.size() - 1;
@@ -3139,11 +3175,19 @@ atf_status atf_space_level_view(const atf_space* s, int32_t g, int32_t k, atf_le
   return ATF_OK;
 }
 
+static bool space_v64(const atf_space* s) {
+  for (auto& p : s->params)
+    if (p.v64) return true;
+  return false;
+}
+
+// out: int32 SoA, or int64 SoA when w64 (reading #22; the int32 decoders refuse int64 spaces)
 static atf_status decode_common(const atf_space* cs, const uint64_t* idx, const uint64_t* digits, int64_t n,
-                                int32_t* out, int64_t ld, void* stream) {
+                                void* out, int64_t ld, void* stream, bool w64 = false) {
   atf_space* s = (atf_space*)cs;
   if (!s || (!idx && !digits) || !out || n < 0 || ld < n) return fail(s, ATF_ERR_INVALID_ARG, "bad decode arguments");
   if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "decode needs a generated (non-shard) space");
+  if (!w64 && space_v64(s)) return fail(s, ATF_ERR_OVERFLOW, "values outside int32: use the *_i64 decoders");
   if (idx) {
     u128 S = 1;
     for (uint64_t z : s->gsize) S *= z;
@@ -3156,7 +3200,7 @@ static atf_status decode_common(const atf_space* cs, const uint64_t* idx, const 
   make_decode_args(s, a);
   CUDA_TRY(s, cudaMemsetAsync(s->d_bad, 0, 4, st));
   // large batches: the decoder specialised for this space (NVRTC, compiled once per space)
-  if (n >= (1 << 18) && !(s->opts.flags & ATF_FLAG_NO_JIT) && !s->decode_jit_tried) {
+  if (!w64 && n >= (1 << 18) && !(s->opts.flags & ATF_FLAG_NO_JIT) && !s->decode_jit_tried) {
     s->decode_jit = jit_decode_kernel(a);
     s->decode_jit_tried = true;
   }
@@ -3167,10 +3211,10 @@ static atf_status decode_common(const atf_space* cs, const uint64_t* idx, const 
   if (big && cudaDeviceGetLimit(&gran, cudaLimitMaxL2FetchGranularity) == cudaSuccess && gran != 32)
     cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, 32);
   cudaGetLastError();
-  int ce = (big && s->decode_jit && !(s->opts.flags & ATF_FLAG_NO_JIT))
-               ? jit_decode_launch(s->decode_jit, a, idx, digits, n, out, ld, s->d_bad, st)
-               : (idx ? launch_decode_indices(a, idx, n, out, ld, s->d_bad, st)
-                      : launch_decode_digits(a, digits, n, out, ld, s->d_bad, st));
+  int ce = (!w64 && big && s->decode_jit && !(s->opts.flags & ATF_FLAG_NO_JIT))
+               ? jit_decode_launch(s->decode_jit, a, idx, digits, n, (int32_t*)out, ld, s->d_bad, st)
+               : (idx ? launch_decode_indices(a, idx, n, out, w64 ? 1 : 0, ld, s->d_bad, st)
+                      : launch_decode_digits(a, digits, n, out, w64 ? 1 : 0, ld, s->d_bad, st));
   if (big && gran && gran != 32) cudaDeviceSetLimit(cudaLimitMaxL2FetchGranularity, gran);
   cudaGetLastError();
   if (ce) return fail(s, ATF_ERR_CUDA, "decode launch: %s", cudaGetErrorString((cudaError_t)ce));
@@ -3179,7 +3223,8 @@ static atf_status decode_common(const atf_space* cs, const uint64_t* idx, const 
   // synchronise the stream here to report ATF_ERR_INDEX deterministically.
   CUDA_TRY(s, cudaMemcpyAsync(s->h_flags, s->d_bad, 4, cudaMemcpyDeviceToHost, st));
   CUDA_TRY(s, cudaStreamSynchronize(st));
-  if (s->h_flags[0]) return fail(s, ATF_ERR_INDEX, "index/digit out of range (rows set to INT32_MIN)");
+  if (s->h_flags[0])
+    return fail(s, ATF_ERR_INDEX, "index/digit out of range (rows set to %s)", w64 ? "INT64_MIN" : "INT32_MIN");
   return ATF_OK;
 }
 
@@ -3221,6 +3266,7 @@ static atf_status encode_common(const atf_space* cs, const int32_t* vals, int64_
   atf_space* s = (atf_space*)cs;
   if (!s || !vals || !digits || n < 0 || ld < n) return fail(s, ATF_ERR_INVALID_ARG, "bad encode arguments");
   if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "encode needs a generated (non-shard) space");
+  if (space_v64(s)) return fail(s, ATF_ERR_LIMIT, "encode takes int32 configurations (int64 space)");
   if (idx) {
     u128 S = 1;
     for (uint64_t z : s->gsize) S *= z;
@@ -3240,6 +3286,7 @@ atf_status atf_space_filter_product(atf_space* s, uint64_t* h_count, uint64_t* h
   if (!s || !h_count) return ATF_ERR_INVALID_ARG;
   atf_status e = plan(s);  // validation + static analysis (the product path needs no tree)
   if (e) return e;
+  if (space_v64(s)) return fail(s, ATF_ERR_LIMIT, "the full-product filter takes int32 values (int64 space)");
   {
     u128 prod = 1;
     for (auto& p : s->params) prod *= (u128)p.values.size();
@@ -3311,6 +3358,7 @@ atf_status atf_space_neighbors(const atf_space* cs, const int32_t* d_in, int64_t
   if (!s || !d_in || !d_out || !d_moved || n < 0 || ld_in < n || ld_out < n || max_tries < 0)
     return fail(s, ATF_ERR_INVALID_ARG, "bad neighbour arguments");
   if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "neighbours need a generated (non-shard) space");
+  if (space_v64(s)) return fail(s, ATF_ERR_LIMIT, "neighbours take int32 configurations (int64 space)");
   if (n == 0) return ATF_OK;
   EncodeArgs a;
   make_encode_args(s, a);
@@ -3339,10 +3387,11 @@ atf_status atf_space_decode_indices(const atf_space* s, const uint64_t* d_idx, i
 }
 
 static atf_status decode128_common(const atf_space* cs, const uint64_t* lo, const uint64_t* hi, uint64_t first_lo,
-                                   uint64_t first_hi, int64_t n, int32_t* out, int64_t ld, void* stream) {
+                                   uint64_t first_hi, int64_t n, void* out, int64_t ld, void* stream, bool w64 = false) {
   atf_space* s = (atf_space*)cs;
   if (!s || !out || n < 0 || ld < n) return fail(s, ATF_ERR_INVALID_ARG, "bad decode arguments");
   if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "decode needs a generated (non-shard) space");
+  if (!w64 && space_v64(s)) return fail(s, ATF_ERR_OVERFLOW, "values outside int32: use the *_i64 decoders");
   u128 S = 1;
   for (uint64_t z : s->gsize) {
     if (z && S > (~(u128)0) / z) return fail(s, ATF_ERR_OVERFLOW, "S >= 2^128");
@@ -3354,11 +3403,13 @@ static atf_status decode128_common(const atf_space* cs, const uint64_t* lo, cons
   DecodeArgs a;
   make_decode_args(s, a);
   CUDA_TRY(s, cudaMemsetAsync(s->d_bad, 0, 4, st));
-  int ce = launch_decode128(a, lo, hi, first_lo, first_hi, n, out, ld, s->d_bad, (uint64_t)S, (uint64_t)(S >> 64), st);
+  int ce = launch_decode128(a, lo, hi, first_lo, first_hi, n, out, w64 ? 1 : 0, ld, s->d_bad, (uint64_t)S,
+                            (uint64_t)(S >> 64), st);
   if (ce) return fail(s, ATF_ERR_CUDA, "decode launch: %s", cudaGetErrorString((cudaError_t)ce));
   CUDA_TRY(s, cudaMemcpyAsync(s->h_flags, s->d_bad, 4, cudaMemcpyDeviceToHost, st));
   CUDA_TRY(s, cudaStreamSynchronize(st));
-  if (s->h_flags[0]) return fail(s, ATF_ERR_INDEX, "index out of range (rows set to INT32_MIN)");
+  if (s->h_flags[0])
+    return fail(s, ATF_ERR_INDEX, "index out of range (rows set to %s)", w64 ? "INT64_MIN" : "INT32_MIN");
   return ATF_OK;
 }
 
@@ -3377,6 +3428,29 @@ atf_status atf_space_decode_digits(const atf_space* s, const uint64_t* d_digits,
                                    int64_t ld, void* stream) {
   if (!d_digits) return fail((atf_space*)s, ATF_ERR_INVALID_ARG, "null digits");
   return decode_common(s, nullptr, d_digits, n, d_out, ld, stream);
+}
+
+atf_status atf_space_decode_indices_i64(const atf_space* s, const uint64_t* d_idx, int64_t n, int64_t* d_out,
+                                        int64_t ld, void* stream) {
+  if (!d_idx) return fail((atf_space*)s, ATF_ERR_INVALID_ARG, "null indices");
+  return decode_common(s, d_idx, nullptr, n, d_out, ld, stream, true);
+}
+
+atf_status atf_space_decode_digits_i64(const atf_space* s, const uint64_t* d_digits, int64_t n, int64_t* d_out,
+                                       int64_t ld, void* stream) {
+  if (!d_digits) return fail((atf_space*)s, ATF_ERR_INVALID_ARG, "null digits");
+  return decode_common(s, nullptr, d_digits, n, d_out, ld, stream, true);
+}
+
+atf_status atf_space_decode_range_i64(const atf_space* s, uint64_t first_lo, uint64_t first_hi, int64_t n,
+                                      int64_t* d_out, int64_t ld, void* stream) {
+  return decode128_common(s, nullptr, nullptr, first_lo, first_hi, n, d_out, ld, stream, true);
+}
+
+atf_status atf_space_value_bits(const atf_space* s, int32_t* bits) {
+  if (!s || !bits) return ATF_ERR_INVALID_ARG;
+  *bits = space_v64(s) ? 64 : 32;
+  return ATF_OK;
 }
 
 atf_status atf_space_stats(const atf_space* s, atf_level_stats* out, int32_t cap, int32_t* n_out) {

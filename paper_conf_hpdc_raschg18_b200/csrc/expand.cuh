@@ -51,9 +51,10 @@ __device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, 
     case T_CMP:
       if (T.variant == V32) return rel_holds32(T.rel, (int32_t)A * x, (int32_t)Bv);
       return rel_holds(T.rel, A * (int64_t)x, Bv);
-    default: {  // T_GENERIC: interpret the conjunct
+    default: {  // T_GENERIC: interpret the conjunct (int64 parameter: x is the position, reading #22)
       bool poison = false;
-      const int64_t v = run_code(a.code + T.code_off, T.code_len, x, slots, stride, poison);
+      const int64_t xv = a.cand64 ? __ldg(a.cand64 + x) : (int64_t)x;
+      const int64_t v = run_code(a.code + T.code_off, T.code_len, xv, slots, stride, poison);
       return !poison && v != 0;
     }
   }
@@ -168,7 +169,7 @@ __device__ __forceinline__ bool prologue_node_impl(const LevelArgs& a, uint64_t 
       if (w == a.pv_word[s]) word = rec[w];
     const uint32_t bits = (uint32_t)a.pv_bits[s];
     const uint32_t pos = bits ? (word >> a.pv_shift[s]) & ((bits >= 32) ? 0xffffffffu : ((1u << bits) - 1u)) : 0u;
-    slots[s] = a.pv_range[s][pos];
+    slots[s] = a.pv_range64[s] ? a.pv_range64[s][pos] : (int64_t)a.pv_range[s][pos];
   }
   bool poison = false;
   for (int s = a.n_pv; s < a.n_slots; s++)

@@ -188,9 +188,24 @@ int launch_level_emit(const LevelArgs& a, int words, void* stream) {
 
 // ---------------------------------------------------------------- decode
 // index -> mixed-radix digits (group 0 most significant, P:229-231 reading #11) ->
-// per group: leaf record -> positions -> values; int32 SoA output.
+// per group: leaf record -> positions -> values; int32 SoA output, or int64 (OutT = int64_t,
+// reading #22: an int64 parameter's position indexes its int64 table lvl_range64).
+template <typename OutT>
+__device__ __forceinline__ OutT level_value(const DecodeArgs& a, int l, uint32_t pos) {
+  if constexpr (sizeof(OutT) == 8) {
+    if (a.lvl_range64[l]) return __ldg(a.lvl_range64[l] + pos);
+  }
+  return (OutT)__ldg(a.lvl_range[l] + pos);
+}
+template <typename OutT>
+__device__ __forceinline__ OutT bad_value() {
+  if constexpr (sizeof(OutT) == 8) return (OutT)INT64_MIN;
+  return (OutT)INT32_MIN;
+}
+
+template <typename OutT>
 __global__ void decode_kernel(const __grid_constant__ DecodeArgs a, const uint64_t* __restrict__ idx,
-                              const uint64_t* __restrict__ digits, int64_t n, int32_t* __restrict__ out,
+                              const uint64_t* __restrict__ digits, int64_t n, OutT* __restrict__ out,
                               int64_t ld, unsigned int* bad, uint64_t S, int s_fits) {
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     bool valid = true;
@@ -202,7 +217,7 @@ __global__ void decode_kernel(const __grid_constant__ DecodeArgs a, const uint64
       for (int g = 0; g < a.n_groups; g++) valid = valid && __ldg(digits + (int64_t)g * n + i) < a.gsize[g];
     }
     if (!valid) {
-      for (int p = 0; p < a.n_params; p++) out[(int64_t)p * ld + i] = INT32_MIN;
+      for (int p = 0; p < a.n_params; p++) out[(int64_t)p * ld + i] = bad_value<OutT>();
       atomicOr(bad, 1u);
       continue;
     }
@@ -247,14 +262,14 @@ __global__ void decode_kernel(const __grid_constant__ DecodeArgs a, const uint64
           if (lw == w) word = rec[w];
         const uint32_t bits = (uint32_t)a.lvl_bits[l];
         const uint32_t pos = bits ? (word >> a.lvl_shift[l]) & ((1u << bits) - 1u) : 0u;
-        out[(int64_t)a.lvl_param[l] * ld + i] = __ldg(a.lvl_range[l] + pos);
+        out[(int64_t)a.lvl_param[l] * ld + i] = level_value<OutT>(a, l, pos);
       }
     }
   }
 }
 
-static int launch_decode(const DecodeArgs& a, const uint64_t* idx, const uint64_t* digits, int64_t n, int32_t* out,
-                         int64_t ld, unsigned int* bad, void* stream) {
+static int launch_decode(const DecodeArgs& a, const uint64_t* idx, const uint64_t* digits, int64_t n, void* out,
+                         int w64, int64_t ld, unsigned int* bad, void* stream) {
   if (n <= 0) return 0;
   uint64_t S = 1;
   int fits = 1;
@@ -267,23 +282,29 @@ static int launch_decode(const DecodeArgs& a, const uint64_t* idx, const uint64_
   int64_t blocks = (n + 255) / 256;
   const int64_t cap = (int64_t)sms * 8;
   if (blocks > cap) blocks = cap;
-  decode_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, idx, digits, n, out, ld, bad, S, fits);
+  if (w64)
+    decode_kernel<int64_t><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, idx, digits, n, (int64_t*)out, ld,
+                                                                                bad, S, fits);
+  else
+    decode_kernel<int32_t><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, idx, digits, n, (int32_t*)out, ld,
+                                                                                bad, S, fits);
   return (int)cudaGetLastError();
 }
 
 // Indices beyond 2^64 (S >= 2^64, P:280 mentions spaces of ~10^19): u128 index = hi * 2^64 + lo,
 // either per row (idx_lo / idx_hi) or the consecutive range first + i (exhaustive search).
 // Mixed radix in u128 (group 0 most significant), then the same leaf gather as decode_kernel.
+template <typename OutT>
 __global__ void decode128_kernel(const __grid_constant__ DecodeArgs a, const uint64_t* __restrict__ idx_lo,
                                  const uint64_t* __restrict__ idx_hi, uint64_t first_lo, uint64_t first_hi, int64_t n,
-                                 int32_t* __restrict__ out, int64_t ld, unsigned int* bad, uint64_t S_lo, uint64_t S_hi) {
+                                 OutT* __restrict__ out, int64_t ld, unsigned int* bad, uint64_t S_lo, uint64_t S_hi) {
   typedef unsigned __int128 u128;
   const u128 S = ((u128)S_hi << 64) | S_lo;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
     u128 rem = idx_lo ? (((u128)__ldg(idx_hi + i) << 64) | __ldg(idx_lo + i))
                       : ((((u128)first_hi << 64) | first_lo) + (u128)i);
     if (rem >= S) {
-      for (int p = 0; p < a.n_params; p++) out[(int64_t)p * ld + i] = INT32_MIN;
+      for (int p = 0; p < a.n_params; p++) out[(int64_t)p * ld + i] = bad_value<OutT>();
       atomicOr(bad, 1u);
       continue;
     }
@@ -304,32 +325,36 @@ __global__ void decode128_kernel(const __grid_constant__ DecodeArgs a, const uin
           if (lw == w) word = rec[w];
         const uint32_t bits = (uint32_t)a.lvl_bits[l];
         const uint32_t pos = bits ? (word >> a.lvl_shift[l]) & ((1u << bits) - 1u) : 0u;
-        out[(int64_t)a.lvl_param[l] * ld + i] = __ldg(a.lvl_range[l] + pos);
+        out[(int64_t)a.lvl_param[l] * ld + i] = level_value<OutT>(a, l, pos);
       }
     }
   }
 }
 
 int launch_decode128(const DecodeArgs& a, const uint64_t* idx_lo, const uint64_t* idx_hi, uint64_t first_lo,
-                     uint64_t first_hi, int64_t n, int32_t* out, int64_t ld, unsigned int* bad, uint64_t S_lo,
+                     uint64_t first_hi, int64_t n, void* out, int w64, int64_t ld, unsigned int* bad, uint64_t S_lo,
                      uint64_t S_hi, void* stream) {
   if (n <= 0) return 0;
   const int sms = cached_sm_count();
   int64_t blocks = (n + 255) / 256;
   const int64_t cap = (int64_t)sms * 8;
   if (blocks > cap) blocks = cap;
-  decode128_kernel<<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(a, idx_lo, idx_hi, first_lo, first_hi, n, out,
-                                                                       ld, bad, S_lo, S_hi);
+  if (w64)
+    decode128_kernel<int64_t><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(
+        a, idx_lo, idx_hi, first_lo, first_hi, n, (int64_t*)out, ld, bad, S_lo, S_hi);
+  else
+    decode128_kernel<int32_t><<<(unsigned)blocks, 256, 0, (cudaStream_t)stream>>>(
+        a, idx_lo, idx_hi, first_lo, first_hi, n, (int32_t*)out, ld, bad, S_lo, S_hi);
   return (int)cudaGetLastError();
 }
 
-int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, int32_t* out, int64_t ld,
+int launch_decode_indices(const DecodeArgs& a, const uint64_t* idx, int64_t n, void* out, int w64, int64_t ld,
                           unsigned int* bad, void* stream) {
-  return launch_decode(a, idx, nullptr, n, out, ld, bad, stream);
+  return launch_decode(a, idx, nullptr, n, out, w64, ld, bad, stream);
 }
-int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, int32_t* out, int64_t ld,
+int launch_decode_digits(const DecodeArgs& a, const uint64_t* digits, int64_t n, void* out, int w64, int64_t ld,
                          unsigned int* bad, void* stream) {
-  return launch_decode(a, nullptr, digits, n, out, ld, bad, stream);
+  return launch_decode(a, nullptr, digits, n, out, w64, ld, bad, stream);
 }
 
 // ---------------------------------------------------------------- encode

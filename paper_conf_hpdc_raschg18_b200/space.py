@@ -24,8 +24,12 @@ def _range_struct(rng: dict):
         return L.atf_range(L.ATF_RANGE_GEN, rng["begin"], rng["end"], rng.get("step", 1),
                            C.cast(code, C.POINTER(C.c_int32)), len(rng["code"])), code
     if kind == "set":
-        vals = (C.c_int32 * max(1, len(rng["values"])))(*rng["values"])
-        return L.atf_range(L.ATF_RANGE_SET, 0, 0, 0, C.cast(vals, C.POINTER(C.c_int32)), len(rng["values"])), vals
+        v = [int(x) for x in rng["values"]]
+        if any(x < -2 ** 31 or x >= 2 ** 31 for x in v):  # int64 values (reading #22)
+            vals = (C.c_int64 * max(1, len(v)))(*v)
+            return L.atf_range(L.ATF_RANGE_SET64, 0, 0, 0, None, len(v), C.cast(vals, C.POINTER(C.c_int64))), vals
+        vals = (C.c_int32 * max(1, len(v)))(*v)
+        return L.atf_range(L.ATF_RANGE_SET, 0, 0, 0, C.cast(vals, C.POINTER(C.c_int32)), len(v)), vals
     raise ValueError(f"unknown range kind {kind}")
 
 
@@ -224,27 +228,37 @@ class Space:
         return [{f: getattr(arr[i], f) for f, _ in L.atf_level_stats._fields_} for i in range(n.value)]
 
     # ---- decode (device tensors in, device tensor out)
-    def decode(self, idx, out=None, stream=None):
-        """idx: CUDA tensor of uint64/int64 indices [n] -> int32 tensor [P, n] (SoA)."""
+    def value_bits(self) -> int:
+        """32 if every parameter value fits int32, else 64 (configurations are then int64)."""
+        b = C.c_int32()
+        L.check(L.atf_space_value_bits(self._h, C.byref(b)), self._h)
+        return b.value
+
+    def _out(self, out, P, n, device):
         import torch
+        if out is not None:
+            return out, out.dtype == torch.int64
+        w64 = self.value_bits() == 64
+        return torch.empty((P, n), dtype=torch.int64 if w64 else torch.int32, device=device), w64
+
+    def decode(self, idx, out=None, stream=None):
+        """idx: CUDA tensor of uint64/int64 indices [n] -> int32 tensor [P, n] (SoA); int64 for a
+        space with values outside int32 (or when `out` is int64)."""
         n = idx.numel()
-        P = len(self.names)
-        if out is None:
-            out = torch.empty((P, n), dtype=torch.int32, device=idx.device)
+        out, w64 = self._out(out, len(self.names), n, idx.device)
         sp = stream.cuda_stream if stream is not None else None
-        L.check(L.atf_space_decode_indices(self._h, idx.data_ptr(), n, out.data_ptr(), out.stride(0), sp), self._h)
+        fn = L.atf_space_decode_indices_i64 if w64 else L.atf_space_decode_indices
+        L.check(fn(self._h, idx.data_ptr(), n, out.data_ptr(), out.stride(0), sp), self._h)
         return out
 
     def decode_range(self, first: int, n: int, out=None, stream=None):
         """The n consecutive indices first, first + 1, ... (any S, u128 in the library) ->
-        int32 tensor [P, n]."""
+        int32 tensor [P, n] (int64 as for decode)."""
         import torch
-        P = len(self.names)
-        if out is None:
-            out = torch.empty((P, n), dtype=torch.int32, device=torch.device("cuda", self._device))
+        out, w64 = self._out(out, len(self.names), n, torch.device("cuda", self._device))
         sp = stream.cuda_stream if stream is not None else None
-        L.check(L.atf_space_decode_range(self._h, first & ((1 << 64) - 1), first >> 64, n, out.data_ptr(),
-                                         out.stride(0), sp), self._h)
+        fn = L.atf_space_decode_range_i64 if w64 else L.atf_space_decode_range
+        L.check(fn(self._h, first & ((1 << 64) - 1), first >> 64, n, out.data_ptr(), out.stride(0), sp), self._h)
         return out
 
     def decode128(self, idx_lo, idx_hi, out=None, stream=None):
@@ -261,15 +275,14 @@ class Space:
         return out
 
     def decode_digits(self, digits, out=None, stream=None):
-        """digits: CUDA tensor [G, n] of per-group indices -> int32 tensor [P, n]."""
-        import torch
+        """digits: CUDA tensor [G, n] of per-group indices -> int32 tensor [P, n] (int64 as for
+        decode)."""
         n = digits.shape[1]
-        P = len(self.names)
-        if out is None:
-            out = torch.empty((P, n), dtype=torch.int32, device=digits.device)
+        out, w64 = self._out(out, len(self.names), n, digits.device)
         digits = digits.contiguous()
         sp = stream.cuda_stream if stream is not None else None
-        L.check(L.atf_space_decode_digits(self._h, digits.data_ptr(), n, out.data_ptr(), out.stride(0), sp), self._h)
+        fn = L.atf_space_decode_digits_i64 if w64 else L.atf_space_decode_digits
+        L.check(fn(self._h, digits.data_ptr(), n, out.data_ptr(), out.stride(0), sp), self._h)
         return out
 
     # ---- encode (inverse of decode; membership)

@@ -126,7 +126,7 @@ def test_validation_errors():
     assert _err(lambda: sp.add_param("a", interval(1, 2))) == -9                    # duplicate name
     assert _err(lambda: sp.add_param("s", set_(1, 2, 2))) == -9                      # duplicate set value
     assert _err(lambda: sp.add_param("t", {"kind": "interval", "begin": 1, "end": 4, "step": 0})) == -1
-    assert _err(lambda: sp.add_param("u", {"kind": "pow2", "begin": 0, "end": 31, "step": 1})) == -1
+    assert _err(lambda: sp.add_param("u", {"kind": "pow2", "begin": 0, "end": 63, "step": 1})) == -1  # 2^63 > int64
     assert _err(lambda: sp.add_constraint(a, P(1).code + [1, 17])) == -6           # forward reference
     assert _err(lambda: sp.add_constraint(b, [1, 17])) == -5                         # stack underflow
     assert _err(lambda: sp.add_constraint(b, [1, 1])) == -5                          # two results
@@ -208,7 +208,8 @@ def test_generator_range_abi_validation(L):
     assert add(A.gen(-2, 2, A.X * A.X)["code"], -2, 2) == -9           # duplicate
     assert add(A.gen(0, 3, A.C(12) // A.X)["code"], 0, 3) == -5         # 12 / 0: poison
     assert add([2, 0], 0, 3) == -5                                       # PARAM 0
-    assert add(A.gen(0, 3, A.X * A.C(1 << 40))["code"], 0, 3) == -5     # > int32
+    assert add(A.gen(0, 3, A.X * A.C(1 << 40))["code"], 0, 3) == 0      # int64 values (reading #22)
+    assert add(A.gen(0, 3, A.X * A.C(1 << 62))["code"], 0, 3) == -7     # > int64: overflow
 
 
 def test_jit_level_sources_compile_for_sm100a(L, tmp_path):

@@ -292,3 +292,170 @@ def test_overflow_int64_values(oracle_bin):
     """Exact int64 arithmetic (reading #9): 2^62 * x overflows for x = 2^62."""
     s = Spec("ovf64"); s.add("x", set_(2 ** 62, 3), (X * X) > 0)
     assert orc.info(s)["overflow"] is True
+
+
+# ---------------------------------------------------------------- library host side (CPU)
+def _lib_space(spec, **kw):
+    from paper_conf_hpdc_raschg18_b200 import Space
+    return Space(spec, torch_alloc=False, **kw)
+
+
+def _status(fn):
+    from paper_conf_hpdc_raschg18_b200 import AtfError
+    with pytest.raises(AtfError) as e:
+        fn()
+    return e.value.status
+
+
+def test_library_value_bits_and_generic_levels():
+    """An int64 parameter's own level is compiled to generic (interpreted, int64) terms; the
+    int32 group of the same space keeps its divisibility atoms (plan_json kinds: 2 = x | n,
+    6 = generic)."""
+    assert _lib_space(A.c1_toy()).value_bits() == 32
+    sp = _lib_space(mixed_groups64())
+    assert sp.value_bits() == 64
+    sp.plan()
+    pj = sp.plan_json()
+    g0, g1 = pj["groups"]
+    assert all(t["kind"] == 6 for t in g0["levels"][0]["terms"] + g0["levels"][2]["terms"])
+    assert [t["kind"] for t in g1["levels"][1]["terms"]] == [2]
+    assert _lib_space(pow2_pairs(30)).value_bits() == 32
+
+
+def test_library_int64_range_validation():
+    from paper_conf_hpdc_raschg18_b200 import Space
+    sp = Space(None, torch_alloc=False)
+    sp.add_param("a", pow2(0, 62))
+    assert _status(lambda: sp.add_param("b", pow2(0, 63))) == -1                 # 2^63 outside int64
+    assert _status(lambda: sp.add_param("c", set_(2 ** 40, 5, 2 ** 40))) == -9   # duplicate (reading #5)
+    sp.add_param("d", interval(2 ** 62, 2 ** 62 + 10))
+    sp.add_param("e", A.gen(0, 3, X * (2 ** 40)))
+    sp.add_param("f", set_(-(2 ** 63), 2 ** 63 - 1))
+    assert sp.value_bits() == 64
+    s = Spec("ovf64"); s.add("x", set_(2 ** 62, 3), (X * X) > 0)
+    assert _status(_lib_space(s).plan) == -7   # static analysis: int64 overflow (reading #9)
+
+
+def test_library_int32_entry_points_refuse_int64_spaces():
+    sp = _lib_space(mixed_groups64())
+    assert _status(sp.filter_product) == -10
+
+
+# ---------------------------------------------------------------- GPU parity (-m gpu)
+def wide64(n_x=5000, n_y=300):
+    """An int64 level with r > 64 over a frontier of several warp tiles with a ragged tail
+    (the warp-tile kernel's dense path), and an int32 level reading an int64 ancestor
+    (64-bit atoms, generic kernels): y_j = j * 2^33 (j = 1..n_y), y / 2^33 a multiple of x;
+    z | y / 2^33 with z in 1..96."""
+    s = Spec(f"wide64_{n_x}x{n_y}")
+    s.add("x", interval(1, n_x))
+    s.add("y", set_(*[j * 2 ** 33 for j in range(1, n_y + 1)]), A.is_multiple_of(P(0) * 2 ** 33))
+    s.add("z", interval(1, 96), divides(P(1) // 2 ** 33))
+    return s
+
+
+GPU_SPECS = {
+    "saxpy64": saxpy64, "pow2pairs": pow2_pairs, "ivmul64": interval_multiples,
+    "ivmul64neg": lambda: interval_multiples(-(2 ** 35) - 3), "ivmul64top": lambda: interval_multiples(2 ** 62 - 500),
+    "edge64": edge_order, "prod64": lambda: products64()[0], "mixed64": mixed_groups64, "wide64": wide64,
+}
+
+
+@pytest.fixture(scope="module")
+def GSpace():
+    torch = pytest.importorskip("torch")
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_hpdc_raschg18_b200 import Space as S
+    return S
+
+
+def _gpu_check(Space, spec, flags=0, regenerate=False):
+    import torch
+    ref = orc.info(spec, threads=8)
+    with Space(spec, flags=flags) as sp:
+        sp.generate()
+        if regenerate:          # replay, then the CUDA graph capture and its launch
+            for _ in range(3):
+                sp.generate()
+        assert sp.value_bits() == 64
+        assert sp.groups() == [g["members"] for g in ref["groups"]]
+        assert sp.size() == int(ref["S"])
+        for g, grp in enumerate(ref["groups"]):
+            assert sp.level_sizes(g) == [lv["f"] for lv in grp["levels"]], (spec.name, g)
+        S = sp.size()
+        if S == 0:
+            return
+        idx = torch.arange(S, dtype=torch.int64, device="cuda")
+        got = sp.decode(idx)
+        assert got.dtype == torch.int64
+        _, want = orc.decode(spec, np.arange(S, dtype=np.uint64))
+        assert np.array_equal(got.cpu().numpy(), want), spec.name
+        # decode_range (u128 path) over a window and decode_digits of group 0's leaves
+        n = min(S, 4096)
+        first = S - n
+        assert np.array_equal(sp.decode_range(first, n).cpu().numpy(), want[:, first:])
+        G = sp.num_groups()
+        sz0 = sp.group_sizes()[0]
+        dig = torch.zeros((G, sz0), dtype=torch.int64, device="cuda")
+        dig[0] = torch.arange(sz0, dtype=torch.int64, device="cuda")
+        lv = sp.decode_digits(dig)[ref["groups"][0]["members"]].T.cpu().numpy()
+        assert np.array_equal(lv, orc.leaves(spec, 0, len(ref["groups"][0]["members"])))
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("name", sorted(GPU_SPECS))
+def test_gpu_int64_named(GSpace, name):
+    _gpu_check(GSpace, GPU_SPECS[name]())
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("seed", range(12))
+def test_gpu_int64_fuzz(GSpace, seed):
+    spec = fuzz64(seed)
+    if not orc.width(spec):
+        pytest.skip("draw without int64 values")
+    _gpu_check(GSpace, spec)
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("variant", ["legacy_wide", "no_replay_regen", "regen", "no_seg_bounds"])
+def test_gpu_int64_flags(GSpace, variant):
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    flags = {"legacy_wide": L.ATF_FLAG_LEGACY_WIDE, "no_replay_regen": L.ATF_FLAG_NO_REPLAY,
+             "regen": 0, "no_seg_bounds": L.ATF_FLAG_NO_SEG_BOUNDS}[variant]
+    for spec in (wide64(), mixed_groups64()):
+        _gpu_check(GSpace, spec, flags=flags, regenerate=variant.endswith("regen"))
+
+
+@pytest.mark.gpu
+def test_gpu_int64_errors(GSpace):
+    """The int32 decoders and encode refuse an int64 space (ATF_ERR_OVERFLOW / ATF_ERR_LIMIT);
+    out-of-range indices give INT64_MIN rows and ATF_ERR_INDEX; the int64 decoders sign-extend
+    an int32 space's values."""
+    import torch
+    from paper_conf_hpdc_raschg18_b200 import AtfError
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    spec = mixed_groups64()
+    with GSpace(spec) as sp:
+        sp.generate()
+        S = sp.size()
+        idx = torch.tensor([0, S, S - 1], dtype=torch.int64, device="cuda")
+        with pytest.raises(AtfError) as e:
+            sp.decode(idx, out=torch.empty((5, 3), dtype=torch.int32, device="cuda"))
+        assert e.value.status == -7
+        out = torch.empty((5, 3), dtype=torch.int64, device="cuda")
+        with pytest.raises(AtfError) as e:
+            sp.decode(idx, out=out)
+        assert e.value.status == -8
+        assert (out[:, 1] == -(2 ** 63)).all()
+        with pytest.raises(AtfError) as e:
+            sp.encode(torch.zeros((5, 2), dtype=torch.int32, device="cuda"))
+        assert e.value.status == -10
+    c1 = A.c1_toy()
+    with GSpace(c1) as sp:
+        sp.generate()
+        idx = torch.arange(sp.size(), dtype=torch.int64, device="cuda")
+        a = sp.decode(idx)
+        b = sp.decode(idx, out=torch.empty((2, sp.size()), dtype=torch.int64, device="cuda"))
+        assert a.dtype == torch.int32 and torch.equal(a.to(torch.int64), b)
