@@ -60,8 +60,7 @@ struct LevelArgs {
   const uint32_t* parent_rec;
   uint64_t n_parents;
   // candidates = materialised range of the level's parameter
-  const int32_t* cand;         // int64 parameter (reading #22): the positions 0..r-1
-  const int64_t* cand64;       // int64 parameter: its values (else null); generic terms only
+  const int32_t* cand;         // int64 parameter (reading #22): the positions 0..r-1 (cand64 below)
   const uint32_t* cand_magic;  // ceil(2^32/|x|) mod 2^32 per candidate (2^16 for x == 0), host-computed
   const uint32_t* cand_abs;    // |x| per candidate; both padded to a multiple of 128
   int32_t r;
@@ -70,8 +69,7 @@ struct LevelArgs {
   // slots [0, n_pv): values of ancestor levels, decoded from the parent record
   int32_t n_pv;
   int32_t pv_word[kMaxSlots], pv_shift[kMaxSlots], pv_bits[kMaxSlots];
-  const int32_t* pv_range[kMaxSlots];
-  const int64_t* pv_range64[kMaxSlots];  // int64 ancestors: their value tables (else null)
+  const int32_t* pv_range[kMaxSlots];  // int64 ancestors: pv_range64 below
   // slots [n_pv, n_slots): hoisted node-invariant expressions (code[inv_off..+inv_len))
   int32_t n_slots;
   int16_t inv_off[kMaxSlots], inv_len[kMaxSlots];
@@ -127,6 +125,13 @@ struct LevelArgs {
   uint64_t n_tiles;
   uint32_t qmax;            // T_QDIV table covers quotients [0, qmax]
   int32_t smem_bytes;
+  // int64 parameters (reading #22), at the end so the int32 kernels' parameter layout is unchanged:
+  // the level's own values (its cand holds positions; generic terms only) and the referenced
+  // int64 ancestors' value tables (else null).  pv64_any: some pv_range64 is set (no hot filter,
+  // the generic prologue).
+  const int64_t* cand64;
+  const int64_t* pv_range64[kMaxSlots];
+  int32_t pv64_any;
 };
 enum KernelKind : int32_t { K_NARROW = 0, K_WIDE = 1, K_WTILE = 2, K_NFAST = 3 };
 

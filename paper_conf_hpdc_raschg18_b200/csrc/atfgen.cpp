@@ -921,7 +921,8 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide, bool seg_
       if (cost < best - 1e-9) { best = cost; best_cpt = cpt; best_nseg = (int)nseg; }
     }
     if (best_cpt) {
-      for (int t = 0; t < a.n_terms; t++) {
+      // (levels reading an int64 ancestor take the generic prologue: no hot filter, reading #22)
+      for (int t = 0; t < a.n_terms && !a.pv64_any; t++) {
         const Term& T = a.terms[t];
         if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) { a.hot = HOT_DIVX; a.hot_term = t; break; }
         if (T.kind == T_MULX && T.variant == V16) { a.hot = HOT_MULX; a.hot_term = t; break; }
@@ -976,7 +977,7 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide, bool seg_
     a.chunk = r;
   } else {
     a.kind = K_WIDE;
-    for (int t = 0; t < a.n_terms; t++) {
+    for (int t = 0; t < a.n_terms && !a.pv64_any; t++) {
       const Term& T = a.terms[t];
       if ((T.kind == T_DIVX || T.kind == T_DIVPROD) && T.variant == V16) { a.hot = HOT_DIVX; a.hot_term = t; break; }
       if (T.kind == T_MULX && T.variant == V16) { a.hot = HOT_MULX; a.hot_term = t; break; }
@@ -1260,9 +1261,11 @@ static void fill_level_ptrs(atf_space* s, const LevelPlan& lp, LevelArgs& a) {
   a.cand_magic = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + rp;
   a.cand_abs = reinterpret_cast<const uint32_t*>(s->d_range[lp.param]) + 2 * rp;
   a.r = lp.r;
+  a.pv64_any = 0;
   for (int i = 0; i < a.n_pv; i++) {
     a.pv_range[i] = s->d_range[lp.pv_param[i]];
     a.pv_range64[i] = s->d_range64[lp.pv_param[i]];
+    if (a.pv_range64[i]) a.pv64_any = 1;
     const size_t rpi = (s->params[lp.pv_param[i]].values.size() + 127) / 128 * 128;
     a.pv_magic[i] = reinterpret_cast<const uint32_t*>(s->d_range[lp.pv_param[i]]) + rpi;
   }

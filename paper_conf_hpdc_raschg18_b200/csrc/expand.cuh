@@ -12,6 +12,10 @@ namespace atf {
 // planner's atoms are exact rewrites of the bytecode).  A, Bv: the
 // node's operands of T (prologue); x: candidate value, ax = |x|, m32 = ceil(2^32/ax)
 // (0 for ax <= 1).  slots/stride: the node's slot column (generic terms only).
+// X64: the level may be an int64 parameter's (reading #22): a generic term maps the candidate
+// position x to its int64 value.  Hot-filter levels never are (their callers pass false and keep
+// the code of the int32 path).
+template <bool X64>
 __device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, int64_t A, int64_t Bv, int32_t x,
                                              uint32_t ax, uint32_t m32, const uint32_t* s_q, const int64_t* slots,
                                              int stride) {
@@ -53,7 +57,7 @@ __device__ __forceinline__ bool term_accepts(const LevelArgs& a, const Term& T, 
       return rel_holds(T.rel, A * (int64_t)x, Bv);
     default: {  // T_GENERIC: interpret the conjunct (int64 parameter: x is the position, reading #22)
       bool poison = false;
-      const int64_t xv = a.cand64 ? __ldg(a.cand64 + x) : (int64_t)x;
+      const int64_t xv = (X64 && a.cand64) ? __ldg(a.cand64 + x) : (int64_t)x;
       const int64_t v = run_code(a.code + T.code_off, T.code_len, xv, slots, stride, poison);
       return !poison && v != 0;
     }
@@ -94,7 +98,7 @@ __device__ __forceinline__ uint64_t term_mask_narrow(const LevelArgs& a, const T
     mm &= mm - 1;
     const int32_t x = s_cx[c];
     const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-    if (term_accepts(a, T, A, Bv, x, ax, s_cm[c], s_q, slots, stride)) out |= 1ull << c;
+    if (term_accepts<true>(a, T, A, Bv, x, ax, s_cm[c], s_q, slots, stride)) out |= 1ull << c;
   }
   return out;
 }
@@ -106,7 +110,7 @@ static __device__ __noinline__ bool node_accepts(const LevelArgs& a, int i, int 
   if (!s_ok[i]) return false;
   const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
   for (int t = 0; t < a.n_terms; t++)
-    if (!term_accepts(a, a.terms[t], s_opa[t * tn + i], s_opb[t * tn + i], x, ax, m32, s_q,
+    if (!term_accepts<true>(a, a.terms[t], s_opa[t * tn + i], s_opb[t * tn + i], x, ax, m32, s_q,
                       s_slots ? s_slots + i : nullptr, tn))
       return false;
   return true;
@@ -146,7 +150,8 @@ __device__ __forceinline__ void load_record(const uint32_t* src, uint32_t* rec) 
 // Per-node prologue: unpack ancestor values from the parent's path record, evaluate the
 // hoisted node-invariant expressions, the node gates and every conjunct's operands into
 // shared memory (node `i` of the tile, global index gnode).  Returns the gate result.
-template <int W>
+// X64: int64 ancestors possible (reading #22; never on hot-filter levels, see choose_geometry).
+template <int W, bool X64 = true>
 __device__ __forceinline__ bool prologue_node_impl(const LevelArgs& a, uint64_t gnode, int i, int tn, uint32_t* s_ok, uint32_t* s_rec,
                               int64_t* s_opa, int64_t* s_opb, int64_t* s_slots, bool rec_staged = false) {
   uint32_t rec[W];
@@ -169,7 +174,7 @@ __device__ __forceinline__ bool prologue_node_impl(const LevelArgs& a, uint64_t 
       if (w == a.pv_word[s]) word = rec[w];
     const uint32_t bits = (uint32_t)a.pv_bits[s];
     const uint32_t pos = bits ? (word >> a.pv_shift[s]) & ((bits >= 32) ? 0xffffffffu : ((1u << bits) - 1u)) : 0u;
-    slots[s] = a.pv_range64[s] ? a.pv_range64[s][pos] : (int64_t)a.pv_range[s][pos];
+    slots[s] = (X64 && a.pv_range64[s]) ? a.pv_range64[s][pos] : (int64_t)a.pv_range[s][pos];
   }
   bool poison = false;
   for (int s = a.n_pv; s < a.n_slots; s++)
@@ -210,11 +215,11 @@ __device__ __forceinline__ bool prologue_node_impl(const LevelArgs& a, uint64_t 
 }
 
 // Out-of-line copy for the wide kernel (keeps the hot loop's registers free).
-template <int W>
+template <int W, bool X64>
 __device__ __noinline__ bool prologue_node(const LevelArgs& a, uint64_t gnode, int i, int tn, uint32_t* s_ok,
                                            uint32_t* s_rec, int64_t* s_opa, int64_t* s_opb, int64_t* s_slots,
                                            bool rec_staged) {
-  return prologue_node_impl<W>(a, gnode, i, tn, s_ok, s_rec, s_opa, s_opb, s_slots, rec_staged);
+  return prologue_node_impl<W, X64>(a, gnode, i, tn, s_ok, s_rec, s_opa, s_opb, s_slots, rec_staged);
 }
 
 // Block-wide exclusive scan of one u32 per thread (B <= 1024); returns the exclusive
@@ -389,7 +394,8 @@ static __device__ __noinline__ uint32_t other_terms_mask(const LevelArgs& a, int
       m &= m - 1;
       const int32_t x = __ldg(a.cand + jg0 + c);
       const uint32_t ax = x < 0 ? 0u - (uint32_t)x : (uint32_t)x;
-      if (!term_accepts(a, T, A, Bv, x, ax, __ldg(a.cand_magic + jg0 + c), s_q, s_slots ? s_slots + i : nullptr, tn))
+      if (!term_accepts<false>(a, T, A, Bv, x, ax, __ldg(a.cand_magic + jg0 + c), s_q, s_slots ? s_slots + i : nullptr,
+                               tn))
         mask &= ~(1u << c);
     }
   }
@@ -557,7 +563,7 @@ __global__ void __launch_bounds__(256, 4) expand_wide(const __grid_constant__ Le
 #pragma unroll
           for (int w = 0; w < W; w++) s_rec[i * W + w] = pre[w];
         }
-        const bool ok = prologue_node<W>(a, node0 + i, i, NT, s_ok, s_rec, s_opa, s_opb, s_slots, staged);
+        const bool ok = prologue_node<W, HOT == HOT_NONE>(a, node0 + i, i, NT, s_ok, s_rec, s_opa, s_opb, s_slots, staged);
         if (HOT == HOT_DIVX) {
           s_hot[i] = ok ? (uint32_t)s_opa[hot_t * NT + i] : kHotSentinel;
         } else if (HOT == HOT_MULX) {
@@ -894,7 +900,7 @@ __global__ void __launch_bounds__(256, 3) expand_wtile(const __grid_constant__ L
 #pragma unroll
         for (int w = 0; w < W; w++) s_rec[lane * W + w] = pre[w];
       }
-      ok = prologue_node<W>(a, node0 + lane, lane, kWT, s_ok, s_rec, s_opa, s_opb, s_slots, staged);
+      ok = prologue_node<W, HOT == HOT_NONE>(a, node0 + lane, lane, kWT, s_ok, s_rec, s_opa, s_opb, s_slots, staged);
     } else {
       s_ok[lane] = 0u;
     }
