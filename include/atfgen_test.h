@@ -45,6 +45,9 @@ atf_status atf_test_set_tail_stage(int32_t bytes);
  * warp tiles per SM below which the warp-tile kernel halves its nodes per tile (256), and
  * log2 of the candidate-pair count below which generate_dist replicates a level (28). */
 atf_status atf_test_set_geometry(int32_t tiles_per_sm, int32_t repl_log2);
+/* Warp-tile levels of at most n tiles are written in place behind a decoupled look-back (one
+ * launch, no scan / copy kernels); 0 restores the default 16.  Tuning experiments. */
+atf_status atf_test_set_direct_tiles(int32_t n);
 #ifdef __cplusplus
 }
 #endif

@@ -900,6 +900,7 @@ static atf_status plan(atf_space* s) {
 // replicates a level instead of distributing it.
 static std::atomic<int> g_tiles_per_sm{256};
 static std::atomic<int> g_repl_log2{28};
+static std::atomic<int> g_direct_tiles{16};  // in-place (look-back) levels: at most this many warp tiles
 
 static void choose_geometry(LevelArgs& a, int words, bool legacy_wide, bool seg_bounds = true) {
   const int r = a.r;
@@ -1338,7 +1339,8 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   // tiny wide levels: one launch, in place (decoupled look-back over <= 16 warp tiles; with
   // more tiles the waits cost more than the two saved launches: DESIGN.md §5).  Otherwise
   // children go to per-tile stash segments and scan_kernel + level_emit_kernel place them.
-  a.direct = (a.kind == K_WTILE && !wide_jit && !(s->opts.flags & ATF_FLAG_LEGACY_WIDE) && a.n_tiles <= 16) ? 1 : 0;
+  a.direct = (a.kind == K_WTILE && !wide_jit && !(s->opts.flags & ATF_FLAG_LEGACY_WIDE) &&
+              a.n_tiles <= (uint64_t)g_direct_tiles.load()) ? 1 : 0;
   if (a.kind == K_WTILE) a.smem_bytes = wtile_layout(a, gp.words).total;
   if (a.smem_bytes > 227 * 1024)
     return fail(s, ATF_ERR_LIMIT, "level %d of group %d needs %d bytes of shared memory", k, g, a.smem_bytes);
@@ -3709,6 +3711,12 @@ atf_status atf_test_set_geometry(int32_t tiles_per_sm, int32_t repl_log2) {
   if (tiles_per_sm < 0 || tiles_per_sm > 4096 || repl_log2 < 0 || repl_log2 > 62) return ATF_ERR_INVALID_ARG;
   g_tiles_per_sm.store(tiles_per_sm ? tiles_per_sm : 256);
   g_repl_log2.store(repl_log2 ? repl_log2 : 28);
+  return ATF_OK;
+}
+
+atf_status atf_test_set_direct_tiles(int32_t n) {
+  if (n < 0 || n > (1 << 20)) return ATF_ERR_INVALID_ARG;
+  g_direct_tiles.store(n ? n : 16);
   return ATF_OK;
 }
 
