@@ -32,6 +32,17 @@ for spec in SPECS:
             back = sp.encode_digits(rows)
             assert torch.equal(back, dig), spec.name
             print(spec.name, fl, sp.size(), flush=True)
+# int64-valued parameters (reading #22): generic kernels over int64 value tables, int64 decode
+sys.path.insert(0, os.path.join(ROOT, "tests"))
+from test_int64_values import mixed_groups64, wide64  # noqa: E402
+for spec in (wide64(600, 120), mixed_groups64()):
+    with Space(spec) as sp:
+        sp.generate()
+        sp.generate()
+        S = sp.size()
+        out = sp.decode(torch.arange(min(S, 8192), dtype=torch.int64, device="cuda"))
+        assert out.dtype == torch.int64
+        print(spec.name, S, flush=True)
 torch.cuda.synchronize()
 # balanced multi-GPU generation: two virtual ranks on their own streams, three generations
 # (synchronous, log-sized, replay with device round flags)
