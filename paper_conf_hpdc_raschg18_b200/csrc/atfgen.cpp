@@ -12,6 +12,9 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <chrono>
+#include <mutex>
+#include <thread>
 #include <array>
 #include <atomic>
 #include <cstdarg>
@@ -174,8 +177,11 @@ struct atf_space {
     size_t pbuf_cap = 0;                   // from the ranks' level arrays (P2P copies)
     cudaStream_t stream = nullptr;
     cudaEvent_t fork = nullptr, join = nullptr;
+    cudaEvent_t done = nullptr;  // run_levels_async: the group's level and its result copies finished
   };
   std::vector<GroupBufs> gb;
+  // run_levels_async: pinned per-group result slots [total u64 | overflow u32 | pad | tail totals u64[4]]
+  unsigned long long* h_pin = nullptr;
   uint64_t stash_hint = 0;     // records: exact size of the last level that overflowed
   unsigned int* d_counter = nullptr;     // [kMaxGroups] tile counters
   unsigned long long* d_totals = nullptr;  // [kMaxGroups]
@@ -1017,6 +1023,35 @@ static void choose_geometry(LevelArgs& a, int words, bool legacy_wide, bool seg_
   a.smem_bytes = expand_layout(a, words).total;
 }
 
+// ---------------------------------------------------------------- pinned result slots
+// run_levels_async reads each group's level total through a pinned 4 KB block (an asynchronous
+// copy per group instead of one synchronising copy per round).  The blocks are pooled per
+// process: a fresh space (one per request) does not pay a cudaMallocHost.
+constexpr size_t kPinSlotBytes = 64;  // per group: total u64 | overflow u32 | pad | tail totals u64[4]
+static std::mutex g_pin_mu;
+static std::vector<void*> g_pin_free;
+static unsigned long long* pinned_slot_acquire() {
+  {
+    std::lock_guard<std::mutex> lk(g_pin_mu);
+    if (!g_pin_free.empty()) {
+      void* p = g_pin_free.back();
+      g_pin_free.pop_back();
+      return (unsigned long long*)p;
+    }
+  }
+  void* p = nullptr;
+  if (cudaMallocHost(&p, kMaxGroups * kPinSlotBytes) != cudaSuccess) {
+    cudaGetLastError();
+    return nullptr;
+  }
+  return (unsigned long long*)p;
+}
+static void pinned_slot_release(unsigned long long* p) {
+  if (!p) return;
+  std::lock_guard<std::mutex> lk(g_pin_mu);
+  g_pin_free.push_back(p);
+}
+
 // ---------------------------------------------------------------- device setup
 static atf_status ensure_device(atf_space* s) {
   CUDA_TRY(s, cudaSetDevice(s->opts.device));
@@ -1117,6 +1152,7 @@ static atf_status ensure_device(atf_space* s) {
     CUDA_TRY(s, cudaStreamCreateWithFlags(&b.stream, cudaStreamNonBlocking));
     CUDA_TRY(s, cudaEventCreateWithFlags(&b.fork, cudaEventDisableTiming));
     CUDA_TRY(s, cudaEventCreateWithFlags(&b.join, cudaEventDisableTiming));
+    CUDA_TRY(s, cudaEventCreateWithFlags(&b.done, cudaEventDisableTiming));
   }
   s->dev_ready = true;
   return ATF_OK;
@@ -1214,8 +1250,11 @@ static void release_device(atf_space* s) {
     }
     if (b.fork) cudaEventDestroy(b.fork);
     if (b.join) cudaEventDestroy(b.join);
+    if (b.done) cudaEventDestroy(b.done);
   }
   s->gb.clear();
+  pinned_slot_release(s->h_pin);
+  s->h_pin = nullptr;
   for (auto& pm : s->peers) cudaIpcCloseMemHandle(pm.base);
   s->peers.clear();
   s->d_counter = nullptr;
@@ -1278,6 +1317,10 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   LevelPlan& lp = gp.levels[k];
   cudaStream_t st = (cudaStream_t)s->opts.stream;  // allocations, memsets
   auto& gbf = s->gb[g];                            // this group's buffers and launch stream
+#ifdef ATF_HOST_PROF
+  using hclk = std::chrono::steady_clock;
+  const auto q0 = hclk::now();
+#endif
   LevelArgs a = lp.proto;
   a.parent_rec = parents;
   a.n_parents = n_parents;
@@ -1429,6 +1472,9 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
     a.piece_tile = piece_tile;
     CUDA_TRY(s, cudaMemsetAsync(d_scratch + o_scan, 0, o_top + 16 - o_scan, st));
   }
+#ifdef ATF_HOST_PROF
+  const auto q1 = hclk::now();
+#endif
   if (a.direct) {
     const size_t need = (size_t)a.n_tiles + 1;
     if (need > gbf.status_cap) {
@@ -1492,6 +1538,13 @@ static atf_status queue_level(atf_space* s, int g, int k, const uint32_t* parent
   }
   if (timing) CUDA_TRY(s, cudaEventRecord(s->events[g][k].second, ls));
   if (!serial) CUDA_TRY(s, cudaEventRecord(gbf.join, ls));
+#ifdef ATF_HOST_PROF
+  {
+    auto us = [](hclk::time_point x, hclk::time_point y) { return std::chrono::duration<double, std::micro>(y - x).count(); };
+    const auto q2 = hclk::now();
+    fprintf(stderr, "[atf host]   g%d k%d: setup+alloc %.1f us, launch %.1f us\n", g, k, us(q0, q1), us(q1, q2));
+  }
+#endif
   pd.joined = !serial;
   pd = Pending{g, k, n_parents, parents, (uint64_t*)csr, child, cap, which, off, pd.joined};
   return ATF_OK;
@@ -1771,7 +1824,14 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
                              std::vector<const uint32_t*> frontier, std::vector<uint64_t> fsize) {
   cudaStream_t st = (cudaStream_t)s->opts.stream;
   std::vector<int> k = k_from;
+#ifdef ATF_HOST_PROF  // host phases of the level-by-level rounds (diagnostic builds only)
+  using hclk = std::chrono::steady_clock;
+  auto hus = [](hclk::time_point a, hclk::time_point b) { return std::chrono::duration<double, std::micro>(b - a).count(); };
+#endif
   for (int round = 0;; round++) {
+#ifdef ATF_HOST_PROF
+    const auto hp0 = hclk::now();
+#endif
     char rname[48];
     snprintf(rname, sizeof rname, "atf level round %d", round);
     NvtxRange nvtx_round(rname);
@@ -1822,6 +1882,9 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       pend.push_back(pd);
     }
     if (pend.empty()) break;
+#ifdef ATF_HOST_PROF
+    const auto hpq = hclk::now();
+#endif
     for (auto& pd : pend)
       if (pd.joined) CUDA_TRY(s, cudaStreamWaitEvent(st, s->gb[pd.g].join, 0));  // join the group streams
     // one copy brings back [totals | overflow flags] of every group
@@ -1834,6 +1897,10 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
                                       cudaMemcpyDeviceToHost, st));
       }
     CUDA_TRY(s, cudaStreamSynchronize(st));
+#ifdef ATF_HOST_PROF
+    fprintf(stderr, "[atf host] round %d: %zu levels, host queue %.1f us, copy+sync %.1f us\n", round, pend.size(),
+            hus(hp0, hpq), hus(hpq, hclk::now()));
+#endif
     unsigned long long h_pairs[kMaxGroups] = {};
     if (s->opts.flags & ATF_FLAG_TIMING)
       CUDA_TRY(s, cudaMemcpy(h_pairs, s->d_pairs, sizeof(h_pairs), cudaMemcpyDeviceToHost));
@@ -1874,6 +1941,138 @@ static atf_status run_levels(atf_space* s, std::vector<int> gs, std::vector<int>
       fsize[i] = total;
       k[i]++;
     }
+  }
+  return ATF_OK;
+}
+
+// Level-by-level generation of every group with NO round barrier between the groups (a fresh
+// space: level sizes unknown).  Each group advances on its own stream: its level's total and
+// overflow flag come back through an asynchronous copy into a pinned slot, an event marks the
+// group done, and the host queues that group's next level as soon as it is -- while the other
+// groups' kernels keep the GPU busy, instead of every group waiting for the slowest one and the
+// GPU idling while the host queues the next round (~60 us of host work per level).  Same kernels,
+// same allocations and the same level data as run_levels.  Not used with ATF_FLAG_TIMING (per-round
+// statistics) or ATF_FLAG_SERIAL_GROUPS.
+static atf_status run_levels_async(atf_space* s) {
+  cudaStream_t st = (cudaStream_t)s->opts.stream;
+  const int G = (int)s->groups.size();
+  if (!s->h_pin && !(s->h_pin = pinned_slot_acquire())) return fail(s, ATF_ERR_OOM, "pinned result slots");
+  std::vector<int> k(G, 0);
+  std::vector<const uint32_t*> frontier(G, s->d_root);
+  std::vector<uint64_t> fsize(G, 1);
+  std::vector<char> busy(G, 0), finished(G, 0);
+  std::vector<Pending> pend(G);
+  auto slot = [&](int g) { return s->h_pin + (size_t)g * (kPinSlotBytes / 8); };
+  // queue group g's next level (or finish it); returns with busy[g] set when work is in flight
+  auto queue = [&](int g) -> atf_status {
+    const int L = (int)s->groups[g].levels.size();
+    if (k[g] >= L) { finished[g] = 1; return ATF_OK; }
+    if (fsize[g] == 0 || s->groups[g].levels[k[g]].r == 0) {
+      // empty frontier or empty range: every deeper level is empty
+      for (int kk = k[g]; kk < L; kk++) {
+        LevelData& d = s->data[g][kk];
+        d.rec = nullptr;
+        d.n = 0;
+        d.evals = (kk == k[g]) ? fsize[g] * (uint64_t)s->groups[g].levels[kk].r : 0;
+        if (kk > 0 && kk == k[g] && fsize[g] > 0) {
+          atf_status e = ATF_OK;
+          char* csr = arena_take(s, g, (fsize[g] + 1) * 8, &e);
+          if (!csr) return e ? e : fail(s, ATF_ERR_OOM, "CSR");
+          CUDA_TRY(s, cudaMemsetAsync(csr, 0, (fsize[g] + 1) * 8, st));
+          s->data[g][kk - 1].csr = (uint64_t*)csr;
+        }
+      }
+      k[g] = L;
+      finished[g] = 1;
+      return ATF_OK;
+    }
+    // this group's level total, overflow flag and tile counter (the kernels fork from st)
+    CUDA_TRY(s, cudaMemsetAsync(s->d_totals + g, 0, 8, st));
+    CUDA_TRY(s, cudaMemsetAsync(s->d_ovf + g, 0, 4, st));
+    CUDA_TRY(s, cudaMemsetAsync(s->d_counter + g, 0, 4, st));
+    Pending& pd = pend[g];
+    atf_status e;
+    if (s->tails[g].phase == 1) e = queue_tail_emit(s, g, pd, true);
+    else if (tail_here(s, g, k[g], fsize[g])) e = queue_tail_count(s, g, k[g], frontier[g], fsize[g], pd, true);
+    else e = queue_level(s, g, k[g], frontier[g], fsize[g], pd, true);
+    if (e) return e;
+    cudaStream_t ls = s->gb[g].stream;
+    unsigned long long* h = slot(g);
+    CUDA_TRY(s, cudaMemcpyAsync(h, s->d_totals + g, 8, cudaMemcpyDeviceToHost, ls));
+    CUDA_TRY(s, cudaMemcpyAsync(h + 1, s->d_ovf + g, 4, cudaMemcpyDeviceToHost, ls));
+    if (pd.kind == 1) {
+      auto& T = s->tails[g];
+      for (int d = 0; d < T.nl; d++)
+        CUDA_TRY(s, cudaMemcpyAsync(h + 2 + d, T.t.tile_base + d * (T.t.n_tiles + 1) + T.t.n_tiles, 8,
+                                    cudaMemcpyDeviceToHost, ls));
+    }
+    CUDA_TRY(s, cudaEventRecord(s->gb[g].done, ls));
+    busy[g] = 1;
+    return ATF_OK;
+  };
+  // a finished level of group g: the bookkeeping of run_levels
+  auto complete = [&](int g) -> atf_status {
+    busy[g] = 0;
+    Pending& pd = pend[g];
+    const unsigned long long* h = slot(g);
+    if (pd.kind == 1) {
+      auto& T = s->tails[g];
+      for (int d = 0; d < T.nl; d++) T.tot[d] = h[2 + d];
+      T.phase = 1;
+      return ATF_OK;
+    }
+    if (pd.kind == 2) {
+      finish_tail(s, g);
+      k[g] = (int)s->groups[g].levels.size();
+      return ATF_OK;
+    }
+    const uint64_t total = h[0];
+    const uint32_t ovf = (uint32_t)(h[1] & 0xffffffffu);
+    GroupPlan& gp = s->groups[g];
+    if (ovf || total > pd.cap) {  // child region or stash too small: grow and redo the level
+      s->stash_hint = std::max<uint64_t>(s->stash_hint, total);
+      return arena_grow(s, g, total * gp.words * 4 + (pd.n_parents + 1) * 8);
+    }
+    Chunk& c = s->arena[g][pd.chunk];
+    c.used = pd.child_off + ((total * gp.words * 4 + 255) & ~(uint64_t)255);
+    LevelData& d = s->data[g][pd.k];
+    d.rec = pd.child;
+    d.n = total;
+    d.evals = pd.n_parents * (uint64_t)gp.levels[pd.k].r;
+    if (pd.k > 0) s->data[g][pd.k - 1].csr = pd.csr;
+    frontier[g] = pd.child;
+    fsize[g] = total;
+    k[g]++;
+    return ATF_OK;
+  };
+  atf_status e = ATF_OK;
+  for (int g = 0; g < G && !e; g++) e = queue(g);
+  while (!e) {
+    int inflight = 0;
+    for (int g = 0; g < G; g++) inflight += busy[g];
+    if (!inflight) break;
+    bool progressed = false;
+    for (int g = 0; g < G && !e; g++) {
+      if (!busy[g]) continue;
+      const cudaError_t q = cudaEventQuery(s->gb[g].done);
+      if (q == cudaErrorNotReady) continue;
+      if (q != cudaSuccess) {
+        e = fail(s, ATF_ERR_CUDA, "group %d level %d: %s", g, k[g], cudaGetErrorString(q));
+        break;
+      }
+      progressed = true;
+      if ((e = complete(g))) break;
+      e = queue(g);
+    }
+    if (!progressed && !e) std::this_thread::yield();
+  }
+  // every group's work precedes what the caller queues on the space's stream next
+  for (int g = 0; g < G; g++)
+    if (s->gb[g].done) cudaStreamWaitEvent(st, s->gb[g].done, 0);
+  if (e) {
+    for (int g = 0; g < G; g++)
+      if (s->gb[g].stream) cudaStreamSynchronize(s->gb[g].stream);
+    return e;
   }
   return ATF_OK;
 }
@@ -2773,7 +2972,11 @@ static atf_status generate_impl(atf_space* s) {
     std::iota(gs.begin(), gs.end(), 0);
     std::vector<const uint32_t*> fr(G, s->d_root);
     std::vector<uint64_t> fz(G, 1);
-    if ((e = run_levels(s, gs, kf, fr, fz))) return e;
+    if (G > 1 && !(s->opts.flags & (ATF_FLAG_TIMING | ATF_FLAG_SERIAL_GROUPS))) {
+      if ((e = run_levels_async(s))) return e;
+    } else if ((e = run_levels(s, gs, kf, fr, fz))) {
+      return e;
+    }
     s->replay_f.assign(G, {});
     for (size_t g = 0; g < G; g++)
       for (auto& d : s->data[g]) s->replay_f[g].push_back(d.n);
