@@ -192,6 +192,9 @@ atf_status atf_space_add_constraint(atf_space* s, int32_t param_id, const int32_
 atf_status atf_space_plan(atf_space* s);
 
 atf_status atf_space_num_params(const atf_space* s, int32_t* out);
+/* Name of parameter p (NUL-terminated, truncated to cap - 1 bytes); *len_out (optional) = its
+ * full length.  ATF_ERR_INVALID_ARG for a bad p. */
+atf_status atf_space_param_name(const atf_space* s, int32_t p, char* buf, size_t cap, size_t* len_out);
 atf_status atf_space_num_groups(const atf_space* s, int32_t* out);           /* >= PLANNED */
 /* members of group g (declaration order) -> out[0..n), n written to *n_out */
 atf_status atf_space_group_members(const atf_space* s, int32_t g, int32_t* out, int32_t cap,
@@ -358,6 +361,20 @@ atf_status atf_space_filter_product(atf_space* s, uint64_t* h_count, uint64_t* h
  * generate and on shard spaces; ATF_ERR_LIMIT on an int64 space. */
 atf_status atf_space_neighbors(const atf_space* s, const int32_t* d_in, int64_t ld_in, int64_t n, uint64_t seed,
                                int32_t max_tries, int32_t* d_out, int64_t ld_out, int32_t* d_moved, void* stream);
+
+/* Checkpoint / resume ("serialise spec + level arrays"): a generated space to a
+ * file and back, so that a tuning run (decode / encode / neighbours) resumes without
+ * regenerating.  atf_space_save writes the spec (names, int64 range values in range order,
+ * constraint programs) and every group's level arrays (path records, CSR); synchronous.
+ * ATF_ERR_STATE unless GENERATED by atf_space_generate (not a shard / rank part);
+ * ATF_ERR_INVALID_ARG if the file cannot be written.
+ * atf_space_load creates a space with `opts` (device, stream, allocator, flags), re-plans the
+ * stored spec (groups and record layout must match the file), uploads the arrays and leaves it
+ * GENERATED (size / decode / encode / neighbours / stats work; a later generate recomputes it).
+ * A malformed, truncated or corrupted file (FNV-1a checksum) -> ATF_ERR_INVALID_ARG.  *out is
+ * set even on error (atf_space_last_error explains; destroy it). */
+atf_status atf_space_save(const atf_space* s, const char* path);
+atf_status atf_space_load(const atf_space_opts* opts, const char* path, atf_space** out);
 
 /* Per (group, level) statistics, in (group, level) order. */
 typedef struct {

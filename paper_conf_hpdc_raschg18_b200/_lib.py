@@ -89,6 +89,9 @@ _SIGS = {
     "atf_space_decode_digits_i64": (_st, [SP, C.c_void_p, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_space_decode_range_i64": (_st, [SP, C.c_uint64, C.c_uint64, C.c_int64, C.c_void_p, C.c_int64, C.c_void_p]),
     "atf_space_value_bits": (_st, [SP, C.POINTER(C.c_int32)]),
+    "atf_space_save": (_st, [SP, C.c_char_p]),
+    "atf_space_load": (_st, [C.POINTER(atf_space_opts), C.c_char_p, C.POINTER(SP)]),
+    "atf_space_param_name": (_st, [SP, C.c_int32, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "atf_space_encode_digits": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p]),
     "atf_space_encode_indices": (_st, [SP, C.c_void_p, C.c_int64, C.c_int64, C.c_void_p, C.c_void_p, C.c_void_p]),
     "atf_space_filter_product": (_st, [SP, C.POINTER(C.c_uint64), C.POINTER(C.c_uint64)]),

@@ -2996,6 +2996,211 @@ static atf_status generate_impl(atf_space* s) {
   return ATF_OK;
 }
 
+// ---------------------------------------------------------------- checkpoint / resume
+// A generated space on disk (SURVEY.md §5 "Checkpoint / resume: serialise spec + level arrays"):
+// the spec (names, int64 range values in range order, constraint programs) and every group's
+// level arrays (path records, CSR), so a tuning run resumes without regenerating.  Loading
+// re-plans the spec (deterministic: same groups and record layout, checked against the file)
+// and uploads the arrays.  Little-endian; FNV-1a 64 checksum of everything before it.
+static const char kCkptMagic[8] = {'A', 'T', 'F', 'S', 'P', 'C', '0', '1'};
+constexpr uint32_t kCkptVersion = 1;
+
+namespace {
+struct CkWriter {
+  FILE* f;
+  uint64_t h = 1469598103934665603ull;
+  bool ok = true;
+  void put(const void* p, size_t n) {
+    const unsigned char* b = (const unsigned char*)p;
+    for (size_t i = 0; i < n; i++) h = (h ^ b[i]) * 1099511628211ull;
+    if (n && std::fwrite(p, 1, n, f) != n) ok = false;
+  }
+  template <typename T> void val(T v) { put(&v, sizeof v); }
+};
+struct CkReader {
+  FILE* f;
+  uint64_t h = 1469598103934665603ull;
+  bool ok = true;
+  bool get(void* p, size_t n) {
+    if (!ok || (n && std::fread(p, 1, n, f) != n)) return ok = false;
+    const unsigned char* b = (const unsigned char*)p;
+    for (size_t i = 0; i < n; i++) h = (h ^ b[i]) * 1099511628211ull;
+    return true;
+  }
+  template <typename T> bool val(T& v) { return get(&v, sizeof v); }
+};
+}  // namespace
+
+atf_status atf_space_save(const atf_space* cs, const char* path) {
+  atf_space* s = (atf_space*)cs;
+  if (!s || !path) return ATF_ERR_INVALID_ARG;
+  if (s->state != GENERATED) return fail(s, ATF_ERR_STATE, "save needs a generated (non-shard) space");
+  for (size_t g = 0; g < s->groups.size(); g++)
+    for (auto& d : s->data[g])
+      if (d.offset != 0 || (d.csr_n != UINT64_MAX && d.csr_n != d.n))
+        return fail(s, ATF_ERR_STATE, "save: the space holds a rank's part of a distributed generation");
+  CUDA_TRY(s, cudaSetDevice(s->opts.device));
+  CUDA_TRY(s, cudaStreamSynchronize((cudaStream_t)s->opts.stream));
+  FILE* f = std::fopen(path, "wb");
+  if (!f) return fail(s, ATF_ERR_INVALID_ARG, "cannot open %s for writing", path);
+  CkWriter w{f};
+  w.put(kCkptMagic, 8);
+  w.val<uint32_t>(kCkptVersion);
+  w.val<uint32_t>((uint32_t)s->params.size());
+  for (auto& p : s->params) {
+    w.val<uint32_t>((uint32_t)p.name.size());
+    w.put(p.name.data(), p.name.size());
+    const uint64_t n = p.values.size();
+    w.val<uint64_t>(n);
+    for (uint64_t j = 0; j < n; j++) w.val<int64_t>(p.v64 ? p.values64[j] : (int64_t)p.values[j]);
+    w.val<uint32_t>((uint32_t)p.programs.size());
+    for (auto& prog : p.programs) {
+      w.val<uint32_t>((uint32_t)prog.size());
+      w.put(prog.data(), prog.size() * 4);
+    }
+  }
+  w.val<uint32_t>((uint32_t)s->groups.size());
+  std::vector<char> buf;
+  atf_status st = ATF_OK;
+  for (size_t g = 0; g < s->groups.size() && st == ATF_OK && w.ok; g++) {
+    const GroupPlan& gp = s->groups[g];
+    w.val<uint32_t>((uint32_t)gp.levels.size());
+    w.val<uint32_t>((uint32_t)gp.words);
+    for (size_t k = 0; k < gp.levels.size() && w.ok; k++) {
+      const LevelData& d = s->data[g][k];
+      const uint64_t n = d.rec ? d.n : 0;
+      const uint64_t nc = (k + 1 < gp.levels.size() && d.csr && n) ? n + 1 : 0;
+      w.val<uint64_t>(n);
+      w.val<uint64_t>(nc);
+      const size_t rb = (size_t)n * gp.words * 4, cb = (size_t)nc * 8;
+      buf.resize(std::max<size_t>(rb, cb) + 1);
+      if (rb) {
+        if (cudaMemcpy(buf.data(), d.rec, rb, cudaMemcpyDeviceToHost) != cudaSuccess) { st = ATF_ERR_CUDA; break; }
+        w.put(buf.data(), rb);
+      }
+      if (cb) {
+        if (cudaMemcpy(buf.data(), d.csr, cb, cudaMemcpyDeviceToHost) != cudaSuccess) { st = ATF_ERR_CUDA; break; }
+        w.put(buf.data(), cb);
+      }
+    }
+  }
+  const uint64_t h = w.h;
+  if (st == ATF_OK) w.put(&h, 8);
+  const bool ok = w.ok && std::fclose(f) == 0;
+  if (st != ATF_OK) return fail(s, st, "save: device copy failed: %s", cudaGetErrorString(cudaGetLastError()));
+  if (!ok) return fail(s, ATF_ERR_INVALID_ARG, "save: write to %s failed", path);
+  return ATF_OK;
+}
+
+static atf_status load_impl(atf_space* s, FILE* f) {
+  CkReader r{f};
+  char magic[8];
+  uint32_t ver = 0, np = 0;
+  if (!r.get(magic, 8) || std::memcmp(magic, kCkptMagic, 8) != 0) return fail(s, ATF_ERR_INVALID_ARG, "load: not an atfgen checkpoint");
+  if (!r.val(ver) || ver != kCkptVersion) return fail(s, ATF_ERR_INVALID_ARG, "load: unsupported checkpoint version");
+  if (!r.val(np) || np > ATF_MAX_PARAMS) return fail(s, ATF_ERR_INVALID_ARG, "load: bad parameter count");
+  for (uint32_t p = 0; p < np; p++) {
+    uint32_t nl = 0;
+    if (!r.val(nl) || nl == 0 || nl > 4096) return fail(s, ATF_ERR_INVALID_ARG, "load: bad name");
+    std::string name(nl, '\0');
+    uint64_t n = 0;
+    if (!r.get(&name[0], nl) || !r.val(n) || n > ATF_MAX_RANGE) return fail(s, ATF_ERR_INVALID_ARG, "load: bad range");
+    std::vector<int64_t> vals(n);
+    if (n && !r.get(vals.data(), n * 8)) return fail(s, ATF_ERR_INVALID_ARG, "load: truncated range");
+    atf_range rg{};
+    rg.kind = ATF_RANGE_SET64;
+    rg.values64 = vals.data();
+    rg.n_values = (int64_t)n;
+    int32_t id = -1;
+    atf_status e = atf_space_add_param(s, name.c_str(), &rg, &id);
+    if (e) return e;
+    uint32_t nprog = 0;
+    if (!r.val(nprog) || nprog > 1024) return fail(s, ATF_ERR_INVALID_ARG, "load: bad program count");
+    for (uint32_t q = 0; q < nprog; q++) {
+      uint32_t nw = 0;
+      if (!r.val(nw) || nw == 0 || nw > ATF_MAX_PROGRAM_WORDS) return fail(s, ATF_ERR_INVALID_ARG, "load: bad program");
+      std::vector<int32_t> code(nw);
+      if (!r.get(code.data(), nw * 4)) return fail(s, ATF_ERR_INVALID_ARG, "load: truncated program");
+      if ((e = atf_space_add_constraint(s, id, code.data(), (int32_t)nw))) return e;
+    }
+  }
+  atf_status e = plan(s);
+  if (e) return e;
+  uint32_t G = 0;
+  if (!r.val(G) || G != s->groups.size()) return fail(s, ATF_ERR_INVALID_ARG, "load: group structure differs from the plan");
+  if ((e = ensure_device(s))) return e;
+  s->data.assign(G, {});
+  s->tails.assign(G, {});
+  std::vector<char> buf;
+  for (uint32_t g = 0; g < G; g++) {
+    const GroupPlan& gp = s->groups[g];
+    uint32_t L = 0, W = 0;
+    if (!r.val(L) || !r.val(W) || L != gp.levels.size() || W != (uint32_t)gp.words)
+      return fail(s, ATF_ERR_INVALID_ARG, "load: level layout of group %u differs from the plan", g);
+    s->data[g].assign(L, LevelData{});
+    uint64_t above = 1;
+    for (uint32_t k = 0; k < L; k++) {
+      uint64_t n = 0, nc = 0;
+      if (!r.val(n) || !r.val(nc)) return fail(s, ATF_ERR_INVALID_ARG, "load: truncated level");
+      if (n > above * (uint64_t)gp.levels[k].r || (nc && nc != n + 1) || (nc && k + 1 == L))
+        return fail(s, ATF_ERR_INVALID_ARG, "load: inconsistent level sizes");
+      LevelData& d = s->data[g][k];
+      d.n = n;
+      d.evals = above * (uint64_t)gp.levels[k].r;
+      const size_t rb = (size_t)n * W * 4, cb = (size_t)nc * 8;
+      buf.resize(std::max<size_t>(rb, cb) + 1);
+      if (rb) {
+        if (!r.get(buf.data(), rb)) return fail(s, ATF_ERR_INVALID_ARG, "load: truncated records");
+        char* p = arena_take(s, (int)g, rb, &e);
+        if (!p) return e ? e : fail(s, ATF_ERR_OOM, "load: records");
+        CUDA_TRY(s, cudaMemcpy(p, buf.data(), rb, cudaMemcpyHostToDevice));
+        d.rec = (uint32_t*)p;
+      }
+      if (cb) {
+        if (!r.get(buf.data(), cb)) return fail(s, ATF_ERR_INVALID_ARG, "load: truncated CSR");
+        char* p = arena_take(s, (int)g, cb, &e);
+        if (!p) return e ? e : fail(s, ATF_ERR_OOM, "load: CSR");
+        CUDA_TRY(s, cudaMemcpy(p, buf.data(), cb, cudaMemcpyHostToDevice));
+        d.csr = (uint64_t*)p;
+      }
+      above = n;
+    }
+  }
+  const uint64_t want = r.h;
+  uint64_t got = 0;
+  if (!r.get(&got, 8) || got != want) return fail(s, ATF_ERR_INVALID_ARG, "load: checksum mismatch");
+  s->gsize.assign(G, 0);
+  s->group_work.assign(G, 0.0);
+  for (uint32_t g = 0; g < G; g++) {
+    s->gsize[g] = s->groups[g].levels.empty() ? 0 : s->data[g].back().n;
+    uint64_t fr = 1;
+    for (size_t k = 0; k < s->data[g].size(); k++) {
+      s->group_work[g] += (double)fr * (double)s->groups[g].levels[k].r;
+      fr = s->data[g][k].n;
+    }
+  }
+  s->replay_ok = false;  // a later generate recomputes level by level
+  s->state = GENERATED;
+  return ATF_OK;
+}
+
+atf_status atf_space_load(const atf_space_opts* opts, const char* path, atf_space** out) {
+  if (!out || !path) return ATF_ERR_INVALID_ARG;
+  *out = nullptr;
+  atf_space* s = nullptr;
+  atf_status e = atf_space_create(opts, &s);
+  if (e) return e;
+  FILE* f = std::fopen(path, "rb");
+  if (!f) {
+    e = fail(s, ATF_ERR_INVALID_ARG, "cannot open %s", path);
+  } else {
+    e = load_impl(s, f);
+    std::fclose(f);
+  }
+  *out = s;  // also on error: atf_space_last_error(s) says why; the caller destroys it
+  return e;
+}
+
 // ---------------------------------------------------------------- decode args
 static atf_status make_decode_args(const atf_space* s, DecodeArgs& a) {
   std::memset(&a, 0, sizeof a);
@@ -3246,6 +3451,18 @@ atf_status atf_space_plan(atf_space* s) {
 atf_status atf_space_num_params(const atf_space* s, int32_t* out) {
   if (!s || !out) return ATF_ERR_INVALID_ARG;
   *out = (int32_t)s->params.size();
+  return ATF_OK;
+}
+
+atf_status atf_space_param_name(const atf_space* s, int32_t p, char* buf, size_t cap, size_t* len_out) {
+  if (!s || p < 0 || p >= (int32_t)s->params.size() || (!buf && cap)) return ATF_ERR_INVALID_ARG;
+  const std::string& n = s->params[p].name;
+  if (len_out) *len_out = n.size();
+  if (cap) {
+    const size_t m = std::min(cap - 1, n.size());
+    std::memcpy(buf, n.data(), m);
+    buf[m] = '\0';
+  }
   return ATF_OK;
 }
 

@@ -40,7 +40,8 @@ class Space:
     (interpret every candidate with the generic bytecode interpreter).
     """
 
-    def __init__(self, spec=None, device: int = 0, stream=None, flags: int = 0, torch_alloc: bool = True):
+    def __init__(self, spec=None, device: int = 0, stream=None, flags: int = 0, torch_alloc: bool = True,
+                 _load_path: Optional[str] = None):
         self._h = C.c_void_p()
         self._bufs: Dict[int, object] = {}
         self._device = device
@@ -74,11 +75,38 @@ class Space:
                     self._alloc_cb = L.ALLOC_FN(_alloc)
                     self._free_cb = L.FREE_FN(_free)
         opts = L.atf_space_opts(device, stream_ptr, self._alloc_cb, self._free_cb, None, flags)
-        L.check(L.atf_space_create(C.byref(opts), C.byref(self._h)))
         self.names: List[str] = []
         self._labels: List[Optional[List[str]]] = []  # enum names per parameter (atfspec.enum)
+        if _load_path is not None:
+            st = L.atf_space_load(C.byref(opts), str(_load_path).encode(), C.byref(self._h))
+            if st != L.ATF_OK:
+                try:
+                    L.check(st, self._h)
+                finally:
+                    L.atf_space_destroy(self._h)
+                    self._h = C.c_void_p()
+            n = C.c_int32()
+            L.check(L.atf_space_num_params(self._h, C.byref(n)), self._h)
+            for p in range(n.value):
+                ln = C.c_size_t()
+                L.check(L.atf_space_param_name(self._h, p, None, 0, C.byref(ln)), self._h)
+                buf = C.create_string_buffer(ln.value + 1)
+                L.check(L.atf_space_param_name(self._h, p, buf, ln.value + 1, None), self._h)
+                self.names.append(buf.value.decode())
+                self._labels.append(None)
+            return
+        L.check(L.atf_space_create(C.byref(opts), C.byref(self._h)))
         if spec is not None:
             self.add_spec(spec)
+
+    @classmethod
+    def load(cls, path, device: int = 0, stream=None, flags: int = 0, torch_alloc: bool = True) -> "Space":
+        """A space saved by `save` (checkpoint / resume): GENERATED, ready for decode / encode."""
+        return cls(None, device=device, stream=stream, flags=flags, torch_alloc=torch_alloc, _load_path=path)
+
+    def save(self, path) -> None:
+        """Write the generated space (spec + level arrays) to `path` (atf_space_save)."""
+        L.check(L.atf_space_save(self._h, str(path).encode()), self._h)
 
     # ---- building
     def add_spec(self, spec) -> None:
