@@ -1813,7 +1813,10 @@ static void finish_tail(atf_space* s, int g) {
     if (timing) {  // the whole tail is attributed to its first level
       ld.ms = d == 0 ? ms_count + ms_emit : 0.f;
       ld.expand_ms = d == 0 ? ms_count_k + ms_emit : 0.f;
-      ld.pairs = ld.evals;
+      // product-structured tail: a level's mask is a function of the frontier node and is
+      // evaluated once per frontier node (r_d pairs), not once per level-(d-1) node
+      const bool prod = !(s->opts.flags & ATF_FLAG_NO_JIT) && gp.tail_jit && jit_tail_product(gp.tail_jit);
+      ld.pairs = (prod && d > 0) ? t.n_parents * (uint64_t)gp.levels[T.k0 + d].r : ld.evals;
     }
   }
   T.phase = 2;
@@ -4137,6 +4140,11 @@ atf_status atf_test_set_geometry(int32_t tiles_per_sm, int32_t repl_log2) {
 atf_status atf_test_set_direct_tiles(int32_t n) {
   if (n < 0 || n > (1 << 20)) return ATF_ERR_INVALID_ARG;
   g_direct_tiles.store(n ? n : 16);
+  return ATF_OK;
+}
+
+atf_status atf_test_set_tail_product(int32_t on) {
+  jit_set_tail_product(on != 0);
   return ATF_OK;
 }
 

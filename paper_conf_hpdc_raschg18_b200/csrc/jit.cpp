@@ -387,10 +387,11 @@ struct TailJitArgs { const u32* parent_rec; u64 n_parents, n_tiles; u32* tile_to
 //                   frontier lane they descend from, whose node constants sit in shared memory),
 //                   written out as coalesced vectors, CSR entries of every chunk.
 std::atomic<int> g_tail_stage{8192};  // tail emit staging bytes per warp (atf_test_set_tail_stage)
+std::atomic<bool> g_tail_product{true};  // product-structured tails (atf_test_set_tail_product)
 
 std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vector<int32_t>>& cx,
                             const std::vector<std::vector<uint32_t>>& cm, int k0,
-                            const std::vector<std::vector<int>>& pv_level, int* warp_bytes) {
+                            const std::vector<std::vector<int>>& pv_level, int* warp_bytes, bool* product_out = nullptr) {
   const int nl = t.nl;
   if (nl < 2 || nl > kMaxTail || (int)pv_level.size() < nl) return "";
   std::string s = kPrelude;
@@ -456,6 +457,39 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
     }
     s += "  return m;\n}\n";
   }
+  // ---- product-structured count: every term of every tail level reads only ancestors above the
+  // tail (all node constants), so under one frontier node level d's mask m_d is the same at every
+  // level-(d-1) node and level d holds P_d = c_0 ... c_d nodes (c_e = popc m_e): the count is a
+  // product instead of a depth-first walk (C3-IS2 145 -> 108 us).  The emit stays the depth-first
+  // kernel below (a lane-parallel emit over the product grid was built and measured slower: 0.97 vs
+  // 0.69 ms).
+  bool product = g_tail_product.load();
+  for (int d = 0; d < nl && product; d++)
+    for (int tt = 0; tt < t.lv[d].n_terms; tt++)
+      if (ncoff[d][tt] < 0) product = false;
+  if (product_out) *product_out = product;
+  if (product) {
+    const std::string NLs = std::to_string(nl);
+    // count: thread per frontier node
+    s += "extern \"C\" __global__ void __launch_bounds__(256) atf_tail_count(const __grid_constant__ TailJitArgs a) {\n";
+    s += "  const int lane = threadIdx.x & 31;\n  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n";
+    s += "  for (u64 tile = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile < a.n_tiles; tile += nw) {\n";
+    s += "    const u64 nd = tile * 32 + lane;\n    u32 P[" + NLs + "] = {};\n";
+    s += "    if (nd < a.n_parents) {\n      u32 w[" + Ws + "];\n";
+    s += "      for (int i = 0; i < " + Ws + "; i++) w[i] = __ldg(a.parent_rec + nd * " + Ws + " + i);\n";
+    s += "      u32 nc[" + std::to_string(NC) + "];\n      tnc(a, w, nc);\n      u32 p = 1u;\n";
+    for (int d = 0; d < nl; d++)
+      s += "      p *= (u32)__popcll((u64)tmask" + std::to_string(d) + "(a, w, nc)); P[" + std::to_string(d) + "] = p;\n";
+    for (int d = 0; d < nl; d++)
+      s += "      a.node_cnt[(u64)" + std::to_string(d) + " * a.n_parents + nd] = P[" + std::to_string(d) + "];\n";
+    s += "    }\n";
+    for (int d = 0; d < nl; d++) {
+      const std::string ds = std::to_string(d);
+      s += "    { u32 v = P[" + ds + "];\n#pragma unroll\n      for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);\n";
+      s += "      if (lane == 0) a.tile_total[(u64)" + ds + " * a.n_tiles + tile] = v; }\n";
+    }
+    s += "  }\n}\n";
+  }
   auto child = [&](int d, const std::string& src, const std::string& dst, const std::string& ind) {
     std::string c;
     const int fw = t.lv[d].field_word, fs = t.lv[d].field_shift;
@@ -464,34 +498,36 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
            (w == fw && t.lv[d].r > 1 ? " | (cc << " + std::to_string(fs) + ")" : "") + ";\n";  // r == 1: no field bits
     return c;
   };
-  // ---- count: depth-first per frontier node
-  for (int d = nl - 1; d >= 0; d--) {
-    const std::string ds = std::to_string(d);
-    s += "__device__ __forceinline__ void cnt" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cnt) {\n";
-    s += "  auto m = tmask" + ds + "(a, w, nc);\n  cnt[" + ds + "] += __popcll((u64)m);\n";
-    if (d + 1 < nl) {
-      s += "  while (m) {\n    const u32 cc = __ffsll((long long)m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
-      s += child(d, "w", "cw", "    ");
-      s += "    cnt" + std::to_string(d + 1) + "(a, cw, nc, cnt);\n  }\n";
+  if (!product) {  // (the product count above replaces it)
+    // ---- count: depth-first per frontier node
+    for (int d = nl - 1; d >= 0; d--) {
+      const std::string ds = std::to_string(d);
+      s += "__device__ __forceinline__ void cnt" + ds + "(const TailJitArgs& a, const u32* w, const u32* nc, u32* cnt) {\n";
+      s += "  auto m = tmask" + ds + "(a, w, nc);\n  cnt[" + ds + "] += __popcll((u64)m);\n";
+      if (d + 1 < nl) {
+        s += "  while (m) {\n    const u32 cc = __ffsll((long long)m) - 1;\n    m &= m - 1;\n    u32 cw[" + Ws + "];\n";
+        s += child(d, "w", "cw", "    ");
+        s += "    cnt" + std::to_string(d + 1) + "(a, cw, nc, cnt);\n  }\n";
+      }
+      s += "}\n";
     }
-    s += "}\n";
+    s += "extern \"C\" __global__ void __launch_bounds__(256) atf_tail_count(const __grid_constant__ TailJitArgs a) {\n";
+    s += "  const int lane = threadIdx.x & 31;\n  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n";
+    s += "  for (u64 tile = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile < a.n_tiles; tile += nw) {\n";
+    s += "    const u64 nd = tile * 32 + lane;\n    u32 cnt[" + std::to_string(nl) + "] = {};\n";
+    s += "    if (nd < a.n_parents) {\n      u32 w[" + Ws + "];\n";
+    s += "      for (int i = 0; i < " + Ws + "; i++) w[i] = __ldg(a.parent_rec + nd * " + Ws + " + i);\n";
+    s += "      u32 nc[" + std::to_string(NC) + "];\n      tnc(a, w, nc);\n      cnt0(a, w, nc, cnt);\n";
+    for (int d = 0; d < nl; d++)
+      s += "      a.node_cnt[(u64)" + std::to_string(d) + " * a.n_parents + nd] = cnt[" + std::to_string(d) + "];\n";
+    s += "    }\n";
+    for (int d = 0; d < nl; d++) {
+      const std::string ds = std::to_string(d);
+      s += "    { u32 v = cnt[" + ds + "];\n#pragma unroll\n      for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);\n";
+      s += "      if (lane == 0) a.tile_total[(u64)" + ds + " * a.n_tiles + tile] = v; }\n";
+    }
+    s += "  }\n}\n";
   }
-  s += "extern \"C\" __global__ void __launch_bounds__(256) atf_tail_count(const __grid_constant__ TailJitArgs a) {\n";
-  s += "  const int lane = threadIdx.x & 31;\n  const u64 nw = ((u64)gridDim.x * blockDim.x) >> 5;\n";
-  s += "  for (u64 tile = ((u64)blockIdx.x * blockDim.x + threadIdx.x) >> 5; tile < a.n_tiles; tile += nw) {\n";
-  s += "    const u64 nd = tile * 32 + lane;\n    u32 cnt[" + std::to_string(nl) + "] = {};\n";
-  s += "    if (nd < a.n_parents) {\n      u32 w[" + Ws + "];\n";
-  s += "      for (int i = 0; i < " + Ws + "; i++) w[i] = __ldg(a.parent_rec + nd * " + Ws + " + i);\n";
-  s += "      u32 nc[" + std::to_string(NC) + "];\n      tnc(a, w, nc);\n      cnt0(a, w, nc, cnt);\n";
-  for (int d = 0; d < nl; d++)
-    s += "      a.node_cnt[(u64)" + std::to_string(d) + " * a.n_parents + nd] = cnt[" + std::to_string(d) + "];\n";
-  s += "    }\n";
-  for (int d = 0; d < nl; d++) {
-    const std::string ds = std::to_string(d);
-    s += "    { u32 v = cnt[" + ds + "];\n#pragma unroll\n      for (int o = 16; o > 0; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);\n";
-    s += "      if (lane == 0) a.tile_total[(u64)" + ds + " * a.n_tiles + tile] = v; }\n";
-  }
-  s += "  }\n}\n";
   // ---- emit: lane = frontier node, depth-first (like the count), output staged per warp.
   // Each lane recounts its subtree (cnt_d); warp scans give its nodes' tile-local positions per
   // level (a node's level-d descendants come out of a depth-first walk in canonical order).  The
@@ -968,6 +1004,7 @@ cudaKernel_t compile(const std::string& src, const char* name = "atf_nfast_jit")
 struct TailJit {
   cudaKernel_t count = nullptr, emit = nullptr;
   int warp_bytes = 0, per_sm = 0, per_sm_count = 0;
+  bool product = false;  // the count kernel is the product-structured one
 };
 std::unordered_map<std::string, TailJit> g_tails;  // source -> kernels (under g_mu)
 
@@ -1027,7 +1064,8 @@ void* jit_tail_kernels(const TailArgs& t, int words, const std::vector<std::vect
                        const std::vector<std::vector<uint32_t>>& cand_magics, int k0,
                        const std::vector<std::vector<int>>& pv_level) {
   int wb = 0;
-  const std::string src = gen_tail_source(t, words, cand_values, cand_magics, k0, pv_level, &wb);
+  bool prod = false;
+  const std::string src = gen_tail_source(t, words, cand_values, cand_magics, k0, pv_level, &wb, &prod);
   if (src.empty()) return nullptr;
   {
     std::lock_guard<std::mutex> lk(g_mu);
@@ -1038,6 +1076,7 @@ void* jit_tail_kernels(const TailArgs& t, int words, const std::vector<std::vect
   tj.count = compile(src, "atf_tail_count");
   tj.emit = compile(src, "atf_tail_emit");
   tj.warp_bytes = wb;
+  tj.product = prod;
   if (tj.count && tj.emit) {
     const int smem = 4 * wb;
     bool ok = !(smem > 48 * 1024 &&
@@ -1059,6 +1098,8 @@ void* jit_tail_kernels(const TailArgs& t, int words, const std::vector<std::vect
   slot = tj;
   return slot.count ? (void*)&slot : nullptr;
 }
+
+bool jit_tail_product(void* handle) { return handle && reinterpret_cast<const TailJit*>(handle)->product; }
 
 int jit_tail_launch(void* handle, const TailArgs& t, bool emit, void* stream) {
   const TailJit& tj = *reinterpret_cast<const TailJit*>(handle);
@@ -1202,4 +1243,5 @@ int jit_decode_launch(void* kernel, const DecodeArgs& a, const uint64_t* idx, co
 
 namespace atf {
 void jit_set_tail_stage(int bytes) { g_tail_stage.store(bytes > 0 ? bytes : 8192); }
+void jit_set_tail_product(bool on) { g_tail_product.store(on); }
 }  // namespace atf

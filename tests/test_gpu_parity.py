@@ -237,14 +237,28 @@ def test_fuzz_specs_without_tail(Space, seed):
 
 def test_tail_kernel_runs(Space):
     """C3's trailing narrow levels KWI, VWM, VWN (and C2's VWMD, VWND) run as one fused tail
-    (kernel id 5), with every pair of those levels evaluated."""
+    (kernel id 5 / 6).  Their terms read only ancestors above the tail, so the tail is
+    product-structured: the first tail level evaluates every (frontier node, candidate) pair, a
+    deeper level's mask is evaluated once per frontier node (stats "pairs" = f_frontier x r_d);
+    with the product count off, every pair counts."""
     from paper_conf_hpdc_raschg18_b200 import _lib as L
     for spec, want in ((A.c3_xgemm("IS1"), [7, 8, 9]), (A.c2_xgemm_direct(256), [6, 7])):
         with Space(spec, flags=L.ATF_FLAG_TIMING) as sp:
             sp.generate()
             st = [x for x in sp.stats() if x["group"] == 0]
             assert [x["level"] for x in st if x["kernel"] == 6] == want   # NVRTC-specialised tail
-            assert all(x["pairs"] == x["evals"] for x in st if x["kernel"] == 6)
+            tail = [x for x in st if x["kernel"] == 6]
+            f_front = st[want[0] - 1]["f"]
+            assert tail[0]["pairs"] == tail[0]["evals"]
+            assert all(x["pairs"] == f_front * x["r"] for x in tail[1:])
+        L.check(L.atf_test_set_tail_product(0))
+        try:
+            with Space(spec, flags=L.ATF_FLAG_TIMING) as sp:
+                sp.generate()
+                st = [x for x in sp.stats() if x["group"] == 0]
+                assert all(x["pairs"] == x["evals"] for x in st if x["kernel"] == 6)
+        finally:
+            L.check(L.atf_test_set_tail_product(1))
         with Space(spec, flags=L.ATF_FLAG_TIMING | L.ATF_FLAG_NO_JIT) as sp:
             sp.generate()
             assert [x["level"] for x in sp.stats() if x["group"] == 0 and x["kernel"] == 5] == want
