@@ -239,7 +239,8 @@ def e2e_generation(spec, steps, dist_ctx=None):
         n = len(r["values"]) if r["kind"] == "set" else max(0, (r["end"] - r["begin"]) // r["step"] + 1)
         h2d += 12 * ((n + 127) // 128 * 128) + 8 * n
     times, d2h = [], 0
-    for i in range(steps + 1):
+    warm = 3  # fresh-space steps discarded (allocator cache, NVRTC / module loads), as the device timing's W >= 3
+    for i in range(steps + warm):
         torch.cuda.synchronize()
         if dist_ctx:
             dist_ctx["dist"].barrier()
@@ -259,10 +260,12 @@ def e2e_generation(spec, steps, dist_ctx=None):
             t = torch.tensor([dt], dtype=torch.float64, device=dist_ctx["dev"])
             dist_ctx["dist"].all_reduce(t, op=dist_ctx["dist"].ReduceOp.MAX)
             dt = float(t.item())
-        if i:
+        if i >= warm:
             times.append(dt)
         d2h = 12 * nlev
-    return {"s_per_step": float(np.mean(times)), "h2d": h2d, "d2h": d2h, "S": S}
+    print(f"[bench] e2e steps (ms): {[round(t * 1e3, 2) for t in times]}", file=sys.stderr, flush=True)
+    return {"s_per_step": float(np.mean(times)), "h2d": h2d, "d2h": d2h, "S": S,
+            "median_s": float(np.median(times)), "steps": len(times)}
 
 
 def secondary_n1(steps, warmup, sm_mhz):
@@ -521,7 +524,8 @@ def main():
                 "clocks": clocks,
                 "e2e": {"value": leaves / e2e["s_per_step"], "unit": "configs/s",
                         "h2d_bytes_per_step": e2e["h2d"], "d2h_bytes_per_step": e2e["d2h"],
-                        "s_per_step": e2e["s_per_step"]}}
+                        "s_per_step": e2e["s_per_step"], "median_s_per_step": e2e["median_s"],
+                        "steps": e2e["steps"], "warmup": 3}}
         if world == 1:
             evals_total = sum(s["evals"] for s in res["stats"])
             # every pair evaluated (headline flags): evaluated = decided = f_{k-1} r_k

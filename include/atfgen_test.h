@@ -45,6 +45,9 @@ atf_status atf_test_set_tail_stage(int32_t bytes);
  * tail: the subtree under a frontier node is a grid of the levels' masks): on (1,
  * default) or off (0, the depth-first kernels) for tails compiled afterwards. */
 atf_status atf_test_set_tail_product(int32_t on);
+/* Fresh spaces with several groups: per-group level rounds without a barrier (1, default) or one
+ * synchronising round for all groups (0).  A/B experiments. */
+atf_status atf_test_set_async_rounds(int32_t on);
 /* Geometry knobs for spaces planned / generated afterwards (tuning experiments; 0 = default):
  * warp tiles per SM below which the warp-tile kernel halves its nodes per tile (256), and
  * log2 of the candidate-pair count below which generate_dist replicates a level (28). */

@@ -907,6 +907,7 @@ static atf_status plan(atf_space* s) {
 static std::atomic<int> g_tiles_per_sm{256};
 static std::atomic<int> g_repl_log2{28};
 static std::atomic<int> g_direct_tiles{16};  // in-place (look-back) levels: at most this many warp tiles
+static std::atomic<int> g_async_rounds{1};   // fresh spaces: per-group rounds without a barrier
 
 static void choose_geometry(LevelArgs& a, int words, bool legacy_wide, bool seg_bounds = true) {
   const int r = a.r;
@@ -2975,7 +2976,7 @@ static atf_status generate_impl(atf_space* s) {
     std::iota(gs.begin(), gs.end(), 0);
     std::vector<const uint32_t*> fr(G, s->d_root);
     std::vector<uint64_t> fz(G, 1);
-    if (G > 1 && !(s->opts.flags & (ATF_FLAG_TIMING | ATF_FLAG_SERIAL_GROUPS))) {
+    if (G > 1 && g_async_rounds.load() && !(s->opts.flags & (ATF_FLAG_TIMING | ATF_FLAG_SERIAL_GROUPS))) {
       if ((e = run_levels_async(s))) return e;
     } else if ((e = run_levels(s, gs, kf, fr, fz))) {
       return e;
@@ -4140,6 +4141,11 @@ atf_status atf_test_set_geometry(int32_t tiles_per_sm, int32_t repl_log2) {
 atf_status atf_test_set_direct_tiles(int32_t n) {
   if (n < 0 || n > (1 << 20)) return ATF_ERR_INVALID_ARG;
   g_direct_tiles.store(n ? n : 16);
+  return ATF_OK;
+}
+
+atf_status atf_test_set_async_rounds(int32_t on) {
+  g_async_rounds.store(on ? 1 : 0);
   return ATF_OK;
 }
 
