@@ -7,7 +7,7 @@ nvidia-smi --query-gpu=name,clocks.sm,clocks.max.sm --format=csv > gpurun_out/${
 timeout 2400 python -m pytest tests -m gpu -q --maxfail=10 --durations=15 > gpurun_out/${T}_pytest_gpu.txt 2>&1
 echo "pytest rc=$?" >> gpurun_out/${T}_pytest_gpu.txt; tail -3 gpurun_out/${T}_pytest_gpu.txt
 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${T}_smoke.txt 2>&1; echo "smoke rc=$?"
-for tool in memcheck racecheck synccheck; do
+for tool in ${SANITIZE:-}; do
   timeout 1500 compute-sanitizer --tool $tool --print-limit 50 python tools/sanitize_run.py > gpurun_out/${T}_sanitize_$tool.txt 2>&1
   echo "sanitize $tool rc=$?"; tail -2 gpurun_out/${T}_sanitize_$tool.txt
 done
