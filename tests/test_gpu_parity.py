@@ -1074,3 +1074,18 @@ def test_float_parameters_by_position(Space):
         assert all(isinstance(r["TOL"], float) for r in named)
         assert all(r["TOL"] <= 1.0 or r["TS"] >= 16 for r in named)
         assert {r["TOL"] for r in named} == {0.25 * i for i in range(1, 9)}
+
+
+@pytest.mark.parametrize("name", ["C2-256", "C3-IS1", "C5-300x4"])
+def test_sync_rounds_and_dfs_tail_count_parity(Space, name):
+    """The A/B alternatives stay exact: one synchronising level round for all groups
+    (atf_test_set_async_rounds(0)) instead of per-group rounds, and the depth-first tail count
+    (atf_test_set_tail_product(0)) instead of the product count."""
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    L.check(L.atf_test_set_async_rounds(0))
+    L.check(L.atf_test_set_tail_product(0))
+    try:
+        _check_against_oracle(Space, SMALL[name]())
+    finally:
+        L.check(L.atf_test_set_async_rounds(1))
+        L.check(L.atf_test_set_tail_product(1))
