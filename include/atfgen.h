@@ -132,10 +132,14 @@ typedef struct {
                                      synchronisation per level round) instead of replaying the
                                      previous generation's level sizes (one synchronisation,
                                      totals verified; DESIGN.md §5 "Steady state")              */
-#define ATF_FLAG_DIST_SUBSETS 512u /* atf_space_generate_dist: from the second generation on, each
-                                     group on a subset of the ranks in proportion to its candidate
-                                     pairs (off by default: rounds stay in lock step
-                                     and the groups' per-level profiles differ, measured no gain) */
+#define ATF_FLAG_DIST_SUBSETS 512u /* (the default since round 2; kept for compatibility) */
+#define ATF_FLAG_DIST_NO_SUBSETS 1024u /* atf_space_generate_dist: every group on every rank in every
+                                     generation.  By default, from the second generation on, each
+                                     group works on a subset of the ranks in proportion to its
+                                     candidate pairs in the previous generation (DESIGN.md §6:
+                                     fewer, larger kernels per rank; one-GPU steady-state
+                                     prediction for C5 at N = 4 / 8: 5.2 / 3.4-3.6 ms vs
+                                     5.4 / 3.75 ms) */
 #define ATF_FLAG_NO_TAIL 128u     /* expand a group's trailing narrow levels one at a time instead
                                      of the fused narrow tail (two launches for up to 4 levels,
                                      DESIGN.md §5); kept for parity coverage and A/B timing    */

@@ -28,7 +28,8 @@ ATF_FLAG_TIMING, ATF_FLAG_GENERIC_ONLY, ATF_FLAG_LEGACY_WIDE, ATF_FLAG_NO_JIT, A
 ATF_FLAG_NO_SEG_BOUNDS = 64
 ATF_FLAG_NO_TAIL = 128
 ATF_FLAG_NO_REPLAY = 256
-ATF_FLAG_DIST_SUBSETS = 512
+ATF_FLAG_DIST_SUBSETS = 512        # default since round 2 (no-op)
+ATF_FLAG_DIST_NO_SUBSETS = 1024
 
 
 class atf_range(C.Structure):

@@ -2396,7 +2396,7 @@ static void dist_assignment(const atf_space* s, int world, std::vector<uint64_t>
   u.assign(G, units);
   double W = 0;
   for (double w : s->group_work) W += w;
-  if (!(s->opts.flags & ATF_FLAG_DIST_SUBSETS) || world == 1 || G < 2 || s->group_work.size() != G || !(W > 0)) return;
+  if ((s->opts.flags & ATF_FLAG_DIST_NO_SUBSETS) || world == 1 || G < 2 || s->group_work.size() != G || !(W > 0)) return;
   uint64_t used = 0;
   size_t big = 0;
   for (size_t g = 0; g < G; g++) {

@@ -949,31 +949,39 @@ def test_dist_replay_virtual_ranks(Space, world, name):
     """Steady state of generate_dist: the first generation synchronises per round, the second
     sizes every level from the log, the third and later replay with device flags (one all-gather
     per generation, the verdicts) -- every generation identical to the single-GPU space."""
-    calls = _dist_check(Space, SMALL[name](), world, gens=4, streams=True)
+    from paper_conf_hpdc_raschg18_b200 import _lib as L
+    # default (rank subsets from generation 2): the assignment changes once, so the replay starts a
+    # generation later (fresh log, log-sized, then replays)
+    calls = _dist_check(Space, SMALL[name](), world, gens=5, streams=True)
+    assert calls[3] == calls[4] == 1, calls
+    # the plain partition (every group on every rank): generation 2 repeats generation 1's rounds
+    calls = _dist_check(Space, SMALL[name](), world, flags=L.ATF_FLAG_DIST_NO_SUBSETS, gens=4, streams=True)
     assert calls[2] == calls[3] == 1, calls
     assert calls[0] == calls[1], calls   # (0 when every level is replicated)
 
 
 @pytest.mark.parametrize("seed", range(0, 24, 5))
 def test_dist_replay_fuzz(Space, seed):
-    calls = _dist_check(Space, A.random_spec(seed), 3, gens=3, streams=True)
-    assert calls[2] == 1, calls
+    calls = _dist_check(Space, A.random_spec(seed), 3, gens=4, streams=True)
+    assert calls[3] == 1, calls
 
 
 def test_dist_replay_headline_flags(Space):
     from paper_conf_hpdc_raschg18_b200 import _lib as L
-    calls = _dist_check(Space, A.c5_chains(4096, 4), 4, flags=L.ATF_FLAG_NO_SEG_BOUNDS, gens=3, streams=True)
-    assert calls[2] == 1, calls
-    calls = _dist_check(Space, A.c5_chains(4096, 5), 2, flags=L.ATF_FLAG_NO_SEG_BOUNDS, gens=3, streams=True)
+    calls = _dist_check(Space, A.c5_chains(4096, 4), 4, flags=L.ATF_FLAG_NO_SEG_BOUNDS, gens=4, streams=True)
+    assert calls[3] == 1, calls
+    plain = L.ATF_FLAG_DIST_NO_SUBSETS
+    calls = _dist_check(Space, A.c5_chains(4096, 5), 2, flags=L.ATF_FLAG_NO_SEG_BOUNDS | plain, gens=3, streams=True)
     assert calls == [2, 2, 1], calls   # levels 4, 5 distributed; then the replay
-    calls = _dist_check(Space, A.c5_chains(4096, 5), 2, flags=L.ATF_FLAG_NO_REPLAY, gens=3, streams=True)
+    calls = _dist_check(Space, A.c5_chains(4096, 5), 2, flags=L.ATF_FLAG_NO_REPLAY | plain, gens=3, streams=True)
     assert calls == [2, 2, 2], calls   # replay off: one all-gather per distributed round every time
 
 
 @pytest.mark.parametrize("world", [2, 3, 8])
 @pytest.mark.parametrize("name", ["C5-300x4", "C5-4096x3", "C3-IS1", "fig1"])
 def test_dist_group_subsets(Space, world, name):
-    """ATF_FLAG_DIST_SUBSETS: from the second generation each group owns a subset of the ranks
+    """Rank subsets (the default; ATF_FLAG_DIST_SUBSETS is a no-op since round 2): from the second
+    generation each group owns a subset of the ranks
     (in proportion to its candidate pairs); the non-members follow its rounds with empty slices.
     Every generation identical to the single-GPU space; the fourth and later replay."""
     from paper_conf_hpdc_raschg18_b200 import _lib as L
@@ -1007,7 +1015,7 @@ def ag(b):
     return o.numpy().tobytes()
 with Space(A.c5_chains(300, 4), stream=torch.cuda.Stream()) as sp:
     ncalls = []
-    for _ in range(4):   # synchronous, log-sized, then two replays (device flags across processes)
+    for _ in range(5):   # synchronous; rank subsets: fresh log, log-sized, then two replays (device flags across processes)
         n0 = len(calls)
         sp.generate_dist(r, 2, ag)
         ncalls.append(len(calls) - n0)
@@ -1031,7 +1039,7 @@ dist.destroy_process_group()
     res = [np.load(tmp_path / f"rank{r}.npy", allow_pickle=True).item() for r in range(2)]
     spec = A.c5_chains(300, 4)
     for r in range(2):
-        assert res[r]["calls"][2] == res[r]["calls"][3] == 1, res[r]["calls"]
+        assert res[r]["calls"][3] == res[r]["calls"][4] == 1, res[r]["calls"]
     with Space(spec) as one:
         one.generate()
         assert res[0]["sizes"] == res[1]["sizes"] == one.group_sizes()

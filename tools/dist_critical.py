@@ -1,7 +1,8 @@
 """Critical-path prediction of the steady-state (replay) balanced generation vs the lock-step one.
 
 In the replay protocol a rank waits only on the device flags of the ranks that own its next parent
-slice, not on every rank: with groups on rank subsets (ATF_FLAG_DIST_SUBSETS) the
+slice, not on every rank: with groups on rank subsets (the default; plain partition:
+ATF_FLAG_DIST_NO_SUBSETS) the
 groups' rank sets progress independently.  From the per-rank per-round device times of N virtual
 ranks (one rank's round alone on the GPU, ATF_FLAG_TIMING), this prints
   lockstep: sum over rounds of the slowest rank's round (the bench's "replay" model), and
@@ -25,7 +26,7 @@ AG_US = 25.0
 
 
 def predict(spec, N, subsets, reps=3):
-    flags = L.ATF_FLAG_NO_SEG_BOUNDS | L.ATF_FLAG_TIMING | (L.ATF_FLAG_DIST_SUBSETS if subsets else 0)
+    flags = L.ATF_FLAG_NO_SEG_BOUNDS | L.ATF_FLAG_TIMING | (0 if subsets else L.ATF_FLAG_DIST_NO_SUBSETS)
     spaces = [Space(spec, flags=flags) for _ in range(N)]
     try:
         for _ in range(2):          # first generation: plain partition; subsets from the second on
