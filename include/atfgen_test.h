@@ -48,6 +48,10 @@ atf_status atf_test_set_tail_product(int32_t on);
 /* Fresh spaces with several groups: per-group level rounds without a barrier (1, default) or one
  * synchronising round for all groups (0).  A/B experiments. */
 atf_status atf_test_set_async_rounds(int32_t on);
+/* Fused-tail emit: the balanced leaf pass writes the leaves to global memory (1) or to the warp's
+ * staging area (0); 2 (default): to global memory when the tail's first level has more than 32
+ * candidates.  A/B experiments. */
+atf_status atf_test_set_tail_leaf_direct(int32_t mode);
 /* Geometry knobs for spaces planned / generated afterwards (tuning experiments; 0 = default):
  * warp tiles per SM below which the warp-tile kernel halves its nodes per tile (256), and
  * log2 of the candidate-pair count below which generate_dist replicates a level (28). */

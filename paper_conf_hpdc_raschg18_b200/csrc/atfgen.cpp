@@ -4149,6 +4149,12 @@ atf_status atf_test_set_async_rounds(int32_t on) {
   return ATF_OK;
 }
 
+atf_status atf_test_set_tail_leaf_direct(int32_t mode) {
+  if (mode < 0 || mode > 2) return ATF_ERR_INVALID_ARG;
+  jit_set_tail_leaf_direct(mode);
+  return ATF_OK;
+}
+
 atf_status atf_test_set_tail_product(int32_t on) {
   jit_set_tail_product(on != 0);
   return ATF_OK;

@@ -388,6 +388,10 @@ struct TailJitArgs { const u32* parent_rec; u64 n_parents, n_tiles; u32* tile_to
 //                   written out as coalesced vectors, CSR entries of every chunk.
 std::atomic<int> g_tail_stage{8192};  // tail emit staging bytes per warp (atf_test_set_tail_stage)
 std::atomic<bool> g_tail_product{true};  // product-structured tails (atf_test_set_tail_product)
+// leaf pass writes global memory instead of the staging area: 0 never, 1 always, 2 (default) when the
+// tail's first level has more than 32 candidates (u64 masks: C3-IS4 1.62 -> 1.58 ms; C3-IS2, r = 25,
+// measured 1.69 -> 1.77 ms the other way; tools/tail_leaf_ab.py)
+std::atomic<int> g_tail_leaf_direct{2};
 
 std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vector<int32_t>>& cx,
                             const std::vector<std::vector<uint32_t>>& cm, int k0,
@@ -605,7 +609,10 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "      u32 incl = cnt[d];\n#pragma unroll\n      for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, incl, o); "
        "if (lane >= o) incl += y; }\n";
   s += "      off[d] = incl - cnt[d];\n";
-  s += "      bytes += cnt[d] * (" + RB + "u + (d + 1 < " + NLs + " ? 4u : 0u) + (d == " + std::to_string(nl - 2) + " ? 4u : 0u));\n    }\n";
+  const int ldm = g_tail_leaf_direct.load();  // leaves straight to global memory (no staging)?
+  const bool leaf_direct = ldm == 1 || (ldm == 2 && t.lv[0].r > 32);
+  s += "      bytes += cnt[d] * (" + (leaf_direct ? "(d + 1 < " + NLs + " ? " + RB + "u : 0u)" : RB + "u") + " + (d + 1 < " + NLs +
+       " ? 4u : 0u) + (d == " + std::to_string(nl - 2) + " ? 4u : 0u));\n    }\n";
   s += "    if (valid) a.csr[0][nd] = base[0] + off[0];\n";
   // inclusive byte prefix per lane
   s += "    u32 bincl = bytes;\n#pragma unroll\n    for (int o = 1; o < 32; o <<= 1) { const u32 y = __shfl_up_sync(0xffffffffu, bincl, o); "
@@ -624,7 +631,8 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   s += "      const u32 lmo = o;  // leaf masks of the part's level-" + std::to_string(nl - 2) + " nodes\n";
   s += "      o += (pe[" + std::to_string(nl - 2) + "] - pb[" + std::to_string(nl - 2) + "]) * 4u;\n";
   s += "      o = (o + 15u) & ~15u;\n";
-  s += "#pragma unroll\n      for (int d = 0; d < " + NLs + "; d++) { roff[d] = o; o += (pe[d] - pb[d]) * " + RB + "u; }\n";
+  s += "#pragma unroll\n      for (int d = 0; d < " + NLs + "; d++) { roff[d] = o; o += " +
+       (leaf_direct ? "(d + 1 < " + NLs + " ? (pe[d] - pb[d]) * " + RB + "u : 0u)" : "(pe[d] - pb[d]) * " + RB + "u") + "; }\n";
   s += "      if (lane >= p0 && lane < p1 && valid) {\n        u32 cur[" + NLs + "];\n";
   s += "#pragma unroll\n        for (int d = 0; d < " + NLs + "; d++) cur[d] = off[d];\n";
   s += "        dfs0(a, w, nc, cur, base, pb, sm, staged, roff, coff, lmo);\n      }\n";
@@ -642,14 +650,17 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
     s += "            u32 pw[" + Ws + "];\n";
     for (int w = 0; w < W; w++) s += "            pw[" + std::to_string(w) + "] = pr[" + std::to_string(w) + "];\n";
     s += "            while (lm) {\n              const u32 cc = __ffs(lm) - 1;\n              lm &= lm - 1;\n";
-    s += "              u32* dst = reinterpret_cast<u32*>(sm + roff[" + ll + "]) + k * " + Ws + ";\n";
+    if (leaf_direct)
+      s += "              u32* dst = a.rec[" + ll + "] + (base[" + ll + "] + pb[" + ll + "] + k) * " + Ws + ";\n";
+    else
+      s += "              u32* dst = reinterpret_cast<u32*>(sm + roff[" + ll + "]) + k * " + Ws + ";\n";
     for (int w = 0; w < W; w++)
       s += "              dst[" + std::to_string(w) + "] = pw[" + std::to_string(w) + "]" +
            (w == fw && t.lv[nl - 1].r > 1 ? " | (cc << " + std::to_string(fs) + ")" : "") + ";\n";
     s += "              k++;\n            }\n          }\n          __syncwarp();\n        }\n";
   }
   s += "#pragma unroll\n        for (int d = 0; d < " + NLs + "; d++) {\n";
-  s += "          const u32 n = (pe[d] - pb[d]) * " + Ws + "u;\n";
+  s += "          const u32 n = " + (leaf_direct ? "d + 1 < " + NLs + " ? (pe[d] - pb[d]) * " + Ws + "u : 0u" : "(pe[d] - pb[d]) * " + Ws + "u") + ";\n";
   s += "          const u32* src = reinterpret_cast<const u32*>(sm + roff[d]);\n          u32* dst = a.rec[d] + (base[d] + pb[d]) * " + Ws + ";\n";
   if (W % 2 == 0)  // 8-byte aligned on both sides (records of even W, 8-byte CSR regions before them)
     s += "          { const uint2* s2 = reinterpret_cast<const uint2*>(src); uint2* d2 = reinterpret_cast<uint2*>(dst);\n"
@@ -1244,4 +1255,5 @@ int jit_decode_launch(void* kernel, const DecodeArgs& a, const uint64_t* idx, co
 namespace atf {
 void jit_set_tail_stage(int bytes) { g_tail_stage.store(bytes > 0 ? bytes : 8192); }
 void jit_set_tail_product(bool on) { g_tail_product.store(on); }
+void jit_set_tail_leaf_direct(int mode) { g_tail_leaf_direct.store(mode); }
 }  // namespace atf

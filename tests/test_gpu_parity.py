@@ -1084,7 +1084,7 @@ def test_float_parameters_by_position(Space):
         assert {r["TOL"] for r in named} == {0.25 * i for i in range(1, 9)}
 
 
-@pytest.mark.parametrize("name", ["C2-256", "C3-IS1", "C5-300x4"])
+@pytest.mark.parametrize("name", ["C2-256", "C3-IS1", "C5-300x4", "C3-12x30x8"])
 def test_sync_rounds_and_dfs_tail_count_parity(Space, name):
     """The A/B alternatives stay exact: one synchronising level round for all groups
     (atf_test_set_async_rounds(0)) instead of per-group rounds, and the depth-first tail count
@@ -1092,8 +1092,12 @@ def test_sync_rounds_and_dfs_tail_count_parity(Space, name):
     from paper_conf_hpdc_raschg18_b200 import _lib as L
     L.check(L.atf_test_set_async_rounds(0))
     L.check(L.atf_test_set_tail_product(0))
+    L.check(L.atf_test_set_tail_leaf_direct(1))   # leaves straight to global memory in every tail
     try:
+        _check_against_oracle(Space, SMALL[name]())
+        L.check(L.atf_test_set_tail_leaf_direct(0))   # leaves staged in every tail
         _check_against_oracle(Space, SMALL[name]())
     finally:
         L.check(L.atf_test_set_async_rounds(1))
         L.check(L.atf_test_set_tail_product(1))
+        L.check(L.atf_test_set_tail_leaf_direct(2))
