@@ -39,7 +39,8 @@ atf_status atf_test_jit_source(atf_space* s, int32_t g, int32_t k, char* buf, si
  * *k0_out (optional) = the tail's first level (-1 if none). */
 atf_status atf_test_tail_source(atf_space* s, int32_t g, char* buf, size_t cap, size_t* len_out, int32_t* k0_out);
 /* Staging bytes per warp of the fused tail's emit kernel for spaces planned afterwards (tuning
- * experiments; 0 restores the default 8192, a multiple of 16 in [2048, 49152] otherwise). */
+ * experiments; 0 restores the default -- 12 KB when the tail's first level has more than 32
+ * candidates, else 8 KB --, a multiple of 16 in [2048, 49152] otherwise). */
 atf_status atf_test_set_tail_stage(int32_t bytes);
 /* Product-structured fused tails (every term of every tail level reads only ancestors above the
  * tail: the subtree under a frontier node is a grid of the levels' masks): on (1,

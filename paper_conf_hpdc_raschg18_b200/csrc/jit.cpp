@@ -386,7 +386,10 @@ struct TailJitArgs { const u32* parent_rec; u64 n_parents, n_tiles; u32* tile_to
 //                   canonical order; children staged in per-warp shared-memory buffers (with the
 //                   frontier lane they descend from, whose node constants sit in shared memory),
 //                   written out as coalesced vectors, CSR entries of every chunk.
-std::atomic<int> g_tail_stage{8192};  // tail emit staging bytes per warp (atf_test_set_tail_stage)
+// tail emit staging bytes per warp (atf_test_set_tail_stage); 0 = by the tail: 12 KB when its first
+// level has more than 32 candidates (C3-IS4 1.59 -> 1.54 ms), else 8 KB (C3-IS2: 6 KB 1.72, 8 KB 1.69,
+// 12 KB 1.75 ms; profiles/r02_tail_stage_sweep.txt)
+std::atomic<int> g_tail_stage{0};
 std::atomic<bool> g_tail_product{true};  // product-structured tails (atf_test_set_tail_product)
 // leaf pass writes global memory instead of the staging area: 0 never, 1 always, 2 (default) when the
 // tail's first level has more than 32 candidates (u64 masks: C3-IS4 1.62 -> 1.58 ms; C3-IS2, r = 25,
@@ -540,7 +543,7 @@ std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vec
   // the lanes of a part write their subtrees into shared memory, the warp copies every level's
   // run out as coalesced words.  A single lane whose subtree alone exceeds the area writes
   // straight to global memory.
-  const int kStage = g_tail_stage.load();  // staging bytes per warp (8192; test hook)
+  const int kStage = g_tail_stage.load() > 0 ? g_tail_stage.load() : (t.lv[0].r > 32 ? 12288 : 8192);  // per warp
   if (warp_bytes) *warp_bytes = kStage;
   const std::string NLs = std::to_string(nl), NCs = std::to_string(NC), RB = std::to_string(W * 4);
   // The leaf level is not written by the depth-first walk when staged: a level-(nl-2) node stores
@@ -1253,7 +1256,7 @@ int jit_decode_launch(void* kernel, const DecodeArgs& a, const uint64_t* idx, co
 }  // namespace atf
 
 namespace atf {
-void jit_set_tail_stage(int bytes) { g_tail_stage.store(bytes > 0 ? bytes : 8192); }
+void jit_set_tail_stage(int bytes) { g_tail_stage.store(bytes > 0 ? bytes : 0); }
 void jit_set_tail_product(bool on) { g_tail_product.store(on); }
 void jit_set_tail_leaf_direct(int mode) { g_tail_leaf_direct.store(mode); }
 }  // namespace atf
