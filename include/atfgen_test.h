@@ -53,6 +53,9 @@ atf_status atf_test_set_async_rounds(int32_t on);
  * staging area (0); 2 (default): to global memory when the tail's first level has more than 32
  * candidates.  A/B experiments. */
 atf_status atf_test_set_tail_leaf_direct(int32_t mode);
+/* Mid-width exact-mask kernel (atf_wide_jit): candidates per superset group of the first conjunct
+ * (2, 4 = default, 8, 16; 0 restores 4), for kernels compiled afterwards.  A/B experiments. */
+atf_status atf_test_set_wide_group(int32_t n);
 /* Geometry knobs for spaces planned / generated afterwards (tuning experiments; 0 = default):
  * warp tiles per SM below which the warp-tile kernel halves its nodes per tile (256), and
  * log2 of the candidate-pair count below which generate_dist replicates a level (28). */

@@ -112,6 +112,7 @@ _SIGS = {
     "atf_test_set_tail_product": (_st, [C.c_int32]),
     "atf_test_set_async_rounds": (_st, [C.c_int32]),
     "atf_test_set_tail_leaf_direct": (_st, [C.c_int32]),
+    "atf_test_set_wide_group": (_st, [C.c_int32]),
     "atf_test_jit_source": (_st, [SP, C.c_int32, C.c_int32, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t)]),
     "atf_test_tail_source": (_st, [SP, C.c_int32, C.c_char_p, C.c_size_t, C.POINTER(C.c_size_t),
                                    C.POINTER(C.c_int32)]),

@@ -355,7 +355,8 @@ int launch_add_offset(uint64_t* data, uint64_t n, uint64_t add, void* stream);
 void jit_set_tail_stage(int bytes);  // test hook: tail emit staging bytes per warp (0: default)
 void jit_set_tail_product(bool on);  // test hook: product-structured tails on (default) / off
 bool jit_tail_product(void* handle);  // the compiled tail's count is product-structured
-void jit_set_tail_leaf_direct(int mode);  // test hook: leaf pass writes global memory (0 / 1 / 2 auto)
+void jit_set_tail_leaf_direct(int mode);
+void jit_set_wide_group(int n);  // test hook: atf_wide_jit superset group size (4 or 8)  // test hook: leaf pass writes global memory (0 / 1 / 2 auto)
 int launch_host_gate(const unsigned int* flag, unsigned int v, void* stream);
 int launch_dist_flag_set(unsigned long long* f, unsigned long long v, void* stream);
 int launch_dist_flag_wait(const unsigned long long* f, unsigned long long v, unsigned long long* err, void* stream);

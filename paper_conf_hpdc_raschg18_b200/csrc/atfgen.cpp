@@ -4149,6 +4149,12 @@ atf_status atf_test_set_async_rounds(int32_t on) {
   return ATF_OK;
 }
 
+atf_status atf_test_set_wide_group(int32_t n) {
+  if (n != 0 && n != 2 && n != 4 && n != 8 && n != 16) return ATF_ERR_INVALID_ARG;
+  jit_set_wide_group(n ? n : 4);
+  return ATF_OK;
+}
+
 atf_status atf_test_set_tail_leaf_direct(int32_t mode) {
   if (mode < 0 || mode > 2) return ATF_ERR_INVALID_ARG;
   jit_set_tail_leaf_direct(mode);

@@ -395,6 +395,7 @@ std::atomic<bool> g_tail_product{true};  // product-structured tails (atf_test_s
 // tail's first level has more than 32 candidates (u64 masks: C3-IS4 1.62 -> 1.58 ms; C3-IS2, r = 25,
 // measured 1.69 -> 1.77 ms the other way; tools/tail_leaf_ab.py)
 std::atomic<int> g_tail_leaf_direct{2};
+std::atomic<int> g_wide_group{4};  // atf_wide_jit: candidates per superset group (atf_test_set_wide_group)
 
 std::string gen_tail_source(const TailArgs& t, int W, const std::vector<std::vector<int32_t>>& cx,
                             const std::vector<std::vector<uint32_t>>& cm, int k0,
@@ -806,18 +807,22 @@ std::string gen_wide_source(const LevelArgs& a, int W, const std::vector<int32_t
     s += "      u32 mw = 0u;\n";
     if (grouped) {
       const bool mulx = a.terms[0].kind == T_MULX;
-      for (int c0 = 0; c0 < 32 && 32 * j + c0 < r; c0 += 4) {
-        const int nc = std::min(4, r - (32 * j + c0));
+      const int GS = g_wide_group.load();  // candidates per superset group (4; test hook)
+      for (int c0 = 0; c0 < 32 && 32 * j + c0 < r; c0 += GS) {
+        const int nc = std::min(GS, r - (32 * j + c0));
         std::vector<std::string> pr;
         for (int c = c0; c < c0 + nc; c++) {
           const int ci = 32 * j + c;
           const uint32_t ax = cx[ci] < 0 ? 0u - (uint32_t)cx[ci] : (uint32_t)cx[ci];
           pr.push_back(mulx ? hex(ax) + " * md0" : "n0 * " + hex(cm[ci]));
         }
-        std::string q = pr[0];
-        if (pr.size() == 2) q = "min(" + pr[0] + ", " + pr[1] + ")";
-        if (pr.size() == 3) q = "min(min(" + pr[0] + ", " + pr[1] + "), " + pr[2] + ")";
-        if (pr.size() == 4) q = "min(min(" + pr[0] + ", " + pr[1] + "), min(" + pr[2] + ", " + pr[3] + "))";
+        while (pr.size() > 1) {  // balanced min tree
+          std::vector<std::string> nx;
+          for (size_t i = 0; i + 1 < pr.size(); i += 2) nx.push_back("min(" + pr[i] + ", " + pr[i + 1] + ")");
+          if (pr.size() % 2) nx.push_back(pr.back());
+          pr.swap(nx);
+        }
+        const std::string q = pr[0];
         s += "      { const u32 q = " + q + "; if (q " + (mulx ? "<= mq0" : "< 0x10000u") + ") mw |= " +
              hex(((1u << nc) - 1u) << c0) + "; }\n";
       }
@@ -1259,4 +1264,5 @@ namespace atf {
 void jit_set_tail_stage(int bytes) { g_tail_stage.store(bytes > 0 ? bytes : 0); }
 void jit_set_tail_product(bool on) { g_tail_product.store(on); }
 void jit_set_tail_leaf_direct(int mode) { g_tail_leaf_direct.store(mode); }
+void jit_set_wide_group(int n) { g_wide_group.store(n); }
 }  // namespace atf
