@@ -1348,6 +1348,7 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
     const uint64_t base = a.tile_base[t];
     const uint32_t tt = (uint32_t)(a.tile_base[t + 1] - base);  // the tile's children
     const bool staged = tt <= (uint32_t)CAP;
+    const bool coop = tt >= 32u * (uint32_t)TN;
     uint32_t run = 0;
 #pragma unroll
     for (int q = 0; q < kNfNPL; q++) {
@@ -1362,6 +1363,33 @@ __global__ void __launch_bounds__(256) nfast_emit(const __grid_constant__ LevelA
       uint32_t rank = run + (incl - c);  // tile-local
       run += __shfl_sync(FULL, incl, 31);
       if (nd < a.n_parents) a.csr[nd] = base + rank;
+      if (coop) {
+        // a dense tile (>= 32 children per parent on average, C3-IS4's unconstrained KWG level):
+        // the warp writes each node's children together -- lane l takes candidate bits l and
+        // l + 32 -- so the stores are coalesced instead of every lane walking its own node's mask
+        // (32 scattered streams): C3-IS4 1.54 -> 1.50 ms; sparser tiles keep the per-lane walk
+        for (int src = 0; src < 32; src++) {
+          const unsigned long long ms = __shfl_sync(FULL, mask[q], src);
+          if (!ms) continue;  // warp-uniform
+          const uint32_t r0 = __shfl_sync(FULL, rank, src);
+          uint32_t rr[W];
+#pragma unroll
+          for (int w = 0; w < W; w++) rr[w] = __shfl_sync(FULL, rec[q][w], src);
+#pragma unroll
+          for (int h = 0; h < 2; h++) {
+            if (h == 1 && a.r <= 32) break;  // (warp-uniform) no candidate bits above 31
+            const int pos = lane + 32 * h;
+            if ((ms >> pos) & 1ull) {
+              const uint32_t k = (uint32_t)__popcll(ms & ((1ull << pos) - 1ull));
+              uint32_t out[W];
+#pragma unroll
+              for (int w = 0; w < W; w++) out[w] = rr[w] | (w == a.field_word ? (uint32_t)pos << a.field_shift : 0u);
+              store_record<W>(a.child_rec + (base + r0 + k) * W, out);
+            }
+          }
+        }
+        continue;
+      }
       unsigned long long m = mask[q];
       while (m) {
         const int cc = __ffsll((long long)m) - 1;
